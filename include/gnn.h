@@ -1,0 +1,319 @@
+/*
+ * gnn.h — C-ABI of the B200 (sm_100a) GNN neighbor-aggregation library.
+ *
+ * The operations are those of Huang et al., "Understanding and Bridging the
+ * Gaps in Current GNN Performance Optimizations", PPoPP'21 (cited as P:<line>
+ * of /root/reference/PAPER.md).  Readings of silent or garbled passages are
+ * R1..R14 in DESIGN.md §2.
+ *
+ * Conventions (all entry points):
+ *  - Graph: CSR by destination (Fig 2): row v lists the sources u
+ *    of edges u -> v.  Host arrays: rowptr int64[n+1] with
+ *    rowptr[0] = 0, non-decreasing, rowptr[n] = nnz < 2^31; colidx int32[nnz]
+ *    with 0 <= colidx < n_src.  Multi-edges count separately; self loops only
+ *    if present (R1).
+ *  - Features: row-major fp32 with row stride ld (elements), ld >= width.
+ *    Pointers named *_h are HOST pointers; every other array pointer is a
+ *    DEVICE pointer on the device that was current when the plan was made.
+ *  - Ownership: the caller allocates and owns every feature/weight/output/
+ *    workspace buffer (torch tensors in practice).  The plan owns copies of the
+ *    graph and its schedule on host and device and frees them in
+ *    gnn_plan_destroy (caller guarantees no call is in flight, like cudaFree).
+ *  - Streams: compute calls only enqueue work on `stream` (NULL = legacy
+ *    default stream); they never synchronise or allocate and can be captured
+ *    into CUDA graphs.  gnn_plan_create / gnn_plan_export* are synchronous.
+ *  - Errors: every entry point returns gnn_status; nothing aborts, nothing
+ *    throws across the ABI.  gnn_last_error() returns a thread-local message
+ *    for the last failing call.  Device faults surface at the caller's next
+ *    synchronisation.
+ *  - Y is fully overwritten; rows with no in-edges get 0 for every reducer (R3).
+ *  - Thread-safety: a plan is immutable after creation; concurrent calls on
+ *    different streams are safe if each has its own workspace.
+ */
+#ifndef GNN_H
+#define GNN_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  GNN_OK = 0,
+  GNN_ERR_INVALID_ARG = 1,   /* null pointer, bad size/stride, aliasing */
+  GNN_ERR_INVALID_GRAPH = 2, /* CSR validation failed */
+  GNN_ERR_WORKSPACE = 3,     /* workspace smaller than gnn_workspace_size() */
+  GNN_ERR_CUDA = 4,          /* CUDA runtime error (message has cudaGetErrorString) */
+  GNN_ERR_NOMEM = 5,         /* host or device allocation failed */
+  GNN_ERR_UNSUPPORTED = 6,   /* valid request this build does not implement */
+  GNN_ERR_INTERNAL = 7
+} gnn_status;
+
+typedef struct gnn_plan_s *gnn_plan_t;
+typedef struct CUstream_st *gnn_stream_t; /* identical to cudaStream_t */
+
+/* Reducers: Table 1 sum / mean / pooling-max. */
+typedef enum { GNN_SUM = 0, GNN_MEAN = 1, GNN_MAX = 2 } gnn_reduce;
+/* Edge weights: Table 2 Const, GCN 1/sqrt(d_u d_v) with
+ * d_u = out-degree of u, d_v = in-degree of v (R1), or an explicit per-CSR-entry
+ * array. */
+typedef enum { GNN_W_ONE = 0, GNN_W_GCN = 1, GNN_W_EDGE = 2 } gnn_weight;
+
+/*
+ * Plan options.  Locality-aware task scheduling (LAS) and
+ * neighbor grouping (NG).
+ */
+typedef struct {
+  uint32_t struct_size;  /* sizeof(gnn_plan_opts), for ABI versioning */
+  int32_t reorder;       /* 0 = identity task order, 1 = LAS (MinHash+LSH+merge) */
+  int32_t group_size;    /* NG upper bound ng; -1 = auto (R8-ii); 0 = never split */
+  int32_t tile_groups;   /* T: max groups per CTA work tile (0 -> 32) */
+  int32_t cluster_cap;   /* LAS cluster size cap (32) */
+  int32_t minhash_k;     /* K signature length (32) */
+  int32_t lsh_rows;      /* r rows per band (2); b = K / r bands */
+  int32_t pair_window;   /* W: candidate pairs (m_i, m_{i+d}), 1 <= d <= W (8) */
+  int32_t min_sim;       /* re-enqueue threshold; -1 -> lsh_rows */
+  int32_t deterministic; /* 1: fixed-order combine (R9); 0: float atomics */
+  uint64_t seed;         /* MinHash salt stream seed */
+} gnn_plan_opts;
+
+/* Fill defaults: reorder 0, group_size -1, tile_groups 32, cluster_cap 32,
+ * minhash_k 32, lsh_rows 2, pair_window 8, min_sim -1, deterministic 1, seed 0. */
+void gnn_plan_opts_default(gnn_plan_opts *opts);
+
+typedef struct {
+  int64_t n;            /* destination rows */
+  int64_t n_src;        /* source rows (== n for gnn_plan_create) */
+  int64_t nnz;
+  int64_t n_groups;     /* G = sum ceil(d_v / ng) */
+  int64_t n_tiles;
+  int64_t n_split_rows; /* rows whose groups span more than one tile */
+  int64_t n_empty_rows;
+  int64_t n_clusters;   /* LAS clusters (n if reorder == 0) */
+  int64_t n_pairs;      /* LSH candidate pairs (0 if reorder == 0) */
+  int32_t group_size;   /* ng actually used */
+  int32_t tile_groups;
+  int32_t max_degree;
+  int32_t reorder;
+  double ms_validate, ms_upload, ms_degrees, ms_minhash, ms_lsh, ms_merge, ms_ng;
+} gnn_plan_info;
+
+/*
+ * Build a plan (a1 CSR ingest + degrees, a2 LAS if opts->reorder, a3 NG and
+ * CTA tiles).  Synchronous; copies the host CSR.  Validates in O(n + nnz):
+ * on failure returns GNN_ERR_INVALID_GRAPH and sets *out = NULL.
+ * opts may be NULL (defaults).
+ */
+gnn_status gnn_plan_create(int64_t n, int64_t nnz, const int64_t *rowptr_h,
+                           const int32_t *colidx_h, const gnn_plan_opts *opts,
+                           gnn_plan_t *out);
+
+/*
+ * Rectangular variant: n destination rows, sources indexed in [0, n_src).
+ * src_degree_h (nullable, int32[n_src]) overrides the source out-degrees used
+ * by GNN_W_GCN (multi-GPU local plans pass the GLOBAL out-degrees in the padded
+ * all-gather layout); NULL = count colidx.
+ */
+gnn_status gnn_plan_create_ex(int64_t n, int64_t n_src, int64_t nnz,
+                              const int64_t *rowptr_h, const int32_t *colidx_h,
+                              const int32_t *src_degree_h,
+                              const gnn_plan_opts *opts, gnn_plan_t *out);
+
+gnn_status gnn_plan_get_info(gnn_plan_t plan, gnn_plan_info *info);
+
+/*
+ * Copy the schedule to host buffers sized from gnn_plan_info (any may be NULL):
+ * perm_h int32[n] (task order), grp_row_h int32[G], grp_beg_h int64[G] (first
+ * CSR entry of each group), tile_beg_h int64[n_tiles+1] (group offsets).
+ * Bit-exact with the oracle's orc_las_merge / orc_neighbor_groups / orc_tiles.
+ */
+gnn_status gnn_plan_export(gnn_plan_t plan, int32_t *perm_h, int32_t *grp_row_h,
+                           int64_t *grp_beg_h, int64_t *tile_beg_h);
+
+/*
+ * LAS intermediates (reorder == 1 only): sig_h uint64[n * minhash_k] (GPU
+ * MinHash), pairs_h int32[2 * n_pairs] (sorted (a, b), a < b),
+ * cluster_of_h int32[n] (representative of each node).  Any may be NULL.
+ */
+gnn_status gnn_plan_export_las(gnn_plan_t plan, uint64_t *sig_h, int32_t *pairs_h,
+                               int32_t *cluster_of_h);
+
+/* Device arrays of the plan's per-node normalisers (read-only, owned by the
+ * plan): nsrc = 1/sqrtf(d_out) [n_src], ndst = 1/sqrtf(d_in) [n] (0 if degree 0). */
+gnn_status gnn_plan_normalizers(gnn_plan_t plan, const float **nsrc, const float **ndst);
+
+gnn_status gnn_plan_destroy(gnn_plan_t plan);
+
+/* Workspace operations */
+typedef enum {
+  GNN_OP_AGGREGATE = 0,     /* f_out = F */
+  GNN_OP_GAT_AGGREGATE = 1, /* f_out = H * Fh, heads = H */
+  GNN_OP_EDGECONV = 2,      /* f_in, f_out */
+  GNN_OP_GCN_LAYER = 3,     /* f_in, f_out */
+  GNN_OP_GAT_LAYER = 4      /* f_in, f_out = H * Fh, heads = H */
+} gnn_op;
+
+/* Bytes of device workspace a call needs (may be 0; pass NULL then).  The
+ * workspace must be 256-byte aligned.  Unused size arguments are ignored. */
+size_t gnn_workspace_size(gnn_plan_t plan, int op, int32_t f_in, int32_t f_out, int32_t heads);
+
+/*
+ * a6 + a9: graph operation y_v = REDUCE_{u->v} e_uv * x_u (Table 1 x Table 2,
+ * Eq 1 inner part P:217), evaluated over the plan's neighbor groups in task
+ * order; split rows combined in fixed group order (R9) or with atomics
+ * (deterministic == 0, sum/mean only).  Epilogue (linear property):
+ * GCN x ndst[v], mean / D_v, then + add_row[v] (nullable, EdgeConv's Q), then
+ * ReLU if relu != 0.
+ *   edge_w: [nnz] in CSR order, required iff weight == GNN_W_EDGE.
+ *   X: [n_src, ldx] with F <= ldx; Y: [n, ldy]; X and Y must not overlap.
+ *   add_row: [n, ld_add] or NULL.
+ * F == 0 is a no-op.
+ */
+gnn_status gnn_aggregate(gnn_plan_t plan, int reduce, int weight, const float *edge_w,
+                         const float *X, int64_t ldx, int32_t F, float *Y, int64_t ldy,
+                         int32_t relu, const float *add_row, int64_t ld_add,
+                         void *ws, size_t ws_bytes, gnn_stream_t stream);
+
+/*
+ * a7: fused GAT graph operation (Eq 2; Listing 1 P:622-646 fused, DVRA
+ * P:943-968, division postponed by the linear property).  Per head h:
+ * e_uv = LeakyReLU(s_u[h] + t_v[h], neg_slope), alpha = softmax_v(e),
+ * y_v[h] = SUM_u alpha_uv z_u[h].  Edge scores never reach HBM.
+ *   Zs: [n_src, ldz] rows = [z_u (H*Fh floats) | s_u (H floats)], ldz >= H*Fh+H.
+ *   t:  [n, ldt] (t_v per head).  Y: [n, ldy], ldy >= H*Fh.
+ */
+gnn_status gnn_gat_aggregate(gnn_plan_t plan, const float *Zs, int64_t ldz,
+                             const float *t, int64_t ldt, int32_t H, int32_t Fh,
+                             float neg_slope, float *Y, int64_t ldy,
+                             void *ws, size_t ws_bytes, gnn_stream_t stream);
+
+/*
+ * Full GAT layer: Z = X W (W: [f_in, H*Fh] row-major), s = Z_h . a_src_h,
+ * t = Z_h . a_dst_h (computed as extra GEMM columns X (W_h a_h)), then
+ * gnn_gat_aggregate.  Requires n_src == n.  Workspace from
+ * gnn_workspace_size(plan, GNN_OP_GAT_LAYER, f_in, H * Fh, H).
+ */
+gnn_status gnn_gat_layer(gnn_plan_t plan, const float *X, int64_t ldx, int32_t f_in,
+                         const float *W, const float *a_src, const float *a_dst,
+                         int32_t H, int32_t Fh, float neg_slope, float *Y, int64_t ldy,
+                         void *ws, size_t ws_bytes, gnn_stream_t stream);
+
+/*
+ * a8: EdgeConv max aggregation given the pre-transformed [P | Q] rows
+ * (redundancy bypass P:1014-1021, reading R6): y_v = ReLU(Q_v + MAX_u P_u),
+ * empty row -> 0.  PQ: [n, ldpq], P = columns [0, f_out), Q = [f_out, 2 f_out).
+ */
+gnn_status gnn_edgeconv_aggregate(gnn_plan_t plan, const float *PQ, int64_t ldpq,
+                                  int32_t f_out, float *Y, int64_t ldy,
+                                  void *ws, size_t ws_bytes, gnn_stream_t stream);
+
+/*
+ * Full EdgeConv layer y_v = MAX_u ReLU(Theta(x_u - x_v) + Phi x_v + b):
+ * [P | Q] = X [Theta^T | (Phi - Theta)^T] (+ b on Q) by gnn_gemm, then
+ * gnn_edgeconv_aggregate.  theta, phi: [f_out, f_in] row-major; bias nullable.
+ */
+gnn_status gnn_edgeconv(gnn_plan_t plan, const float *X, int64_t ldx, int32_t f_in,
+                        const float *theta, const float *phi, const float *bias,
+                        int32_t f_out, float *Y, int64_t ldy, void *ws, size_t ws_bytes,
+                        gnn_stream_t stream);
+
+/*
+ * a5: dense transform H = X W (Eq 1 "(x) W") in fp32 accuracy,
+ * X: [m, ldx] (k used), W: [k, ldw] (n used), H: [m, ldh].
+ * Epilogue: row_scale (nullable, [m]) multiplies row i; col_bias (nullable, [n])
+ * is added after the scale; relu != 0 clamps.  H must not overlap X or W.
+ */
+gnn_status gnn_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H,
+                    int64_t ldh, int64_t m, int32_t k, int32_t n, const float *row_scale,
+                    const float *col_bias, int32_t relu, gnn_stream_t stream);
+
+/* GEMM implementation selector (process-wide): 0 = auto, 1 = SIMT FFMA,
+ * 2 = tcgen05 3xTF32.  Returns the previous value. */
+int gnn_set_gemm_impl(int impl);
+
+/*
+ * GCN layer (Eq 1): Y = ACT((A_gcn X) W).  order: 0 = auto (aggregate at
+ * min(f_in, f_out)), 1 = transform first (H = X W scaled by nsrc, aggregate,
+ * x ndst), 2 = aggregate first.  Workspace: gnn_workspace_size(plan,
+ * GNN_OP_GCN_LAYER, f_in, f_out, 0).  X has n_src rows; Y has n rows.
+ */
+gnn_status gnn_gcn_layer(gnn_plan_t plan, const float *X, int64_t ldx, int32_t f_in,
+                         const float *W, int64_t ldw, int32_t f_out, int32_t relu,
+                         int32_t order, float *Y, int64_t ldy, void *ws, size_t ws_bytes,
+                         gnn_stream_t stream);
+
+/*
+ * Second half of a transform-first GCN layer (Eq 1 reassociated, R4-i; linear
+ * property): y_v = ACT(ndst[v] * SUM_{u->v} Hs[u]) where the caller's
+ * Hs rows are already scaled by nsrc[u] (gnn_gemm row_scale = the plan's nsrc
+ * from gnn_plan_normalizers).  Hs: [n_src, ldh]; Y: [n, ldy].
+ */
+gnn_status gnn_gcn_aggregate_prescaled(gnn_plan_t plan, const float *Hs, int64_t ldh, int32_t F,
+                                       float *Y, int64_t ldy, int32_t relu, void *ws,
+                                       size_t ws_bytes, gnn_stream_t stream);
+
+/*
+ * GAT parameter fold (device, O(f_in * H * Fh)): Wext[:, 0:H*Fh] = W,
+ * Wext[:, H*Fh + h] = W_h . a_src_h, Wext[:, H*Fh + H + h] = W_h . a_dst_h, so
+ * X Wext = [Z | s | t] (Table 2 GAT scores as extra GEMM columns).
+ * W: [f_in, H*Fh] row-major; Wext: [f_in, ldwe], ldwe >= H*Fh + 2H.
+ */
+gnn_status gnn_gat_fold_weights(const float *W, const float *a_src, const float *a_dst,
+                                int32_t f_in, int32_t H, int32_t Fh, float *Wext, int64_t ldwe,
+                                gnn_stream_t stream);
+
+/*
+ * a10: multi-GPU destination-row partition (host only, reading R10):
+ * bounds[p] = smallest i with rowptr[i] >= ceil(p * nnz / P), bounds[0] = 0,
+ * bounds[P] = n.  bounds_h: int64[nparts + 1].
+ */
+gnn_status gnn_partition_rows(int64_t n, const int64_t *rowptr_h, int32_t nparts,
+                              int64_t *bounds_h);
+
+/*
+ * Local CSR of rank `rank` (host only): rows [bounds[rank], bounds[rank+1]),
+ * every source u translated to the padded all-gather layout
+ * owner(u) * r_max + (u - bounds[owner(u)]), r_max = max part size.
+ * Outputs (caller-allocated, sizes from a NULL-output query):
+ *   *r_max, *local_nnz; local_rowptr_h int64[rows+1]; local_colidx_h
+ *   int32[local_nnz]; src_degree_h int32[nparts * r_max] = global out-degree of
+ *   each padded source slot (0 for pad slots).
+ */
+gnn_status gnn_local_csr(int64_t n, const int64_t *rowptr_h, const int32_t *colidx_h,
+                         const int64_t *bounds_h, int32_t nparts, int32_t rank,
+                         int64_t *r_max, int64_t *local_nnz, int64_t *local_rowptr_h,
+                         int32_t *local_colidx_h, int32_t *src_degree_h);
+
+/*
+ * Host-only planner steps (no GPU needed).  gnn_plan_create runs exactly these
+ * after the GPU MinHash; they are exported so the host logic can be checked
+ * against the oracle without a device.
+ *
+ * gnn_las_host: a2 steps 2-5 (LSH banding P:819-825, pair merging P:827-844,
+ *   task scheduling P:846-853; reading R7) from MinHash signatures sig_h
+ *   uint64[n * K].  Outputs perm_h int32[n], cluster_of_h int32[n] (nullable),
+ *   *n_pairs, *n_clusters.
+ * gnn_groups_host: a3 neighbor groups in task order and CTA tiles (P:855-884,
+ *   reading R8).  ng <= 0 = one group per row.  Call with NULL arrays first to
+ *   get *n_groups / *n_tiles; then grp_row_h int32[G], grp_beg_h int64[G],
+ *   tile_beg_h int64[n_tiles + 1].
+ */
+gnn_status gnn_las_host(int64_t n, const int64_t *rowptr_h, const uint64_t *sig_h, int32_t K,
+                        int32_t r, int32_t W, int32_t cap, int32_t min_sim, int32_t *perm_h,
+                        int32_t *cluster_of_h, int64_t *n_pairs, int64_t *n_clusters);
+gnn_status gnn_groups_host(int64_t n, const int64_t *rowptr_h, const int32_t *perm_h, int32_t ng,
+                           int32_t T, int64_t *n_groups, int64_t *n_tiles, int32_t *grp_row_h,
+                           int64_t *grp_beg_h, int64_t *tile_beg_h);
+
+/* Number of kernels this library launched since load (for bench accounting). */
+uint64_t gnn_launch_count(void);
+
+const char *gnn_last_error(void);
+const char *gnn_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GNN_H */

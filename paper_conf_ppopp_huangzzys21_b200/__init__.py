@@ -1,0 +1,24 @@
+"""paper_conf_ppopp_huangzzys21_b200 — B200-native (sm_100a) GNN neighbor aggregation.
+
+The hot path of Huang et al., "Understanding and Bridging the Gaps in Current
+GNN Performance Optimizations" (PPoPP'21): CSR graph operations (sum / mean /
+max), the fused GAT edge-softmax aggregation, EdgeConv max aggregation, the
+X.W transform, locality-aware task scheduling and neighbor grouping.
+
+The product is ``libgnn.so`` (C-ABI, ``include/gnn.h``); ``gnn`` is its thin
+Python binding.  Touching any public name loads the library and fails loudly
+if it is not built — there is no CPU fallback.  (The submodule ``build`` can
+be imported without loading the library, so it can rebuild it.)
+"""
+_PUBLIC = ("Plan", "aggregate", "gat_aggregate", "gat_layer", "edgeconv", "edgeconv_aggregate", "gemm",
+           "gcn_layer", "partition_rows", "local_csr", "launch_count", "set_gemm_impl", "las_host", "groups_host",
+           "GnnError")
+__all__ = ["gnn", *_PUBLIC]
+
+
+def __getattr__(name):
+    if name == "gnn" or name in _PUBLIC:
+        import importlib
+        _gnn = importlib.import_module(__name__ + ".gnn")
+        return _gnn if name == "gnn" else getattr(_gnn, name)
+    raise AttributeError(name)

@@ -1,0 +1,695 @@
+// api.cpp — the C-ABI of libgnn.so (include/gnn.h): validation, plan
+// lifetime, dispatch to the sm_100a kernels.  No exception crosses the ABI.
+#include <atomic>
+#include <chrono>
+#include <climits>
+#include <cstring>
+#include <exception>
+#include <new>
+#include <string>
+
+#include "gnn_internal.h"
+
+namespace gnn {
+
+static thread_local std::string t_last_error;
+static std::atomic<uint64_t> g_launches{0};
+
+void set_error(const std::string &msg) { t_last_error = msg; }
+void count_launch(uint64_t k) { g_launches.fetch_add(k, std::memory_order_relaxed); }
+
+gnn_status cuda_status(cudaError_t e, const char *what) {
+  if (e == cudaSuccess) return GNN_OK;
+  set_error(std::string(what) + ": " + cudaGetErrorString(e));
+  return e == cudaErrorMemoryAllocation ? GNN_ERR_NOMEM : GNN_ERR_CUDA;
+}
+
+static double ms_since(std::chrono::steady_clock::time_point t0) {
+  return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+}
+
+static size_t align256(size_t b) { return (b + 255) & ~(size_t)255; }
+
+static void free_plan(gnn_plan_s *p) {
+  if (!p) return;
+  int cur = 0;
+  cudaGetDevice(&cur);
+  cudaSetDevice(p->device);
+  for (void *d : p->dev_allocs) cudaFree(d);
+  cudaSetDevice(cur);
+  delete p;
+}
+
+#define GNN_TRY(...)                                       \
+  try {                                                     \
+    __VA_ARGS__                                             \
+  } catch (const std::bad_alloc &) {                        \
+    gnn::set_error("host allocation failed");               \
+    return GNN_ERR_NOMEM;                                   \
+  } catch (const std::exception &ex) {                      \
+    gnn::set_error(std::string("internal: ") + ex.what()); \
+    return GNN_ERR_INTERNAL;                                \
+  } catch (...) {                                           \
+    gnn::set_error("internal: unknown exception");          \
+    return GNN_ERR_INTERNAL;                                \
+  }
+
+static gnn_status check(bool ok, const char *msg) {
+  if (ok) return GNN_OK;
+  set_error(msg);
+  return GNN_ERR_INVALID_ARG;
+}
+
+// overlap of [a, a + na) and [b, b + nb) in bytes
+static bool overlaps(const void *a, size_t na, const void *b, size_t nb) {
+  if (!a || !b || na == 0 || nb == 0) return false;
+  const char *x = (const char *)a, *y = (const char *)b;
+  return x < y + nb && y < x + na;
+}
+static size_t span_bytes(int64_t rows, int64_t ld, int64_t width) {
+  return rows <= 0 ? 0 : sizeof(float) * (size_t)((rows - 1) * ld + width);
+}
+
+}  // namespace gnn
+
+using namespace gnn;
+
+extern "C" {
+
+const char *gnn_last_error(void) { return t_last_error.c_str(); }
+const char *gnn_version(void) { return "gnn-b200 0.1 (sm_100a)"; }
+uint64_t gnn_launch_count(void) { return g_launches.load(); }
+
+void gnn_plan_opts_default(gnn_plan_opts *o) {
+  if (!o) return;
+  std::memset(o, 0, sizeof(*o));
+  o->struct_size = sizeof(gnn_plan_opts);
+  o->reorder = 0;
+  o->group_size = -1;
+  o->tile_groups = 32;
+  o->cluster_cap = 32;
+  o->minhash_k = 32;
+  o->lsh_rows = 2;
+  o->pair_window = 8;
+  o->min_sim = -1;
+  o->deterministic = 1;
+  o->seed = 0;
+}
+
+gnn_status gnn_plan_create_ex(int64_t n, int64_t n_src, int64_t nnz, const int64_t *rowptr_h,
+                              const int32_t *colidx_h, const int32_t *src_degree_h,
+                              const gnn_plan_opts *opts_in, gnn_plan_t *out) {
+  GNN_TRY({
+    if (!out) return check(false, "out is NULL");
+    *out = nullptr;
+    auto t0 = std::chrono::steady_clock::now();
+    gnn_plan_opts opts;
+    gnn_plan_opts_default(&opts);
+    if (opts_in) {
+      if (opts_in->struct_size != sizeof(gnn_plan_opts)) return check(false, "opts.struct_size mismatch");
+      opts = *opts_in;
+    }
+    if (n < 0 || n_src < 0 || nnz < 0 || n >= INT32_MAX || n_src >= INT32_MAX) {
+      set_error("negative or too large sizes");
+      return GNN_ERR_INVALID_GRAPH;
+    }
+    if (nnz >= INT32_MAX) {
+      set_error("nnz >= 2^31 is not supported (int32 device indices)");
+      return GNN_ERR_INVALID_GRAPH;
+    }
+    if (!rowptr_h || (nnz > 0 && !colidx_h)) return check(false, "rowptr/colidx is NULL");
+    if (opts.tile_groups == 0) opts.tile_groups = 32;
+    if (opts.tile_groups < 1 || opts.tile_groups > 256) return check(false, "tile_groups out of [1, 256]");
+    if (opts.reorder) {
+      if (opts.minhash_k < 1 || opts.minhash_k > 64) return check(false, "minhash_k out of [1, 64]");
+      if (opts.lsh_rows < 1 || opts.minhash_k % opts.lsh_rows) return check(false, "lsh_rows must divide minhash_k");
+      if (opts.pair_window < 1) return check(false, "pair_window < 1");
+      if (opts.cluster_cap < 1) return check(false, "cluster_cap < 1");
+    }
+    // a1: CSR validation, O(n + nnz)
+    if (rowptr_h[0] != 0 || rowptr_h[n] != nnz) {
+      set_error("rowptr[0] != 0 or rowptr[n] != nnz");
+      return GNN_ERR_INVALID_GRAPH;
+    }
+    int32_t maxd = 0;
+    for (int64_t v = 0; v < n; ++v) {
+      const int64_t d = rowptr_h[v + 1] - rowptr_h[v];
+      if (d < 0) {
+        set_error("rowptr is decreasing at row " + std::to_string(v));
+        return GNN_ERR_INVALID_GRAPH;
+      }
+      if (d > maxd) maxd = (int32_t)d;
+    }
+    for (int64_t k = 0; k < nnz; ++k)
+      if (colidx_h[k] < 0 || colidx_h[k] >= n_src) {
+        set_error("colidx out of range at entry " + std::to_string(k));
+        return GNN_ERR_INVALID_GRAPH;
+      }
+    gnn_plan_s *p = new gnn_plan_s();
+    p->n = n;
+    p->n_src = n_src;
+    p->nnz = nnz;
+    p->opts = opts;
+    p->max_degree = maxd;
+    p->T = opts.tile_groups;
+    // NG bound (R8-ii): largest multiple of 16 <= min(64, 10 * avg degree), >= 16
+    int64_t ng = opts.group_size;
+    if (ng < 0) {
+      const double avg = n > 0 ? (double)nnz / (double)n : 0.0;
+      ng = (int64_t)(std::min(64.0, 10.0 * avg) / 16.0) * 16;
+      if (ng < 16) ng = 16;
+    }
+    p->info.group_size = (int32_t)ng;
+    if (ng == 0) ng = 1 << 30;  // never split
+    p->ng = (int32_t)ng;
+    p->rowptr.assign(rowptr_h, rowptr_h + n + 1);
+    cudaGetDevice(&p->device);
+    p->info.ms_validate = ms_since(t0);
+
+    auto fail = [&](gnn_status st) {
+      free_plan(p);
+      return st;
+    };
+    // upload CSR (int32 on device)
+    t0 = std::chrono::steady_clock::now();
+    std::vector<int32_t> rp32((size_t)n + 1);
+    for (int64_t v = 0; v <= n; ++v) rp32[v] = (int32_t)rowptr_h[v];
+    void *d_rowptr = nullptr, *d_colidx = nullptr, *d_nsrc = nullptr, *d_ndst = nullptr, *d_dout = nullptr;
+    cudaError_t e = cudaMalloc(&d_rowptr, sizeof(int32_t) * (n + 1));
+    if (e == cudaSuccess) p->dev_allocs.push_back(d_rowptr);
+    if (e == cudaSuccess) e = cudaMalloc(&d_colidx, sizeof(int32_t) * (nnz > 0 ? nnz : 1));
+    if (e == cudaSuccess) p->dev_allocs.push_back(d_colidx);
+    if (e == cudaSuccess) e = cudaMalloc(&d_nsrc, sizeof(float) * (n_src > 0 ? n_src : 1));
+    if (e == cudaSuccess) p->dev_allocs.push_back(d_nsrc);
+    if (e == cudaSuccess) e = cudaMalloc(&d_ndst, sizeof(float) * (n > 0 ? n : 1));
+    if (e == cudaSuccess) p->dev_allocs.push_back(d_ndst);
+    if (e == cudaSuccess) e = cudaMalloc(&d_dout, sizeof(int32_t) * (n_src > 0 ? n_src : 1));
+    if (e == cudaSuccess) p->dev_allocs.push_back(d_dout);
+    if (e == cudaSuccess) e = cudaMemcpy(d_rowptr, rp32.data(), sizeof(int32_t) * (n + 1), cudaMemcpyHostToDevice);
+    if (e == cudaSuccess && nnz > 0)
+      e = cudaMemcpy(d_colidx, colidx_h, sizeof(int32_t) * nnz, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess && src_degree_h && n_src > 0)
+      e = cudaMemcpy(d_dout, src_degree_h, sizeof(int32_t) * n_src, cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) return fail(cuda_status(e, "plan allocation/upload"));
+    p->dg.rowptr = (const int32_t *)d_rowptr;
+    p->dg.colidx = (const int32_t *)d_colidx;
+    p->dg.nsrc = (const float *)d_nsrc;
+    p->dg.ndst = (const float *)d_ndst;
+    p->info.ms_upload = ms_since(t0);
+    // a1: degrees + normalisers on the GPU
+    t0 = std::chrono::steady_clock::now();
+    e = launch_degrees(p->dg.rowptr, p->dg.colidx, n, n_src, nnz,
+                       src_degree_h ? (const int32_t *)d_dout : nullptr, (int32_t *)d_dout,
+                       (float *)d_nsrc, (float *)d_ndst, nullptr);
+    if (e == cudaSuccess) e = cudaDeviceSynchronize();
+    if (e != cudaSuccess) return fail(cuda_status(e, "degrees"));
+    p->info.ms_degrees = ms_since(t0);
+    // a2: locality-aware task scheduling
+    if (opts.reorder && n > 0) {
+      t0 = std::chrono::steady_clock::now();
+      const int32_t K = opts.minhash_k;
+      uint64_t *d_sig = nullptr;
+      e = cudaMalloc(&d_sig, sizeof(uint64_t) * (size_t)n * K);
+      if (e != cudaSuccess) return fail(cuda_status(e, "minhash alloc"));
+      e = launch_minhash(p->dg.rowptr, p->dg.colidx, n, K, opts.seed, d_sig, nullptr);
+      p->sig.resize((size_t)n * K);
+      if (e == cudaSuccess)
+        e = cudaMemcpy(p->sig.data(), d_sig, sizeof(uint64_t) * (size_t)n * K, cudaMemcpyDeviceToHost);
+      cudaFree(d_sig);
+      if (e != cudaSuccess) return fail(cuda_status(e, "minhash"));
+      p->info.ms_minhash = ms_since(t0);
+      t0 = std::chrono::steady_clock::now();
+      const int64_t np = las_lsh_pairs(n, rowptr_h, p->sig.data(), K, opts.lsh_rows, opts.pair_window, p->pairs);
+      p->info.n_pairs = np;
+      p->info.ms_lsh = ms_since(t0);
+      t0 = std::chrono::steady_clock::now();
+      const int32_t min_sim = opts.min_sim < 0 ? opts.lsh_rows : opts.min_sim;
+      p->n_clusters = las_merge(n, p->sig.data(), K, p->pairs, opts.cluster_cap, min_sim, p->perm, p->cluster_of);
+      p->info.ms_merge = ms_since(t0);
+    } else {
+      p->perm.resize((size_t)n);
+      for (int64_t v = 0; v < n; ++v) p->perm[v] = (int32_t)v;
+      p->n_clusters = n;
+    }
+    // a3: neighbor grouping + tiles
+    t0 = std::chrono::steady_clock::now();
+    gnn_status st = build_schedule(p);
+    if (st != GNN_OK) return fail(st);
+    p->info.ms_ng = ms_since(t0);
+    p->info.n = n;
+    p->info.n_src = n_src;
+    p->info.nnz = nnz;
+    p->info.n_clusters = p->n_clusters;
+    p->info.tile_groups = p->T;
+    p->info.max_degree = maxd;
+    p->info.reorder = opts.reorder;
+    *out = p;
+    return GNN_OK;
+  })
+}
+
+gnn_status gnn_plan_create(int64_t n, int64_t nnz, const int64_t *rowptr_h, const int32_t *colidx_h,
+                           const gnn_plan_opts *opts, gnn_plan_t *out) {
+  return gnn_plan_create_ex(n, n, nnz, rowptr_h, colidx_h, nullptr, opts, out);
+}
+
+gnn_status gnn_plan_get_info(gnn_plan_t p, gnn_plan_info *info) {
+  if (!p || !info) return check(false, "plan/info is NULL");
+  *info = p->info;
+  return GNN_OK;
+}
+
+gnn_status gnn_plan_export(gnn_plan_t p, int32_t *perm_h, int32_t *grp_row_h, int64_t *grp_beg_h,
+                           int64_t *tile_beg_h) {
+  if (!p) return check(false, "plan is NULL");
+  if (perm_h) std::memcpy(perm_h, p->perm.data(), sizeof(int32_t) * p->perm.size());
+  if (grp_row_h) std::memcpy(grp_row_h, p->grp_row.data(), sizeof(int32_t) * p->grp_row.size());
+  if (grp_beg_h) std::memcpy(grp_beg_h, p->grp_beg.data(), sizeof(int64_t) * p->grp_beg.size());
+  if (tile_beg_h) std::memcpy(tile_beg_h, p->tile_beg.data(), sizeof(int64_t) * p->tile_beg.size());
+  return GNN_OK;
+}
+
+gnn_status gnn_plan_export_las(gnn_plan_t p, uint64_t *sig_h, int32_t *pairs_h, int32_t *cluster_of_h) {
+  if (!p) return check(false, "plan is NULL");
+  if (!p->opts.reorder) {
+    set_error("plan was built without reorder");
+    return GNN_ERR_INVALID_ARG;
+  }
+  if (sig_h) std::memcpy(sig_h, p->sig.data(), sizeof(uint64_t) * p->sig.size());
+  if (pairs_h) std::memcpy(pairs_h, p->pairs.data(), sizeof(int32_t) * p->pairs.size());
+  if (cluster_of_h) std::memcpy(cluster_of_h, p->cluster_of.data(), sizeof(int32_t) * p->cluster_of.size());
+  return GNN_OK;
+}
+
+gnn_status gnn_plan_normalizers(gnn_plan_t p, const float **nsrc, const float **ndst) {
+  if (!p) return check(false, "plan is NULL");
+  if (nsrc) *nsrc = p->dg.nsrc;
+  if (ndst) *ndst = p->dg.ndst;
+  return GNN_OK;
+}
+
+gnn_status gnn_plan_destroy(gnn_plan_t p) {
+  GNN_TRY({
+    free_plan(p);
+    return GNN_OK;
+  })
+}
+
+static size_t ws_gat_layer_head(int64_t n, int32_t f_in, int32_t HF, int32_t H, int32_t *ldwe) {
+  const int32_t ld = ((HF + 2 * H) + 7) / 8 * 8;
+  if (ldwe) *ldwe = ld;
+  return align256(sizeof(float) * (size_t)f_in * ld) + align256(sizeof(float) * (size_t)n * ld);
+}
+static size_t ws_edgeconv_head(int64_t n, int32_t f_in, int32_t f_out) {
+  const size_t ld = 2 * (size_t)f_out;
+  return align256(sizeof(float) * (size_t)f_in * ld) + align256(sizeof(float) * ld) +
+         align256(sizeof(float) * (size_t)n * ld);
+}
+static int32_t ld8(int32_t f) { return (f + 7) / 8 * 8; }
+
+size_t gnn_workspace_size(gnn_plan_t p, int op, int32_t f_in, int32_t f_out, int32_t heads) {
+  if (!p) return 0;
+  switch (op) {
+    case GNN_OP_AGGREGATE: return agg_workspace_bytes(p, 0, f_out, 0);
+    case GNN_OP_GAT_AGGREGATE: return agg_workspace_bytes(p, 3, f_out, heads);
+    case GNN_OP_EDGECONV: return ws_edgeconv_head(p->n, f_in, f_out) + agg_workspace_bytes(p, 2, f_out, 0);
+    case GNN_OP_GAT_LAYER:
+      return ws_gat_layer_head(p->n, f_in, f_out, heads, nullptr) + agg_workspace_bytes(p, 3, f_out, heads);
+    case GNN_OP_GCN_LAYER: {
+      const bool tf = f_out <= f_in;  // auto order; both orders fit in max()
+      (void)tf;
+      const size_t a = align256(sizeof(float) * (size_t)p->n_src * ld8(f_out)) + agg_workspace_bytes(p, 0, f_out, 0);
+      const size_t b = align256(sizeof(float) * (size_t)p->n * ld8(f_in)) + agg_workspace_bytes(p, 0, f_in, 0);
+      return a > b ? a : b;
+    }
+    default: return 0;
+  }
+}
+
+static gnn_status agg_common(gnn_plan_t p, AggArgs &a, void *ws, size_t ws_bytes, gnn_stream_t stream) {
+  a.deterministic = p->opts.deterministic;
+  return launch_aggregate(p, a, ws, ws_bytes, (cudaStream_t)stream);
+}
+
+gnn_status gnn_aggregate(gnn_plan_t p, int reduce, int weight, const float *edge_w, const float *X,
+                         int64_t ldx, int32_t F, float *Y, int64_t ldy, int32_t relu, const float *add_row,
+                         int64_t ld_add, void *ws, size_t ws_bytes, gnn_stream_t stream) {
+  GNN_TRY({
+    if (!p) return check(false, "plan is NULL");
+    if (reduce < 0 || reduce > 2) return check(false, "reduce out of range");
+    if (weight < 0 || weight > 2) return check(false, "weight out of range");
+    if (F < 0) return check(false, "F < 0");
+    if (F == 0) return GNN_OK;
+    if (!Y || (p->nnz > 0 && !X)) return check(false, "X/Y is NULL");
+    if (ldx < F || ldy < F) return check(false, "ld < F");
+    if (weight == GNN_W_EDGE && !edge_w && p->nnz > 0) return check(false, "edge_w required for GNN_W_EDGE");
+    if (add_row && ld_add < F) return check(false, "ld_add < F");
+    if (overlaps(X, span_bytes(p->n_src, ldx, F), Y, span_bytes(p->n, ldy, F)))
+      return check(false, "X and Y overlap");
+    AggArgs a{};
+    a.mode = reduce;
+    a.weight = weight;
+    a.edge_w = edge_w;
+    a.X = X;
+    a.ldx = ldx;
+    a.F = F;
+    a.Y = Y;
+    a.ldy = ldy;
+    a.add_row = add_row;
+    a.ld_add = ld_add;
+    a.relu = relu;
+    return agg_common(p, a, ws, ws_bytes, stream);
+  })
+}
+
+gnn_status gnn_gat_aggregate(gnn_plan_t p, const float *Zs, int64_t ldz, const float *t, int64_t ldt,
+                             int32_t H, int32_t Fh, float neg_slope, float *Y, int64_t ldy, void *ws,
+                             size_t ws_bytes, gnn_stream_t stream) {
+  GNN_TRY({
+    if (!p) return check(false, "plan is NULL");
+    if (H < 1 || Fh < 1) return check(false, "H and Fh must be >= 1");
+    const int32_t F = H * Fh;
+    if (!Y || !t || (p->nnz > 0 && !Zs)) return check(false, "Zs/t/Y is NULL");
+    if (ldz < F + H || ldt < H || ldy < F) return check(false, "ldz < H*Fh+H or ldt < H or ldy < H*Fh");
+    if (overlaps(Zs, span_bytes(p->n_src, ldz, F + H), Y, span_bytes(p->n, ldy, F)))
+      return check(false, "Zs and Y overlap");
+    AggArgs a{};
+    a.mode = 3;
+    a.X = Zs;
+    a.ldx = ldz;
+    a.F = F;
+    a.Y = Y;
+    a.ldy = ldy;
+    a.t = t;
+    a.ldt = ldt;
+    a.H = H;
+    a.Fh = Fh;
+    a.slope = neg_slope;
+    return agg_common(p, a, ws, ws_bytes, stream);
+  })
+}
+
+gnn_status gnn_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H, int64_t ldh,
+                    int64_t m, int32_t k, int32_t n, const float *row_scale, const float *col_bias,
+                    int32_t relu, gnn_stream_t stream) {
+  GNN_TRY({
+    if (m < 0 || k < 0 || n < 0) return check(false, "negative GEMM size");
+    if (m == 0 || n == 0) return GNN_OK;
+    if (!H || (k > 0 && (!X || !W))) return check(false, "X/W/H is NULL");
+    if (ldx < k || ldw < n || ldh < n) return check(false, "GEMM leading dimension too small");
+    if (overlaps(H, span_bytes(m, ldh, n), X, span_bytes(m, ldx, k)) ||
+        overlaps(H, span_bytes(m, ldh, n), W, span_bytes(k, ldw, n)))
+      return check(false, "H overlaps X or W");
+    return launch_gemm(X, ldx, W, ldw, H, ldh, m, k, n, row_scale, col_bias, relu, (cudaStream_t)stream);
+  })
+}
+
+int gnn_set_gemm_impl(int impl) { return set_gemm_impl(impl); }
+
+gnn_status gnn_gat_layer(gnn_plan_t p, const float *X, int64_t ldx, int32_t f_in, const float *W,
+                         const float *a_src, const float *a_dst, int32_t H, int32_t Fh, float neg_slope,
+                         float *Y, int64_t ldy, void *ws, size_t ws_bytes, gnn_stream_t stream) {
+  GNN_TRY({
+    if (!p) return check(false, "plan is NULL");
+    if (p->n != p->n_src) return check(false, "gnn_gat_layer needs a square plan (n_src == n)");
+    if (H < 1 || Fh < 1 || f_in < 1) return check(false, "H, Fh, f_in must be >= 1");
+    if (!X || !W || !a_src || !a_dst || !Y) return check(false, "NULL argument");
+    if (ldx < f_in || ldy < (int64_t)H * Fh) return check(false, "leading dimension too small");
+    const int32_t HF = H * Fh;
+    int32_t ldwe = 0;
+    const size_t head = ws_gat_layer_head(p->n, f_in, HF, H, &ldwe);
+    const size_t need = head + agg_workspace_bytes(p, 3, HF, H);
+    if (!ws || ws_bytes < need) {
+      set_error("workspace too small: need " + std::to_string(need));
+      return GNN_ERR_WORKSPACE;
+    }
+    char *base = (char *)ws;
+    float *Wext = (float *)base;
+    float *Zst = (float *)(base + align256(sizeof(float) * (size_t)f_in * ldwe));
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e = launch_gat_weights(W, a_src, a_dst, f_in, H, Fh, Wext, ldwe, s);
+    if (e != cudaSuccess) return cuda_status(e, "gat weights");
+    gnn_status st = launch_gemm(X, ldx, Wext, ldwe, Zst, ldwe, p->n, f_in, ldwe, nullptr, nullptr, 0, s);
+    if (st != GNN_OK) return st;
+    AggArgs a{};
+    a.mode = 3;
+    a.X = Zst;
+    a.ldx = ldwe;
+    a.F = HF;
+    a.Y = Y;
+    a.ldy = ldy;
+    a.t = Zst + HF + H;
+    a.ldt = ldwe;
+    a.H = H;
+    a.Fh = Fh;
+    a.slope = neg_slope;
+    return agg_common(p, a, base + head, ws_bytes - head, stream);
+  })
+}
+
+gnn_status gnn_edgeconv_aggregate(gnn_plan_t p, const float *PQ, int64_t ldpq, int32_t f_out, float *Y,
+                                  int64_t ldy, void *ws, size_t ws_bytes, gnn_stream_t stream) {
+  GNN_TRY({
+    if (!p) return check(false, "plan is NULL");
+    if (p->n != p->n_src) return check(false, "EdgeConv needs a square plan");
+    if (f_out < 1) return check(false, "f_out < 1");
+    if (!PQ || !Y) return check(false, "PQ/Y is NULL");
+    if (ldpq < 2 * (int64_t)f_out || ldy < f_out) return check(false, "leading dimension too small");
+    if (overlaps(PQ, span_bytes(p->n, ldpq, 2 * f_out), Y, span_bytes(p->n, ldy, f_out)))
+      return check(false, "PQ and Y overlap");
+    AggArgs a{};
+    a.mode = 2;
+    a.weight = GNN_W_ONE;
+    a.X = PQ;
+    a.ldx = ldpq;
+    a.F = f_out;
+    a.Y = Y;
+    a.ldy = ldy;
+    a.add_row = PQ + f_out;
+    a.ld_add = ldpq;
+    a.relu = 1;
+    return agg_common(p, a, ws, ws_bytes, stream);
+  })
+}
+
+gnn_status gnn_edgeconv(gnn_plan_t p, const float *X, int64_t ldx, int32_t f_in, const float *theta,
+                        const float *phi, const float *bias, int32_t f_out, float *Y, int64_t ldy, void *ws,
+                        size_t ws_bytes, gnn_stream_t stream) {
+  GNN_TRY({
+    if (!p) return check(false, "plan is NULL");
+    if (p->n != p->n_src) return check(false, "EdgeConv needs a square plan");
+    if (f_in < 1 || f_out < 1) return check(false, "f_in/f_out < 1");
+    if (!X || !theta || !phi || !Y) return check(false, "NULL argument");
+    if (ldx < f_in || ldy < f_out) return check(false, "leading dimension too small");
+    const size_t head = ws_edgeconv_head(p->n, f_in, f_out);
+    const size_t need = head + agg_workspace_bytes(p, 2, f_out, 0);
+    if (!ws || ws_bytes < need) {
+      set_error("workspace too small: need " + std::to_string(need));
+      return GNN_ERR_WORKSPACE;
+    }
+    const int64_t ld = 2 * (int64_t)f_out;
+    char *base = (char *)ws;
+    float *Wpq = (float *)base;
+    float *bpq = (float *)(base + align256(sizeof(float) * (size_t)f_in * ld));
+    float *PQ = (float *)((char *)bpq + align256(sizeof(float) * ld));
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e = launch_edgeconv_weights(theta, phi, bias, f_in, f_out, Wpq, bpq, s);
+    if (e != cudaSuccess) return cuda_status(e, "edgeconv weights");
+    gnn_status st = launch_gemm(X, ldx, Wpq, ld, PQ, ld, p->n, f_in, (int32_t)ld, nullptr, bpq, 0, s);
+    if (st != GNN_OK) return st;
+    return gnn_edgeconv_aggregate(p, PQ, ld, f_out, Y, ldy, base + head, ws_bytes - head, stream);
+  })
+}
+
+gnn_status gnn_gcn_layer(gnn_plan_t p, const float *X, int64_t ldx, int32_t f_in, const float *W, int64_t ldw,
+                         int32_t f_out, int32_t relu, int32_t order, float *Y, int64_t ldy, void *ws,
+                         size_t ws_bytes, gnn_stream_t stream) {
+  GNN_TRY({
+    if (!p) return check(false, "plan is NULL");
+    if (f_in < 1 || f_out < 1) return check(false, "f_in/f_out < 1");
+    if (!X || !W || !Y) return check(false, "NULL argument");
+    if (ldx < f_in || ldw < f_out || ldy < f_out) return check(false, "leading dimension too small");
+    if (order < 0 || order > 2) return check(false, "order out of range");
+    if (order == 0) order = f_out <= f_in ? 1 : 2;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (order == 1) {
+      // transform first: Hs = (X W) * nsrc[u]; y = ndst[v] * sum_u Hs[u]  (Eq 1 reassociated, R4-i)
+      const int32_t ldh = ld8(f_out);
+      const size_t head = align256(sizeof(float) * (size_t)p->n_src * ldh);
+      const size_t need = head + agg_workspace_bytes(p, 0, f_out, 0);
+      if (!ws || ws_bytes < need) {
+        set_error("workspace too small: need " + std::to_string(need));
+        return GNN_ERR_WORKSPACE;
+      }
+      float *Hs = (float *)ws;
+      gnn_status st = launch_gemm(X, ldx, W, ldw, Hs, ldh, p->n_src, f_in, f_out, p->dg.nsrc, nullptr, 0, s);
+      if (st != GNN_OK) return st;
+      AggArgs a{};
+      a.mode = 0;
+      a.weight = 3;  // W_DST_ONLY
+      a.X = Hs;
+      a.ldx = ldh;
+      a.F = f_out;
+      a.Y = Y;
+      a.ldy = ldy;
+      a.relu = relu;
+      return agg_common(p, a, (char *)ws + head, ws_bytes - head, stream);
+    }
+    // aggregate first: A = A_gcn X; Y = ACT(A W)
+    const int32_t lda = ld8(f_in);
+    const size_t head = align256(sizeof(float) * (size_t)p->n * lda);
+    const size_t need = head + agg_workspace_bytes(p, 0, f_in, 0);
+    if (!ws || ws_bytes < need) {
+      set_error("workspace too small: need " + std::to_string(need));
+      return GNN_ERR_WORKSPACE;
+    }
+    float *A = (float *)ws;
+    AggArgs a{};
+    a.mode = 0;
+    a.weight = GNN_W_GCN;
+    a.X = X;
+    a.ldx = ldx;
+    a.F = f_in;
+    a.Y = A;
+    a.ldy = lda;
+    gnn_status st = agg_common(p, a, (char *)ws + head, ws_bytes - head, stream);
+    if (st != GNN_OK) return st;
+    return launch_gemm(A, lda, W, ldw, Y, ldy, p->n, f_in, f_out, nullptr, nullptr, relu, s);
+  })
+}
+
+gnn_status gnn_gcn_aggregate_prescaled(gnn_plan_t p, const float *Hs, int64_t ldh, int32_t F, float *Y,
+                                       int64_t ldy, int32_t relu, void *ws, size_t ws_bytes, gnn_stream_t stream) {
+  GNN_TRY({
+    if (!p) return check(false, "plan is NULL");
+    if (F < 0) return check(false, "F < 0");
+    if (F == 0) return GNN_OK;
+    if (!Y || (p->nnz > 0 && !Hs)) return check(false, "Hs/Y is NULL");
+    if (ldh < F || ldy < F) return check(false, "ld < F");
+    if (overlaps(Hs, span_bytes(p->n_src, ldh, F), Y, span_bytes(p->n, ldy, F)))
+      return check(false, "Hs and Y overlap");
+    AggArgs a{};
+    a.mode = 0;
+    a.weight = 3;  // W_DST_ONLY: weight 1 in the loop, x ndst[v] in the epilogue
+    a.X = Hs;
+    a.ldx = ldh;
+    a.F = F;
+    a.Y = Y;
+    a.ldy = ldy;
+    a.relu = relu;
+    return agg_common(p, a, ws, ws_bytes, stream);
+  })
+}
+
+gnn_status gnn_gat_fold_weights(const float *W, const float *a_src, const float *a_dst, int32_t f_in, int32_t H,
+                                int32_t Fh, float *Wext, int64_t ldwe, gnn_stream_t stream) {
+  GNN_TRY({
+    if (!W || !a_src || !a_dst || !Wext) return check(false, "NULL argument");
+    if (f_in < 1 || H < 1 || Fh < 1) return check(false, "f_in, H, Fh must be >= 1");
+    if (ldwe < (int64_t)H * Fh + 2 * H) return check(false, "ldwe < H*Fh + 2H");
+    return cuda_status(launch_gat_weights(W, a_src, a_dst, f_in, H, Fh, Wext, (int32_t)ldwe, (cudaStream_t)stream),
+                       "gat fold");
+  })
+}
+
+gnn_status gnn_partition_rows(int64_t n, const int64_t *rowptr_h, int32_t nparts, int64_t *bounds_h) {
+  GNN_TRY({
+    if (n < 0 || nparts < 1 || !rowptr_h || !bounds_h) return check(false, "bad partition arguments");
+    const int64_t E = rowptr_h[n];
+    bounds_h[0] = 0;
+    for (int32_t q = 1; q < nparts; ++q) {
+      const int64_t target = (q * E + nparts - 1) / nparts;
+      // smallest i in [bounds[q-1], n] with rowptr[i] >= target (binary search)
+      int64_t lo = bounds_h[q - 1], hi = n;
+      while (lo < hi) {
+        const int64_t mid = lo + (hi - lo) / 2;
+        if (rowptr_h[mid] >= target) hi = mid;
+        else lo = mid + 1;
+      }
+      bounds_h[q] = lo;
+    }
+    bounds_h[nparts] = n;
+    return GNN_OK;
+  })
+}
+
+gnn_status gnn_local_csr(int64_t n, const int64_t *rowptr_h, const int32_t *colidx_h, const int64_t *bounds_h,
+                         int32_t nparts, int32_t rank, int64_t *r_max, int64_t *local_nnz,
+                         int64_t *local_rowptr_h, int32_t *local_colidx_h, int32_t *src_degree_h) {
+  GNN_TRY({
+    if (n < 0 || !rowptr_h || !bounds_h || nparts < 1 || rank < 0 || rank >= nparts || !r_max || !local_nnz)
+      return check(false, "bad local_csr arguments");
+    int64_t rm = 0;
+    for (int32_t q = 0; q < nparts; ++q) rm = std::max<int64_t>(rm, bounds_h[q + 1] - bounds_h[q]);
+    const int64_t lo = bounds_h[rank], hi = bounds_h[rank + 1];
+    *r_max = rm;
+    *local_nnz = rowptr_h[hi] - rowptr_h[lo];
+    if (!local_rowptr_h && !local_colidx_h && !src_degree_h) return GNN_OK;  // size query
+    // owner lookup: owner of u = the q with bounds[q] <= u < bounds[q+1]
+    auto owner = [&](int64_t u) {
+      int64_t a = 0, b = nparts - 1;
+      while (a < b) {
+        const int64_t mid = (a + b + 1) / 2;
+        if (bounds_h[mid] <= u) a = mid;
+        else b = mid - 1;
+      }
+      // skip empty parts that share the same bound
+      while (a + 1 < nparts && bounds_h[a + 1] <= u) ++a;
+      return a;
+    };
+    if (local_rowptr_h)
+      for (int64_t v = lo; v <= hi; ++v) local_rowptr_h[v - lo] = rowptr_h[v] - rowptr_h[lo];
+    if (local_colidx_h)
+      for (int64_t k = rowptr_h[lo]; k < rowptr_h[hi]; ++k) {
+        const int64_t u = colidx_h[k];
+        const int64_t q = owner(u);
+        local_colidx_h[k - rowptr_h[lo]] = (int32_t)(q * rm + (u - bounds_h[q]));
+      }
+    if (src_degree_h) {
+      std::memset(src_degree_h, 0, sizeof(int32_t) * (size_t)(nparts * rm));
+      for (int64_t k = 0; k < rowptr_h[n]; ++k) {
+        const int64_t u = colidx_h[k];
+        const int64_t q = owner(u);
+        src_degree_h[q * rm + (u - bounds_h[q])] += 1;
+      }
+    }
+    return GNN_OK;
+  })
+}
+
+gnn_status gnn_las_host(int64_t n, const int64_t *rowptr_h, const uint64_t *sig_h, int32_t K, int32_t r,
+                        int32_t W, int32_t cap, int32_t min_sim, int32_t *perm_h, int32_t *cluster_of_h,
+                        int64_t *n_pairs, int64_t *n_clusters) {
+  GNN_TRY({
+    if (n < 0 || !rowptr_h || (n > 0 && !sig_h) || !perm_h) return check(false, "bad las_host arguments");
+    if (K < 1 || r < 1 || K % r || W < 1 || cap < 1) return check(false, "bad LAS parameters");
+    std::vector<int32_t> pairs, perm, cl;
+    const int64_t np = las_lsh_pairs(n, rowptr_h, sig_h, K, r, W, pairs);
+    const int64_t nc = las_merge(n, sig_h, K, pairs, cap, min_sim < 0 ? r : min_sim, perm, cl);
+    std::memcpy(perm_h, perm.data(), sizeof(int32_t) * (size_t)n);
+    if (cluster_of_h) std::memcpy(cluster_of_h, cl.data(), sizeof(int32_t) * (size_t)n);
+    if (n_pairs) *n_pairs = np;
+    if (n_clusters) *n_clusters = nc;
+    return GNN_OK;
+  })
+}
+
+gnn_status gnn_groups_host(int64_t n, const int64_t *rowptr_h, const int32_t *perm_h, int32_t ng, int32_t T,
+                           int64_t *n_groups, int64_t *n_tiles, int32_t *grp_row_h, int64_t *grp_beg_h,
+                           int64_t *tile_beg_h) {
+  GNN_TRY({
+    if (n < 0 || !rowptr_h || !n_groups || !n_tiles || T < 1) return check(false, "bad groups_host arguments");
+    std::vector<int32_t> gr, ts, so, sf, sn;
+    std::vector<int64_t> gb, tb;
+    int64_t slots = 0;
+    schedule_host(n, rowptr_h, perm_h, ng > 0 ? ng : (1 << 30), T, gr, gb, tb, ts, so, sf, sn, slots);
+    *n_groups = (int64_t)gr.size();
+    *n_tiles = (int64_t)tb.size() - 1;
+    if (grp_row_h) std::memcpy(grp_row_h, gr.data(), sizeof(int32_t) * gr.size());
+    if (grp_beg_h) std::memcpy(grp_beg_h, gb.data(), sizeof(int64_t) * gb.size());
+    if (tile_beg_h) std::memcpy(tile_beg_h, tb.data(), sizeof(int64_t) * tb.size());
+    return GNN_OK;
+  })
+}
+
+}  // extern "C"

@@ -1,0 +1,121 @@
+// gnn_internal.h — private declarations of libgnn.so (never installed).
+// The public boundary is include/gnn.h.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "../../include/gnn.h"
+
+namespace gnn {
+
+// Device-side view of a plan handed to the graph kernels (all int32: the
+// plan rejects nnz >= 2^31).
+struct DevGraph {
+  const int32_t *rowptr;       // [n+1]
+  const int32_t *colidx;       // [nnz]
+  const float *nsrc;           // [n_src] 1/sqrtf(d_out)
+  const float *ndst;           // [n]     1/sqrtf(d_in)
+  const int32_t *grp_row;      // [G]
+  const int32_t *grp_beg;      // [G]
+  const int32_t *tile_beg;     // [n_tiles+1]
+  const int32_t *tile_split;   // [n_tiles] split-row index or -1
+  const int32_t *split_off;    // [n_split] first workspace slot of the split row
+  const int32_t *split_first;  // [n_split] global index of the row's first group
+  const int32_t *split_ntiles; // [n_split]
+  const int32_t *empty_rows;   // [n_empty]
+  int32_t n_tiles, n_split, n_empty, ng;
+};
+
+}  // namespace gnn
+
+struct gnn_plan_s {
+  int device = 0;
+  int64_t n = 0, n_src = 0, nnz = 0;
+  gnn_plan_opts opts{};
+  int32_t ng = 0;      // effective group bound (INT32_MAX-ish when "never split")
+  int32_t T = 32;
+  int32_t max_degree = 0;
+  // host copies
+  std::vector<int64_t> rowptr;
+  std::vector<int32_t> perm, grp_row;
+  std::vector<int64_t> grp_beg, tile_beg;
+  std::vector<uint64_t> sig;
+  std::vector<int32_t> pairs, cluster_of;
+  int64_t n_clusters = 0, n_split = 0, n_empty = 0, split_slots = 0;
+  gnn_plan_info info{};
+  // device allocations (owned)
+  std::vector<void *> dev_allocs;
+  gnn::DevGraph dg{};
+};
+
+namespace gnn {
+
+// error plumbing (api.cpp)
+void set_error(const std::string &msg);
+gnn_status cuda_status(cudaError_t e, const char *what);
+void count_launch(uint64_t k = 1);
+
+// planner (plan.cpp) — host side
+gnn_status build_schedule(gnn_plan_s *p);
+void schedule_host(int64_t n, const int64_t *rowptr, const int32_t *perm, int64_t ng, int32_t T,
+                   std::vector<int32_t> &grp_row, std::vector<int64_t> &grp_beg,
+                   std::vector<int64_t> &tile_beg, std::vector<int32_t> &tile_split,
+                   std::vector<int32_t> &split_off, std::vector<int32_t> &split_first,
+                   std::vector<int32_t> &split_ntiles, int64_t &slots);
+int64_t las_lsh_pairs(int64_t n, const int64_t *rowptr, const uint64_t *sig, int32_t K, int32_t r,
+                      int32_t W, std::vector<int32_t> &pairs);
+int64_t las_merge(int64_t n, const uint64_t *sig, int32_t K, const std::vector<int32_t> &pairs,
+                  int32_t cap, int32_t min_sim, std::vector<int32_t> &perm,
+                  std::vector<int32_t> &cluster_of);
+
+// kernels (k_graph.cu)
+cudaError_t launch_degrees(const int32_t *rowptr, const int32_t *colidx, int64_t n, int64_t n_src,
+                           int64_t nnz, const int32_t *src_degree_override, int32_t *d_out_tmp,
+                           float *nsrc, float *ndst, cudaStream_t s);
+cudaError_t launch_minhash(const int32_t *rowptr, const int32_t *colidx, int64_t n, int32_t K,
+                           uint64_t seed, uint64_t *sig, cudaStream_t s);
+
+struct AggArgs {
+  int mode;            // 0 sum, 1 mean, 2 max, 3 gat
+  int weight;          // gnn_weight (sum/mean/max)
+  const float *edge_w;
+  const float *X;
+  int64_t ldx;
+  int32_t F;
+  float *Y;
+  int64_t ldy;
+  const float *add_row;
+  int64_t ld_add;
+  int32_t relu;
+  // GAT
+  const float *t;
+  int64_t ldt;
+  int32_t H, Fh;
+  float slope;
+  // split-row workspace
+  float *ws_part;
+  int32_t *ws_cnt;
+  int32_t deterministic;
+};
+size_t agg_workspace_bytes(const gnn_plan_s *p, int mode, int32_t F, int32_t H);
+gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, size_t ws_bytes,
+                            cudaStream_t s);
+
+// GEMM (k_gemm.cu)
+gnn_status launch_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H,
+                       int64_t ldh, int64_t m, int32_t k, int32_t n, const float *row_scale,
+                       const float *col_bias, int32_t relu, cudaStream_t s);
+int set_gemm_impl(int impl);
+
+// small helper kernels (k_graph.cu)
+cudaError_t launch_gat_weights(const float *W, const float *a_src, const float *a_dst, int32_t f_in,
+                               int32_t H, int32_t Fh, float *Wext, int32_t ldwe, cudaStream_t s);
+cudaError_t launch_edgeconv_weights(const float *theta, const float *phi, const float *bias,
+                                    int32_t f_in, int32_t f_out, float *Wpq, float *bpq,
+                                    cudaStream_t s);
+
+}  // namespace gnn

@@ -1,0 +1,336 @@
+// plan.cpp — host side of the planner (libgnn.so):
+//   a2 steps 2-5 of locality-aware task scheduling (LSH banding, candidate
+//      pairs, similarity, capped pair merging, cluster schedule);
+//   a3 neighbor grouping and CTA work tiles (reading R8).
+// MinHash signatures (a2 step 1) come from the GPU kernel in k_graph.cu.
+// This is an independent implementation of the same integer specification
+// the oracle follows (R7/R8): results must be bit-identical.
+#include <algorithm>
+#include <chrono>
+#include <cstring>
+#include <queue>
+#include <thread>
+#include <vector>
+
+#include "gnn_internal.h"
+
+namespace gnn {
+
+namespace {
+
+struct BandKey {
+  uint64_t b0, b1;  // band tuple (r <= 2 handled directly; r > 2 hashed into rank order below)
+  uint32_t rank;    // position of the node in (full signature, id) order
+  uint32_t id;
+  bool operator<(const BandKey &o) const {
+    if (b0 != o.b0) return b0 < o.b0;
+    if (b1 != o.b1) return b1 < o.b1;
+    return rank < o.rank;
+  }
+};
+
+}  // namespace
+
+// LSH banding: for band j, non-empty nodes ordered by (band
+// tuple, full signature, id); buckets = runs of equal band tuple; candidate
+// pairs (m_i, m_{i+d}), 1 <= d <= W.  Union over bands, dedup, sorted.
+int64_t las_lsh_pairs(int64_t n, const int64_t *rowptr, const uint64_t *sig, int32_t K, int32_t r,
+                      int32_t W, std::vector<int32_t> &pairs) {
+  const int32_t nb = K / r;
+  std::vector<uint32_t> nodes;
+  nodes.reserve((size_t)n);
+  for (int64_t v = 0; v < n; ++v)
+    if (rowptr[v + 1] > rowptr[v]) nodes.push_back((uint32_t)v);
+  // rank by (full signature, id)
+  std::vector<uint32_t> order(nodes);
+  std::sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) {
+    const uint64_t *sa = sig + (size_t)a * K, *sb = sig + (size_t)b * K;
+    for (int32_t k = 0; k < K; ++k)
+      if (sa[k] != sb[k]) return sa[k] < sb[k];
+    return a < b;
+  });
+  std::vector<uint32_t> rank((size_t)n, 0);
+  for (size_t i = 0; i < order.size(); ++i) rank[order[i]] = (uint32_t)i;
+
+  const unsigned nthreads = std::max(1u, std::min(8u, std::thread::hardware_concurrency()));
+  std::vector<std::vector<uint64_t>> local(nthreads);
+  auto work = [&](unsigned tid) {
+    std::vector<BandKey> keys(nodes.size());
+    std::vector<uint64_t> &out = local[tid];
+    for (int32_t j = (int32_t)tid; j < nb; j += (int32_t)nthreads) {
+      for (size_t i = 0; i < nodes.size(); ++i) {
+        const uint32_t v = nodes[i];
+        const uint64_t *s = sig + (size_t)v * K + (size_t)j * r;
+        BandKey bk;
+        bk.b0 = s[0];
+        bk.b1 = r > 1 ? s[1] : 0;
+        bk.rank = rank[v];
+        bk.id = v;
+        keys[i] = bk;
+      }
+      std::sort(keys.begin(), keys.end());
+      auto same_band = [&](const BandKey &x, const BandKey &y) {
+        if (x.b0 != y.b0 || x.b1 != y.b1) return false;
+        for (int32_t q = 2; q < r; ++q)
+          if (sig[(size_t)x.id * K + (size_t)j * r + q] != sig[(size_t)y.id * K + (size_t)j * r + q])
+            return false;
+        return true;
+      };
+      size_t s0 = 0;
+      while (s0 < keys.size()) {
+        size_t e = s0 + 1;
+        while (e < keys.size() && same_band(keys[s0], keys[e])) ++e;
+        for (size_t i = s0; i < e; ++i)
+          for (int32_t d = 1; d <= W && i + (size_t)d < e; ++d) {
+            uint32_t a = keys[i].id, b = keys[i + d].id;
+            if (a > b) std::swap(a, b);
+            out.push_back(((uint64_t)a << 32) | b);
+          }
+        s0 = e;
+      }
+    }
+  };
+  if (r > 2) {
+    // band tuples longer than 2: fall back to an exact comparator on the tuple
+    // (rank order still breaks ties), single-threaded
+    for (int32_t j = 0; j < nb; ++j) {
+      std::vector<uint32_t> ord(nodes);
+      std::sort(ord.begin(), ord.end(), [&](uint32_t a, uint32_t b) {
+        const uint64_t *sa = sig + (size_t)a * K + (size_t)j * r, *sb = sig + (size_t)b * K + (size_t)j * r;
+        for (int32_t q = 0; q < r; ++q)
+          if (sa[q] != sb[q]) return sa[q] < sb[q];
+        return rank[a] < rank[b];
+      });
+      auto eq = [&](uint32_t a, uint32_t b) {
+        return std::memcmp(sig + (size_t)a * K + (size_t)j * r, sig + (size_t)b * K + (size_t)j * r,
+                           sizeof(uint64_t) * r) == 0;
+      };
+      size_t s0 = 0;
+      while (s0 < ord.size()) {
+        size_t e = s0 + 1;
+        while (e < ord.size() && eq(ord[s0], ord[e])) ++e;
+        for (size_t i = s0; i < e; ++i)
+          for (int32_t d = 1; d <= W && i + (size_t)d < e; ++d) {
+            uint32_t a = ord[i], b = ord[i + d];
+            if (a > b) std::swap(a, b);
+            local[0].push_back(((uint64_t)a << 32) | b);
+          }
+        s0 = e;
+      }
+    }
+  } else {
+    std::vector<std::thread> th;
+    for (unsigned t = 0; t < nthreads; ++t) th.emplace_back(work, t);
+    for (auto &t : th) t.join();
+  }
+  size_t tot = 0;
+  for (auto &l : local) tot += l.size();
+  std::vector<uint64_t> all;
+  all.reserve(tot);
+  for (auto &l : local) {
+    all.insert(all.end(), l.begin(), l.end());
+    std::vector<uint64_t>().swap(l);
+  }
+  std::sort(all.begin(), all.end());
+  all.erase(std::unique(all.begin(), all.end()), all.end());
+  pairs.resize(all.size() * 2);
+  for (size_t i = 0; i < all.size(); ++i) {
+    pairs[2 * i] = (int32_t)(all[i] >> 32);
+    pairs[2 * i + 1] = (int32_t)(all[i] & 0xffffffffu);
+  }
+  return (int64_t)all.size();
+}
+
+namespace {
+struct HEnt {
+  int32_t sim, a, b;
+};
+struct HCmp {  // priority_queue pops the "largest": sim desc, a asc, b asc
+  bool operator()(const HEnt &x, const HEnt &y) const {
+    if (x.sim != y.sim) return x.sim < y.sim;
+    if (x.a != y.a) return x.a > y.a;
+    return x.b > y.b;
+  }
+};
+inline int32_t sim_of(const uint64_t *sig, int32_t K, int64_t a, int64_t b) {
+  const uint64_t *sa = sig + (size_t)a * K, *sb = sig + (size_t)b * K;
+  int32_t s = 0;
+  for (int32_t k = 0; k < K; ++k) s += sa[k] == sb[k];
+  return s;
+}
+}  // namespace
+
+// Pair merging and task scheduling; spec R7.
+int64_t las_merge(int64_t n, const uint64_t *sig, int32_t K, const std::vector<int32_t> &pairs,
+                  int32_t cap, int32_t min_sim, std::vector<int32_t> &perm,
+                  std::vector<int32_t> &cluster_of) {
+  std::vector<int32_t> parent((size_t)n), size((size_t)n, 1);
+  for (int64_t v = 0; v < n; ++v) parent[v] = (int32_t)v;
+  auto find = [&](int64_t x) {
+    int64_t r = x;
+    while (parent[r] != r) r = parent[r];
+    while (parent[x] != r) {
+      int64_t nx = parent[x];
+      parent[x] = (int32_t)r;
+      x = nx;
+    }
+    return r;
+  };
+  const size_t np = pairs.size() / 2;
+  std::vector<HEnt> init(np);
+  for (size_t i = 0; i < np; ++i)
+    init[i] = HEnt{sim_of(sig, K, pairs[2 * i], pairs[2 * i + 1]), pairs[2 * i], pairs[2 * i + 1]};
+  std::priority_queue<HEnt, std::vector<HEnt>, HCmp> pq(HCmp(), std::move(init));
+  while (!pq.empty()) {
+    const HEnt e = pq.top();
+    pq.pop();
+    if (parent[e.a] == e.a && parent[e.b] == e.b) {
+      if (size[e.a] + size[e.b] <= cap) {
+        int32_t keep = (size[e.a] != size[e.b]) ? (size[e.a] > size[e.b] ? e.a : e.b) : std::min(e.a, e.b);
+        int32_t gone = keep == e.a ? e.b : e.a;
+        parent[gone] = keep;
+        size[keep] += size[gone];
+      }
+    } else {
+      const int64_t ra = find(e.a), rb = find(e.b);
+      if (ra != rb && size[ra] + size[rb] <= cap) {
+        const int32_t s = sim_of(sig, K, ra, rb);
+        if (s >= min_sim) pq.push(HEnt{s, (int32_t)std::min(ra, rb), (int32_t)std::max(ra, rb)});
+      }
+    }
+  }
+  // clusters ordered by smallest member, members ascending
+  std::vector<int64_t> cnt((size_t)n, 0), off((size_t)n, -1);
+  for (int64_t v = 0; v < n; ++v) cnt[find(v)]++;
+  perm.assign((size_t)n, 0);
+  cluster_of.assign((size_t)n, 0);
+  int64_t pos = 0, nc = 0;
+  for (int64_t v = 0; v < n; ++v) {
+    const int64_t r = find(v);
+    if (off[r] < 0) {
+      off[r] = pos;
+      pos += cnt[r];
+      ++nc;
+    }
+    perm[off[r]++] = (int32_t)v;
+    cluster_of[v] = (int32_t)r;
+  }
+  return nc;
+}
+
+// a3: neighbor groups in schedule order + tiles + split-row
+// tables (reading R8).  Pure host function, also exported as gnn_groups_host.
+void schedule_host(int64_t n, const int64_t *rowptr, const int32_t *perm, int64_t ng, int32_t T,
+                   std::vector<int32_t> &grp_row, std::vector<int64_t> &grp_beg,
+                   std::vector<int64_t> &tile_beg, std::vector<int32_t> &tile_split,
+                   std::vector<int32_t> &split_off, std::vector<int32_t> &split_first,
+                   std::vector<int32_t> &split_ntiles, int64_t &slots) {
+  grp_row.clear();
+  grp_beg.clear();
+  for (int64_t i = 0; i < n; ++i) {
+    const int64_t v = perm ? perm[i] : i;
+    const int64_t beg = rowptr[v], end = rowptr[v + 1];
+    for (int64_t b = beg; b < end; b += ng) {
+      grp_row.push_back((int32_t)v);
+      grp_beg.push_back(b);
+      if (end - b <= ng) break;
+    }
+  }
+  const int64_t G = (int64_t)grp_row.size();
+  // tiles: first-fit of whole runs, runs longer than T get their own tiles
+  tile_beg.assign(1, 0);
+  tile_split.clear();
+  split_off.clear();
+  split_first.clear();
+  split_ntiles.clear();
+  slots = 0;
+  int64_t cur = 0, g = 0;
+  while (g < G) {
+    int64_t e = g + 1;
+    while (e < G && grp_row[e] == grp_row[g]) ++e;
+    const int64_t run = e - g;
+    if (run > T) {
+      if (cur > 0) {
+        tile_beg.push_back(g);
+        tile_split.push_back(-1);
+        cur = 0;
+      }
+      const int32_t s = (int32_t)split_off.size();
+      split_off.push_back((int32_t)slots);
+      split_first.push_back((int32_t)g);
+      split_ntiles.push_back((int32_t)((run + T - 1) / T));
+      slots += run;
+      for (int64_t s0 = g; s0 < e; s0 += T) {
+        tile_beg.push_back(std::min<int64_t>(s0 + T, e));
+        tile_split.push_back(s);
+      }
+    } else {
+      if (cur + run > T) {
+        tile_beg.push_back(g);
+        tile_split.push_back(-1);
+        cur = 0;
+      }
+      cur += run;
+    }
+    g = e;
+  }
+  if (cur > 0) {
+    tile_beg.push_back(G);
+    tile_split.push_back(-1);
+  }
+}
+
+gnn_status build_schedule(gnn_plan_s *p) {
+  const int64_t n = p->n;
+  std::vector<int32_t> tile_split, split_off, split_first, split_ntiles;
+  int64_t slots = 0;
+  schedule_host(n, p->rowptr.data(), p->perm.data(), p->ng, p->T, p->grp_row, p->grp_beg, p->tile_beg,
+                tile_split, split_off, split_first, split_ntiles, slots);
+  const int64_t G = (int64_t)p->grp_row.size();
+  const int64_t n_tiles = (int64_t)p->tile_beg.size() - 1;
+  p->n_split = (int64_t)split_off.size();
+  p->split_slots = slots;
+  std::vector<int32_t> empty;
+  for (int64_t v = 0; v < n; ++v)
+    if (p->rowptr[v + 1] == p->rowptr[v]) empty.push_back((int32_t)v);
+  p->n_empty = (int64_t)empty.size();
+
+  // upload (int32 on device)
+  auto upload = [&](const void *src, size_t bytes, void **dst) -> cudaError_t {
+    *dst = nullptr;
+    cudaError_t e = cudaMalloc(dst, bytes > 0 ? bytes : 4);
+    if (e != cudaSuccess) return e;
+    p->dev_allocs.push_back(*dst);
+    if (bytes > 0) e = cudaMemcpy(*dst, src, bytes, cudaMemcpyHostToDevice);
+    return e;
+  };
+  std::vector<int32_t> grp_beg32((size_t)G), tile_beg32((size_t)n_tiles + 1);
+  for (int64_t i = 0; i < G; ++i) grp_beg32[i] = (int32_t)p->grp_beg[i];
+  for (int64_t i = 0; i <= n_tiles; ++i) tile_beg32[i] = (int32_t)p->tile_beg[i];
+  void *d;
+  cudaError_t e;
+#define UP(vec, field)                                                                 \
+  e = upload((vec).data(), sizeof(int32_t) * (vec).size(), &d);                       \
+  if (e != cudaSuccess) return cuda_status(e, "plan upload");                         \
+  p->dg.field = reinterpret_cast<const int32_t *>(d);
+  UP(p->grp_row, grp_row)
+  UP(grp_beg32, grp_beg)
+  UP(tile_beg32, tile_beg)
+  UP(tile_split, tile_split)
+  UP(split_off, split_off)
+  UP(split_first, split_first)
+  UP(split_ntiles, split_ntiles)
+  UP(empty, empty_rows)
+#undef UP
+  p->dg.n_tiles = (int32_t)n_tiles;
+  p->dg.n_split = (int32_t)p->n_split;
+  p->dg.n_empty = (int32_t)p->n_empty;
+  p->dg.ng = p->ng;
+  p->info.n_groups = G;
+  p->info.n_tiles = n_tiles;
+  p->info.n_split_rows = p->n_split;
+  p->info.n_empty_rows = p->n_empty;
+  return GNN_OK;
+}
+
+}  // namespace gnn

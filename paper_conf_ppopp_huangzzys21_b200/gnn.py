@@ -1,0 +1,361 @@
+"""Thin Python binding of libgnn.so (include/gnn.h) — argument marshalling only.
+
+Every C entry point is exposed under its C name (``gnn_plan_create``,
+``gnn_aggregate``, ...) taking raw pointers/ints exactly like the C-ABI.  On
+top sit small torch-tensor conveniences (``Plan``, ``aggregate``,
+``gat_aggregate``, ...) that only read ``data_ptr()``/``stride()`` and allocate
+outputs/workspace with torch; every step of the path runs in the library's
+sm_100a kernels.  There is NO CPU or Python fallback: if libgnn.so is missing
+or fails to load, importing this module raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libgnn.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"{LIB_PATH} not built: run `python -m paper_conf_ppopp_huangzzys21_b200.build` "
+                      "(or __graft_entry__.build()); there is no fallback path")
+_lib = ctypes.CDLL(LIB_PATH)
+
+GNN_OK = 0
+STATUS = {0: "GNN_OK", 1: "GNN_ERR_INVALID_ARG", 2: "GNN_ERR_INVALID_GRAPH", 3: "GNN_ERR_WORKSPACE",
+          4: "GNN_ERR_CUDA", 5: "GNN_ERR_NOMEM", 6: "GNN_ERR_UNSUPPORTED", 7: "GNN_ERR_INTERNAL"}
+GNN_SUM, GNN_MEAN, GNN_MAX = 0, 1, 2
+GNN_W_ONE, GNN_W_GCN, GNN_W_EDGE = 0, 1, 2
+GNN_OP_AGGREGATE, GNN_OP_GAT_AGGREGATE, GNN_OP_EDGECONV, GNN_OP_GCN_LAYER, GNN_OP_GAT_LAYER = range(5)
+REDUCE = {"sum": GNN_SUM, "mean": GNN_MEAN, "max": GNN_MAX}
+WEIGHT = {"one": GNN_W_ONE, "gcn": GNN_W_GCN, "edge": GNN_W_EDGE}
+
+
+class GnnError(RuntimeError):
+    def __init__(self, fn, status):
+        self.status = status
+        super().__init__(f"{fn} -> {STATUS.get(status, status)}: {gnn_last_error()}")
+
+
+class gnn_plan_opts(ctypes.Structure):
+    _fields_ = [("struct_size", ctypes.c_uint32), ("reorder", ctypes.c_int32), ("group_size", ctypes.c_int32),
+                ("tile_groups", ctypes.c_int32), ("cluster_cap", ctypes.c_int32), ("minhash_k", ctypes.c_int32),
+                ("lsh_rows", ctypes.c_int32), ("pair_window", ctypes.c_int32), ("min_sim", ctypes.c_int32),
+                ("deterministic", ctypes.c_int32), ("seed", ctypes.c_uint64)]
+
+
+class gnn_plan_info(ctypes.Structure):
+    _fields_ = [(k, ctypes.c_int64) for k in ("n", "n_src", "nnz", "n_groups", "n_tiles", "n_split_rows",
+                                                "n_empty_rows", "n_clusters", "n_pairs")] + \
+               [(k, ctypes.c_int32) for k in ("group_size", "tile_groups", "max_degree", "reorder")] + \
+               [(k, ctypes.c_double) for k in ("ms_validate", "ms_upload", "ms_degrees", "ms_minhash", "ms_lsh",
+                                                 "ms_merge", "ms_ng")]
+
+
+_P = ctypes.c_void_p
+_I64 = ctypes.c_int64
+_I32 = ctypes.c_int32
+_SZ = ctypes.c_size_t
+_F = ctypes.c_float
+
+_SIGS = {
+    "gnn_plan_opts_default": (None, [ctypes.POINTER(gnn_plan_opts)]),
+    "gnn_plan_create": (ctypes.c_int, [_I64, _I64, _P, _P, ctypes.POINTER(gnn_plan_opts), ctypes.POINTER(_P)]),
+    "gnn_plan_create_ex": (ctypes.c_int, [_I64, _I64, _I64, _P, _P, _P, ctypes.POINTER(gnn_plan_opts),
+                                          ctypes.POINTER(_P)]),
+    "gnn_plan_get_info": (ctypes.c_int, [_P, ctypes.POINTER(gnn_plan_info)]),
+    "gnn_plan_export": (ctypes.c_int, [_P, _P, _P, _P, _P]),
+    "gnn_plan_export_las": (ctypes.c_int, [_P, _P, _P, _P]),
+    "gnn_plan_normalizers": (ctypes.c_int, [_P, ctypes.POINTER(_P), ctypes.POINTER(_P)]),
+    "gnn_plan_destroy": (ctypes.c_int, [_P]),
+    "gnn_workspace_size": (_SZ, [_P, ctypes.c_int, _I32, _I32, _I32]),
+    "gnn_aggregate": (ctypes.c_int, [_P, ctypes.c_int, ctypes.c_int, _P, _P, _I64, _I32, _P, _I64, _I32, _P, _I64,
+                                     _P, _SZ, _P]),
+    "gnn_gat_aggregate": (ctypes.c_int, [_P, _P, _I64, _P, _I64, _I32, _I32, _F, _P, _I64, _P, _SZ, _P]),
+    "gnn_gat_layer": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _P, _P, _I32, _I32, _F, _P, _I64, _P, _SZ, _P]),
+    "gnn_edgeconv_aggregate": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _I64, _P, _SZ, _P]),
+    "gnn_edgeconv": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _P, _P, _I32, _P, _I64, _P, _SZ, _P]),
+    "gnn_gemm": (ctypes.c_int, [_P, _I64, _P, _I64, _P, _I64, _I64, _I32, _I32, _P, _P, _I32, _P]),
+    "gnn_set_gemm_impl": (ctypes.c_int, [ctypes.c_int]),
+    "gnn_gcn_layer": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _I64, _I32, _I32, _I32, _P, _I64, _P, _SZ, _P]),
+    "gnn_gcn_aggregate_prescaled": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _I64, _I32, _P, _SZ, _P]),
+    "gnn_gat_fold_weights": (ctypes.c_int, [_P, _P, _P, _I32, _I32, _I32, _P, _I64, _P]),
+    "gnn_partition_rows": (ctypes.c_int, [_I64, _P, _I32, _P]),
+    "gnn_local_csr": (ctypes.c_int, [_I64, _P, _P, _P, _I32, _I32, ctypes.POINTER(_I64), ctypes.POINTER(_I64),
+                                     _P, _P, _P]),
+    "gnn_las_host": (ctypes.c_int, [_I64, _P, _P, _I32, _I32, _I32, _I32, _I32, _P, _P, ctypes.POINTER(_I64),
+                                    ctypes.POINTER(_I64)]),
+    "gnn_groups_host": (ctypes.c_int, [_I64, _P, _P, _I32, _I32, ctypes.POINTER(_I64), ctypes.POINTER(_I64), _P, _P,
+                                       _P]),
+    "gnn_launch_count": (ctypes.c_uint64, []),
+    "gnn_last_error": (ctypes.c_char_p, []),
+    "gnn_version": (ctypes.c_char_p, []),
+}
+
+EXPORTED = sorted(_SIGS)
+
+for _name, (_res, _args) in _SIGS.items():
+    _f = getattr(_lib, _name)
+    _f.restype = _res
+    _f.argtypes = _args
+    globals()[_name] = _f
+
+
+def gnn_last_error() -> str:  # noqa: F811 — decode the C string
+    return _lib.gnn_last_error().decode()
+
+
+def gnn_version() -> str:  # noqa: F811
+    return _lib.gnn_version().decode()
+
+
+def _call(name, *args):
+    st = getattr(_lib, name)(*args)
+    if st != GNN_OK:
+        raise GnnError(name, st)
+
+
+# --------------------------------------------------------------------------- #
+# torch conveniences (marshalling only)
+# --------------------------------------------------------------------------- #
+def _torch():
+    import torch
+    return torch
+
+
+def _np_ptr(a):
+    return None if a is None else a.ctypes.data
+
+
+def _tp(t):
+    return None if t is None else ctypes.c_void_p(t.data_ptr())
+
+
+def _ld(t, width):
+    assert t.dtype == _torch().float32, "fp32 tensors only"
+    assert t.dim() == 2 and t.stride(1) == 1, "row-major 2-D tensors only"
+    assert t.shape[1] >= width
+    return t.stride(0)
+
+
+def _stream(stream):
+    torch = _torch()
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def default_opts(**kw) -> gnn_plan_opts:
+    o = gnn_plan_opts()
+    _lib.gnn_plan_opts_default(ctypes.byref(o))
+    for k, v in kw.items():
+        setattr(o, k, v)
+    return o
+
+
+class Plan:
+    """Owns a gnn_plan_t built from a host CSR (numpy int64 rowptr, int32 colidx)."""
+
+    def __init__(self, rowptr, colidx, n_src=None, src_degree=None, **opts):
+        rowptr = np.ascontiguousarray(rowptr, dtype=np.int64)
+        colidx = np.ascontiguousarray(colidx, dtype=np.int32)
+        self.n = len(rowptr) - 1
+        self.nnz = int(rowptr[-1])
+        self.n_src = self.n if n_src is None else int(n_src)
+        self.opts = default_opts(**opts)
+        h = ctypes.c_void_p()
+        sd = None if src_degree is None else np.ascontiguousarray(src_degree, dtype=np.int32)
+        _call("gnn_plan_create_ex", self.n, self.n_src, self.nnz, _np_ptr(rowptr), _np_ptr(colidx), _np_ptr(sd),
+              ctypes.byref(self.opts), ctypes.byref(h))
+        self.handle = h
+        self._ws = {}
+
+    @property
+    def info(self) -> dict:
+        i = gnn_plan_info()
+        _call("gnn_plan_get_info", self.handle, ctypes.byref(i))
+        return {k: getattr(i, k) for k, _ in gnn_plan_info._fields_}
+
+    def export(self):
+        info = self.info
+        perm = np.empty(self.n, np.int32)
+        gr = np.empty(max(info["n_groups"], 1), np.int32)
+        gb = np.empty(max(info["n_groups"], 1), np.int64)
+        tb = np.empty(info["n_tiles"] + 1, np.int64)
+        _call("gnn_plan_export", self.handle, _np_ptr(perm), _np_ptr(gr), _np_ptr(gb), _np_ptr(tb))
+        G = info["n_groups"]
+        return perm, gr[:G], gb[:G], tb
+
+    def export_las(self):
+        info = self.info
+        K = self.opts.minhash_k
+        sig = np.empty((self.n, K), np.uint64)
+        pairs = np.empty((max(info["n_pairs"], 1), 2), np.int32)
+        cl = np.empty(self.n, np.int32)
+        _call("gnn_plan_export_las", self.handle, _np_ptr(sig), _np_ptr(pairs), _np_ptr(cl))
+        return sig, pairs[:info["n_pairs"]], cl
+
+    def normalizers(self):
+        a, b = ctypes.c_void_p(), ctypes.c_void_p()
+        _call("gnn_plan_normalizers", self.handle, ctypes.byref(a), ctypes.byref(b))
+        return a.value, b.value
+
+    def workspace(self, op, f_in=0, f_out=0, heads=0, device=None):
+        nbytes = _lib.gnn_workspace_size(self.handle, op, f_in, f_out, heads)
+        if nbytes == 0:
+            return None, 0
+        key = (op, f_in, f_out, heads)
+        ws = self._ws.get(key)
+        if ws is None:
+            torch = _torch()
+            ws = torch.empty(nbytes, dtype=torch.uint8, device=device or "cuda")
+            self._ws[key] = ws
+        return ws, nbytes
+
+    def destroy(self):
+        if getattr(self, "handle", None):
+            _lib.gnn_plan_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.destroy()
+        except Exception:
+            pass
+
+
+def aggregate(plan: Plan, X, reduce="sum", weight="one", edge_w=None, relu=False, add_row=None, out=None,
+              stream=None):
+    torch = _torch()
+    F = X.shape[1]
+    Y = out if out is not None else torch.empty((plan.n, F), dtype=torch.float32, device=X.device)
+    ws, nb = plan.workspace(GNN_OP_AGGREGATE, 0, F, 0, X.device)
+    _call("gnn_aggregate", plan.handle, REDUCE[reduce], WEIGHT[weight], _tp(edge_w), _tp(X), _ld(X, F), F, _tp(Y),
+          _ld(Y, F), int(relu), _tp(add_row), 0 if add_row is None else _ld(add_row, F), _tp(ws), nb,
+          _stream(stream))
+    return Y
+
+
+def gat_aggregate(plan: Plan, Zs, t, H, Fh, neg_slope=0.2, out=None, stream=None):
+    torch = _torch()
+    F = H * Fh
+    Y = out if out is not None else torch.empty((plan.n, F), dtype=torch.float32, device=Zs.device)
+    ws, nb = plan.workspace(GNN_OP_GAT_AGGREGATE, 0, F, H, Zs.device)
+    _call("gnn_gat_aggregate", plan.handle, _tp(Zs), _ld(Zs, F + H), _tp(t), _ld(t, H), H, Fh, float(neg_slope),
+          _tp(Y), _ld(Y, F), _tp(ws), nb, _stream(stream))
+    return Y
+
+
+def gat_layer(plan: Plan, X, W, a_src, a_dst, H, Fh, neg_slope=0.2, out=None, stream=None):
+    torch = _torch()
+    F = H * Fh
+    f_in = X.shape[1]
+    Y = out if out is not None else torch.empty((plan.n, F), dtype=torch.float32, device=X.device)
+    ws, nb = plan.workspace(GNN_OP_GAT_LAYER, f_in, F, H, X.device)
+    _call("gnn_gat_layer", plan.handle, _tp(X), _ld(X, f_in), f_in, _tp(W.contiguous()), _tp(a_src.contiguous()),
+          _tp(a_dst.contiguous()), H, Fh, float(neg_slope), _tp(Y), _ld(Y, F), _tp(ws), nb, _stream(stream))
+    return Y
+
+
+def edgeconv_aggregate(plan: Plan, PQ, f_out, out=None, stream=None):
+    torch = _torch()
+    Y = out if out is not None else torch.empty((plan.n, f_out), dtype=torch.float32, device=PQ.device)
+    ws, nb = plan.workspace(GNN_OP_AGGREGATE, 0, f_out, 0, PQ.device)
+    _call("gnn_edgeconv_aggregate", plan.handle, _tp(PQ), _ld(PQ, 2 * f_out), f_out, _tp(Y), _ld(Y, f_out),
+          _tp(ws), nb, _stream(stream))
+    return Y
+
+
+def edgeconv(plan: Plan, X, theta, phi, bias=None, out=None, stream=None):
+    torch = _torch()
+    f_out, f_in = theta.shape
+    Y = out if out is not None else torch.empty((plan.n, f_out), dtype=torch.float32, device=X.device)
+    ws, nb = plan.workspace(GNN_OP_EDGECONV, f_in, f_out, 0, X.device)
+    _call("gnn_edgeconv", plan.handle, _tp(X), _ld(X, f_in), f_in, _tp(theta.contiguous()), _tp(phi.contiguous()),
+          _tp(bias), f_out, _tp(Y), _ld(Y, f_out), _tp(ws), nb, _stream(stream))
+    return Y
+
+
+def gemm(X, W, row_scale=None, col_bias=None, relu=False, out=None, stream=None):
+    torch = _torch()
+    m, k = X.shape
+    n = W.shape[1]
+    H = out if out is not None else torch.empty((m, n), dtype=torch.float32, device=X.device)
+    _call("gnn_gemm", _tp(X), _ld(X, k), _tp(W), _ld(W, n), _tp(H), _ld(H, n), m, k, n, _tp(row_scale),
+          _tp(col_bias), int(relu), _stream(stream))
+    return H
+
+
+def set_gemm_impl(impl: int) -> int:
+    return _lib.gnn_set_gemm_impl(impl)
+
+
+def gcn_layer(plan: Plan, X, W, relu=True, order=0, out=None, stream=None):
+    torch = _torch()
+    f_in = X.shape[1]
+    f_out = W.shape[1]
+    Y = out if out is not None else torch.empty((plan.n, f_out), dtype=torch.float32, device=X.device)
+    ws, nb = plan.workspace(GNN_OP_GCN_LAYER, f_in, f_out, 0, X.device)
+    _call("gnn_gcn_layer", plan.handle, _tp(X), _ld(X, f_in), f_in, _tp(W), _ld(W, f_out), f_out, int(relu),
+          int(order), _tp(Y), _ld(Y, f_out), _tp(ws), nb, _stream(stream))
+    return Y
+
+
+def partition_rows(rowptr, nparts):
+    rowptr = np.ascontiguousarray(rowptr, dtype=np.int64)
+    b = np.empty(nparts + 1, np.int64)
+    _call("gnn_partition_rows", len(rowptr) - 1, _np_ptr(rowptr), nparts, _np_ptr(b))
+    return b
+
+
+def local_csr(rowptr, colidx, bounds, rank):
+    """Rank-local CSR in the padded all-gather layout (host only)."""
+    rowptr = np.ascontiguousarray(rowptr, dtype=np.int64)
+    colidx = np.ascontiguousarray(colidx, dtype=np.int32)
+    bounds = np.ascontiguousarray(bounds, dtype=np.int64)
+    n = len(rowptr) - 1
+    P = len(bounds) - 1
+    rmax, lnnz = ctypes.c_int64(), ctypes.c_int64()
+    _call("gnn_local_csr", n, _np_ptr(rowptr), _np_ptr(colidx), _np_ptr(bounds), P, rank, ctypes.byref(rmax),
+          ctypes.byref(lnnz), None, None, None)
+    rows = int(bounds[rank + 1] - bounds[rank])
+    lrp = np.empty(rows + 1, np.int64)
+    lci = np.empty(max(lnnz.value, 1), np.int32)
+    sdeg = np.empty(max(P * rmax.value, 1), np.int32)
+    _call("gnn_local_csr", n, _np_ptr(rowptr), _np_ptr(colidx), _np_ptr(bounds), P, rank, ctypes.byref(rmax),
+          ctypes.byref(lnnz), _np_ptr(lrp), _np_ptr(lci), _np_ptr(sdeg))
+    return lrp, lci[:lnnz.value], sdeg[:P * rmax.value], rmax.value
+
+
+def las_host(rowptr, sig, r=2, W=8, cap=32, min_sim=-1):
+    """a2 steps 2-5 on the host from given MinHash signatures (no GPU)."""
+    rowptr = np.ascontiguousarray(rowptr, dtype=np.int64)
+    sig = np.ascontiguousarray(sig, dtype=np.uint64)
+    n, K = sig.shape
+    perm = np.empty(n, np.int32)
+    cl = np.empty(n, np.int32)
+    npairs, nc = ctypes.c_int64(), ctypes.c_int64()
+    _call("gnn_las_host", n, _np_ptr(rowptr), _np_ptr(sig), K, r, W, cap, min_sim, _np_ptr(perm), _np_ptr(cl),
+          ctypes.byref(npairs), ctypes.byref(nc))
+    return perm, cl, npairs.value, nc.value
+
+
+def groups_host(rowptr, ng, T=32, perm=None):
+    """a3 neighbor groups + tiles on the host (no GPU)."""
+    rowptr = np.ascontiguousarray(rowptr, dtype=np.int64)
+    n = len(rowptr) - 1
+    p = None if perm is None else np.ascontiguousarray(perm, dtype=np.int32)
+    G, NT = ctypes.c_int64(), ctypes.c_int64()
+    _call("gnn_groups_host", n, _np_ptr(rowptr), _np_ptr(p), ng, T, ctypes.byref(G), ctypes.byref(NT), None, None,
+          None)
+    gr = np.empty(max(G.value, 1), np.int32)
+    gb = np.empty(max(G.value, 1), np.int64)
+    tb = np.empty(NT.value + 1, np.int64)
+    _call("gnn_groups_host", n, _np_ptr(rowptr), _np_ptr(p), ng, T, ctypes.byref(G), ctypes.byref(NT), _np_ptr(gr),
+          _np_ptr(gb), _np_ptr(tb))
+    return gr[:G.value], gb[:G.value], tb
+
+
+def launch_count() -> int:
+    return int(_lib.gnn_launch_count())

@@ -1,0 +1,328 @@
+"""GPU parity: the sm_100a path (through the C-ABI) vs the CPU oracle.
+
+Bar (BASELINE.json north_star): fp32 within |g - r| <= 1e-5 + 1e-4 |r| of the
+fp64 oracle rounded to fp32; plans bit-exact; the deterministic variant
+bit-identical across reruns, schedules and tile sizes, and bit-identical to
+the oracle's fp32 order replica (R9); integer work bit-exact.
+"""
+import numpy as np
+import pytest
+
+import gnn_synth as gs
+import oracle
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+if not torch.cuda.is_available():  # pragma: no cover - CPU box
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+import paper_conf_ppopp_huangzzys21_b200 as G  # noqa: E402  (loads libgnn.so, no fallback)
+
+DEV = "cuda"
+RTOL, ATOL = 1e-4, 1e-5
+
+
+def T(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).to(DEV)
+
+
+def H(t):
+    torch.cuda.synchronize()
+    return t.detach().cpu().numpy()
+
+
+def assert_close(got, ref, rtol=RTOL, atol=ATOL, what=""):
+    got = np.asarray(got, np.float64)
+    ref = np.asarray(ref, np.float64)
+    assert got.shape == ref.shape, (got.shape, ref.shape)
+    err = np.abs(got - ref)
+    bad = err > atol + rtol * np.abs(ref)
+    assert not bad.any(), f"{what}: {bad.sum()} / {bad.size} outside tol; max abs {err.max():.3e}; " \
+                          f"first {np.argwhere(bad)[:3].tolist()}"
+
+
+def hub_graph(seed=0):
+    """Mixed graph with a 5,000-degree hub (rows spanning many tiles), empty rows,
+    self loops and multi-edges."""
+    rng = np.random.default_rng(seed)
+    n = 700
+    rows = []
+    for v in range(n):
+        if v == 3:
+            rows.append(sorted(rng.integers(0, n, size=5000).tolist()))
+        elif v % 11 == 0:
+            rows.append([])
+        else:
+            rows.append(sorted(rng.integers(0, n, size=int(rng.integers(1, 90))).tolist()))
+    return gs.from_rows(rows)
+
+
+GRAPHS = {
+    "cora": lambda: gs.config_graph("C1"),
+    "small": lambda: gs.random_small(300, avg_deg=7, seed=3, self_loops=True),
+    "hub": hub_graph,
+}
+
+
+@pytest.fixture(scope="module")
+def graphs():
+    return {k: f() for k, f in GRAPHS.items()}
+
+
+# --------------------------------------------------------------------------- #
+# a6 aggregation
+# --------------------------------------------------------------------------- #
+@pytest.mark.parametrize("gname,F", [("cora", 16), ("small", 1), ("small", 3), ("small", 40), ("small", 100),
+                                     ("hub", 64), ("hub", 256), ("small", 602)])
+@pytest.mark.parametrize("reduce", ["sum", "mean", "max"])
+@pytest.mark.parametrize("weight", ["one", "gcn", "edge"])
+def test_aggregate_parity(graphs, gname, F, reduce, weight):
+    g = graphs[gname]
+    X = gs.uniform(g.n, F, seed=F)
+    ew = gs.uniform(g.nnz, 1, lo=0.1, hi=1.0, seed=2)[:, 0] if weight == "edge" else None
+    relu = (F % 2 == 0)
+    ref = oracle.aggregate(g.rowptr, g.colidx, X, reduce, weight, ew, relu=relu)
+    plan = G.Plan(g.rowptr, g.colidx, group_size=16 if gname == "hub" else -1, tile_groups=8)
+    Y = G.aggregate(plan, T(X), reduce, weight, None if ew is None else T(ew), relu=relu)
+    assert_close(H(Y), ref, what=f"{gname} F={F} {reduce}/{weight}")
+    if reduce == "max" and weight == "one":
+        assert np.array_equal(H(Y), ref)  # max is exact
+
+
+@pytest.mark.parametrize("reduce", ["sum", "mean", "max"])
+@pytest.mark.parametrize("weight", ["one", "gcn", "edge"])
+@pytest.mark.parametrize("ng,Tg", [(16, 2), (16, 32), (64, 32), (0, 32), (1, 4)])
+def test_aggregate_bit_exact_vs_order_replica(graphs, reduce, weight, ng, Tg):
+    """Deterministic variant == the oracle's fp32 order replica (R9) bit for bit,
+    including rows split across CTAs (hub, T=2)."""
+    g = graphs["hub"]
+    F = 24
+    X = gs.uniform(g.n, F, seed=11)
+    ew = gs.uniform(g.nnz, 1, seed=12)[:, 0] if weight == "edge" else None
+    rep = oracle.aggregate_ng_f32(g.rowptr, g.colidx, X, ng, reduce, weight, ew, relu=True)
+    plan = G.Plan(g.rowptr, g.colidx, group_size=ng, tile_groups=Tg)
+    Y = H(G.aggregate(plan, T(X), reduce, weight, None if ew is None else T(ew), relu=True))
+    assert np.array_equal(Y.view(np.uint32), rep.view(np.uint32)), np.abs(Y - rep).max()
+
+
+def test_integer_features_exact(graphs):
+    g = graphs["hub"]
+    X = gs.integer_features(g.n, 32, seed=1)
+    plan = G.Plan(g.rowptr, g.colidx, group_size=16, tile_groups=2)
+    for red in ("sum", "mean", "max"):
+        assert np.array_equal(H(G.aggregate(plan, T(X), red)), oracle.aggregate(g.rowptr, g.colidx, X, red))
+
+
+def test_rerun_schedule_and_tile_invariance():
+    """Bit-identical across reruns, LAS on/off and tile sizes (deterministic variant)."""
+    g = gs.powerlaw(20000, 400000, 20, 3000, 2500, comm=32, rho=0.8, seed=7)
+    X = T(gs.uniform(g.n, 64, seed=1))
+    outs = []
+    for reorder, Tg in [(0, 32), (1, 32), (0, 4), (1, 7)]:
+        plan = G.Plan(g.rowptr, g.colidx, reorder=reorder, tile_groups=Tg, group_size=32)
+        a = H(G.aggregate(plan, X, "sum", "gcn", relu=True))
+        b = H(G.aggregate(plan, X, "sum", "gcn", relu=True))
+        assert np.array_equal(a, b)
+        outs.append(a)
+    for o in outs[1:]:
+        assert np.array_equal(o, outs[0])
+
+
+def test_nondeterministic_variant_within_tolerance(graphs):
+    g = graphs["hub"]
+    X = gs.uniform(g.n, 32, seed=5)
+    plan = G.Plan(g.rowptr, g.colidx, group_size=16, tile_groups=2, deterministic=0)
+    for red, w in [("sum", "gcn"), ("mean", "one")]:
+        ref = oracle.aggregate(g.rowptr, g.colidx, X, red, w)
+        assert_close(H(G.aggregate(plan, T(X), red, w)), ref, what=f"atomic {red}")
+
+
+def test_strided_and_offset_views():
+    """ld > F and unaligned column offsets fall back to narrower vectors."""
+    g = gs.random_small(200, avg_deg=6, seed=9)
+    Xbig = gs.uniform(g.n, 70, seed=3)
+    X = T(Xbig)[:, 1:65]  # ld 70, base offset 4 B
+    Y = torch.zeros((g.n, 80), device=DEV)[:, 3:67]
+    plan = G.Plan(g.rowptr, g.colidx)
+    G.aggregate(plan, X, "sum", "gcn", out=Y)
+    assert_close(H(Y), oracle.aggregate(g.rowptr, g.colidx, Xbig[:, 1:65], "sum", "gcn"))
+
+
+# --------------------------------------------------------------------------- #
+# a2/a3 plans bit-exact
+# --------------------------------------------------------------------------- #
+@pytest.mark.parametrize("rho", [0.0, 0.8])
+def test_plan_bit_exact_vs_oracle(rho):
+    g = gs.powerlaw(8000, 90000, 11, 900, 800, comm=32, rho=rho, seed=3)
+    plan = G.Plan(g.rowptr, g.colidx, reorder=1, group_size=16, tile_groups=8, seed=42)
+    sig, pairs, cl = plan.export_las()
+    perm, gr, gb, tb = plan.export()
+    operm, info = oracle.las_schedule(g.rowptr, g.colidx, seed=42)
+    assert np.array_equal(sig, info["sig"])        # GPU MinHash == oracle MinHash
+    assert np.array_equal(pairs, info["pairs"])
+    assert np.array_equal(cl, info["cluster_of"])
+    assert np.array_equal(perm, operm)
+    ogr, ogb = oracle.neighbor_groups(g.rowptr, 16, operm)
+    assert np.array_equal(gr, ogr) and np.array_equal(gb, ogb)
+    assert np.array_equal(tb, oracle.tiles(ogr, 8))
+
+
+# --------------------------------------------------------------------------- #
+# a7 fused GAT
+# --------------------------------------------------------------------------- #
+@pytest.mark.parametrize("Hh,Fh", [(8, 8), (8, 32), (1, 1), (2, 3), (4, 16)])
+@pytest.mark.parametrize("gname", ["small", "hub"])
+def test_gat_aggregate_parity(graphs, Hh, Fh, gname):
+    g = graphs[gname]
+    F = Hh * Fh
+    Zs = gs.uniform(g.n, F + Hh, seed=Fh)
+    Zs[:, F:] *= 3.0
+    t = gs.uniform(g.n, Hh, lo=-3, hi=3, seed=Hh)
+    ref = oracle.gat_aggregate(g.rowptr, g.colidx, Zs, t, Hh, Fh, 0.2)
+    plan = G.Plan(g.rowptr, g.colidx, group_size=16, tile_groups=4)
+    Y = G.gat_aggregate(plan, T(Zs), T(t), Hh, Fh, 0.2)
+    assert_close(H(Y), ref, what=f"gat {gname} {Hh}x{Fh}")
+
+
+def test_gat_invariants(graphs):
+    g = graphs["hub"]
+    Hh, Fh = 2, 4
+    F = Hh * Fh
+    plan = G.Plan(g.rowptr, g.colidx, group_size=16, tile_groups=2)
+    # (1) softmax rows sum to 1: a ones column in z
+    Zs = gs.uniform(g.n, F + Hh, lo=-2, hi=2, seed=1)
+    Zs[:, Fh - 1] = 1.0
+    Zs[:, 2 * Fh - 1] = 1.0
+    t = gs.uniform(g.n, Hh, lo=-2, hi=2, seed=2)
+    Y = H(G.gat_aggregate(plan, T(Zs), T(t), Hh, Fh))
+    nonempty = np.diff(g.rowptr) > 0
+    assert np.allclose(Y[nonempty][:, [Fh - 1, 2 * Fh - 1]], 1.0, atol=2e-6)
+    assert np.all(Y[~nonempty] == 0)
+    # (2) zero scores -> uniform attention -> mean aggregation
+    Zs[:, F:] = 0
+    Y0 = H(G.gat_aggregate(plan, T(Zs), T(np.zeros_like(t)), Hh, Fh))
+    assert_close(Y0, oracle.aggregate(g.rowptr, g.colidx, Zs[:, :F], "mean"), 1e-5, 1e-6)
+    # (3) single-neighbour rows reproduce z_u bit-exactly
+    g1 = gs.from_rows([[5], [0], [], [1], [2], [3]])
+    p1 = G.Plan(g1.rowptr, g1.colidx)
+    Z1 = gs.uniform(6, F + Hh, lo=-50, hi=50, seed=3)
+    Y1 = H(G.gat_aggregate(p1, T(Z1), T(gs.uniform(6, Hh, lo=-50, hi=50, seed=4)), Hh, Fh))
+    assert np.array_equal(Y1[[0, 1, 3, 4, 5]], Z1[[5, 0, 1, 2, 3], :F])
+    assert np.all(Y1[2] == 0)
+
+
+def test_gat_layer_parity():
+    g = gs.random_small(500, avg_deg=8, seed=4)
+    Hh, Fh, f_in = 8, 8, 128
+    X = gs.uniform(g.n, f_in, seed=1)
+    W = gs.uniform(f_in, Hh * Fh, lo=-0.2, hi=0.2, seed=2)
+    a_s = gs.uniform(1, Hh * Fh, lo=-0.6, hi=0.6, seed=3)[0]
+    a_d = gs.uniform(1, Hh * Fh, lo=-0.6, hi=0.6, seed=4)[0]
+    ref = oracle.gat_layer(g.rowptr, g.colidx, X, W, a_s, a_d, Hh, Fh, 0.2)
+    plan = G.Plan(g.rowptr, g.colidx)
+    Y = G.gat_layer(plan, T(X), T(W), T(a_s), T(a_d), Hh, Fh, 0.2)
+    assert_close(H(Y), ref, what="gat layer")
+
+
+# --------------------------------------------------------------------------- #
+# a8 EdgeConv
+# --------------------------------------------------------------------------- #
+def test_edgeconv_aggregate_bit_exact_subpin():
+    """Given the GPU's own [P|Q], y_v = max_u fl(Q_v + P_u) clamped at 0 must match
+    an fp32 per-edge recompute bit-for-bit (rounding is monotone, R6)."""
+    g = gs.config_graph("C4")
+    f_out = 64
+    PQ = gs.uniform(g.n, 2 * f_out, seed=5)
+    plan = G.Plan(g.rowptr, g.colidx)
+    Y = H(G.edgeconv_aggregate(plan, T(PQ), f_out))
+    src = g.colidx.astype(np.int64)
+    dst = np.repeat(np.arange(g.n), np.diff(g.rowptr))
+    msg = (PQ[dst, f_out:] + PQ[src, :f_out]).astype(np.float32)
+    want = np.full((g.n, f_out), -np.inf, np.float32)
+    np.maximum.at(want, dst, msg)
+    want = np.maximum(want, np.float32(0))
+    assert np.array_equal(Y, want)
+
+
+def test_edgeconv_layer_parity():
+    g = gs.config_graph("C4")
+    fin, fout = 64, 64
+    X = gs.uniform(g.n, fin, seed=1)
+    lim = np.sqrt(6 / (fin + fout))
+    th = gs.uniform(fout, fin, lo=-lim, hi=lim, seed=2)
+    ph = gs.uniform(fout, fin, lo=-lim, hi=lim, seed=3)
+    b = gs.uniform(1, fout, lo=-0.1, hi=0.1, seed=4)[0]
+    rows = np.random.default_rng(0).choice(g.n, 3000, replace=False)
+    ref = oracle.edgeconv(g.rowptr, g.colidx, X, th, ph, b, rows=rows)
+    plan = G.Plan(g.rowptr, g.colidx)
+    Y = H(G.edgeconv(plan, T(X), T(th), T(ph), T(b)))
+    assert_close(Y[rows], ref, what="edgeconv")
+
+
+# --------------------------------------------------------------------------- #
+# a5 GEMM and the GCN layer
+# --------------------------------------------------------------------------- #
+@pytest.mark.parametrize("m,k,n", [(1, 1, 1), (300, 17, 5), (2708, 1433, 16), (4099, 602, 256), (5000, 100, 256),
+                                   (3333, 64, 128), (1000, 256, 272)])
+def test_gemm_parity(m, k, n):
+    X = gs.uniform(m, k, seed=1)
+    lim = np.sqrt(6 / (k + n))
+    W = gs.uniform(k, n, lo=-lim, hi=lim, seed=2)
+    rs = gs.uniform(m, 1, lo=0.1, hi=1.0, seed=3)[:, 0]
+    ref = oracle.gemm(X, W, rs)
+    Hh = G.gemm(T(X), T(W), row_scale=T(rs))
+    assert_close(H(Hh), ref, what=f"gemm {m}x{k}x{n}")
+
+
+@pytest.mark.parametrize("order", [1, 2])
+def test_gcn_layer_parity(order):
+    g = gs.config_graph("C1")
+    X = (np.random.default_rng(1).random((g.n, 1433)) < 0.0127).astype(np.float32)
+    lim = np.sqrt(6 / (1433 + 16))
+    W = gs.uniform(1433, 16, lo=-lim, hi=lim, seed=2)
+    ref = oracle.gcn_layer(g.rowptr, g.colidx, X, W, relu=True)
+    plan = G.Plan(g.rowptr, g.colidx)
+    Y = G.gcn_layer(plan, T(X), T(W), relu=True, order=order)
+    assert_close(H(Y), ref, what=f"gcn order {order}")
+
+
+# --------------------------------------------------------------------------- #
+# full-size BASELINE.json configs (sampled rows: rows are independent)
+# --------------------------------------------------------------------------- #
+def sample_rows(g, k=4096, seed=0):
+    rng = np.random.default_rng(seed)
+    deg = np.diff(g.rowptr)
+    top = np.argsort(deg)[-64:]
+    return np.unique(np.concatenate([rng.choice(g.n, min(k, g.n), replace=False), top]))
+
+
+def test_c2_gat_layer_full():
+    c = gs.CONFIGS["C2"]
+    g = gs.config_graph("C2")
+    Hh, Fh, f_in = c["H"], c["Fh"], c["F_in"]
+    X = gs.uniform(g.n, f_in, seed=gs.seed_of("C2", 1))
+    lim = np.sqrt(6 / (f_in + Hh * Fh))
+    W = gs.uniform(f_in, Hh * Fh, lo=-lim, hi=lim, seed=gs.seed_of("C2", 2))
+    al = np.sqrt(6 / (Fh + 1))
+    a_s = gs.uniform(1, Hh * Fh, lo=-al, hi=al, seed=gs.seed_of("C2", 3))[0]
+    a_d = gs.uniform(1, Hh * Fh, lo=-al, hi=al, seed=gs.seed_of("C2", 3) + 1)[0]
+    plan = G.Plan(g.rowptr, g.colidx, reorder=1)
+    Y = H(G.gat_layer(plan, T(X), T(W), T(a_s), T(a_d), Hh, Fh, 0.2))
+    rows = sample_rows(g)
+    ref = oracle.gat_layer(g.rowptr, g.colidx, X, W, a_s, a_d, Hh, Fh, 0.2, rows=rows)
+    assert_close(Y[rows], ref, what="C2 GAT layer")
+
+
+@pytest.mark.parametrize("cfg", ["C3", "C5"])
+def test_full_size_gcn_aggregate(cfg):
+    """The bench's launch configuration at full size: LAS plan, transform-first
+    aggregation at F=256 (sampled rows incl. the 64 largest)."""
+    g = gs.config_graph(cfg)
+    F = 256
+    Hs = gs.uniform(g.n, F, seed=gs.seed_of(cfg, 1))
+    plan = G.Plan(g.rowptr, g.colidx, reorder=1)
+    Y = H(G.aggregate(plan, T(Hs), "sum", "gcn", relu=True))
+    rows = sample_rows(g, 2048)
+    ref = oracle.aggregate(g.rowptr, g.colidx, Hs, "sum", "gcn", relu=True, rows=rows)
+    assert_close(Y[rows], ref, what=f"{cfg} aggregate")
