@@ -1,0 +1,97 @@
+"""Kernel micro-benchmarks on the GPU (dev tool, not the bench contract).
+
+    python scripts/kbench.py gemm            # SIMT vs tcgen05 3xTF32 at the C5 shapes (+ parity)
+    python scripts/kbench.py agg [--cfg C5]  # aggregation kernels on a config graph
+"""
+import os
+import sys
+import time
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import gnn_synth as gs  # noqa: E402
+import paper_conf_ppopp_huangzzys21_b200 as G  # noqa: E402
+
+
+def timeit(fn, iters=10, warm=3):
+    for _ in range(warm):
+        fn()
+    torch.cuda.synchronize()
+    a = torch.cuda.Event(enable_timing=True)
+    b = torch.cuda.Event(enable_timing=True)
+    a.record()
+    for _ in range(iters):
+        fn()
+    b.record()
+    torch.cuda.synchronize()
+    return a.elapsed_time(b) / iters
+
+
+def gemm():
+    import oracle
+    shapes = [(2449029, 100, 256), (2449029, 256, 256), (2449029, 256, 272), (232965, 602, 256),
+              (169343, 128, 80), (32768, 64, 128), (4099, 602, 256), (1000, 37, 5)]
+    for (m, k, n) in shapes:
+        X = torch.rand(m, k, device="cuda") * 2 - 1
+        W = (torch.rand(k, n, device="cuda") * 2 - 1) * float(np.sqrt(6 / (k + n)))
+        rs = torch.rand(m, device="cuda") + 0.1
+        res = {}
+        for impl, name in [(1, "simt"), (2, "tc")]:
+            G.set_gemm_impl(impl)
+            try:
+                H = G.gemm(X, W, row_scale=rs)
+                torch.cuda.synchronize()
+                ms = timeit(lambda: G.gemm(X, W, row_scale=rs, out=H))
+                res[name] = (ms, H.clone())
+            except Exception as e:  # noqa: BLE001
+                res[name] = (None, repr(e))
+        G.set_gemm_impl(0)
+        rows = torch.randint(0, m, (512,), device="cuda")
+        ref = oracle.gemm(X[rows].cpu().numpy(), W.cpu().numpy(), rs[rows].cpu().numpy())
+        line = f"m={m} k={k} n={n}"
+        for name, (ms, H) in res.items():
+            if ms is None:
+                line += f" | {name}: FAILED {H}"
+                continue
+            got = H[rows].cpu().numpy()
+            err = np.abs(got - ref)
+            ok = np.all(err <= 1e-5 + 1e-4 * np.abs(ref))
+            tf = 2 * m * k * n / (ms * 1e-3) / 1e12
+            gbs = 4 * (m * k + k * n + m * n) / (ms * 1e-3) / 1e9
+            line += f" | {name}: {ms:.3f} ms {tf:.1f} TF/s {gbs:.0f} GB/s maxerr {err.max():.2e} ok={ok}"
+        print(line, flush=True)
+
+
+def agg(cfg="C5"):
+    t0 = time.time()
+    g = gs.config_graph(cfg)
+    print(f"{cfg}: n={g.n} nnz={g.nnz} gen {time.time() - t0:.1f}s", flush=True)
+    for reorder in (0, 1):
+        t0 = time.time()
+        plan = G.Plan(g.rowptr, g.colidx, reorder=reorder)
+        print(f" plan reorder={reorder}: {time.time() - t0:.1f}s info={plan.info}", flush=True)
+        for F in (64, 100, 256):
+            X = torch.rand(g.n, F, device="cuda")
+            Y = torch.empty_like(X)
+            ms = timeit(lambda: G.aggregate(plan, X, "sum", "gcn", out=Y), iters=5, warm=2)
+            alg = g.nnz * (4 + 4 * F + 4) + g.n * (8 + 4 * F)
+            print(f"  F={F}: {ms:.3f} ms  {alg / ms / 1e6:.0f} GB/s algorithmic  "
+                  f"{g.nnz * F / ms / 1e6:.1f} Gedge*F/s", flush=True)
+        Hh, Fh = 8, 32
+        Zs = torch.rand(g.n, Hh * Fh + 2 * Hh, device="cuda")
+        Y = torch.empty(g.n, Hh * Fh, device="cuda")
+        t = Zs[:, Hh * Fh + Hh:]
+        ms = timeit(lambda: G.gat_aggregate(plan, Zs, t, Hh, Fh, out=Y), iters=5, warm=2)
+        alg = g.nnz * (4 + 4 * (Hh * Fh + Hh)) + g.n * (8 + 4 * Hh * Fh + 4 * Hh)
+        print(f"  GAT 8x32: {ms:.3f} ms  {alg / ms / 1e6:.0f} GB/s algorithmic", flush=True)
+
+
+if __name__ == "__main__":
+    what = sys.argv[1] if len(sys.argv) > 1 else "gemm"
+    if what == "gemm":
+        gemm()
+    else:
+        agg(sys.argv[sys.argv.index("--cfg") + 1] if "--cfg" in sys.argv else "C5")

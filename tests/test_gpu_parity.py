@@ -32,12 +32,20 @@ def H(t):
     return t.detach().cpu().numpy()
 
 
-def assert_close(got, ref, rtol=RTOL, atol=ATOL, what=""):
+def assert_close(got, ref, rtol=RTOL, atol=ATOL, what="", S=None, deg=None):
+    """R11: |g - r| <= atol + rtol |r|.  Conditioned fallback only for
+    raw (unnormalised) sums on rows with more than 1,000 terms, where fp32
+    reassociation alone can exceed the primary bound: |g - r| <= 1e-6 * S,
+    S = sum |terms| from the oracle."""
     got = np.asarray(got, np.float64)
     ref = np.asarray(ref, np.float64)
     assert got.shape == ref.shape, (got.shape, ref.shape)
     err = np.abs(got - ref)
-    bad = err > atol + rtol * np.abs(ref)
+    allowed = atol + rtol * np.abs(ref)
+    if S is not None and deg is not None:
+        long_rows = (deg > 1000)[:, None]
+        allowed = np.where(long_rows, np.maximum(allowed, 1e-6 * S), allowed)
+    bad = err > allowed
     assert not bad.any(), f"{what}: {bad.sum()} / {bad.size} outside tol; max abs {err.max():.3e}; " \
                           f"first {np.argwhere(bad)[:3].tolist()}"
 
@@ -82,10 +90,12 @@ def test_aggregate_parity(graphs, gname, F, reduce, weight):
     X = gs.uniform(g.n, F, seed=F)
     ew = gs.uniform(g.nnz, 1, lo=0.1, hi=1.0, seed=2)[:, 0] if weight == "edge" else None
     relu = (F % 2 == 0)
-    ref = oracle.aggregate(g.rowptr, g.colidx, X, reduce, weight, ew, relu=relu)
+    ref, S = oracle.aggregate(g.rowptr, g.colidx, X, reduce, weight, ew, relu=relu, return_abs=True)
     plan = G.Plan(g.rowptr, g.colidx, group_size=16 if gname == "hub" else -1, tile_groups=8)
     Y = G.aggregate(plan, T(X), reduce, weight, None if ew is None else T(ew), relu=relu)
-    assert_close(H(Y), ref, what=f"{gname} F={F} {reduce}/{weight}")
+    raw = weight == "edge" and reduce == "sum"  # unnormalised sum: conditioned fallback allowed
+    assert_close(H(Y), ref, what=f"{gname} F={F} {reduce}/{weight}", S=S if raw else None,
+                 deg=np.diff(g.rowptr) if raw else None)
     if reduce == "max" and weight == "one":
         assert np.array_equal(H(Y), ref)  # max is exact
 
@@ -136,6 +146,9 @@ def test_nondeterministic_variant_within_tolerance(graphs):
     for red, w in [("sum", "gcn"), ("mean", "one")]:
         ref = oracle.aggregate(g.rowptr, g.colidx, X, red, w)
         assert_close(H(G.aggregate(plan, T(X), red, w)), ref, what=f"atomic {red}")
+    # raw sums over the 5,000-entry hub: conditioned bound (R11)
+    ref, S = oracle.aggregate(g.rowptr, g.colidx, X, "sum", "one", return_abs=True)
+    assert_close(H(G.aggregate(plan, T(X), "sum", "one")), ref, what="atomic raw sum", S=S, deg=np.diff(g.rowptr))
 
 
 def test_strided_and_offset_views():
