@@ -145,6 +145,7 @@ def run_ours(args):
     import torch
     import torch.distributed as dist
     import paper_conf_ppopp_huangzzys21_b200 as G
+    from paper_conf_ppopp_huangzzys21_b200.model import RowPartitionedGCNGAT
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -158,101 +159,18 @@ def run_ours(args):
     F_in, F, Hh, Fh = inp["F_in"], inp["F"], inp["H"], inp["Fh"]
     HF = Hh * Fh
     t0 = time.time()
-    if world == 1:
-        bounds = np.array([0, n], np.int64)
-        lo, hi, rmax = 0, n, n
-        plan = G.Plan(g.rowptr, g.colidx, reorder=args.reorder)
-    else:
-        bounds = G.partition_rows(g.rowptr, world)
-        lo, hi = int(bounds[rank]), int(bounds[rank + 1])
-        lrp, lci, sdeg, rmax = G.local_csr(g.rowptr, g.colidx, bounds, rank)
-        plan = G.Plan(lrp, lci, n_src=world * rmax, src_degree=sdeg, reorder=args.reorder)
+    model = RowPartitionedGCNGAT(g.rowptr, g.colidx, inp["W1"], inp["W2"], inp["W3"], inp["a_src"], inp["a_dst"],
+                                 Hh, Fh, rank=rank, world=world, reorder=args.reorder, device=dev)
     plan_s = time.time() - t0
-    info = plan.info
-    rows = hi - lo
-    lnnz = int(g.rowptr[hi] - g.rowptr[lo])
-    # device-resident inputs (X replicated: layer 1 aggregates first, R4-i / SURVEY §8(e) lever i)
-    Xd = torch.from_numpy(inp["X"]).to(dev)
-    W1 = torch.from_numpy(inp["W1"]).to(dev)
-    W2 = torch.from_numpy(inp["W2"]).to(dev)
-    W3 = torch.from_numpy(inp["W3"]).to(dev)
-    a_s = torch.from_numpy(inp["a_src"]).to(dev)
-    a_d = torch.from_numpy(inp["a_dst"]).to(dev)
-    ldwe = (HF + 2 * Hh + 7) // 8 * 8
-    A1 = torch.empty((rows, F_in), device=dev)
-    Y1 = torch.empty((rows, F), device=dev)
-    Hs2 = torch.empty((world * rmax, F), device=dev)  # padded all-gather layout
-    Y2 = torch.empty((rows, F), device=dev)
-    Wext = torch.empty((F, ldwe), device=dev)
-    Zst = torch.empty((world * rmax, ldwe), device=dev)
-    Y3 = torch.empty((rows, HF), device=dev)
-    nsrc_ptr, _ = plan.normalizers()
-    ws_agg, ws_agg_b = plan.workspace(G.gnn.GNN_OP_AGGREGATE, 0, max(F, F_in), 0, dev)
-    ws_gat, ws_gat_b = plan.workspace(G.gnn.GNN_OP_GAT_AGGREGATE, 0, HF, Hh, dev)
-    import ctypes
-    lib = G.gnn
-    X_local = Xd if world == 1 else Xd  # full X, plan rows are the local ones
-    if world > 1:
-        # local plan indexes the padded layout; X must be laid out the same way
-        Xpad = torch.zeros((world * rmax, F_in), device=dev)
-        for q in range(world):
-            Xpad[q * rmax:q * rmax + int(bounds[q + 1] - bounds[q])] = Xd[int(bounds[q]):int(bounds[q + 1])]
-        X_local = Xpad
-        del Xd
+    info = model.plan.info
+    rows, lnnz = model.rows, model.nnz_local
+    model.load_input(torch.from_numpy(inp["X"]), non_blocking=False)  # inputs resident in HBM
     stream = torch.cuda.current_stream(dev)
-    sp = ctypes.c_void_p(stream.cuda_stream)
-    nsrc_c = ctypes.c_void_p(nsrc_ptr)
-
-    def P(t):
-        return ctypes.c_void_p(t.data_ptr())
-
-    def chk(st, what):
-        if st != 0:
-            raise RuntimeError(f"{what}: {lib.gnn_last_error()}")
-
-    # the GAT weight fold W' = [W3 | W3_h a_src_h | W3_h a_dst_h] is a per-layer
-    # parameter transform: done inside the step by gnn_gat_layer's helper path
-    def step(ev=None):
-        rec = (lambda i: ev[i].record(stream)) if ev else (lambda i: None)
-        rec(0)
-        # layer 1: aggregate-first at F_in (exchange-free: X replicated)
-        chk(lib.gnn_aggregate(plan.handle, 0, 1, None, P(X_local), F_in, F_in, P(A1), F_in, 0, None, 0,
-                              P(ws_agg), ws_agg_b, sp), "agg1")
-        rec(1)
-        chk(lib.gnn_gemm(P(A1), F_in, P(W1), F, P(Y1), F, rows, F_in, F, None, None, 1, sp), "gemm1")
-        rec(2)
-        # layer 2: transform-first, nsrc folded into the GEMM epilogue
-        if world == 1:
-            chk(lib.gnn_gemm(P(Y1), F, P(W2), F, P(Hs2), F, rows, F, F, nsrc_c, None, 0, sp), "gemm2")
-        else:
-            loc = Hs2[rank * rmax:rank * rmax + rows]
-            # nsrc of the local rows lives at the rank's slot of the padded source space
-            chk(lib.gnn_gemm(P(Y1), F, P(W2), F, P(loc), F, rows, F, F,
-                             ctypes.c_void_p(nsrc_ptr + 4 * rank * rmax), None, 0, sp), "gemm2")
-            dist.all_gather_into_tensor(Hs2, Hs2[rank * rmax:(rank + 1) * rmax].clone())
-        rec(3)
-        chk(lib.gnn_gcn_aggregate_prescaled(plan.handle, P(Hs2), F, F, P(Y2), F, 0, P(ws_agg), ws_agg_b, sp),
-            "agg2")
-        rec(4)
-        # layer 3: GAT 8x32: Z|s|t = Y2 W', fused edge-softmax aggregation
-        chk(lib.gnn_gat_fold_weights(P(W3), P(a_s), P(a_d), F, Hh, Fh, P(Wext), ldwe, sp), "gat fold")
-        zloc = Zst if world == 1 else Zst[rank * rmax:rank * rmax + rows]
-        chk(lib.gnn_gemm(P(Y2), F, P(Wext), ldwe, P(zloc), ldwe, rows, F, ldwe, None, None, 0, sp), "gemm3")
-        if world > 1:
-            dist.all_gather_into_tensor(Zst, Zst[rank * rmax:(rank + 1) * rmax].clone())
-        rec(5)
-        tptr = ctypes.c_void_p(zloc.data_ptr() + 4 * (HF + Hh))
-        chk(lib.gnn_gat_aggregate(plan.handle, P(Zst), ldwe, tptr, ldwe, Hh, Fh, ctypes.c_float(0.2), P(Y3), HF,
-                                  P(ws_gat), ws_gat_b, sp), "gat agg")
-        rec(6)
-
-    # warm-up
     for _ in range(args.warmup):
-        step()
+        model.step()
     torch.cuda.synchronize(dev)
     if world > 1:
         dist.barrier()
-    # timed region: K steps, per-call events on the launching stream
     nev = 7
     evs = [[torch.cuda.Event(enable_timing=True) for _ in range(nev)] for _ in range(args.steps)]
     clk = ClockSampler(local)
@@ -266,15 +184,14 @@ def run_ours(args):
     t_end = torch.cuda.Event(enable_timing=True)
     t_start.record(stream)
     for k in range(args.steps):
-        step(evs[k])
+        model.step(events=evs[k])
     t_end.record(stream)
     torch.cuda.synchronize(dev)
     if world > 1:
         dist.barrier()
     launches = G.launch_count() - launches0
     clocks = clk.stop()
-    ms_total = t_start.elapsed_time(t_end)
-    ms = torch.tensor([ms_total], device=dev)
+    ms = torch.tensor([t_start.elapsed_time(t_end)], device=dev)
     if world > 1:
         dist.all_reduce(ms, op=dist.ReduceOp.MAX)
     ms_step = float(ms.item()) / args.steps
@@ -287,17 +204,14 @@ def run_ours(args):
     edge_feats = float(nnz) * (F_in + F + HF)  # whole job (all ranks)
     value = edge_feats / (ms_step * 1e-3) / 1e9
 
-    # roofline of the dominant graph kernel
-    dom = int(np.argmax(parts))
+    # roofline of the dominant graph kernel (algorithmic bytes per launch / event time)
     per_launch = {
-        "agg1_F100": agg_bytes(lnnz, rows, F_in, per_edge_extra=4),  # + nsrc[u] gather
-        "agg2_F256": agg_bytes(lnnz, rows, F, extra_row=4),          # + ndst[v]
+        "agg1_F100": agg_bytes(lnnz, rows, F_in, per_edge_extra=4),                # + nsrc[u] gather
+        "agg2_F256": agg_bytes(lnnz, rows, F, extra_row=4),                        # + ndst[v]
         "gat_agg_8x32": agg_bytes(lnnz, rows, HF, per_edge_extra=4 * Hh, extra_row=4 * Hh),
     }
-    dom_name = names[dom]
-    if dom_name not in per_launch:
-        dom_name = max(per_launch, key=lambda k: parts[names.index(k)])
-        dom = names.index(dom_name)
+    dom_name = max(per_launch, key=lambda k: parts[names.index(k)])
+    dom = names.index(dom_name)
     peaks = {}
     try:
         peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -305,39 +219,34 @@ def run_ours(args):
         pass
     peak = float(peaks.get("hbm_gbs", 6650.0))
     achieved = per_launch[dom_name] / (parts[dom] * 1e-3) / 1e9
+    traffic = None
+    try:  # ncu DRAM bytes per launch of this kernel, from the committed profile summary
+        traffic = json.load(open(os.path.join(ROOT, "profiles", "traffic.json"))).get(dom_name)
+    except Exception:
+        pass
     roofline = {"bound": "hbm", "kernel": dom_name, "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                "frac": round(achieved / peak, 4), "traffic": None,
+                "frac": round(achieved / peak, 4), "traffic": traffic,
+                "algorithmic_bytes": int(per_launch[dom_name]), "launch_ms": round(float(parts[dom]), 4),
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)" if "hbm_gbs" in peaks else "fallback 6650"}
 
-    # e2e: same step through the public API with host buffers (pinned), copies inside the timed region
+    # e2e: same step through the public API with host buffers, copies inside the timed region
     e2e = None
     if not args.no_e2e:
         Xh = torch.from_numpy(inp["X"]).pin_memory()
         Yh = torch.empty((rows, HF), dtype=torch.float32).pin_memory()
         h2d = Xh.numel() * 4
         d2h = Yh.numel() * 4
-
-        def upload():
-            if world == 1:
-                X_local.copy_(Xh, non_blocking=True)
-            else:
-                for q in range(world):
-                    a, b = int(bounds[q]), int(bounds[q + 1])
-                    X_local[q * rmax:q * rmax + (b - a)].copy_(Xh[a:b], non_blocking=True)
-
         for _ in range(2):
-            upload()
-            step()
-            Yh.copy_(Y3, non_blocking=True)
+            model.load_input(Xh)
+            Yh.copy_(model.step(), non_blocking=True)
         torch.cuda.synchronize(dev)
         e_s = torch.cuda.Event(enable_timing=True)
         e_e = torch.cuda.Event(enable_timing=True)
         ke = max(1, min(args.steps, 5))
         e_s.record(stream)
         for _ in range(ke):
-            upload()
-            step()
-            Yh.copy_(Y3, non_blocking=True)
+            model.load_input(Xh)
+            Yh.copy_(model.step(), non_blocking=True)
         e_e.record(stream)
         torch.cuda.synchronize(dev)
         me = torch.tensor([e_s.elapsed_time(e_e) / ke], device=dev)
@@ -354,7 +263,7 @@ def run_ours(args):
         "config": {"workload": WORKLOAD, "graph": args.config, "n": n, "nnz": nnz, "rho": args.rho,
                    "reorder": args.reorder, "F": [F_in, F, HF], "heads": Hh, "scale": args.scale,
                    "group_size": info["group_size"], "tile_groups": info["tile_groups"],
-                   "l2": "inputs larger than L2 (X 980 MB, H 2.5 GB vs 126 MB); no flush",
+                   "l2": "inputs larger than L2 (X 980 MB, activations 2.5 GB vs 126 MB); no flush",
                    "parallelism": f"row-partition x{world}" + (" + NCCL all-gather" if world > 1 else "")},
         "breakdown_ms": {k: round(float(v), 4) for k, v in zip(names, parts)},
         "plan": {"build_s": round(plan_s, 2), "gen_s": round(inp["gen_s"], 2), "n_groups": info["n_groups"],

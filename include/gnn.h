@@ -76,11 +76,13 @@ typedef struct {
   int32_t pair_window;   /* W: candidate pairs (m_i, m_{i+d}), 1 <= d <= W (8) */
   int32_t min_sim;       /* re-enqueue threshold; -1 -> lsh_rows */
   int32_t deterministic; /* 1: fixed-order combine (R9); 0: float atomics */
+  int32_t cluster_order; /* LAS schedule: 1 = clusters by representative signature, 0 = by smallest member */
   uint64_t seed;         /* MinHash salt stream seed */
 } gnn_plan_opts;
 
 /* Fill defaults: reorder 0, group_size -1, tile_groups 32, cluster_cap 32,
- * minhash_k 32, lsh_rows 2, pair_window 8, min_sim -1, deterministic 1, seed 0. */
+ * minhash_k 32, lsh_rows 2, pair_window 8, min_sim -1, deterministic 1,
+ * cluster_order 1, seed 0. */
 void gnn_plan_opts_default(gnn_plan_opts *opts);
 
 typedef struct {
@@ -301,7 +303,8 @@ gnn_status gnn_local_csr(int64_t n, const int64_t *rowptr_h, const int32_t *coli
  *   tile_beg_h int64[n_tiles + 1].
  */
 gnn_status gnn_las_host(int64_t n, const int64_t *rowptr_h, const uint64_t *sig_h, int32_t K,
-                        int32_t r, int32_t W, int32_t cap, int32_t min_sim, int32_t *perm_h,
+                        int32_t r, int32_t W, int32_t cap, int32_t min_sim, int32_t cluster_order,
+                        int32_t *perm_h,
                         int32_t *cluster_of_h, int64_t *n_pairs, int64_t *n_clusters);
 gnn_status gnn_groups_host(int64_t n, const int64_t *rowptr_h, const int32_t *perm_h, int32_t ng,
                            int32_t T, int64_t *n_groups, int64_t *n_tiles, int32_t *grp_row_h,

@@ -70,7 +70,7 @@ def lib():
             "orc_minhash": (None, [_i64, _p, _p, _i32, ctypes.c_uint64, _p]),
             "orc_sim": (_i32, [_p, _i32, _i64, _i64]),
             "orc_lsh_pairs": (_i64, [_i64, _p, _p, _i32, _i32, _i32, _p, _i64]),
-            "orc_las_merge": (_i64, [_i64, _p, _i32, _p, _i64, _i32, _i32, _p, _p, _p]),
+            "orc_las_merge": (_i64, [_i64, _p, _i32, _p, _i64, _i32, _i32, _i32, _p, _p, _p]),
             "orc_neighbor_groups": (_i64, [_i64, _p, _p, _i32, _p, _p]),
             "orc_tiles": (_i64, [_i64, _p, _i32, _p]),
             "orc_partition_rows": (None, [_i64, _p, _i32, _p]),
@@ -243,22 +243,23 @@ def lsh_pairs(rowptr, sig, r=2, W=8):
     return pairs[:cnt]
 
 
-def las_merge(sig, pairs, cap=32, min_sim=2):
+def las_merge(sig, pairs, cap=32, min_sim=2, cluster_order=1):
     sig = np.ascontiguousarray(sig, dtype=np.uint64)
     pairs = np.ascontiguousarray(pairs, dtype=np.int32)
     n, K = sig.shape
     perm = np.empty(n, np.int32)
     cl = np.empty(n, np.int32)
     st = np.zeros(3, np.int64)
-    nc = lib().orc_las_merge(n, _ptr(sig), K, _ptr(pairs), len(pairs), cap, min_sim, _ptr(perm), _ptr(cl), _ptr(st))
+    nc = lib().orc_las_merge(n, _ptr(sig), K, _ptr(pairs), len(pairs), cap, min_sim, cluster_order, _ptr(perm),
+                             _ptr(cl), _ptr(st))
     return perm, cl, int(nc), {"merges": int(st[0]), "pops": int(st[1]), "repush": int(st[2])}
 
 
-def las_schedule(rowptr, colidx, K=32, r=2, W=8, cap=32, min_sim=None, seed=0):
+def las_schedule(rowptr, colidx, K=32, r=2, W=8, cap=32, min_sim=None, seed=0, cluster_order=1):
     """Full a2 pipeline: MinHash -> LSH -> merge -> schedule."""
     sig = minhash(rowptr, colidx, K, seed)
     pairs = lsh_pairs(rowptr, sig, r, W)
-    perm, cl, nc, st = las_merge(sig, pairs, cap, r if min_sim is None else min_sim)
+    perm, cl, nc, st = las_merge(sig, pairs, cap, r if min_sim is None else min_sim, cluster_order)
     return perm, {"sig": sig, "pairs": pairs, "cluster_of": cl, "n_clusters": nc, **st}
 
 

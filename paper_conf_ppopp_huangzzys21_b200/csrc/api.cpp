@@ -93,6 +93,7 @@ void gnn_plan_opts_default(gnn_plan_opts *o) {
   o->pair_window = 8;
   o->min_sim = -1;
   o->deterministic = 1;
+  o->cluster_order = 1;
   o->seed = 0;
 }
 
@@ -224,7 +225,8 @@ gnn_status gnn_plan_create_ex(int64_t n, int64_t n_src, int64_t nnz, const int64
       p->info.ms_lsh = ms_since(t0);
       t0 = std::chrono::steady_clock::now();
       const int32_t min_sim = opts.min_sim < 0 ? opts.lsh_rows : opts.min_sim;
-      p->n_clusters = las_merge(n, p->sig.data(), K, p->pairs, opts.cluster_cap, min_sim, p->perm, p->cluster_of);
+      p->n_clusters = las_merge(n, p->sig.data(), K, p->pairs, opts.cluster_cap, min_sim, opts.cluster_order, p->perm,
+                                p->cluster_of);
       p->info.ms_merge = ms_since(t0);
     } else {
       p->perm.resize((size_t)n);
@@ -658,14 +660,15 @@ gnn_status gnn_local_csr(int64_t n, const int64_t *rowptr_h, const int32_t *coli
 }
 
 gnn_status gnn_las_host(int64_t n, const int64_t *rowptr_h, const uint64_t *sig_h, int32_t K, int32_t r,
-                        int32_t W, int32_t cap, int32_t min_sim, int32_t *perm_h, int32_t *cluster_of_h,
+                        int32_t W, int32_t cap, int32_t min_sim, int32_t cluster_order, int32_t *perm_h,
+                        int32_t *cluster_of_h,
                         int64_t *n_pairs, int64_t *n_clusters) {
   GNN_TRY({
     if (n < 0 || !rowptr_h || (n > 0 && !sig_h) || !perm_h) return check(false, "bad las_host arguments");
     if (K < 1 || r < 1 || K % r || W < 1 || cap < 1) return check(false, "bad LAS parameters");
     std::vector<int32_t> pairs, perm, cl;
     const int64_t np = las_lsh_pairs(n, rowptr_h, sig_h, K, r, W, pairs);
-    const int64_t nc = las_merge(n, sig_h, K, pairs, cap, min_sim < 0 ? r : min_sim, perm, cl);
+    const int64_t nc = las_merge(n, sig_h, K, pairs, cap, min_sim < 0 ? r : min_sim, cluster_order, perm, cl);
     std::memcpy(perm_h, perm.data(), sizeof(int32_t) * (size_t)n);
     if (cluster_of_h) std::memcpy(cluster_of_h, cl.data(), sizeof(int32_t) * (size_t)n);
     if (n_pairs) *n_pairs = np;

@@ -69,7 +69,7 @@ void schedule_host(int64_t n, const int64_t *rowptr, const int32_t *perm, int64_
 int64_t las_lsh_pairs(int64_t n, const int64_t *rowptr, const uint64_t *sig, int32_t K, int32_t r,
                       int32_t W, std::vector<int32_t> &pairs);
 int64_t las_merge(int64_t n, const uint64_t *sig, int32_t K, const std::vector<int32_t> &pairs,
-                  int32_t cap, int32_t min_sim, std::vector<int32_t> &perm,
+                  int32_t cap, int32_t min_sim, int32_t cluster_order, std::vector<int32_t> &perm,
                   std::vector<int32_t> &cluster_of);
 
 // kernels (k_graph.cu)

@@ -254,13 +254,17 @@ __device__ __forceinline__ void gat_merge(float &m1, float &l1, float *a1, float
   m1 = m;
 }
 
-// group partial over CSR entries [beg, end) of destination `row`
+// group partial over CSR entries [beg, end) of destination `row`.
+// Rolling register ring: U source rows stay in flight per worker (a row is
+// re-requested as soon as its slot is consumed); the next batch of LANES
+// indices is requested before the current batch is consumed.  Consumption
+// order is CSR order, so the fp32 chain is exactly R9's.
 template <int MODE, int VEC, int NV, int LANES>
 __device__ __forceinline__ void group_partial(const KParams &p, int32_t beg, int32_t end, int32_t row,
                                               int32_t c0, int lane, unsigned mask,
                                               Part<MODE, VEC, NV> &P) {
   constexpr int FPL = VEC * NV;  // floats per lane per source row
-  constexpr int U = FPL <= 8 ? 8 : (FPL <= 16 ? 4 : 2);
+  constexpr int U = FPL >= 32 ? 1 : (32 / FPL > 8 ? 8 : 32 / FPL);
   part_init(P);
   bool valid[NV];
   int32_t head[NV];
@@ -277,57 +281,64 @@ __device__ __forceinline__ void group_partial(const KParams &p, int32_t beg, int
     }
   }
   const int weight = p.weight;
-  for (int32_t k = beg; k < end; k += LANES) {
-    const int32_t cnt = min(LANES, end - k);
-    int32_t my_u = 0;
-    float my_w = 1.0f;
+  auto load_idx = [&](int32_t k, int32_t cnt, int32_t &u, float &w) {
+    u = 0;
+    w = 1.0f;
     if (lane < cnt) {
-      my_u = ld_stream_i32(p.g.colidx + k + lane);
+      u = ld_stream_i32(p.g.colidx + k + lane);
       if constexpr (MODE != M_GAT) {
-        if (weight == GNN_W_GCN) my_w = __ldg(p.g.nsrc + my_u);
-        else if (weight == GNN_W_EDGE) my_w = ld_stream_f32(p.edge_w + k + lane);
+        if (weight == GNN_W_GCN) w = __ldg(p.g.nsrc + u);
+        else if (weight == GNN_W_EDGE) w = ld_stream_f32(p.edge_w + k + lane);
       }
     }
+  };
+  float v[U][NV][VEC];
+  float sc[U][NV];
+  auto load_row = [&](int q, int32_t u) {
+    const float *xr = p.X + (int64_t)u * p.ldx;
+#pragma unroll
+    for (int n = 0; n < NV; ++n) {
+      if (valid[n]) ldv<VEC>(xr + c0 + (n * LANES + lane) * VEC, v[q][n]);
+      if constexpr (MODE == M_GAT) sc[q][n] = valid[n] ? __ldg(xr + p.F + head[n]) : 0.0f;
+    }
+  };
+  int32_t k = beg;
+  int32_t cnt = min(LANES, end - k);
+  int32_t my_u;
+  float my_w;
+  load_idx(k, cnt, my_u, my_w);
+  for (;;) {
+    // next index batch in flight while this one is consumed
+    const int32_t kn = k + LANES;
+    const int32_t cnt_n = kn < end ? min(LANES, end - kn) : 0;
+    int32_t nx_u;
+    float nx_w;
+    load_idx(kn, cnt_n, nx_u, nx_w);
+#pragma unroll
+    for (int q = 0; q < U; ++q)
+      if (q < cnt) load_row(q, __shfl_sync(mask, my_u, q, LANES));
     for (int32_t j = 0; j < cnt; j += U) {
-      float v[U][NV][VEC];
-      float sc[U][NV];
-      int32_t uu[U];
 #pragma unroll
       for (int q = 0; q < U; ++q) {
-        uu[q] = 0;
-        if (j + q < cnt) uu[q] = __shfl_sync(mask, my_u, j + q, LANES);
-      }
-#pragma unroll
-      for (int q = 0; q < U; ++q) {
-        if (j + q < cnt) {
-          const float *xr = p.X + (int64_t)uu[q] * p.ldx;
-#pragma unroll
-          for (int n = 0; n < NV; ++n) {
-            if (valid[n]) ldv<VEC>(xr + c0 + (n * LANES + lane) * VEC, v[q][n]);
-            if constexpr (MODE == M_GAT) sc[q][n] = valid[n] ? __ldg(xr + p.F + head[n]) : 0.0f;
-          }
-        }
-      }
-#pragma unroll
-      for (int q = 0; q < U; ++q) {
-        if (j + q < cnt) {
+        const int32_t e = j + q;
+        if (e < cnt) {
           if constexpr (MODE == M_GAT) {
 #pragma unroll
             for (int n = 0; n < NV; ++n) {
               if (!valid[n]) continue;
-              float e = sc[q][n] + tv[n];
-              e = e > 0.0f ? e : p.slope * e;  // LeakyReLU (Table 2 GAT)
-              const float d = e - P.m[n];
+              float sco = sc[q][n] + tv[n];
+              sco = sco > 0.0f ? sco : p.slope * sco;  // LeakyReLU (Table 2 GAT)
+              const float d = sco - P.m[n];
               const float ex = __expf(-fabsf(d));
               const bool up = d > 0.0f;
 #pragma unroll
               for (int i = 0; i < VEC; ++i)
                 P.a[n][i] = fmaf(up ? P.a[n][i] : v[q][n][i], ex, up ? v[q][n][i] : P.a[n][i]);
               P.l[n] = fmaf(up ? P.l[n] : 1.0f, ex, up ? 1.0f : P.l[n]);
-              P.m[n] = up ? e : P.m[n];
+              P.m[n] = up ? sco : P.m[n];
             }
           } else {
-            const float w = __shfl_sync(mask, my_w, j + q, LANES);
+            const float w = __shfl_sync(mask, my_w, e, LANES);
 #pragma unroll
             for (int n = 0; n < NV; ++n) {
               if (!valid[n]) continue;
@@ -338,9 +349,15 @@ __device__ __forceinline__ void group_partial(const KParams &p, int32_t beg, int
               }
             }
           }
+          if (e + U < cnt) load_row(q, __shfl_sync(mask, my_u, e + U, LANES));
         }
       }
     }
+    if (cnt_n == 0) break;
+    k = kn;
+    cnt = cnt_n;
+    my_u = nx_u;
+    my_w = nx_w;
   }
 }
 
@@ -432,8 +449,11 @@ __device__ __forceinline__ void slot_load(const float *smem, int T, int j, int l
   }
 }
 
+#ifndef GNN_AGG_MINB
+#define GNN_AGG_MINB 4
+#endif
 template <int MODE, int VEC, int NV, int LANES>
-__global__ void __launch_bounds__(256) k_aggregate(const KParams p) {
+__global__ void __launch_bounds__(256, MODE == M_GAT ? GNN_AGG_MINB - 1 : GNN_AGG_MINB) k_aggregate(const KParams p) {
   extern __shared__ float smem[];
   constexpr int CW = LANES * VEC * NV;
   __shared__ int s_last;

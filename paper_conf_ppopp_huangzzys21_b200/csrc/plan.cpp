@@ -162,7 +162,7 @@ inline int32_t sim_of(const uint64_t *sig, int32_t K, int64_t a, int64_t b) {
 
 // Pair merging and task scheduling; spec R7.
 int64_t las_merge(int64_t n, const uint64_t *sig, int32_t K, const std::vector<int32_t> &pairs,
-                  int32_t cap, int32_t min_sim, std::vector<int32_t> &perm,
+                  int32_t cap, int32_t min_sim, int32_t cluster_order, std::vector<int32_t> &perm,
                   std::vector<int32_t> &cluster_of) {
   std::vector<int32_t> parent((size_t)n), size((size_t)n, 1);
   for (int64_t v = 0; v < n; ++v) parent[v] = (int32_t)v;
@@ -199,22 +199,36 @@ int64_t las_merge(int64_t n, const uint64_t *sig, int32_t K, const std::vector<i
       }
     }
   }
-  // clusters ordered by smallest member, members ascending
+  // schedule (R7): clusters ordered by (representative signature,
+  // smallest member) when cluster_order == 1, by smallest member when 0;
+  // members ascending
   std::vector<int64_t> cnt((size_t)n, 0), off((size_t)n, -1);
-  for (int64_t v = 0; v < n; ++v) cnt[find(v)]++;
-  perm.assign((size_t)n, 0);
-  cluster_of.assign((size_t)n, 0);
-  int64_t pos = 0, nc = 0;
+  std::vector<std::pair<int64_t, int64_t>> cl;  // (representative, smallest member)
   for (int64_t v = 0; v < n; ++v) {
     const int64_t r = find(v);
-    if (off[r] < 0) {
-      off[r] = pos;
-      pos += cnt[r];
-      ++nc;
-    }
+    if (cnt[r]++ == 0) cl.emplace_back(r, v);
+  }
+  if (cluster_order == 1) {
+    std::sort(cl.begin(), cl.end(), [&](const std::pair<int64_t, int64_t> &x, const std::pair<int64_t, int64_t> &y) {
+      const uint64_t *sa = sig + (size_t)x.first * K, *sb = sig + (size_t)y.first * K;
+      for (int32_t k = 0; k < K; ++k)
+        if (sa[k] != sb[k]) return sa[k] < sb[k];
+      return x.second < y.second;
+    });
+  }
+  int64_t pos = 0;
+  for (const auto &c : cl) {
+    off[c.first] = pos;
+    pos += cnt[c.first];
+  }
+  perm.assign((size_t)n, 0);
+  cluster_of.assign((size_t)n, 0);
+  for (int64_t v = 0; v < n; ++v) {
+    const int64_t r = find(v);
     perm[off[r]++] = (int32_t)v;
     cluster_of[v] = (int32_t)r;
   }
+  const int64_t nc = (int64_t)cl.size();
   return nc;
 }
 

@@ -16,7 +16,7 @@ import os
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libgnn.so")
+LIB_PATH = os.environ.get("GNN_LIB_PATH") or os.path.join(_PKG, "libgnn.so")  # override: dev A/B builds only
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} not built: run `python -m paper_conf_ppopp_huangzzys21_b200.build` "
@@ -43,7 +43,7 @@ class gnn_plan_opts(ctypes.Structure):
     _fields_ = [("struct_size", ctypes.c_uint32), ("reorder", ctypes.c_int32), ("group_size", ctypes.c_int32),
                 ("tile_groups", ctypes.c_int32), ("cluster_cap", ctypes.c_int32), ("minhash_k", ctypes.c_int32),
                 ("lsh_rows", ctypes.c_int32), ("pair_window", ctypes.c_int32), ("min_sim", ctypes.c_int32),
-                ("deterministic", ctypes.c_int32), ("seed", ctypes.c_uint64)]
+                ("deterministic", ctypes.c_int32), ("cluster_order", ctypes.c_int32), ("seed", ctypes.c_uint64)]
 
 
 class gnn_plan_info(ctypes.Structure):
@@ -85,7 +85,7 @@ _SIGS = {
     "gnn_partition_rows": (ctypes.c_int, [_I64, _P, _I32, _P]),
     "gnn_local_csr": (ctypes.c_int, [_I64, _P, _P, _P, _I32, _I32, ctypes.POINTER(_I64), ctypes.POINTER(_I64),
                                      _P, _P, _P]),
-    "gnn_las_host": (ctypes.c_int, [_I64, _P, _P, _I32, _I32, _I32, _I32, _I32, _P, _P, ctypes.POINTER(_I64),
+    "gnn_las_host": (ctypes.c_int, [_I64, _P, _P, _I32, _I32, _I32, _I32, _I32, _I32, _P, _P, ctypes.POINTER(_I64),
                                     ctypes.POINTER(_I64)]),
     "gnn_groups_host": (ctypes.c_int, [_I64, _P, _P, _I32, _I32, ctypes.POINTER(_I64), ctypes.POINTER(_I64), _P, _P,
                                        _P]),
@@ -328,7 +328,7 @@ def local_csr(rowptr, colidx, bounds, rank):
     return lrp, lci[:lnnz.value], sdeg[:P * rmax.value], rmax.value
 
 
-def las_host(rowptr, sig, r=2, W=8, cap=32, min_sim=-1):
+def las_host(rowptr, sig, r=2, W=8, cap=32, min_sim=-1, cluster_order=1):
     """a2 steps 2-5 on the host from given MinHash signatures (no GPU)."""
     rowptr = np.ascontiguousarray(rowptr, dtype=np.int64)
     sig = np.ascontiguousarray(sig, dtype=np.uint64)
@@ -336,7 +336,8 @@ def las_host(rowptr, sig, r=2, W=8, cap=32, min_sim=-1):
     perm = np.empty(n, np.int32)
     cl = np.empty(n, np.int32)
     npairs, nc = ctypes.c_int64(), ctypes.c_int64()
-    _call("gnn_las_host", n, _np_ptr(rowptr), _np_ptr(sig), K, r, W, cap, min_sim, _np_ptr(perm), _np_ptr(cl),
+    _call("gnn_las_host", n, _np_ptr(rowptr), _np_ptr(sig), K, r, W, cap, min_sim, cluster_order, _np_ptr(perm),
+          _np_ptr(cl),
           ctypes.byref(npairs), ctypes.byref(nc))
     return perm, cl, npairs.value, nc.value
 

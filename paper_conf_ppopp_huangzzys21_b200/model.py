@@ -1,0 +1,132 @@
+"""The C5 forward step on 1..P GPUs (a10: destination-row partitioning with a
+per-layer all-gather of transformed source rows, reading R10).
+
+Every arithmetic step runs in libgnn.so kernels through the C-ABI; this module
+only owns buffers, the order of calls and the collective.
+
+    layer 1  Y1 = ReLU((A_gcn X) W1)   aggregate-first (X replicated: no exchange)
+    layer 2  Y2 = A_gcn (Y1 W2)        transform-first: Hs = (Y1 W2) * nsrc, all-gather, aggregate * ndst
+    layer 3  Y3 = GAT_HxFh(Y2)         [Z|s|t] = Y2 W', all-gather, fused edge-softmax aggregation
+
+Rank p owns destination rows [bounds[p], bounds[p+1]); sources live in the
+padded layout u -> owner(u) * r_max + (u - bounds[owner]).  With the
+deterministic plan option the concatenated P-rank output is bit-identical to
+P = 1 (the per-row arithmetic depends only on (CSR, ng, F), R9).
+"""
+from __future__ import annotations
+
+import ctypes
+
+import numpy as np
+import torch
+
+from . import gnn as _g
+
+
+class RowPartitionedGCNGAT:
+    def __init__(self, rowptr, colidx, W1, W2, W3, a_src, a_dst, heads, head_dim, neg_slope=0.2,
+                 rank=0, world=1, group=None, reorder=1, device=None, plan_opts=None, staged_allgather=False):
+        self.rank, self.world, self.group = rank, world, group
+        self.dev = device or torch.device("cuda", torch.cuda.current_device())
+        self.staged = staged_allgather  # gloo: exchange through host memory (tests only)
+        n = len(rowptr) - 1
+        self.n = n
+        opts = dict(reorder=reorder, **(plan_opts or {}))
+        if world == 1:
+            self.bounds = np.array([0, n], np.int64)
+            self.rmax = n
+            self.plan = _g.Plan(rowptr, colidx, **opts)
+        else:
+            self.bounds = _g.partition_rows(rowptr, world)
+            lrp, lci, sdeg, rmax = _g.local_csr(rowptr, colidx, self.bounds, rank)
+            self.rmax = rmax
+            self.plan = _g.Plan(lrp, lci, n_src=world * rmax, src_degree=sdeg, **opts)
+        self.lo, self.hi = int(self.bounds[rank]), int(self.bounds[rank + 1])
+        self.rows = self.hi - self.lo
+        self.nnz_local = int(rowptr[self.hi] - rowptr[self.lo])
+        d = self.dev
+        self.W1 = torch.as_tensor(W1, device=d).contiguous()
+        self.W2 = torch.as_tensor(W2, device=d).contiguous()
+        self.W3 = torch.as_tensor(W3, device=d).contiguous()
+        self.a_s = torch.as_tensor(a_src, device=d).contiguous()
+        self.a_d = torch.as_tensor(a_dst, device=d).contiguous()
+        self.F_in, self.F = self.W1.shape
+        self.H, self.Fh = heads, head_dim
+        self.HF = heads * head_dim
+        self.slope = float(neg_slope)
+        self.ldwe = (self.HF + 2 * heads + 7) // 8 * 8
+        R, P = self.rows, world * self.rmax
+        self.Xs = torch.zeros((P, self.F_in), device=d)          # replicated input, padded layout
+        self.A1 = torch.empty((R, self.F_in), device=d)
+        self.Y1 = torch.empty((R, self.F), device=d)
+        self.Hs2 = torch.zeros((P, self.F), device=d)
+        self.Y2 = torch.empty((R, self.F), device=d)
+        self.Wext = torch.empty((self.F, self.ldwe), device=d)
+        self.Zst = torch.zeros((P, self.ldwe), device=d)
+        self.Y3 = torch.empty((R, self.HF), device=d)
+        self.nsrc_ptr, _ = self.plan.normalizers()
+        self.ws_agg, self.ws_agg_b = self.plan.workspace(_g.GNN_OP_AGGREGATE, 0, max(self.F, self.F_in), 0, d)
+        self.ws_gat, self.ws_gat_b = self.plan.workspace(_g.GNN_OP_GAT_AGGREGATE, 0, self.HF, heads, d)
+        self.names = ["agg1", "gemm1", "gemm2+xchg", "agg2", "gemm3+xchg", "gat_agg"]
+
+    # -- inputs -------------------------------------------------------------
+    def load_input(self, X_host_or_dev, non_blocking=True):
+        """X [n, F_in] (host pinned or device) -> the replicated padded buffer."""
+        for q in range(self.world):
+            a, b = int(self.bounds[q]), int(self.bounds[q + 1])
+            self.Xs[q * self.rmax:q * self.rmax + (b - a)].copy_(X_host_or_dev[a:b], non_blocking=non_blocking)
+
+    # -- exchange -----------------------------------------------------------
+    def _allgather(self, buf):
+        if self.world == 1:
+            return
+        import torch.distributed as dist
+        mine = buf[self.rank * self.rmax:(self.rank + 1) * self.rmax]
+        if self.staged:
+            out = torch.empty((self.world * self.rmax, buf.shape[1]), dtype=buf.dtype)
+            dist.all_gather_into_tensor(out, mine.cpu(), group=self.group)
+            buf.copy_(out)
+        else:
+            dist.all_gather_into_tensor(buf, mine.clone(), group=self.group)
+
+    # -- the step -----------------------------------------------------------
+    def step(self, stream=None, events=None):
+        lib = _g._lib
+        s = torch.cuda.current_stream(self.dev) if stream is None else stream
+        sp = ctypes.c_void_p(s.cuda_stream)
+        P = lambda t: ctypes.c_void_p(t.data_ptr())  # noqa: E731
+        rec = (lambda i: events[i].record(s)) if events else (lambda i: None)
+        R, F, Fi, HF, H = self.rows, self.F, self.F_in, self.HF, self.H
+        off = self.rank * self.rmax
+
+        def chk(st, what):
+            if st != 0:
+                raise _g.GnnError(what, st)
+
+        rec(0)
+        chk(lib.gnn_aggregate(self.plan.handle, _g.GNN_SUM, _g.GNN_W_GCN, None, P(self.Xs), Fi, Fi, P(self.A1), Fi,
+                              0, None, 0, P(self.ws_agg), self.ws_agg_b, sp), "agg1")
+        rec(1)
+        chk(lib.gnn_gemm(P(self.A1), Fi, P(self.W1), F, P(self.Y1), F, R, Fi, F, None, None, 1, sp), "gemm1")
+        rec(2)
+        h_loc = self.Hs2[off:off + R]
+        chk(lib.gnn_gemm(P(self.Y1), F, P(self.W2), F, P(h_loc), F, R, F, F,
+                         ctypes.c_void_p(self.nsrc_ptr + 4 * off), None, 0, sp), "gemm2")
+        self._allgather(self.Hs2)
+        rec(3)
+        chk(lib.gnn_gcn_aggregate_prescaled(self.plan.handle, P(self.Hs2), F, F, P(self.Y2), F, 0, P(self.ws_agg),
+                                            self.ws_agg_b, sp), "agg2")
+        rec(4)
+        chk(lib.gnn_gat_fold_weights(P(self.W3), P(self.a_s), P(self.a_d), F, H, self.Fh, P(self.Wext), self.ldwe,
+                                     sp), "gat fold")
+        z_loc = self.Zst[off:off + R]
+        chk(lib.gnn_gemm(P(self.Y2), F, P(self.Wext), self.ldwe, P(z_loc), self.ldwe, R, F, self.ldwe, None, None, 0,
+                         sp), "gemm3")
+        self._allgather(self.Zst)
+        rec(5)
+        tptr = ctypes.c_void_p(z_loc.data_ptr() + 4 * (HF + H))
+        chk(lib.gnn_gat_aggregate(self.plan.handle, P(self.Zst), self.ldwe, tptr, self.ldwe, H, self.Fh,
+                                  ctypes.c_float(self.slope), P(self.Y3), HF, P(self.ws_gat), self.ws_gat_b, sp),
+            "gat agg")
+        rec(6)
+        return self.Y3

@@ -42,7 +42,7 @@ def test_version_and_defaults():
     assert "sm_100a" in P.gnn.gnn_version()
     o = P.gnn.default_opts()
     assert (o.reorder, o.group_size, o.tile_groups, o.cluster_cap, o.minhash_k, o.lsh_rows, o.pair_window,
-            o.min_sim, o.deterministic) == (0, -1, 32, 32, 32, 2, 8, -1, 1)
+            o.min_sim, o.deterministic, o.cluster_order) == (0, -1, 32, 32, 32, 2, 8, -1, 1, 1)
 
 
 def _create(rowptr, colidx, n=None, **kw):
@@ -106,6 +106,9 @@ def test_las_host_bit_exact_vs_oracle(seed, rho):
     assert nc == info["n_clusters"]
     assert np.array_equal(perm, perm_o)
     assert np.array_equal(cl, info["cluster_of"])
+    perm0, _, _, _ = P.las_host(g.rowptr, info["sig"], cluster_order=0)
+    operm0, _, _, _ = oracle.las_merge(info["sig"], info["pairs"], 32, 2, cluster_order=0)
+    assert np.array_equal(perm0, operm0)
 
 
 def test_las_host_other_parameters():

@@ -457,7 +457,9 @@ def test_las_invariants_powerlaw(seed):
     cl = info["cluster_of"]
     sizes = np.bincount(cl, minlength=n)
     assert sizes.max() <= 32
-    # members of a cluster are contiguous in perm and ascending; clusters ordered by min member
+    # members of a cluster are contiguous in perm and ascending; clusters ordered by
+    # (representative signature, min member) (R7)
+    sig_ = info["sig"]
     seen = []
     i = 0
     while i < n:
@@ -467,9 +469,13 @@ def test_las_invariants_powerlaw(seed):
             j += 1
         assert j - i == sizes[c]
         assert np.all(np.diff(perm[i:j]) > 0)
-        seen.append(perm[i])
+        seen.append((tuple(int(x) for x in sig_[c]), int(perm[i])))
         i = j
-    assert np.all(np.diff(seen) > 0)
+    assert seen == sorted(seen)
+    # the smallest-member order (cluster_order 0) is the other option
+    perm0, _, _, _ = oracle.las_merge(info["sig"], info["pairs"], 32, 2, cluster_order=0)
+    heads = [int(v) for k, v in enumerate(perm0) if k == 0 or cl[perm0[k - 1]] != cl[v]]
+    assert heads == sorted(heads)
     # every candidate pair shares a full band (LSH bucket); sim >= r
     sig, pairs = info["sig"], info["pairs"]
     for a, b in pairs[:2000]:
