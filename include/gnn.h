@@ -226,10 +226,15 @@ gnn_status gnn_edgeconv(gnn_plan_t plan, const float *X, int64_t ldx, int32_t f_
  * X: [m, ldx] (k used), W: [k, ldw] (n used), H: [m, ldh].
  * Epilogue: row_scale (nullable, [m]) multiplies row i; col_bias (nullable, [n])
  * is added after the scale; relu != 0 clamps.  H must not overlap X or W.
+ * With ws (>= gnn_gemm_workspace_size(m, k, n) bytes, 256-byte aligned) and
+ * n <= 512 the tcgen05 3xTF32 tensor-core kernel runs (the workspace holds the
+ * split, pre-swizzled W image); with ws == NULL the SIMT fp32 FFMA kernel runs.
  */
 gnn_status gnn_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H,
                     int64_t ldh, int64_t m, int32_t k, int32_t n, const float *row_scale,
-                    const float *col_bias, int32_t relu, gnn_stream_t stream);
+                    const float *col_bias, int32_t relu, void *ws, size_t ws_bytes,
+                    gnn_stream_t stream);
+size_t gnn_gemm_workspace_size(int64_t m, int32_t k, int32_t n);
 
 /* GEMM implementation selector (process-wide): 0 = auto, 1 = SIMT FFMA,
  * 2 = tcgen05 3xTF32.  Returns the previous value. */

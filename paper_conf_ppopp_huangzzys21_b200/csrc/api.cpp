@@ -297,15 +297,17 @@ gnn_status gnn_plan_destroy(gnn_plan_t p) {
   })
 }
 
+// layer workspaces: [GEMM W image][layer buffers][aggregation workspace]
 static size_t ws_gat_layer_head(int64_t n, int32_t f_in, int32_t HF, int32_t H, int32_t *ldwe) {
   const int32_t ld = ((HF + 2 * H) + 7) / 8 * 8;
   if (ldwe) *ldwe = ld;
-  return align256(sizeof(float) * (size_t)f_in * ld) + align256(sizeof(float) * (size_t)n * ld);
+  return align256(gemm_tc_workspace(n, f_in, ld)) + align256(sizeof(float) * (size_t)f_in * ld) +
+         align256(sizeof(float) * (size_t)n * ld);
 }
 static size_t ws_edgeconv_head(int64_t n, int32_t f_in, int32_t f_out) {
   const size_t ld = 2 * (size_t)f_out;
-  return align256(sizeof(float) * (size_t)f_in * ld) + align256(sizeof(float) * ld) +
-         align256(sizeof(float) * (size_t)n * ld);
+  return align256(gemm_tc_workspace(n, f_in, (int32_t)ld)) + align256(sizeof(float) * (size_t)f_in * ld) +
+         align256(sizeof(float) * ld) + align256(sizeof(float) * (size_t)n * ld);
 }
 static int32_t ld8(int32_t f) { return (f + 7) / 8 * 8; }
 
@@ -320,8 +322,10 @@ size_t gnn_workspace_size(gnn_plan_t p, int op, int32_t f_in, int32_t f_out, int
     case GNN_OP_GCN_LAYER: {
       const bool tf = f_out <= f_in;  // auto order; both orders fit in max()
       (void)tf;
-      const size_t a = align256(sizeof(float) * (size_t)p->n_src * ld8(f_out)) + agg_workspace_bytes(p, 0, f_out, 0);
-      const size_t b = align256(sizeof(float) * (size_t)p->n * ld8(f_in)) + agg_workspace_bytes(p, 0, f_in, 0);
+      const size_t a = align256(gemm_tc_workspace(p->n_src, f_in, f_out)) +
+                       align256(sizeof(float) * (size_t)p->n_src * ld8(f_out)) + agg_workspace_bytes(p, 0, f_out, 0);
+      const size_t b = align256(gemm_tc_workspace(p->n, f_in, f_out)) +
+                       align256(sizeof(float) * (size_t)p->n * ld8(f_in)) + agg_workspace_bytes(p, 0, f_in, 0);
       return a > b ? a : b;
     }
     default: return 0;
@@ -391,9 +395,11 @@ gnn_status gnn_gat_aggregate(gnn_plan_t p, const float *Zs, int64_t ldz, const f
   })
 }
 
+size_t gnn_gemm_workspace_size(int64_t m, int32_t k, int32_t n) { return gemm_tc_workspace(m, k, n); }
+
 gnn_status gnn_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H, int64_t ldh,
                     int64_t m, int32_t k, int32_t n, const float *row_scale, const float *col_bias,
-                    int32_t relu, gnn_stream_t stream) {
+                    int32_t relu, void *ws, size_t ws_bytes, gnn_stream_t stream) {
   GNN_TRY({
     if (m < 0 || k < 0 || n < 0) return check(false, "negative GEMM size");
     if (m == 0 || n == 0) return GNN_OK;
@@ -402,7 +408,8 @@ gnn_status gnn_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw, fl
     if (overlaps(H, span_bytes(m, ldh, n), X, span_bytes(m, ldx, k)) ||
         overlaps(H, span_bytes(m, ldh, n), W, span_bytes(k, ldw, n)))
       return check(false, "H overlaps X or W");
-    return launch_gemm(X, ldx, W, ldw, H, ldh, m, k, n, row_scale, col_bias, relu, (cudaStream_t)stream);
+    return launch_gemm(X, ldx, W, ldw, H, ldh, m, k, n, row_scale, col_bias, relu, ws, ws_bytes,
+                       (cudaStream_t)stream);
   })
 }
 
@@ -426,12 +433,13 @@ gnn_status gnn_gat_layer(gnn_plan_t p, const float *X, int64_t ldx, int32_t f_in
       return GNN_ERR_WORKSPACE;
     }
     char *base = (char *)ws;
-    float *Wext = (float *)base;
-    float *Zst = (float *)(base + align256(sizeof(float) * (size_t)f_in * ldwe));
+    const size_t gws = align256(gemm_tc_workspace(p->n, f_in, ldwe));
+    float *Wext = (float *)(base + gws);
+    float *Zst = (float *)(base + gws + align256(sizeof(float) * (size_t)f_in * ldwe));
     cudaStream_t s = (cudaStream_t)stream;
     cudaError_t e = launch_gat_weights(W, a_src, a_dst, f_in, H, Fh, Wext, ldwe, s);
     if (e != cudaSuccess) return cuda_status(e, "gat weights");
-    gnn_status st = launch_gemm(X, ldx, Wext, ldwe, Zst, ldwe, p->n, f_in, ldwe, nullptr, nullptr, 0, s);
+    gnn_status st = launch_gemm(X, ldx, Wext, ldwe, Zst, ldwe, p->n, f_in, ldwe, nullptr, nullptr, 0, base, gws, s);
     if (st != GNN_OK) return st;
     AggArgs a{};
     a.mode = 3;
@@ -491,13 +499,14 @@ gnn_status gnn_edgeconv(gnn_plan_t p, const float *X, int64_t ldx, int32_t f_in,
     }
     const int64_t ld = 2 * (int64_t)f_out;
     char *base = (char *)ws;
-    float *Wpq = (float *)base;
-    float *bpq = (float *)(base + align256(sizeof(float) * (size_t)f_in * ld));
+    const size_t gws = align256(gemm_tc_workspace(p->n, f_in, (int32_t)ld));
+    float *Wpq = (float *)(base + gws);
+    float *bpq = (float *)(base + gws + align256(sizeof(float) * (size_t)f_in * ld));
     float *PQ = (float *)((char *)bpq + align256(sizeof(float) * ld));
     cudaStream_t s = (cudaStream_t)stream;
     cudaError_t e = launch_edgeconv_weights(theta, phi, bias, f_in, f_out, Wpq, bpq, s);
     if (e != cudaSuccess) return cuda_status(e, "edgeconv weights");
-    gnn_status st = launch_gemm(X, ldx, Wpq, ld, PQ, ld, p->n, f_in, (int32_t)ld, nullptr, bpq, 0, s);
+    gnn_status st = launch_gemm(X, ldx, Wpq, ld, PQ, ld, p->n, f_in, (int32_t)ld, nullptr, bpq, 0, base, gws, s);
     if (st != GNN_OK) return st;
     return gnn_edgeconv_aggregate(p, PQ, ld, f_out, Y, ldy, base + head, ws_bytes - head, stream);
   })
@@ -517,14 +526,15 @@ gnn_status gnn_gcn_layer(gnn_plan_t p, const float *X, int64_t ldx, int32_t f_in
     if (order == 1) {
       // transform first: Hs = (X W) * nsrc[u]; y = ndst[v] * sum_u Hs[u]  (Eq 1 reassociated, R4-i)
       const int32_t ldh = ld8(f_out);
-      const size_t head = align256(sizeof(float) * (size_t)p->n_src * ldh);
+      const size_t gws = align256(gemm_tc_workspace(p->n_src, f_in, f_out));
+      const size_t head = gws + align256(sizeof(float) * (size_t)p->n_src * ldh);
       const size_t need = head + agg_workspace_bytes(p, 0, f_out, 0);
       if (!ws || ws_bytes < need) {
         set_error("workspace too small: need " + std::to_string(need));
         return GNN_ERR_WORKSPACE;
       }
-      float *Hs = (float *)ws;
-      gnn_status st = launch_gemm(X, ldx, W, ldw, Hs, ldh, p->n_src, f_in, f_out, p->dg.nsrc, nullptr, 0, s);
+      float *Hs = (float *)((char *)ws + gws);
+      gnn_status st = launch_gemm(X, ldx, W, ldw, Hs, ldh, p->n_src, f_in, f_out, p->dg.nsrc, nullptr, 0, ws, gws, s);
       if (st != GNN_OK) return st;
       AggArgs a{};
       a.mode = 0;
@@ -539,13 +549,14 @@ gnn_status gnn_gcn_layer(gnn_plan_t p, const float *X, int64_t ldx, int32_t f_in
     }
     // aggregate first: A = A_gcn X; Y = ACT(A W)
     const int32_t lda = ld8(f_in);
-    const size_t head = align256(sizeof(float) * (size_t)p->n * lda);
+    const size_t gws = align256(gemm_tc_workspace(p->n, f_in, f_out));
+    const size_t head = gws + align256(sizeof(float) * (size_t)p->n * lda);
     const size_t need = head + agg_workspace_bytes(p, 0, f_in, 0);
     if (!ws || ws_bytes < need) {
       set_error("workspace too small: need " + std::to_string(need));
       return GNN_ERR_WORKSPACE;
     }
-    float *A = (float *)ws;
+    float *A = (float *)((char *)ws + gws);
     AggArgs a{};
     a.mode = 0;
     a.weight = GNN_W_GCN;
@@ -556,7 +567,7 @@ gnn_status gnn_gcn_layer(gnn_plan_t p, const float *X, int64_t ldx, int32_t f_in
     a.ldy = lda;
     gnn_status st = agg_common(p, a, (char *)ws + head, ws_bytes - head, stream);
     if (st != GNN_OK) return st;
-    return launch_gemm(A, lda, W, ldw, Y, ldy, p->n, f_in, f_out, nullptr, nullptr, relu, s);
+    return launch_gemm(A, lda, W, ldw, Y, ldy, p->n, f_in, f_out, nullptr, nullptr, relu, ws, gws, s);
   })
 }
 

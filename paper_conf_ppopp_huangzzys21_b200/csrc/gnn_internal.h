@@ -108,7 +108,8 @@ gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, siz
 // GEMM (k_gemm.cu)
 gnn_status launch_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H,
                        int64_t ldh, int64_t m, int32_t k, int32_t n, const float *row_scale,
-                       const float *col_bias, int32_t relu, cudaStream_t s);
+                       const float *col_bias, int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s);
+size_t gemm_tc_workspace(int64_t m, int32_t k, int32_t n);
 int set_gemm_impl(int impl);
 
 // small helper kernels (k_graph.cu)

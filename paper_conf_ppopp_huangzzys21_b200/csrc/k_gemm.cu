@@ -124,21 +124,24 @@ int set_gemm_impl(int impl) {
 // is outside what the tcgen05 kernel takes
 cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H,
                            int64_t ldh, int64_t m, int32_t k, int32_t n, const float *row_scale,
-                           const float *col_bias, int32_t relu, cudaStream_t s);
+                           const float *col_bias, int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s);
 
 gnn_status launch_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H,
                        int64_t ldh, int64_t m, int32_t k, int32_t n, const float *row_scale,
-                       const float *col_bias, int32_t relu, cudaStream_t s) {
+                       const float *col_bias, int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s) {
   if (m == 0 || n == 0) return GNN_OK;
-  if (g_gemm_impl != 1) {
-    cudaError_t e = launch_gemm_tc(X, ldx, W, ldw, H, ldh, m, k, n, row_scale, col_bias, relu, s);
+  if (g_gemm_impl != 1 && ws != nullptr) {
+    cudaError_t e = launch_gemm_tc(X, ldx, W, ldw, H, ldh, m, k, n, row_scale, col_bias, relu, ws, ws_bytes, s);
     if (e == cudaSuccess) return GNN_OK;
     if (e != cudaErrorNotSupported) return cuda_status(e, "gemm tcgen05 launch");
     if (g_gemm_impl == 2) {
-      set_error("tcgen05 GEMM does not support this shape/alignment");
+      set_error("tcgen05 GEMM does not support this shape/alignment/workspace");
       return GNN_ERR_UNSUPPORTED;
     }
     (void)cudaGetLastError();
+  } else if (g_gemm_impl == 2) {
+    set_error("tcgen05 GEMM needs a workspace (gnn_gemm_workspace_size)");
+    return GNN_ERR_UNSUPPORTED;
   }
   dim3 grid((n + BN - 1) / BN, (unsigned)((m + BM - 1) / BM));
   if (grid.y > 65535u) {

@@ -1,18 +1,28 @@
 // k_gemm_tc.cu — a5: H = X W on the 5th-generation tensor cores (tcgen05,
-// kind::tf32, accumulator in TMEM) with a 3xTF32 split so the result has fp32
-// accuracy (plain TF32 fails the 1e-4 bar):
-//     X = Xhi + Xlo, W = Whi + Wlo  (hi = fp32 with the low 13 mantissa bits
-//     cleared — exactly representable in TF32; lo = x - hi, exact in fp32)
-//     H = Xhi Whi + Xhi Wlo + Xlo Whi      (Xlo Wlo ~ 2^-22 relative, dropped)
+// kind::tf32, accumulators in TMEM) with a 3xTF32 split so the result keeps
+// fp32 accuracy (plain TF32 fails the 1e-4 bar):
+//     X = Xhi + Xlo, W = Whi + Wlo  (hi = fp32 with the 13 low mantissa bits
+//     cleared, exactly representable in TF32; lo = x - hi, exact in fp32)
+//     H = Xlo Whi + Xhi Wlo + Xhi Whi      (Xlo Wlo ~ 2^-22 relative: dropped)
 // Epilogue fused: row scale (GCN nsrc[u]), column bias, ReLU.
 //
-// CTA = 128 rows x N (N <= 512; one MMA per 256 columns).  Warps 0-3 load
-// X/W tiles from global memory, split them into hi/lo and write them to
-// shared memory in the UMMA K-major SWIZZLE_128B layout (32 fp32 of K per
-// 128-byte row), then signal an mbarrier; warp 4 (one elected lane) issues
-// tcgen05.mma and releases stages with tcgen05.commit; warps 0-3 finally
-// read the accumulator with tcgen05.ld (32x32b: one TMEM lane = one row per
-// thread) and store it.
+// Structure (persistent, one CTA per SM, 288 threads):
+//   warps 0-3  producers: per 32-wide K block, load the 128 x 32 X tile from
+//              global memory, split it into hi/lo and store both in the UMMA
+//              K-major SWIZZLE_128B layout; thread 0 also issues one bulk
+//              async copy (cp.async.bulk, the TMA engine) of the pre-split,
+//              pre-swizzled W image for that K block (built once per call by
+//              k_gemm_wimage into the caller's workspace).
+//   warp 4     MMA issuer: one elected lane issues 3 tcgen05.mma per 8-wide K
+//              step per 256-column slice, commits stage release / tile done.
+//   warps 5-8  epilogue: tcgen05.ld (32x32b: one TMEM lane = one row per
+//              thread), fp32 sum of the partial accumulators, scale/bias/ReLU,
+//              store.  Runs concurrently with the next tile's MMAs when TMEM
+//              holds two tile buffers.
+// Accumulation drift: the tensor core's internal accumulation is not IEEE
+// round-to-nearest, so long K chains drift; K blocks are spread round-robin
+// over n_acc partial accumulators (summed in fp32 in the epilogue) so that no
+// accumulator sees more than ~8 K blocks (<= 96 MMA accumulations).
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -22,14 +32,15 @@ namespace gnn {
 namespace tc {
 
 constexpr int BM = 128;
-constexpr int BK = 32;           // fp32 elements per 128-byte swizzle row
-constexpr int NUM_LOAD_WARPS = 4;
-constexpr int THREADS = 32 * (NUM_LOAD_WARPS + 1);
-constexpr int TILE_A_BYTES = BM * BK * 4;  // 16 KB
+constexpr int BK = 32;  // fp32 elements per 128-byte swizzle row
+constexpr int NUM_PRODUCER_WARPS = 4;
+constexpr int MMA_WARP = 4;
+constexpr int EPI_WARP0 = 5;
+constexpr int THREADS = 32 * 9;
+constexpr int TILE_A_BYTES = BM * BK * 4;  // 16 KB per hi or lo
+constexpr int MAX_STAGES = 6;
 
-__device__ __forceinline__ uint32_t smem_u32(const void *p) {
-  return (uint32_t)__cvta_generic_to_shared(p);
-}
+__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
 __device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
@@ -37,31 +48,40 @@ __device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
 __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
 __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
-  const uint32_t addr = smem_u32(bar);
   asm volatile(
       "{\n\t"
       ".reg .pred P1;\n\t"
       "WAIT_%=:\n\t"
       "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
       "@!P1 bra WAIT_%=;\n\t"
-      "}\n" ::"r"(addr),
+      "}\n" ::"r"(smem_u32(bar)),
       "r"(parity)
       : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
 }
 
 // UMMA shared-memory descriptor: K-major, SWIZZLE_128B, 8-row atoms of 1024 B
 __device__ __forceinline__ uint64_t sw128_desc(uint32_t saddr) {
   uint64_t d = 0;
-  d |= (uint64_t)((saddr & 0x3FFFF) >> 4);  // start address (>>4), bits 0-13
-  d |= (uint64_t)1 << 16;                   // leading byte offset (unused for swizzled K-major)
+  d |= (uint64_t)((saddr & 0x3FFFF) >> 4);  // start address >> 4 (bits 0-13)
+  d |= (uint64_t)1 << 16;                   // leading byte offset (unused: swizzled K-major)
   d |= (uint64_t)(1024 >> 4) << 32;         // stride byte offset: 8 rows x 128 B
   d |= (uint64_t)1 << 46;                   // descriptor version (sm_100)
-  d |= (uint64_t)2 << 61;                   // layout: SWIZZLE_128B
+  d |= (uint64_t)2 << 61;                   // SWIZZLE_128B
   return d;
 }
 
-// instruction descriptor: D f32, A/B tf32, K-major both, M = 128, N
+// instruction descriptor: D f32, A/B tf32, both K-major, M = 128, N = n
 __host__ __device__ constexpr uint32_t idesc_tf32(int n) {
   return (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
 }
@@ -76,76 +96,83 @@ __device__ __forceinline__ void mma_tf32(uint32_t tmem_d, uint64_t da, uint64_t 
       "}\n" ::"r"(tmem_d),
       "l"(da), "l"(db), "r"(idesc), "r"(accumulate));
 }
-
 __device__ __forceinline__ void mma_commit(uint64_t *bar) {
-  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
-                   smem_u32(bar))
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
                : "memory");
 }
 
-// split x into (hi, lo): hi = x with 13 low mantissa bits cleared (TF32-exact), lo = x - hi (exact)
-__device__ __forceinline__ void split4(const float4 &x, float4 &hi, float4 &lo) {
-  hi.x = __uint_as_float(__float_as_uint(x.x) & 0xFFFFE000u);
-  hi.y = __uint_as_float(__float_as_uint(x.y) & 0xFFFFE000u);
-  hi.z = __uint_as_float(__float_as_uint(x.z) & 0xFFFFE000u);
-  hi.w = __uint_as_float(__float_as_uint(x.w) & 0xFFFFE000u);
-  lo.x = x.x - hi.x;
-  lo.y = x.y - hi.y;
-  lo.z = x.z - hi.z;
-  lo.w = x.w - hi.w;
-}
+__device__ __forceinline__ float hi_of(float x) { return __uint_as_float(__float_as_uint(x) & 0xFFFFE000u); }
 
 // byte offset of 16-byte chunk c (0..7) of row r inside a SW128 K-major tile
-__device__ __forceinline__ uint32_t sw128_off(int r, int c) {
+__host__ __device__ __forceinline__ uint32_t sw128_off(int r, int c) {
   return (uint32_t)((r >> 3) * 1024 + (r & 7) * 128 + ((c ^ (r & 7)) << 4));
+}
+
+// W image: for each K block kb: [hi tile | lo tile], each NP rows (n) x 128 B,
+// K-major, swizzled exactly as in shared memory.
+__global__ void k_gemm_wimage(const float *__restrict__ W, int64_t ldw, int32_t k, int32_t n, int32_t np,
+                              int32_t num_kb, uint8_t *img) {
+  const int64_t total = (int64_t)num_kb * np * 8;
+  for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < total; q += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t kb = (int32_t)(q / (np * 8));
+    const int32_t rem = (int32_t)(q % (np * 8));
+    const int32_t nn = rem >> 3, c = rem & 7;
+    const int32_t gk = kb * BK + 4 * c;
+    float w[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) w[i] = (nn < n && gk + i < k) ? W[(int64_t)(gk + i) * ldw + nn] : 0.0f;
+    float4 hi = make_float4(hi_of(w[0]), hi_of(w[1]), hi_of(w[2]), hi_of(w[3]));
+    float4 lo = make_float4(w[0] - hi.x, w[1] - hi.y, w[2] - hi.z, w[3] - hi.w);
+    uint8_t *base = img + (size_t)kb * 2 * np * 128;
+    const uint32_t off = sw128_off(nn, c);
+    *reinterpret_cast<float4 *>(base + off) = hi;
+    *reinterpret_cast<float4 *>(base + (size_t)np * 128 + off) = lo;
+  }
 }
 
 struct TcParams {
   const float *X;
   int64_t ldx;
-  const float *W;
-  int64_t ldw;
   float *H;
   int64_t ldh;
+  const uint8_t *wimg;
   int64_t m;
-  int32_t k, n, np;  // np = n rounded up to 16
+  int32_t k, n, np, npa;  // np = n rounded to 16; npa = TMEM columns per accumulator
+  int32_t num_kb, num_tiles;
+  int32_t stages, n_acc, n_buf;
   const float *row_scale;
   const float *col_bias;
   int32_t relu;
-  int32_t stages;
-  int32_t tmem_cols;
 };
 
 template <bool VEC_X, bool VEC_H>
 __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
-  // carve: [stage][A_hi | A_lo | B_hi | B_lo], 1024-aligned
   uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   const int NP = p.np;
   const int B_BYTES = NP * 128;
   const int STAGE_BYTES = 2 * TILE_A_BYTES + 2 * B_BYTES;
-  __shared__ uint64_t full_bar[4], empty_bar[4], accum_bar;
+  __shared__ uint64_t full_bar[MAX_STAGES], empty_bar[MAX_STAGES], tfull_bar[2], tempty_bar[2];
   __shared__ uint32_t tmem_base_sh;
 
   const int tid = threadIdx.x;
   const int warp = tid >> 5;
   const int lane = tid & 31;
-  const int64_t m0 = (int64_t)blockIdx.x * BM;
-  const int num_kb = (p.k + BK - 1) / BK;
   const int S = p.stages;
 
   if (tid == 0) {
     for (int s = 0; s < S; ++s) {
-      mbar_init(&full_bar[s], NUM_LOAD_WARPS * 32);
+      mbar_init(&full_bar[s], NUM_PRODUCER_WARPS * 32 + 1);  // 128 A arrivals + 1 expect_tx for W
       mbar_init(&empty_bar[s], 1);
     }
-    mbar_init(&accum_bar, 1);
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&tfull_bar[b], 1);
+      mbar_init(&tempty_bar[b], 128);
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (warp == 0) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
-                     smem_u32(&tmem_base_sh)),
-                 "r"(p.tmem_cols));
+  if (warp == MMA_WARP) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_u32(&tmem_base_sh)));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
   asm volatile("tcgen05.fence::before_thread_sync;");
@@ -153,163 +180,232 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p) {
   asm volatile("tcgen05.fence::after_thread_sync;");
   const uint32_t tmem = tmem_base_sh;
 
-  if (warp < NUM_LOAD_WARPS) {
-    // ---------------- producers: global -> split -> swizzled smem ----------------
-    for (int kb = 0; kb < num_kb; ++kb) {
-      const int s = kb % S, use = kb / S;
-      if (use > 0) mbar_wait(&empty_bar[s], (use - 1) & 1);
-      uint8_t *st = smem + (size_t)s * STAGE_BYTES;
-      uint8_t *a_hi = st, *a_lo = st + TILE_A_BYTES, *b_hi = st + 2 * TILE_A_BYTES, *b_lo = b_hi + B_BYTES;
-      const int k0 = kb * BK;
-      // A: 128 rows x 8 chunks of 4 fp32
-#pragma unroll 2
-      for (int q = tid; q < BM * 8; q += NUM_LOAD_WARPS * 32) {
-        const int r = q >> 3, c = q & 7;
-        const int64_t gm = m0 + r;
-        const int gk = k0 + 4 * c;
-        float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (gm < p.m) {
-          const float *src = p.X + gm * p.ldx + gk;
-          if (VEC_X && gk + 3 < p.k) {
-            x = __ldg(reinterpret_cast<const float4 *>(src));
-          } else {
-            if (gk + 0 < p.k) x.x = __ldg(src + 0);
-            if (gk + 1 < p.k) x.y = __ldg(src + 1);
-            if (gk + 2 < p.k) x.z = __ldg(src + 2);
-            if (gk + 3 < p.k) x.w = __ldg(src + 3);
+  if (warp < NUM_PRODUCER_WARPS) {
+    // ------------------------------ producers ------------------------------
+    int it = 0;  // global K-block counter across tiles (stage/phase tracking)
+    for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
+      const int64_t m0 = (int64_t)tile * BM;
+      for (int kb = 0; kb < p.num_kb; ++kb, ++it) {
+        const int s = it % S, use = it / S;
+        if (use > 0) mbar_wait(&empty_bar[s], (use - 1) & 1);
+        uint8_t *st = smem + (size_t)s * STAGE_BYTES;
+        uint8_t *a_hi = st, *a_lo = st + TILE_A_BYTES, *b_img = st + 2 * TILE_A_BYTES;
+        if (tid == 0) {
+          mbar_arrive_expect_tx(&full_bar[s], 2 * B_BYTES);
+          const uint8_t *src = p.wimg + (size_t)kb * 2 * B_BYTES;
+          for (int off = 0; off < 2 * B_BYTES; off += 16384) {
+            const int bytes = 2 * B_BYTES - off < 16384 ? 2 * B_BYTES - off : 16384;
+            bulk_g2s(b_img + off, src + off, bytes, &full_bar[s]);
           }
         }
-        float4 hi, lo;
-        split4(x, hi, lo);
-        const uint32_t off = sw128_off(r, c);
-        *reinterpret_cast<float4 *>(a_hi + off) = hi;
-        *reinterpret_cast<float4 *>(a_lo + off) = lo;
-      }
-      // B (K-major W^T tile): NP rows (n) x 8 chunks of 4 k; W is [k, n] row-major
-      for (int q = tid; q < NP * 8; q += NUM_LOAD_WARPS * 32) {
-        const int c = q / NP, nn = q % NP;  // consecutive threads -> consecutive n (coalesced)
-        const int gk = k0 + 4 * c;
-        float4 w = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (nn < p.n) {
-          const float *src = p.W + (int64_t)gk * p.ldw + nn;
-          if (gk + 0 < p.k) w.x = __ldg(src);
-          if (gk + 1 < p.k) w.y = __ldg(src + p.ldw);
-          if (gk + 2 < p.k) w.z = __ldg(src + 2 * p.ldw);
-          if (gk + 3 < p.k) w.w = __ldg(src + 3 * p.ldw);
+        const int k0 = kb * BK;
+#pragma unroll 4
+        for (int q = tid; q < BM * 8; q += NUM_PRODUCER_WARPS * 32) {
+          const int r = q >> 3, c = q & 7;
+          const int64_t gm = m0 + r;
+          const int gk = k0 + 4 * c;
+          float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
+          if (gm < p.m) {
+            const float *src = p.X + gm * p.ldx + gk;
+            if (VEC_X && gk + 3 < p.k) {
+              x = __ldg(reinterpret_cast<const float4 *>(src));
+            } else {
+              if (gk + 0 < p.k) x.x = __ldg(src + 0);
+              if (gk + 1 < p.k) x.y = __ldg(src + 1);
+              if (gk + 2 < p.k) x.z = __ldg(src + 2);
+              if (gk + 3 < p.k) x.w = __ldg(src + 3);
+            }
+          }
+          const float4 hi = make_float4(hi_of(x.x), hi_of(x.y), hi_of(x.z), hi_of(x.w));
+          const float4 lo = make_float4(x.x - hi.x, x.y - hi.y, x.z - hi.z, x.w - hi.w);
+          const uint32_t off = sw128_off(r, c);
+          *reinterpret_cast<float4 *>(a_hi + off) = hi;
+          *reinterpret_cast<float4 *>(a_lo + off) = lo;
         }
-        float4 hi, lo;
-        split4(w, hi, lo);
-        const uint32_t off = sw128_off(nn, c);
-        *reinterpret_cast<float4 *>(b_hi + off) = hi;
-        *reinterpret_cast<float4 *>(b_lo + off) = lo;
+        // generic-proxy smem writes -> visible to the tensor core (async proxy)
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        mbar_arrive(&full_bar[s]);
       }
-      // make generic-proxy smem writes visible to the tensor core (async proxy)
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-      mbar_arrive(&full_bar[s]);
     }
-    // ---------------- epilogue: TMEM -> registers -> global ----------------
-    mbar_wait(&accum_bar, 0);
-    asm volatile("tcgen05.fence::after_thread_sync;");
-    const int r = warp * 32 + lane;
-    const int64_t gm = m0 + r;
-    const float sc = (p.row_scale && gm < p.m) ? __ldg(p.row_scale + gm) : 1.0f;
-    for (int c0 = 0; c0 < NP; c0 += 32) {
-      uint32_t v[32];
-      const uint32_t taddr = tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)c0;
-      asm volatile(
-          "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
-          "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
-          : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]),
-            "=r"(v[7]), "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]),
-            "=r"(v[14]), "=r"(v[15]), "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]),
-            "=r"(v[21]), "=r"(v[22]), "=r"(v[23]), "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]),
-            "=r"(v[28]), "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
-          : "r"(taddr));
-      asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-      if (gm >= p.m) continue;
-      float y[32];
+  } else if (warp == MMA_WARP) {
+    // ------------------------------ MMA issuer ------------------------------
+    int it = 0, tcount = 0;
+    for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++tcount) {
+      const int b = tcount % p.n_buf, buse = tcount / p.n_buf;
+      if (buse > 0) mbar_wait(&tempty_bar[b], (buse - 1) & 1);
+      asm volatile("tcgen05.fence::after_thread_sync;");
+      const uint32_t tbase = tmem + (uint32_t)(b * p.n_acc * p.npa);
+      for (int kb = 0; kb < p.num_kb; ++kb, ++it) {
+        const int s = it % S, use = it / S;
+        mbar_wait(&full_bar[s], use & 1);
+        asm volatile("tcgen05.fence::after_thread_sync;");
+        if (lane == 0) {
+          const uint32_t st = smem_u32(smem + (size_t)s * STAGE_BYTES);
+          const uint32_t a_hi = st, a_lo = st + TILE_A_BYTES, b_hi = st + 2 * TILE_A_BYTES, b_lo = b_hi + B_BYTES;
+          const int acc = kb % p.n_acc;
+          const uint32_t d0 = tbase + (uint32_t)(acc * p.npa);
+          const uint32_t first = (kb < p.n_acc) ? 1u : 0u;  // first K block of this accumulator
 #pragma unroll
-      for (int i = 0; i < 32; ++i) {
-        const int col = c0 + i;
-        float t = __uint_as_float(v[i]);
-        if (p.row_scale) t = t * sc;
-        if (p.col_bias && col < p.n) t = t + __ldg(p.col_bias + col);
-        if (p.relu) t = t > 0.0f ? t : 0.0f;
-        y[i] = t;
-      }
-      float *dst = p.H + gm * p.ldh + c0;
-      if (VEC_H && c0 + 32 <= p.n) {
-#pragma unroll
-        for (int i = 0; i < 32; i += 4)
-          *reinterpret_cast<float4 *>(dst + i) = make_float4(y[i], y[i + 1], y[i + 2], y[i + 3]);
-      } else {
-#pragma unroll
-        for (int i = 0; i < 32; ++i)
-          if (c0 + i < p.n) dst[i] = y[i];
+          for (int j = 0; j < BK / 8; ++j) {  // 8 tf32 (32 B) per MMA K step
+            const uint32_t ko = j * 32;
+            for (int n0 = 0; n0 < NP; n0 += 256) {
+              const int nn = NP - n0 < 256 ? NP - n0 : 256;
+              const uint32_t id = idesc_tf32(nn);
+              const uint32_t bo = (uint32_t)n0 * 128;
+              const uint32_t d = d0 + (uint32_t)n0;
+              mma_tf32(d, sw128_desc(a_lo + ko), sw128_desc(b_hi + bo + ko), id, (first && j == 0) ? 0u : 1u);
+              mma_tf32(d, sw128_desc(a_hi + ko), sw128_desc(b_lo + bo + ko), id, 1u);
+              mma_tf32(d, sw128_desc(a_hi + ko), sw128_desc(b_hi + bo + ko), id, 1u);
+            }
+          }
+          mma_commit(&empty_bar[s]);
+          if (kb == p.num_kb - 1) mma_commit(&tfull_bar[b]);
+        }
+        __syncwarp();
       }
     }
   } else {
-    // ---------------- MMA issuer: warp 4, one elected lane ----------------
-    for (int kb = 0; kb < num_kb; ++kb) {
-      const int s = kb % S, use = kb / S;
-      mbar_wait(&full_bar[s], use & 1);
+    // ------------------------------ epilogue ------------------------------
+    const int ew = warp - EPI_WARP0;  // 0..3 -> TMEM lanes 32*ew (warp % 4 == ew + 1 ... see note)
+    // TMEM lane quadrant accessible by a warp is (warp id % 4): warps 5,6,7,8 -> 1,2,3,0
+    const int quad = warp & 3;
+    (void)ew;
+    int tcount = 0;
+    for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++tcount) {
+      const int b = tcount % p.n_buf, buse = tcount / p.n_buf;
+      mbar_wait(&tfull_bar[b], buse & 1);
       asm volatile("tcgen05.fence::after_thread_sync;");
-      if (lane == 0) {
-        const uint32_t st = smem_u32(smem + (size_t)s * STAGE_BYTES);
-        const uint32_t a_hi = st, a_lo = st + TILE_A_BYTES, b_hi = st + 2 * TILE_A_BYTES, b_lo = b_hi + B_BYTES;
+      const int r = quad * 32 + lane;
+      const int64_t gm = (int64_t)tile * BM + r;
+      const float sc = (p.row_scale && gm < p.m) ? __ldg(p.row_scale + gm) : 1.0f;
+      const uint32_t tbase = tmem + (uint32_t)(b * p.n_acc * p.npa) + ((uint32_t)(quad * 32) << 16);
+      const int n_acc_used = p.num_kb < p.n_acc ? p.num_kb : p.n_acc;
+      for (int c0 = 0; c0 < NP; c0 += 32) {
+        float y[32];
 #pragma unroll
-        for (int j = 0; j < BK / 8; ++j) {  // 8 tf32 (32 B) per MMA K step
-          const uint32_t ko = j * 32;
-          for (int n0 = 0; n0 < NP; n0 += 256) {
-            const int nn = NP - n0 < 256 ? NP - n0 : 256;
-            const uint32_t id = idesc_tf32(nn);
-            const uint32_t bo = (uint32_t)n0 * 128;  // row n0 of the B tile
-            const uint32_t d = tmem + (uint32_t)n0;
-            const uint32_t acc0 = (kb > 0 || j > 0) ? 1u : 0u;
-            mma_tf32(d, sw128_desc(a_lo + ko), sw128_desc(b_hi + bo + ko), id, acc0);
-            mma_tf32(d, sw128_desc(a_hi + ko), sw128_desc(b_lo + bo + ko), id, 1u);
-            mma_tf32(d, sw128_desc(a_hi + ko), sw128_desc(b_hi + bo + ko), id, 1u);
-          }
+        for (int i = 0; i < 32; ++i) y[i] = 0.0f;
+        for (int a = 0; a < n_acc_used; ++a) {
+          uint32_t v[32];
+          const uint32_t taddr = tbase + (uint32_t)(a * p.npa + c0);
+          asm volatile(
+              "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+              "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+              : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+                "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
+                "=r"(v[15]), "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]),
+                "=r"(v[22]), "=r"(v[23]), "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]),
+                "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
+              : "r"(taddr));
+          asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+          for (int i = 0; i < 32; ++i) y[i] = (a == 0) ? __uint_as_float(v[i]) : y[i] + __uint_as_float(v[i]);
         }
-        mma_commit(&empty_bar[s]);
-        if (kb == num_kb - 1) mma_commit(&accum_bar);
+        if (gm >= p.m) continue;
+#pragma unroll
+        for (int i = 0; i < 32; ++i) {
+          const int col = c0 + i;
+          float t = y[i];
+          if (p.row_scale) t = t * sc;
+          if (p.col_bias && col < p.n) t = t + __ldg(p.col_bias + col);
+          if (p.relu) t = t > 0.0f ? t : 0.0f;
+          y[i] = t;
+        }
+        float *dst = p.H + gm * p.ldh + c0;
+        if (VEC_H && c0 + 32 <= p.n) {
+#pragma unroll
+          for (int i = 0; i < 32; i += 4) *reinterpret_cast<float4 *>(dst + i) = make_float4(y[i], y[i + 1], y[i + 2], y[i + 3]);
+        } else {
+#pragma unroll
+          for (int i = 0; i < 32; ++i)
+            if (c0 + i < p.n) dst[i] = y[i];
+        }
       }
-      __syncwarp();
+      asm volatile("tcgen05.fence::before_thread_sync;");
+      mbar_arrive(&tempty_bar[b]);
     }
   }
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
-  if (warp == 0) {
+  if (warp == MMA_WARP) {
     asm volatile("tcgen05.fence::after_thread_sync;");
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(p.tmem_cols));
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem));
   }
+}
+
+struct Config {
+  int np, npa, num_kb, stages, n_acc, n_buf;
+  size_t smem, wimg_bytes;
+};
+
+static bool configure(int64_t m, int32_t k, int32_t n, Config &c) {
+  if (n < 1 || n > 512 || k < 1 || m < 1) return false;
+  c.np = (n + 15) / 16 * 16;
+  c.npa = 32;
+  while (c.npa < c.np) c.npa *= 2;
+  c.num_kb = (k + BK - 1) / BK;
+  c.wimg_bytes = (size_t)c.num_kb * 2 * c.np * 128;
+  const int stage_bytes = 2 * TILE_A_BYTES + 2 * c.np * 128;
+  c.stages = 6;
+  while (c.stages > 2 && (size_t)c.stages * stage_bytes + 2048 > 200 * 1024) --c.stages;
+  c.smem = (size_t)c.stages * stage_bytes + 1024;
+  if (c.smem > 227 * 1024) return false;
+  // TMEM: n_buf tile buffers x n_acc accumulators x npa columns <= 512
+  const int slots = 512 / c.npa;  // accumulators that fit
+  if (slots < 1) return false;
+  if (c.num_kb <= 8 && slots >= 2) {
+    c.n_buf = 2;  // overlap the epilogue with the next tile
+    c.n_acc = slots / 2;
+  } else {
+    c.n_buf = 1;
+    c.n_acc = slots;
+  }
+  const int need_acc = (c.num_kb + 7) / 8;  // keep <= 8 K blocks per accumulator when possible
+  if (c.n_acc > need_acc) c.n_acc = need_acc;
+  if (c.n_acc < 1) c.n_acc = 1;
+  return true;
 }
 
 }  // namespace tc
 
+size_t gemm_tc_workspace(int64_t m, int32_t k, int32_t n) {
+  tc::Config c;
+  if (!tc::configure(m > 0 ? m : 1, k, n, c)) return 0;
+  return (c.wimg_bytes + 255) & ~(size_t)255;
+}
+
 cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H, int64_t ldh,
                            int64_t m, int32_t k, int32_t n, const float *row_scale, const float *col_bias,
-                           int32_t relu, cudaStream_t s) {
+                           int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s) {
   using namespace tc;
-  if (n < 1 || n > 512 || k < 1 || m < 1) return cudaErrorNotSupported;
-  const int np = (n + 15) / 16 * 16;
-  const int stage_bytes = 2 * TILE_A_BYTES + 2 * np * 128;
-  int stages = 4;
-  while (stages > 2 && stages * stage_bytes > 160 * 1024) --stages;
-  const size_t smem = (size_t)stages * stage_bytes + 1024;
-  if (smem > 227 * 1024) return cudaErrorNotSupported;
-  int cols = 32;
-  while (cols < np) cols *= 2;
-  TcParams p{X, ldx, W, ldw, H, ldh, m, k, n, np, row_scale, col_bias, relu, stages, cols};
+  Config c;
+  if (!configure(m, k, n, c)) return cudaErrorNotSupported;
+  if (!ws || ws_bytes < c.wimg_bytes || ((uintptr_t)ws & 15)) return cudaErrorNotSupported;
+  static int num_sms = 0;
+  if (num_sms == 0) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&num_sms, cudaDevAttrMultiProcessorCount, dev);
+    if (num_sms <= 0) num_sms = 148;
+  }
+  uint8_t *img = (uint8_t *)ws;
+  {
+    const int64_t total = (int64_t)c.num_kb * c.np * 8;
+    const int blocks = (int)((total + 255) / 256 < 4096 ? (total + 255) / 256 : 4096);
+    k_gemm_wimage<<<blocks, 256, 0, s>>>(W, ldw, k, n, c.np, c.num_kb, img);
+    count_launch();
+  }
+  const int64_t num_tiles = (m + BM - 1) / BM;
+  if (num_tiles > 0x7fffffff) return cudaErrorNotSupported;
+  TcParams p{X, ldx, H, ldh, img, m, k, n, c.np, c.npa, c.num_kb, (int32_t)num_tiles, c.stages, c.n_acc, c.n_buf,
+             row_scale, col_bias, relu};
   const bool vx = (ldx % 4 == 0) && ((uintptr_t)X % 16 == 0);
   const bool vh = (ldh % 4 == 0) && ((uintptr_t)H % 16 == 0);
   auto fn = vx ? (vh ? k_gemm_tc<true, true> : k_gemm_tc<true, false>)
                : (vh ? k_gemm_tc<false, true> : k_gemm_tc<false, false>);
-  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c.smem);
   if (e != cudaSuccess) return e;
-  const int64_t grid = (m + BM - 1) / BM;
-  if (grid > 0x7fffffff) return cudaErrorNotSupported;
-  fn<<<(unsigned)grid, THREADS, smem, s>>>(p);
+  const int grid = (int)(num_tiles < num_sms ? num_tiles : num_sms);
+  fn<<<grid, THREADS, c.smem, s>>>(p);
   count_launch();
   return cudaGetLastError();
 }

@@ -77,7 +77,8 @@ _SIGS = {
     "gnn_gat_layer": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _P, _P, _I32, _I32, _F, _P, _I64, _P, _SZ, _P]),
     "gnn_edgeconv_aggregate": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _I64, _P, _SZ, _P]),
     "gnn_edgeconv": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _P, _P, _I32, _P, _I64, _P, _SZ, _P]),
-    "gnn_gemm": (ctypes.c_int, [_P, _I64, _P, _I64, _P, _I64, _I64, _I32, _I32, _P, _P, _I32, _P]),
+    "gnn_gemm": (ctypes.c_int, [_P, _I64, _P, _I64, _P, _I64, _I64, _I32, _I32, _P, _P, _I32, _P, _SZ, _P]),
+    "gnn_gemm_workspace_size": (_SZ, [_I64, _I32, _I32]),
     "gnn_set_gemm_impl": (ctypes.c_int, [ctypes.c_int]),
     "gnn_gcn_layer": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _I64, _I32, _I32, _I32, _P, _I64, _P, _SZ, _P]),
     "gnn_gcn_aggregate_prescaled": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _I64, _I32, _P, _SZ, _P]),
@@ -277,13 +278,31 @@ def edgeconv(plan: Plan, X, theta, phi, bias=None, out=None, stream=None):
     return Y
 
 
-def gemm(X, W, row_scale=None, col_bias=None, relu=False, out=None, stream=None):
+_GEMM_WS = {}
+
+
+def gemm_workspace(m, k, n, device):
+    """Workspace for the tcgen05 path (the split, swizzled W image); cached per device/size."""
+    nbytes = _lib.gnn_gemm_workspace_size(m, k, n)
+    if nbytes == 0:
+        return None, 0
+    torch = _torch()
+    key = (str(device), nbytes)
+    ws = _GEMM_WS.get(key)
+    if ws is None:
+        ws = torch.empty(nbytes, dtype=torch.uint8, device=device)
+        _GEMM_WS[key] = ws
+    return ws, nbytes
+
+
+def gemm(X, W, row_scale=None, col_bias=None, relu=False, out=None, stream=None, simt=False):
     torch = _torch()
     m, k = X.shape
     n = W.shape[1]
     H = out if out is not None else torch.empty((m, n), dtype=torch.float32, device=X.device)
+    ws, nb = (None, 0) if simt else gemm_workspace(m, k, n, X.device)
     _call("gnn_gemm", _tp(X), _ld(X, k), _tp(W), _ld(W, n), _tp(H), _ld(H, n), m, k, n, _tp(row_scale),
-          _tp(col_bias), int(relu), _stream(stream))
+          _tp(col_bias), int(relu), _tp(ws), nb, _stream(stream))
     return H
 
 

@@ -68,6 +68,10 @@ class RowPartitionedGCNGAT:
         self.ws_agg, self.ws_agg_b = self.plan.workspace(_g.GNN_OP_AGGREGATE, 0, max(self.F, self.F_in), 0, d)
         self.ws_gat, self.ws_gat_b = self.plan.workspace(_g.GNN_OP_GAT_AGGREGATE, 0, self.HF, heads, d)
         self.names = ["agg1", "gemm1", "gemm2+xchg", "agg2", "gemm3+xchg", "gat_agg"]
+        gw = max(_g._lib.gnn_gemm_workspace_size(R, self.F_in, self.F), _g._lib.gnn_gemm_workspace_size(R, self.F, self.F),
+                 _g._lib.gnn_gemm_workspace_size(R, self.F, self.ldwe))
+        self.ws_gemm = torch.empty(max(gw, 256), dtype=torch.uint8, device=d)
+        self.ws_gemm_b = gw
 
     # -- inputs -------------------------------------------------------------
     def load_input(self, X_host_or_dev, non_blocking=True):
@@ -107,11 +111,12 @@ class RowPartitionedGCNGAT:
         chk(lib.gnn_aggregate(self.plan.handle, _g.GNN_SUM, _g.GNN_W_GCN, None, P(self.Xs), Fi, Fi, P(self.A1), Fi,
                               0, None, 0, P(self.ws_agg), self.ws_agg_b, sp), "agg1")
         rec(1)
-        chk(lib.gnn_gemm(P(self.A1), Fi, P(self.W1), F, P(self.Y1), F, R, Fi, F, None, None, 1, sp), "gemm1")
+        gws = (P(self.ws_gemm), self.ws_gemm_b) if self.ws_gemm_b else (None, 0)
+        chk(lib.gnn_gemm(P(self.A1), Fi, P(self.W1), F, P(self.Y1), F, R, Fi, F, None, None, 1, *gws, sp), "gemm1")
         rec(2)
         h_loc = self.Hs2[off:off + R]
         chk(lib.gnn_gemm(P(self.Y1), F, P(self.W2), F, P(h_loc), F, R, F, F,
-                         ctypes.c_void_p(self.nsrc_ptr + 4 * off), None, 0, sp), "gemm2")
+                         ctypes.c_void_p(self.nsrc_ptr + 4 * off), None, 0, *gws, sp), "gemm2")
         self._allgather(self.Hs2)
         rec(3)
         chk(lib.gnn_gcn_aggregate_prescaled(self.plan.handle, P(self.Hs2), F, F, P(self.Y2), F, 0, P(self.ws_agg),
@@ -121,7 +126,7 @@ class RowPartitionedGCNGAT:
                                      sp), "gat fold")
         z_loc = self.Zst[off:off + R]
         chk(lib.gnn_gemm(P(self.Y2), F, P(self.Wext), self.ldwe, P(z_loc), self.ldwe, R, F, self.ldwe, None, None, 0,
-                         sp), "gemm3")
+                         *gws, sp), "gemm3")
         self._allgather(self.Zst)
         rec(5)
         tptr = ctypes.c_void_p(z_loc.data_ptr() + 4 * (HF + H))

@@ -42,9 +42,9 @@ def gemm():
         for impl, name in [(1, "simt"), (2, "tc")]:
             G.set_gemm_impl(impl)
             try:
-                H = G.gemm(X, W, row_scale=rs)
+                H = G.gemm(X, W, row_scale=rs, simt=(impl == 1))
                 torch.cuda.synchronize()
-                ms = timeit(lambda: G.gemm(X, W, row_scale=rs, out=H))
+                ms = timeit(lambda: G.gemm(X, W, row_scale=rs, out=H, simt=(impl == 1)))
                 res[name] = (ms, H.clone())
             except Exception as e:  # noqa: BLE001
                 res[name] = (None, repr(e))

@@ -79,7 +79,7 @@ def test_plan_create_rejects_invalid_csr(case):
 
 def test_invalid_args_return_status_not_crash():
     assert P.gnn.gnn_aggregate(None, 0, 0, None, None, 1, 1, None, 1, 0, None, 0, None, 0, None) == 1
-    assert P.gnn.gnn_gemm(None, 1, None, 1, None, 1, 4, 4, 4, None, None, 0, None) == 1
+    assert P.gnn.gnn_gemm(None, 1, None, 1, None, 1, 4, 4, 4, None, None, 0, None, 0, None) == 1
     assert P.gnn.gnn_plan_destroy(None) == 0
 
 
