@@ -19,15 +19,17 @@ struct DevGraph {
   const int32_t *colidx;       // [nnz]
   const float *nsrc;           // [n_src] 1/sqrtf(d_out)
   const float *ndst;           // [n]     1/sqrtf(d_in)
+  const int32_t *grp_beg;      // [G] first CSR entry of each group
   const int32_t *grp_row;      // [G]
-  const int32_t *grp_beg;      // [G]
-  const int32_t *tile_beg;     // [n_tiles+1]
-  const int32_t *tile_split;   // [n_tiles] split-row index or -1
+  const int32_t *whole_rows;   // [n_whole] whole-row tasks in task order
+  const int32_t *tile_lo;      // [n_tiles] split-row tile: group range [lo, hi)
+  const int32_t *tile_hi;      // [n_tiles]
+  const int32_t *tile_split;   // [n_tiles] split-row index
   const int32_t *split_off;    // [n_split] first workspace slot of the split row
   const int32_t *split_first;  // [n_split] global index of the row's first group
   const int32_t *split_ntiles; // [n_split]
   const int32_t *empty_rows;   // [n_empty]
-  int32_t n_tiles, n_split, n_empty, ng;
+  int32_t n_whole, n_tiles, n_split, n_empty, ng;
 };
 
 }  // namespace gnn
@@ -38,11 +40,13 @@ struct gnn_plan_s {
   gnn_plan_opts opts{};
   int32_t ng = 0;      // effective group bound (INT32_MAX-ish when "never split")
   int32_t T = 32;
+  int32_t R = 4;
   int32_t max_degree = 0;
   // host copies
   std::vector<int64_t> rowptr;
   std::vector<int32_t> perm, grp_row;
-  std::vector<int64_t> grp_beg, tile_beg;
+  std::vector<int64_t> grp_beg, tile_lo, tile_hi;
+  std::vector<int32_t> whole_rows;
   std::vector<uint64_t> sig;
   std::vector<int32_t> pairs, cluster_of;
   int64_t n_clusters = 0, n_split = 0, n_empty = 0, split_slots = 0;
@@ -61,9 +65,10 @@ void count_launch(uint64_t k = 1);
 
 // planner (plan.cpp) — host side
 gnn_status build_schedule(gnn_plan_s *p);
-void schedule_host(int64_t n, const int64_t *rowptr, const int32_t *perm, int64_t ng, int32_t T,
-                   std::vector<int32_t> &grp_row, std::vector<int64_t> &grp_beg,
-                   std::vector<int64_t> &tile_beg, std::vector<int32_t> &tile_split,
+void schedule_host(int64_t n, const int64_t *rowptr, const int32_t *perm, int64_t ng, int32_t R,
+                   int32_t T, std::vector<int32_t> &grp_row, std::vector<int64_t> &grp_beg,
+                   std::vector<int32_t> &whole_rows, std::vector<int64_t> &tile_lo,
+                   std::vector<int64_t> &tile_hi, std::vector<int32_t> &tile_split,
                    std::vector<int32_t> &split_off, std::vector<int32_t> &split_first,
                    std::vector<int32_t> &split_ntiles, int64_t &slots);
 int64_t las_lsh_pairs(int64_t n, const int64_t *rowptr, const uint64_t *sig, int32_t K, int32_t r,

@@ -176,6 +176,7 @@ struct KParams {
   int32_t FW;      // F (+ 2H for GAT)
   int32_t deterministic;
   int32_t T;
+  int32_t n_persist;  // blocks of the persistent whole-row phase
 };
 
 template <int VEC>
@@ -254,18 +255,35 @@ __device__ __forceinline__ void gat_merge(float &m1, float &l1, float *a1, float
   m1 = m;
 }
 
-// group partial over CSR entries [beg, end) of destination `row`.
-// Rolling register ring: U source rows stay in flight per worker (a row is
-// re-requested as soon as its slot is consumed); the next batch of LANES
-// indices is requested before the current batch is consumed.  Consumption
-// order is CSR order, so the fp32 chain is exactly R9's.
+// combine partial B into A (A = A (+) B) in fixed form
+template <int MODE, int VEC, int NV>
+__device__ __forceinline__ void part_combine(Part<MODE, VEC, NV> &A, const Part<MODE, VEC, NV> &B) {
+#pragma unroll
+  for (int n = 0; n < NV; ++n) {
+    if constexpr (MODE == M_GAT) {
+      gat_merge(A.m[n], A.l[n], A.a[n], B.m[n], B.l[n], B.a[n], VEC);
+    } else {
+#pragma unroll
+      for (int i = 0; i < VEC; ++i)
+        A.a[n][i] = (MODE == M_MAX) ? fmaxf(A.a[n][i], B.a[n][i]) : A.a[n][i] + B.a[n][i];
+    }
+  }
+}
+
+// Chain over CSR entries [beg, end) of destination `row`, neighbour groups
+// of ng entries starting at beg (R9): a fresh fp32 group partial G runs in CSR
+// order and is folded into the row accumulator A at every group boundary
+// (A = G for the first group, then A = A (+) G).  One rolling register ring
+// keeps U source rows in flight per worker across group boundaries; the next
+// batch of LANES indices is requested before the current batch is consumed.
 template <int MODE, int VEC, int NV, int LANES>
-__device__ __forceinline__ void group_partial(const KParams &p, int32_t beg, int32_t end, int32_t row,
-                                              int32_t c0, int lane, unsigned mask,
-                                              Part<MODE, VEC, NV> &P) {
+__device__ __forceinline__ void row_chain(const KParams &p, int32_t beg, int32_t end, int32_t row, int32_t c0,
+                                          int lane, unsigned mask, Part<MODE, VEC, NV> &A) {
   constexpr int FPL = VEC * NV;  // floats per lane per source row
   constexpr int U = FPL >= 32 ? 1 : (32 / FPL > 8 ? 8 : 32 / FPL);
-  part_init(P);
+  const int32_t ng = p.g.ng;
+  Part<MODE, VEC, NV> G;
+  part_init(G);
   bool valid[NV];
   int32_t head[NV];
   float tv[NV];
@@ -307,8 +325,9 @@ __device__ __forceinline__ void group_partial(const KParams &p, int32_t beg, int
   int32_t my_u;
   float my_w;
   load_idx(k, cnt, my_u, my_w);
+  int32_t next_fold = (end - beg > ng) ? beg + ng : end;  // absolute index ending the current group
+  bool first = true;
   for (;;) {
-    // next index batch in flight while this one is consumed
     const int32_t kn = k + LANES;
     const int32_t cnt_n = kn < end ? min(LANES, end - kn) : 0;
     int32_t nx_u;
@@ -328,14 +347,14 @@ __device__ __forceinline__ void group_partial(const KParams &p, int32_t beg, int
               if (!valid[n]) continue;
               float sco = sc[q][n] + tv[n];
               sco = sco > 0.0f ? sco : p.slope * sco;  // LeakyReLU (Table 2 GAT)
-              const float d = sco - P.m[n];
+              const float d = sco - G.m[n];
               const float ex = __expf(-fabsf(d));
               const bool up = d > 0.0f;
 #pragma unroll
               for (int i = 0; i < VEC; ++i)
-                P.a[n][i] = fmaf(up ? P.a[n][i] : v[q][n][i], ex, up ? v[q][n][i] : P.a[n][i]);
-              P.l[n] = fmaf(up ? P.l[n] : 1.0f, ex, up ? 1.0f : P.l[n]);
-              P.m[n] = up ? sco : P.m[n];
+                G.a[n][i] = fmaf(up ? G.a[n][i] : v[q][n][i], ex, up ? v[q][n][i] : G.a[n][i]);
+              G.l[n] = fmaf(up ? G.l[n] : 1.0f, ex, up ? 1.0f : G.l[n]);
+              G.m[n] = up ? sco : G.m[n];
             }
           } else {
             const float w = __shfl_sync(mask, my_w, e, LANES);
@@ -344,12 +363,22 @@ __device__ __forceinline__ void group_partial(const KParams &p, int32_t beg, int
               if (!valid[n]) continue;
 #pragma unroll
               for (int i = 0; i < VEC; ++i) {
-                if constexpr (MODE == M_MAX) P.a[n][i] = fmaxf(P.a[n][i], w * v[q][n][i]);
-                else P.a[n][i] = fmaf(w, v[q][n][i], P.a[n][i]);
+                if constexpr (MODE == M_MAX) G.a[n][i] = fmaxf(G.a[n][i], w * v[q][n][i]);
+                else G.a[n][i] = fmaf(w, v[q][n][i], G.a[n][i]);
               }
             }
           }
           if (e + U < cnt) load_row(q, __shfl_sync(mask, my_u, e + U, LANES));
+          if (k + e + 1 == next_fold) {  // group boundary: fold G into A, restart G
+            if (first) {
+              A = G;
+              first = false;
+            } else {
+              part_combine<MODE, VEC, NV>(A, G);
+            }
+            part_init(G);
+            next_fold = (end - next_fold > ng) ? next_fold + ng : end;
+          }
         }
       }
     }
@@ -358,21 +387,6 @@ __device__ __forceinline__ void group_partial(const KParams &p, int32_t beg, int
     cnt = cnt_n;
     my_u = nx_u;
     my_w = nx_w;
-  }
-}
-
-// combine partial B into A (A = A (+) B) in fixed form
-template <int MODE, int VEC, int NV>
-__device__ __forceinline__ void part_combine(Part<MODE, VEC, NV> &A, const Part<MODE, VEC, NV> &B) {
-#pragma unroll
-  for (int n = 0; n < NV; ++n) {
-    if constexpr (MODE == M_GAT) {
-      gat_merge(A.m[n], A.l[n], A.a[n], B.m[n], B.l[n], B.a[n], VEC);
-    } else {
-#pragma unroll
-      for (int i = 0; i < VEC; ++i)
-        A.a[n][i] = (MODE == M_MAX) ? fmaxf(A.a[n][i], B.a[n][i]) : A.a[n][i] + B.a[n][i];
-    }
   }
 }
 
@@ -410,51 +424,11 @@ __device__ __forceinline__ void store_row(const KParams &p, int32_t row, int32_t
   }
 }
 
-// shared-memory slot layout: [T][CW] accumulators, then [T][NV*LANES][2] (m, l)
-template <int MODE, int VEC, int NV, int LANES>
-__device__ __forceinline__ void slot_store(float *smem, int T, int j, int lane,
-                                           const Part<MODE, VEC, NV> &P) {
-  constexpr int CW = LANES * VEC * NV;
-  float *s = smem + (size_t)j * CW;
-#pragma unroll
-  for (int n = 0; n < NV; ++n)
-#pragma unroll
-    for (int i = 0; i < VEC; ++i) s[(n * LANES + lane) * VEC + i] = P.a[n][i];
-  if constexpr (MODE == M_GAT) {
-    float *ml = smem + (size_t)T * CW + ((size_t)j * NV * LANES) * 2;
-#pragma unroll
-    for (int n = 0; n < NV; ++n) {
-      ml[(n * LANES + lane) * 2] = P.m[n];
-      ml[(n * LANES + lane) * 2 + 1] = P.l[n];
-    }
-  }
-}
-
-template <int MODE, int VEC, int NV, int LANES>
-__device__ __forceinline__ void slot_load(const float *smem, int T, int j, int lane,
-                                          Part<MODE, VEC, NV> &P) {
-  constexpr int CW = LANES * VEC * NV;
-  const float *s = smem + (size_t)j * CW;
-#pragma unroll
-  for (int n = 0; n < NV; ++n)
-#pragma unroll
-    for (int i = 0; i < VEC; ++i) P.a[n][i] = s[(n * LANES + lane) * VEC + i];
-  if constexpr (MODE == M_GAT) {
-    const float *ml = smem + (size_t)T * CW + ((size_t)j * NV * LANES) * 2;
-#pragma unroll
-    for (int n = 0; n < NV; ++n) {
-      P.m[n] = ml[(n * LANES + lane) * 2];
-      P.l[n] = ml[(n * LANES + lane) * 2 + 1];
-    }
-  }
-}
-
 #ifndef GNN_AGG_MINB
 #define GNN_AGG_MINB 4
 #endif
 template <int MODE, int VEC, int NV, int LANES>
 __global__ void __launch_bounds__(256, MODE == M_GAT ? GNN_AGG_MINB - 1 : GNN_AGG_MINB) k_aggregate(const KParams p) {
-  extern __shared__ float smem[];
   constexpr int CW = LANES * VEC * NV;
   __shared__ int s_last;
   const int tid = threadIdx.x;
@@ -465,20 +439,40 @@ __global__ void __launch_bounds__(256, MODE == M_GAT ? GNN_AGG_MINB - 1 : GNN_AG
       LANES == 32 ? 0xffffffffu : (((1u << LANES) - 1u) << ((tid & 31) & ~(LANES - 1)));
   const DevGraph &g = p.g;
 
-  if ((int)blockIdx.x >= g.n_tiles) {
+  const int32_t nb_split = g.n_tiles;
+  if ((int32_t)blockIdx.x >= nb_split) {
+    const int32_t b = (int32_t)blockIdx.x - nb_split;
+    if (b < p.n_persist) {
+      // ---- whole-row tasks (<= R groups): statically interleaved over every
+      // worker of the persistent grid, so rows adjacent in the LAS task order
+      // are processed at the same time; one worker runs a row's
+      // groups in order and combines them in registers (R9)
+      const int64_t gw = (int64_t)b * nwk + wk, GW = (int64_t)p.n_persist * nwk;
+      for (int32_t c0 = 0; c0 < p.F; c0 += CW) {
+        for (int64_t i = gw; i < g.n_whole; i += GW) {
+          const int32_t row = g.whole_rows[i];
+          const int32_t rb = g.rowptr[row], re = g.rowptr[row + 1];
+          Part<MODE, VEC, NV> A;
+          row_chain<MODE, VEC, NV, LANES>(p, rb, re, row, c0, lane, mask, A);
+          store_row<MODE, VEC, NV, LANES>(p, row, re - rb, c0, lane, A);
+        }
+      }
+      return;
+    }
     // zero-fill rows without in-edges (R3-i): 32 rows per block
-    const int64_t r0 = (int64_t)(blockIdx.x - g.n_tiles) * 32;
+    const int64_t r0 = (int64_t)(b - p.n_persist) * 32;
     for (int64_t r = r0; r < r0 + 32 && r < g.n_empty; ++r) {
       float *y = p.Y + (int64_t)g.empty_rows[r] * p.ldy;
       for (int f = tid; f < p.F; f += blockDim.x) y[f] = 0.0f;
     }
     return;
   }
+  // ---- split-row tile: a row with more than R groups; groups spread over the
+  // CTA's workers, partials to the workspace, last-arriving CTA merges them
   const int32_t t = blockIdx.x;
-  const int32_t gb = g.tile_beg[t], ngr = g.tile_beg[t + 1] - gb;
+  const int32_t gb = g.tile_lo[t], ngr = g.tile_hi[t] - gb;
   const int32_t split = g.tile_split[t];
-
-  if (split >= 0) {
+  {
     // ---- a row spanning several tiles: partials -> workspace, last CTA merges
     const int32_t row = g.grp_row[gb];
     const int32_t rb = g.rowptr[row], re = g.rowptr[row + 1];
@@ -489,7 +483,7 @@ __global__ void __launch_bounds__(256, MODE == M_GAT ? GNN_AGG_MINB - 1 : GNN_AG
         const int32_t gi = gb + j;
         const int32_t beg = g.grp_beg[gi], end = (re - beg > g.ng) ? beg + g.ng : re;
         Part<MODE, VEC, NV> P;
-        group_partial<MODE, VEC, NV, LANES>(p, beg, end, row, c0, lane, mask, P);
+        row_chain<MODE, VEC, NV, LANES>(p, beg, end, row, c0, lane, mask, P);
         float *dst = part + (size_t)(gi - first) * p.FW;
 #pragma unroll
         for (int n = 0; n < NV; ++n) {
@@ -556,38 +550,6 @@ __global__ void __launch_bounds__(256, MODE == M_GAT ? GNN_AGG_MINB - 1 : GNN_AG
     return;
   }
 
-  for (int32_t c0 = 0; c0 < p.F; c0 += CW) {
-    // ---- phase 1: one group per worker
-    for (int32_t j = wk; j < ngr; j += nwk) {
-      const int32_t gi = gb + j;
-      const int32_t row = g.grp_row[gi];
-      const int32_t beg = g.grp_beg[gi];
-      const int32_t rb = g.rowptr[row], re = g.rowptr[row + 1];
-      const int32_t end = (re - beg > g.ng) ? beg + g.ng : re;
-      Part<MODE, VEC, NV> P;
-      group_partial<MODE, VEC, NV, LANES>(p, beg, end, row, c0, lane, mask, P);
-      if (beg == rb && end == re) store_row<MODE, VEC, NV, LANES>(p, row, re - rb, c0, lane, P);
-      else slot_store<MODE, VEC, NV, LANES>(smem, p.T, j, lane, P);
-    }
-    __syncthreads();
-    // ---- phase 2: rows with several groups in this tile, combined in group order
-    for (int32_t j = wk; j < ngr; j += nwk) {
-      const int32_t gi = gb + j;
-      const int32_t row = g.grp_row[gi];
-      if (j > 0 && g.grp_row[gi - 1] == row) continue;  // not the first group of the row
-      const int32_t rb = g.rowptr[row], re = g.rowptr[row + 1];
-      const int32_t ngrp = 1 + (re - rb - 1) / g.ng;
-      if (ngrp <= 1) continue;
-      Part<MODE, VEC, NV> A, B;
-      slot_load<MODE, VEC, NV, LANES>(smem, p.T, j, lane, A);
-      for (int32_t k = 1; k < ngrp; ++k) {
-        slot_load<MODE, VEC, NV, LANES>(smem, p.T, j + k, lane, B);
-        part_combine<MODE, VEC, NV>(A, B);
-      }
-      store_row<MODE, VEC, NV, LANES>(p, row, re - rb, c0, lane, A);
-    }
-    if (c0 + CW < p.F) __syncthreads();
-  }
 }
 
 // ---------------------------------------------------------------------------
@@ -632,14 +594,35 @@ size_t agg_workspace_bytes(const gnn_plan_s *p, int mode, int32_t F, int32_t H) 
   return b + sizeof(float) * slots * FW;
 }
 
-template <int MODE, int VEC, int NV, int LANES>
-static cudaError_t launch_one(const KParams &kp, int threads, size_t smem, int64_t blocks,
-                              cudaStream_t s) {
-  auto fn = k_aggregate<MODE, VEC, NV, LANES>;
-  if (smem > 48 * 1024) {
-    cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
+static int num_sms() {
+  static int n = 0;
+  if (n == 0) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    if (n <= 0) n = 148;
   }
+  return n;
+}
+
+template <int MODE, int VEC, int NV, int LANES>
+static cudaError_t launch_one(const KParams &kp_in, int threads, size_t smem, int64_t blocks_unused,
+                              cudaStream_t s) {
+  (void)blocks_unused;
+  auto fn = k_aggregate<MODE, VEC, NV, LANES>;
+  static int occ = 0;  // resident CTAs per SM for this instantiation
+  if (occ == 0) {
+    // no shared memory on the hot path: the whole unified array goes to L1
+    cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, threads, smem);
+    if (occ <= 0) occ = 1;
+  }
+  KParams kp = kp_in;
+  const int64_t workers = threads / LANES;
+  const int64_t want = (kp.g.n_whole + workers - 1) / workers;
+  kp.n_persist = (int32_t)std::min<int64_t>(want, (int64_t)num_sms() * occ);
+  const int64_t blocks = (int64_t)kp.g.n_tiles + kp.n_persist + (kp.g.n_empty + 31) / 32;
+  if (blocks == 0) return cudaSuccess;
   fn<<<(unsigned)blocks, threads, smem, s>>>(kp);
   count_launch();
   return cudaGetLastError();
@@ -715,11 +698,10 @@ gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, siz
   }
   const Mapping m = choose_mapping(a, mode == M_GAT ? a.Fh : 0);
   const int CW = m.lanes * m.vec * m.nv;
-  const int threads = std::min(256, std::max(32, p->T * m.lanes));
-  size_t smem = sizeof(float) * (size_t)p->T * CW;
-  if (mode == M_GAT) smem += sizeof(float) * (size_t)p->T * m.nv * m.lanes * 2;
-  const int64_t blocks = (int64_t)p->dg.n_tiles + (p->dg.n_empty + 31) / 32;
-  if (blocks == 0) return GNN_OK;
+  (void)CW;
+  const int threads = 256;
+  const size_t smem = 0;
+  const int64_t blocks = 0;  // computed per instantiation (occupancy)
   cudaError_t e;
   switch (mode) {
     case M_SUM:

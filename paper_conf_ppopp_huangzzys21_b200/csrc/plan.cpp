@@ -232,65 +232,51 @@ int64_t las_merge(int64_t n, const uint64_t *sig, int32_t K, const std::vector<i
   return nc;
 }
 
-// a3: neighbor groups in schedule order + tiles + split-row
-// tables (reading R8).  Pure host function, also exported as gnn_groups_host.
-void schedule_host(int64_t n, const int64_t *rowptr, const int32_t *perm, int64_t ng, int32_t T,
-                   std::vector<int32_t> &grp_row, std::vector<int64_t> &grp_beg,
-                   std::vector<int64_t> &tile_beg, std::vector<int32_t> &tile_split,
+// a3: neighbor groups in schedule order and tasks (reading R8):
+// a row with <= R groups is one whole-row task (one worker runs its groups in
+// order); a longer row is cut into T-group split tiles whose group partials
+// are merged in group order by the last tile to finish.  Pure host function,
+// also exported as gnn_groups_host.
+void schedule_host(int64_t n, const int64_t *rowptr, const int32_t *perm, int64_t ng, int32_t R, int32_t T,
+                   std::vector<int32_t> &grp_row, std::vector<int64_t> &grp_beg, std::vector<int32_t> &whole_rows,
+                   std::vector<int64_t> &tile_lo, std::vector<int64_t> &tile_hi, std::vector<int32_t> &tile_split,
                    std::vector<int32_t> &split_off, std::vector<int32_t> &split_first,
                    std::vector<int32_t> &split_ntiles, int64_t &slots) {
   grp_row.clear();
   grp_beg.clear();
-  for (int64_t i = 0; i < n; ++i) {
-    const int64_t v = perm ? perm[i] : i;
-    const int64_t beg = rowptr[v], end = rowptr[v + 1];
-    for (int64_t b = beg; b < end; b += ng) {
-      grp_row.push_back((int32_t)v);
-      grp_beg.push_back(b);
-      if (end - b <= ng) break;
-    }
-  }
-  const int64_t G = (int64_t)grp_row.size();
-  // tiles: first-fit of whole runs, runs longer than T get their own tiles
-  tile_beg.assign(1, 0);
+  whole_rows.clear();
+  tile_lo.clear();
+  tile_hi.clear();
   tile_split.clear();
   split_off.clear();
   split_first.clear();
   split_ntiles.clear();
   slots = 0;
-  int64_t cur = 0, g = 0;
-  while (g < G) {
-    int64_t e = g + 1;
-    while (e < G && grp_row[e] == grp_row[g]) ++e;
-    const int64_t run = e - g;
-    if (run > T) {
-      if (cur > 0) {
-        tile_beg.push_back(g);
-        tile_split.push_back(-1);
-        cur = 0;
-      }
+  for (int64_t i = 0; i < n; ++i) {
+    const int64_t v = perm ? perm[i] : i;
+    const int64_t beg = rowptr[v], end = rowptr[v + 1];
+    if (end == beg) continue;
+    const int64_t g0 = (int64_t)grp_row.size();
+    for (int64_t b = beg; b < end; b += ng) {
+      grp_row.push_back((int32_t)v);
+      grp_beg.push_back(b);
+      if (end - b <= ng) break;
+    }
+    const int64_t run = (int64_t)grp_row.size() - g0;
+    if (run <= R) {
+      whole_rows.push_back((int32_t)v);
+    } else {
       const int32_t s = (int32_t)split_off.size();
       split_off.push_back((int32_t)slots);
-      split_first.push_back((int32_t)g);
+      split_first.push_back((int32_t)g0);
       split_ntiles.push_back((int32_t)((run + T - 1) / T));
       slots += run;
-      for (int64_t s0 = g; s0 < e; s0 += T) {
-        tile_beg.push_back(std::min<int64_t>(s0 + T, e));
+      for (int64_t s0 = g0; s0 < g0 + run; s0 += T) {
+        tile_lo.push_back(s0);
+        tile_hi.push_back(std::min<int64_t>(s0 + T, g0 + run));
         tile_split.push_back(s);
       }
-    } else {
-      if (cur + run > T) {
-        tile_beg.push_back(g);
-        tile_split.push_back(-1);
-        cur = 0;
-      }
-      cur += run;
     }
-    g = e;
-  }
-  if (cur > 0) {
-    tile_beg.push_back(G);
-    tile_split.push_back(-1);
   }
 }
 
@@ -298,10 +284,10 @@ gnn_status build_schedule(gnn_plan_s *p) {
   const int64_t n = p->n;
   std::vector<int32_t> tile_split, split_off, split_first, split_ntiles;
   int64_t slots = 0;
-  schedule_host(n, p->rowptr.data(), p->perm.data(), p->ng, p->T, p->grp_row, p->grp_beg, p->tile_beg,
-                tile_split, split_off, split_first, split_ntiles, slots);
+  schedule_host(n, p->rowptr.data(), p->perm.data(), p->ng, p->R, p->T, p->grp_row, p->grp_beg, p->whole_rows,
+                p->tile_lo, p->tile_hi, tile_split, split_off, split_first, split_ntiles, slots);
   const int64_t G = (int64_t)p->grp_row.size();
-  const int64_t n_tiles = (int64_t)p->tile_beg.size() - 1;
+  const int64_t n_tiles = (int64_t)p->tile_lo.size();
   p->n_split = (int64_t)split_off.size();
   p->split_slots = slots;
   std::vector<int32_t> empty;
@@ -309,7 +295,6 @@ gnn_status build_schedule(gnn_plan_s *p) {
     if (p->rowptr[v + 1] == p->rowptr[v]) empty.push_back((int32_t)v);
   p->n_empty = (int64_t)empty.size();
 
-  // upload (int32 on device)
   auto upload = [&](const void *src, size_t bytes, void **dst) -> cudaError_t {
     *dst = nullptr;
     cudaError_t e = cudaMalloc(dst, bytes > 0 ? bytes : 4);
@@ -318,9 +303,12 @@ gnn_status build_schedule(gnn_plan_s *p) {
     if (bytes > 0) e = cudaMemcpy(*dst, src, bytes, cudaMemcpyHostToDevice);
     return e;
   };
-  std::vector<int32_t> grp_beg32((size_t)G), tile_beg32((size_t)n_tiles + 1);
+  std::vector<int32_t> grp_beg32((size_t)G), lo32((size_t)n_tiles), hi32((size_t)n_tiles);
   for (int64_t i = 0; i < G; ++i) grp_beg32[i] = (int32_t)p->grp_beg[i];
-  for (int64_t i = 0; i <= n_tiles; ++i) tile_beg32[i] = (int32_t)p->tile_beg[i];
+  for (int64_t i = 0; i < n_tiles; ++i) {
+    lo32[i] = (int32_t)p->tile_lo[i];
+    hi32[i] = (int32_t)p->tile_hi[i];
+  }
   void *d;
   cudaError_t e;
 #define UP(vec, field)                                                                 \
@@ -329,19 +317,23 @@ gnn_status build_schedule(gnn_plan_s *p) {
   p->dg.field = reinterpret_cast<const int32_t *>(d);
   UP(p->grp_row, grp_row)
   UP(grp_beg32, grp_beg)
-  UP(tile_beg32, tile_beg)
+  UP(p->whole_rows, whole_rows)
+  UP(lo32, tile_lo)
+  UP(hi32, tile_hi)
   UP(tile_split, tile_split)
   UP(split_off, split_off)
   UP(split_first, split_first)
   UP(split_ntiles, split_ntiles)
   UP(empty, empty_rows)
 #undef UP
+  p->dg.n_whole = (int32_t)p->whole_rows.size();
   p->dg.n_tiles = (int32_t)n_tiles;
   p->dg.n_split = (int32_t)p->n_split;
   p->dg.n_empty = (int32_t)p->n_empty;
   p->dg.ng = p->ng;
   p->info.n_groups = G;
   p->info.n_tiles = n_tiles;
+  p->info.n_whole_rows = (int64_t)p->whole_rows.size();
   p->info.n_split_rows = p->n_split;
   p->info.n_empty_rows = p->n_empty;
   return GNN_OK;

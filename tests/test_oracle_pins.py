@@ -512,21 +512,25 @@ def test_neighbor_groups_cover_edges(ng):
     assert order == [int(v) for v in perm if deg[v] > 0]
 
 
-@pytest.mark.parametrize("T", [1, 4, 32])
-def test_tiles(T):
-    g = gs.powerlaw(2000, 40000, 20, 2000, 600, comm=32, rho=0.0, seed=T)
+@pytest.mark.parametrize("R,T", [(1, 1), (4, 32), (4, 3), (32, 32), (0, 8)])
+def test_tasks(R, T):
+    """R8: every group belongs to exactly one task; rows with <= R groups are
+    whole-row tasks in group order; longer runs are cut into T-group tiles."""
+    g = gs.powerlaw(2000, 40000, 20, 2000, 600, comm=32, rho=0.0, seed=T + R)
     gr, gb = oracle.neighbor_groups(g.rowptr, 16)
-    tb = oracle.tiles(gr, T)
-    assert tb[0] == 0 and tb[-1] == len(gr) and np.all(np.diff(tb) >= 1)
-    for a, b in zip(tb[:-1], tb[1:]):
-        rows = gr[a:b]
-        if b - a > 1 and len(set(rows)) > 1:
-            assert b - a <= T
-        # a row is split across tiles only when its run exceeds T
-        if a > 0 and gr[a - 1] == gr[a]:
-            run = np.sum(gr == gr[a])
-            assert run > T
-        assert b - a <= T
+    whole, lo, hi = oracle.tasks(gr, R, T)
+    runs = {}
+    for r in gr:
+        runs[r] = runs.get(r, 0) + 1
+    assert list(whole) == [r for r in dict.fromkeys(gr.tolist()) if runs[r] <= R]
+    covered = np.zeros(len(gr), np.int64)
+    for a, b in zip(lo, hi):
+        assert 0 < b - a <= T
+        assert len(set(gr[a:b])) == 1 and runs[gr[a]] > R
+        covered[a:b] += 1
+    for r in whole:
+        covered[gr == r] += 1
+    assert np.all(covered == 1)
 
 
 def test_partition_rows():
