@@ -69,7 +69,7 @@ typedef struct {
   uint32_t struct_size;  /* sizeof(gnn_plan_opts), for ABI versioning */
   int32_t reorder;       /* 0 = identity task order, 1 = LAS (MinHash+LSH+merge) */
   int32_t group_size;    /* NG upper bound ng; -1 = auto (R8-ii); 0 = never split */
-  int32_t tile_groups;   /* T: groups per split-row CTA tile (0 -> 32) */
+  int32_t tile_groups;   /* T: consecutive groups per CTA work tile (0 -> 32) */
   int32_t cluster_cap;   /* LAS cluster size cap (32) */
   int32_t minhash_k;     /* K signature length (32) */
   int32_t lsh_rows;      /* r rows per band (2); b = K / r bands */
@@ -77,13 +77,12 @@ typedef struct {
   int32_t min_sim;       /* re-enqueue threshold; -1 -> lsh_rows */
   int32_t deterministic; /* 1: fixed-order combine (R9); 0: float atomics */
   int32_t cluster_order; /* LAS schedule: 1 = clusters by representative signature, 0 = by smallest member */
-  int32_t worker_groups; /* R: a row with <= R groups is one whole-row task (0 -> 4) */
   uint64_t seed;         /* MinHash salt stream seed */
 } gnn_plan_opts;
 
 /* Fill defaults: reorder 0, group_size -1, tile_groups 32, cluster_cap 32,
  * minhash_k 32, lsh_rows 2, pair_window 8, min_sim -1, deterministic 1,
- * cluster_order 1, worker_groups 4, seed 0. */
+ * cluster_order 1, seed 0. */
 void gnn_plan_opts_default(gnn_plan_opts *opts);
 
 typedef struct {
@@ -91,9 +90,8 @@ typedef struct {
   int64_t n_src;        /* source rows (== n for gnn_plan_create) */
   int64_t nnz;
   int64_t n_groups;     /* G = sum ceil(d_v / ng) */
-  int64_t n_tiles;      /* split-row tiles (T groups each) */
-  int64_t n_whole_rows; /* whole-row tasks (rows with <= R groups) */
-  int64_t n_split_rows; /* rows with more than R groups */
+  int64_t n_tiles;      /* CTA tiles = ceil(G / T) */
+  int64_t n_split_rows; /* rows with more than one group (combined through the workspace) */
   int64_t n_empty_rows;
   int64_t n_clusters;   /* LAS clusters (n if reorder == 0) */
   int64_t n_pairs;      /* LSH candidate pairs (0 if reorder == 0) */
@@ -130,14 +128,11 @@ gnn_status gnn_plan_get_info(gnn_plan_t plan, gnn_plan_info *info);
 /*
  * Copy the schedule to host buffers sized from gnn_plan_info (any may be NULL):
  * perm_h int32[n] (task order), grp_row_h int32[G], grp_beg_h int64[G] (first
- * CSR entry of each group), whole_rows_h int32[n_whole_rows] (whole-row tasks
- * in order), tile_lo_h / tile_hi_h int64[n_tiles] (group range of each
- * split-row tile).  Bit-exact with the oracle's orc_las_merge /
- * orc_neighbor_groups / orc_tasks.
+ * CSR entry of each group).  CTA tile t is groups [t*T, min((t+1)*T, G)).
+ * Bit-exact with the oracle's orc_las_merge / orc_neighbor_groups.
  */
 gnn_status gnn_plan_export(gnn_plan_t plan, int32_t *perm_h, int32_t *grp_row_h,
-                           int64_t *grp_beg_h, int32_t *whole_rows_h, int64_t *tile_lo_h,
-                           int64_t *tile_hi_h);
+                           int64_t *grp_beg_h);
 
 /*
  * LAS intermediates (reorder == 1 only): sig_h uint64[n * minhash_k] (GPU
@@ -169,8 +164,10 @@ size_t gnn_workspace_size(gnn_plan_t plan, int op, int32_t f_in, int32_t f_out, 
 /*
  * a6 + a9: graph operation y_v = REDUCE_{u->v} e_uv * x_u (Table 1 x Table 2,
  * Eq 1 inner part P:217), evaluated over the plan's neighbor groups in task
- * order; split rows combined in fixed group order (R9) or with atomics
- * (deterministic == 0, sum/mean only).  Epilogue (linear property):
+ * order (one CTA per tile of T consecutive groups, groups round-robin over its
+ * workers); the groups of a multi-group row are combined in fixed group order
+ * by the last worker to finish one (R9), or with atomics (deterministic == 0,
+ * sum/mean only).  Epilogue (linear property):
  * GCN x ndst[v], mean / D_v, then + add_row[v] (nullable, EdgeConv's Q), then
  * ReLU if relu != 0.
  *   edge_w: [nnz] in CSR order, required iff weight == GNN_W_EDGE.
@@ -307,20 +304,16 @@ gnn_status gnn_local_csr(int64_t n, const int64_t *rowptr_h, const int32_t *coli
  *   task scheduling P:846-853; reading R7) from MinHash signatures sig_h
  *   uint64[n * K].  Outputs perm_h int32[n], cluster_of_h int32[n] (nullable),
  *   *n_pairs, *n_clusters.
- * gnn_groups_host: a3 neighbor groups in task order and tasks (P:855-884,
- *   reading R8): whole-row tasks for rows with <= R groups, T-group split
- *   tiles for longer rows.  ng <= 0 = one group per row.  Call with NULL
- *   arrays first to get the counts; then grp_row_h int32[G], grp_beg_h
- *   int64[G], whole_rows_h int32[n_whole], tile_lo_h / tile_hi_h int64[n_tiles].
+ * gnn_groups_host: a3 neighbor groups in task order (reading R8).
+ *   ng <= 0 = one group per row.  Call with NULL arrays first to get
+ *   *n_groups; then grp_row_h int32[G], grp_beg_h int64[G].
  */
 gnn_status gnn_las_host(int64_t n, const int64_t *rowptr_h, const uint64_t *sig_h, int32_t K,
                         int32_t r, int32_t W, int32_t cap, int32_t min_sim, int32_t cluster_order,
                         int32_t *perm_h,
                         int32_t *cluster_of_h, int64_t *n_pairs, int64_t *n_clusters);
 gnn_status gnn_groups_host(int64_t n, const int64_t *rowptr_h, const int32_t *perm_h, int32_t ng,
-                           int32_t R, int32_t T, int64_t *n_groups, int64_t *n_whole,
-                           int64_t *n_tiles, int32_t *grp_row_h, int64_t *grp_beg_h,
-                           int32_t *whole_rows_h, int64_t *tile_lo_h, int64_t *tile_hi_h);
+                           int64_t *n_groups, int32_t *grp_row_h, int64_t *grp_beg_h);
 
 /* Number of kernels this library launched since load (for bench accounting). */
 uint64_t gnn_launch_count(void);

@@ -9,7 +9,7 @@ never imports it.
 
 Parity status per function (DESIGN.md §4 lists the pins):
   aggregate, aggregate_ng_f32, gemm, gcn_layer, gat_aggregate, gat_layer,
-  edgeconv, minhash, lsh_pairs, las_merge, neighbor_groups, tiles,
+  edgeconv, minhash, lsh_pairs, las_merge, neighbor_groups,
   partition_rows: pinned by tests/test_oracle_pins.py.
   LAS *quality* (how much L2 reuse the schedule buys) is "parity unpinned":
   the paper's real graphs are unavailable.
@@ -72,7 +72,6 @@ def lib():
             "orc_lsh_pairs": (_i64, [_i64, _p, _p, _i32, _i32, _i32, _p, _i64]),
             "orc_las_merge": (_i64, [_i64, _p, _i32, _p, _i64, _i32, _i32, _i32, _p, _p, _p]),
             "orc_neighbor_groups": (_i64, [_i64, _p, _p, _i32, _p, _p]),
-            "orc_tasks": (_i64, [_i64, _p, _i32, _i32, _p, _p, _p, _p]),
             "orc_partition_rows": (None, [_i64, _p, _i32, _p]),
             "orc_forget_degrees": (None, []),
         }
@@ -272,18 +271,6 @@ def neighbor_groups(rowptr, ng, perm=None):
     grp_beg = np.empty(max(G, 1), np.int64)
     lib().orc_neighbor_groups(n, _ptr(rowptr), _ptr(p), ng, _ptr(grp_row), _ptr(grp_beg))
     return grp_row[:G], grp_beg[:G]
-
-
-def tasks(grp_row, R=4, T=32):
-    """Whole-row tasks and split tiles (R8): returns (whole_rows, tile_lo, tile_hi)."""
-    grp_row = np.ascontiguousarray(grp_row, dtype=np.int32)
-    nw = ctypes.c_int64()
-    nt = lib().orc_tasks(len(grp_row), _ptr(grp_row), R, T, None, None, None, ctypes.byref(nw))
-    whole = np.empty(max(nw.value, 1), np.int32)
-    lo = np.empty(max(nt, 1), np.int64)
-    hi = np.empty(max(nt, 1), np.int64)
-    lib().orc_tasks(len(grp_row), _ptr(grp_row), R, T, _ptr(whole), _ptr(lo), _ptr(hi), ctypes.byref(nw))
-    return whole[:nw.value], lo[:nt], hi[:nt]
 
 
 def partition_rows(rowptr, P):

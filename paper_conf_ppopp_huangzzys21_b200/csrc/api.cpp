@@ -94,7 +94,6 @@ void gnn_plan_opts_default(gnn_plan_opts *o) {
   o->min_sim = -1;
   o->deterministic = 1;
   o->cluster_order = 1;
-  o->worker_groups = 4;
   o->seed = 0;
 }
 
@@ -122,8 +121,6 @@ gnn_status gnn_plan_create_ex(int64_t n, int64_t n_src, int64_t nnz, const int64
     if (!rowptr_h || (nnz > 0 && !colidx_h)) return check(false, "rowptr/colidx is NULL");
     if (opts.tile_groups == 0) opts.tile_groups = 32;
     if (opts.tile_groups < 1 || opts.tile_groups > 256) return check(false, "tile_groups out of [1, 256]");
-    if (opts.worker_groups == 0) opts.worker_groups = 4;
-    if (opts.worker_groups < 0) return check(false, "worker_groups < 0");
     if (opts.reorder) {
       if (opts.minhash_k < 1 || opts.minhash_k > 64) return check(false, "minhash_k out of [1, 64]");
       if (opts.lsh_rows < 1 || opts.minhash_k % opts.lsh_rows) return check(false, "lsh_rows must divide minhash_k");
@@ -156,7 +153,6 @@ gnn_status gnn_plan_create_ex(int64_t n, int64_t n_src, int64_t nnz, const int64
     p->opts = opts;
     p->max_degree = maxd;
     p->T = opts.tile_groups;
-    p->R = opts.worker_groups;
     // NG bound (R8-ii): largest multiple of 16 <= min(64, 10 * avg degree), >= 16
     int64_t ng = opts.group_size;
     if (ng < 0) {
@@ -265,15 +261,11 @@ gnn_status gnn_plan_get_info(gnn_plan_t p, gnn_plan_info *info) {
   return GNN_OK;
 }
 
-gnn_status gnn_plan_export(gnn_plan_t p, int32_t *perm_h, int32_t *grp_row_h, int64_t *grp_beg_h,
-                           int32_t *whole_rows_h, int64_t *tile_lo_h, int64_t *tile_hi_h) {
+gnn_status gnn_plan_export(gnn_plan_t p, int32_t *perm_h, int32_t *grp_row_h, int64_t *grp_beg_h) {
   if (!p) return check(false, "plan is NULL");
   if (perm_h) std::memcpy(perm_h, p->perm.data(), sizeof(int32_t) * p->perm.size());
   if (grp_row_h) std::memcpy(grp_row_h, p->grp_row.data(), sizeof(int32_t) * p->grp_row.size());
   if (grp_beg_h) std::memcpy(grp_beg_h, p->grp_beg.data(), sizeof(int64_t) * p->grp_beg.size());
-  if (whole_rows_h) std::memcpy(whole_rows_h, p->whole_rows.data(), sizeof(int32_t) * p->whole_rows.size());
-  if (tile_lo_h) std::memcpy(tile_lo_h, p->tile_lo.data(), sizeof(int64_t) * p->tile_lo.size());
-  if (tile_hi_h) std::memcpy(tile_hi_h, p->tile_hi.data(), sizeof(int64_t) * p->tile_hi.size());
   return GNN_OK;
 }
 
@@ -694,24 +686,17 @@ gnn_status gnn_las_host(int64_t n, const int64_t *rowptr_h, const uint64_t *sig_
   })
 }
 
-gnn_status gnn_groups_host(int64_t n, const int64_t *rowptr_h, const int32_t *perm_h, int32_t ng, int32_t R,
-                           int32_t T, int64_t *n_groups, int64_t *n_whole, int64_t *n_tiles, int32_t *grp_row_h,
-                           int64_t *grp_beg_h, int32_t *whole_rows_h, int64_t *tile_lo_h, int64_t *tile_hi_h) {
+gnn_status gnn_groups_host(int64_t n, const int64_t *rowptr_h, const int32_t *perm_h, int32_t ng,
+                           int64_t *n_groups, int32_t *grp_row_h, int64_t *grp_beg_h) {
   GNN_TRY({
-    if (n < 0 || !rowptr_h || !n_groups || !n_whole || !n_tiles || T < 1 || R < 0)
-      return check(false, "bad groups_host arguments");
-    std::vector<int32_t> gr, wr, ts, so, sf, sn;
-    std::vector<int64_t> gb, lo, hi;
+    if (n < 0 || !rowptr_h || !n_groups) return check(false, "bad groups_host arguments");
+    std::vector<int32_t> gr, gm, ms;
+    std::vector<int64_t> gb;
     int64_t slots = 0;
-    schedule_host(n, rowptr_h, perm_h, ng > 0 ? ng : (1 << 30), R, T, gr, gb, wr, lo, hi, ts, so, sf, sn, slots);
+    schedule_host(n, rowptr_h, perm_h, ng > 0 ? ng : (1 << 30), gr, gb, gm, ms, slots);
     *n_groups = (int64_t)gr.size();
-    *n_whole = (int64_t)wr.size();
-    *n_tiles = (int64_t)lo.size();
     if (grp_row_h) std::memcpy(grp_row_h, gr.data(), sizeof(int32_t) * gr.size());
     if (grp_beg_h) std::memcpy(grp_beg_h, gb.data(), sizeof(int64_t) * gb.size());
-    if (whole_rows_h) std::memcpy(whole_rows_h, wr.data(), sizeof(int32_t) * wr.size());
-    if (tile_lo_h) std::memcpy(tile_lo_h, lo.data(), sizeof(int64_t) * lo.size());
-    if (tile_hi_h) std::memcpy(tile_hi_h, hi.data(), sizeof(int64_t) * hi.size());
     return GNN_OK;
   })
 }

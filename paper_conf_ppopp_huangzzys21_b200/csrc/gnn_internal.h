@@ -15,21 +15,16 @@ namespace gnn {
 // Device-side view of a plan handed to the graph kernels (all int32: the
 // plan rejects nnz >= 2^31).
 struct DevGraph {
-  const int32_t *rowptr;       // [n+1]
-  const int32_t *colidx;       // [nnz]
-  const float *nsrc;           // [n_src] 1/sqrtf(d_out)
-  const float *ndst;           // [n]     1/sqrtf(d_in)
-  const int32_t *grp_beg;      // [G] first CSR entry of each group
-  const int32_t *grp_row;      // [G]
-  const int32_t *whole_rows;   // [n_whole] whole-row tasks in task order
-  const int32_t *tile_lo;      // [n_tiles] split-row tile: group range [lo, hi)
-  const int32_t *tile_hi;      // [n_tiles]
-  const int32_t *tile_split;   // [n_tiles] split-row index
-  const int32_t *split_off;    // [n_split] first workspace slot of the split row
-  const int32_t *split_first;  // [n_split] global index of the row's first group
-  const int32_t *split_ntiles; // [n_split]
-  const int32_t *empty_rows;   // [n_empty]
-  int32_t n_whole, n_tiles, n_split, n_empty, ng;
+  const int32_t *rowptr;        // [n+1]
+  const int32_t *colidx;        // [nnz]
+  const float *nsrc;            // [n_src] 1/sqrtf(d_out)
+  const float *ndst;            // [n]     1/sqrtf(d_in)
+  const int32_t *grp_row;       // [G] groups in task order
+  const int32_t *grp_beg;       // [G] first CSR entry of each group
+  const int32_t *grp_multi;     // [G] index m of the group's multi-group row, -1 if the row has one group
+  const int32_t *multi_slot;    // [n_multi] workspace slot of the row's first group
+  const int32_t *empty_rows;    // [n_empty]
+  int32_t n_groups, n_tiles, T, n_multi, n_empty, ng;
 };
 
 }  // namespace gnn
@@ -40,16 +35,14 @@ struct gnn_plan_s {
   gnn_plan_opts opts{};
   int32_t ng = 0;      // effective group bound (INT32_MAX-ish when "never split")
   int32_t T = 32;
-  int32_t R = 4;
   int32_t max_degree = 0;
   // host copies
   std::vector<int64_t> rowptr;
   std::vector<int32_t> perm, grp_row;
-  std::vector<int64_t> grp_beg, tile_lo, tile_hi;
-  std::vector<int32_t> whole_rows;
+  std::vector<int64_t> grp_beg;
   std::vector<uint64_t> sig;
   std::vector<int32_t> pairs, cluster_of;
-  int64_t n_clusters = 0, n_split = 0, n_empty = 0, split_slots = 0;
+  int64_t n_clusters = 0, n_multi = 0, n_empty = 0, multi_slots = 0;
   gnn_plan_info info{};
   // device allocations (owned)
   std::vector<void *> dev_allocs;
@@ -65,12 +58,9 @@ void count_launch(uint64_t k = 1);
 
 // planner (plan.cpp) — host side
 gnn_status build_schedule(gnn_plan_s *p);
-void schedule_host(int64_t n, const int64_t *rowptr, const int32_t *perm, int64_t ng, int32_t R,
-                   int32_t T, std::vector<int32_t> &grp_row, std::vector<int64_t> &grp_beg,
-                   std::vector<int32_t> &whole_rows, std::vector<int64_t> &tile_lo,
-                   std::vector<int64_t> &tile_hi, std::vector<int32_t> &tile_split,
-                   std::vector<int32_t> &split_off, std::vector<int32_t> &split_first,
-                   std::vector<int32_t> &split_ntiles, int64_t &slots);
+void schedule_host(int64_t n, const int64_t *rowptr, const int32_t *perm, int64_t ng,
+                   std::vector<int32_t> &grp_row, std::vector<int64_t> &grp_beg,
+                   std::vector<int32_t> &grp_multi, std::vector<int32_t> &multi_slot, int64_t &slots);
 int64_t las_lsh_pairs(int64_t n, const int64_t *rowptr, const uint64_t *sig, int32_t K, int32_t r,
                       int32_t W, std::vector<int32_t> &pairs);
 int64_t las_merge(int64_t n, const uint64_t *sig, int32_t K, const std::vector<int32_t> &pairs,

@@ -182,50 +182,79 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p) {
 
   if (warp < NUM_PRODUCER_WARPS) {
     // ------------------------------ producers ------------------------------
-    int it = 0;  // global K-block counter across tiles (stage/phase tracking)
-    for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
-      const int64_t m0 = (int64_t)tile * BM;
-      for (int kb = 0; kb < p.num_kb; ++kb, ++it) {
-        const int s = it % S, use = it / S;
-        if (use > 0) mbar_wait(&empty_bar[s], (use - 1) & 1);
-        uint8_t *st = smem + (size_t)s * STAGE_BYTES;
-        uint8_t *a_hi = st, *a_lo = st + TILE_A_BYTES, *b_img = st + 2 * TILE_A_BYTES;
-        if (tid == 0) {
-          mbar_arrive_expect_tx(&full_bar[s], 2 * B_BYTES);
-          const uint8_t *src = p.wimg + (size_t)kb * 2 * B_BYTES;
-          for (int off = 0; off < 2 * B_BYTES; off += 16384) {
-            const int bytes = 2 * B_BYTES - off < 16384 ? 2 * B_BYTES - off : 16384;
-            bulk_g2s(b_img + off, src + off, bytes, &full_bar[s]);
+    // The X tile of the NEXT K block is loaded into registers before waiting
+    // for the current stage to free up, so global-memory latency overlaps the
+    // MMAs of earlier stages (one K block of register look-ahead).
+    constexpr int PER_THREAD = BM * 8 / (NUM_PRODUCER_WARPS * 32);  // float4 chunks per thread per K block
+    float4 buf[2][PER_THREAD];
+    auto load_a = [&](float4 (&dst)[PER_THREAD], int64_t m0, int kb) {
+      const int k0 = kb * BK;
+#pragma unroll
+      for (int i = 0; i < PER_THREAD; ++i) {
+        const int q = tid + i * NUM_PRODUCER_WARPS * 32;
+        const int r = q >> 3, c = q & 7;
+        const int64_t gm = m0 + r;
+        const int gk = k0 + 4 * c;
+        float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (gm < p.m) {
+          const float *src = p.X + gm * p.ldx + gk;
+          if (VEC_X && gk + 3 < p.k) {
+            x = __ldg(reinterpret_cast<const float4 *>(src));
+          } else {
+            if (gk + 0 < p.k) x.x = __ldg(src + 0);
+            if (gk + 1 < p.k) x.y = __ldg(src + 1);
+            if (gk + 2 < p.k) x.z = __ldg(src + 2);
+            if (gk + 3 < p.k) x.w = __ldg(src + 3);
           }
         }
-        const int k0 = kb * BK;
-#pragma unroll 4
-        for (int q = tid; q < BM * 8; q += NUM_PRODUCER_WARPS * 32) {
-          const int r = q >> 3, c = q & 7;
-          const int64_t gm = m0 + r;
-          const int gk = k0 + 4 * c;
-          float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
-          if (gm < p.m) {
-            const float *src = p.X + gm * p.ldx + gk;
-            if (VEC_X && gk + 3 < p.k) {
-              x = __ldg(reinterpret_cast<const float4 *>(src));
-            } else {
-              if (gk + 0 < p.k) x.x = __ldg(src + 0);
-              if (gk + 1 < p.k) x.y = __ldg(src + 1);
-              if (gk + 2 < p.k) x.z = __ldg(src + 2);
-              if (gk + 3 < p.k) x.w = __ldg(src + 3);
-            }
-          }
-          const float4 hi = make_float4(hi_of(x.x), hi_of(x.y), hi_of(x.z), hi_of(x.w));
-          const float4 lo = make_float4(x.x - hi.x, x.y - hi.y, x.z - hi.z, x.w - hi.w);
-          const uint32_t off = sw128_off(r, c);
-          *reinterpret_cast<float4 *>(a_hi + off) = hi;
-          *reinterpret_cast<float4 *>(a_lo + off) = lo;
-        }
-        // generic-proxy smem writes -> visible to the tensor core (async proxy)
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        mbar_arrive(&full_bar[s]);
+        dst[i] = x;
       }
+    };
+    int it = 0;  // global K-block counter across tiles (stage/phase tracking)
+    int tile = blockIdx.x;
+    int kb = 0;
+    if (tile < p.num_tiles) load_a(buf[0], (int64_t)tile * BM, 0);
+    while (tile < p.num_tiles) {
+      // next (tile, kb) to prefetch
+      int ntile = tile, nkb = kb + 1;
+      if (nkb == p.num_kb) {
+        nkb = 0;
+        ntile += gridDim.x;
+      }
+      const int cur = it & 1;
+      if (ntile < p.num_tiles) {
+        if (cur == 0) load_a(buf[1], (int64_t)ntile * BM, nkb);
+        else load_a(buf[0], (int64_t)ntile * BM, nkb);
+      }
+      const int s = it % S, use = it / S;
+      if (use > 0) mbar_wait(&empty_bar[s], (use - 1) & 1);
+      uint8_t *st = smem + (size_t)s * STAGE_BYTES;
+      uint8_t *a_hi = st, *a_lo = st + TILE_A_BYTES, *b_img = st + 2 * TILE_A_BYTES;
+      if (tid == 0) {
+        mbar_arrive_expect_tx(&full_bar[s], 2 * B_BYTES);
+        const uint8_t *src = p.wimg + (size_t)kb * 2 * B_BYTES;
+        for (int off = 0; off < 2 * B_BYTES; off += 16384) {
+          const int bytes = 2 * B_BYTES - off < 16384 ? 2 * B_BYTES - off : 16384;
+          bulk_g2s(b_img + off, src + off, bytes, &full_bar[s]);
+        }
+      }
+#pragma unroll
+      for (int i = 0; i < PER_THREAD; ++i) {
+        const int q = tid + i * NUM_PRODUCER_WARPS * 32;
+        const int r = q >> 3, c = q & 7;
+        const float4 x = cur == 0 ? buf[0][i] : buf[1][i];
+        const float4 hi = make_float4(hi_of(x.x), hi_of(x.y), hi_of(x.z), hi_of(x.w));
+        const float4 lo = make_float4(x.x - hi.x, x.y - hi.y, x.z - hi.z, x.w - hi.w);
+        const uint32_t off = sw128_off(r, c);
+        *reinterpret_cast<float4 *>(a_hi + off) = hi;
+        *reinterpret_cast<float4 *>(a_lo + off) = lo;
+      }
+      // generic-proxy smem writes -> visible to the tensor core (async proxy)
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      mbar_arrive(&full_bar[s]);
+      ++it;
+      tile = ntile;
+      kb = nkb;
     }
   } else if (warp == MMA_WARP) {
     // ------------------------------ MMA issuer ------------------------------

@@ -170,13 +170,12 @@ struct KParams {
   int64_t ldt;
   int32_t H, Fh;
   float slope;
-  float *ws_acc;   // [n_split][FW] atomic accumulators (deterministic == 0)
-  float *ws_part;  // [split slots][FW] per-group partials (deterministic)
-  int32_t *ws_cnt; // [n_split]
+  float *ws_acc;   // [n_multi][FW] atomic accumulators (deterministic == 0)
+  float *ws_part;  // [multi slots][FW] per-group partials (deterministic)
+  int32_t *ws_cnt; // [n_multi][nch] arrival counters
   int32_t FW;      // F (+ 2H for GAT)
   int32_t deterministic;
-  int32_t T;
-  int32_t n_persist;  // blocks of the persistent whole-row phase
+  int32_t nch;  // feature chunks per row (arrival counters per multi-group row)
 };
 
 template <int VEC>
@@ -424,13 +423,108 @@ __device__ __forceinline__ void store_row(const KParams &p, int32_t row, int32_t
   }
 }
 
+// load VEC floats from L2 (bypassing L1: data written by other SMs in this launch)
+template <int VEC>
+__device__ __forceinline__ void ldv_cg(const float *p, float (&v)[VEC]) {
+  if constexpr (VEC == 8) {
+    const float4 a = __ldcg(reinterpret_cast<const float4 *>(p));
+    const float4 b = __ldcg(reinterpret_cast<const float4 *>(p) + 1);
+    v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w; v[4] = b.x; v[5] = b.y; v[6] = b.z; v[7] = b.w;
+  } else if constexpr (VEC == 4) {
+    const float4 a = __ldcg(reinterpret_cast<const float4 *>(p));
+    v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
+  } else if constexpr (VEC == 2) {
+    const float2 a = __ldcg(reinterpret_cast<const float2 *>(p));
+    v[0] = a.x; v[1] = a.y;
+  } else {
+    v[0] = __ldcg(p);
+  }
+}
+
+// a9: a group of a multi-group row.  Deterministic: the group partial goes to
+// its workspace slot; the worker that completes the row's last group merges
+// all partials in group order (R9) and applies the postponed epilogue
+// (P:970-986).  Atomic variant (sum/mean): partials are added into one
+// accumulator row and the last worker applies the epilogue.
+template <int MODE, int VEC, int NV, int LANES>
+__device__ __forceinline__ void multi_group_combine(const KParams &p, int32_t m, int32_t row, int32_t rb, int32_t re,
+                                                    int32_t beg, int32_t c0, int32_t ci, int lane, unsigned mask,
+                                                    const Part<MODE, VEC, NV> &P) {
+  const int32_t ng = p.g.ng;
+  const int32_t ngrp = 1 + (re - rb - 1) / ng;
+  const int32_t k = (beg - rb) / ng;
+  const bool atomic_acc = !p.deterministic && MODE == M_SUM;
+  float *base = p.ws_part + (size_t)p.g.multi_slot[m] * p.FW;
+  float *acc = p.ws_acc + (size_t)m * p.FW;
+#pragma unroll
+  for (int n = 0; n < NV; ++n) {
+    const int32_t f = c0 + (n * LANES + lane) * VEC;
+    if (f >= p.F) continue;
+    if (atomic_acc) {
+#pragma unroll
+      for (int i = 0; i < VEC; ++i) atomicAdd(acc + f + i, P.a[n][i]);
+    } else {
+      stv<VEC>(base + (size_t)k * p.FW + f, P.a[n]);
+      if constexpr (MODE == M_GAT) {
+        if (f % p.Fh == 0) {
+          base[(size_t)k * p.FW + p.F + f / p.Fh] = P.m[n];
+          base[(size_t)k * p.FW + p.F + p.H + f / p.Fh] = P.l[n];
+        }
+      }
+    }
+  }
+  __threadfence();
+  __syncwarp(mask);
+  int last = 0;
+  int32_t *cnt = p.ws_cnt + (size_t)m * p.nch + ci;
+  if (lane == 0) last = atomicAdd(cnt, 1) == ngrp - 1;
+  last = __shfl_sync(mask, last, 0, LANES);
+  if (!last) return;
+  __threadfence();
+  Part<MODE, VEC, NV> A;
+  part_init(A);
+#pragma unroll
+  for (int n = 0; n < NV; ++n) {
+    const int32_t f = c0 + (n * LANES + lane) * VEC;
+    if (f >= p.F) continue;
+    if (atomic_acc) {
+      ldv_cg<VEC>(acc + f, A.a[n]);
+      continue;
+    }
+    for (int32_t q = 0; q < ngrp; ++q) {
+      float b[VEC];
+      ldv_cg<VEC>(base + (size_t)q * p.FW + f, b);
+      if constexpr (MODE == M_GAT) {
+        const float bm = __ldcg(base + (size_t)q * p.FW + p.F + f / p.Fh);
+        const float bl = __ldcg(base + (size_t)q * p.FW + p.F + p.H + f / p.Fh);
+        if (q == 0) {
+#pragma unroll
+          for (int i = 0; i < VEC; ++i) A.a[n][i] = b[i];
+          A.m[n] = bm;
+          A.l[n] = bl;
+        } else {
+          gat_merge(A.m[n], A.l[n], A.a[n], bm, bl, b, VEC);
+        }
+      } else {
+#pragma unroll
+        for (int i = 0; i < VEC; ++i)
+          A.a[n][i] = (q == 0) ? b[i] : (MODE == M_MAX ? fmaxf(A.a[n][i], b[i]) : A.a[n][i] + b[i]);
+      }
+    }
+  }
+  store_row<MODE, VEC, NV, LANES>(p, row, re - rb, c0, lane, A);
+  if (lane == 0) *cnt = 0;  // leave the counter at 0 for the next call
+}
+
 #ifndef GNN_AGG_MINB
 #define GNN_AGG_MINB 4
 #endif
+// One CTA per tile of T consecutive groups in task order (a LAS cluster stays
+// on one SM); groups round-robin over the CTA's workers (NG load
+// balance).  No shared memory and no CTA barrier on the hot path.
 template <int MODE, int VEC, int NV, int LANES>
 __global__ void __launch_bounds__(256, MODE == M_GAT ? GNN_AGG_MINB - 1 : GNN_AGG_MINB) k_aggregate(const KParams p) {
   constexpr int CW = LANES * VEC * NV;
-  __shared__ int s_last;
   const int tid = threadIdx.x;
   const int lane = tid & (LANES - 1);
   const int wk = tid / LANES;
@@ -438,118 +532,31 @@ __global__ void __launch_bounds__(256, MODE == M_GAT ? GNN_AGG_MINB - 1 : GNN_AG
   const unsigned mask =
       LANES == 32 ? 0xffffffffu : (((1u << LANES) - 1u) << ((tid & 31) & ~(LANES - 1)));
   const DevGraph &g = p.g;
-
-  const int32_t nb_split = g.n_tiles;
-  if ((int32_t)blockIdx.x >= nb_split) {
-    const int32_t b = (int32_t)blockIdx.x - nb_split;
-    if (b < p.n_persist) {
-      // ---- whole-row tasks (<= R groups): statically interleaved over every
-      // worker of the persistent grid, so rows adjacent in the LAS task order
-      // are processed at the same time; one worker runs a row's
-      // groups in order and combines them in registers (R9)
-      const int64_t gw = (int64_t)b * nwk + wk, GW = (int64_t)p.n_persist * nwk;
-      for (int32_t c0 = 0; c0 < p.F; c0 += CW) {
-        for (int64_t i = gw; i < g.n_whole; i += GW) {
-          const int32_t row = g.whole_rows[i];
-          const int32_t rb = g.rowptr[row], re = g.rowptr[row + 1];
-          Part<MODE, VEC, NV> A;
-          row_chain<MODE, VEC, NV, LANES>(p, rb, re, row, c0, lane, mask, A);
-          store_row<MODE, VEC, NV, LANES>(p, row, re - rb, c0, lane, A);
-        }
-      }
-      return;
-    }
+  if ((int32_t)blockIdx.x >= g.n_tiles) {
     // zero-fill rows without in-edges (R3-i): 32 rows per block
-    const int64_t r0 = (int64_t)(b - p.n_persist) * 32;
+    const int64_t r0 = (int64_t)(blockIdx.x - g.n_tiles) * 32;
     for (int64_t r = r0; r < r0 + 32 && r < g.n_empty; ++r) {
       float *y = p.Y + (int64_t)g.empty_rows[r] * p.ldy;
       for (int f = tid; f < p.F; f += blockDim.x) y[f] = 0.0f;
     }
     return;
   }
-  // ---- split-row tile: a row with more than R groups; groups spread over the
-  // CTA's workers, partials to the workspace, last-arriving CTA merges them
-  const int32_t t = blockIdx.x;
-  const int32_t gb = g.tile_lo[t], ngr = g.tile_hi[t] - gb;
-  const int32_t split = g.tile_split[t];
-  {
-    // ---- a row spanning several tiles: partials -> workspace, last CTA merges
-    const int32_t row = g.grp_row[gb];
-    const int32_t rb = g.rowptr[row], re = g.rowptr[row + 1];
-    const int32_t first = g.split_first[split];
-    float *part = p.ws_part + (size_t)g.split_off[split] * p.FW;
-    for (int32_t c0 = 0; c0 < p.F; c0 += CW) {
-      for (int32_t j = wk; j < ngr; j += nwk) {
-        const int32_t gi = gb + j;
-        const int32_t beg = g.grp_beg[gi], end = (re - beg > g.ng) ? beg + g.ng : re;
-        Part<MODE, VEC, NV> P;
-        row_chain<MODE, VEC, NV, LANES>(p, beg, end, row, c0, lane, mask, P);
-        float *dst = part + (size_t)(gi - first) * p.FW;
-#pragma unroll
-        for (int n = 0; n < NV; ++n) {
-          const int32_t f = c0 + (n * LANES + lane) * VEC;
-          if (f >= p.F) continue;
-          if (!p.deterministic && MODE != M_GAT && MODE != M_MAX) {
-            float *acc = p.ws_acc + (size_t)split * p.FW;  // one accumulator row per split row
-#pragma unroll
-            for (int i = 0; i < VEC; ++i) atomicAdd(acc + f + i, P.a[n][i]);
-          } else {
-            stv<VEC>(dst + f, P.a[n]);
-          }
-          if constexpr (MODE == M_GAT) {
-            if (f % p.Fh == 0) {
-              dst[p.F + f / p.Fh] = P.m[n];
-              dst[p.F + p.H + f / p.Fh] = P.l[n];
-            }
-          }
-        }
-      }
+  const int32_t gb = (int32_t)blockIdx.x * g.T;
+  const int32_t ngr = min(g.T, g.n_groups - gb);
+  int32_t ci = 0;
+  for (int32_t c0 = 0; c0 < p.F; c0 += CW, ++ci) {
+    for (int32_t j = wk; j < ngr; j += nwk) {
+      const int32_t gi = gb + j;
+      const int32_t row = g.grp_row[gi], beg = g.grp_beg[gi];
+      const int32_t rb = g.rowptr[row], re = g.rowptr[row + 1];
+      const int32_t end = (re - beg > g.ng) ? beg + g.ng : re;
+      Part<MODE, VEC, NV> P;
+      row_chain<MODE, VEC, NV, LANES>(p, beg, end, row, c0, lane, mask, P);  // exactly one group
+      const int32_t m = g.grp_multi[gi];
+      if (m < 0) store_row<MODE, VEC, NV, LANES>(p, row, re - rb, c0, lane, P);
+      else multi_group_combine<MODE, VEC, NV, LANES>(p, m, row, rb, re, beg, c0, ci, lane, mask, P);
     }
-    __threadfence();
-    __syncthreads();
-    if (tid == 0) {
-      const int old = atomicAdd(p.ws_cnt + split, 1);
-      s_last = old == g.split_ntiles[split] - 1;
-    }
-    __syncthreads();
-    if (!s_last) return;
-    __threadfence();
-    const int32_t ngrp = 1 + (re - rb - 1) / g.ng;
-    const float ndst = (MODE != M_GAT && scales_dst(p.weight)) ? __ldg(g.ndst + row) : 1.0f;
-    const float deg_f = (float)(re - rb);
-    const bool atomic_acc = !p.deterministic && MODE != M_GAT && MODE != M_MAX;
-    for (int32_t f = tid; f < p.F; f += blockDim.x) {
-      float a, l = 1.0f, m = 0.0f;
-      if (atomic_acc) {
-        float *acc = p.ws_acc + (size_t)split * p.FW + f;
-        a = __ldcg(acc);
-        *acc = 0.0f;  // leave the accumulator zeroed for the next call
-      } else {
-        a = __ldcg(part + f);
-        if (MODE == M_GAT) {
-          m = __ldcg(part + p.F + f / p.Fh);
-          l = __ldcg(part + p.F + p.H + f / p.Fh);
-        }
-        for (int32_t k = 1; k < ngrp; ++k) {
-          const float *q = part + (size_t)k * p.FW;
-          const float b = __ldcg(q + f);
-          if (MODE == M_GAT) {
-            const float m2 = __ldcg(q + p.F + f / p.Fh), l2 = __ldcg(q + p.F + p.H + f / p.Fh);
-            gat_merge(m, l, &a, m2, l2, &b, 1);
-          } else if (MODE == M_MAX) {
-            a = fmaxf(a, b);
-          } else {
-            a = a + b;
-          }
-        }
-      }
-      const float *addp = p.add_row ? p.add_row + (int64_t)row * p.ld_add + f : nullptr;
-      p.Y[(int64_t)row * p.ldy + f] = epi(p, p.mode, a, l, ndst, deg_f, addp);
-    }
-    if (tid == 0) p.ws_cnt[split] = 0;  // reset for the next call
-    return;
   }
-
 }
 
 // ---------------------------------------------------------------------------
@@ -568,11 +575,13 @@ static Mapping choose_mapping(const AggArgs &a, int32_t fh_or_0) {
   Mapping m{1, 4, 1};
   const int cands[4] = {8, 4, 2, 1};
   for (int v : cands) {
-    bool ok = a.F % v == 0 && a.ldx % v == 0 && a.ldy % v == 0 && aligned(a.X, 4 * v) &&
-              aligned(a.Y, 4 * v);
+    bool ok = a.F % v == 0 && a.ldx % v == 0 && a.ldy % v == 0 && aligned(a.X, 4 * v) && aligned(a.Y, 4 * v);
     if (a.add_row) ok = ok && a.ld_add % v == 0 && aligned(a.add_row, 4 * v);
     if (fh_or_0) ok = ok && fh_or_0 % v == 0;
-    if (ok) { m.vec = v; break; }
+    if (ok) {
+      m.vec = v;
+      break;
+    }
   }
   const int nvec = a.F / m.vec;  // vectors per row
   int lanes = 4;
@@ -580,48 +589,41 @@ static Mapping choose_mapping(const AggArgs &a, int32_t fh_or_0) {
   m.lanes = lanes;
   m.nv = 1;
   if (lanes == 32) {
-    const int max_nv = m.vec == 8 ? 2 : 4;  // keep T*CW*4 <= 64 KB at T = 32
+    const int max_nv = m.vec == 8 ? 2 : 4;
     while (m.nv < max_nv && 32 * m.nv < nvec) m.nv *= 2;
   }
   return m;
 }
 
-size_t agg_workspace_bytes(const gnn_plan_s *p, int mode, int32_t F, int32_t H) {
-  const size_t FW = (size_t)F + (mode == M_GAT ? 2 * (size_t)H : 0);
-  const size_t slots = (size_t)p->split_slots + (size_t)p->n_split;  // + atomic accumulators
-  size_t b = sizeof(int32_t) * (size_t)(p->n_split > 0 ? p->n_split : 0);
-  b = (b + 255) & ~(size_t)255;
-  return b + sizeof(float) * slots * FW;
-}
+static int32_t max_chunks(int32_t F) { return F <= 128 ? 1 : (F + 31) / 32; }
 
-static int num_sms() {
-  static int n = 0;
-  if (n == 0) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
-    if (n <= 0) n = 148;
-  }
-  return n;
+size_t agg_workspace_bytes(const gnn_plan_s *p, int mode, int32_t F, int32_t H) {
+  if (p->n_multi == 0) return 0;
+  const size_t FW = (size_t)F + (mode == M_GAT ? 2 * (size_t)H : 0);
+  size_t b = sizeof(int32_t) * (size_t)p->n_multi * max_chunks(F);
+  b = (b + 255) & ~(size_t)255;
+  return b + sizeof(float) * ((size_t)p->multi_slots + (size_t)p->n_multi) * FW;
 }
 
 template <int MODE, int VEC, int NV, int LANES>
-static cudaError_t launch_one(const KParams &kp_in, int threads, size_t smem, int64_t blocks_unused,
-                              cudaStream_t s) {
-  (void)blocks_unused;
+static cudaError_t launch_one(const KParams &kp_in, int threads, size_t smem, int64_t blocks, cudaStream_t s) {
   auto fn = k_aggregate<MODE, VEC, NV, LANES>;
-  static int occ = 0;  // resident CTAs per SM for this instantiation
-  if (occ == 0) {
-    // no shared memory on the hot path: the whole unified array goes to L1
+  static bool configured = false;  // per instantiation
+  if (!configured) {
+    // no shared memory on the hot path: the unified array goes to L1, which
+    // serves the source rows a LAS cluster (one tile, one SM) shares
     cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, 0);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, threads, smem);
-    if (occ <= 0) occ = 1;
+    configured = true;
   }
   KParams kp = kp_in;
-  const int64_t workers = threads / LANES;
-  const int64_t want = (kp.g.n_whole + workers - 1) / workers;
-  kp.n_persist = (int32_t)std::min<int64_t>(want, (int64_t)num_sms() * occ);
-  const int64_t blocks = (int64_t)kp.g.n_tiles + kp.n_persist + (kp.g.n_empty + 31) / 32;
+  constexpr int CW = LANES * VEC * NV;
+  kp.nch = (kp.F + CW - 1) / CW;
+  if (kp.g.n_multi > 0) {
+    cudaError_t e = cudaMemsetAsync(kp.ws_cnt, 0, sizeof(int32_t) * (size_t)kp.g.n_multi * kp.nch, s);
+    if (e == cudaSuccess && !kp.deterministic && MODE == M_SUM)
+      e = cudaMemsetAsync(kp.ws_acc, 0, sizeof(float) * (size_t)kp.g.n_multi * kp.FW, s);
+    if (e != cudaSuccess) return e;
+  }
   if (blocks == 0) return cudaSuccess;
   fn<<<(unsigned)blocks, threads, smem, s>>>(kp);
   count_launch();
@@ -629,8 +631,8 @@ static cudaError_t launch_one(const KParams &kp_in, int threads, size_t smem, in
 }
 
 template <int MODE, int VEC>
-static cudaError_t dispatch_lanes(const KParams &kp, const Mapping &m, int threads, size_t smem,
-                                  int64_t blocks, cudaStream_t s) {
+static cudaError_t dispatch_lanes(const KParams &kp, const Mapping &m, int threads, size_t smem, int64_t blocks,
+                                  cudaStream_t s) {
   switch (m.lanes) {
     case 4: return launch_one<MODE, VEC, 1, 4>(kp, threads, smem, blocks, s);
     case 8: return launch_one<MODE, VEC, 1, 8>(kp, threads, smem, blocks, s);
@@ -644,8 +646,8 @@ static cudaError_t dispatch_lanes(const KParams &kp, const Mapping &m, int threa
 }
 
 template <int MODE>
-static cudaError_t dispatch_vec(const KParams &kp, const Mapping &m, int threads, size_t smem,
-                                int64_t blocks, cudaStream_t s) {
+static cudaError_t dispatch_vec(const KParams &kp, const Mapping &m, int threads, size_t smem, int64_t blocks,
+                                cudaStream_t s) {
   switch (m.vec) {
     case 8: return dispatch_lanes<MODE, 8>(kp, m, threads, smem, blocks, s);
     case 4: return dispatch_lanes<MODE, 4>(kp, m, threads, smem, blocks, s);
@@ -654,12 +656,11 @@ static cudaError_t dispatch_vec(const KParams &kp, const Mapping &m, int threads
   }
 }
 
-gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, size_t ws_bytes,
-                            cudaStream_t s) {
+gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, size_t ws_bytes, cudaStream_t s) {
   if (a.F <= 0) return GNN_OK;
   const int mode = a.mode;
   const size_t need = agg_workspace_bytes(p, mode, a.F, a.H);
-  if (p->n_split > 0 && (ws == nullptr || ws_bytes < need)) {
+  if (p->n_multi > 0 && (ws == nullptr || ws_bytes < need)) {
     set_error("workspace too small: need " + std::to_string(need) + " bytes");
     return GNN_ERR_WORKSPACE;
   }
@@ -683,25 +684,17 @@ gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, siz
   kp.slope = a.slope;
   kp.FW = a.F + (mode == M_GAT ? 2 * a.H : 0);
   kp.deterministic = a.deterministic;
-  kp.T = p->T;
-  if (p->n_split > 0) {
-    // layout: [counters n_split int32 | pad to 256 B][accumulators n_split x FW][slots x FW]
-    const size_t cnt_bytes = (sizeof(int32_t) * (size_t)p->n_split + 255) & ~(size_t)255;
+  if (p->n_multi > 0) {
+    // layout: [counters n_multi x nch int32 | pad to 256 B][accumulators n_multi x FW][slots x FW]
+    const size_t cnt_bytes = (sizeof(int32_t) * (size_t)p->n_multi * max_chunks(a.F) + 255) & ~(size_t)255;
     kp.ws_cnt = reinterpret_cast<int32_t *>(ws);
     kp.ws_acc = reinterpret_cast<float *>(reinterpret_cast<char *>(ws) + cnt_bytes);
-    kp.ws_part = kp.ws_acc + (size_t)p->n_split * kp.FW;
-    // counters (and the atomic accumulators) start at 0 every call
-    cudaError_t e = cudaMemsetAsync(kp.ws_cnt, 0, sizeof(int32_t) * (size_t)p->n_split, s);
-    if (e == cudaSuccess && !a.deterministic && mode != M_GAT && mode != M_MAX)
-      e = cudaMemsetAsync(kp.ws_acc, 0, sizeof(float) * (size_t)p->n_split * kp.FW, s);
-    if (e != cudaSuccess) return cuda_status(e, "workspace memset");
+    kp.ws_part = kp.ws_acc + (size_t)p->n_multi * kp.FW;
   }
   const Mapping m = choose_mapping(a, mode == M_GAT ? a.Fh : 0);
-  const int CW = m.lanes * m.vec * m.nv;
-  (void)CW;
-  const int threads = 256;
+  const int threads = std::min(256, std::max(32, p->T * m.lanes));
   const size_t smem = 0;
-  const int64_t blocks = 0;  // computed per instantiation (occupancy)
+  const int64_t blocks = (int64_t)p->dg.n_tiles + (p->dg.n_empty + 31) / 32;
   cudaError_t e;
   switch (mode) {
     case M_SUM:

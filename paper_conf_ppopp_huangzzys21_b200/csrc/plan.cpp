@@ -232,64 +232,44 @@ int64_t las_merge(int64_t n, const uint64_t *sig, int32_t K, const std::vector<i
   return nc;
 }
 
-// a3: neighbor groups in schedule order and tasks (reading R8):
-// a row with <= R groups is one whole-row task (one worker runs its groups in
-// order); a longer row is cut into T-group split tiles whose group partials
-// are merged in group order by the last tile to finish.  Pure host function,
-// also exported as gnn_groups_host.
-void schedule_host(int64_t n, const int64_t *rowptr, const int32_t *perm, int64_t ng, int32_t R, int32_t T,
-                   std::vector<int32_t> &grp_row, std::vector<int64_t> &grp_beg, std::vector<int32_t> &whole_rows,
-                   std::vector<int64_t> &tile_lo, std::vector<int64_t> &tile_hi, std::vector<int32_t> &tile_split,
-                   std::vector<int32_t> &split_off, std::vector<int32_t> &split_first,
-                   std::vector<int32_t> &split_ntiles, int64_t &slots) {
+// a3: neighbor groups in task order (reading R8).  CTA tile t is
+// groups [t*T, (t+1)*T).  A row with more than one group ("multi-group") gets
+// workspace slots for its group partials, merged in group order by the last
+// worker to finish one of them (R9).  Pure host function (gnn_groups_host).
+void schedule_host(int64_t n, const int64_t *rowptr, const int32_t *perm, int64_t ng,
+                   std::vector<int32_t> &grp_row, std::vector<int64_t> &grp_beg, std::vector<int32_t> &grp_multi,
+                   std::vector<int32_t> &multi_slot, int64_t &slots) {
   grp_row.clear();
   grp_beg.clear();
-  whole_rows.clear();
-  tile_lo.clear();
-  tile_hi.clear();
-  tile_split.clear();
-  split_off.clear();
-  split_first.clear();
-  split_ntiles.clear();
+  grp_multi.clear();
+  multi_slot.clear();
   slots = 0;
   for (int64_t i = 0; i < n; ++i) {
     const int64_t v = perm ? perm[i] : i;
     const int64_t beg = rowptr[v], end = rowptr[v + 1];
     if (end == beg) continue;
-    const int64_t g0 = (int64_t)grp_row.size();
+    const bool multi = end - beg > ng;
+    const int32_t m = multi ? (int32_t)multi_slot.size() : -1;
+    if (multi) multi_slot.push_back((int32_t)slots);
     for (int64_t b = beg; b < end; b += ng) {
       grp_row.push_back((int32_t)v);
       grp_beg.push_back(b);
+      grp_multi.push_back(m);
+      if (multi) ++slots;
       if (end - b <= ng) break;
-    }
-    const int64_t run = (int64_t)grp_row.size() - g0;
-    if (run <= R) {
-      whole_rows.push_back((int32_t)v);
-    } else {
-      const int32_t s = (int32_t)split_off.size();
-      split_off.push_back((int32_t)slots);
-      split_first.push_back((int32_t)g0);
-      split_ntiles.push_back((int32_t)((run + T - 1) / T));
-      slots += run;
-      for (int64_t s0 = g0; s0 < g0 + run; s0 += T) {
-        tile_lo.push_back(s0);
-        tile_hi.push_back(std::min<int64_t>(s0 + T, g0 + run));
-        tile_split.push_back(s);
-      }
     }
   }
 }
 
 gnn_status build_schedule(gnn_plan_s *p) {
   const int64_t n = p->n;
-  std::vector<int32_t> tile_split, split_off, split_first, split_ntiles;
+  std::vector<int32_t> grp_multi, multi_slot;
   int64_t slots = 0;
-  schedule_host(n, p->rowptr.data(), p->perm.data(), p->ng, p->R, p->T, p->grp_row, p->grp_beg, p->whole_rows,
-                p->tile_lo, p->tile_hi, tile_split, split_off, split_first, split_ntiles, slots);
+  schedule_host(n, p->rowptr.data(), p->perm.data(), p->ng, p->grp_row, p->grp_beg, grp_multi, multi_slot, slots);
   const int64_t G = (int64_t)p->grp_row.size();
-  const int64_t n_tiles = (int64_t)p->tile_lo.size();
-  p->n_split = (int64_t)split_off.size();
-  p->split_slots = slots;
+  const int64_t n_tiles = (G + p->T - 1) / p->T;
+  p->n_multi = (int64_t)multi_slot.size();
+  p->multi_slots = slots;
   std::vector<int32_t> empty;
   for (int64_t v = 0; v < n; ++v)
     if (p->rowptr[v + 1] == p->rowptr[v]) empty.push_back((int32_t)v);
@@ -303,12 +283,8 @@ gnn_status build_schedule(gnn_plan_s *p) {
     if (bytes > 0) e = cudaMemcpy(*dst, src, bytes, cudaMemcpyHostToDevice);
     return e;
   };
-  std::vector<int32_t> grp_beg32((size_t)G), lo32((size_t)n_tiles), hi32((size_t)n_tiles);
+  std::vector<int32_t> grp_beg32((size_t)G);
   for (int64_t i = 0; i < G; ++i) grp_beg32[i] = (int32_t)p->grp_beg[i];
-  for (int64_t i = 0; i < n_tiles; ++i) {
-    lo32[i] = (int32_t)p->tile_lo[i];
-    hi32[i] = (int32_t)p->tile_hi[i];
-  }
   void *d;
   cudaError_t e;
 #define UP(vec, field)                                                                 \
@@ -317,24 +293,19 @@ gnn_status build_schedule(gnn_plan_s *p) {
   p->dg.field = reinterpret_cast<const int32_t *>(d);
   UP(p->grp_row, grp_row)
   UP(grp_beg32, grp_beg)
-  UP(p->whole_rows, whole_rows)
-  UP(lo32, tile_lo)
-  UP(hi32, tile_hi)
-  UP(tile_split, tile_split)
-  UP(split_off, split_off)
-  UP(split_first, split_first)
-  UP(split_ntiles, split_ntiles)
+  UP(grp_multi, grp_multi)
+  UP(multi_slot, multi_slot)
   UP(empty, empty_rows)
 #undef UP
-  p->dg.n_whole = (int32_t)p->whole_rows.size();
+  p->dg.n_groups = (int32_t)G;
   p->dg.n_tiles = (int32_t)n_tiles;
-  p->dg.n_split = (int32_t)p->n_split;
+  p->dg.T = p->T;
+  p->dg.n_multi = (int32_t)p->n_multi;
   p->dg.n_empty = (int32_t)p->n_empty;
   p->dg.ng = p->ng;
   p->info.n_groups = G;
   p->info.n_tiles = n_tiles;
-  p->info.n_whole_rows = (int64_t)p->whole_rows.size();
-  p->info.n_split_rows = p->n_split;
+  p->info.n_split_rows = p->n_multi;
   p->info.n_empty_rows = p->n_empty;
   return GNN_OK;
 }

@@ -43,13 +43,12 @@ class gnn_plan_opts(ctypes.Structure):
     _fields_ = [("struct_size", ctypes.c_uint32), ("reorder", ctypes.c_int32), ("group_size", ctypes.c_int32),
                 ("tile_groups", ctypes.c_int32), ("cluster_cap", ctypes.c_int32), ("minhash_k", ctypes.c_int32),
                 ("lsh_rows", ctypes.c_int32), ("pair_window", ctypes.c_int32), ("min_sim", ctypes.c_int32),
-                ("deterministic", ctypes.c_int32), ("cluster_order", ctypes.c_int32), ("worker_groups", ctypes.c_int32),
-                ("seed", ctypes.c_uint64)]
+                ("deterministic", ctypes.c_int32), ("cluster_order", ctypes.c_int32), ("seed", ctypes.c_uint64)]
 
 
 class gnn_plan_info(ctypes.Structure):
-    _fields_ = [(k, ctypes.c_int64) for k in ("n", "n_src", "nnz", "n_groups", "n_tiles", "n_whole_rows",
-                                                "n_split_rows", "n_empty_rows", "n_clusters", "n_pairs")] + \
+    _fields_ = [(k, ctypes.c_int64) for k in ("n", "n_src", "nnz", "n_groups", "n_tiles", "n_split_rows",
+                                                "n_empty_rows", "n_clusters", "n_pairs")] + \
                [(k, ctypes.c_int32) for k in ("group_size", "tile_groups", "max_degree", "reorder")] + \
                [(k, ctypes.c_double) for k in ("ms_validate", "ms_upload", "ms_degrees", "ms_minhash", "ms_lsh",
                                                  "ms_merge", "ms_ng")]
@@ -67,7 +66,7 @@ _SIGS = {
     "gnn_plan_create_ex": (ctypes.c_int, [_I64, _I64, _I64, _P, _P, _P, ctypes.POINTER(gnn_plan_opts),
                                           ctypes.POINTER(_P)]),
     "gnn_plan_get_info": (ctypes.c_int, [_P, ctypes.POINTER(gnn_plan_info)]),
-    "gnn_plan_export": (ctypes.c_int, [_P, _P, _P, _P, _P, _P, _P]),
+    "gnn_plan_export": (ctypes.c_int, [_P, _P, _P, _P]),
     "gnn_plan_export_las": (ctypes.c_int, [_P, _P, _P, _P]),
     "gnn_plan_normalizers": (ctypes.c_int, [_P, ctypes.POINTER(_P), ctypes.POINTER(_P)]),
     "gnn_plan_destroy": (ctypes.c_int, [_P]),
@@ -89,8 +88,7 @@ _SIGS = {
                                      _P, _P, _P]),
     "gnn_las_host": (ctypes.c_int, [_I64, _P, _P, _I32, _I32, _I32, _I32, _I32, _I32, _P, _P, ctypes.POINTER(_I64),
                                     ctypes.POINTER(_I64)]),
-    "gnn_groups_host": (ctypes.c_int, [_I64, _P, _P, _I32, _I32, _I32, ctypes.POINTER(_I64), ctypes.POINTER(_I64),
-                                       ctypes.POINTER(_I64), _P, _P, _P, _P, _P]),
+    "gnn_groups_host": (ctypes.c_int, [_I64, _P, _P, _I32, ctypes.POINTER(_I64), _P, _P]),
     "gnn_launch_count": (ctypes.c_uint64, []),
     "gnn_last_error": (ctypes.c_char_p, []),
     "gnn_version": (ctypes.c_char_p, []),
@@ -180,18 +178,13 @@ class Plan:
         return {k: getattr(i, k) for k, _ in gnn_plan_info._fields_}
 
     def export(self):
-        """(perm, grp_row, grp_beg, whole_rows, tile_lo, tile_hi)"""
-        info = self.info
-        G, W, NT = info["n_groups"], info["n_whole_rows"], info["n_tiles"]
+        """(perm, grp_row, grp_beg); CTA tile t = groups [t*T, (t+1)*T)."""
+        G = self.info["n_groups"]
         perm = np.empty(self.n, np.int32)
         gr = np.empty(max(G, 1), np.int32)
         gb = np.empty(max(G, 1), np.int64)
-        wr = np.empty(max(W, 1), np.int32)
-        lo = np.empty(max(NT, 1), np.int64)
-        hi = np.empty(max(NT, 1), np.int64)
-        _call("gnn_plan_export", self.handle, _np_ptr(perm), _np_ptr(gr), _np_ptr(gb), _np_ptr(wr), _np_ptr(lo),
-              _np_ptr(hi))
-        return perm, gr[:G], gb[:G], wr[:W], lo[:NT], hi[:NT]
+        _call("gnn_plan_export", self.handle, _np_ptr(perm), _np_ptr(gr), _np_ptr(gb))
+        return perm, gr[:G], gb[:G]
 
     def export_las(self):
         info = self.info
@@ -366,23 +359,17 @@ def las_host(rowptr, sig, r=2, W=8, cap=32, min_sim=-1, cluster_order=1):
     return perm, cl, npairs.value, nc.value
 
 
-def groups_host(rowptr, ng, R=4, T=32, perm=None):
-    """a3 neighbor groups + tasks on the host (no GPU):
-    (grp_row, grp_beg, whole_rows, tile_lo, tile_hi)."""
+def groups_host(rowptr, ng, perm=None):
+    """a3 neighbor groups in task order on the host (no GPU): (grp_row, grp_beg)."""
     rowptr = np.ascontiguousarray(rowptr, dtype=np.int64)
     n = len(rowptr) - 1
     p = None if perm is None else np.ascontiguousarray(perm, dtype=np.int32)
-    G, W, NT = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
-    _call("gnn_groups_host", n, _np_ptr(rowptr), _np_ptr(p), ng, R, T, ctypes.byref(G), ctypes.byref(W),
-          ctypes.byref(NT), None, None, None, None, None)
+    G = ctypes.c_int64()
+    _call("gnn_groups_host", n, _np_ptr(rowptr), _np_ptr(p), ng, ctypes.byref(G), None, None)
     gr = np.empty(max(G.value, 1), np.int32)
     gb = np.empty(max(G.value, 1), np.int64)
-    wr = np.empty(max(W.value, 1), np.int32)
-    lo = np.empty(max(NT.value, 1), np.int64)
-    hi = np.empty(max(NT.value, 1), np.int64)
-    _call("gnn_groups_host", n, _np_ptr(rowptr), _np_ptr(p), ng, R, T, ctypes.byref(G), ctypes.byref(W),
-          ctypes.byref(NT), _np_ptr(gr), _np_ptr(gb), _np_ptr(wr), _np_ptr(lo), _np_ptr(hi))
-    return gr[:G.value], gb[:G.value], wr[:W.value], lo[:NT.value], hi[:NT.value]
+    _call("gnn_groups_host", n, _np_ptr(rowptr), _np_ptr(p), ng, ctypes.byref(G), _np_ptr(gr), _np_ptr(gb))
+    return gr[:G.value], gb[:G.value]
 
 
 def launch_count() -> int:

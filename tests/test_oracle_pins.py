@@ -489,7 +489,7 @@ def test_las_invariants_powerlaw(seed):
 
 
 # --------------------------------------------------------------------------- #
-# a3 neighbor grouping + tiles (reading R8)
+# a3 neighbor grouping (reading R8)
 # --------------------------------------------------------------------------- #
 @pytest.mark.parametrize("ng", [0, 1, 4, 16, 64])
 def test_neighbor_groups_cover_edges(ng):
@@ -510,27 +510,6 @@ def test_neighbor_groups_cover_edges(ng):
     # schedule order: rows appear in perm order
     order = [r for i, r in enumerate(gr) if i == 0 or gr[i - 1] != r]
     assert order == [int(v) for v in perm if deg[v] > 0]
-
-
-@pytest.mark.parametrize("R,T", [(1, 1), (4, 32), (4, 3), (32, 32), (0, 8)])
-def test_tasks(R, T):
-    """R8: every group belongs to exactly one task; rows with <= R groups are
-    whole-row tasks in group order; longer runs are cut into T-group tiles."""
-    g = gs.powerlaw(2000, 40000, 20, 2000, 600, comm=32, rho=0.0, seed=T + R)
-    gr, gb = oracle.neighbor_groups(g.rowptr, 16)
-    whole, lo, hi = oracle.tasks(gr, R, T)
-    runs = {}
-    for r in gr:
-        runs[r] = runs.get(r, 0) + 1
-    assert list(whole) == [r for r in dict.fromkeys(gr.tolist()) if runs[r] <= R]
-    covered = np.zeros(len(gr), np.int64)
-    for a, b in zip(lo, hi):
-        assert 0 < b - a <= T
-        assert len(set(gr[a:b])) == 1 and runs[gr[a]] > R
-        covered[a:b] += 1
-    for r in whole:
-        covered[gr == r] += 1
-    assert np.all(covered == 1)
 
 
 def test_partition_rows():
