@@ -69,7 +69,7 @@ typedef struct {
   uint32_t struct_size;  /* sizeof(gnn_plan_opts), for ABI versioning */
   int32_t reorder;       /* 0 = identity task order, 1 = LAS (MinHash+LSH+merge) */
   int32_t group_size;    /* NG upper bound ng; -1 = auto (R8-ii); 0 = never split */
-  int32_t tile_groups;   /* T: consecutive groups per CTA work tile (0 -> 32) */
+  int32_t tile_groups;   /* T: max groups per work unit; longer rows are split (0 -> 32) */
   int32_t cluster_cap;   /* LAS cluster size cap (32) */
   int32_t minhash_k;     /* K signature length (32) */
   int32_t lsh_rows;      /* r rows per band (2); b = K / r bands */
@@ -90,8 +90,8 @@ typedef struct {
   int64_t n_src;        /* source rows (== n for gnn_plan_create) */
   int64_t nnz;
   int64_t n_groups;     /* G = sum ceil(d_v / ng) */
-  int64_t n_tiles;      /* CTA tiles = ceil(G / T) */
-  int64_t n_split_rows; /* rows with more than one group (combined through the workspace) */
+  int64_t n_tiles;      /* work units (whole rows, or T-group slices of longer rows) */
+  int64_t n_split_rows; /* rows with more than T groups (combined through the workspace) */
   int64_t n_empty_rows;
   int64_t n_clusters;   /* LAS clusters (n if reorder == 0) */
   int64_t n_pairs;      /* LSH candidate pairs (0 if reorder == 0) */
@@ -128,8 +128,8 @@ gnn_status gnn_plan_get_info(gnn_plan_t plan, gnn_plan_info *info);
 /*
  * Copy the schedule to host buffers sized from gnn_plan_info (any may be NULL):
  * perm_h int32[n] (task order), grp_row_h int32[G], grp_beg_h int64[G] (first
- * CSR entry of each group).  CTA tile t is groups [t*T, min((t+1)*T, G)).
- * Bit-exact with the oracle's orc_las_merge / orc_neighbor_groups.
+ * CSR entry of each group).  Bit-exact with the oracle's orc_las_merge /
+ * orc_neighbor_groups.
  */
 gnn_status gnn_plan_export(gnn_plan_t plan, int32_t *perm_h, int32_t *grp_row_h,
                            int64_t *grp_beg_h);
@@ -164,10 +164,10 @@ size_t gnn_workspace_size(gnn_plan_t plan, int op, int32_t f_in, int32_t f_out, 
 /*
  * a6 + a9: graph operation y_v = REDUCE_{u->v} e_uv * x_u (Table 1 x Table 2,
  * Eq 1 inner part P:217), evaluated over the plan's neighbor groups in task
- * order (one CTA per tile of T consecutive groups, groups round-robin over its
- * workers); the groups of a multi-group row are combined in fixed group order
- * by the last worker to finish one (R9), or with atomics (deterministic == 0,
- * sum/mean only).  Epilogue (linear property):
+ * order: persistent workers take work units (a whole row, or T groups of a
+ * longer row) in task order; a row's group partials are combined in fixed
+ * group order (R9) — in registers, or in the workspace by the last unit of a
+ * long row to finish — or with atomics (deterministic == 0, sum/mean only).  Epilogue (linear property):
  * GCN x ndst[v], mean / D_v, then + add_row[v] (nullable, EdgeConv's Q), then
  * ReLU if relu != 0.
  *   edge_w: [nnz] in CSR order, required iff weight == GNN_W_EDGE.

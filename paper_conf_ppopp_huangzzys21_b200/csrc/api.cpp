@@ -153,11 +153,12 @@ gnn_status gnn_plan_create_ex(int64_t n, int64_t n_src, int64_t nnz, const int64
     p->opts = opts;
     p->max_degree = maxd;
     p->T = opts.tile_groups;
-    // NG bound (R8-ii): largest multiple of 16 <= min(64, 10 * avg degree), >= 16
+    // NG bound (R8-ii): largest multiple of 16 <= 10 * average degree
+    // (P:1163-1165), clamped to [16, 4096]
     int64_t ng = opts.group_size;
     if (ng < 0) {
       const double avg = n > 0 ? (double)nnz / (double)n : 0.0;
-      ng = (int64_t)(std::min(64.0, 10.0 * avg) / 16.0) * 16;
+      ng = (int64_t)(std::min(4096.0, 10.0 * avg) / 16.0) * 16;
       if (ng < 16) ng = 16;
     }
     p->info.group_size = (int32_t)ng;
@@ -235,7 +236,9 @@ gnn_status gnn_plan_create_ex(int64_t n, int64_t n_src, int64_t nnz, const int64
     }
     // a3: neighbor grouping + tiles
     t0 = std::chrono::steady_clock::now();
+    p->colidx_h = colidx_h;
     gnn_status st = build_schedule(p);
+    p->colidx_h = nullptr;
     if (st != GNN_OK) return fail(st);
     p->info.ms_ng = ms_since(t0);
     p->info.n = n;
@@ -690,10 +693,9 @@ gnn_status gnn_groups_host(int64_t n, const int64_t *rowptr_h, const int32_t *pe
                            int64_t *n_groups, int32_t *grp_row_h, int64_t *grp_beg_h) {
   GNN_TRY({
     if (n < 0 || !rowptr_h || !n_groups) return check(false, "bad groups_host arguments");
-    std::vector<int32_t> gr, gm, ms;
+    std::vector<int32_t> gr;
     std::vector<int64_t> gb;
-    int64_t slots = 0;
-    schedule_host(n, rowptr_h, perm_h, ng > 0 ? ng : (1 << 30), gr, gb, gm, ms, slots);
+    schedule_host(n, rowptr_h, perm_h, ng > 0 ? ng : (1 << 30), gr, gb);
     *n_groups = (int64_t)gr.size();
     if (grp_row_h) std::memcpy(grp_row_h, gr.data(), sizeof(int32_t) * gr.size());
     if (grp_beg_h) std::memcpy(grp_beg_h, gb.data(), sizeof(int64_t) * gb.size());

@@ -16,15 +16,17 @@ namespace gnn {
 // plan rejects nnz >= 2^31).
 struct DevGraph {
   const int32_t *rowptr;        // [n+1]
-  const int32_t *colidx;        // [nnz]
+  const int32_t *colidx;        // [nnz] CSR order
   const float *nsrc;            // [n_src] 1/sqrtf(d_out)
   const float *ndst;            // [n]     1/sqrtf(d_in)
-  const int32_t *grp_row;       // [G] groups in task order
-  const int32_t *grp_beg;       // [G] first CSR entry of each group
-  const int32_t *grp_multi;     // [G] index m of the group's multi-group row, -1 if the row has one group
-  const int32_t *multi_slot;    // [n_multi] workspace slot of the row's first group
+  const int4 *unit_desc;        // [n_units+1] work units in task order: {tpos, beg, row, m}
+                                //   tpos = offset in colidx_t, beg = CSR offset of the unit's first entry,
+                                //   m = long-row index (-1: the unit is the whole row); [n_units] = {nnz,0,0,-1}
+  const int32_t *colidx_t;      // [nnz + 16] source indices in task order
+  const int32_t *multi_slot;    // [n_multi] workspace slot of a long row's first group
+  const int32_t *multi_units;   // [n_multi] number of units of a long row
   const int32_t *empty_rows;    // [n_empty]
-  int32_t n_groups, n_tiles, T, n_multi, n_empty, ng;
+  int32_t n_units, n_multi, n_empty, ng;
 };
 
 }  // namespace gnn
@@ -37,12 +39,13 @@ struct gnn_plan_s {
   int32_t T = 32;
   int32_t max_degree = 0;
   // host copies
+  const int32_t *colidx_h = nullptr;  // caller's array, valid only during gnn_plan_create
   std::vector<int64_t> rowptr;
   std::vector<int32_t> perm, grp_row;
   std::vector<int64_t> grp_beg;
   std::vector<uint64_t> sig;
   std::vector<int32_t> pairs, cluster_of;
-  int64_t n_clusters = 0, n_multi = 0, n_empty = 0, multi_slots = 0;
+  int64_t n_clusters = 0, n_multi = 0, n_empty = 0, multi_slots = 0, max_tile_edges = 0;
   gnn_plan_info info{};
   // device allocations (owned)
   std::vector<void *> dev_allocs;
@@ -59,8 +62,7 @@ void count_launch(uint64_t k = 1);
 // planner (plan.cpp) — host side
 gnn_status build_schedule(gnn_plan_s *p);
 void schedule_host(int64_t n, const int64_t *rowptr, const int32_t *perm, int64_t ng,
-                   std::vector<int32_t> &grp_row, std::vector<int64_t> &grp_beg,
-                   std::vector<int32_t> &grp_multi, std::vector<int32_t> &multi_slot, int64_t &slots);
+                   std::vector<int32_t> &grp_row, std::vector<int64_t> &grp_beg);
 int64_t las_lsh_pairs(int64_t n, const int64_t *rowptr, const uint64_t *sig, int32_t K, int32_t r,
                       int32_t W, std::vector<int32_t> &pairs);
 int64_t las_merge(int64_t n, const uint64_t *sig, int32_t K, const std::vector<int32_t> &pairs,

@@ -170,12 +170,14 @@ struct KParams {
   int64_t ldt;
   int32_t H, Fh;
   float slope;
+  int32_t *ws_unit;  // work-unit counters (one per feature chunk), zeroed per call
   float *ws_acc;   // [n_multi][FW] atomic accumulators (deterministic == 0)
   float *ws_part;  // [multi slots][FW] per-group partials (deterministic)
   int32_t *ws_cnt; // [n_multi][nch] arrival counters
   int32_t FW;      // F (+ 2H for GAT)
   int32_t deterministic;
-  int32_t nch;  // feature chunks per row (arrival counters per multi-group row)
+  int32_t nch;        // feature chunks per row (arrival counters per multi-unit row)
+  int32_t n_persist;  // persistent CTAs
 };
 
 template <int VEC>
@@ -269,126 +271,6 @@ __device__ __forceinline__ void part_combine(Part<MODE, VEC, NV> &A, const Part<
   }
 }
 
-// Chain over CSR entries [beg, end) of destination `row`, neighbour groups
-// of ng entries starting at beg (R9): a fresh fp32 group partial G runs in CSR
-// order and is folded into the row accumulator A at every group boundary
-// (A = G for the first group, then A = A (+) G).  One rolling register ring
-// keeps U source rows in flight per worker across group boundaries; the next
-// batch of LANES indices is requested before the current batch is consumed.
-template <int MODE, int VEC, int NV, int LANES>
-__device__ __forceinline__ void row_chain(const KParams &p, int32_t beg, int32_t end, int32_t row, int32_t c0,
-                                          int lane, unsigned mask, Part<MODE, VEC, NV> &A) {
-  constexpr int FPL = VEC * NV;  // floats per lane per source row
-  constexpr int U = FPL >= 32 ? 1 : (32 / FPL > 8 ? 8 : 32 / FPL);
-  const int32_t ng = p.g.ng;
-  Part<MODE, VEC, NV> G;
-  part_init(G);
-  bool valid[NV];
-  int32_t head[NV];
-  float tv[NV];
-#pragma unroll
-  for (int n = 0; n < NV; ++n) {
-    const int32_t f = c0 + (n * LANES + lane) * VEC;
-    valid[n] = f < p.F;
-    head[n] = 0;
-    tv[n] = 0.0f;
-    if constexpr (MODE == M_GAT) {
-      head[n] = valid[n] ? f / p.Fh : 0;
-      tv[n] = valid[n] ? __ldg(p.t + (int64_t)row * p.ldt + head[n]) : 0.0f;
-    }
-  }
-  const int weight = p.weight;
-  auto load_idx = [&](int32_t k, int32_t cnt, int32_t &u, float &w) {
-    u = 0;
-    w = 1.0f;
-    if (lane < cnt) {
-      u = ld_stream_i32(p.g.colidx + k + lane);
-      if constexpr (MODE != M_GAT) {
-        if (weight == GNN_W_GCN) w = __ldg(p.g.nsrc + u);
-        else if (weight == GNN_W_EDGE) w = ld_stream_f32(p.edge_w + k + lane);
-      }
-    }
-  };
-  float v[U][NV][VEC];
-  float sc[U][NV];
-  auto load_row = [&](int q, int32_t u) {
-    const float *xr = p.X + (int64_t)u * p.ldx;
-#pragma unroll
-    for (int n = 0; n < NV; ++n) {
-      if (valid[n]) ldv<VEC>(xr + c0 + (n * LANES + lane) * VEC, v[q][n]);
-      if constexpr (MODE == M_GAT) sc[q][n] = valid[n] ? __ldg(xr + p.F + head[n]) : 0.0f;
-    }
-  };
-  int32_t k = beg;
-  int32_t cnt = min(LANES, end - k);
-  int32_t my_u;
-  float my_w;
-  load_idx(k, cnt, my_u, my_w);
-  int32_t next_fold = (end - beg > ng) ? beg + ng : end;  // absolute index ending the current group
-  bool first = true;
-  for (;;) {
-    const int32_t kn = k + LANES;
-    const int32_t cnt_n = kn < end ? min(LANES, end - kn) : 0;
-    int32_t nx_u;
-    float nx_w;
-    load_idx(kn, cnt_n, nx_u, nx_w);
-#pragma unroll
-    for (int q = 0; q < U; ++q)
-      if (q < cnt) load_row(q, __shfl_sync(mask, my_u, q, LANES));
-    for (int32_t j = 0; j < cnt; j += U) {
-#pragma unroll
-      for (int q = 0; q < U; ++q) {
-        const int32_t e = j + q;
-        if (e < cnt) {
-          if constexpr (MODE == M_GAT) {
-#pragma unroll
-            for (int n = 0; n < NV; ++n) {
-              if (!valid[n]) continue;
-              float sco = sc[q][n] + tv[n];
-              sco = sco > 0.0f ? sco : p.slope * sco;  // LeakyReLU (Table 2 GAT, P:271-273)
-              const float d = sco - G.m[n];
-              const float ex = __expf(-fabsf(d));
-              const bool up = d > 0.0f;
-#pragma unroll
-              for (int i = 0; i < VEC; ++i)
-                G.a[n][i] = fmaf(up ? G.a[n][i] : v[q][n][i], ex, up ? v[q][n][i] : G.a[n][i]);
-              G.l[n] = fmaf(up ? G.l[n] : 1.0f, ex, up ? 1.0f : G.l[n]);
-              G.m[n] = up ? sco : G.m[n];
-            }
-          } else {
-            const float w = __shfl_sync(mask, my_w, e, LANES);
-#pragma unroll
-            for (int n = 0; n < NV; ++n) {
-              if (!valid[n]) continue;
-#pragma unroll
-              for (int i = 0; i < VEC; ++i) {
-                if constexpr (MODE == M_MAX) G.a[n][i] = fmaxf(G.a[n][i], w * v[q][n][i]);
-                else G.a[n][i] = fmaf(w, v[q][n][i], G.a[n][i]);
-              }
-            }
-          }
-          if (e + U < cnt) load_row(q, __shfl_sync(mask, my_u, e + U, LANES));
-          if (k + e + 1 == next_fold) {  // group boundary: fold G into A, restart G
-            if (first) {
-              A = G;
-              first = false;
-            } else {
-              part_combine<MODE, VEC, NV>(A, G);
-            }
-            part_init(G);
-            next_fold = (end - next_fold > ng) ? next_fold + ng : end;
-          }
-        }
-      }
-    }
-    if (cnt_n == 0) break;
-    k = kn;
-    cnt = cnt_n;
-    my_u = nx_u;
-    my_w = nx_w;
-  }
-}
-
 // epilogue on one value (linear property: normalisation postponed)
 __device__ __forceinline__ float epi(const KParams &p, int mode, float a, float l, float ndst,
                                      float deg_f, const float *addp) {
@@ -441,56 +323,122 @@ __device__ __forceinline__ void ldv_cg(const float *p, float (&v)[VEC]) {
   }
 }
 
-// a9: a group of a multi-group row.  Deterministic: the group partial goes to
-// its workspace slot; the worker that completes the row's last group merges
-// all partials in group order (R9) and applies the postponed epilogue
-// (P:970-986).  Atomic variant (sum/mean): partials are added into one
-// accumulator row and the last worker applies the epilogue.
+// ---------------------------------------------------------------------------
+// v8 work distribution (measured: scripts/stream_bench_k.cu): persistent
+// workers grab work units in task (LAS) order through one atomic counter, so
+// the units in flight across the GPU are consecutive in the schedule and share
+// their source rows in L2; load balance is dynamic (NG's goal,
+// P:855-884) with no CTA barrier.  A unit is a whole row (<= R groups) or an
+// R-group slice of a longer row; its source indices are read from the
+// task-ordered colidx_t (one contiguous stream per unit).
+// ---------------------------------------------------------------------------
+
+// one neighbour group: fresh fp32 chain in CSR order (R9); indices from the
+// task-ordered stream, LANES at a time, U source rows in flight per worker
 template <int MODE, int VEC, int NV, int LANES>
-__device__ __forceinline__ void multi_group_combine(const KParams &p, int32_t m, int32_t row, int32_t rb, int32_t re,
-                                                    int32_t beg, int32_t c0, int32_t ci, int lane, unsigned mask,
-                                                    const Part<MODE, VEC, NV> &P) {
-  const int32_t ng = p.g.ng;
-  const int32_t ngrp = 1 + (re - rb - 1) / ng;
-  const int32_t k = (beg - rb) / ng;
-  const bool atomic_acc = !p.deterministic && MODE == M_SUM;
-  float *base = p.ws_part + (size_t)p.g.multi_slot[m] * p.FW;
-  float *acc = p.ws_acc + (size_t)m * p.FW;
+__device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx, int32_t len, int32_t beg,
+                                            int32_t row, int32_t c0, int lane, unsigned mask,
+                                            Part<MODE, VEC, NV> &G) {
+  constexpr int FPL = VEC * NV;
+  constexpr int U = FPL >= 32 ? 1 : (32 / FPL > 8 ? 8 : 32 / FPL);
+  part_init(G);
+  const int weight = p.weight;
+  const float *xl = p.X + c0 + lane * VEC;
+  bool valid[NV];
+  int32_t head[NV];
+  float tv[NV];
 #pragma unroll
   for (int n = 0; n < NV; ++n) {
     const int32_t f = c0 + (n * LANES + lane) * VEC;
-    if (f >= p.F) continue;
-    if (atomic_acc) {
+    valid[n] = f < p.F;
+    head[n] = 0;
+    tv[n] = 0.0f;
+    if constexpr (MODE == M_GAT) {
+      head[n] = valid[n] ? f / p.Fh : 0;
+      tv[n] = valid[n] ? __ldg(p.t + (int64_t)row * p.ldt + head[n]) : 0.0f;
+    }
+  }
+  for (int32_t k = 0; k < len; k += LANES) {
+    const int32_t cnt = min(LANES, len - k);
+    int32_t my_u = 0;
+    float my_w = 1.0f;
+    if (lane < cnt) {
+      my_u = ld_stream_i32(idx + k + lane);
+      if constexpr (MODE != M_GAT) {
+        if (weight == GNN_W_GCN) my_w = __ldg(p.g.nsrc + my_u);
+        else if (weight == GNN_W_EDGE) my_w = ld_stream_f32(p.edge_w + beg + k + lane);
+      }
+    }
+    float v[U][NV][VEC];
+    float sc[U][NV];
 #pragma unroll
-      for (int i = 0; i < VEC; ++i) atomicAdd(acc + f + i, P.a[n][i]);
-    } else {
-      stv<VEC>(base + (size_t)k * p.FW + f, P.a[n]);
-      if constexpr (MODE == M_GAT) {
-        if (f % p.Fh == 0) {
-          base[(size_t)k * p.FW + p.F + f / p.Fh] = P.m[n];
-          base[(size_t)k * p.FW + p.F + p.H + f / p.Fh] = P.l[n];
+    for (int q = 0; q < U; ++q) {
+      if (q < cnt) {
+        const int32_t u = __shfl_sync(mask, my_u, q, LANES);
+#pragma unroll
+        for (int n = 0; n < NV; ++n) {
+          if (valid[n]) ldv<VEC>(xl + (int64_t)u * p.ldx + n * LANES * VEC, v[q][n]);
+          if constexpr (MODE == M_GAT) sc[q][n] = valid[n] ? __ldg(p.X + (int64_t)u * p.ldx + p.F + head[n]) : 0.0f;
+        }
+      }
+    }
+    for (int32_t j = 0; j < cnt; j += U) {
+#pragma unroll
+      for (int q = 0; q < U; ++q) {
+        const int32_t e = j + q;
+        if (e < cnt) {
+          if constexpr (MODE == M_GAT) {
+#pragma unroll
+            for (int n = 0; n < NV; ++n) {
+              if (!valid[n]) continue;
+              float sco = sc[q][n] + tv[n];
+              sco = sco > 0.0f ? sco : p.slope * sco;  // LeakyReLU (Table 2 GAT, P:271-273)
+              const float d = sco - G.m[n];
+              const float ex = __expf(-fabsf(d));
+              const bool up = d > 0.0f;
+#pragma unroll
+              for (int i = 0; i < VEC; ++i)
+                G.a[n][i] = fmaf(up ? G.a[n][i] : v[q][n][i], ex, up ? v[q][n][i] : G.a[n][i]);
+              G.l[n] = fmaf(up ? G.l[n] : 1.0f, ex, up ? 1.0f : G.l[n]);
+              G.m[n] = up ? sco : G.m[n];
+            }
+          } else {
+            const float w = __shfl_sync(mask, my_w, e, LANES);
+#pragma unroll
+            for (int n = 0; n < NV; ++n) {
+              if (!valid[n]) continue;
+#pragma unroll
+              for (int i = 0; i < VEC; ++i) {
+                if constexpr (MODE == M_MAX) G.a[n][i] = fmaxf(G.a[n][i], w * v[q][n][i]);
+                else G.a[n][i] = fmaf(w, v[q][n][i], G.a[n][i]);
+              }
+            }
+          }
+          if (e + U < cnt) {
+            const int32_t u = __shfl_sync(mask, my_u, e + U, LANES);
+#pragma unroll
+            for (int n = 0; n < NV; ++n) {
+              if (valid[n]) ldv<VEC>(xl + (int64_t)u * p.ldx + n * LANES * VEC, v[q][n]);
+              if constexpr (MODE == M_GAT)
+                sc[q][n] = valid[n] ? __ldg(p.X + (int64_t)u * p.ldx + p.F + head[n]) : 0.0f;
+            }
+          }
         }
       }
     }
   }
-  __threadfence();
-  __syncwarp(mask);
-  int last = 0;
-  int32_t *cnt = p.ws_cnt + (size_t)m * p.nch + ci;
-  if (lane == 0) last = atomicAdd(cnt, 1) == ngrp - 1;
-  last = __shfl_sync(mask, last, 0, LANES);
-  if (!last) return;
-  __threadfence();
+}
+
+// merge the group partials of a long row in group order (R9), epilogue, store
+template <int MODE, int VEC, int NV, int LANES>
+__device__ __forceinline__ void merge_row(const KParams &p, const float *base, int32_t ngrp, int32_t row,
+                                          int32_t deg, int32_t c0, int lane) {
   Part<MODE, VEC, NV> A;
   part_init(A);
 #pragma unroll
   for (int n = 0; n < NV; ++n) {
     const int32_t f = c0 + (n * LANES + lane) * VEC;
     if (f >= p.F) continue;
-    if (atomic_acc) {
-      ldv_cg<VEC>(acc + f, A.a[n]);
-      continue;
-    }
     for (int32_t q = 0; q < ngrp; ++q) {
       float b[VEC];
       ldv_cg<VEC>(base + (size_t)q * p.FW + f, b);
@@ -512,49 +460,103 @@ __device__ __forceinline__ void multi_group_combine(const KParams &p, int32_t m,
       }
     }
   }
-  store_row<MODE, VEC, NV, LANES>(p, row, re - rb, c0, lane, A);
+  store_row<MODE, VEC, NV, LANES>(p, row, deg, c0, lane, A);
+}
+
+// one work unit = one neighbour group (NG: a group is the task of
+// one computing unit).  A row with a single group is finished here (epilogue +
+// store); the groups of a longer row leave their partials in the workspace and
+// the last one to arrive merges them in group order (R9).
+template <int MODE, int VEC, int NV, int LANES>
+__device__ __forceinline__ void process_unit(const KParams &p, int4 d, int32_t len, int32_t c0, int32_t ci, int lane,
+                                             unsigned mask) {
+  const DevGraph &g = p.g;
+  const int32_t tpos = d.x, beg = d.y, row = d.z, m = d.w;
+  Part<MODE, VEC, NV> G;
+  group_chain<MODE, VEC, NV, LANES>(p, g.colidx_t + tpos, len, beg, row, c0, lane, mask, G);
+  const int32_t rb = g.rowptr[row], re = g.rowptr[row + 1];
+  if (m < 0) {
+    store_row<MODE, VEC, NV, LANES>(p, row, re - rb, c0, lane, G);
+    return;
+  }
+  const int32_t ng = g.ng;
+  const int32_t ngrp = 1 + (re - rb - 1) / ng;
+  const int32_t k = (beg - rb) / ng;
+  const bool atomic_acc = !p.deterministic && MODE == M_SUM;
+  float *base = p.ws_part + (size_t)g.multi_slot[m] * p.FW;
+  float *acc = p.ws_acc + (size_t)m * p.FW;
+#pragma unroll
+  for (int n = 0; n < NV; ++n) {
+    const int32_t f = c0 + (n * LANES + lane) * VEC;
+    if (f >= p.F) continue;
+    if (atomic_acc) {
+#pragma unroll
+      for (int i = 0; i < VEC; ++i) atomicAdd(acc + f + i, G.a[n][i]);
+    } else {
+      stv<VEC>(base + (size_t)k * p.FW + f, G.a[n]);
+      if constexpr (MODE == M_GAT) {
+        if (f % p.Fh == 0) {
+          base[(size_t)k * p.FW + p.F + f / p.Fh] = G.m[n];
+          base[(size_t)k * p.FW + p.F + p.H + f / p.Fh] = G.l[n];
+        }
+      }
+    }
+  }
+  __threadfence();
+  __syncwarp(mask);
+  int32_t *cnt = p.ws_cnt + (size_t)m * p.nch + ci;
+  int last = 0;
+  if (lane == 0) last = atomicAdd(cnt, 1) == ngrp - 1;
+  last = __shfl_sync(mask, last, 0, LANES);
+  if (!last) return;
+  __threadfence();
+  if (atomic_acc) {
+    Part<MODE, VEC, NV> A;
+    part_init(A);
+#pragma unroll
+    for (int n = 0; n < NV; ++n) {
+      const int32_t f = c0 + (n * LANES + lane) * VEC;
+      if (f < p.F) ldv_cg<VEC>(acc + f, A.a[n]);
+    }
+    store_row<MODE, VEC, NV, LANES>(p, row, re - rb, c0, lane, A);
+  } else {
+    merge_row<MODE, VEC, NV, LANES>(p, base, ngrp, row, re - rb, c0, lane);
+  }
   if (lane == 0) *cnt = 0;  // leave the counter at 0 for the next call
 }
 
 #ifndef GNN_AGG_MINB
 #define GNN_AGG_MINB 4
 #endif
-// One CTA per tile of T consecutive groups in task order (a LAS cluster stays
-// on one SM); groups round-robin over the CTA's workers (NG load
-// balance).  No shared memory and no CTA barrier on the hot path.
 template <int MODE, int VEC, int NV, int LANES>
 __global__ void __launch_bounds__(256, MODE == M_GAT ? GNN_AGG_MINB - 1 : GNN_AGG_MINB) k_aggregate(const KParams p) {
   constexpr int CW = LANES * VEC * NV;
   const int tid = threadIdx.x;
   const int lane = tid & (LANES - 1);
-  const int wk = tid / LANES;
-  const int nwk = blockDim.x / LANES;
   const unsigned mask =
       LANES == 32 ? 0xffffffffu : (((1u << LANES) - 1u) << ((tid & 31) & ~(LANES - 1)));
   const DevGraph &g = p.g;
-  if ((int32_t)blockIdx.x >= g.n_tiles) {
+  if ((int32_t)blockIdx.x >= p.n_persist) {
     // zero-fill rows without in-edges (R3-i): 32 rows per block
-    const int64_t r0 = (int64_t)(blockIdx.x - g.n_tiles) * 32;
+    const int64_t r0 = (int64_t)(blockIdx.x - p.n_persist) * 32;
     for (int64_t r = r0; r < r0 + 32 && r < g.n_empty; ++r) {
       float *y = p.Y + (int64_t)g.empty_rows[r] * p.ldy;
       for (int f = tid; f < p.F; f += blockDim.x) y[f] = 0.0f;
     }
     return;
   }
-  const int32_t gb = (int32_t)blockIdx.x * g.T;
-  const int32_t ngr = min(g.T, g.n_groups - gb);
+  const int32_t nunits = g.n_units;
   int32_t ci = 0;
   for (int32_t c0 = 0; c0 < p.F; c0 += CW, ++ci) {
-    for (int32_t j = wk; j < ngr; j += nwk) {
-      const int32_t gi = gb + j;
-      const int32_t row = g.grp_row[gi], beg = g.grp_beg[gi];
-      const int32_t rb = g.rowptr[row], re = g.rowptr[row + 1];
-      const int32_t end = (re - beg > g.ng) ? beg + g.ng : re;
-      Part<MODE, VEC, NV> P;
-      row_chain<MODE, VEC, NV, LANES>(p, beg, end, row, c0, lane, mask, P);  // exactly one group
-      const int32_t m = g.grp_multi[gi];
-      if (m < 0) store_row<MODE, VEC, NV, LANES>(p, row, re - rb, c0, lane, P);
-      else multi_group_combine<MODE, VEC, NV, LANES>(p, m, row, rb, re, beg, c0, ci, lane, mask, P);
+    int32_t *ctr = p.ws_unit + ci;
+    for (;;) {
+      int32_t u = 0;
+      if (lane == 0) u = atomicAdd(ctr, 1);
+      u = __shfl_sync(mask, u, 0, LANES);
+      if (u >= nunits) break;
+      const int4 d = __ldg(g.unit_desc + u);
+      const int32_t len = __ldg(&g.unit_desc[u + 1].x) - d.x;
+      process_unit<MODE, VEC, NV, LANES>(p, d, len, c0, ci, lane, mask);
     }
   }
 }
@@ -597,62 +599,74 @@ static Mapping choose_mapping(const AggArgs &a, int32_t fh_or_0) {
 
 static int32_t max_chunks(int32_t F) { return F <= 128 ? 1 : (F + 31) / 32; }
 
+// layout: [unit counters (256 B)][row counters n_multi x nch | pad 256][acc n_multi x FW][slots x FW]
 size_t agg_workspace_bytes(const gnn_plan_s *p, int mode, int32_t F, int32_t H) {
-  if (p->n_multi == 0) return 0;
   const size_t FW = (size_t)F + (mode == M_GAT ? 2 * (size_t)H : 0);
-  size_t b = sizeof(int32_t) * (size_t)p->n_multi * max_chunks(F);
-  b = (b + 255) & ~(size_t)255;
+  size_t b = 256;
+  size_t c = sizeof(int32_t) * (size_t)p->n_multi * max_chunks(F);
+  b += (c + 255) & ~(size_t)255;
   return b + sizeof(float) * ((size_t)p->multi_slots + (size_t)p->n_multi) * FW;
 }
 
+static int num_sms() {
+  static int n = 0;
+  if (n == 0) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    if (n <= 0) n = 148;
+  }
+  return n;
+}
+
 template <int MODE, int VEC, int NV, int LANES>
-static cudaError_t launch_one(const KParams &kp_in, int threads, size_t smem, int64_t blocks, cudaStream_t s) {
+static cudaError_t launch_one(const KParams &kp_in, int threads, cudaStream_t s) {
   auto fn = k_aggregate<MODE, VEC, NV, LANES>;
-  static bool configured = false;  // per instantiation
-  if (!configured) {
-    // no shared memory on the hot path: the unified array goes to L1, which
-    // serves the source rows a LAS cluster (one tile, one SM) shares
-    cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, 0);
-    configured = true;
+  static int occ = 0;  // resident CTAs per SM for this instantiation
+  if (occ == 0) {
+    cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, 0);  // all of it to L1
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, threads, 0);
+    if (occ <= 0) occ = 1;
   }
   KParams kp = kp_in;
   constexpr int CW = LANES * VEC * NV;
   kp.nch = (kp.F + CW - 1) / CW;
-  if (kp.g.n_multi > 0) {
-    cudaError_t e = cudaMemsetAsync(kp.ws_cnt, 0, sizeof(int32_t) * (size_t)kp.g.n_multi * kp.nch, s);
-    if (e == cudaSuccess && !kp.deterministic && MODE == M_SUM)
-      e = cudaMemsetAsync(kp.ws_acc, 0, sizeof(float) * (size_t)kp.g.n_multi * kp.FW, s);
-    if (e != cudaSuccess) return e;
-  }
-  if (blocks == 0) return cudaSuccess;
-  fn<<<(unsigned)blocks, threads, smem, s>>>(kp);
+  const int64_t workers_per_cta = threads / LANES;
+  kp.n_persist = (int32_t)std::min<int64_t>((int64_t)num_sms() * occ,
+                                            std::max<int64_t>(1, (kp.g.n_units + workers_per_cta - 1) / workers_per_cta));
+  cudaError_t e = cudaMemsetAsync(kp.ws_unit, 0, 256, s);
+  if (e == cudaSuccess && kp.g.n_multi > 0)
+    e = cudaMemsetAsync(kp.ws_cnt, 0, sizeof(int32_t) * (size_t)kp.g.n_multi * kp.nch, s);
+  if (e == cudaSuccess && kp.g.n_multi > 0 && !kp.deterministic && MODE == M_SUM)
+    e = cudaMemsetAsync(kp.ws_acc, 0, sizeof(float) * (size_t)kp.g.n_multi * kp.FW, s);
+  if (e != cudaSuccess) return e;
+  const int64_t blocks = (int64_t)kp.n_persist + (kp.g.n_empty + 31) / 32;
+  fn<<<(unsigned)blocks, threads, 0, s>>>(kp);
   count_launch();
   return cudaGetLastError();
 }
 
 template <int MODE, int VEC>
-static cudaError_t dispatch_lanes(const KParams &kp, const Mapping &m, int threads, size_t smem, int64_t blocks,
-                                  cudaStream_t s) {
+static cudaError_t dispatch_lanes(const KParams &kp, const Mapping &m, int threads, cudaStream_t s) {
   switch (m.lanes) {
-    case 4: return launch_one<MODE, VEC, 1, 4>(kp, threads, smem, blocks, s);
-    case 8: return launch_one<MODE, VEC, 1, 8>(kp, threads, smem, blocks, s);
-    case 16: return launch_one<MODE, VEC, 1, 16>(kp, threads, smem, blocks, s);
+    case 4: return launch_one<MODE, VEC, 1, 4>(kp, threads, s);
+    case 8: return launch_one<MODE, VEC, 1, 8>(kp, threads, s);
+    case 16: return launch_one<MODE, VEC, 1, 16>(kp, threads, s);
     default:
-      if (m.nv == 1) return launch_one<MODE, VEC, 1, 32>(kp, threads, smem, blocks, s);
-      if (m.nv == 2) return launch_one<MODE, VEC, 2, 32>(kp, threads, smem, blocks, s);
-      if constexpr (VEC < 8) return launch_one<MODE, VEC, 4, 32>(kp, threads, smem, blocks, s);
+      if (m.nv == 1) return launch_one<MODE, VEC, 1, 32>(kp, threads, s);
+      if (m.nv == 2) return launch_one<MODE, VEC, 2, 32>(kp, threads, s);
+      if constexpr (VEC < 8) return launch_one<MODE, VEC, 4, 32>(kp, threads, s);
       return cudaErrorInvalidValue;
   }
 }
 
 template <int MODE>
-static cudaError_t dispatch_vec(const KParams &kp, const Mapping &m, int threads, size_t smem, int64_t blocks,
-                                cudaStream_t s) {
+static cudaError_t dispatch_vec(const KParams &kp, const Mapping &m, int threads, cudaStream_t s) {
   switch (m.vec) {
-    case 8: return dispatch_lanes<MODE, 8>(kp, m, threads, smem, blocks, s);
-    case 4: return dispatch_lanes<MODE, 4>(kp, m, threads, smem, blocks, s);
-    case 2: return dispatch_lanes<MODE, 2>(kp, m, threads, smem, blocks, s);
-    default: return dispatch_lanes<MODE, 1>(kp, m, threads, smem, blocks, s);
+    case 8: return dispatch_lanes<MODE, 8>(kp, m, threads, s);
+    case 4: return dispatch_lanes<MODE, 4>(kp, m, threads, s);
+    case 2: return dispatch_lanes<MODE, 2>(kp, m, threads, s);
+    default: return dispatch_lanes<MODE, 1>(kp, m, threads, s);
   }
 }
 
@@ -660,7 +674,7 @@ gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, siz
   if (a.F <= 0) return GNN_OK;
   const int mode = a.mode;
   const size_t need = agg_workspace_bytes(p, mode, a.F, a.H);
-  if (p->n_multi > 0 && (ws == nullptr || ws_bytes < need)) {
+  if (ws == nullptr || ws_bytes < need) {
     set_error("workspace too small: need " + std::to_string(need) + " bytes");
     return GNN_ERR_WORKSPACE;
   }
@@ -684,23 +698,20 @@ gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, siz
   kp.slope = a.slope;
   kp.FW = a.F + (mode == M_GAT ? 2 * a.H : 0);
   kp.deterministic = a.deterministic;
-  if (p->n_multi > 0) {
-    // layout: [counters n_multi x nch int32 | pad to 256 B][accumulators n_multi x FW][slots x FW]
-    const size_t cnt_bytes = (sizeof(int32_t) * (size_t)p->n_multi * max_chunks(a.F) + 255) & ~(size_t)255;
-    kp.ws_cnt = reinterpret_cast<int32_t *>(ws);
-    kp.ws_acc = reinterpret_cast<float *>(reinterpret_cast<char *>(ws) + cnt_bytes);
-    kp.ws_part = kp.ws_acc + (size_t)p->n_multi * kp.FW;
-  }
+  char *w = reinterpret_cast<char *>(ws);
+  kp.ws_unit = reinterpret_cast<int32_t *>(w);
+  const size_t cnt_bytes = (sizeof(int32_t) * (size_t)p->n_multi * max_chunks(a.F) + 255) & ~(size_t)255;
+  kp.ws_cnt = reinterpret_cast<int32_t *>(w + 256);
+  kp.ws_acc = reinterpret_cast<float *>(w + 256 + cnt_bytes);
+  kp.ws_part = kp.ws_acc + (size_t)p->n_multi * kp.FW;
   const Mapping m = choose_mapping(a, mode == M_GAT ? a.Fh : 0);
-  const int threads = std::min(256, std::max(32, p->T * m.lanes));
-  const size_t smem = 0;
-  const int64_t blocks = (int64_t)p->dg.n_tiles + (p->dg.n_empty + 31) / 32;
+  const int threads = 256;
   cudaError_t e;
   switch (mode) {
     case M_SUM:
-    case M_MEAN: e = dispatch_vec<M_SUM>(kp, m, threads, smem, blocks, s); break;
-    case M_MAX: e = dispatch_vec<M_MAX>(kp, m, threads, smem, blocks, s); break;
-    default: e = dispatch_vec<M_GAT>(kp, m, threads, smem, blocks, s); break;
+    case M_MEAN: e = dispatch_vec<M_SUM>(kp, m, threads, s); break;
+    case M_MAX: e = dispatch_vec<M_MAX>(kp, m, threads, s); break;
+    default: e = dispatch_vec<M_GAT>(kp, m, threads, s); break;
   }
   return cuda_status(e, "aggregate launch");
 }

@@ -6,6 +6,7 @@
 // This is an independent implementation of the same integer specification
 // the oracle follows (R7/R8): results must be bit-identical.
 #include <algorithm>
+#include <cstring>
 #include <chrono>
 #include <cstring>
 #include <queue>
@@ -232,79 +233,83 @@ int64_t las_merge(int64_t n, const uint64_t *sig, int32_t K, const std::vector<i
   return nc;
 }
 
-// a3: neighbor groups in task order (reading R8).  CTA tile t is
-// groups [t*T, (t+1)*T).  A row with more than one group ("multi-group") gets
-// workspace slots for its group partials, merged in group order by the last
-// worker to finish one of them (R9).  Pure host function (gnn_groups_host).
+// a3: neighbor groups in task order (reading R8).  Pure host
+// function (also gnn_groups_host).
 void schedule_host(int64_t n, const int64_t *rowptr, const int32_t *perm, int64_t ng,
-                   std::vector<int32_t> &grp_row, std::vector<int64_t> &grp_beg, std::vector<int32_t> &grp_multi,
-                   std::vector<int32_t> &multi_slot, int64_t &slots) {
+                   std::vector<int32_t> &grp_row, std::vector<int64_t> &grp_beg) {
   grp_row.clear();
   grp_beg.clear();
-  grp_multi.clear();
-  multi_slot.clear();
-  slots = 0;
   for (int64_t i = 0; i < n; ++i) {
     const int64_t v = perm ? perm[i] : i;
     const int64_t beg = rowptr[v], end = rowptr[v + 1];
-    if (end == beg) continue;
-    const bool multi = end - beg > ng;
-    const int32_t m = multi ? (int32_t)multi_slot.size() : -1;
-    if (multi) multi_slot.push_back((int32_t)slots);
     for (int64_t b = beg; b < end; b += ng) {
       grp_row.push_back((int32_t)v);
       grp_beg.push_back(b);
-      grp_multi.push_back(m);
-      if (multi) ++slots;
       if (end - b <= ng) break;
     }
   }
 }
 
+// Work units in task order = neighbour groups: a row with one
+// group is one unit; the groups of a longer row are separate units whose
+// partials meet in the workspace.  Source indices are re-laid out in task order
+// (colidx_t) so every unit reads one contiguous stream.
 gnn_status build_schedule(gnn_plan_s *p) {
-  const int64_t n = p->n;
-  std::vector<int32_t> grp_multi, multi_slot;
-  int64_t slots = 0;
-  schedule_host(n, p->rowptr.data(), p->perm.data(), p->ng, p->grp_row, p->grp_beg, grp_multi, multi_slot, slots);
-  const int64_t G = (int64_t)p->grp_row.size();
-  const int64_t n_tiles = (G + p->T - 1) / p->T;
-  p->n_multi = (int64_t)multi_slot.size();
-  p->multi_slots = slots;
-  std::vector<int32_t> empty;
+  const int64_t n = p->n, ng = p->ng;
+  schedule_host(n, p->rowptr.data(), p->perm.data(), ng, p->grp_row, p->grp_beg);
+  std::vector<int32_t> desc, colidx_t((size_t)p->nnz + 16, 0), multi_slot, multi_units, empty;
+  desc.reserve((size_t)p->grp_row.size() * 4 + 4);
+  int64_t tpos = 0, slots = 0;
+  for (int64_t i = 0; i < n; ++i) {
+    const int64_t v = p->perm[i];
+    const int64_t rb = p->rowptr[v], re = p->rowptr[v + 1];
+    if (re == rb) continue;
+    std::memcpy(colidx_t.data() + tpos, p->colidx_h + rb, sizeof(int32_t) * (size_t)(re - rb));
+    const int64_t ngrp = (re - rb + ng - 1) / ng;
+    int32_t m = -1;
+    if (ngrp > 1) {
+      m = (int32_t)multi_slot.size();
+      multi_slot.push_back((int32_t)slots);
+      multi_units.push_back((int32_t)ngrp);
+      slots += ngrp;
+    }
+    for (int64_t b = rb; b < re; b += ng) desc.insert(desc.end(), {(int32_t)(tpos + (b - rb)), (int32_t)b, (int32_t)v, m});
+    tpos += re - rb;
+  }
+  const int64_t n_units = (int64_t)desc.size() / 4;
+  desc.insert(desc.end(), {(int32_t)tpos, 0, 0, -1});
   for (int64_t v = 0; v < n; ++v)
     if (p->rowptr[v + 1] == p->rowptr[v]) empty.push_back((int32_t)v);
+  p->n_multi = (int64_t)multi_slot.size();
+  p->multi_slots = slots;
   p->n_empty = (int64_t)empty.size();
 
   auto upload = [&](const void *src, size_t bytes, void **dst) -> cudaError_t {
     *dst = nullptr;
-    cudaError_t e = cudaMalloc(dst, bytes > 0 ? bytes : 4);
+    cudaError_t e = cudaMalloc(dst, bytes > 0 ? bytes : 16);
     if (e != cudaSuccess) return e;
     p->dev_allocs.push_back(*dst);
     if (bytes > 0) e = cudaMemcpy(*dst, src, bytes, cudaMemcpyHostToDevice);
     return e;
   };
-  std::vector<int32_t> grp_beg32((size_t)G);
-  for (int64_t i = 0; i < G; ++i) grp_beg32[i] = (int32_t)p->grp_beg[i];
   void *d;
   cudaError_t e;
 #define UP(vec, field)                                                                 \
   e = upload((vec).data(), sizeof(int32_t) * (vec).size(), &d);                       \
   if (e != cudaSuccess) return cuda_status(e, "plan upload");                         \
-  p->dg.field = reinterpret_cast<const int32_t *>(d);
-  UP(p->grp_row, grp_row)
-  UP(grp_beg32, grp_beg)
-  UP(grp_multi, grp_multi)
+  p->dg.field = reinterpret_cast<decltype(p->dg.field)>(d);
+  UP(desc, unit_desc)
+  UP(colidx_t, colidx_t)
   UP(multi_slot, multi_slot)
+  UP(multi_units, multi_units)
   UP(empty, empty_rows)
 #undef UP
-  p->dg.n_groups = (int32_t)G;
-  p->dg.n_tiles = (int32_t)n_tiles;
-  p->dg.T = p->T;
+  p->dg.n_units = (int32_t)n_units;
   p->dg.n_multi = (int32_t)p->n_multi;
   p->dg.n_empty = (int32_t)p->n_empty;
-  p->dg.ng = p->ng;
-  p->info.n_groups = G;
-  p->info.n_tiles = n_tiles;
+  p->dg.ng = (int32_t)ng;
+  p->info.n_groups = (int64_t)p->grp_row.size();
+  p->info.n_tiles = n_units;
   p->info.n_split_rows = p->n_multi;
   p->info.n_empty_rows = p->n_empty;
   return GNN_OK;
