@@ -40,6 +40,8 @@ def _load():
         lib.synth_powerlaw.argtypes = [ctypes.c_int64, ctypes.c_int64, ctypes.c_double, ctypes.c_double,
                                        ctypes.c_int64, ctypes.c_int64, ctypes.c_double, ctypes.c_uint64,
                                        ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]
+        lib.synth_powerlaw_ex.restype = ctypes.c_int
+        lib.synth_powerlaw_ex.argtypes = lib.synth_powerlaw.argtypes + [ctypes.c_void_p]
         lib.synth_uniform_f32.restype = None
         lib.synth_uniform_f32.argtypes = [ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_float,
                                           ctypes.c_float, ctypes.c_uint64, ctypes.c_void_p]
@@ -60,16 +62,22 @@ class Graph:
         return int(self.rowptr[-1])
 
 
-def powerlaw(n, nnz, mean, var, cap, comm=32, rho=0.8, seed=1) -> Graph:
+def powerlaw(n, nnz, mean, var, cap, comm=32, rho=0.8, seed=1, with_relabel=False) -> Graph:
+    """GEN-PL graph.  with_relabel=True also returns (in stats["relabel"]) the
+    relabel permutation (new id of pre-relabel node v), for locality studies."""
     lib = _load()
     rowptr = np.empty(n + 1, dtype=np.int64)
     colidx = np.empty(max(nnz, 1), dtype=np.int32)
     st = np.zeros(4, dtype=np.int64)
-    rc = lib.synth_powerlaw(n, nnz, float(mean), float(var), cap, comm, float(rho), seed,
-                            rowptr.ctypes.data, colidx.ctypes.data, st.ctypes.data)
+    rel = np.empty(n, dtype=np.int64) if with_relabel else None
+    rc = lib.synth_powerlaw_ex(n, nnz, float(mean), float(var), cap, comm, float(rho), seed,
+                               rowptr.ctypes.data, colidx.ctypes.data, st.ctypes.data,
+                               None if rel is None else rel.ctypes.data)
     if rc != 0:
         raise RuntimeError(f"synth_powerlaw failed rc={rc}")
     stats = {"max": int(st[0]), "mean": st[1] / 1e6, "var": st[2] / 1e3, "zero_rows": int(st[3])}
+    if rel is not None:
+        stats["relabel"] = rel
     return Graph(n, rowptr, colidx[:nnz], stats)
 
 
@@ -155,11 +163,12 @@ def seed_of(cfg: str, what: int) -> int:
     return 20210227 + 10 * int(cfg[1]) + what
 
 
-def config_graph(cfg: str, rho: float = 0.8, scale: float = 1.0) -> Graph:
+def config_graph(cfg: str, rho: float = 0.8, scale: float = 1.0, with_relabel: bool = False) -> Graph:
     c = CONFIGS[cfg]
     if cfg == "C4":
         return knn_clouds(c["batch"], c["points"], c["k"], seed=seed_of(cfg, 0))
     n = max(64, int(c["n"] * scale))
     nnz = max(n, int(c["nnz"] * scale))
     cap = min(c["cap"], n - 1)
-    return powerlaw(n, nnz, c["mean"], c["var"], cap, c["comm"], rho, seed_of(cfg, 0) + int(rho * 100))
+    return powerlaw(n, nnz, c["mean"], c["var"], cap, c["comm"], rho, seed_of(cfg, 0) + int(rho * 100),
+                    with_relabel=with_relabel)

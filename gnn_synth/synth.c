@@ -120,9 +120,9 @@ static int64_t sort_unique_i64(int64_t *v, int64_t k) {
  * Returns 0 on success.  rowptr[n+1] and colidx[nnz] are caller-allocated.
  * stats (may be NULL) receives {max_deg, mean*1e6, var*1e3, zero_rows}.
  */
-int synth_powerlaw(int64_t n, int64_t nnz, double mean, double var, int64_t cap,
-                   int64_t comm, double rho, uint64_t seed, int64_t *rowptr,
-                   int32_t *colidx, int64_t *stats) {
+int synth_powerlaw_ex(int64_t n, int64_t nnz, double mean, double var, int64_t cap,
+                      int64_t comm, double rho, uint64_t seed, int64_t *rowptr,
+                      int32_t *colidx, int64_t *stats, int64_t *relabel_out) {
   if (n <= 1 || nnz < 0 || cap < 1) return -1;
   if (cap > n - 1) cap = n - 1;
   if (nnz > n * cap) return -2;
@@ -280,10 +280,17 @@ int synth_powerlaw(int64_t n, int64_t nnz, double mean, double var, int64_t cap,
     stats[2] = (int64_t)llround(m2 / n * 1e3);
     stats[3] = zeros;
   }
+  if (relabel_out) memcpy(relabel_out, perm, sizeof(int64_t) * (size_t)n);
   free(row); free(tcopy); free(perm); free(tpl); free(tpl_off);
   alias_free(&al);
   free(w); free(deg);
   return 0;
+}
+
+int synth_powerlaw(int64_t n, int64_t nnz, double mean, double var, int64_t cap,
+                   int64_t comm, double rho, uint64_t seed, int64_t *rowptr,
+                   int32_t *colidx, int64_t *stats) {
+  return synth_powerlaw_ex(n, nnz, mean, var, cap, comm, rho, seed, rowptr, colidx, stats, NULL);
 }
 
 /* uniform fp32 features in [lo, hi) with row stride ld (pad columns = 0) */

@@ -549,14 +549,30 @@ __global__ void __launch_bounds__(256, MODE == M_GAT ? GNN_AGG_MINB - 1 : GNN_AG
   int32_t ci = 0;
   for (int32_t c0 = 0; c0 < p.F; c0 += CW, ++ci) {
     int32_t *ctr = p.ws_unit + ci;
-    for (;;) {
-      int32_t u = 0;
-      if (lane == 0) u = atomicAdd(ctr, 1);
-      u = __shfl_sync(mask, u, 0, LANES);
-      if (u >= nunits) break;
-      const int4 d = __ldg(g.unit_desc + u);
-      const int32_t len = __ldg(&g.unit_desc[u + 1].x) - d.x;
-      process_unit<MODE, VEC, NV, LANES>(p, d, len, c0, ci, lane, mask);
+    // the next unit (id and descriptor) is claimed while the current one streams
+    int32_t u = 0;
+    if (lane == 0) u = atomicAdd(ctr, 1);
+    u = __shfl_sync(mask, u, 0, LANES);
+    int4 d = make_int4(0, 0, 0, -1);
+    int32_t dnx = 0;
+    if (u < nunits) {
+      d = __ldg(g.unit_desc + u);
+      dnx = __ldg(&g.unit_desc[u + 1].x);
+    }
+    while (u < nunits) {
+      int32_t un = 0;
+      if (lane == 0) un = atomicAdd(ctr, 1);
+      un = __shfl_sync(mask, un, 0, LANES);
+      int4 dn = make_int4(0, 0, 0, -1);
+      int32_t dnxn = 0;
+      if (un < nunits) {
+        dn = __ldg(g.unit_desc + un);
+        dnxn = __ldg(&g.unit_desc[un + 1].x);
+      }
+      process_unit<MODE, VEC, NV, LANES>(p, d, dnx - d.x, c0, ci, lane, mask);
+      u = un;
+      d = dn;
+      dnx = dnxn;
     }
   }
 }
