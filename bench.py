@@ -229,32 +229,28 @@ def run_ours(args):
                 "algorithmic_bytes": int(per_launch[dom_name]), "launch_ms": round(float(parts[dom]), 4),
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)" if "hbm_gbs" in peaks else "fallback 6650"}
 
-    # e2e: same step through the public API with host buffers, copies inside the timed region
+    # e2e: the same steps through the public API from pinned host input to
+    # pinned host output, the copies inside the timed region (pipelined over
+    # the host links: input of step k+1 and output of step k overlap compute)
     e2e = None
     if not args.no_e2e:
         Xh = torch.from_numpy(inp["X"]).pin_memory()
         Yh = torch.empty((rows, HF), dtype=torch.float32).pin_memory()
         h2d = Xh.numel() * 4
         d2h = Yh.numel() * 4
-        for _ in range(2):
-            model.load_input(Xh)
-            Yh.copy_(model.step(), non_blocking=True)
+        s0, s1 = model.run_pipelined(Xh, Yh, 2)
         torch.cuda.synchronize(dev)
-        e_s = torch.cuda.Event(enable_timing=True)
-        e_e = torch.cuda.Event(enable_timing=True)
-        ke = max(1, min(args.steps, 5))
-        e_s.record(stream)
-        for _ in range(ke):
-            model.load_input(Xh)
-            Yh.copy_(model.step(), non_blocking=True)
-        e_e.record(stream)
+        ke = max(2, min(args.steps, 5))
+        e_s, e_e = model.run_pipelined(Xh, Yh, ke)
         torch.cuda.synchronize(dev)
         me = torch.tensor([e_s.elapsed_time(e_e) / ke], device=dev)
         if world > 1:
             dist.all_reduce(me, op=dist.ReduceOp.MAX)
         e2e = {"value": round(edge_feats / (float(me.item()) * 1e-3) / 1e9, 3), "unit": UNIT,
                "ms_per_step": round(float(me.item()), 3), "h2d_bytes_per_step": int(h2d),
-               "d2h_bytes_per_step": int(d2h)}
+               "d2h_bytes_per_step": int(d2h), "steps": ke,
+               "note": "pinned host X -> device, step, device -> pinned host Y3 every step; copies of "
+                       "step k+1 / k overlap compute on separate streams"}
 
     out = {
         "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": world, "steps": args.steps,

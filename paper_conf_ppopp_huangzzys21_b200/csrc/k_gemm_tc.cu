@@ -162,7 +162,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p) {
 
   if (tid == 0) {
     for (int s = 0; s < S; ++s) {
-      mbar_init(&full_bar[s], NUM_PRODUCER_WARPS * 32 + 1);  // 128 A arrivals + 1 expect_tx for W
+      mbar_init(&full_bar[s], NUM_PRODUCER_WARPS * 32 / 2 + 1);  // 64 A arrivals (one group) + 1 expect_tx
       mbar_init(&empty_bar[s], 1);
     }
     for (int b = 0; b < 2; ++b) {
@@ -182,16 +182,20 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p) {
 
   if (warp < NUM_PRODUCER_WARPS) {
     // ------------------------------ producers ------------------------------
-    // The X tile of the NEXT K block is loaded into registers before waiting
-    // for the current stage to free up, so global-memory latency overlaps the
-    // MMAs of earlier stages (one K block of register look-ahead).
-    constexpr int PER_THREAD = BM * 8 / (NUM_PRODUCER_WARPS * 32);  // float4 chunks per thread per K block
-    float4 buf[2][PER_THREAD];
-    auto load_a = [&](float4 (&dst)[PER_THREAD], int64_t m0, int kb) {
+    // Two producer groups of 2 warps take alternate K blocks (group g handles
+    // the global K-block counter it = g, g+2, ...); each group loads its next
+    // X tile into registers before waiting for its stage, so two K blocks of
+    // X are in flight per CTA while the MMAs run.
+    constexpr int GROUP_THREADS = NUM_PRODUCER_WARPS * 32 / 2;           // 64
+    constexpr int PER_THREAD = BM * 8 / GROUP_THREADS;                     // 16 float4 chunks
+    const int grp = warp >> 1;                                             // 0 or 1
+    const int gtid = tid - grp * GROUP_THREADS;
+    float4 buf[PER_THREAD];
+    auto load_a = [&](int64_t m0, int kb) {
       const int k0 = kb * BK;
 #pragma unroll
       for (int i = 0; i < PER_THREAD; ++i) {
-        const int q = tid + i * NUM_PRODUCER_WARPS * 32;
+        const int q = gtid + i * GROUP_THREADS;
         const int r = q >> 3, c = q & 7;
         const int64_t gm = m0 + r;
         const int gk = k0 + 4 * c;
@@ -207,30 +211,21 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p) {
             if (gk + 3 < p.k) x.w = __ldg(src + 3);
           }
         }
-        dst[i] = x;
+        buf[i] = x;
       }
     };
-    int it = 0;  // global K-block counter across tiles (stage/phase tracking)
-    int tile = blockIdx.x;
-    int kb = 0;
-    if (tile < p.num_tiles) load_a(buf[0], (int64_t)tile * BM, 0);
-    while (tile < p.num_tiles) {
-      // next (tile, kb) to prefetch
-      int ntile = tile, nkb = kb + 1;
-      if (nkb == p.num_kb) {
-        nkb = 0;
-        ntile += gridDim.x;
-      }
-      const int cur = it & 1;
-      if (ntile < p.num_tiles) {
-        if (cur == 0) load_a(buf[1], (int64_t)ntile * BM, nkb);
-        else load_a(buf[0], (int64_t)ntile * BM, nkb);
-      }
+    const int my_tiles = p.num_tiles > (int)blockIdx.x ? (p.num_tiles - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0;
+    const int total_it = my_tiles * p.num_kb;
+    auto tile_of = [&](int it) { return (int)blockIdx.x + (it / p.num_kb) * (int)gridDim.x; };
+    int it = grp;
+    if (it < total_it) load_a((int64_t)tile_of(it) * BM, it % p.num_kb);
+    while (it < total_it) {
+      const int kb = it % p.num_kb;
       const int s = it % S, use = it / S;
       if (use > 0) mbar_wait(&empty_bar[s], (use - 1) & 1);
       uint8_t *st = smem + (size_t)s * STAGE_BYTES;
       uint8_t *a_hi = st, *a_lo = st + TILE_A_BYTES, *b_img = st + 2 * TILE_A_BYTES;
-      if (tid == 0) {
+      if (gtid == 0) {
         mbar_arrive_expect_tx(&full_bar[s], 2 * B_BYTES);
         const uint8_t *src = p.wimg + (size_t)kb * 2 * B_BYTES;
         for (int off = 0; off < 2 * B_BYTES; off += 16384) {
@@ -240,9 +235,9 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p) {
       }
 #pragma unroll
       for (int i = 0; i < PER_THREAD; ++i) {
-        const int q = tid + i * NUM_PRODUCER_WARPS * 32;
+        const int q = gtid + i * GROUP_THREADS;
         const int r = q >> 3, c = q & 7;
-        const float4 x = cur == 0 ? buf[0][i] : buf[1][i];
+        const float4 x = buf[i];
         const float4 hi = make_float4(hi_of(x.x), hi_of(x.y), hi_of(x.z), hi_of(x.w));
         const float4 lo = make_float4(x.x - hi.x, x.y - hi.y, x.z - hi.z, x.w - hi.w);
         const uint32_t off = sw128_off(r, c);
@@ -252,9 +247,8 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p) {
       // generic-proxy smem writes -> visible to the tensor core (async proxy)
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       mbar_arrive(&full_bar[s]);
-      ++it;
-      tile = ntile;
-      kb = nkb;
+      it += 2;
+      if (it < total_it) load_a((int64_t)tile_of(it) * BM, it % p.num_kb);
     }
   } else if (warp == MMA_WARP) {
     // ------------------------------ MMA issuer ------------------------------

@@ -358,17 +358,28 @@ __device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx
       tv[n] = valid[n] ? __ldg(p.t + (int64_t)row * p.ldt + head[n]) : 0.0f;
     }
   }
-  for (int32_t k = 0; k < len; k += LANES) {
-    const int32_t cnt = min(LANES, len - k);
-    int32_t my_u = 0;
-    float my_w = 1.0f;
-    if (lane < cnt) {
-      my_u = ld_stream_i32(idx + k + lane);
+  // index batches: the next batch (and its weights) is requested before the
+  // current one is consumed
+  auto load_batch = [&](int32_t k, int32_t &u, float &w) {
+    const int32_t c = min(LANES, len - k);
+    u = 0;
+    w = 1.0f;
+    if (lane < c) {
+      u = ld_stream_i32(idx + k + lane);
       if constexpr (MODE != M_GAT) {
-        if (weight == GNN_W_GCN) my_w = __ldg(p.g.nsrc + my_u);
-        else if (weight == GNN_W_EDGE) my_w = ld_stream_f32(p.edge_w + beg + k + lane);
+        if (weight == GNN_W_GCN) w = __ldg(p.g.nsrc + u);
+        else if (weight == GNN_W_EDGE) w = ld_stream_f32(p.edge_w + beg + k + lane);
       }
     }
+  };
+  int32_t nx_u = 0;
+  float nx_w = 1.0f;
+  if (len > 0) load_batch(0, nx_u, nx_w);
+  for (int32_t k = 0; k < len; k += LANES) {
+    const int32_t cnt = min(LANES, len - k);
+    const int32_t my_u = nx_u;
+    const float my_w = nx_w;
+    if (k + LANES < len) load_batch(k + LANES, nx_u, nx_w);
     float v[U][NV][VEC];
     float sc[U][NV];
 #pragma unroll
@@ -388,6 +399,7 @@ __device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx
         const int32_t e = j + q;
         if (e < cnt) {
           if constexpr (MODE == M_GAT) {
+            // online softmax (R9 GAT): one exp per edge and head
 #pragma unroll
             for (int n = 0; n < NV; ++n) {
               if (!valid[n]) continue;

@@ -73,6 +73,54 @@ class RowPartitionedGCNGAT:
         self.ws_gemm = torch.empty(max(gw, 256), dtype=torch.uint8, device=d)
         self.ws_gemm_b = gw
 
+    # -- end to end over a stream of inputs ---------------------------------
+    def run_pipelined(self, X_host, Y_host, steps, stream=None):
+        """`steps` forward passes from pinned host input to pinned host output.
+
+        Three streams overlap the host links with compute: the input of step
+        k+1 is uploaded once step k's layer-1 aggregation has consumed the
+        previous input, and the output of step k is downloaded while step k+1
+        computes (the GAT output alternates between two device buffers).
+        Returns the device-side events (start, end) bracketing the whole run.
+        """
+        dev = self.dev
+        comp = torch.cuda.current_stream(dev) if stream is None else stream
+        cin = torch.cuda.Stream(device=dev)
+        cout = torch.cuda.Stream(device=dev)
+        if not hasattr(self, "Y3b"):
+            self.Y3b = [self.Y3, torch.empty_like(self.Y3)]
+        E = lambda: torch.cuda.Event()  # noqa: E731
+        start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        start.record(comp)
+        cin.wait_event(start)
+        cout.wait_event(start)
+        consumed = None  # layer 1 of the previous step has read Xs
+        downloaded = [None, None]
+        for k in range(steps):
+            with torch.cuda.stream(cin):
+                if consumed is not None:
+                    cin.wait_event(consumed)
+                self.load_input(X_host, non_blocking=True)
+                up = E()
+                up.record(cin)
+            comp.wait_event(up)
+            b = k % 2
+            if downloaded[b] is not None:
+                comp.wait_event(downloaded[b])
+            self.Y3 = self.Y3b[b]
+            evs = [E() for _ in range(7)]
+            self.step(stream=comp, events=evs)
+            consumed = evs[1]
+            with torch.cuda.stream(cout):
+                cout.wait_event(evs[6])
+                Y_host.copy_(self.Y3b[b], non_blocking=True)
+                dl = E()
+                dl.record(cout)
+                downloaded[b] = dl
+        comp.wait_stream(cout)
+        end.record(comp)
+        return start, end
+
     # -- inputs -------------------------------------------------------------
     def load_input(self, X_host_or_dev, non_blocking=True):
         """X [n, F_in] (host pinned or device) -> the replicated padded buffer."""
