@@ -243,6 +243,21 @@ size_t gnn_gemm_workspace_size(int64_t m, int32_t k, int32_t n);
 int gnn_set_gemm_impl(int impl);
 
 /*
+ * a4 mapping override (process-wide; the hook of the paper's mapping tuner,
+ * P:1128-1168): every later graph op whose F, strides and pointers
+ * admit it uses vec floats per lane-vector (1, 2, 4 or 8), `lanes` lanes per
+ * worker (4, 8, 16 or 32) and nv vectors per lane (1, 2 or 4; nv > 1 needs
+ * lanes == 32; vec 8 allows nv <= 2).  The feature chunk lanes*vec*nv bounds
+ * the width of H one sweep over the schedule gathers (wider rows take several
+ * sweeps).  An op whose shapes do not admit the override uses the automatic
+ * rule.  vec = lanes = nv = 0 restores the automatic rule.
+ * Returns GNN_ERR_INVALID_ARG for an unsupported combination.  Results are
+ * unchanged bit for bit in the deterministic variant (the chain of R9 is per
+ * feature and does not depend on the mapping).
+ */
+gnn_status gnn_set_agg_mapping(int32_t vec, int32_t lanes, int32_t nv);
+
+/*
  * GCN layer (Eq 1): Y = ACT((A_gcn X) W).  order: 0 = auto (aggregate at
  * min(f_in, f_out)), 1 = transform first (H = X W scaled by nsrc, aggregate,
  * x ndst), 2 = aggregate first.  Workspace: gnn_workspace_size(plan,

@@ -416,6 +416,16 @@ gnn_status gnn_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw, fl
 
 int gnn_set_gemm_impl(int impl) { return set_gemm_impl(impl); }
 
+gnn_status gnn_set_agg_mapping(int32_t vec, int32_t lanes, int32_t nv) {
+  GNN_TRY({
+    if (!set_agg_mapping(vec, lanes, nv)) {
+      set_error("gnn_set_agg_mapping: unsupported (vec, lanes, nv)");
+      return GNN_ERR_INVALID_ARG;
+    }
+    return GNN_OK;
+  })
+}
+
 gnn_status gnn_gat_layer(gnn_plan_t p, const float *X, int64_t ldx, int32_t f_in, const float *W,
                          const float *a_src, const float *a_dst, int32_t H, int32_t Fh, float neg_slope,
                          float *Y, int64_t ldy, void *ws, size_t ws_bytes, gnn_stream_t stream) {

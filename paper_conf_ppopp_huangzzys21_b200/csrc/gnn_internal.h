@@ -98,6 +98,7 @@ struct AggArgs {
   int32_t *ws_cnt;
   int32_t deterministic;
 };
+bool set_agg_mapping(int32_t vec, int32_t lanes, int32_t nv);
 size_t agg_workspace_bytes(const gnn_plan_s *p, int mode, int32_t F, int32_t H);
 gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, size_t ws_bytes,
                             cudaStream_t s);

@@ -600,15 +600,45 @@ struct Mapping {
   int vec, lanes, nv;
 };
 
+// feature chunks one call may sweep (sizes the per-chunk counters): the
+// automatic rule needs <= ceil(F/32); an override up to 8
+static int32_t max_chunks(int32_t F) { return std::max<int32_t>(8, (F + 31) / 32); }
+
+// process-wide mapping override (gnn_set_agg_mapping; the tuner hook)
+static Mapping g_override{0, 0, 0};
+
+bool set_agg_mapping(int32_t vec, int32_t lanes, int32_t nv) {
+  if (vec == 0 && lanes == 0 && nv == 0) {
+    g_override = Mapping{0, 0, 0};
+    return true;
+  }
+  const bool vec_ok = vec == 1 || vec == 2 || vec == 4 || vec == 8;
+  const bool lanes_ok = lanes == 4 || lanes == 8 || lanes == 16 || lanes == 32;
+  const bool nv_ok = nv == 1 || ((nv == 2 || nv == 4) && lanes == 32 && !(vec == 8 && nv == 4));
+  if (!vec_ok || !lanes_ok || !nv_ok) return false;
+  g_override = Mapping{vec, lanes, nv};
+  return true;
+}
+
+static bool vec_admissible(const AggArgs &a, int32_t fh_or_0, int v) {
+  bool ok = a.F % v == 0 && a.ldx % v == 0 && a.ldy % v == 0 && aligned(a.X, 4 * v) && aligned(a.Y, 4 * v);
+  if (a.add_row) ok = ok && a.ld_add % v == 0 && aligned(a.add_row, 4 * v);
+  if (fh_or_0) ok = ok && fh_or_0 % v == 0;
+  return ok;
+}
+
 // a4: feature-length-adaptive mapping rule
 static Mapping choose_mapping(const AggArgs &a, int32_t fh_or_0) {
   Mapping m{1, 4, 1};
+  if (g_override.vec != 0 && vec_admissible(a, fh_or_0, g_override.vec)) {
+    // GAT: a chunk must hold whole heads (the softmax state is per head)
+    const int cw = g_override.vec * g_override.lanes * g_override.nv;
+    const bool heads_ok = !fh_or_0 || cw >= a.F || cw % fh_or_0 == 0;
+    if (heads_ok && (a.F + cw - 1) / cw <= max_chunks(a.F)) return g_override;
+  }
   const int cands[4] = {8, 4, 2, 1};
   for (int v : cands) {
-    bool ok = a.F % v == 0 && a.ldx % v == 0 && a.ldy % v == 0 && aligned(a.X, 4 * v) && aligned(a.Y, 4 * v);
-    if (a.add_row) ok = ok && a.ld_add % v == 0 && aligned(a.add_row, 4 * v);
-    if (fh_or_0) ok = ok && fh_or_0 % v == 0;
-    if (ok) {
+    if (vec_admissible(a, fh_or_0, v)) {
       m.vec = v;
       break;
     }
@@ -625,7 +655,6 @@ static Mapping choose_mapping(const AggArgs &a, int32_t fh_or_0) {
   return m;
 }
 
-static int32_t max_chunks(int32_t F) { return F <= 128 ? 1 : (F + 31) / 32; }
 
 // layout: [unit counters (256 B)][row counters n_multi x nch | pad 256][acc n_multi x FW][slots x FW]
 size_t agg_workspace_bytes(const gnn_plan_s *p, int mode, int32_t F, int32_t H) {

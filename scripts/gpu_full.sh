@@ -1,0 +1,16 @@
+# full round session: GPU tests, bench, launch list, ncu --set full of the graph kernels
+# usage: bash scripts/gpu_full.sh TAG
+TAG=${1:-cur}
+set -x
+cd $GRAFT_REPO_ROOT; mkdir -p gpurun_out
+nvidia-smi > gpurun_out/smi.txt 2>&1
+nproc > gpurun_out/nproc.txt; grep -m1 "model name" /proc/cpuinfo >> gpurun_out/nproc.txt
+timeout 1500 python -m pytest tests -m gpu -x -q -p no:cacheprovider > gpurun_out/pytest_gpu_$TAG.log 2>&1
+echo "pytest rc=$?" >> gpurun_out/pytest_gpu_$TAG.log
+timeout 900 python bench.py --steps 10 --warmup 3 > gpurun_out/bench_$TAG.log 2>&1
+echo "bench rc=$?" >> gpurun_out/bench_$TAG.log
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_$TAG.csv python bench.py --steps 2 --warmup 1 --no-e2e --no-cpu > gpurun_out/ncu_launch_$TAG.log 2>&1
+echo "ncu rc=$?" >> gpurun_out/ncu_launch_$TAG.log
+timeout 1500 ncu --set full --clock-control none --import-source on -k regex:"k_aggregate|k_gemm_tc" -c 6 -o gpurun_out/prof_$TAG -f \
+  python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu > gpurun_out/ncu_full_$TAG.log 2>&1
+echo "ncu rc=$?" >> gpurun_out/ncu_full_$TAG.log

@@ -89,9 +89,36 @@ def agg(cfg="C5"):
         print(f"  GAT 8x32: {ms:.3f} ms  {alg / ms / 1e6:.0f} GB/s algorithmic", flush=True)
 
 
+def mapsweep(cfg="C5"):
+    """a4 mapping sweep: feature chunk width vs time (sum at F=256, GAT 8x32)."""
+    t0 = time.time()
+    g = gs.config_graph(cfg)
+    print(f"{cfg}: n={g.n} nnz={g.nnz} gen {time.time() - t0:.1f}s", flush=True)
+    plan = G.Plan(g.rowptr, g.colidx, reorder=1)
+    print(f" plan: {plan.info}", flush=True)
+    F = 256
+    X = torch.rand(g.n, F, device="cuda")
+    Y = torch.empty_like(X)
+    Hh, Fh = 8, 32
+    Zs = torch.rand(g.n, Hh * Fh + 2 * Hh, device="cuda")
+    Yg = torch.empty(g.n, Hh * Fh, device="cuda")
+    t = Zs[:, Hh * Fh + Hh:]
+    maps = [(0, 0, 0), (8, 32, 1), (4, 32, 2), (8, 16, 1), (4, 32, 1), (8, 8, 1), (4, 16, 1), (4, 8, 1), (8, 4, 1),
+            (2, 32, 1), (4, 4, 1)]
+    for (v, l, nv) in maps:
+        G.set_agg_mapping(v, l, nv)
+        ms = timeit(lambda: G.aggregate(plan, X, "sum", "gcn", out=Y), iters=5, warm=2)
+        msg = timeit(lambda: G.gat_aggregate(plan, Zs, t, Hh, Fh, out=Yg), iters=5, warm=2)
+        print(f" map vec={v} lanes={l} nv={nv} cw={v * l * nv}: sum F=256 {ms:.3f} ms | GAT 8x32 {msg:.3f} ms",
+              flush=True)
+    G.set_agg_mapping(0, 0, 0)
+
+
 if __name__ == "__main__":
     what = sys.argv[1] if len(sys.argv) > 1 else "gemm"
     if what == "gemm":
         gemm()
+    elif what == "map":
+        mapsweep(sys.argv[sys.argv.index("--cfg") + 1] if "--cfg" in sys.argv else "C5")
     else:
         agg(sys.argv[sys.argv.index("--cfg") + 1] if "--cfg" in sys.argv else "C5")

@@ -83,6 +83,18 @@ def test_invalid_args_return_status_not_crash():
     assert P.gnn.gnn_plan_destroy(None) == 0
 
 
+@pytest.mark.parametrize("vec,lanes,nv", [(3, 32, 1), (8, 2, 1), (8, 32, 4), (4, 16, 2), (0, 32, 1)])
+def test_agg_mapping_rejects_unsupported(vec, lanes, nv):
+    assert P.gnn.gnn_set_agg_mapping(vec, lanes, nv) == 1
+    assert P.gnn.gnn_set_agg_mapping(0, 0, 0) == 0
+
+
+def test_agg_mapping_accepts_supported():
+    for m in [(8, 32, 1), (8, 32, 2), (4, 32, 4), (8, 8, 1), (1, 4, 1)]:
+        assert P.gnn.gnn_set_agg_mapping(*m) == 0
+    assert P.gnn.gnn_set_agg_mapping(0, 0, 0) == 0
+
+
 @pytest.mark.parametrize("ng", [0, 1, 5, 16, 64])
 def test_groups_host_bit_exact_vs_oracle(ng):
     g = gs.powerlaw(1500, 25000, 16, 1500, 900, comm=32, rho=0.5, seed=ng)

@@ -116,6 +116,41 @@ def test_aggregate_bit_exact_vs_order_replica(graphs, reduce, weight, ng, Tg):
     assert np.array_equal(Y.view(np.uint32), rep.view(np.uint32)), np.abs(Y - rep).max()
 
 
+@pytest.mark.parametrize("mapping", [(8, 8, 1), (4, 16, 1), (8, 16, 1), (2, 32, 1), (4, 32, 2), (1, 4, 1)])
+@pytest.mark.parametrize("reduce", ["sum", "max"])
+def test_mapping_override_bit_exact(graphs, mapping, reduce):
+    """a4 override (tuner hook): any admissible mapping / feature-chunk width
+    gives the same deterministic result bit for bit (R9 is per feature)."""
+    g = graphs["hub"]
+    F = 256
+    X = gs.uniform(g.n, F, seed=21)
+    rep = oracle.aggregate_ng_f32(g.rowptr, g.colidx, X, 16, reduce, "gcn", None, relu=False)
+    plan = G.Plan(g.rowptr, g.colidx, group_size=16, tile_groups=4)
+    try:
+        G.set_agg_mapping(*mapping)
+        Y = H(G.aggregate(plan, T(X), reduce, "gcn"))
+    finally:
+        G.set_agg_mapping(0, 0, 0)
+    assert np.array_equal(Y.view(np.uint32), rep.view(np.uint32)), np.abs(Y - rep).max()
+
+
+@pytest.mark.parametrize("mapping", [(8, 8, 1), (8, 16, 1), (4, 16, 1)])
+def test_gat_mapping_override_parity(graphs, mapping):
+    g = graphs["hub"]
+    Hh, Fh = 8, 32
+    F = Hh * Fh
+    Zs = gs.uniform(g.n, F + Hh, seed=5)
+    t = gs.uniform(g.n, Hh, lo=-3, hi=3, seed=6)
+    ref = oracle.gat_aggregate(g.rowptr, g.colidx, Zs, t, Hh, Fh, 0.2)
+    plan = G.Plan(g.rowptr, g.colidx, group_size=16, tile_groups=4)
+    try:
+        G.set_agg_mapping(*mapping)
+        Y = H(G.gat_aggregate(plan, T(Zs), T(t), Hh, Fh, 0.2))
+    finally:
+        G.set_agg_mapping(0, 0, 0)
+    assert_close(Y, ref, what=f"gat mapping {mapping}")
+
+
 def test_integer_features_exact(graphs):
     g = graphs["hub"]
     X = gs.integer_features(g.n, 32, seed=1)
