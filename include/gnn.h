@@ -69,7 +69,8 @@ typedef struct {
   uint32_t struct_size;  /* sizeof(gnn_plan_opts), for ABI versioning */
   int32_t reorder;       /* 0 = identity task order, 1 = LAS (MinHash+LSH+merge) */
   int32_t group_size;    /* NG upper bound ng; -1 = auto (R8-ii); 0 = never split */
-  int32_t tile_groups;   /* T: max groups per work unit; longer rows are split (0 -> 32) */
+  int32_t tile_groups;   /* T: max neighbor groups per work unit (a run of consecutive groups in
+                            task order streamed by one worker; capped at 32) (0 -> 32) */
   int32_t cluster_cap;   /* LAS cluster size cap (32) */
   int32_t minhash_k;     /* K signature length (32) */
   int32_t lsh_rows;      /* r rows per band (2); b = K / r bands */
@@ -90,7 +91,7 @@ typedef struct {
   int64_t n_src;        /* source rows (== n for gnn_plan_create) */
   int64_t nnz;
   int64_t n_groups;     /* G = sum ceil(d_v / ng) */
-  int64_t n_tiles;      /* work units (whole rows, or T-group slices of longer rows) */
+  int64_t n_tiles;      /* work units (runs of <= T consecutive groups, <= E_u edges) */
   int64_t n_split_rows; /* rows with more than T groups (combined through the workspace) */
   int64_t n_empty_rows;
   int64_t n_clusters;   /* LAS clusters (n if reorder == 0) */
@@ -256,6 +257,12 @@ int gnn_set_gemm_impl(int impl);
  * feature and does not depend on the mapping).
  */
 gnn_status gnn_set_agg_mapping(int32_t vec, int32_t lanes, int32_t nv);
+
+/* Aggregation kernel selector (process-wide; same results bit for bit):
+ * 0 = stream kernel (default: one worker streams a run of consecutive groups
+ * with its loads in flight across group boundaries), 1 = per-group kernel
+ * (one work unit = one group).  Returns the previous value. */
+int gnn_set_agg_impl(int impl);
 
 /*
  * GCN layer (Eq 1): Y = ACT((A_gcn X) W).  order: 0 = auto (aggregate at

@@ -1,0 +1,874 @@
+// k_agg.cuh — the aggregation kernel family (a6/a7/a8/a9) of libgnn.so:
+// device templates and launch templates, instantiated per reducer in
+// k_agg_sum.cu / k_agg_max.cu / k_agg_gat.cu (parallel compilation).
+//
+// Paper: Huang et al., PPoPP'21 (PAPER.md P:<line>).  Design: DESIGN.md §5.
+#pragma once
+#include <cuda_runtime.h>
+#include <math.h>
+#include <stdint.h>
+
+#include <algorithm>
+
+#include "gnn_internal.h"
+
+namespace gnn {
+
+// ---------------------------------------------------------------------------
+// a6/a7/a8/a9: the aggregation kernel family.
+//
+// Mapping (a4, feature-length-adaptive): a "worker"
+// is LANES consecutive lanes (LANES in {4, 8, 16, 32}); each lane owns NV
+// vectors of VEC consecutive features (VEC in {1,2,4,8}; VEC = 8 is one
+// 256-bit LDG per lane).  Chunk width CW = LANES*VEC*NV features; wider rows
+// loop over chunks.  One CTA processes one plan tile (<= T neighbor groups,
+// P:855-884) per launch block; workers take groups round-robin.
+//
+// Per group: indices are loaded LANES at a time (one coalesced load), then
+// broadcast with sub-warp shuffles; U source rows are in flight per worker.
+// Group partial = sequential fp32 chain in CSR order (reading R9).
+// Single-group rows finish in the worker (epilogue + store).  Multi-group
+// rows inside one tile are combined in shared memory in group order (TB-level
+// data-visible-range adapter).  Rows spanning several tiles write
+// per-group partials to the workspace; the last-arriving CTA (per-row counter)
+// merges them in group order (P:885-894 with a fixed order) and applies the
+// postponed epilogue (linear property).
+// ---------------------------------------------------------------------------
+enum { M_SUM = 0, M_MEAN = 1, M_MAX = 2, M_GAT = 3 };
+// internal weight code: weight 1 inside the loop, x ndst[v] in the epilogue
+// (transform-first GCN whose GEMM epilogue already applied nsrc[u])
+constexpr int W_DST_ONLY = 3;
+__device__ __forceinline__ bool scales_dst(int w) { return w == GNN_W_GCN || w == W_DST_ONLY; }
+
+struct KParams {
+  DevGraph g;
+  int mode, weight;
+  const float *edge_w;
+  const float *X;
+  int64_t ldx;
+  int32_t F;
+  float *Y;
+  int64_t ldy;
+  const float *add_row;
+  int64_t ld_add;
+  int32_t relu;
+  const float *t;
+  int64_t ldt;
+  int32_t H, Fh;
+  float slope;
+  int32_t *ws_unit;  // work-unit counters (one per feature chunk), zeroed per call
+  float *ws_acc;   // [n_multi][FW] atomic accumulators (deterministic == 0)
+  float *ws_part;  // [multi slots][FW] per-group partials (deterministic)
+  int32_t *ws_cnt; // [n_multi][nch] arrival counters
+  int32_t FW;      // F (+ 2H for GAT)
+  int32_t deterministic;
+  int32_t nch;        // feature chunks per row (arrival counters per multi-unit row)
+  int32_t n_persist;  // persistent CTAs
+};
+
+template <int VEC>
+__device__ __forceinline__ void ldv(const float *p, float (&v)[VEC]) {
+  if constexpr (VEC == 8) {
+    asm volatile("ld.global.nc.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3]), "=f"(v[4]), "=f"(v[5]),
+                   "=f"(v[6]), "=f"(v[7])
+                 : "l"(p));
+  } else if constexpr (VEC == 4) {
+    float4 x = __ldg(reinterpret_cast<const float4 *>(p));
+    v[0] = x.x; v[1] = x.y; v[2] = x.z; v[3] = x.w;
+  } else if constexpr (VEC == 2) {
+    float2 x = __ldg(reinterpret_cast<const float2 *>(p));
+    v[0] = x.x; v[1] = x.y;
+  } else {
+    v[0] = __ldg(p);
+  }
+}
+
+template <int VEC>
+__device__ __forceinline__ void stv(float *p, const float (&v)[VEC]) {
+  if constexpr (VEC == 8) {
+    asm volatile("st.global.v8.f32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "f"(v[0]), "f"(v[1]),
+                 "f"(v[2]), "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]), "f"(v[7])
+                 : "memory");
+  } else if constexpr (VEC == 4) {
+    *reinterpret_cast<float4 *>(p) = make_float4(v[0], v[1], v[2], v[3]);
+  } else if constexpr (VEC == 2) {
+    *reinterpret_cast<float2 *>(p) = make_float2(v[0], v[1]);
+  } else {
+    p[0] = v[0];
+  }
+}
+
+// streaming index load: read once, do not keep in L1
+__device__ __forceinline__ int32_t ld_stream_i32(const int32_t *p) {
+  int32_t r;
+  asm volatile("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(r) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ float ld_stream_f32(const float *p) {
+  float r;
+  asm volatile("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(r) : "l"(p));
+  return r;
+}
+
+// fixed ReLU: y > 0 ? y : +0 (matches the oracle replica, R9)
+__device__ __forceinline__ float relu_f(float y) { return y > 0.0f ? y : 0.0f; }
+
+template <int MODE, int VEC, int NV>
+struct Part {
+  float a[NV][VEC];
+  float m[NV];  // GAT running max
+  float l[NV];  // GAT running sum
+};
+
+template <int MODE, int VEC, int NV>
+__device__ __forceinline__ void part_init(Part<MODE, VEC, NV> &P) {
+#pragma unroll
+  for (int n = 0; n < NV; ++n) {
+#pragma unroll
+    for (int i = 0; i < VEC; ++i) P.a[n][i] = (MODE == M_MAX) ? -INFINITY : 0.0f;
+    P.m[n] = -INFINITY;
+    P.l[n] = 0.0f;
+  }
+}
+
+// (m1,l1,a1) <- (m1,l1,a1) (+) (m2,l2,a2): online-softmax merge, fixed form.
+__device__ __forceinline__ void gat_merge(float &m1, float &l1, float *a1, float m2, float l2,
+                                          const float *a2, int cnt) {
+  const float m = fmaxf(m1, m2);
+  const float c1 = __expf(m1 - m), c2 = __expf(m2 - m);
+  l1 = fmaf(l2, c2, l1 * c1);
+  for (int i = 0; i < cnt; ++i) a1[i] = fmaf(a2[i], c2, a1[i] * c1);
+  m1 = m;
+}
+
+// combine partial B into A (A = A (+) B) in fixed form
+template <int MODE, int VEC, int NV>
+__device__ __forceinline__ void part_combine(Part<MODE, VEC, NV> &A, const Part<MODE, VEC, NV> &B) {
+#pragma unroll
+  for (int n = 0; n < NV; ++n) {
+    if constexpr (MODE == M_GAT) {
+      gat_merge(A.m[n], A.l[n], A.a[n], B.m[n], B.l[n], B.a[n], VEC);
+    } else {
+#pragma unroll
+      for (int i = 0; i < VEC; ++i)
+        A.a[n][i] = (MODE == M_MAX) ? fmaxf(A.a[n][i], B.a[n][i]) : A.a[n][i] + B.a[n][i];
+    }
+  }
+}
+
+// epilogue on one value (linear property: normalisation postponed)
+__device__ __forceinline__ float epi(const KParams &p, int mode, float a, float l, float ndst,
+                                     float deg_f, const float *addp) {
+  float y;
+  if (mode == M_GAT) {
+    y = a / l;
+  } else {
+    y = a;
+    if (scales_dst(p.weight)) y = y * ndst;
+    if (mode == M_MEAN) y = y / deg_f;
+    if (addp) y = y + *addp;
+  }
+  if (p.relu) y = relu_f(y);
+  return y;
+}
+
+template <int MODE, int VEC, int NV, int LANES>
+__device__ __forceinline__ void store_row(const KParams &p, int32_t row, int32_t deg, int32_t c0,
+                                          int lane, const Part<MODE, VEC, NV> &P) {
+  const float ndst = (MODE != M_GAT && scales_dst(p.weight)) ? __ldg(p.g.ndst + row) : 1.0f;
+  const float deg_f = (float)deg;
+#pragma unroll
+  for (int n = 0; n < NV; ++n) {
+    const int32_t f = c0 + (n * LANES + lane) * VEC;
+    if (f >= p.F) continue;
+    float y[VEC];
+    float addv[VEC];
+    if (p.add_row) ldv<VEC>(p.add_row + (int64_t)row * p.ld_add + f, addv);
+#pragma unroll
+    for (int i = 0; i < VEC; ++i) y[i] = epi(p, p.mode, P.a[n][i], P.l[n], ndst, deg_f, p.add_row ? &addv[i] : nullptr);
+    stv<VEC>(p.Y + (int64_t)row * p.ldy + f, y);
+  }
+}
+
+// load VEC floats from L2 (bypassing L1: data written by other SMs in this launch)
+template <int VEC>
+__device__ __forceinline__ void ldv_cg(const float *p, float (&v)[VEC]) {
+  if constexpr (VEC == 8) {
+    const float4 a = __ldcg(reinterpret_cast<const float4 *>(p));
+    const float4 b = __ldcg(reinterpret_cast<const float4 *>(p) + 1);
+    v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w; v[4] = b.x; v[5] = b.y; v[6] = b.z; v[7] = b.w;
+  } else if constexpr (VEC == 4) {
+    const float4 a = __ldcg(reinterpret_cast<const float4 *>(p));
+    v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
+  } else if constexpr (VEC == 2) {
+    const float2 a = __ldcg(reinterpret_cast<const float2 *>(p));
+    v[0] = a.x; v[1] = a.y;
+  } else {
+    v[0] = __ldcg(p);
+  }
+}
+
+// ---------------------------------------------------------------------------
+// v8 work distribution (measured: scripts/stream_bench_k.cu): persistent
+// workers grab work units in task (LAS) order through one atomic counter, so
+// the units in flight across the GPU are consecutive in the schedule and share
+// their source rows in L2; load balance is dynamic (NG's goal,
+// P:855-884) with no CTA barrier.  A unit is a whole row (<= R groups) or an
+// R-group slice of a longer row; its source indices are read from the
+// task-ordered colidx_t (one contiguous stream per unit).
+// ---------------------------------------------------------------------------
+
+// one neighbour group: fresh fp32 chain in CSR order (R9); indices from the
+// task-ordered stream, LANES at a time, U source rows in flight per worker
+template <int MODE, int VEC, int NV, int LANES>
+__device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx, int32_t len, int32_t beg,
+                                            int32_t row, int32_t c0, int lane, unsigned mask,
+                                            Part<MODE, VEC, NV> &G) {
+  constexpr int FPL = VEC * NV;
+  constexpr int U = FPL >= 32 ? 1 : (32 / FPL > 8 ? 8 : 32 / FPL);
+  part_init(G);
+  const int weight = p.weight;
+  const float *xl = p.X + c0 + lane * VEC;
+  bool valid[NV];
+  int32_t head[NV];
+  float tv[NV];
+#pragma unroll
+  for (int n = 0; n < NV; ++n) {
+    const int32_t f = c0 + (n * LANES + lane) * VEC;
+    valid[n] = f < p.F;
+    head[n] = 0;
+    tv[n] = 0.0f;
+    if constexpr (MODE == M_GAT) {
+      head[n] = valid[n] ? f / p.Fh : 0;
+      tv[n] = valid[n] ? __ldg(p.t + (int64_t)row * p.ldt + head[n]) : 0.0f;
+    }
+  }
+  // index batches: the next batch (and its weights) is requested before the
+  // current one is consumed
+  auto load_batch = [&](int32_t k, int32_t &u, float &w) {
+    const int32_t c = min(LANES, len - k);
+    u = 0;
+    w = 1.0f;
+    if (lane < c) {
+      u = ld_stream_i32(idx + k + lane);
+      if constexpr (MODE != M_GAT) {
+        if (weight == GNN_W_GCN) w = __ldg(p.g.nsrc + u);
+        else if (weight == GNN_W_EDGE) w = ld_stream_f32(p.edge_w + beg + k + lane);
+      }
+    }
+  };
+  int32_t nx_u = 0;
+  float nx_w = 1.0f;
+  if (len > 0) load_batch(0, nx_u, nx_w);
+  for (int32_t k = 0; k < len; k += LANES) {
+    const int32_t cnt = min(LANES, len - k);
+    const int32_t my_u = nx_u;
+    const float my_w = nx_w;
+    if (k + LANES < len) load_batch(k + LANES, nx_u, nx_w);
+    float v[U][NV][VEC];
+    float sc[U][NV];
+#pragma unroll
+    for (int q = 0; q < U; ++q) {
+      if (q < cnt) {
+        const int32_t u = __shfl_sync(mask, my_u, q, LANES);
+#pragma unroll
+        for (int n = 0; n < NV; ++n) {
+          if (valid[n]) ldv<VEC>(xl + (int64_t)u * p.ldx + n * LANES * VEC, v[q][n]);
+          if constexpr (MODE == M_GAT) sc[q][n] = valid[n] ? __ldg(p.X + (int64_t)u * p.ldx + p.F + head[n]) : 0.0f;
+        }
+      }
+    }
+    for (int32_t j = 0; j < cnt; j += U) {
+#pragma unroll
+      for (int q = 0; q < U; ++q) {
+        const int32_t e = j + q;
+        if (e < cnt) {
+          if constexpr (MODE == M_GAT) {
+            // online softmax (R9 GAT): one exp per edge and head
+#pragma unroll
+            for (int n = 0; n < NV; ++n) {
+              if (!valid[n]) continue;
+              float sco = sc[q][n] + tv[n];
+              sco = sco > 0.0f ? sco : p.slope * sco;  // LeakyReLU (Table 2 GAT)
+              const float d = sco - G.m[n];
+              const float ex = __expf(-fabsf(d));
+              const bool up = d > 0.0f;
+#pragma unroll
+              for (int i = 0; i < VEC; ++i)
+                G.a[n][i] = fmaf(up ? G.a[n][i] : v[q][n][i], ex, up ? v[q][n][i] : G.a[n][i]);
+              G.l[n] = fmaf(up ? G.l[n] : 1.0f, ex, up ? 1.0f : G.l[n]);
+              G.m[n] = up ? sco : G.m[n];
+            }
+          } else {
+            const float w = __shfl_sync(mask, my_w, e, LANES);
+#pragma unroll
+            for (int n = 0; n < NV; ++n) {
+              if (!valid[n]) continue;
+#pragma unroll
+              for (int i = 0; i < VEC; ++i) {
+                if constexpr (MODE == M_MAX) G.a[n][i] = fmaxf(G.a[n][i], w * v[q][n][i]);
+                else G.a[n][i] = fmaf(w, v[q][n][i], G.a[n][i]);
+              }
+            }
+          }
+          if (e + U < cnt) {
+            const int32_t u = __shfl_sync(mask, my_u, e + U, LANES);
+#pragma unroll
+            for (int n = 0; n < NV; ++n) {
+              if (valid[n]) ldv<VEC>(xl + (int64_t)u * p.ldx + n * LANES * VEC, v[q][n]);
+              if constexpr (MODE == M_GAT)
+                sc[q][n] = valid[n] ? __ldg(p.X + (int64_t)u * p.ldx + p.F + head[n]) : 0.0f;
+            }
+          }
+        }
+      }
+    }
+  }
+}
+
+// merge the group partials of a long row in group order (R9), epilogue, store
+template <int MODE, int VEC, int NV, int LANES>
+__device__ __forceinline__ void merge_row(const KParams &p, const float *base, int32_t ngrp, int32_t row,
+                                          int32_t deg, int32_t c0, int lane) {
+  Part<MODE, VEC, NV> A;
+  part_init(A);
+#pragma unroll
+  for (int n = 0; n < NV; ++n) {
+    const int32_t f = c0 + (n * LANES + lane) * VEC;
+    if (f >= p.F) continue;
+    for (int32_t q = 0; q < ngrp; ++q) {
+      float b[VEC];
+      ldv_cg<VEC>(base + (size_t)q * p.FW + f, b);
+      if constexpr (MODE == M_GAT) {
+        const float bm = __ldcg(base + (size_t)q * p.FW + p.F + f / p.Fh);
+        const float bl = __ldcg(base + (size_t)q * p.FW + p.F + p.H + f / p.Fh);
+        if (q == 0) {
+#pragma unroll
+          for (int i = 0; i < VEC; ++i) A.a[n][i] = b[i];
+          A.m[n] = bm;
+          A.l[n] = bl;
+        } else {
+          gat_merge(A.m[n], A.l[n], A.a[n], bm, bl, b, VEC);
+        }
+      } else {
+#pragma unroll
+        for (int i = 0; i < VEC; ++i)
+          A.a[n][i] = (q == 0) ? b[i] : (MODE == M_MAX ? fmaxf(A.a[n][i], b[i]) : A.a[n][i] + b[i]);
+      }
+    }
+  }
+  store_row<MODE, VEC, NV, LANES>(p, row, deg, c0, lane, A);
+}
+
+// one work unit = one neighbour group (NG: a group is the task of
+// one computing unit).  A row with a single group is finished here (epilogue +
+// store); the groups of a longer row leave their partials in the workspace and
+// the last one to arrive merges them in group order (R9).
+template <int MODE, int VEC, int NV, int LANES>
+__device__ __forceinline__ void process_unit(const KParams &p, int4 d, int32_t len, int32_t c0, int32_t ci, int lane,
+                                             unsigned mask) {
+  const DevGraph &g = p.g;
+  const int32_t tpos = d.x, beg = d.y, row = d.z, m = d.w;
+  Part<MODE, VEC, NV> G;
+  group_chain<MODE, VEC, NV, LANES>(p, g.colidx_t + tpos, len, beg, row, c0, lane, mask, G);
+  const int32_t rb = g.rowptr[row], re = g.rowptr[row + 1];
+  if (m < 0) {
+    store_row<MODE, VEC, NV, LANES>(p, row, re - rb, c0, lane, G);
+    return;
+  }
+  const int32_t ng = g.ng;
+  const int32_t ngrp = 1 + (re - rb - 1) / ng;
+  const int32_t k = (beg - rb) / ng;
+  const bool atomic_acc = !p.deterministic && MODE == M_SUM;
+  float *base = p.ws_part + (size_t)g.multi_slot[m] * p.FW;
+  float *acc = p.ws_acc + (size_t)m * p.FW;
+#pragma unroll
+  for (int n = 0; n < NV; ++n) {
+    const int32_t f = c0 + (n * LANES + lane) * VEC;
+    if (f >= p.F) continue;
+    if (atomic_acc) {
+#pragma unroll
+      for (int i = 0; i < VEC; ++i) atomicAdd(acc + f + i, G.a[n][i]);
+    } else {
+      stv<VEC>(base + (size_t)k * p.FW + f, G.a[n]);
+      if constexpr (MODE == M_GAT) {
+        if (f % p.Fh == 0) {
+          base[(size_t)k * p.FW + p.F + f / p.Fh] = G.m[n];
+          base[(size_t)k * p.FW + p.F + p.H + f / p.Fh] = G.l[n];
+        }
+      }
+    }
+  }
+  __threadfence();
+  __syncwarp(mask);
+  int32_t *cnt = p.ws_cnt + (size_t)m * p.nch + ci;
+  int last = 0;
+  if (lane == 0) last = atomicAdd(cnt, 1) == ngrp - 1;
+  last = __shfl_sync(mask, last, 0, LANES);
+  if (!last) return;
+  __threadfence();
+  if (atomic_acc) {
+    Part<MODE, VEC, NV> A;
+    part_init(A);
+#pragma unroll
+    for (int n = 0; n < NV; ++n) {
+      const int32_t f = c0 + (n * LANES + lane) * VEC;
+      if (f < p.F) ldv_cg<VEC>(acc + f, A.a[n]);
+    }
+    store_row<MODE, VEC, NV, LANES>(p, row, re - rb, c0, lane, A);
+  } else {
+    merge_row<MODE, VEC, NV, LANES>(p, base, ngrp, row, re - rb, c0, lane);
+  }
+  if (lane == 0) *cnt = 0;  // leave the counter at 0 for the next call
+}
+
+// ---------------------------------------------------------------------------
+// v10 stream kernel.  A work unit is a run of consecutive neighbour groups in
+// task order (plan: <= 32 groups, <= E_u edges); its source indices are one
+// contiguous range [T0, T1) of colidx_t.  The worker streams that range with
+// U source rows in flight and never drains its load pipeline at group or row
+// boundaries: when the edge that ends a group is consumed, the group's chain
+// (R9, unchanged: a fresh fp32 chain per group in CSR order) is finished —
+// epilogue + store, or partial + fixed-order merge for split rows — while the
+// loads of the next group's first rows are already in flight.
+//
+// Index stream: three LANES-wide batches (A = being issued, B, C = loading);
+// per-edge weights (GCN nsrc[u], explicit edge_w via the task->CSR map) are
+// fetched one batch ahead from indices that already arrived, so no load in
+// the loop waits on another load.
+// ---------------------------------------------------------------------------
+template <int MODE, int VEC, int NV, int LANES, bool WGT>
+struct Stream {
+  static constexpr int FPL = VEC * NV;
+  static constexpr int U0 = FPL >= 32 ? 1 : (32 / FPL > 8 ? 8 : 32 / FPL);
+  static constexpr int U = (MODE == M_GAT && U0 > 4) ? 4 : (U0 > LANES ? LANES : U0);
+};
+
+// finish one group: epilogue + store (whole row), or the group's partial to
+// its workspace slot (atomics into one accumulator row in the non-deterministic
+// variant); split rows are merged by k_merge after the stream kernel
+template <int MODE, int VEC, int NV, int LANES>
+__device__ __forceinline__ void finish_group(const KParams &p, const Part<MODE, VEC, NV> &G, int32_t row, int32_t m,
+                                             int32_t gbeg, int32_t len, int32_t c0, int32_t ci, int lane,
+                                             unsigned mask) {
+  if (m < 0) {
+    store_row<MODE, VEC, NV, LANES>(p, row, len, c0, lane, G);
+    return;
+  }
+  const DevGraph &g = p.g;
+  const int32_t k = (gbeg - __ldg(g.rowptr + row)) / g.ng;
+  const bool atomic_acc = !p.deterministic && MODE == M_SUM;
+  float *base = p.ws_part + (size_t)__ldg(g.multi_slot + m) * p.FW;
+  float *acc = p.ws_acc + (size_t)m * p.FW;
+#pragma unroll
+  for (int n = 0; n < NV; ++n) {
+    const int32_t f = c0 + (n * LANES + lane) * VEC;
+    if (f >= p.F) continue;
+    if (atomic_acc) {
+#pragma unroll
+      for (int i = 0; i < VEC; ++i) atomicAdd(acc + f + i, G.a[n][i]);
+    } else {
+      stv<VEC>(base + (size_t)k * p.FW + f, G.a[n]);
+      if constexpr (MODE == M_GAT) {
+        if (f % p.Fh == 0) {
+          base[(size_t)k * p.FW + p.F + f / p.Fh] = G.m[n];
+          base[(size_t)k * p.FW + p.F + p.H + f / p.Fh] = G.l[n];
+        }
+      }
+    }
+  }
+}
+
+// split rows (more than one group): merge the group partials in group order
+// (R9) and apply the postponed epilogue.  One worker per row.
+template <int MODE, int VEC, int NV, int LANES>
+__global__ void __launch_bounds__(256) k_merge(const KParams p) {
+  constexpr int CW = LANES * VEC * NV;
+  const int lane = threadIdx.x & (LANES - 1);
+  const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / LANES;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) / LANES;
+  const DevGraph &g = p.g;
+  for (int64_t m = w; m < g.n_multi; m += nw) {
+    const int32_t row = __ldg(g.multi_row + m);
+    const int32_t rb = __ldg(g.rowptr + row), re = __ldg(g.rowptr + row + 1);
+    const int32_t ngrp = 1 + (re - rb - 1) / g.ng;
+    for (int32_t c0 = 0; c0 < p.F; c0 += CW) {
+      if (!p.deterministic && MODE == M_SUM) {
+        const float *acc = p.ws_acc + (size_t)m * p.FW;
+        Part<MODE, VEC, NV> A;
+        part_init(A);
+#pragma unroll
+        for (int n = 0; n < NV; ++n) {
+          const int32_t f = c0 + (n * LANES + lane) * VEC;
+          if (f < p.F) ldv_cg<VEC>(acc + f, A.a[n]);
+        }
+        store_row<MODE, VEC, NV, LANES>(p, row, re - rb, c0, lane, A);
+      } else {
+        const float *base = p.ws_part + (size_t)__ldg(g.multi_slot + m) * p.FW;
+        merge_row<MODE, VEC, NV, LANES>(p, base, ngrp, row, re - rb, c0, lane);
+      }
+    }
+  }
+}
+
+template <int MODE, int VEC, int NV, int LANES, bool WGT>
+__device__ __forceinline__ void stream_unit(const KParams &p, int32_t g0, int32_t g1, int32_t T0, int32_t T1,
+                                            int32_t c0, int32_t ci, int lane, unsigned mask) {
+  constexpr int U = Stream<MODE, VEC, NV, LANES, WGT>::U;
+  const DevGraph &g = p.g;
+  // group table: lane j holds group gw + j
+  int32_t gw = g0;
+  int32_t gtp = 0, gend = 0, grow = 0, gm = -1, gbg = 0;
+  auto load_table = [&]() {
+    if (gw + lane < g1) {
+      const int4 d = __ldg(g.unit_desc + gw + lane);
+      gtp = d.x; gbg = d.y; grow = d.z; gm = d.w;
+      gend = __ldg(&g.unit_desc[gw + lane + 1].x);
+    }
+  };
+  load_table();
+  // index batches
+  const int32_t *idx = g.colidx_t;
+  auto ld_idx = [&](int32_t pos) -> int32_t { return pos < T1 ? ld_stream_i32(idx + pos) : 0; };
+  auto ld_pos = [&](int32_t pos) -> int32_t { return pos < T1 ? ld_stream_i32(g.pos_t + pos) : 0; };
+  auto weight_of = [&](int32_t u, int32_t cpos, int32_t pos) -> float {
+    if constexpr (WGT) {
+      if (pos >= T1) return 0.0f;
+      return p.weight == GNN_W_GCN ? __ldg(g.nsrc + u) : ld_stream_f32(p.edge_w + cpos);
+    } else {
+      return 1.0f;
+    }
+  };
+  int32_t ibase = T0;
+  int32_t a_u = ld_idx(T0 + lane), b_u = ld_idx(T0 + LANES + lane), c_u = ld_idx(T0 + 2 * LANES + lane);
+  int32_t a_c = 0, b_c = 0, c_c = 0;
+  if (WGT && p.weight == GNN_W_EDGE) {
+    a_c = ld_pos(T0 + lane); b_c = ld_pos(T0 + LANES + lane); c_c = ld_pos(T0 + 2 * LANES + lane);
+  }
+  float a_w = weight_of(a_u, a_c, T0 + lane), b_w = weight_of(b_u, b_c, T0 + LANES + lane);
+  // per-lane feature slice
+  bool valid[NV];
+  int32_t head[NV];
+#pragma unroll
+  for (int n = 0; n < NV; ++n) {
+    const int32_t f = c0 + (n * LANES + lane) * VEC;
+    valid[n] = f < p.F;
+    head[n] = (MODE == M_GAT && valid[n]) ? f / p.Fh : 0;
+  }
+  const float *xl = p.X + c0 + lane * VEC;
+  // current group
+  int32_t gi = g0;
+  int32_t cur_end = __shfl_sync(mask, gend, 0, LANES);
+  float tv[NV], tvn[NV];
+  auto load_tv = [&](int32_t row, float (&out)[NV]) {
+#pragma unroll
+    for (int n = 0; n < NV; ++n) out[n] = valid[n] ? __ldg(p.t + (int64_t)row * p.ldt + head[n]) : 0.0f;
+  };
+  if constexpr (MODE == M_GAT) {
+    load_tv(__shfl_sync(mask, grow, 0, LANES), tv);
+    if (g0 + 1 < g1 && 1 < LANES) load_tv(__shfl_sync(mask, grow, 1, LANES), tvn);
+  }
+  Part<MODE, VEC, NV> G;
+  part_init(G);
+  float v[U][NV][VEC];
+  float sc[U][NV];
+  float wq[U];
+  // issue the load of edge `pos` into slot q (pos is the next position in
+  // order; a macro so that q is a compile-time constant after unrolling and
+  // the slot arrays stay in registers)
+#define GNN_ISSUE(q, pos)                                                                             \
+  do {                                                                                                \
+    int32_t off_ = (pos) - ibase;                                                                     \
+    if (off_ == LANES) { /* batch A fully issued: rotate */                                          \
+      a_u = b_u; a_w = b_w; a_c = b_c;                                                                \
+      b_u = c_u; b_c = c_c;                                                                           \
+      b_w = weight_of(b_u, b_c, ibase + 2 * LANES + lane);                                            \
+      c_u = ld_idx(ibase + 3 * LANES + lane);                                                         \
+      if (WGT && p.weight == GNN_W_EDGE) c_c = ld_pos(ibase + 3 * LANES + lane);                      \
+      ibase += LANES;                                                                                 \
+      off_ = 0;                                                                                       \
+    }                                                                                                 \
+    const int32_t u_ = __shfl_sync(mask, a_u, off_, LANES);                                           \
+    if constexpr (WGT) wq[q] = __shfl_sync(mask, a_w, off_, LANES);                                   \
+    _Pragma("unroll") for (int n = 0; n < NV; ++n) {                                                  \
+      if (valid[n]) ldv<VEC>(xl + (int64_t)u_ * p.ldx + n * LANES * VEC, v[q][n]);                    \
+      if constexpr (MODE == M_GAT)                                                                    \
+        sc[q][n] = valid[n] ? __ldg(p.X + (int64_t)u_ * p.ldx + p.F + head[n]) : 0.0f;                \
+    }                                                                                                 \
+  } while (0)
+  int32_t pi = T0;
+#pragma unroll
+  for (int q = 0; q < U; ++q)
+    if (pi < T1) {
+      GNN_ISSUE(q, pi);
+      ++pi;
+    }
+  int32_t pe = T0;
+  while (pe < T1) {
+#pragma unroll
+    for (int q = 0; q < U; ++q) {
+      if (pe < T1) {
+        // consume edge pe (slot q)
+        if constexpr (MODE == M_GAT) {
+#pragma unroll
+          for (int n = 0; n < NV; ++n) {
+            if (!valid[n]) continue;
+            float sco = sc[q][n] + tv[n];
+            sco = sco > 0.0f ? sco : p.slope * sco;  // LeakyReLU (Table 2 GAT)
+            const float d = sco - G.m[n];
+            const float ex = __expf(-fabsf(d));
+            const bool up = d > 0.0f;
+#pragma unroll
+            for (int i = 0; i < VEC; ++i)
+              G.a[n][i] = fmaf(up ? G.a[n][i] : v[q][n][i], ex, up ? v[q][n][i] : G.a[n][i]);
+            G.l[n] = fmaf(up ? G.l[n] : 1.0f, ex, up ? 1.0f : G.l[n]);
+            G.m[n] = up ? sco : G.m[n];
+          }
+        } else {
+          const float w = WGT ? wq[q] : 1.0f;
+#pragma unroll
+          for (int n = 0; n < NV; ++n) {
+            if (!valid[n]) continue;
+#pragma unroll
+            for (int i = 0; i < VEC; ++i) {
+              if constexpr (MODE == M_MAX) G.a[n][i] = fmaxf(G.a[n][i], WGT ? w * v[q][n][i] : v[q][n][i]);
+              else G.a[n][i] = WGT ? fmaf(w, v[q][n][i], G.a[n][i]) : G.a[n][i] + v[q][n][i];
+            }
+          }
+        }
+        ++pe;
+        if (pe == cur_end) {
+          const int j = gi - gw;
+          const int32_t row = __shfl_sync(mask, grow, j, LANES);
+          const int32_t m = __shfl_sync(mask, gm, j, LANES);
+          const int32_t gb = __shfl_sync(mask, gbg, j, LANES);
+          const int32_t tp = __shfl_sync(mask, gtp, j, LANES);
+          finish_group<MODE, VEC, NV, LANES>(p, G, row, m, gb, cur_end - tp, c0, ci, lane, mask);
+          part_init(G);
+          ++gi;
+          if (gi < g1) {
+            if (gi - gw == LANES) {  // next window of the group table
+              gw += LANES;
+              load_table();
+              if constexpr (MODE == M_GAT) load_tv(__shfl_sync(mask, grow, 0, LANES), tvn);
+            }
+            cur_end = __shfl_sync(mask, gend, gi - gw, LANES);
+            if constexpr (MODE == M_GAT) {
+#pragma unroll
+              for (int n = 0; n < NV; ++n) tv[n] = tvn[n];
+              const int jn = gi + 1 - gw;
+              const int32_t rn = __shfl_sync(mask, grow, jn < LANES ? jn : 0, LANES);
+              if (gi + 1 < g1 && jn < LANES) load_tv(rn, tvn);
+            }
+          }
+        }
+        if (pi < T1) {
+          GNN_ISSUE(q, pi);
+          ++pi;
+        }
+      }
+    }
+  }
+#undef GNN_ISSUE
+}
+
+template <int MODE, int VEC, int NV, int LANES, bool WGT>
+__global__ void __launch_bounds__(256, MODE == M_GAT ? 3 : 4) k_stream(const KParams p) {
+  constexpr int CW = LANES * VEC * NV;
+  const int tid = threadIdx.x;
+  const int lane = tid & (LANES - 1);
+  const unsigned mask =
+      LANES == 32 ? 0xffffffffu : (((1u << LANES) - 1u) << ((tid & 31) & ~(LANES - 1)));
+  const DevGraph &g = p.g;
+  if ((int32_t)blockIdx.x >= p.n_persist) {
+    const int64_t r0 = (int64_t)(blockIdx.x - p.n_persist) * 32;
+    for (int64_t r = r0; r < r0 + 32 && r < g.n_empty; ++r) {
+      float *y = p.Y + (int64_t)g.empty_rows[r] * p.ldy;
+      for (int f = tid; f < p.F; f += blockDim.x) y[f] = 0.0f;
+    }
+    return;
+  }
+  const int32_t nunits = g.n_sunits;
+  int32_t ci = 0;
+  for (int32_t c0 = 0; c0 < p.F; c0 += CW, ++ci) {
+    int32_t *ctr = p.ws_unit + ci;
+    // the next unit (id, group range, index range) is claimed while the current one streams
+    int32_t u = 0;
+    if (lane == 0) u = atomicAdd(ctr, 1);
+    u = __shfl_sync(mask, u, 0, LANES);
+    int32_t g0 = 0, g1 = 0, t0 = 0, t1 = 0;
+    if (u < nunits) {
+      g0 = __ldg(g.sunit_beg + u);
+      g1 = __ldg(g.sunit_beg + u + 1);
+      t0 = __ldg(&g.unit_desc[g0].x);
+      t1 = __ldg(&g.unit_desc[g1].x);
+    }
+    while (u < nunits) {
+      int32_t un = 0;
+      if (lane == 0) un = atomicAdd(ctr, 1);
+      un = __shfl_sync(mask, un, 0, LANES);
+      int32_t h0 = 0, h1 = 0, s0 = 0, s1 = 0;
+      if (un < nunits) {
+        h0 = __ldg(g.sunit_beg + un);
+        h1 = __ldg(g.sunit_beg + un + 1);
+      }
+      stream_unit<MODE, VEC, NV, LANES, WGT>(p, g0, g1, t0, t1, c0, ci, lane, mask);
+      if (un < nunits) {
+        s0 = __ldg(&g.unit_desc[h0].x);
+        s1 = __ldg(&g.unit_desc[h1].x);
+      }
+      u = un; g0 = h0; g1 = h1; t0 = s0; t1 = s1;
+    }
+  }
+}
+
+#ifndef GNN_AGG_MINB
+#define GNN_AGG_MINB 4
+#endif
+template <int MODE, int VEC, int NV, int LANES>
+__global__ void __launch_bounds__(256, MODE == M_GAT ? GNN_AGG_MINB - 1 : GNN_AGG_MINB) k_aggregate(const KParams p) {
+  constexpr int CW = LANES * VEC * NV;
+  const int tid = threadIdx.x;
+  const int lane = tid & (LANES - 1);
+  const unsigned mask =
+      LANES == 32 ? 0xffffffffu : (((1u << LANES) - 1u) << ((tid & 31) & ~(LANES - 1)));
+  const DevGraph &g = p.g;
+  if ((int32_t)blockIdx.x >= p.n_persist) {
+    // zero-fill rows without in-edges (R3-i): 32 rows per block
+    const int64_t r0 = (int64_t)(blockIdx.x - p.n_persist) * 32;
+    for (int64_t r = r0; r < r0 + 32 && r < g.n_empty; ++r) {
+      float *y = p.Y + (int64_t)g.empty_rows[r] * p.ldy;
+      for (int f = tid; f < p.F; f += blockDim.x) y[f] = 0.0f;
+    }
+    return;
+  }
+  const int32_t nunits = g.n_units;
+  int32_t ci = 0;
+  for (int32_t c0 = 0; c0 < p.F; c0 += CW, ++ci) {
+    int32_t *ctr = p.ws_unit + ci;
+    // the next unit (id and descriptor) is claimed while the current one streams
+    int32_t u = 0;
+    if (lane == 0) u = atomicAdd(ctr, 1);
+    u = __shfl_sync(mask, u, 0, LANES);
+    int4 d = make_int4(0, 0, 0, -1);
+    int32_t dnx = 0;
+    if (u < nunits) {
+      d = __ldg(g.unit_desc + u);
+      dnx = __ldg(&g.unit_desc[u + 1].x);
+    }
+    while (u < nunits) {
+      int32_t un = 0;
+      if (lane == 0) un = atomicAdd(ctr, 1);
+      un = __shfl_sync(mask, un, 0, LANES);
+      int4 dn = make_int4(0, 0, 0, -1);
+      int32_t dnxn = 0;
+      if (un < nunits) {
+        dn = __ldg(g.unit_desc + un);
+        dnxn = __ldg(&g.unit_desc[un + 1].x);
+      }
+      process_unit<MODE, VEC, NV, LANES>(p, d, dnx - d.x, c0, ci, lane, mask);
+      u = un;
+      d = dn;
+      dnx = dnxn;
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------
+// launch templates
+// ---------------------------------------------------------------------------
+struct Mapping {
+  int vec, lanes, nv;
+};
+int num_sms();
+int agg_impl();
+
+template <typename KFN>
+cudaError_t launch_persistent(KFN fn, int &occ, const KParams &kp_in, int32_t units, int cw, int lanes,
+                                     int threads, cudaStream_t s) {
+  if (occ == 0) {
+    cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, 0);  // all of it to L1
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, threads, 0);
+    if (occ <= 0) occ = 1;
+  }
+  KParams kp = kp_in;
+  kp.nch = (kp.F + cw - 1) / cw;
+  const int64_t workers_per_cta = threads / lanes;
+  kp.n_persist = (int32_t)std::min<int64_t>((int64_t)num_sms() * occ,
+                                            std::max<int64_t>(1, (units + workers_per_cta - 1) / workers_per_cta));
+  cudaError_t e = cudaMemsetAsync(kp.ws_unit, 0, 256, s);
+  if (e == cudaSuccess && kp.g.n_multi > 0)
+    e = cudaMemsetAsync(kp.ws_cnt, 0, sizeof(int32_t) * (size_t)kp.g.n_multi * kp.nch, s);
+  if (e == cudaSuccess && kp.g.n_multi > 0 && !kp.deterministic && kp.mode != M_MAX && kp.mode != M_GAT)
+    e = cudaMemsetAsync(kp.ws_acc, 0, sizeof(float) * (size_t)kp.g.n_multi * kp.FW, s);
+  if (e != cudaSuccess) return e;
+  const int64_t blocks = (int64_t)kp.n_persist + (kp.g.n_empty + 31) / 32;
+  fn<<<(unsigned)blocks, threads, 0, s>>>(kp);
+  count_launch();
+  return cudaGetLastError();
+}
+
+template <int MODE, int VEC, int NV, int LANES>
+cudaError_t launch_one(const KParams &kp, int threads, cudaStream_t s) {
+  constexpr int CW = LANES * VEC * NV;
+  if (agg_impl() == 1) {
+    static int occ = 0;
+    return launch_persistent(k_aggregate<MODE, VEC, NV, LANES>, occ, kp, kp.g.n_units, CW, LANES, threads, s);
+  }
+  const bool wgt = MODE != M_GAT && (kp.weight == GNN_W_GCN || kp.weight == GNN_W_EDGE);
+  cudaError_t e;
+  if constexpr (MODE != M_GAT) {
+    static int occ_w = 0;
+    static int occ = 0;
+    e = wgt ? launch_persistent(k_stream<MODE, VEC, NV, LANES, true>, occ_w, kp, kp.g.n_sunits, CW, LANES, threads, s)
+            : launch_persistent(k_stream<MODE, VEC, NV, LANES, false>, occ, kp, kp.g.n_sunits, CW, LANES, threads, s);
+  } else {
+    static int occ = 0;
+    e = launch_persistent(k_stream<MODE, VEC, NV, LANES, false>, occ, kp, kp.g.n_sunits, CW, LANES, threads, s);
+  }
+  if (e != cudaSuccess || kp.g.n_multi == 0) return e;
+  // split rows: fixed-order merge of the group partials (R9)
+  KParams km = kp;
+  km.nch = (kp.F + CW - 1) / CW;
+  const int64_t blocks = std::max<int64_t>(1, std::min<int64_t>((kp.g.n_multi * LANES + 255) / 256, 148 * 8));
+  k_merge<MODE, VEC, NV, LANES><<<(unsigned)blocks, 256, 0, s>>>(km);
+  count_launch();
+  return cudaGetLastError();
+}
+
+template <int MODE, int VEC>
+cudaError_t dispatch_lanes(const KParams &kp, const Mapping &m, int threads, cudaStream_t s) {
+  switch (m.lanes) {
+    case 4: return launch_one<MODE, VEC, 1, 4>(kp, threads, s);
+    case 8: return launch_one<MODE, VEC, 1, 8>(kp, threads, s);
+    case 16: return launch_one<MODE, VEC, 1, 16>(kp, threads, s);
+    default:
+      if (m.nv == 1) return launch_one<MODE, VEC, 1, 32>(kp, threads, s);
+      if (m.nv == 2) return launch_one<MODE, VEC, 2, 32>(kp, threads, s);
+      if constexpr (VEC < 8) return launch_one<MODE, VEC, 4, 32>(kp, threads, s);
+      return cudaErrorInvalidValue;
+  }
+}
+
+template <int MODE>
+cudaError_t dispatch_vec(const KParams &kp, const Mapping &m, int threads, cudaStream_t s) {
+#ifdef GNN_DEV_SUBSET  // dev builds: only the C5 bench instantiations (fast compile)
+  if (m.lanes == 32 && m.nv == 1 && m.vec == 8) return launch_one<MODE, 8, 1, 32>(kp, threads, s);
+  if (m.lanes == 32 && m.nv == 1 && m.vec == 4) return launch_one<MODE, 4, 1, 32>(kp, threads, s);
+  return cudaErrorInvalidValue;
+#else
+  switch (m.vec) {
+    case 8: return dispatch_lanes<MODE, 8>(kp, m, threads, s);
+    case 4: return dispatch_lanes<MODE, 4>(kp, m, threads, s);
+    case 2: return dispatch_lanes<MODE, 2>(kp, m, threads, s);
+    default: return dispatch_lanes<MODE, 1>(kp, m, threads, s);
+  }
+#endif
+}
+
+cudaError_t dispatch_sum(const KParams &kp, const Mapping &m, int threads, cudaStream_t s);
+cudaError_t dispatch_max(const KParams &kp, const Mapping &m, int threads, cudaStream_t s);
+cudaError_t dispatch_gat(const KParams &kp, const Mapping &m, int threads, cudaStream_t s);
+
+}  // namespace gnn
