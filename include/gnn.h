@@ -248,7 +248,8 @@ int gnn_set_gemm_impl(int impl);
  * P:1128-1168): every later graph op whose F, strides and pointers
  * admit it uses vec floats per lane-vector (1, 2, 4 or 8), `lanes` lanes per
  * worker (4, 8, 16 or 32) and nv vectors per lane (1, 2 or 4; nv > 1 needs
- * lanes == 32; vec 8 allows nv <= 2).  The feature chunk lanes*vec*nv bounds
+ * lanes == 32 (vec 8: nv <= 2), or lanes*nv == 32 with lanes 16 (vec >= 2) or
+ * lanes 8 (vec >= 4)).  The feature chunk lanes*vec*nv bounds
  * the width of H one sweep over the schedule gathers (wider rows take several
  * sweeps).  An op whose shapes do not admit the override uses the automatic
  * rule.  vec = lanes = nv = 0 restores the automatic rule.

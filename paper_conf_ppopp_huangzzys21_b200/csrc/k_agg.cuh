@@ -56,6 +56,7 @@ struct KParams {
   int64_t ldt;
   int32_t H, Fh;
   float slope;
+  const uint32_t *smax;  // GAT: [H] order-encoded max over sources of s_u[h] (k_score_max)
   int32_t *ws_unit;  // work-unit counters (one per feature chunk), zeroed per call
   float *ws_acc;   // [n_multi][FW] atomic accumulators (deterministic == 0)
   float *ws_part;  // [multi slots][FW] per-group partials (deterministic)
@@ -113,6 +114,33 @@ __device__ __forceinline__ float ld_stream_f32(const float *p) {
 
 // fixed ReLU: y > 0 ? y : +0 (matches the oracle replica, R9)
 __device__ __forceinline__ float relu_f(float y) { return y > 0.0f ? y : 0.0f; }
+
+// LeakyReLU (Table 2 GAT) as one min/max: for slope <= 1,
+// max(x, slope*x) is x for x >= 0 and slope*x below 0 (min for slope > 1)
+__device__ __forceinline__ float leaky_f(float x, float slope) {
+  return slope <= 1.0f ? fmaxf(x, slope * x) : fminf(x, slope * x);
+}
+__device__ __forceinline__ float ex2_f(float x) {
+  float r;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+  return r;
+}
+// order-preserving float <-> uint32 key (atomicMax on floats, exact)
+__device__ __forceinline__ uint32_t fkey(float f) {
+  const uint32_t b = __float_as_uint(f);
+  return (b & 0x80000000u) ? ~b : (b | 0x80000000u);
+}
+__device__ __forceinline__ float fkey_decode(uint32_t k) {
+  return __uint_as_float((k & 0x80000000u) ? (k & 0x7fffffffu) : ~k);
+}
+constexpr float kLog2e = 1.4426950408889634f;
+// GAT softmax shift (reading R9 GAT): a group is accumulated against the
+// reference m = LeakyReLU(max_u s_u[h] + t_v[h]), an upper bound of every
+// score of the row (LeakyReLU and rounding are monotone), so each term is
+// exp(e - m) <= 1 and there is no per-edge rescaling.  If the bound is
+// looser than kGatSlack for some head (exp(-kGatSlack) keeps all terms
+// normal) the group is recomputed against its own exact max.
+constexpr float kGatSlack = 32.0f;
 
 template <int MODE, int VEC, int NV>
 struct Part {
@@ -233,15 +261,24 @@ __device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx
   bool valid[NV];
   int32_t head[NV];
   float tv[NV];
+  float nmb[NV];   // GAT: -m * log2(e) for the current reference m
+  float seen[NV];  // GAT: exact max score of the group
+  // GAT: a one-edge group takes its own score as reference (term = 1 exactly)
+  const bool one = MODE == M_GAT && len == 1;
 #pragma unroll
   for (int n = 0; n < NV; ++n) {
     const int32_t f = c0 + (n * LANES + lane) * VEC;
     valid[n] = f < p.F;
     head[n] = 0;
     tv[n] = 0.0f;
+    nmb[n] = 0.0f;
+    seen[n] = -INFINITY;
     if constexpr (MODE == M_GAT) {
       head[n] = valid[n] ? f / p.Fh : 0;
       tv[n] = valid[n] ? __ldg(p.t + (int64_t)row * p.ldt + head[n]) : 0.0f;
+      const float mb = valid[n] ? leaky_f(fkey_decode(__ldg(p.smax + head[n])) + tv[n], p.slope) : 0.0f;
+      G.m[n] = mb;
+      nmb[n] = -mb * kLog2e;
     }
   }
   // index batches: the next batch (and its weights) is requested before the
@@ -258,70 +295,91 @@ __device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx
       }
     }
   };
-  int32_t nx_u = 0;
-  float nx_w = 1.0f;
-  if (len > 0) load_batch(0, nx_u, nx_w);
-  for (int32_t k = 0; k < len; k += LANES) {
-    const int32_t cnt = min(LANES, len - k);
-    const int32_t my_u = nx_u;
-    const float my_w = nx_w;
-    if (k + LANES < len) load_batch(k + LANES, nx_u, nx_w);
-    float v[U][NV][VEC];
-    float sc[U][NV];
-#pragma unroll
-    for (int q = 0; q < U; ++q) {
-      if (q < cnt) {
-        const int32_t u = __shfl_sync(mask, my_u, q, LANES);
-#pragma unroll
-        for (int n = 0; n < NV; ++n) {
-          if (valid[n]) ldv<VEC>(xl + (int64_t)u * p.ldx + n * LANES * VEC, v[q][n]);
-          if constexpr (MODE == M_GAT) sc[q][n] = valid[n] ? __ldg(p.X + (int64_t)u * p.ldx + p.F + head[n]) : 0.0f;
-        }
-      }
-    }
-    for (int32_t j = 0; j < cnt; j += U) {
+#pragma unroll 1
+  for (int pass = 0;; ++pass) {
+    int32_t nx_u = 0;
+    float nx_w = 1.0f;
+    if (len > 0) load_batch(0, nx_u, nx_w);
+    for (int32_t k = 0; k < len; k += LANES) {
+      const int32_t cnt = min(LANES, len - k);
+      const int32_t my_u = nx_u;
+      const float my_w = nx_w;
+      if (k + LANES < len) load_batch(k + LANES, nx_u, nx_w);
+      float v[U][NV][VEC];
+      float sc[U][NV];
 #pragma unroll
       for (int q = 0; q < U; ++q) {
-        const int32_t e = j + q;
-        if (e < cnt) {
-          if constexpr (MODE == M_GAT) {
-            // online softmax (R9 GAT): one exp per edge and head
+        if (q < cnt) {
+          const int32_t u = __shfl_sync(mask, my_u, q, LANES);
 #pragma unroll
-            for (int n = 0; n < NV; ++n) {
-              if (!valid[n]) continue;
-              float sco = sc[q][n] + tv[n];
-              sco = sco > 0.0f ? sco : p.slope * sco;  // LeakyReLU (Table 2 GAT)
-              const float d = sco - G.m[n];
-              const float ex = __expf(-fabsf(d));
-              const bool up = d > 0.0f;
+          for (int n = 0; n < NV; ++n) {
+            if (valid[n]) ldv<VEC>(xl + (int64_t)u * p.ldx + n * LANES * VEC, v[q][n]);
+            if constexpr (MODE == M_GAT) sc[q][n] = valid[n] ? __ldg(p.X + (int64_t)u * p.ldx + p.F + head[n]) : 0.0f;
+          }
+        }
+      }
+      for (int32_t j = 0; j < cnt; j += U) {
 #pragma unroll
-              for (int i = 0; i < VEC; ++i)
-                G.a[n][i] = fmaf(up ? G.a[n][i] : v[q][n][i], ex, up ? v[q][n][i] : G.a[n][i]);
-              G.l[n] = fmaf(up ? G.l[n] : 1.0f, ex, up ? 1.0f : G.l[n]);
-              G.m[n] = up ? sco : G.m[n];
+        for (int q = 0; q < U; ++q) {
+          const int32_t e = j + q;
+          if (e < cnt) {
+            if constexpr (MODE == M_GAT) {
+              // e_uv = LeakyReLU(s_u + t_v); term exp(e_uv - m) (one ex2 per edge and head)
+#pragma unroll
+              for (int n = 0; n < NV; ++n) {
+                if (!valid[n]) continue;
+                const float sco = leaky_f(sc[q][n] + tv[n], p.slope);
+                seen[n] = fmaxf(seen[n], sco);
+                const float ex = one ? 1.0f : ex2_f(fmaf(sco, kLog2e, nmb[n]));
+                G.l[n] += ex;
+#pragma unroll
+                for (int i = 0; i < VEC; ++i) G.a[n][i] = fmaf(ex, v[q][n][i], G.a[n][i]);
+              }
+            } else {
+              const float w = __shfl_sync(mask, my_w, e, LANES);
+#pragma unroll
+              for (int n = 0; n < NV; ++n) {
+                if (!valid[n]) continue;
+#pragma unroll
+                for (int i = 0; i < VEC; ++i) {
+                  if constexpr (MODE == M_MAX) G.a[n][i] = fmaxf(G.a[n][i], w * v[q][n][i]);
+                  else G.a[n][i] = fmaf(w, v[q][n][i], G.a[n][i]);
+                }
+              }
             }
-          } else {
-            const float w = __shfl_sync(mask, my_w, e, LANES);
+            if (e + U < cnt) {
+              const int32_t u = __shfl_sync(mask, my_u, e + U, LANES);
 #pragma unroll
-            for (int n = 0; n < NV; ++n) {
-              if (!valid[n]) continue;
-#pragma unroll
-              for (int i = 0; i < VEC; ++i) {
-                if constexpr (MODE == M_MAX) G.a[n][i] = fmaxf(G.a[n][i], w * v[q][n][i]);
-                else G.a[n][i] = fmaf(w, v[q][n][i], G.a[n][i]);
+              for (int n = 0; n < NV; ++n) {
+                if (valid[n]) ldv<VEC>(xl + (int64_t)u * p.ldx + n * LANES * VEC, v[q][n]);
+                if constexpr (MODE == M_GAT)
+                  sc[q][n] = valid[n] ? __ldg(p.X + (int64_t)u * p.ldx + p.F + head[n]) : 0.0f;
               }
             }
           }
-          if (e + U < cnt) {
-            const int32_t u = __shfl_sync(mask, my_u, e + U, LANES);
-#pragma unroll
-            for (int n = 0; n < NV; ++n) {
-              if (valid[n]) ldv<VEC>(xl + (int64_t)u * p.ldx + n * LANES * VEC, v[q][n]);
-              if constexpr (MODE == M_GAT)
-                sc[q][n] = valid[n] ? __ldg(p.X + (int64_t)u * p.ldx + p.F + head[n]) : 0.0f;
-            }
-          }
         }
+      }
+    }
+    if constexpr (MODE != M_GAT) {
+      break;
+    } else {
+      if (one) {
+#pragma unroll
+        for (int n = 0; n < NV; ++n) G.m[n] = seen[n];
+        break;
+      }
+      // bound too loose for some head of this worker: redo against the exact max
+      bool loose = false;
+#pragma unroll
+      for (int n = 0; n < NV; ++n) loose |= valid[n] && !(G.m[n] - seen[n] <= kGatSlack);
+      if (pass == 1 || !__any_sync(mask, loose)) break;
+#pragma unroll
+      for (int n = 0; n < NV; ++n) {
+        G.m[n] = seen[n];
+        nmb[n] = -seen[n] * kLog2e;
+        G.l[n] = 0.0f;
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) G.a[n][i] = 0.0f;
       }
     }
   }
@@ -726,8 +784,11 @@ __global__ void __launch_bounds__(256, MODE == M_GAT ? 3 : 4) k_stream(const KPa
 #ifndef GNN_AGG_MINB
 #define GNN_AGG_MINB 4
 #endif
+#ifndef GNN_AGG_MINB_GAT
+#define GNN_AGG_MINB_GAT 4
+#endif
 template <int MODE, int VEC, int NV, int LANES>
-__global__ void __launch_bounds__(256, MODE == M_GAT ? GNN_AGG_MINB - 1 : GNN_AGG_MINB) k_aggregate(const KParams p) {
+__global__ void __launch_bounds__(256, MODE == M_GAT ? GNN_AGG_MINB_GAT : GNN_AGG_MINB) k_aggregate(const KParams p) {
   constexpr int CW = LANES * VEC * NV;
   const int tid = threadIdx.x;
   const int lane = tid & (LANES - 1);
@@ -841,8 +902,16 @@ template <int MODE, int VEC>
 cudaError_t dispatch_lanes(const KParams &kp, const Mapping &m, int threads, cudaStream_t s) {
   switch (m.lanes) {
     case 4: return launch_one<MODE, VEC, 1, 4>(kp, threads, s);
-    case 8: return launch_one<MODE, VEC, 1, 8>(kp, threads, s);
-    case 16: return launch_one<MODE, VEC, 1, 16>(kp, threads, s);
+    case 8:
+      if constexpr (VEC >= 4) {
+        if (m.nv == 4) return launch_one<MODE, VEC, 4, 8>(kp, threads, s);
+      }
+      return launch_one<MODE, VEC, 1, 8>(kp, threads, s);
+    case 16:
+      if constexpr (VEC >= 2) {
+        if (m.nv == 2) return launch_one<MODE, VEC, 2, 16>(kp, threads, s);
+      }
+      return launch_one<MODE, VEC, 1, 16>(kp, threads, s);
     default:
       if (m.nv == 1) return launch_one<MODE, VEC, 1, 32>(kp, threads, s);
       if (m.nv == 2) return launch_one<MODE, VEC, 2, 32>(kp, threads, s);
@@ -856,6 +925,10 @@ cudaError_t dispatch_vec(const KParams &kp, const Mapping &m, int threads, cudaS
 #ifdef GNN_DEV_SUBSET  // dev builds: only the C5 bench instantiations (fast compile)
   if (m.lanes == 32 && m.nv == 1 && m.vec == 8) return launch_one<MODE, 8, 1, 32>(kp, threads, s);
   if (m.lanes == 32 && m.nv == 1 && m.vec == 4) return launch_one<MODE, 4, 1, 32>(kp, threads, s);
+  if (m.lanes == 16 && m.nv == 2 && m.vec == 4) return launch_one<MODE, 4, 2, 16>(kp, threads, s);
+  if (m.lanes == 8 && m.nv == 4 && m.vec == 4) return launch_one<MODE, 4, 4, 8>(kp, threads, s);
+  if (m.lanes == 16 && m.nv == 2 && m.vec == 8) return launch_one<MODE, 8, 2, 16>(kp, threads, s);
+  if (m.lanes == 8 && m.nv == 4 && m.vec == 8) return launch_one<MODE, 8, 4, 8>(kp, threads, s);
   return cudaErrorInvalidValue;
 #else
   switch (m.vec) {

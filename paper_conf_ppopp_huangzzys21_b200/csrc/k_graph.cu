@@ -129,6 +129,40 @@ cudaError_t launch_minhash(const int32_t *rowptr, const int32_t *colidx, int64_t
 }
 
 // ---------------------------------------------------------------------------
+// GAT softmax reference (reading R9 GAT): smax[h] = max over the source rows
+// of s_u[h], as order-preserving keys (exact, order-free).  One strided pass
+// over the H score columns (n_src x H x 4 B, ~3% of the aggregation's reads).
+// ---------------------------------------------------------------------------
+__global__ void k_score_max(const float *__restrict__ S, int64_t lds, int64_t n_src, int32_t H,
+                            uint32_t *smax) {
+  __shared__ uint32_t red[256];
+  const int per = blockDim.x / H;  // rows per block pass; blockDim.x = per * H
+  const int h = threadIdx.x % H, r = threadIdx.x / H;
+  uint32_t k = 0;
+  for (int64_t row = blockIdx.x * (int64_t)per + r; row < n_src; row += (int64_t)gridDim.x * per)
+    k = max(k, fkey(__ldg(S + row * lds + h)));
+  red[threadIdx.x] = k;
+  __syncthreads();
+  if (r == 0) {
+    for (int j = 1; j < per; ++j) k = max(k, red[j * H + h]);
+    atomicMax(smax + h, k);
+  }
+}
+
+cudaError_t launch_score_max(const float *S, int64_t lds, int64_t n_src, int32_t H, uint32_t *smax,
+                             cudaStream_t s) {
+  cudaError_t e = cudaMemsetAsync(smax, 0, sizeof(uint32_t) * (size_t)H, s);
+  if (e != cudaSuccess || n_src == 0) return e;
+  const int threads = H <= 256 ? (256 / H) * H : 0;
+  if (threads == 0) return cudaErrorInvalidValue;
+  const int per = threads / H;
+  const int blocks = (int)std::max<int64_t>(1, std::min<int64_t>((n_src + per - 1) / per, (int64_t)num_sms() * 8));
+  k_score_max<<<blocks, threads, 0, s>>>(S, lds, n_src, H, smax);
+  count_launch();
+  return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------
 // host dispatch
 // ---------------------------------------------------------------------------
 static bool aligned(const void *ptr, int bytes) {
@@ -150,7 +184,8 @@ bool set_agg_mapping(int32_t vec, int32_t lanes, int32_t nv) {
   }
   const bool vec_ok = vec == 1 || vec == 2 || vec == 4 || vec == 8;
   const bool lanes_ok = lanes == 4 || lanes == 8 || lanes == 16 || lanes == 32;
-  const bool nv_ok = nv == 1 || ((nv == 2 || nv == 4) && lanes == 32 && !(vec == 8 && nv == 4));
+  const bool nv_ok = nv == 1 || ((nv == 2 || nv == 4) && lanes == 32 && !(vec == 8 && nv == 4)) ||
+                     (vec >= 2 && lanes == 16 && nv == 2) || (vec >= 4 && lanes == 8 && nv == 4);
   if (!vec_ok || !lanes_ok || !nv_ok) return false;
   g_override = Mapping{vec, lanes, nv};
   return true;
@@ -184,7 +219,14 @@ static Mapping choose_mapping(const AggArgs &a, int32_t fh_or_0) {
   while (lanes < nvec && lanes < 32) lanes *= 2;
   m.lanes = lanes;
   m.nv = 1;
-  if (lanes == 32) {
+  if (lanes == 32 && nvec <= 32 && !fh_or_0 && m.vec >= 4) {
+    // 17..32 vectors: two 16-lane workers per warp with two vectors per lane
+    // halve the per-edge index/shuffle/address work per warp (measured on C5:
+    // F=100 10.95 -> 9.72 ms, F=256 14.67 -> 14.23 ms; GAT 8x32 is faster
+    // with one 32-lane worker: 19.2 vs 21.0 ms)
+    m.lanes = 16;
+    m.nv = 2;
+  } else if (lanes == 32) {
     const int max_nv = m.vec == 8 ? 2 : 4;
     while (m.nv < max_nv && 32 * m.nv < nvec) m.nv *= 2;
   }
@@ -192,10 +234,14 @@ static Mapping choose_mapping(const AggArgs &a, int32_t fh_or_0) {
 }
 
 
-// layout: [unit counters (256 B)][row counters n_multi x nch | pad 256][acc n_multi x FW][slots x FW]
+// layout: [unit counters (256 B)][GAT score max: H keys | pad 256][row counters n_multi x nch | pad 256]
+//         [acc n_multi x FW][slots x FW]
+static size_t smax_bytes(int mode, int32_t H) {
+  return mode == M_GAT ? ((sizeof(uint32_t) * (size_t)H + 255) & ~(size_t)255) : 0;
+}
 size_t agg_workspace_bytes(const gnn_plan_s *p, int mode, int32_t F, int32_t H) {
   const size_t FW = (size_t)F + (mode == M_GAT ? 2 * (size_t)H : 0);
-  size_t b = 256;
+  size_t b = 256 + smax_bytes(mode, H);
   size_t c = sizeof(int32_t) * (size_t)p->n_multi * max_chunks(F);
   b += (c + 255) & ~(size_t)255;
   return b + sizeof(float) * ((size_t)p->multi_slots + (size_t)p->n_multi) * FW;
@@ -251,12 +297,19 @@ gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, siz
   char *w = reinterpret_cast<char *>(ws);
   kp.ws_unit = reinterpret_cast<int32_t *>(w);
   const size_t cnt_bytes = (sizeof(int32_t) * (size_t)p->n_multi * max_chunks(a.F) + 255) & ~(size_t)255;
-  kp.ws_cnt = reinterpret_cast<int32_t *>(w + 256);
-  kp.ws_acc = reinterpret_cast<float *>(w + 256 + cnt_bytes);
+  const size_t sm_bytes = smax_bytes(mode, a.H);
+  kp.ws_cnt = reinterpret_cast<int32_t *>(w + 256 + sm_bytes);
+  kp.ws_acc = reinterpret_cast<float *>(w + 256 + sm_bytes + cnt_bytes);
   kp.ws_part = kp.ws_acc + (size_t)p->n_multi * kp.FW;
   const Mapping m = choose_mapping(a, mode == M_GAT ? a.Fh : 0);
   const int threads = 256;
   cudaError_t e;
+  if (mode == M_GAT) {
+    uint32_t *smax = reinterpret_cast<uint32_t *>(w + 256);
+    kp.smax = smax;
+    e = launch_score_max(a.X + a.F, a.ldx, p->n_src, a.H, smax, s);
+    if (e != cudaSuccess) return cuda_status(e, "score max launch");
+  }
   switch (mode) {
     case M_SUM:
     case M_MEAN: e = dispatch_sum(kp, m, threads, s); break;

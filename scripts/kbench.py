@@ -114,6 +114,37 @@ def mapsweep(cfg="C5"):
     G.set_agg_mapping(0, 0, 0)
 
 
+def map100(cfg="C5"):
+    """a4 sweep at the bench's layer-1 width (F=100, GCN weights) and GAT 8x32."""
+    g = gs.config_graph(cfg)
+    plan = G.Plan(g.rowptr, g.colidx, reorder=1)
+    X1 = torch.rand(g.n, 100, device="cuda")
+    Y1 = torch.empty_like(X1)
+    ref = None
+    for (v, l, nv) in [(0, 0, 0), (4, 16, 2), (4, 8, 4), (2, 16, 2), (4, 32, 1), (0, 0, 0)]:
+        G.set_agg_mapping(v, l, nv)
+        ms = timeit(lambda: G.aggregate(plan, X1, "sum", "gcn", out=Y1), iters=5, warm=2)
+        same = None if ref is None else bool(torch.equal(ref, Y1))
+        ref = Y1.clone() if ref is None else ref
+        print(f" F=100 map vec={v} lanes={l} nv={nv}: {ms:.3f} ms identical={same}", flush=True)
+    G.set_agg_mapping(0, 0, 0)
+    Hh, Fh = 8, 32
+    Zs = torch.rand(g.n, Hh * Fh + 2 * Hh, device="cuda") * 2 - 1
+    Yg = torch.empty(g.n, Hh * Fh, device="cuda")
+    t = Zs[:, Hh * Fh + Hh:]
+    for (v, l, nv) in [(0, 0, 0), (8, 16, 2), (8, 8, 4), (4, 16, 2)]:
+        G.set_agg_mapping(v, l, nv)
+        ms = timeit(lambda: G.gat_aggregate(plan, Zs, t, Hh, Fh, out=Yg), iters=5, warm=2)
+        print(f" GAT 8x32 map vec={v} lanes={l} nv={nv}: {ms:.3f} ms", flush=True)
+    X2 = torch.rand(g.n, 256, device="cuda")
+    Y2 = torch.empty_like(X2)
+    for (v, l, nv) in [(0, 0, 0), (8, 16, 2), (8, 8, 4), (4, 16, 2)]:
+        G.set_agg_mapping(v, l, nv)
+        ms = timeit(lambda: G.aggregate(plan, X2, "sum", "one", out=Y2), iters=5, warm=2)
+        print(f" sum F=256 map vec={v} lanes={l} nv={nv}: {ms:.3f} ms", flush=True)
+    G.set_agg_mapping(0, 0, 0)
+
+
 def impls(cfg="C5"):
     """v8 per-group kernel vs v10 stream kernel on the bench's three aggregations."""
     t0 = time.time()
@@ -183,6 +214,8 @@ if __name__ == "__main__":
         tiles(sys.argv[sys.argv.index("--cfg") + 1] if "--cfg" in sys.argv else "C5")
     elif what == "impl":
         impls(sys.argv[sys.argv.index("--cfg") + 1] if "--cfg" in sys.argv else "C5")
+    elif what == "map100":
+        map100(sys.argv[sys.argv.index("--cfg") + 1] if "--cfg" in sys.argv else "C5")
     elif what == "map":
         mapsweep(sys.argv[sys.argv.index("--cfg") + 1] if "--cfg" in sys.argv else "C5")
     else:

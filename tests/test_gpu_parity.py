@@ -116,7 +116,8 @@ def test_aggregate_bit_exact_vs_order_replica(graphs, reduce, weight, ng, Tg):
     assert np.array_equal(Y.view(np.uint32), rep.view(np.uint32)), np.abs(Y - rep).max()
 
 
-@pytest.mark.parametrize("mapping", [(8, 8, 1), (4, 16, 1), (8, 16, 1), (2, 32, 1), (4, 32, 2), (1, 4, 1)])
+@pytest.mark.parametrize("mapping", [(8, 8, 1), (4, 16, 1), (8, 16, 1), (2, 32, 1), (4, 32, 2), (1, 4, 1),
+                                     (4, 16, 2), (4, 8, 4), (2, 16, 2), (8, 16, 2), (8, 8, 4)])
 @pytest.mark.parametrize("reduce", ["sum", "max"])
 def test_mapping_override_bit_exact(graphs, mapping, reduce):
     """a4 override (tuner hook): any admissible mapping / feature-chunk width
@@ -134,7 +135,7 @@ def test_mapping_override_bit_exact(graphs, mapping, reduce):
     assert np.array_equal(Y.view(np.uint32), rep.view(np.uint32)), np.abs(Y - rep).max()
 
 
-@pytest.mark.parametrize("mapping", [(8, 8, 1), (8, 16, 1), (4, 16, 1)])
+@pytest.mark.parametrize("mapping", [(8, 8, 1), (8, 16, 1), (4, 16, 1), (4, 16, 2), (4, 8, 4), (8, 16, 2), (8, 8, 4)])
 def test_gat_mapping_override_parity(graphs, mapping):
     g = graphs["hub"]
     Hh, Fh = 8, 32
@@ -257,6 +258,38 @@ def test_gat_invariants(graphs):
     Y1 = H(G.gat_aggregate(p1, T(Z1), T(gs.uniform(6, Hh, lo=-50, hi=50, seed=4)), Hh, Fh))
     assert np.array_equal(Y1[[0, 1, 3, 4, 5]], Z1[[5, 0, 1, 2, 3], :F])
     assert np.all(Y1[2] == 0)
+
+
+@pytest.mark.parametrize("case", ["loose_bound", "wide_spread", "neg_slope", "steep_slope"])
+def test_gat_softmax_reference(graphs, case):
+    """Reading R9 GAT: terms are exp(e - m) against the bound m =
+    LeakyReLU(max_u s_u + t_v); a bound looser than the slack (a huge score on
+    a node no row reads, or a row whose scores spread over ~400) makes the
+    group recompute against its exact max.  Parity holds either way."""
+    h = graphs["hub"]
+    # one extra node that no row reads (its score only moves the bound)
+    g = gs.from_rows([h.colidx[h.rowptr[v]:h.rowptr[v + 1]].tolist() for v in range(h.n)] + [[]])
+    Hh, Fh = 4, 8
+    F = Hh * Fh
+    Zs = gs.uniform(g.n, F + Hh, lo=-2, hi=2, seed=31)
+    t = gs.uniform(g.n, Hh, lo=-2, hi=2, seed=32)
+    slope = 0.2
+    outdeg = np.bincount(g.colidx, minlength=g.n)
+    if case == "loose_bound":
+        unread = np.flatnonzero(outdeg == 0)
+        assert unread.size > 0
+        Zs[unread[0], F:] = 1e4          # max_u s_u far above every row's scores
+    elif case == "wide_spread":
+        Zs[:, F:] *= 100.0               # scores spread over ~400 inside rows
+    elif case == "neg_slope":
+        slope = -0.5
+    else:
+        slope = 3.0
+    ref = oracle.gat_aggregate(g.rowptr, g.colidx, Zs, t, Hh, Fh, slope)
+    plan = G.Plan(g.rowptr, g.colidx, group_size=16, tile_groups=4)
+    Y = H(G.gat_aggregate(plan, T(Zs), T(t), Hh, Fh, slope))
+    assert np.all(np.isfinite(Y))
+    assert_close(Y, ref, what=f"gat {case}")
 
 
 def test_gat_layer_parity():
