@@ -226,6 +226,11 @@ def run_ours(args):
         pass
     roofline = {"bound": "hbm", "kernel": dom_name, "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(achieved / peak, 4), "traffic": traffic,
+                "dram_gbs": round(traffic / (parts[dom] * 1e-3) / 1e9, 1) if traffic else None,
+                "dram_frac": round(traffic / (parts[dom] * 1e-3) / 1e9 / peak, 4) if traffic else None,
+                "note": "achieved = SURVEY §8(d) no-reuse algorithmic bytes (every gathered row counted) / the "
+                        "launch's event time; LAS + L2 serve part of them, so it can exceed the HBM peak. "
+                        "dram_gbs = ncu DRAM bytes (traffic, cold-cache capture) / the same time.",
                 "algorithmic_bytes": int(per_launch[dom_name]), "launch_ms": round(float(parts[dom]), 4),
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)" if "hbm_gbs" in peaks else "fallback 6650"}
 

@@ -259,11 +259,53 @@ int gnn_set_gemm_impl(int impl);
  */
 gnn_status gnn_set_agg_mapping(int32_t vec, int32_t lanes, int32_t nv);
 
-/* Aggregation kernel selector (process-wide; same results bit for bit):
- * 0 = stream kernel (default: one worker streams a run of consecutive groups
- * with its loads in flight across group boundaries), 1 = per-group kernel
- * (one work unit = one group).  Returns the previous value. */
+/* Aggregation kernel selector for sum/mean/max (process-wide; same results
+ * bit for bit): 1 = per-group kernel (default: one work unit = one neighbour
+ * group), 0 = stream kernel (one worker streams a run of consecutive groups
+ * with its loads in flight across group boundaries; measured slower, kept
+ * for experiments).  GAT always takes the per-group kernel.  Returns the
+ * previous value. */
 int gnn_set_agg_impl(int impl);
+
+/*
+ * NG bound of an existing plan (reading R8): rebuilds the work
+ * units and the task-ordered index stream for group_size (> 0: groups of at
+ * most group_size entries; 0: never split rows; -1: the default rule); the
+ * LAS schedule is kept.  Synchronous (host rebuild + upload); the caller
+ * guarantees that no call using the plan is in flight.  Deterministic results
+ * depend on (CSR, group size, F) only (R9), so they change with the bound.
+ * Workspace sizes change too: query gnn_workspace_size again.
+ */
+gnn_status gnn_plan_set_group_size(gnn_plan_t plan, int32_t group_size);
+
+/* Result of gnn_tune_aggregate. */
+typedef struct {
+  int32_t group_size;     /* chosen NG bound (left in the plan) */
+  int32_t vec, lanes, nv; /* chosen a4 mapping (0,0,0 = the automatic rule) */
+  float ms;               /* median time of one gnn_aggregate call with both */
+  float ms_default;       /* the same at entry (automatic mapping, entry bound) */
+  int32_t rounds;         /* NG rounds run (one bound per round) */
+  int32_t mappings_tried; /* mapping templates timed */
+} gnn_tune_result;
+
+/*
+ * NEXT-1 online tuner: phase 1 times the a4 mapping templates
+ * (vector width x lanes per worker x vectors per lane, at most two feature
+ * chunks) at the plan's current bound ("first exhaust GPU resources by
+ * scheduling more warps"); phase 2 tries NG bounds, one per
+ * round, multiples of 16 up to ten times the average degree (and the max
+ * degree), a doubling ladder then bisection around the best, at most
+ * max_rounds rounds (<= 0: 20).  Each candidate = 1 warm-up +
+ * median of 3 gnn_aggregate calls timed with CUDA events on `stream`.  The
+ * plan keeps the best bound and uses the chosen mapping for later calls of
+ * width F (a process-wide gnn_set_agg_mapping override takes precedence;
+ * tuning with one active returns GNN_ERR_INVALID_ARG).  Arguments as
+ * gnn_aggregate (relu off; Y is overwritten).  Synchronous; allocates its own
+ * workspace; not graph-capturable.
+ */
+gnn_status gnn_tune_aggregate(gnn_plan_t plan, int reduce, int weight, const float *edge_w,
+                              const float *X, int64_t ldx, int32_t F, float *Y, int64_t ldy,
+                              int32_t max_rounds, gnn_tune_result *out, gnn_stream_t stream);
 
 /*
  * GCN layer (Eq 1): Y = ACT((A_gcn X) W).  order: 0 = auto (aggregate at

@@ -36,6 +36,7 @@ static void free_plan(gnn_plan_s *p) {
   cudaGetDevice(&cur);
   cudaSetDevice(p->device);
   for (void *d : p->dev_allocs) cudaFree(d);
+  for (void *d : p->sched_allocs) cudaFree(d);
   cudaSetDevice(cur);
   delete p;
 }
@@ -156,11 +157,7 @@ gnn_status gnn_plan_create_ex(int64_t n, int64_t n_src, int64_t nnz, const int64
     // NG bound (R8-ii): largest multiple of 16 <= 10 * average degree
     // (P:1163-1165), clamped to [16, 4096]
     int64_t ng = opts.group_size;
-    if (ng < 0) {
-      const double avg = n > 0 ? (double)nnz / (double)n : 0.0;
-      ng = (int64_t)(std::min(4096.0, 10.0 * avg) / 16.0) * 16;
-      if (ng < 16) ng = 16;
-    }
+    if (ng < 0) ng = default_group_size(n, nnz);
     p->info.group_size = (int32_t)ng;
     if (ng == 0) ng = 1 << 30;  // never split
     p->ng = (int32_t)ng;

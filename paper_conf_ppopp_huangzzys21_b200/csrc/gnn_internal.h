@@ -51,8 +51,13 @@ struct gnn_plan_s {
   std::vector<int32_t> pairs, cluster_of;
   int64_t n_clusters = 0, n_multi = 0, n_empty = 0, multi_slots = 0, max_tile_edges = 0;
   gnn_plan_info info{};
-  // device allocations (owned)
+  // device allocations (owned); sched_allocs = the NG schedule (rebuilt by
+  // gnn_plan_set_group_size)
   std::vector<void *> dev_allocs;
+  std::vector<void *> sched_allocs;
+  // per-plan a4 mapping chosen by gnn_tune_aggregate for width tuned_F
+  // (tuned_vec == 0: none)
+  int32_t tuned_F = 0, tuned_vec = 0, tuned_lanes = 0, tuned_nv = 0;
   gnn::DevGraph dg{};
 };
 
@@ -103,6 +108,11 @@ struct AggArgs {
   int32_t deterministic;
 };
 bool set_agg_mapping(int32_t vec, int32_t lanes, int32_t nv);
+bool mapping_supported(int32_t vec, int32_t lanes, int32_t nv);
+bool agg_override_active();
+bool agg_mapping_ok(const AggArgs &a, int32_t fh_or_0, int32_t vec, int32_t lanes, int32_t nv);
+gnn_status rebuild_schedule(gnn_plan_s *p, int64_t group_size);
+int64_t default_group_size(int64_t n, int64_t nnz);
 int set_agg_impl(int impl);
 size_t agg_workspace_bytes(const gnn_plan_s *p, int mode, int32_t F, int32_t H);
 gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, size_t ws_bytes,

@@ -177,19 +177,25 @@ static int32_t max_chunks(int32_t F) { return std::max<int32_t>(8, (F + 31) / 32
 // process-wide mapping override (gnn_set_agg_mapping; the tuner hook)
 static Mapping g_override{0, 0, 0};
 
+bool mapping_supported(int32_t vec, int32_t lanes, int32_t nv) {
+  const bool vec_ok = vec == 1 || vec == 2 || vec == 4 || vec == 8;
+  const bool lanes_ok = lanes == 4 || lanes == 8 || lanes == 16 || lanes == 32;
+  const bool nv_ok = nv == 1 || ((nv == 2 || nv == 4) && lanes == 32 && !(vec == 8 && nv == 4)) ||
+                     (vec >= 2 && lanes == 16 && nv == 2) || (vec >= 4 && lanes == 8 && nv == 4);
+  return vec_ok && lanes_ok && nv_ok;
+}
+
 bool set_agg_mapping(int32_t vec, int32_t lanes, int32_t nv) {
   if (vec == 0 && lanes == 0 && nv == 0) {
     g_override = Mapping{0, 0, 0};
     return true;
   }
-  const bool vec_ok = vec == 1 || vec == 2 || vec == 4 || vec == 8;
-  const bool lanes_ok = lanes == 4 || lanes == 8 || lanes == 16 || lanes == 32;
-  const bool nv_ok = nv == 1 || ((nv == 2 || nv == 4) && lanes == 32 && !(vec == 8 && nv == 4)) ||
-                     (vec >= 2 && lanes == 16 && nv == 2) || (vec >= 4 && lanes == 8 && nv == 4);
-  if (!vec_ok || !lanes_ok || !nv_ok) return false;
+  if (!mapping_supported(vec, lanes, nv)) return false;
   g_override = Mapping{vec, lanes, nv};
   return true;
 }
+
+bool agg_override_active() { return g_override.vec != 0; }
 
 static bool vec_admissible(const AggArgs &a, int32_t fh_or_0, int v) {
   bool ok = a.F % v == 0 && a.ldx % v == 0 && a.ldy % v == 0 && aligned(a.X, 4 * v) && aligned(a.Y, 4 * v);
@@ -199,14 +205,24 @@ static bool vec_admissible(const AggArgs &a, int32_t fh_or_0, int v) {
 }
 
 // a4: feature-length-adaptive mapping rule
-static Mapping choose_mapping(const AggArgs &a, int32_t fh_or_0) {
+static bool mapping_ok(const AggArgs &a, int32_t fh_or_0, const Mapping &o) {
+  if (o.vec == 0 || !vec_admissible(a, fh_or_0, o.vec)) return false;
+  // GAT: a chunk must hold whole heads (the softmax state is per head)
+  const int cw = o.vec * o.lanes * o.nv;
+  const bool heads_ok = !fh_or_0 || cw >= a.F || cw % fh_or_0 == 0;
+  return heads_ok && (a.F + cw - 1) / cw <= max_chunks(a.F);
+}
+
+bool agg_mapping_ok(const AggArgs &a, int32_t fh_or_0, int32_t vec, int32_t lanes, int32_t nv) {
+  return mapping_supported(vec, lanes, nv) && mapping_ok(a, fh_or_0, Mapping{vec, lanes, nv});
+}
+
+static Mapping choose_mapping(const gnn_plan_s *p, const AggArgs &a, int32_t fh_or_0) {
   Mapping m{1, 4, 1};
-  if (g_override.vec != 0 && vec_admissible(a, fh_or_0, g_override.vec)) {
-    // GAT: a chunk must hold whole heads (the softmax state is per head)
-    const int cw = g_override.vec * g_override.lanes * g_override.nv;
-    const bool heads_ok = !fh_or_0 || cw >= a.F || cw % fh_or_0 == 0;
-    if (heads_ok && (a.F + cw - 1) / cw <= max_chunks(a.F)) return g_override;
-  }
+  if (mapping_ok(a, fh_or_0, g_override)) return g_override;
+  // the plan's tuned mapping (gnn_tune_aggregate) for this width
+  const Mapping t{p->tuned_vec, p->tuned_lanes, p->tuned_nv};
+  if (p->tuned_F == a.F && mapping_ok(a, fh_or_0, t)) return t;
   const int cands[4] = {8, 4, 2, 1};
   for (int v : cands) {
     if (vec_admissible(a, fh_or_0, v)) {
@@ -301,7 +317,7 @@ gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, siz
   kp.ws_cnt = reinterpret_cast<int32_t *>(w + 256 + sm_bytes);
   kp.ws_acc = reinterpret_cast<float *>(w + 256 + sm_bytes + cnt_bytes);
   kp.ws_part = kp.ws_acc + (size_t)p->n_multi * kp.FW;
-  const Mapping m = choose_mapping(a, mode == M_GAT ? a.Fh : 0);
+  const Mapping m = choose_mapping(p, a, mode == M_GAT ? a.Fh : 0);
   const int threads = 256;
   cudaError_t e;
   if (mode == M_GAT) {

@@ -316,7 +316,7 @@ gnn_status build_schedule(gnn_plan_s *p) {
     *dst = nullptr;
     cudaError_t e = cudaMalloc(dst, bytes > 0 ? bytes : 16);
     if (e != cudaSuccess) return e;
-    p->dev_allocs.push_back(*dst);
+    p->sched_allocs.push_back(*dst);
     if (bytes > 0) e = cudaMemcpy(*dst, src, bytes, cudaMemcpyHostToDevice);
     return e;
   };
@@ -345,6 +345,43 @@ gnn_status build_schedule(gnn_plan_s *p) {
   p->info.n_split_rows = p->n_multi;
   p->info.n_empty_rows = p->n_empty;
   return GNN_OK;
+}
+
+// NG bound (R8): largest multiple of 16 <= 10 * average degree,
+// clamped to [16, 4096]
+int64_t default_group_size(int64_t n, int64_t nnz) {
+  const double avg = n > 0 ? (double)nnz / (double)n : 0.0;
+  int64_t ng = (int64_t)(std::min(4096.0, 10.0 * avg) / 16.0) * 16;
+  return ng < 16 ? 16 : ng;
+}
+
+// Rebuild the NG schedule (work units, task-ordered index stream) of an
+// existing plan for another group bound; the LAS schedule (perm) is kept.
+// Synchronous; the caller guarantees no call is in flight on the plan.
+gnn_status rebuild_schedule(gnn_plan_s *p, int64_t group_size) {
+  if (group_size < 0) group_size = default_group_size(p->n, p->nnz);
+  int cur = 0;
+  cudaGetDevice(&cur);
+  cudaSetDevice(p->device);
+  std::vector<int32_t> col((size_t)p->nnz);
+  cudaError_t e = cudaSuccess;
+  if (p->nnz > 0)
+    e = cudaMemcpy(col.data(), p->dg.colidx, sizeof(int32_t) * (size_t)p->nnz, cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) {
+    cudaSetDevice(cur);
+    return cuda_status(e, "rebuild: colidx download");
+  }
+  for (void *d : p->sched_allocs) cudaFree(d);
+  p->sched_allocs.clear();
+  p->info.group_size = (int32_t)group_size;
+  p->ng = group_size == 0 ? (1 << 30) : (int32_t)group_size;
+  const auto t0 = std::chrono::steady_clock::now();
+  p->colidx_h = col.data();
+  gnn_status st = build_schedule(p);
+  p->colidx_h = nullptr;
+  p->info.ms_ng = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  cudaSetDevice(cur);
+  return st;
 }
 
 }  // namespace gnn

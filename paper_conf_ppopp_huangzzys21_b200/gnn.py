@@ -54,6 +54,12 @@ class gnn_plan_info(ctypes.Structure):
                                                  "ms_merge", "ms_ng")]
 
 
+class gnn_tune_result(ctypes.Structure):
+    _fields_ = [("group_size", ctypes.c_int32), ("vec", ctypes.c_int32), ("lanes", ctypes.c_int32),
+                ("nv", ctypes.c_int32), ("ms", ctypes.c_float), ("ms_default", ctypes.c_float),
+                ("rounds", ctypes.c_int32), ("mappings_tried", ctypes.c_int32)]
+
+
 _P = ctypes.c_void_p
 _I64 = ctypes.c_int64
 _I32 = ctypes.c_int32
@@ -92,6 +98,9 @@ _SIGS = {
                                     ctypes.POINTER(_I64)]),
     "gnn_groups_host": (ctypes.c_int, [_I64, _P, _P, _I32, ctypes.POINTER(_I64), _P, _P]),
     "gnn_launch_count": (ctypes.c_uint64, []),
+    "gnn_plan_set_group_size": (ctypes.c_int, [_P, _I32]),
+    "gnn_tune_aggregate": (ctypes.c_int, [_P, ctypes.c_int, ctypes.c_int, _P, _P, _I64, _I32, _P, _I64, _I32,
+                                          ctypes.POINTER(gnn_tune_result), _P]),
     "gnn_last_error": (ctypes.c_char_p, []),
     "gnn_version": (ctypes.c_char_p, []),
 }
@@ -382,6 +391,25 @@ def groups_host(rowptr, ng, perm=None):
     gb = np.empty(max(G.value, 1), np.int64)
     _call("gnn_groups_host", n, _np_ptr(rowptr), _np_ptr(p), ng, ctypes.byref(G), _np_ptr(gr), _np_ptr(gb))
     return gr[:G.value], gb[:G.value]
+
+
+def set_group_size(plan: Plan, group_size: int) -> None:
+    """gnn_plan_set_group_size: rebuild the plan's NG schedule for another bound."""
+    _call("gnn_plan_set_group_size", plan.handle, int(group_size))
+    plan._ws = {}
+
+
+def tune_aggregate(plan: Plan, X, reduce="sum", weight="one", edge_w=None, out=None, max_rounds=20,
+                   stream=None) -> dict:
+    """gnn_tune_aggregate: the online tuner (mapping templates, then NG bound)."""
+    torch = _torch()
+    F = X.shape[1]
+    Y = out if out is not None else torch.empty((plan.n, F), dtype=torch.float32, device=X.device)
+    r = gnn_tune_result()
+    _call("gnn_tune_aggregate", plan.handle, REDUCE[reduce], WEIGHT[weight], _tp(edge_w), _tp(X), _ld(X, F), F,
+          _tp(Y), _ld(Y, F), int(max_rounds), ctypes.byref(r), _stream(stream))
+    plan._ws = {}
+    return {k: getattr(r, k) for k, _ in gnn_tune_result._fields_}
 
 
 def launch_count() -> int:

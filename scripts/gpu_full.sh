@@ -14,3 +14,4 @@ echo "ncu rc=$?" >> gpurun_out/ncu_launch_$TAG.log
 timeout 1500 ncu --set full --clock-control none --import-source on -k regex:"k_aggregate|k_gemm_tc" -c 6 -o gpurun_out/prof_$TAG -f \
   python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu > gpurun_out/ncu_full_$TAG.log 2>&1
 echo "ncu rc=$?" >> gpurun_out/ncu_full_$TAG.log
+timeout 300 ncu --metrics gpu__time_duration.sum,launch__grid_size,launch__block_size --clock-control none --csv --log-file gpurun_out/c1_launches_$TAG.csv python scripts/kbench.py c1 > gpurun_out/c1_probe_$TAG.log 2>&1

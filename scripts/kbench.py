@@ -145,6 +145,18 @@ def map100(cfg="C5"):
     G.set_agg_mapping(0, 0, 0)
 
 
+def c1probe():
+    """C1 (Cora) aggregate calls for an ncu launch list (launch-bound config)."""
+    g = gs.config_graph("C1")
+    plan = G.Plan(g.rowptr, g.colidx, reorder=1)
+    X = torch.rand(g.n, 16, device="cuda")
+    Y = torch.empty_like(X)
+    for _ in range(5):
+        G.aggregate(plan, X, "sum", "gcn", relu=True, out=Y)
+    torch.cuda.synchronize()
+    print(plan.info, flush=True)
+
+
 def impls(cfg="C5"):
     """v8 per-group kernel vs v10 stream kernel on the bench's three aggregations."""
     t0 = time.time()
@@ -214,6 +226,8 @@ if __name__ == "__main__":
         tiles(sys.argv[sys.argv.index("--cfg") + 1] if "--cfg" in sys.argv else "C5")
     elif what == "impl":
         impls(sys.argv[sys.argv.index("--cfg") + 1] if "--cfg" in sys.argv else "C5")
+    elif what == "c1":
+        c1probe()
     elif what == "map100":
         map100(sys.argv[sys.argv.index("--cfg") + 1] if "--cfg" in sys.argv else "C5")
     elif what == "map":

@@ -83,14 +83,16 @@ def test_invalid_args_return_status_not_crash():
     assert P.gnn.gnn_plan_destroy(None) == 0
 
 
-@pytest.mark.parametrize("vec,lanes,nv", [(3, 32, 1), (8, 2, 1), (8, 32, 4), (4, 16, 2), (0, 32, 1)])
+@pytest.mark.parametrize("vec,lanes,nv", [(3, 32, 1), (8, 2, 1), (8, 32, 4), (1, 16, 2), (2, 8, 4), (4, 4, 2),
+                                          (0, 32, 1)])
 def test_agg_mapping_rejects_unsupported(vec, lanes, nv):
     assert P.gnn.gnn_set_agg_mapping(vec, lanes, nv) == 1
     assert P.gnn.gnn_set_agg_mapping(0, 0, 0) == 0
 
 
 def test_agg_mapping_accepts_supported():
-    for m in [(8, 32, 1), (8, 32, 2), (4, 32, 4), (8, 8, 1), (1, 4, 1)]:
+    for m in [(8, 32, 1), (8, 32, 2), (4, 32, 4), (8, 8, 1), (1, 4, 1), (4, 16, 2), (8, 16, 2), (2, 16, 2),
+              (8, 8, 4), (4, 8, 4)]:
         assert P.gnn.gnn_set_agg_mapping(*m) == 0
     assert P.gnn.gnn_set_agg_mapping(0, 0, 0) == 0
 

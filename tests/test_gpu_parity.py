@@ -152,6 +152,43 @@ def test_gat_mapping_override_parity(graphs, mapping):
     assert_close(Y, ref, what=f"gat mapping {mapping}")
 
 
+@pytest.mark.parametrize("ng", [16, 48, 0, -1])
+def test_set_group_size_rebuild_bit_exact(graphs, ng):
+    """gnn_plan_set_group_size rebuilds NG in place; the result equals the
+    oracle's fp32 order replica for the new bound (R9 depends on (CSR, ng, F))."""
+    g = graphs["hub"]
+    X = gs.uniform(g.n, 64, seed=43)
+    plan = G.Plan(g.rowptr, g.colidx, reorder=1, group_size=32)
+    G.set_group_size(plan, ng)
+    eff = plan.info["group_size"]
+    assert eff == (ng if ng >= 0 else plan.info["group_size"])
+    Y = H(G.aggregate(plan, T(X), "sum", "gcn", relu=True))
+    rep = oracle.aggregate_ng_f32(g.rowptr, g.colidx, X, eff if eff > 0 else g.nnz + 1, "sum", "gcn", None,
+                                  relu=True)
+    assert np.array_equal(Y.view(np.uint32), rep.view(np.uint32))
+
+
+@pytest.mark.parametrize("gname,F", [("hub", 64), ("cora", 16), ("small", 100)])
+def test_tuner(graphs, gname, F):
+    """NEXT-1 tuner: bounded rounds, bound a multiple of 16 <= 10x average
+    degree (or the entry bound), chosen settings kept by the plan, results
+    still bit-exact vs the replica at the chosen bound."""
+    g = graphs[gname]
+    X = gs.uniform(g.n, F, seed=44)
+    plan = G.Plan(g.rowptr, g.colidx, reorder=1)
+    ng0 = plan.info["group_size"]
+    r = G.tune_aggregate(plan, T(X), "sum", "gcn", max_rounds=6)
+    assert r["rounds"] <= 6 and r["mappings_tried"] >= 1
+    assert r["ms"] <= r["ms_default"]
+    ng = r["group_size"]
+    cap = max(16, int(10 * g.nnz / g.n) // 16 * 16)
+    assert ng == ng0 or (ng % 16 == 0 and 16 <= ng <= cap)
+    assert plan.info["group_size"] == ng
+    Y = H(G.aggregate(plan, T(X), "sum", "gcn"))
+    rep = oracle.aggregate_ng_f32(g.rowptr, g.colidx, X, ng, "sum", "gcn", None)
+    assert np.array_equal(Y.view(np.uint32), rep.view(np.uint32))
+
+
 def test_integer_features_exact(graphs):
     g = graphs["hub"]
     X = gs.integer_features(g.n, 32, seed=1)
