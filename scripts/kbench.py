@@ -145,6 +145,18 @@ def map100(cfg="C5"):
     G.set_agg_mapping(0, 0, 0)
 
 
+def tune():
+    """NEXT-1 tuner on the config graphs: default vs tuned (bound, mapping)."""
+    for cfg, F in [("C1", 16), ("C2", 64), ("C5", 100), ("C5", 256)]:
+        g = gs.config_graph(cfg)
+        plan = G.Plan(g.rowptr, g.colidx, reorder=1)
+        X = torch.rand(g.n, F, device="cuda")
+        t0 = time.time()
+        r = G.tune_aggregate(plan, X, "sum", "gcn")
+        print(f" {cfg} F={F}: {r} in {time.time() - t0:.1f}s", flush=True)
+        del plan
+
+
 def c1probe():
     """C1 (Cora) aggregate calls for an ncu launch list (launch-bound config)."""
     g = gs.config_graph("C1")
@@ -226,6 +238,8 @@ if __name__ == "__main__":
         tiles(sys.argv[sys.argv.index("--cfg") + 1] if "--cfg" in sys.argv else "C5")
     elif what == "impl":
         impls(sys.argv[sys.argv.index("--cfg") + 1] if "--cfg" in sys.argv else "C5")
+    elif what == "tune":
+        tune()
     elif what == "c1":
         c1probe()
     elif what == "map100":
