@@ -74,6 +74,9 @@ def lib():
             "orc_neighbor_groups": (_i64, [_i64, _p, _p, _i32, _p, _p]),
             "orc_partition_rows": (None, [_i64, _p, _i32, _p]),
             "orc_forget_degrees": (None, []),
+            "orc_sample_neighbors": (None, [_i64, _p, _p, _i32, ctypes.c_uint64, _p]),
+            "orc_sage_lstm": (ctypes.c_int, [_i64, _p, _i64, _i32, _p, _i32, _p, _p, _p, _p, _i32, _p, _p, _p,
+                                             _i32, _p, _i64, _p, _i64]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -278,3 +281,31 @@ def partition_rows(rowptr, P):
     b = np.empty(P + 1, np.int64)
     lib().orc_partition_rows(len(rowptr) - 1, _ptr(rowptr), P, _ptr(b))
     return b
+
+
+def sample_neighbors(rowptr, colidx, T=16, seed=0):
+    """NEXT-3 sampling (reading R13): [n, T] int32 node ids, -1 for empty rows."""
+    rowptr, colidx = _csr(rowptr, colidx)
+    n = len(rowptr) - 1
+    table = np.empty((n, T), np.int32)
+    lib().orc_sample_neighbors(n, _ptr(rowptr), _ptr(colidx), T, seed, _ptr(table))
+    return table
+
+
+def sage_lstm(X, table, W_ih, W_hh, b_ih, b_hh, W_self, W_neigh, bias=None, rows=None):
+    """NEXT-3 GraphSAGE-LSTM layer, fp64 (Fig 6 base implementation): returns [n or len(rows), F_out]."""
+    X = _f32(X)
+    table = np.ascontiguousarray(table, dtype=np.int32)
+    n, T = table.shape
+    F4, f_in = W_ih.shape
+    F = F4 // 4
+    F_out = W_self.shape[0]
+    r, nr = _rows(rows)
+    m = nr if rows is not None else n
+    Y = np.empty((m, F_out), np.float32)
+    W_ih, W_hh, b_ih, b_hh, W_self, W_neigh = (_f32(a) for a in (W_ih, W_hh, b_ih, b_hh, W_self, W_neigh))
+    b = _f32(bias) if bias is not None else None
+    assert lib().orc_sage_lstm(n, _ptr(X), X.shape[1], f_in, _ptr(table), T, _ptr(W_ih), _ptr(W_hh), _ptr(b_ih),
+                               _ptr(b_hh), F, _ptr(W_self), _ptr(W_neigh), _ptr(b), F_out, _ptr(r), nr, _ptr(Y),
+                               F_out) == 0
+    return Y

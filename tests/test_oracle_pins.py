@@ -522,3 +522,105 @@ def test_partition_rows():
         nnz = np.diff(g.rowptr[b])
         assert nnz.sum() == E
         assert np.all(nnz <= E / P + maxd)
+
+
+# --------------------------------------------------------------------------- #
+# NEXT-3 GraphSAGE-LSTM (Fig 6; reading R13)
+# --------------------------------------------------------------------------- #
+def _lstm_params(f_in, F, F_out, seed, scale=0.3):
+    rng = np.random.default_rng(seed)
+    u = lambda *s: (rng.uniform(-scale, scale, size=s)).astype(np.float32)  # noqa: E731
+    return dict(W_ih=u(4 * F, f_in), W_hh=u(4 * F, F), b_ih=u(4 * F), b_hh=u(4 * F), W_self=u(F_out, f_in),
+                W_neigh=u(F_out, F), bias=u(F_out))
+
+
+def test_sage_lstm_matches_torch_lstm():
+    """The LSTM cell chain (Fig 6, gate blocks i, f, z, o) against PyTorch's
+    nn.LSTM in fp64 on the same sampled sequences (a library routine), then
+    the SAGE combine y = W_self x_v + W_neigh h_T + b by numpy."""
+    torch = pytest.importorskip("torch")
+    g = gs.random_small(60, avg_deg=6, seed=11)
+    f_in, F, F_out, T = 12, 8, 5, 7
+    X = gs.uniform(g.n, f_in, seed=12)
+    P = _lstm_params(f_in, F, F_out, 13)
+    table = oracle.sample_neighbors(g.rowptr, g.colidx, T, seed=5)
+    Y = oracle.sage_lstm(X, table, **P)
+    lstm = torch.nn.LSTM(f_in, F, batch_first=True).double()
+    with torch.no_grad():
+        lstm.weight_ih_l0.copy_(torch.from_numpy(P["W_ih"].astype(np.float64)))
+        lstm.weight_hh_l0.copy_(torch.from_numpy(P["W_hh"].astype(np.float64)))
+        lstm.bias_ih_l0.copy_(torch.from_numpy(P["b_ih"].astype(np.float64)))
+        lstm.bias_hh_l0.copy_(torch.from_numpy(P["b_hh"].astype(np.float64)))
+    deg = np.diff(g.rowptr)
+    ref = np.empty_like(Y, dtype=np.float64)
+    for v in range(g.n):
+        h = np.zeros(F)
+        if deg[v] > 0:
+            seq = torch.from_numpy(X[table[v]].astype(np.float64))[None]
+            with torch.no_grad():
+                _, (hT, _) = lstm(seq)
+            h = hT[0, 0].numpy()
+        ref[v] = P["W_self"].astype(np.float64) @ X[v] + P["W_neigh"].astype(np.float64) @ h + P["bias"]
+    assert np.allclose(Y, ref, rtol=1e-6, atol=1e-7)
+
+
+def test_sage_lstm_zero_weights_closed_form():
+    """W = R = 0: every cell sees only its biases, c_t = s_f c_{t-1} + s_i tanh(b_z),
+    so c_T = s_i tanh(b_z) (1 - s_f^T) / (1 - s_f) and h_T = s_o tanh(c_T)."""
+    g = gs.random_small(40, avg_deg=3, seed=2, allow_empty=True)
+    f_in, F, T = 6, 4, 16
+    P = _lstm_params(f_in, F, F, 3, scale=1.0)
+    P["W_ih"][:] = 0
+    P["W_hh"][:] = 0
+    P["W_self"][:] = 0
+    P["W_neigh"] = np.eye(F, dtype=np.float32)
+    P["bias"][:] = 0
+    X = gs.uniform(g.n, f_in, seed=4)
+    table = oracle.sample_neighbors(g.rowptr, g.colidx, T, seed=1)
+    Y = oracle.sage_lstm(X, table, **P)
+    b = P["b_ih"].astype(np.float64) + P["b_hh"]
+    sig = lambda x: 1 / (1 + np.exp(-x))  # noqa: E731
+    si, sf, sz, so = sig(b[:F]), sig(b[F:2 * F]), np.tanh(b[2 * F:3 * F]), sig(b[3 * F:])
+    cT = si * sz * (1 - sf ** T) / (1 - sf)
+    hT = so * np.tanh(cT)
+    deg = np.diff(g.rowptr)
+    assert np.allclose(Y[deg > 0], hT[None, :], rtol=1e-6, atol=1e-7)
+    assert np.all(Y[deg == 0] == 0)
+
+
+def test_sage_lstm_empty_rows_and_single_step():
+    """Empty rows: h_T = 0, y = W_self x_v + b.  T = 1: h_1 = s(o) tanh(s(i) tanh(z))
+    with the gate pre-activations computed by a dense matmul of the one neighbour."""
+    g = gs.from_rows([[1], [], [0], [2]])
+    f_in, F, F_out = 3, 2, 2
+    P = _lstm_params(f_in, F, F_out, 9, scale=0.8)
+    X = gs.uniform(g.n, f_in, seed=10)
+    table = oracle.sample_neighbors(g.rowptr, g.colidx, 1, seed=0)
+    assert table.ravel().tolist() == [1, -1, 0, 2]
+    Y = oracle.sage_lstm(X, table, **P)
+    W = {k: v.astype(np.float64) for k, v in P.items()}
+    assert np.allclose(Y[1], W["W_self"] @ X[1] + W["bias"], rtol=1e-6, atol=1e-7)
+    sig = lambda x: 1 / (1 + np.exp(-x))  # noqa: E731
+    for v, u in ((0, 1), (2, 0), (3, 2)):
+        a = W["W_ih"] @ X[u] + W["b_ih"] + W["b_hh"]
+        h = sig(a[3 * F:]) * np.tanh(sig(a[:F]) * np.tanh(a[2 * F:3 * F]))
+        assert np.allclose(Y[v], W["W_self"] @ X[v] + W["W_neigh"] @ h + W["bias"], rtol=1e-6, atol=1e-7)
+
+
+def test_sample_neighbors_uniform_with_replacement():
+    """Reading R13: every sample is a neighbour of its row; degree-1 rows repeat
+    their neighbour; on a degree-4 row, T = 4000 samples hit each neighbour
+    with frequency 1/4 (within 5 sigma); different seeds give different tables."""
+    g = gs.from_rows([[3, 5, 7, 9], [2], []])
+    t = oracle.sample_neighbors(g.rowptr, g.colidx, 4000, seed=123)
+    cnt = np.array([(t[0] == u).sum() for u in (3, 5, 7, 9)])
+    assert cnt.sum() == 4000
+    assert np.all(np.abs(cnt - 1000) < 5 * math.sqrt(4000 * 0.25 * 0.75))
+    assert np.all(t[1] == 2) and np.all(t[2] == -1)
+    g2 = gs.random_small(200, avg_deg=8, seed=5)
+    a = oracle.sample_neighbors(g2.rowptr, g2.colidx, 16, seed=1)
+    b = oracle.sample_neighbors(g2.rowptr, g2.colidx, 16, seed=2)
+    for v in range(g2.n):
+        nb = set(g2.colidx[g2.rowptr[v]:g2.rowptr[v + 1]].tolist())
+        assert set(a[v].tolist()) <= (nb if nb else {-1})
+    assert (a != b).mean() > 0.5
