@@ -155,7 +155,8 @@ typedef enum {
   GNN_OP_GAT_AGGREGATE = 1, /* f_out = H * Fh, heads = H */
   GNN_OP_EDGECONV = 2,      /* f_in, f_out */
   GNN_OP_GCN_LAYER = 3,     /* f_in, f_out */
-  GNN_OP_GAT_LAYER = 4      /* f_in, f_out = H * Fh, heads = H */
+  GNN_OP_GAT_LAYER = 4,     /* f_in, f_out = H * Fh, heads = H */
+  GNN_OP_SAGE_LSTM_LAYER = 5 /* f_in, f_out = F_out, heads = T (hidden F = 32) */
 } gnn_op;
 
 /* Bytes of device workspace a call needs (may be 0; pass NULL then).  The
@@ -381,6 +382,50 @@ gnn_status gnn_groups_host(int64_t n, const int64_t *rowptr_h, const int32_t *pe
                            int64_t *n_groups, int32_t *grp_row_h, int64_t *grp_beg_h);
 
 /* Number of kernels this library launched since load (for bench accounting). */
+/*
+ * NEXT-3 GraphSAGE-LSTM (Fig 6; setting P:1366-1367: 32 in /
+ * 32 out, 16 sampled neighbours; reading R13).
+ *
+ * gnn_sample_neighbors: table[v*T + t] (device, [n, T] int32) = the t-th
+ * neighbour of row v drawn uniformly with replacement by the counter-based
+ * rule colidx[rowptr[v] + fmix64(seed + (v*T + t + 1) * 0x9E3779B97F4A7C15)
+ * mod d_v]; -1 for every sample of an empty row.  1 <= T <= 32.
+ */
+gnn_status gnn_sample_neighbors(gnn_plan_t plan, int32_t T, uint64_t seed, int32_t *table,
+                                gnn_stream_t stream);
+
+/*
+ * Fused LSTM aggregation with sparse fetching + SAGE combine:
+ * h_T(v) = LSTM over the rows GS[u_1..u_T] of v's sampled neighbours (h_0 =
+ * c_0 = 0; cell of Fig 6: i, f, o sigmoid, z tanh, c = f c + i z,
+ * h = o tanh(c)); y_v = GS[v][4F : 4F+F_out] + W_neigh h_T(v).
+ * GS: [n_src, ldg] device rows = the pre-transformed features (redundancy
+ * bypass): GS[u][4j+g] = gate g (i, f, z, o) of hidden unit j of
+ * x_u W_ih^T + b_ih + b_hh, and GS[u][4F+o] = (x_u W_self^T + b)[o].
+ * R = W_hh [4F, F] (gate blocks i, f, z, o, PyTorch layout), W_neigh
+ * [F_out, F].  F (hidden) must be 32 (else GNN_ERR_UNSUPPORTED), 1 <= F_out
+ * <= 32, 1 <= T <= 32; GS 16-byte aligned, ldg a multiple of 4.
+ * Empty rows: h_T = 0.  Y: [n, ldy].
+ */
+gnn_status gnn_sage_lstm_aggregate(gnn_plan_t plan, const int32_t *table, int32_t T,
+                                   const float *GS, int64_t ldg, int32_t F, const float *R,
+                                   const float *W_neigh, int32_t F_out, float *Y, int64_t ldy,
+                                   gnn_stream_t stream);
+
+/*
+ * One GraphSAGE-LSTM layer: y_v = W_self x_v + W_neigh LSTM(x_{u_1..u_T}) + b,
+ * computed as [W_ih | W_self] folded into one tensor-core GEMM (3xTF32) over
+ * the nodes (GS, above), gnn_sample_neighbors(seed), then the fused cell
+ * kernel.  W_ih [4F, f_in], W_hh [4F, F], b_ih/b_hh [4F], W_self [F_out,
+ * f_in], W_neigh [F_out, F], bias [F_out] (nullable).  Workspace:
+ * gnn_workspace_size(plan, GNN_OP_SAGE_LSTM_LAYER, f_in, F_out, T).
+ */
+gnn_status gnn_sage_lstm_layer(gnn_plan_t plan, const float *X, int64_t ldx, int32_t f_in,
+                               const float *W_ih, const float *W_hh, const float *b_ih,
+                               const float *b_hh, const float *W_self, const float *W_neigh,
+                               const float *bias, int32_t F, int32_t F_out, int32_t T, uint64_t seed,
+                               float *Y, int64_t ldy, void *ws, size_t ws_bytes, gnn_stream_t stream);
+
 uint64_t gnn_launch_count(void);
 
 const char *gnn_last_error(void);

@@ -309,6 +309,16 @@ static size_t ws_edgeconv_head(int64_t n, int32_t f_in, int32_t f_out) {
 }
 static int32_t ld8(int32_t f) { return (f + 7) / 8 * 8; }
 
+// GraphSAGE-LSTM layer workspace: [gemm ws][Wcat f_in x ld][bcat ld][table n x T][GS n_src x ld]
+static constexpr int32_t kSageF = 32;
+static size_t ws_sage_lstm(const gnn_plan_s *p, int32_t f_in, int32_t f_out, int32_t T) {
+  const int32_t ld = 4 * kSageF + f_out;
+  const int32_t ldp = (ld + 7) / 8 * 8;  // GS row stride: 16-byte aligned rows for the cell kernel
+  return align256(gemm_tc_workspace(p->n_src, f_in, ld)) + align256(sizeof(float) * (size_t)f_in * ld) +
+         align256(sizeof(float) * (size_t)ld) + align256(sizeof(int32_t) * (size_t)p->n * (size_t)(T > 0 ? T : 0)) +
+         align256(sizeof(float) * (size_t)p->n_src * ldp);
+}
+
 size_t gnn_workspace_size(gnn_plan_t p, int op, int32_t f_in, int32_t f_out, int32_t heads) {
   if (!p) return 0;
   switch (op) {
@@ -326,6 +336,7 @@ size_t gnn_workspace_size(gnn_plan_t p, int op, int32_t f_in, int32_t f_out, int
                        align256(sizeof(float) * (size_t)p->n * ld8(f_in)) + agg_workspace_bytes(p, 0, f_in, 0);
       return a > b ? a : b;
     }
+    case GNN_OP_SAGE_LSTM_LAYER: return ws_sage_lstm(p, f_in, f_out, heads);
     default: return 0;
   }
 }
@@ -709,6 +720,82 @@ gnn_status gnn_groups_host(int64_t n, const int64_t *rowptr_h, const int32_t *pe
     if (grp_row_h) std::memcpy(grp_row_h, gr.data(), sizeof(int32_t) * gr.size());
     if (grp_beg_h) std::memcpy(grp_beg_h, gb.data(), sizeof(int64_t) * gb.size());
     return GNN_OK;
+  })
+}
+
+
+
+// ---------------------------------------------------------------------------
+// NEXT-3 GraphSAGE-LSTM (Fig 6, reading R13)
+// ---------------------------------------------------------------------------
+gnn_status gnn_sample_neighbors(gnn_plan_t p, int32_t T, uint64_t seed, int32_t *table, gnn_stream_t stream) {
+  GNN_TRY({
+    if (!p || (!table && p->n > 0)) return check(false, "plan/table is NULL");
+    if (T < 1 || T > 32) return check(false, "T must be in [1, 32]");
+    return cuda_status(launch_sample_neighbors(p, T, seed, table, (cudaStream_t)stream), "sample neighbors");
+  })
+}
+
+gnn_status gnn_sage_lstm_aggregate(gnn_plan_t p, const int32_t *table, int32_t T, const float *GS, int64_t ldg,
+                                   int32_t F, const float *R, const float *W_neigh, int32_t F_out, float *Y,
+                                   int64_t ldy, gnn_stream_t stream) {
+  GNN_TRY({
+    if (!p) return check(false, "plan is NULL");
+    if (F != kSageF) {
+      set_error("gnn_sage_lstm_aggregate: hidden size F must be 32");
+      return GNN_ERR_UNSUPPORTED;
+    }
+    if (T < 1 || T > 32) return check(false, "T must be in [1, 32]");
+    if (F_out < 1 || F_out > 32) {
+      set_error("gnn_sage_lstm_aggregate: F_out must be in [1, 32]");
+      return GNN_ERR_UNSUPPORTED;
+    }
+    if (p->n > 0 && (!table || !GS || !R || !W_neigh || !Y)) return check(false, "NULL argument");
+    if (ldg < 4 * F + F_out || ldg % 4 != 0 || ldy < F_out) return check(false, "ldg < 4F+F_out (or not a multiple of 4) or ldy < F_out");
+    if (reinterpret_cast<uintptr_t>(GS) % 16 != 0) return check(false, "GS must be 16-byte aligned");
+    if (overlaps(GS, span_bytes(p->n_src, ldg, 4 * F + F_out), Y, span_bytes(p->n, ldy, F_out)))
+      return check(false, "GS and Y overlap");
+    return cuda_status(launch_sage_lstm(p, table, T, GS, ldg, R, W_neigh, F_out, Y, ldy, (cudaStream_t)stream),
+                       "sage lstm");
+  })
+}
+
+gnn_status gnn_sage_lstm_layer(gnn_plan_t p, const float *X, int64_t ldx, int32_t f_in, const float *W_ih,
+                               const float *W_hh, const float *b_ih, const float *b_hh, const float *W_self,
+                               const float *W_neigh, const float *bias, int32_t F, int32_t F_out, int32_t T,
+                               uint64_t seed, float *Y, int64_t ldy, void *ws, size_t ws_bytes,
+                               gnn_stream_t stream) {
+  GNN_TRY({
+    if (!p) return check(false, "plan is NULL");
+    if (F != kSageF) {
+      set_error("gnn_sage_lstm_layer: hidden size F must be 32");
+      return GNN_ERR_UNSUPPORTED;
+    }
+    if (f_in < 1 || T < 1 || T > 32 || F_out < 1 || F_out > 32) return check(false, "f_in < 1, T or F_out out of [1, 32]");
+    if (!X || !W_ih || !W_hh || !b_ih || !b_hh || !W_self || !W_neigh || !Y) return check(false, "NULL argument");
+    if (ldx < f_in || ldy < F_out) return check(false, "leading dimension too small");
+    const size_t need = ws_sage_lstm(p, f_in, F_out, T);
+    if (!ws || ws_bytes < need) {
+      set_error("workspace too small: need " + std::to_string(need));
+      return GNN_ERR_WORKSPACE;
+    }
+    const int32_t ld = 4 * F + F_out;
+    char *base = (char *)ws;
+    const size_t gws = align256(gemm_tc_workspace(p->n_src, f_in, ld));
+    float *Wcat = (float *)(base + gws);
+    float *bcat = (float *)((char *)Wcat + align256(sizeof(float) * (size_t)f_in * ld));
+    int32_t *table = (int32_t *)((char *)bcat + align256(sizeof(float) * (size_t)ld));
+    float *GS = (float *)((char *)table + align256(sizeof(int32_t) * (size_t)p->n * T));
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e = launch_lstm_weights(W_ih, b_ih, b_hh, W_self, bias, f_in, F, F_out, Wcat, bcat, s);
+    if (e != cudaSuccess) return cuda_status(e, "lstm weights");
+    // redundancy bypass: G = X W_ih^T + b_ih + b_hh and S = X W_self^T + b, once per node
+    const int32_t ldp = (ld + 7) / 8 * 8;
+    gnn_status st = launch_gemm(X, ldx, Wcat, ld, GS, ldp, p->n_src, f_in, ld, nullptr, bcat, 0, base, gws, s);
+    if (st != GNN_OK) return st;
+    e = launch_sample_neighbors(p, T, seed, table, s);
+    if (e != cudaSuccess) return cuda_status(e, "sample neighbors");
+    return cuda_status(launch_sage_lstm(p, table, T, GS, ldp, W_hh, W_neigh, F_out, Y, ldy, s), "sage lstm");
   })
 }
 

@@ -29,6 +29,7 @@ struct DevGraph {
   const int32_t *multi_units;   // [n_multi] number of units of a long row
   const int32_t *multi_row;     // [n_multi] row id of each split row
   const int32_t *empty_rows;    // [n_empty]
+  const int32_t *perm;          // [n] task (LAS) order of the rows
   int32_t n_units, n_multi, n_empty, ng;
   int32_t n_sunits;
 };
@@ -107,6 +108,13 @@ struct AggArgs {
   int32_t *ws_cnt;
   int32_t deterministic;
 };
+// NEXT-3 GraphSAGE-LSTM (k_lstm.cu)
+cudaError_t launch_sample_neighbors(const gnn_plan_s *p, int32_t T, uint64_t seed, int32_t *table, cudaStream_t s);
+cudaError_t launch_lstm_weights(const float *W_ih, const float *b_ih, const float *b_hh, const float *W_self,
+                                const float *bias, int32_t f_in, int32_t F, int32_t F_out, float *Wcat,
+                                float *bcat, cudaStream_t s);
+cudaError_t launch_sage_lstm(const gnn_plan_s *p, const int32_t *table, int32_t T, const float *GS, int64_t ldg,
+                             const float *R, const float *Wn, int32_t F_out, float *Y, int64_t ldy, cudaStream_t s);
 bool set_agg_mapping(int32_t vec, int32_t lanes, int32_t nv);
 bool mapping_supported(int32_t vec, int32_t lanes, int32_t nv);
 bool agg_override_active();

@@ -334,6 +334,7 @@ gnn_status build_schedule(gnn_plan_s *p) {
   UP(multi_units, multi_units)
   UP(multi_row, multi_row)
   UP(empty, empty_rows)
+  UP(p->perm, perm)
 #undef UP
   p->dg.n_units = (int32_t)n_units;
   p->dg.n_sunits = (int32_t)(sunit.size() - 1);

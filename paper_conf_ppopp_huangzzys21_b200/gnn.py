@@ -28,7 +28,8 @@ STATUS = {0: "GNN_OK", 1: "GNN_ERR_INVALID_ARG", 2: "GNN_ERR_INVALID_GRAPH", 3: 
           4: "GNN_ERR_CUDA", 5: "GNN_ERR_NOMEM", 6: "GNN_ERR_UNSUPPORTED", 7: "GNN_ERR_INTERNAL"}
 GNN_SUM, GNN_MEAN, GNN_MAX = 0, 1, 2
 GNN_W_ONE, GNN_W_GCN, GNN_W_EDGE = 0, 1, 2
-GNN_OP_AGGREGATE, GNN_OP_GAT_AGGREGATE, GNN_OP_EDGECONV, GNN_OP_GCN_LAYER, GNN_OP_GAT_LAYER = range(5)
+GNN_OP_AGGREGATE, GNN_OP_GAT_AGGREGATE, GNN_OP_EDGECONV, GNN_OP_GCN_LAYER, GNN_OP_GAT_LAYER, \
+    GNN_OP_SAGE_LSTM_LAYER = range(6)
 REDUCE = {"sum": GNN_SUM, "mean": GNN_MEAN, "max": GNN_MAX}
 WEIGHT = {"one": GNN_W_ONE, "gcn": GNN_W_GCN, "edge": GNN_W_EDGE}
 
@@ -99,6 +100,10 @@ _SIGS = {
     "gnn_groups_host": (ctypes.c_int, [_I64, _P, _P, _I32, ctypes.POINTER(_I64), _P, _P]),
     "gnn_launch_count": (ctypes.c_uint64, []),
     "gnn_plan_set_group_size": (ctypes.c_int, [_P, _I32]),
+    "gnn_sample_neighbors": (ctypes.c_int, [_P, _I32, ctypes.c_uint64, _P, _P]),
+    "gnn_sage_lstm_aggregate": (ctypes.c_int, [_P, _P, _I32, _P, _I64, _I32, _P, _P, _I32, _P, _I64, _P]),
+    "gnn_sage_lstm_layer": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _P, _P, _P, _P, _P, _P, _I32, _I32, _I32,
+                                           ctypes.c_uint64, _P, _I64, _P, _SZ, _P]),
     "gnn_tune_aggregate": (ctypes.c_int, [_P, ctypes.c_int, ctypes.c_int, _P, _P, _I64, _I32, _P, _I64, _I32,
                                           ctypes.POINTER(gnn_tune_result), _P]),
     "gnn_last_error": (ctypes.c_char_p, []),
@@ -410,6 +415,41 @@ def tune_aggregate(plan: Plan, X, reduce="sum", weight="one", edge_w=None, out=N
           _tp(Y), _ld(Y, F), int(max_rounds), ctypes.byref(r), _stream(stream))
     plan._ws = {}
     return {k: getattr(r, k) for k, _ in gnn_tune_result._fields_}
+
+
+def sample_neighbors(plan: Plan, T=16, seed=0, out=None, stream=None):
+    """gnn_sample_neighbors -> [n, T] int32 device table (reading R13)."""
+    torch = _torch()
+    tab = out if out is not None else torch.empty((plan.n, T), dtype=torch.int32, device="cuda")
+    _call("gnn_sample_neighbors", plan.handle, int(T), ctypes.c_uint64(seed), _tp(tab), _stream(stream))
+    return tab
+
+
+def sage_lstm_aggregate(plan: Plan, table, GS, R, W_neigh, out=None, stream=None):
+    """gnn_sage_lstm_aggregate: fused LSTM cells over pre-transformed rows GS + SAGE combine."""
+    torch = _torch()
+    T = table.shape[1]
+    F_out = W_neigh.shape[0]
+    F = R.shape[1]
+    Y = out if out is not None else torch.empty((plan.n, F_out), dtype=torch.float32, device=GS.device)
+    _call("gnn_sage_lstm_aggregate", plan.handle, _tp(table), T, _tp(GS), GS.stride(0), F, _tp(R), _tp(W_neigh),
+          F_out, _tp(Y), _ld(Y, F_out), _stream(stream))
+    return Y
+
+
+def sage_lstm_layer(plan: Plan, X, W_ih, W_hh, b_ih, b_hh, W_self, W_neigh, bias=None, T=16, seed=0, out=None,
+                    stream=None):
+    """gnn_sage_lstm_layer: y = W_self x_v + W_neigh LSTM(sampled neighbours) + b."""
+    torch = _torch()
+    f_in = X.shape[1]
+    F = W_hh.shape[1]
+    F_out = W_self.shape[0]
+    Y = out if out is not None else torch.empty((plan.n, F_out), dtype=torch.float32, device=X.device)
+    ws, nb = plan.workspace(GNN_OP_SAGE_LSTM_LAYER, f_in, F_out, T, X.device)
+    _call("gnn_sage_lstm_layer", plan.handle, _tp(X), _ld(X, f_in), f_in, _tp(W_ih), _tp(W_hh), _tp(b_ih), _tp(b_hh),
+          _tp(W_self), _tp(W_neigh), _tp(bias), F, F_out, int(T), ctypes.c_uint64(seed), _tp(Y), _ld(Y, F_out),
+          _tp(ws), nb, _stream(stream))
+    return Y
 
 
 def launch_count() -> int:
