@@ -347,6 +347,78 @@ def c4():
     return out
 
 
+def lstm_base_torch(X, table, P, T):
+    """Fig 6 base implementation (torch ops): per cell gather the neighbour
+    feature matrix X[u_t], transform it (no redundancy bypass), then the cell."""
+    n = X.shape[0]
+    F = P["W_hh"].shape[1]
+    h = torch.zeros((n, F), device=DEV)
+    c = torch.zeros((n, F), device=DEV)
+    has = (table[:, 0] >= 0)[:, None]
+    idx = table.clamp(min=0).long()
+    b = P["b_ih"] + P["b_hh"]
+    for t in range(T):
+        xg = X[idx[:, t]]                                  # graph op: neighbour feature matrix
+        a = xg @ P["W_ih"].t() + h @ P["W_hh"].t() + b     # neural op on the expanded data
+        i, f, z, o = a.split(F, dim=1)
+        c2 = torch.sigmoid(f) * c + torch.sigmoid(i) * torch.tanh(z)
+        h2 = torch.sigmoid(o) * torch.tanh(c2)
+        c = torch.where(has, c2, c)
+        h = torch.where(has, h2, h)
+    return X @ P["W_self"].t() + h @ P["W_neigh"].t() + P["bias"]
+
+
+def lstm(cfg="C5"):
+    """NEXT-3 GraphSAGE-LSTM layer (32 -> 32, 16 sampled neighbours)
+    on a config graph: layer / cell-kernel ms, rooflines, Fig 11 analogue."""
+    g = gs.config_graph(cfg)
+    f_in, F, F_out, nT = 32, 32, 32, 16
+    rng = np.random.default_rng(gs.seed_of(cfg, 4))
+    Ph = {k: rng.uniform(-0.3, 0.3, size=s).astype(np.float32) for k, s in
+          dict(W_ih=(4 * F, f_in), W_hh=(4 * F, F), b_ih=(4 * F,), b_hh=(4 * F,), W_self=(F_out, f_in),
+               W_neigh=(F_out, F), bias=(F_out,)).items()}
+    P = {k: T(v) for k, v in Ph.items()}
+    X = gs.uniform(g.n, f_in, seed=gs.seed_of(cfg, 1) + 5)
+    Xd = T(X)
+    plan = G.Plan(g.rowptr, g.colidx, reorder=1)
+    args = [P[k] for k in ("W_ih", "W_hh", "b_ih", "b_hh", "W_self", "W_neigh", "bias")]
+    Y = torch.empty((g.n, F_out), device=DEV)
+    out = {"graph": cfg, "n": g.n, "nnz": g.nnz, "T": nT, "f_in": f_in, "F": F, "F_out": F_out}
+    out["layer_ms"] = events_ms(lambda: G.sage_lstm_layer(plan, Xd, *args, T=nT, seed=7, out=Y), iters=10)[0]
+    # the parts: sampling, pre-transform GEMM (redundancy bypass), fused cells
+    tab = G.sample_neighbors(plan, nT, 7)
+    out["sample_ms"] = events_ms(lambda: G.sample_neighbors(plan, nT, 7, out=tab), iters=10)[0]
+    Wcat = torch.cat([P["W_ih"].view(4, F, f_in).permute(1, 0, 2).reshape(4 * F, f_in), P["W_self"]], 0).t()
+    bcat = torch.cat([(P["b_ih"] + P["b_hh"]).view(4, F).t().reshape(-1), P["bias"]])
+    GS = torch.empty((g.n, 4 * F + F_out), device=DEV)
+    out["pretransform_gemm_ms"] = events_ms(lambda: G.gemm(Xd, Wcat.contiguous(), col_bias=bcat, out=GS), iters=10)[0]
+    Ya = torch.empty_like(Y)
+    cell = events_ms(lambda: G.sage_lstm_aggregate(plan, tab, GS, P["W_hh"], P["W_neigh"], out=Ya), iters=10)[0]
+    out["cell_kernel_ms"] = cell
+    out["cell_vs_layer_max_abs_diff"] = float((Ya - Y).abs().max())
+    flop = 2.0 * g.n * nT * (4 * F * F) + 2.0 * g.n * F * F_out
+    byts = g.n * nT * (4 * (4 * F) + 4) + g.n * (4 * F_out * 2 + 4)
+    clk = 1.965e9
+    fp32_peak = 148 * 128 * 2 * clk / 1e12
+    out["cell_roofline"] = {"flop": flop, "algorithmic_bytes": byts, "TFLOPs": flop / (cell * 1e-3) / 1e12,
+                            "fp32_fma_peak_TFLOPs": fp32_peak, "frac_fp32": flop / (cell * 1e-3) / 1e12 / fp32_peak,
+                            "GBps": byts / (cell * 1e-3) / 1e9}
+    # parity on sampled rows (oracle on the same counter-based table)
+    rows = sample_rows(g, k=1024, top=16)
+    table = oracle.sample_neighbors(g.rowptr, g.colidx, nT, 7)
+    ref = oracle.sage_lstm(X, table, **Ph, rows=rows)
+    out["parity_sampled"] = close(Y.cpu().numpy()[rows], ref)
+    out["parity_rows"] = int(len(rows))
+    # Fig 11 analogue: base implementation (expand + transform every cell), torch ops
+    torch.backends.cuda.matmul.allow_tf32 = False
+    base = events_ms(lambda: lstm_base_torch(Xd, tab, P, nT), iters=3, warm=1)[0]
+    out["base_impl_torch_ms"] = base
+    out["speedup_vs_base"] = base / out["layer_ms"]
+    out["base_vs_ours_max_abs_diff"] = float((lstm_base_torch(Xd, tab, P, nT) - Y).abs().max())
+    del plan
+    return out
+
+
 def fsweep():
     """F sweep (Fig 4 / Fig 12 analogue, NEXT-1): sum-aggregation throughput vs
     feature length on the C5 graph with the automatic a4 mapping."""
@@ -455,6 +527,17 @@ def summary(path):
               f"- per-edge MLP (torch, no redundancy bypass) {c['per_edge_mlp_torch_ms']:.3f} ms -> factorised "
               f"**{c['speedup_factorised_vs_per_edge']:.1f}x** ({c['factorised_gemm_GFLOP']:.2f} vs "
               f"{c['per_edge_gemm_GFLOP']:.1f} GFLOP); oracle {c['oracle_edgeconv_ms']:.0f} ms", ""]
+    if "LSTM_C5" in d:
+        c = d["LSTM_C5"]
+        r = c["cell_roofline"]
+        L += [f"## GraphSAGE-LSTM (NEXT-3), {c['graph']}-shaped graph, {c['f_in']}->{c['F_out']}, T={c['T']}", "",
+              f"- layer **{c['layer_ms']:.2f} ms** = sampling {c['sample_ms']:.3f} + pre-transform GEMM "
+              f"{c['pretransform_gemm_ms']:.3f} + fused cells {c['cell_kernel_ms']:.2f} ms",
+              f"- cells: {r['TFLOPs']:.1f} TFLOP/s = {100 * r['frac_fp32']:.0f}% of the fp32 FMA peak "
+              f"({r['fp32_fma_peak_TFLOPs']:.1f}); {r['GBps']:.0f} GB/s algorithmic",
+              f"- base implementation (gather + transform every cell, torch) {c['base_impl_torch_ms']:.1f} ms -> "
+              f"**{c['speedup_vs_base']:.1f}x**; parity ({c['parity_rows']} sampled rows): "
+              f"{c['parity_sampled']['pass']}", ""]
     if "F_sweep" in d:
         L += ["## F sweep (C5 graph, sum, automatic a4 mapping)", "", "| F | ms | Gedge*F/s | alg GB/s |",
               "|---|---|---|---|"]
@@ -500,6 +583,8 @@ def main():
                 rep[f"C3_rho{rho}"] = c3(rho)
         elif c == "C4":
             rep["C4"] = c4()
+        elif c == "LSTM":
+            rep["LSTM_C5"] = lstm("C5")
         elif c == "FS":
             rep["F_sweep"] = fsweep()
         print(f"{c} done in {time.time() - t0:.1f}s", flush=True)
