@@ -74,6 +74,8 @@ def lib():
             "orc_neighbor_groups": (_i64, [_i64, _p, _p, _i32, _p, _p]),
             "orc_partition_rows": (None, [_i64, _p, _i32, _p]),
             "orc_forget_degrees": (None, []),
+            "orc_attn_aggregate": (ctypes.c_int, [_i64, _p, _p, _i32, _p, _i64, _p, _i64, _p, _i32, _i32,
+                                                  ctypes.c_float, _i32, _p, _i64, _p, _i64]),
             "orc_sample_neighbors": (None, [_i64, _p, _p, _i32, ctypes.c_uint64, _p]),
             "orc_sage_lstm": (ctypes.c_int, [_i64, _p, _i64, _i32, _p, _i32, _p, _p, _p, _p, _i32, _p, _p, _p,
                                              _i32, _p, _i64, _p, _i64]),
@@ -308,4 +310,24 @@ def sage_lstm(X, table, W_ih, W_hh, b_ih, b_hh, W_self, W_neigh, bias=None, rows
     assert lib().orc_sage_lstm(n, _ptr(X), X.shape[1], f_in, _ptr(table), T, _ptr(W_ih), _ptr(W_hh), _ptr(b_ih),
                                _ptr(b_hh), F, _ptr(W_self), _ptr(W_neigh), _ptr(b), F_out, _ptr(r), nr, _ptr(Y),
                                F_out) == 0
+    return Y
+
+
+SCORES = {"gat": 0, "sym": 1, "linear": 2, "gaan": 3, "gene": 4}
+
+
+def attn_aggregate(rowptr, colidx, score, Zs, H, Fh, Tv=None, Wa=None, neg_slope=0.2, head_mean=False, rows=None):
+    """NEXT-4 Table 2 edge functions + softmax aggregation (reading R14), fp64."""
+    rowptr, colidx = _csr(rowptr, colidx)
+    Zs = _f32(Zs)
+    n = len(rowptr) - 1
+    Tv = _f32(Tv) if Tv is not None else None
+    Wa = _f32(Wa) if Wa is not None else None
+    r, nr = _rows(rows)
+    m = nr if rows is not None else n
+    width = Fh if head_mean else H * Fh
+    Y = np.empty((m, width), np.float32)
+    assert lib().orc_attn_aggregate(n, _ptr(rowptr), _ptr(colidx), SCORES[score], _ptr(Zs), Zs.shape[1], _ptr(Tv),
+                                    0 if Tv is None else Tv.shape[1], _ptr(Wa), H, Fh, neg_slope, int(head_mean),
+                                    _ptr(r), nr, _ptr(Y), width) == 0
     return Y

@@ -624,3 +624,95 @@ def test_sample_neighbors_uniform_with_replacement():
         nb = set(g2.colidx[g2.rowptr[v]:g2.rowptr[v + 1]].tolist())
         assert set(a[v].tolist()) <= (nb if nb else {-1})
     assert (a != b).mean() > 0.5
+
+
+# --------------------------------------------------------------------------- #
+# NEXT-4 Table 2 edge functions + Softmax_aggr (R14)
+# --------------------------------------------------------------------------- #
+def _dense_softmax_aggr(A, E, Z):
+    """Dense masked softmax (multiplicity weights A[v,u]) then the weighted sum."""
+    out = np.zeros((A.shape[0], Z.shape[1]))
+    for v in range(A.shape[0]):
+        m = A[v] > 0
+        if not m.any():
+            continue
+        ev = np.where(m, E[v], -np.inf)
+        w = A[v] * np.exp(ev - ev[m].max())
+        out[v] = (w / w.sum()) @ Z
+    return out
+
+
+def _dense_adj(g):
+    A = np.zeros((g.n, g.n))
+    for v in range(g.n):
+        for u in g.colidx[g.rowptr[v]:g.rowptr[v + 1]]:
+            A[v, u] += 1
+    return A
+
+
+@pytest.mark.parametrize("score", ["gat", "sym", "linear", "gaan", "gene"])
+def test_attn_scores_vs_dense(score):
+    """Every Table 2 score, evaluated per edge by the oracle, against a dense
+    all-pairs formulation (N x N score matrix, adjacency-masked softmax)."""
+    g = gs.random_small(40, avg_deg=5, seed=17, self_loops=True, multi=True)
+    H, Fh = 3, 4
+    F = H * Fh
+    rng = np.random.default_rng(18)
+    Z = rng.uniform(-2, 2, size=(g.n, F)).astype(np.float32)
+    s = rng.uniform(-2, 2, size=(g.n, H)).astype(np.float32)
+    t = rng.uniform(-2, 2, size=(g.n, H)).astype(np.float32)
+    q = rng.uniform(-1, 1, size=(g.n, F)).astype(np.float32)
+    k = rng.uniform(-1, 1, size=(g.n, F)).astype(np.float32)
+    Wa = rng.uniform(-1, 1, size=(H, Fh)).astype(np.float32)
+    A = _dense_adj(g)
+    lk = lambda x: np.where(x > 0, x, 0.2 * x)  # noqa: E731
+    Tv = None
+    if score == "gat":
+        Zs, Tv = np.concatenate([Z, s], 1), t
+        E = [lk(s[None, :, h].astype(np.float64) + t[:, None, h]) for h in range(H)]
+    elif score == "sym":
+        Zs = np.concatenate([Z, s, t], 1)
+        E = [lk(s[None, :, h].astype(np.float64) + t[:, None, h]) + lk(s[:, None, h].astype(np.float64) + t[None, :, h])
+             for h in range(H)]
+    elif score == "linear":
+        Zs = np.concatenate([Z, s], 1)
+        E = [np.tanh(np.broadcast_to(s[None, :, h].astype(np.float64), (g.n, g.n))) for h in range(H)]
+    elif score == "gaan":
+        Zs, Tv = np.concatenate([Z, q], 1), k
+        E = [k[:, h * Fh:(h + 1) * Fh].astype(np.float64) @ q[:, h * Fh:(h + 1) * Fh].T.astype(np.float64)
+             for h in range(H)]
+    else:
+        Zs, Tv = np.concatenate([Z, q], 1), k
+        E = [np.tanh(q[None, :, h * Fh:(h + 1) * Fh].astype(np.float64) + k[:, None, h * Fh:(h + 1) * Fh]) @
+             Wa[h].astype(np.float64) for h in range(H)]
+    Y = oracle.attn_aggregate(g.rowptr, g.colidx, score, Zs, H, Fh, Tv=Tv, Wa=Wa)
+    ref = np.concatenate([_dense_softmax_aggr(A, E[h], Z[:, h * Fh:(h + 1) * Fh].astype(np.float64))
+                          for h in range(H)], 1)
+    assert np.allclose(Y, ref, rtol=1e-6, atol=1e-6)
+    Ym = oracle.attn_aggregate(g.rowptr, g.colidx, score, Zs, H, Fh, Tv=Tv, Wa=Wa, head_mean=True)
+    assert np.allclose(Ym, ref.reshape(g.n, H, Fh).mean(1), rtol=1e-6, atol=1e-6)
+
+
+def test_attn_special_cases():
+    """Zero attention parameters give uniform weights (= mean aggregation,
+    pinned above by the dense adjacency); the GAT score path equals the
+    separately written GAT oracle (Listing 1 order)."""
+    g = gs.random_small(80, avg_deg=6, seed=19)
+    H, Fh = 2, 3
+    F = H * Fh
+    rng = np.random.default_rng(20)
+    Z = rng.uniform(-1, 1, size=(g.n, F)).astype(np.float32)
+    zeros = np.zeros((g.n, F), np.float32)
+    mean = oracle.aggregate(g.rowptr, g.colidx, Z, "mean")
+    for score, Zs, Tv, Wa in [("gaan", np.concatenate([Z, zeros], 1), rng.uniform(-1, 1, (g.n, F)), None),
+                              ("gene", np.concatenate([Z, rng.uniform(-1, 1, (g.n, F))], 1),
+                               rng.uniform(-1, 1, (g.n, F)), np.zeros((H, Fh))),
+                              ("linear", np.concatenate([Z, np.zeros((g.n, H), np.float32)], 1), None, None)]:
+        Y = oracle.attn_aggregate(g.rowptr, g.colidx, score, Zs, H, Fh, Tv=Tv, Wa=Wa)
+        assert np.allclose(Y, mean, rtol=1e-6, atol=1e-7), score
+    s = rng.uniform(-3, 3, size=(g.n, H)).astype(np.float32)
+    t = rng.uniform(-3, 3, size=(g.n, H)).astype(np.float32)
+    Zs = np.concatenate([Z, s], 1)
+    a = oracle.attn_aggregate(g.rowptr, g.colidx, "gat", Zs, H, Fh, Tv=t)
+    b = oracle.gat_aggregate(g.rowptr, g.colidx, Zs, t, H, Fh, 0.2)
+    assert np.allclose(a, b, rtol=1e-6, atol=1e-7)
