@@ -156,7 +156,9 @@ typedef enum {
   GNN_OP_EDGECONV = 2,      /* f_in, f_out */
   GNN_OP_GCN_LAYER = 3,     /* f_in, f_out */
   GNN_OP_GAT_LAYER = 4,     /* f_in, f_out = H * Fh, heads = H */
-  GNN_OP_SAGE_LSTM_LAYER = 5 /* f_in, f_out = F_out, heads = T (hidden F = 32) */
+  GNN_OP_SAGE_LSTM_LAYER = 5, /* f_in, f_out = F_out, heads = T (hidden F = 32) */
+  GNN_OP_ATTN_AGGREGATE = 6,  /* f_out = H * Fh, heads = H */
+  GNN_OP_ATTN_AGGREGATE_MEAN = 7 /* as 6, with head_mean (adds an n x H*Fh buffer) */
 } gnn_op;
 
 /* Bytes of device workspace a call needs (may be 0; pass NULL then).  The
@@ -425,6 +427,36 @@ gnn_status gnn_sage_lstm_layer(gnn_plan_t plan, const float *X, int64_t ldx, int
                                const float *b_hh, const float *W_self, const float *W_neigh,
                                const float *bias, int32_t F, int32_t F_out, int32_t T, uint64_t seed,
                                float *Y, int64_t ldy, void *ws, size_t ws_bytes, gnn_stream_t stream);
+
+/*
+ * NEXT-4: the edge functions of Table 2 feeding Table 1's
+ * Softmax_aggr, fused like GAT (scores never reach HBM; reading
+ * R14).  Per edge u->v and head h (Fh features per head, F = H*Fh):
+ *   GNN_SCORE_GAT      e = LeakyReLU(s_u + t_v)            Zs = [z | s], Tv = t [n, H]
+ *   GNN_SCORE_SYM_GAT  e = LeakyReLU(s_u + t_v) + LeakyReLU(s_v + t_u)   Zs = [z | s | t]
+ *   GNN_SCORE_LINEAR   e = tanh(s_u)                       Zs = [z | s]
+ *   GNN_SCORE_GAAN     e = <q_u, k_v>                      Zs = [z | q], Tv = k [n, F]
+ *   GNN_SCORE_GENE     e = <W_a, tanh(a_u + b_v)>          Zs = [z | a], Tv = b [n, F], Wa [H, Fh]
+ * y_v[h] = SUM_u softmax_u(e_uv[h]) z_u[h]; head_mean = 1 averages the heads
+ * (Y [n, Fh]) instead of concatenating them (Y [n, F]).  Empty rows give 0.
+ * s, t, q, k, a, b are the W_l h / W_r h projections (caller's GEMM).  Zs:
+ * [n_src, ldz] device, Tv: [n, ldt].  Sym-GAT needs n == n_src.  GaAN and
+ * Gene-linear need Fh / vec to be a power of two <= 32 for some vector width
+ * vec in {8, 4, 2, 1} dividing Fh (else GNN_ERR_UNSUPPORTED).  Workspace:
+ * gnn_workspace_size(plan, head_mean ? GNN_OP_ATTN_AGGREGATE_MEAN :
+ * GNN_OP_ATTN_AGGREGATE, 0, F, H).
+ */
+typedef enum {
+  GNN_SCORE_GAT = 0,
+  GNN_SCORE_SYM_GAT = 1,
+  GNN_SCORE_LINEAR = 2,
+  GNN_SCORE_GAAN = 3,
+  GNN_SCORE_GENE = 4
+} gnn_score;
+gnn_status gnn_attn_aggregate(gnn_plan_t plan, int score, const float *Zs, int64_t ldz,
+                              const float *Tv, int64_t ldt, const float *Wa, int32_t H, int32_t Fh,
+                              float neg_slope, int32_t head_mean, float *Y, int64_t ldy, void *ws,
+                              size_t ws_bytes, gnn_stream_t stream);
 
 uint64_t gnn_launch_count(void);
 

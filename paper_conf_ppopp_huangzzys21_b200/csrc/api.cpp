@@ -337,6 +337,9 @@ size_t gnn_workspace_size(gnn_plan_t p, int op, int32_t f_in, int32_t f_out, int
       return a > b ? a : b;
     }
     case GNN_OP_SAGE_LSTM_LAYER: return ws_sage_lstm(p, f_in, f_out, heads);
+    case GNN_OP_ATTN_AGGREGATE: return agg_workspace_bytes(p, 4, f_out, heads);
+    case GNN_OP_ATTN_AGGREGATE_MEAN:
+      return align256(sizeof(float) * (size_t)p->n * (size_t)(f_out > 0 ? f_out : 0)) + agg_workspace_bytes(p, 4, f_out, heads);
     default: return 0;
   }
 }
@@ -796,6 +799,66 @@ gnn_status gnn_sage_lstm_layer(gnn_plan_t p, const float *X, int64_t ldx, int32_
     e = launch_sample_neighbors(p, T, seed, table, s);
     if (e != cudaSuccess) return cuda_status(e, "sample neighbors");
     return cuda_status(launch_sage_lstm(p, table, T, GS, ldp, W_hh, W_neigh, F_out, Y, ldy, s), "sage lstm");
+  })
+}
+
+// ---------------------------------------------------------------------------
+// NEXT-4: Table 2 edge functions + softmax aggregation (reading R14)
+// ---------------------------------------------------------------------------
+gnn_status gnn_attn_aggregate(gnn_plan_t p, int score, const float *Zs, int64_t ldz, const float *Tv, int64_t ldt,
+                              const float *Wa, int32_t H, int32_t Fh, float neg_slope, int32_t head_mean, float *Y,
+                              int64_t ldy, void *ws, size_t ws_bytes, gnn_stream_t stream) {
+  GNN_TRY({
+    if (!p) return check(false, "plan is NULL");
+    if (score < GNN_SCORE_GAT || score > GNN_SCORE_GENE) return check(false, "score out of range");
+    if (H < 1 || Fh < 1 || H > 256) return check(false, "H in [1, 256] and Fh >= 1 required");
+    const int32_t F = H * Fh;
+    const int32_t extra = (score == GNN_SCORE_GAT || score == GNN_SCORE_LINEAR) ? H
+                          : score == GNN_SCORE_SYM_GAT ? 2 * H : F;
+    const bool needs_tv = score == GNN_SCORE_GAT || score == GNN_SCORE_GAAN || score == GNN_SCORE_GENE;
+    const int32_t tv_w = score == GNN_SCORE_GAT ? H : F;
+    if (!Y || (p->nnz > 0 && !Zs)) return check(false, "Zs/Y is NULL");
+    if (needs_tv && !Tv) return check(false, "Tv (t, k or b) is required for this score");
+    if (score == GNN_SCORE_GENE && !Wa) return check(false, "Wa is required for Gene-linear");
+    if (ldz < F + extra) return check(false, "ldz too small for [z | score columns]");
+    if (needs_tv && ldt < tv_w) return check(false, "ldt too small");
+    if (score == GNN_SCORE_SYM_GAT && p->n != p->n_src) return check(false, "Sym-GAT needs a square plan");
+    const int32_t width = head_mean ? Fh : F;
+    if (ldy < width) return check(false, "ldy too small");
+    if (overlaps(Zs, span_bytes(p->n_src, ldz, F + extra), Y, span_bytes(p->n, ldy, width)))
+      return check(false, "Zs and Y overlap");
+    size_t head = 0;
+    float *Yf = Y;
+    int64_t ldf = ldy;
+    if (head_mean) {
+      head = align256(sizeof(float) * (size_t)p->n * (size_t)F);
+      Yf = (float *)ws;
+      ldf = F;
+    }
+    const size_t need = head + agg_workspace_bytes(p, 4, F, H);  // Sym-GAT (2H keys) bounds every score
+    if (!ws || ws_bytes < need) {
+      set_error("workspace too small: need " + std::to_string(need));
+      return GNN_ERR_WORKSPACE;
+    }
+    static const int kMode[5] = {3, 4, 5, 6, 7};
+    AggArgs a{};
+    a.mode = kMode[score];
+    a.X = Zs;
+    a.ldx = ldz;
+    a.F = F;
+    a.Y = Yf;
+    a.ldy = ldf;
+    a.t = score == GNN_SCORE_GAT ? Tv : nullptr;
+    a.ldt = ldt;
+    a.kb = (score == GNN_SCORE_GAAN || score == GNN_SCORE_GENE) ? Tv : nullptr;
+    a.ldk = ldt;
+    a.Wa = Wa;
+    a.H = H;
+    a.Fh = Fh;
+    a.slope = neg_slope;
+    gnn_status st = agg_common(p, a, (char *)ws + head, ws_bytes - head, stream);
+    if (st != GNN_OK || !head_mean) return st;
+    return cuda_status(launch_head_mean(Yf, ldf, p->n, H, Fh, Y, ldy, (cudaStream_t)stream), "head mean");
   })
 }
 

@@ -87,7 +87,7 @@ cudaError_t launch_minhash(const int32_t *rowptr, const int32_t *colidx, int64_t
                            uint64_t seed, uint64_t *sig, cudaStream_t s);
 
 struct AggArgs {
-  int mode;            // 0 sum, 1 mean, 2 max, 3 gat
+  int mode;            // 0 sum, 1 mean, 2 max, 3 gat, 4 sym-gat, 5 linear, 6 gaan, 7 gene-linear
   int weight;          // gnn_weight (sum/mean/max)
   const float *edge_w;
   const float *X;
@@ -103,6 +103,10 @@ struct AggArgs {
   int64_t ldt;
   int32_t H, Fh;
   float slope;
+  // GaAN k / Gene b per destination row, Gene W_a
+  const float *kb;
+  int64_t ldk;
+  const float *Wa;
   // split-row workspace
   float *ws_part;
   int32_t *ws_cnt;
@@ -123,6 +127,8 @@ gnn_status rebuild_schedule(gnn_plan_s *p, int64_t group_size);
 int64_t default_group_size(int64_t n, int64_t nnz);
 int set_agg_impl(int impl);
 size_t agg_workspace_bytes(const gnn_plan_s *p, int mode, int32_t F, int32_t H);
+cudaError_t launch_head_mean(const float *Yf, int64_t ldf, int64_t n, int32_t H, int32_t Fh, float *Y, int64_t ldy,
+                             cudaStream_t s);
 gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, size_t ws_bytes,
                             cudaStream_t s);
 

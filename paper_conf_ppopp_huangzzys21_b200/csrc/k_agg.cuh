@@ -34,7 +34,11 @@ namespace gnn {
 // merges them in group order (P:885-894 with a fixed order) and applies the
 // postponed epilogue (linear property).
 // ---------------------------------------------------------------------------
-enum { M_SUM = 0, M_MEAN = 1, M_MAX = 2, M_GAT = 3 };
+enum { M_SUM = 0, M_MEAN = 1, M_MAX = 2, M_GAT = 3, M_SYM = 4, M_LIN = 5, M_GAAN = 6, M_GENE = 7 };
+// attention modes (softmax aggregation of Table 1 with a Table 2 score, R9/R14)
+__host__ __device__ constexpr bool is_att(int mode) { return mode >= M_GAT; }
+// scores that are an Fh-vector product per head (GaAN, Gene-linear)
+__host__ __device__ constexpr bool vec_score(int mode) { return mode == M_GAAN || mode == M_GENE; }
 // internal weight code: weight 1 inside the loop, x ndst[v] in the epilogue
 // (transform-first GCN whose GEMM epilogue already applied nsrc[u])
 constexpr int W_DST_ONLY = 3;
@@ -56,7 +60,11 @@ struct KParams {
   int64_t ldt;
   int32_t H, Fh;
   float slope;
-  const uint32_t *smax;  // GAT: [H] order-encoded max over sources of s_u[h] (k_score_max)
+  const uint32_t *smax;  // attention: order-encoded source maxima (k_score_max): [H] s (GAT, Linear),
+                         // [2H] s then t (Sym-GAT), [H] |q_u[h]| (GaAN)
+  const float *kb;       // GaAN k / Gene b: [n, ldk] per destination row
+  int64_t ldk;
+  const float *Wa;       // Gene: [H, Fh]
   int32_t *ws_unit;  // work-unit counters (one per feature chunk), zeroed per call
   float *ws_acc;   // [n_multi][FW] atomic accumulators (deterministic == 0)
   float *ws_part;  // [multi slots][FW] per-group partials (deterministic)
@@ -175,7 +183,7 @@ template <int MODE, int VEC, int NV>
 __device__ __forceinline__ void part_combine(Part<MODE, VEC, NV> &A, const Part<MODE, VEC, NV> &B) {
 #pragma unroll
   for (int n = 0; n < NV; ++n) {
-    if constexpr (MODE == M_GAT) {
+    if constexpr (is_att(MODE)) {
       gat_merge(A.m[n], A.l[n], A.a[n], B.m[n], B.l[n], B.a[n], VEC);
     } else {
 #pragma unroll
@@ -189,7 +197,7 @@ __device__ __forceinline__ void part_combine(Part<MODE, VEC, NV> &A, const Part<
 __device__ __forceinline__ float epi(const KParams &p, int mode, float a, float l, float ndst,
                                      float deg_f, const float *addp) {
   float y;
-  if (mode == M_GAT) {
+  if (is_att(mode)) {
     y = a / l;
   } else {
     y = a;
@@ -204,7 +212,7 @@ __device__ __forceinline__ float epi(const KParams &p, int mode, float a, float 
 template <int MODE, int VEC, int NV, int LANES>
 __device__ __forceinline__ void store_row(const KParams &p, int32_t row, int32_t deg, int32_t c0,
                                           int lane, const Part<MODE, VEC, NV> &P) {
-  const float ndst = (MODE != M_GAT && scales_dst(p.weight)) ? __ldg(p.g.ndst + row) : 1.0f;
+  const float ndst = (!is_att(MODE) && scales_dst(p.weight)) ? __ldg(p.g.ndst + row) : 1.0f;
   const float deg_f = (float)deg;
 #pragma unroll
   for (int n = 0; n < NV; ++n) {
@@ -247,36 +255,85 @@ __device__ __forceinline__ void ldv_cg(const float *p, float (&v)[VEC]) {
 // task-ordered colidx_t (one contiguous stream per unit).
 // ---------------------------------------------------------------------------
 
+// fast tanh for the Linear / Gene-linear scores: 1 - 2 / (e^{2x} + 1), in [-1, 1]
+__device__ __forceinline__ float tanh_fast(float x) { return 1.0f - __fdividef(2.0f, __expf(2.0f * x) + 1.0f); }
+
+// sum over the LPH lanes of one head (LPH a power of two, aligned segments);
+// the butterfly leaves the same value in every lane of the segment
+template <int LANES>
+__device__ __forceinline__ float head_sum(float x, int lph, unsigned mask) {
+  for (int off = 1; off < lph; off <<= 1) x += __shfl_xor_sync(mask, x, off, LANES);
+  return x;
+}
+
 // one neighbour group: fresh fp32 chain in CSR order (R9); indices from the
-// task-ordered stream, LANES at a time, U source rows in flight per worker
+// task-ordered stream, LANES at a time, U source rows in flight per worker.
+// Attention modes (GAT and the other Table 2 scores, R14): softmax terms
+// exp(e - m) against a per-row upper bound m of the scores (R9 GAT), with an
+// exact-max recompute when the bound is loose.
 template <int MODE, int VEC, int NV, int LANES>
 __device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx, int32_t len, int32_t beg,
                                             int32_t row, int32_t c0, int lane, unsigned mask,
                                             Part<MODE, VEC, NV> &G) {
+  constexpr bool ATT = is_att(MODE);
+  constexpr bool VS = vec_score(MODE);
   constexpr int FPL = VEC * NV;
-  constexpr int U = FPL >= 32 ? 1 : (32 / FPL > 8 ? 8 : 32 / FPL);
+  constexpr int U0 = FPL >= 32 ? 1 : (32 / FPL > 8 ? 8 : 32 / FPL);
+  constexpr int U = (VS && U0 > 2) ? 2 : U0;
+  constexpr int VQ = VS ? VEC : 1;  // per-slot score vector (GaAN q_u / Gene a_u slice)
   part_init(G);
   const int weight = p.weight;
   const float *xl = p.X + c0 + lane * VEC;
+  const int lph = VS ? p.Fh / VEC : 1;  // lanes per head
   bool valid[NV];
   int32_t head[NV];
-  float tv[NV];
-  float nmb[NV];   // GAT: -m * log2(e) for the current reference m
-  float seen[NV];  // GAT: exact max score of the group
-  // GAT: a one-edge group takes its own score as reference (term = 1 exactly)
-  const bool one = MODE == M_GAT && len == 1;
+  float tv[NV];     // GAT/Sym: t_v[h]
+  float sv[NV];     // Sym: s_v[h]
+  float kv[NV][VQ];  // GaAN k_v / Gene b_v slice
+  float wa[NV][VQ];  // Gene W_a slice
+  float nmb[NV];    // -m * log2(e) for the current reference m
+  float seen[NV];   // exact max score of the group
+  // a one-edge group takes its own score as reference (term = 1 exactly)
+  const bool one = ATT && len == 1;
 #pragma unroll
   for (int n = 0; n < NV; ++n) {
     const int32_t f = c0 + (n * LANES + lane) * VEC;
     valid[n] = f < p.F;
     head[n] = 0;
     tv[n] = 0.0f;
+    sv[n] = 0.0f;
     nmb[n] = 0.0f;
     seen[n] = -INFINITY;
-    if constexpr (MODE == M_GAT) {
+#pragma unroll
+    for (int i = 0; i < VQ; ++i) kv[n][i] = wa[n][i] = 0.0f;
+    if constexpr (ATT) {
       head[n] = valid[n] ? f / p.Fh : 0;
-      tv[n] = valid[n] ? __ldg(p.t + (int64_t)row * p.ldt + head[n]) : 0.0f;
-      const float mb = valid[n] ? leaky_f(fkey_decode(__ldg(p.smax + head[n])) + tv[n], p.slope) : 0.0f;
+      const int h = head[n];
+      float mb = 0.0f;
+      if constexpr (MODE == M_GAT) {
+        tv[n] = valid[n] ? __ldg(p.t + (int64_t)row * p.ldt + h) : 0.0f;
+        mb = leaky_f(fkey_decode(__ldg(p.smax + h)) + tv[n], p.slope);
+      } else if constexpr (MODE == M_SYM) {
+        const float *zv = p.X + (int64_t)row * p.ldx + p.F;
+        tv[n] = valid[n] ? __ldg(zv + p.H + h) : 0.0f;
+        sv[n] = valid[n] ? __ldg(zv + h) : 0.0f;
+        mb = leaky_f(fkey_decode(__ldg(p.smax + h)) + tv[n], p.slope) +
+             leaky_f(sv[n] + fkey_decode(__ldg(p.smax + p.H + h)), p.slope);
+      } else if constexpr (MODE == M_LIN) {
+        mb = 1.0f;  // tanh <= 1
+      } else {
+        if (valid[n]) {
+          ldv<VEC>(p.kb + (int64_t)row * p.ldk + f, kv[n]);
+          if constexpr (MODE == M_GENE) ldv<VEC>(p.Wa + f, wa[n]);
+        }
+        float part = 0.0f;
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) part = MODE == M_GAAN ? fmaf(kv[n][i], kv[n][i], part) : part + fabsf(wa[n][i]);
+        part = head_sum<LANES>(part, lph, mask);
+        // GaAN: <q_u, k_v> <= max_u |q_u| |k_v| (Cauchy-Schwarz); Gene: |<W_a, tanh(.)>| <= |W_a|_1
+        mb = MODE == M_GAAN ? fkey_decode(__ldg(p.smax + h)) * sqrtf(part) : part;
+      }
+      if (!valid[n]) mb = 0.0f;
       G.m[n] = mb;
       nmb[n] = -mb * kLog2e;
     }
@@ -289,10 +346,24 @@ __device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx
     w = 1.0f;
     if (lane < c) {
       u = ld_stream_i32(idx + k + lane);
-      if constexpr (MODE != M_GAT) {
+      if constexpr (!ATT) {
         if (weight == GNN_W_GCN) w = __ldg(p.g.nsrc + u);
         else if (weight == GNN_W_EDGE) w = ld_stream_f32(p.edge_w + beg + k + lane);
       }
+    }
+  };
+  // per-slot score inputs of source row u
+  auto load_score = [&](int32_t u, int n, float &a, float &b, float (&vq)[VQ]) {
+    if constexpr (MODE == M_GAT || MODE == M_LIN) {
+      a = valid[n] ? __ldg(p.X + (int64_t)u * p.ldx + p.F + head[n]) : 0.0f;
+    } else if constexpr (MODE == M_SYM) {
+      a = valid[n] ? __ldg(p.X + (int64_t)u * p.ldx + p.F + head[n]) : 0.0f;
+      b = valid[n] ? __ldg(p.X + (int64_t)u * p.ldx + p.F + p.H + head[n]) : 0.0f;
+    } else if constexpr (VS) {
+      if (valid[n]) ldv<VEC>(xl + (int64_t)u * p.ldx + p.F + n * LANES * VEC, vq);
+      else
+#pragma unroll
+        for (int i = 0; i < VQ; ++i) vq[i] = 0.0f;
     }
   };
 #pragma unroll 1
@@ -306,7 +377,8 @@ __device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx
       const float my_w = nx_w;
       if (k + LANES < len) load_batch(k + LANES, nx_u, nx_w);
       float v[U][NV][VEC];
-      float sc[U][NV];
+      float sc[U][NV], sc2[U][NV];
+      float vq[U][NV][VQ];
 #pragma unroll
       for (int q = 0; q < U; ++q) {
         if (q < cnt) {
@@ -314,7 +386,7 @@ __device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx
 #pragma unroll
           for (int n = 0; n < NV; ++n) {
             if (valid[n]) ldv<VEC>(xl + (int64_t)u * p.ldx + n * LANES * VEC, v[q][n]);
-            if constexpr (MODE == M_GAT) sc[q][n] = valid[n] ? __ldg(p.X + (int64_t)u * p.ldx + p.F + head[n]) : 0.0f;
+            if constexpr (ATT) load_score(u, n, sc[q][n], sc2[q][n], vq[q][n]);
           }
         }
       }
@@ -323,14 +395,31 @@ __device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx
         for (int q = 0; q < U; ++q) {
           const int32_t e = j + q;
           if (e < cnt) {
-            if constexpr (MODE == M_GAT) {
-              // e_uv = LeakyReLU(s_u + t_v); term exp(e_uv - m) (one ex2 per edge and head)
+            if constexpr (ATT) {
+              // the score e_uv (Table 2), then the term exp(e_uv - m): one ex2 per edge and head
+              float sco[NV];
+#pragma unroll
+              for (int n = 0; n < NV; ++n) {
+                if constexpr (MODE == M_GAT) {
+                  sco[n] = leaky_f(sc[q][n] + tv[n], p.slope);
+                } else if constexpr (MODE == M_SYM) {
+                  sco[n] = leaky_f(sc[q][n] + tv[n], p.slope) + leaky_f(sv[n] + sc2[q][n], p.slope);
+                } else if constexpr (MODE == M_LIN) {
+                  sco[n] = tanh_fast(sc[q][n]);
+                } else {
+                  float part = 0.0f;
+#pragma unroll
+                  for (int i = 0; i < VEC; ++i)
+                    part = MODE == M_GAAN ? fmaf(vq[q][n][i], kv[n][i], part)
+                                          : fmaf(wa[n][i], tanh_fast(vq[q][n][i] + kv[n][i]), part);
+                  sco[n] = head_sum<LANES>(part, lph, mask);
+                }
+              }
 #pragma unroll
               for (int n = 0; n < NV; ++n) {
                 if (!valid[n]) continue;
-                const float sco = leaky_f(sc[q][n] + tv[n], p.slope);
-                seen[n] = fmaxf(seen[n], sco);
-                const float ex = one ? 1.0f : ex2_f(fmaf(sco, kLog2e, nmb[n]));
+                seen[n] = fmaxf(seen[n], sco[n]);
+                const float ex = one ? 1.0f : ex2_f(fmaf(sco[n], kLog2e, nmb[n]));
                 G.l[n] += ex;
 #pragma unroll
                 for (int i = 0; i < VEC; ++i) G.a[n][i] = fmaf(ex, v[q][n][i], G.a[n][i]);
@@ -352,15 +441,14 @@ __device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx
 #pragma unroll
               for (int n = 0; n < NV; ++n) {
                 if (valid[n]) ldv<VEC>(xl + (int64_t)u * p.ldx + n * LANES * VEC, v[q][n]);
-                if constexpr (MODE == M_GAT)
-                  sc[q][n] = valid[n] ? __ldg(p.X + (int64_t)u * p.ldx + p.F + head[n]) : 0.0f;
+                if constexpr (ATT) load_score(u, n, sc[q][n], sc2[q][n], vq[q][n]);
               }
             }
           }
         }
       }
     }
-    if constexpr (MODE != M_GAT) {
+    if constexpr (!ATT) {
       break;
     } else {
       if (one) {
@@ -398,7 +486,7 @@ __device__ __forceinline__ void merge_row(const KParams &p, const float *base, i
     for (int32_t q = 0; q < ngrp; ++q) {
       float b[VEC];
       ldv_cg<VEC>(base + (size_t)q * p.FW + f, b);
-      if constexpr (MODE == M_GAT) {
+      if constexpr (is_att(MODE)) {
         const float bm = __ldcg(base + (size_t)q * p.FW + p.F + f / p.Fh);
         const float bl = __ldcg(base + (size_t)q * p.FW + p.F + p.H + f / p.Fh);
         if (q == 0) {
@@ -450,7 +538,7 @@ __device__ __forceinline__ void process_unit(const KParams &p, int4 d, int32_t l
       for (int i = 0; i < VEC; ++i) atomicAdd(acc + f + i, G.a[n][i]);
     } else {
       stv<VEC>(base + (size_t)k * p.FW + f, G.a[n]);
-      if constexpr (MODE == M_GAT) {
+      if constexpr (is_att(MODE)) {
         if (f % p.Fh == 0) {
           base[(size_t)k * p.FW + p.F + f / p.Fh] = G.m[n];
           base[(size_t)k * p.FW + p.F + p.H + f / p.Fh] = G.l[n];
@@ -500,7 +588,7 @@ template <int MODE, int VEC, int NV, int LANES, bool WGT>
 struct Stream {
   static constexpr int FPL = VEC * NV;
   static constexpr int U0 = FPL >= 32 ? 1 : (32 / FPL > 8 ? 8 : 32 / FPL);
-  static constexpr int U = (MODE == M_GAT && U0 > 4) ? 4 : (U0 > LANES ? LANES : U0);
+  static constexpr int U = (is_att(MODE) && U0 > 4) ? 4 : (U0 > LANES ? LANES : U0);
 };
 
 // finish one group: epilogue + store (whole row), or the group's partial to
@@ -528,7 +616,7 @@ __device__ __forceinline__ void finish_group(const KParams &p, const Part<MODE, 
       for (int i = 0; i < VEC; ++i) atomicAdd(acc + f + i, G.a[n][i]);
     } else {
       stv<VEC>(base + (size_t)k * p.FW + f, G.a[n]);
-      if constexpr (MODE == M_GAT) {
+      if constexpr (is_att(MODE)) {
         if (f % p.Fh == 0) {
           base[(size_t)k * p.FW + p.F + f / p.Fh] = G.m[n];
           base[(size_t)k * p.FW + p.F + p.H + f / p.Fh] = G.l[n];
@@ -612,7 +700,7 @@ __device__ __forceinline__ void stream_unit(const KParams &p, int32_t g0, int32_
   for (int n = 0; n < NV; ++n) {
     const int32_t f = c0 + (n * LANES + lane) * VEC;
     valid[n] = f < p.F;
-    head[n] = (MODE == M_GAT && valid[n]) ? f / p.Fh : 0;
+    head[n] = (is_att(MODE) && valid[n]) ? f / p.Fh : 0;
   }
   const float *xl = p.X + c0 + lane * VEC;
   // current group
@@ -623,7 +711,7 @@ __device__ __forceinline__ void stream_unit(const KParams &p, int32_t g0, int32_
 #pragma unroll
     for (int n = 0; n < NV; ++n) out[n] = valid[n] ? __ldg(p.t + (int64_t)row * p.ldt + head[n]) : 0.0f;
   };
-  if constexpr (MODE == M_GAT) {
+  if constexpr (is_att(MODE)) {
     load_tv(__shfl_sync(mask, grow, 0, LANES), tv);
     if (g0 + 1 < g1 && 1 < LANES) load_tv(__shfl_sync(mask, grow, 1, LANES), tvn);
   }
@@ -651,7 +739,7 @@ __device__ __forceinline__ void stream_unit(const KParams &p, int32_t g0, int32_
     if constexpr (WGT) wq[q] = __shfl_sync(mask, a_w, off_, LANES);                                   \
     _Pragma("unroll") for (int n = 0; n < NV; ++n) {                                                  \
       if (valid[n]) ldv<VEC>(xl + (int64_t)u_ * p.ldx + n * LANES * VEC, v[q][n]);                    \
-      if constexpr (MODE == M_GAT)                                                                    \
+      if constexpr (is_att(MODE))                                                                    \
         sc[q][n] = valid[n] ? __ldg(p.X + (int64_t)u_ * p.ldx + p.F + head[n]) : 0.0f;                \
     }                                                                                                 \
   } while (0)
@@ -668,7 +756,7 @@ __device__ __forceinline__ void stream_unit(const KParams &p, int32_t g0, int32_
     for (int q = 0; q < U; ++q) {
       if (pe < T1) {
         // consume edge pe (slot q)
-        if constexpr (MODE == M_GAT) {
+        if constexpr (is_att(MODE)) {
 #pragma unroll
           for (int n = 0; n < NV; ++n) {
             if (!valid[n]) continue;
@@ -709,10 +797,10 @@ __device__ __forceinline__ void stream_unit(const KParams &p, int32_t g0, int32_
             if (gi - gw == LANES) {  // next window of the group table
               gw += LANES;
               load_table();
-              if constexpr (MODE == M_GAT) load_tv(__shfl_sync(mask, grow, 0, LANES), tvn);
+              if constexpr (is_att(MODE)) load_tv(__shfl_sync(mask, grow, 0, LANES), tvn);
             }
             cur_end = __shfl_sync(mask, gend, gi - gw, LANES);
-            if constexpr (MODE == M_GAT) {
+            if constexpr (is_att(MODE)) {
 #pragma unroll
               for (int n = 0; n < NV; ++n) tv[n] = tvn[n];
               const int jn = gi + 1 - gw;
@@ -732,7 +820,7 @@ __device__ __forceinline__ void stream_unit(const KParams &p, int32_t g0, int32_
 }
 
 template <int MODE, int VEC, int NV, int LANES, bool WGT>
-__global__ void __launch_bounds__(256, MODE == M_GAT ? 3 : 4) k_stream(const KParams p) {
+__global__ void __launch_bounds__(256, is_att(MODE) ? 3 : 4) k_stream(const KParams p) {
   constexpr int CW = LANES * VEC * NV;
   const int tid = threadIdx.x;
   const int lane = tid & (LANES - 1);
@@ -788,7 +876,8 @@ __global__ void __launch_bounds__(256, MODE == M_GAT ? 3 : 4) k_stream(const KPa
 #define GNN_AGG_MINB_GAT 4
 #endif
 template <int MODE, int VEC, int NV, int LANES>
-__global__ void __launch_bounds__(256, MODE == M_GAT ? GNN_AGG_MINB_GAT : GNN_AGG_MINB) k_aggregate(const KParams p) {
+__global__ void __launch_bounds__(256, vec_score(MODE) ? 2 : (is_att(MODE) ? GNN_AGG_MINB_GAT : GNN_AGG_MINB))
+    k_aggregate(const KParams p) {
   constexpr int CW = LANES * VEC * NV;
   const int tid = threadIdx.x;
   const int lane = tid & (LANES - 1);
@@ -861,7 +950,7 @@ cudaError_t launch_persistent(KFN fn, int &occ, const KParams &kp_in, int32_t un
   cudaError_t e = cudaMemsetAsync(kp.ws_unit, 0, 256, s);
   if (e == cudaSuccess && kp.g.n_multi > 0)
     e = cudaMemsetAsync(kp.ws_cnt, 0, sizeof(int32_t) * (size_t)kp.g.n_multi * kp.nch, s);
-  if (e == cudaSuccess && kp.g.n_multi > 0 && !kp.deterministic && kp.mode != M_MAX && kp.mode != M_GAT)
+  if (e == cudaSuccess && kp.g.n_multi > 0 && !kp.deterministic && kp.mode != M_MAX && !is_att(kp.mode))
     e = cudaMemsetAsync(kp.ws_acc, 0, sizeof(float) * (size_t)kp.g.n_multi * kp.FW, s);
   if (e != cudaSuccess) return e;
   const int64_t blocks = (int64_t)kp.n_persist + (kp.g.n_empty + 31) / 32;
@@ -877,9 +966,9 @@ cudaError_t launch_one(const KParams &kp, int threads, cudaStream_t s) {
     static int occ = 0;
     return launch_persistent(k_aggregate<MODE, VEC, NV, LANES>, occ, kp, kp.g.n_units, CW, LANES, threads, s);
   }
-  const bool wgt = MODE != M_GAT && (kp.weight == GNN_W_GCN || kp.weight == GNN_W_EDGE);
+  const bool wgt = !is_att(MODE) && (kp.weight == GNN_W_GCN || kp.weight == GNN_W_EDGE);
   cudaError_t e;
-  if constexpr (MODE != M_GAT) {
+  if constexpr (!is_att(MODE)) {
     static int occ_w = 0;
     static int occ = 0;
     e = wgt ? launch_persistent(k_stream<MODE, VEC, NV, LANES, true>, occ_w, kp, kp.g.n_sunits, CW, LANES, threads, s)
@@ -943,5 +1032,6 @@ cudaError_t dispatch_vec(const KParams &kp, const Mapping &m, int threads, cudaS
 cudaError_t dispatch_sum(const KParams &kp, const Mapping &m, int threads, cudaStream_t s);
 cudaError_t dispatch_max(const KParams &kp, const Mapping &m, int threads, cudaStream_t s);
 cudaError_t dispatch_gat(const KParams &kp, const Mapping &m, int threads, cudaStream_t s);
+cudaError_t dispatch_att(const KParams &kp, const Mapping &m, int threads, cudaStream_t s);
 
 }  // namespace gnn

@@ -133,14 +133,26 @@ cudaError_t launch_minhash(const int32_t *rowptr, const int32_t *colidx, int64_t
 // of s_u[h], as order-preserving keys (exact, order-free).  One strided pass
 // over the H score columns (n_src x H x 4 B, ~3% of the aggregation's reads).
 // ---------------------------------------------------------------------------
-__global__ void k_score_max(const float *__restrict__ S, int64_t lds, int64_t n_src, int32_t H,
+__global__ void k_score_max(const float *__restrict__ S, int64_t lds, int64_t n_src, int32_t H, int32_t len,
                             uint32_t *smax) {
   __shared__ uint32_t red[256];
   const int per = blockDim.x / H;  // rows per block pass; blockDim.x = per * H
   const int h = threadIdx.x % H, r = threadIdx.x / H;
   uint32_t k = 0;
-  for (int64_t row = blockIdx.x * (int64_t)per + r; row < n_src; row += (int64_t)gridDim.x * per)
-    k = max(k, fkey(__ldg(S + row * lds + h)));
+  for (int64_t row = blockIdx.x * (int64_t)per + r; row < n_src; row += (int64_t)gridDim.x * per) {
+    float x;
+    if (len == 1) {
+      x = __ldg(S + row * lds + h);
+    } else {  // Euclidean norm of the head's len-vector (GaAN's Cauchy-Schwarz bound)
+      float q = 0.0f;
+      for (int32_t i = 0; i < len; ++i) {
+        const float y = __ldg(S + row * lds + (int64_t)h * len + i);
+        q = fmaf(y, y, q);
+      }
+      x = sqrtf(q) * 1.0000005f;  // round up past sqrt's rounding (the bound must not fall below)
+    }
+    k = max(k, fkey(x));
+  }
   red[threadIdx.x] = k;
   __syncthreads();
   if (r == 0) {
@@ -149,7 +161,7 @@ __global__ void k_score_max(const float *__restrict__ S, int64_t lds, int64_t n_
   }
 }
 
-cudaError_t launch_score_max(const float *S, int64_t lds, int64_t n_src, int32_t H, uint32_t *smax,
+cudaError_t launch_score_max(const float *S, int64_t lds, int64_t n_src, int32_t H, int32_t len, uint32_t *smax,
                              cudaStream_t s) {
   cudaError_t e = cudaMemsetAsync(smax, 0, sizeof(uint32_t) * (size_t)H, s);
   if (e != cudaSuccess || n_src == 0) return e;
@@ -157,7 +169,28 @@ cudaError_t launch_score_max(const float *S, int64_t lds, int64_t n_src, int32_t
   if (threads == 0) return cudaErrorInvalidValue;
   const int per = threads / H;
   const int blocks = (int)std::max<int64_t>(1, std::min<int64_t>((n_src + per - 1) / per, (int64_t)num_sms() * 8));
-  k_score_max<<<blocks, threads, 0, s>>>(S, lds, n_src, H, smax);
+  k_score_max<<<blocks, threads, 0, s>>>(S, lds, n_src, H, len, smax);
+  count_launch();
+  return cudaGetLastError();
+}
+
+// head mean (final attention layer): y[v][f] = (1/H) sum_h Yf[v][h*Fh + f], heads in order
+__global__ void k_head_mean(const float *__restrict__ Yf, int64_t ldf, int64_t n, int32_t H, int32_t Fh, float *Y,
+                            int64_t ldy) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n * Fh; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t v = i / Fh;
+    const int32_t f = (int32_t)(i % Fh);
+    float y = 0.0f;
+    for (int32_t h = 0; h < H; ++h) y += Yf[v * ldf + (int64_t)h * Fh + f];
+    Y[v * ldy + f] = y / (float)H;
+  }
+}
+
+cudaError_t launch_head_mean(const float *Yf, int64_t ldf, int64_t n, int32_t H, int32_t Fh, float *Y, int64_t ldy,
+                             cudaStream_t s) {
+  if (n == 0) return cudaSuccess;
+  const int blocks = (int)std::min<int64_t>((n * Fh + 255) / 256, (int64_t)num_sms() * 16);
+  k_head_mean<<<blocks, 256, 0, s>>>(Yf, ldf, n, H, Fh, Y, ldy);
   count_launch();
   return cudaGetLastError();
 }
@@ -197,16 +230,24 @@ bool set_agg_mapping(int32_t vec, int32_t lanes, int32_t nv) {
 
 bool agg_override_active() { return g_override.vec != 0; }
 
+static bool is_pow2(int x) { return x > 0 && (x & (x - 1)) == 0; }
+
 static bool vec_admissible(const AggArgs &a, int32_t fh_or_0, int v) {
   bool ok = a.F % v == 0 && a.ldx % v == 0 && a.ldy % v == 0 && aligned(a.X, 4 * v) && aligned(a.Y, 4 * v);
   if (a.add_row) ok = ok && a.ld_add % v == 0 && aligned(a.add_row, 4 * v);
   if (fh_or_0) ok = ok && fh_or_0 % v == 0;
+  if (vec_score(a.mode))  // GaAN / Gene: k_v or b_v (and W_a) read as vectors; the head's lanes a power of 2
+    ok = ok && a.ldk % v == 0 && aligned(a.kb, 4 * v) && aligned(a.Wa, 4 * v) && is_pow2(fh_or_0 / v) &&
+         fh_or_0 / v <= 32;
   return ok;
 }
 
 // a4: feature-length-adaptive mapping rule
 static bool mapping_ok(const AggArgs &a, int32_t fh_or_0, const Mapping &o) {
   if (o.vec == 0 || !vec_admissible(a, fh_or_0, o.vec)) return false;
+  // the Table 2 scores other than GAT are instantiated with one vector per lane
+  if (a.mode > M_GAT && o.nv != 1) return false;
+  if (vec_score(a.mode) && fh_or_0 / o.vec > o.lanes) return false;
   // GAT: a chunk must hold whole heads (the softmax state is per head)
   const int cw = o.vec * o.lanes * o.nv;
   const bool heads_ok = !fh_or_0 || cw >= a.F || cw % fh_or_0 == 0;
@@ -224,12 +265,14 @@ static Mapping choose_mapping(const gnn_plan_s *p, const AggArgs &a, int32_t fh_
   const Mapping t{p->tuned_vec, p->tuned_lanes, p->tuned_nv};
   if (p->tuned_F == a.F && mapping_ok(a, fh_or_0, t)) return t;
   const int cands[4] = {8, 4, 2, 1};
+  m.vec = 0;
   for (int v : cands) {
     if (vec_admissible(a, fh_or_0, v)) {
       m.vec = v;
       break;
     }
   }
+  if (m.vec == 0) return Mapping{0, 0, 0};  // only the vector scores can fail (head size)
   const int nvec = a.F / m.vec;  // vectors per row
   int lanes = 4;
   while (lanes < nvec && lanes < 32) lanes *= 2;
@@ -242,7 +285,7 @@ static Mapping choose_mapping(const gnn_plan_s *p, const AggArgs &a, int32_t fh_
     // with one 32-lane worker: 19.2 vs 21.0 ms)
     m.lanes = 16;
     m.nv = 2;
-  } else if (lanes == 32) {
+  } else if (lanes == 32 && a.mode <= M_GAT) {
     const int max_nv = m.vec == 8 ? 2 : 4;
     while (m.nv < max_nv && 32 * m.nv < nvec) m.nv *= 2;
   }
@@ -250,13 +293,18 @@ static Mapping choose_mapping(const gnn_plan_s *p, const AggArgs &a, int32_t fh_
 }
 
 
-// layout: [unit counters (256 B)][GAT score max: H keys | pad 256][row counters n_multi x nch | pad 256]
-//         [acc n_multi x FW][slots x FW]
+// layout: [unit counters (256 B)][attention score maxima: H or 2H keys | pad 256]
+//         [row counters n_multi x nch | pad 256][acc n_multi x FW][slots x FW]
 static size_t smax_bytes(int mode, int32_t H) {
-  return mode == M_GAT ? ((sizeof(uint32_t) * (size_t)H + 255) & ~(size_t)255) : 0;
+  const size_t keys = (mode == M_GAT || mode == M_GAAN) ? (size_t)H : (mode == M_SYM ? 2 * (size_t)H : 0);
+  return (sizeof(uint32_t) * keys + 255) & ~(size_t)255;
 }
+// partial-slot width: F (+ m, l per head for attention), rounded up to 8 floats
+// so that every slot row is 32-byte aligned for the vector stores
+static int32_t slot_width(int mode, int32_t F, int32_t H) { return (F + (is_att(mode) ? 2 * H : 0) + 7) / 8 * 8; }
+
 size_t agg_workspace_bytes(const gnn_plan_s *p, int mode, int32_t F, int32_t H) {
-  const size_t FW = (size_t)F + (mode == M_GAT ? 2 * (size_t)H : 0);
+  const size_t FW = (size_t)slot_width(mode, F, H);
   size_t b = 256 + smax_bytes(mode, H);
   size_t c = sizeof(int32_t) * (size_t)p->n_multi * max_chunks(F);
   b += (c + 255) & ~(size_t)255;
@@ -308,7 +356,10 @@ gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, siz
   kp.H = a.H;
   kp.Fh = a.Fh;
   kp.slope = a.slope;
-  kp.FW = a.F + (mode == M_GAT ? 2 * a.H : 0);
+  kp.kb = a.kb;
+  kp.ldk = a.ldk;
+  kp.Wa = a.Wa;
+  kp.FW = slot_width(mode, a.F, a.H);
   kp.deterministic = a.deterministic;
   char *w = reinterpret_cast<char *>(ws);
   kp.ws_unit = reinterpret_cast<int32_t *>(w);
@@ -317,20 +368,25 @@ gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, siz
   kp.ws_cnt = reinterpret_cast<int32_t *>(w + 256 + sm_bytes);
   kp.ws_acc = reinterpret_cast<float *>(w + 256 + sm_bytes + cnt_bytes);
   kp.ws_part = kp.ws_acc + (size_t)p->n_multi * kp.FW;
-  const Mapping m = choose_mapping(p, a, mode == M_GAT ? a.Fh : 0);
-  const int threads = 256;
-  cudaError_t e;
-  if (mode == M_GAT) {
-    uint32_t *smax = reinterpret_cast<uint32_t *>(w + 256);
-    kp.smax = smax;
-    e = launch_score_max(a.X + a.F, a.ldx, p->n_src, a.H, smax, s);
-    if (e != cudaSuccess) return cuda_status(e, "score max launch");
+  const Mapping m = choose_mapping(p, a, is_att(mode) ? a.Fh : 0);
+  if (m.vec == 0) {
+    set_error("no supported lane mapping for this width / head size (GaAN, Gene: Fh/vec must be a power of 2 <= 32)");
+    return GNN_ERR_UNSUPPORTED;
   }
+  const int threads = 256;
+  cudaError_t e = cudaSuccess;
+  uint32_t *smax = reinterpret_cast<uint32_t *>(w + 256);
+  kp.smax = smax;
+  if (mode == M_GAT || mode == M_SYM) e = launch_score_max(a.X + a.F, a.ldx, p->n_src, a.H, 1, smax, s);
+  if (e == cudaSuccess && mode == M_SYM) e = launch_score_max(a.X + a.F + a.H, a.ldx, p->n_src, a.H, 1, smax + a.H, s);
+  if (e == cudaSuccess && mode == M_GAAN) e = launch_score_max(a.X + a.F, a.ldx, p->n_src, a.H, a.Fh, smax, s);
+  if (e != cudaSuccess) return cuda_status(e, "score max launch");
   switch (mode) {
     case M_SUM:
     case M_MEAN: e = dispatch_sum(kp, m, threads, s); break;
     case M_MAX: e = dispatch_max(kp, m, threads, s); break;
-    default: e = dispatch_gat(kp, m, threads, s); break;
+    case M_GAT: e = dispatch_gat(kp, m, threads, s); break;
+    default: e = dispatch_att(kp, m, threads, s); break;
   }
   return cuda_status(e, "aggregate launch");
 }

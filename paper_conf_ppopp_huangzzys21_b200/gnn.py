@@ -29,7 +29,8 @@ STATUS = {0: "GNN_OK", 1: "GNN_ERR_INVALID_ARG", 2: "GNN_ERR_INVALID_GRAPH", 3: 
 GNN_SUM, GNN_MEAN, GNN_MAX = 0, 1, 2
 GNN_W_ONE, GNN_W_GCN, GNN_W_EDGE = 0, 1, 2
 GNN_OP_AGGREGATE, GNN_OP_GAT_AGGREGATE, GNN_OP_EDGECONV, GNN_OP_GCN_LAYER, GNN_OP_GAT_LAYER, \
-    GNN_OP_SAGE_LSTM_LAYER = range(6)
+    GNN_OP_SAGE_LSTM_LAYER, GNN_OP_ATTN_AGGREGATE, GNN_OP_ATTN_AGGREGATE_MEAN = range(8)
+SCORES = {"gat": 0, "sym": 1, "linear": 2, "gaan": 3, "gene": 4}
 REDUCE = {"sum": GNN_SUM, "mean": GNN_MEAN, "max": GNN_MAX}
 WEIGHT = {"one": GNN_W_ONE, "gcn": GNN_W_GCN, "edge": GNN_W_EDGE}
 
@@ -100,6 +101,8 @@ _SIGS = {
     "gnn_groups_host": (ctypes.c_int, [_I64, _P, _P, _I32, ctypes.POINTER(_I64), _P, _P]),
     "gnn_launch_count": (ctypes.c_uint64, []),
     "gnn_plan_set_group_size": (ctypes.c_int, [_P, _I32]),
+    "gnn_attn_aggregate": (ctypes.c_int, [_P, ctypes.c_int, _P, _I64, _P, _I64, _P, _I32, _I32, _F, _I32, _P, _I64,
+                                          _P, _SZ, _P]),
     "gnn_sample_neighbors": (ctypes.c_int, [_P, _I32, ctypes.c_uint64, _P, _P]),
     "gnn_sage_lstm_aggregate": (ctypes.c_int, [_P, _P, _I32, _P, _I64, _I32, _P, _P, _I32, _P, _I64, _P]),
     "gnn_sage_lstm_layer": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _P, _P, _P, _P, _P, _P, _I32, _I32, _I32,
@@ -415,6 +418,21 @@ def tune_aggregate(plan: Plan, X, reduce="sum", weight="one", edge_w=None, out=N
           _tp(Y), _ld(Y, F), int(max_rounds), ctypes.byref(r), _stream(stream))
     plan._ws = {}
     return {k: getattr(r, k) for k, _ in gnn_tune_result._fields_}
+
+
+def attn_aggregate(plan: Plan, score, Zs, H, Fh, Tv=None, Wa=None, neg_slope=0.2, head_mean=False, out=None,
+                   stream=None):
+    """gnn_attn_aggregate: a Table 2 score + softmax aggregation, fused (reading R14)."""
+    torch = _torch()
+    F = H * Fh
+    width = Fh if head_mean else F
+    Y = out if out is not None else torch.empty((plan.n, width), dtype=torch.float32, device=Zs.device)
+    op = GNN_OP_ATTN_AGGREGATE_MEAN if head_mean else GNN_OP_ATTN_AGGREGATE
+    ws, nb = plan.workspace(op, 0, F, H, Zs.device)
+    _call("gnn_attn_aggregate", plan.handle, SCORES[score], _tp(Zs), Zs.stride(0), _tp(Tv),
+          0 if Tv is None else Tv.stride(0), _tp(Wa), H, Fh, neg_slope, int(head_mean), _tp(Y), _ld(Y, width),
+          _tp(ws), nb, _stream(stream))
+    return Y
 
 
 def sample_neighbors(plan: Plan, T=16, seed=0, out=None, stream=None):
