@@ -419,6 +419,61 @@ def lstm(cfg="C5"):
     return out
 
 
+def attn(cfg="C5", H=8, Fh=32):
+    """NEXT-4 Table 2 scores + softmax aggregation on a config graph: ms,
+    algorithmic GB/s, sampled parity; GaAN also against an unfused torch
+    SDDMM -> edge softmax -> SpMM pipeline."""
+    g = gs.config_graph(cfg)
+    F = H * Fh
+    plan = G.Plan(g.rowptr, g.colidx, reorder=1)
+    rng = np.random.default_rng(3)
+    rows = sample_rows(g, k=512, top=16)
+    out = {"graph": cfg, "n": g.n, "nnz": g.nnz, "H": H, "Fh": Fh, "scores": {}}
+    extra_edge = {"gat": 4 * H, "sym": 8 * H, "linear": 4 * H, "gaan": 4 * F, "gene": 4 * F}
+    extra_row = {"gat": 4 * H, "sym": 8 * H, "linear": 0, "gaan": 4 * F, "gene": 4 * F}
+    for score in ("gat", "sym", "linear", "gaan", "gene"):
+        w = F + (H if score in ("gat", "linear") else 2 * H if score == "sym" else F)
+        Zs = torch.rand((g.n, w), device=DEV) * 2 - 1
+        Tv = None
+        if score == "gat":
+            Tv = torch.rand((g.n, H), device=DEV) * 2 - 1
+        elif score in ("gaan", "gene"):
+            Tv = (torch.rand((g.n, F), device=DEV) * 2 - 1) * 0.5
+        Wa = torch.from_numpy(rng.uniform(-0.5, 0.5, size=(H, Fh)).astype(np.float32)).to(DEV) if score == "gene" else None
+        Y = torch.empty((g.n, F), device=DEV)
+        ms = events_ms(lambda: G.attn_aggregate(plan, score, Zs, H, Fh, Tv, Wa, out=Y), iters=5, warm=2)[0]
+        alg = g.nnz * (4 + 4 * F + extra_edge[score]) + g.n * (8 + 4 * F + extra_row[score])
+        ref = oracle.attn_aggregate(g.rowptr, g.colidx, score, Zs.cpu().numpy(), H, Fh,
+                                    Tv=None if Tv is None else Tv.cpu().numpy(),
+                                    Wa=None if Wa is None else Wa.cpu().numpy(), rows=rows)
+        r = {"ms": ms, "alg_GBps": alg / (ms * 1e-3) / 1e9, "parity_sampled": close(Y.cpu().numpy()[rows], ref)}
+        if score == "gaan":  # unfused: SDDMM (per-edge dot) -> edge softmax -> SpMM, torch ops
+            deg = np.diff(g.rowptr)
+            row_t = torch.from_numpy(np.repeat(np.arange(g.n), deg)).to(DEV)
+            col_t = torch.from_numpy(g.colidx.astype(np.int64)).to(DEV)
+
+            def unfused():
+                q = Zs[:, F:].view(-1, H, Fh)
+                e = (q[col_t] * Tv.view(-1, H, Fh)[row_t]).sum(-1)
+                m = torch.full((g.n, H), -float("inf"), device=DEV).scatter_reduce(
+                    0, row_t[:, None].expand(-1, H), e, "amax")
+                ex = torch.exp(e - m[row_t])
+                l_ = torch.zeros((g.n, H), device=DEV).index_add_(0, row_t, ex)
+                return torch.zeros((g.n, H, Fh), device=DEV).index_add_(
+                    0, row_t, (ex / l_[row_t])[:, :, None] * Zs[:, :F].view(-1, H, Fh)[col_t]).view(g.n, F)
+            try:
+                r["unfused_torch_ms"] = events_ms(unfused, iters=3, warm=1)[0]
+                r["speedup_vs_unfused"] = r["unfused_torch_ms"] / ms
+            except RuntimeError as exc:  # the expanded [E, H, Fh] tensors may not fit
+                r["unfused_torch_ms"] = f"failed: {str(exc)[:80]}"
+        out["scores"][score] = r
+        print(f"  {score}: {ms:.3f} ms", flush=True)
+        del Zs, Tv, Y
+        torch.cuda.empty_cache()
+    del plan
+    return out
+
+
 def fsweep():
     """F sweep (Fig 4 / Fig 12 analogue, NEXT-1): sum-aggregation throughput vs
     feature length on the C5 graph with the automatic a4 mapping."""
@@ -538,6 +593,16 @@ def summary(path):
               f"- base implementation (gather + transform every cell, torch) {c['base_impl_torch_ms']:.1f} ms -> "
               f"**{c['speedup_vs_base']:.1f}x**; parity ({c['parity_rows']} sampled rows): "
               f"{c['parity_sampled']['pass']}", ""]
+    for key in ("ATTN_C2", "ATTN_C5"):
+        if key not in d:
+            continue
+        c = d[key]
+        L += [f"## Table 2 edge functions (NEXT-4), {c['graph']}-shaped graph, {c['H']} heads x {c['Fh']}", "",
+              "| score | ms | alg GB/s | sampled parity | unfused torch ms |", "|---|---|---|---|---|"]
+        for k, v in c["scores"].items():
+            L.append(f"| {k} | {v['ms']:.3f} | {v['alg_GBps']:.0f} | {v['parity_sampled']['pass']} | "
+                     f"{v.get('unfused_torch_ms', '')} |")
+        L.append("")
     if "F_sweep" in d:
         L += ["## F sweep (C5 graph, sum, automatic a4 mapping)", "", "| F | ms | Gedge*F/s | alg GB/s |",
               "|---|---|---|---|"]
@@ -585,6 +650,9 @@ def main():
             rep["C4"] = c4()
         elif c == "LSTM":
             rep["LSTM_C5"] = lstm("C5")
+        elif c == "ATT":
+            rep["ATTN_C5"] = attn("C5")
+            rep["ATTN_C2"] = attn("C2", H=8, Fh=8)
         elif c == "FS":
             rep["F_sweep"] = fsweep()
         print(f"{c} done in {time.time() - t0:.1f}s", flush=True)
