@@ -24,8 +24,11 @@
 #include <stdint.h>
 
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 
 #include "gnn_internal.h"
+#include "tc_common.cuh"
 
 namespace gnn {
 
@@ -111,8 +114,19 @@ struct LstmParams {
   int64_t n;
 };
 
-__device__ __forceinline__ float sigm(float x) { return 1.0f / (1.0f + __expf(-x)); }
-__device__ __forceinline__ float tanh_f(float x) { return 1.0f - 2.0f / (__expf(2.0f * x) + 1.0f); }
+// sigmoid / tanh from ex2.approx and rcp.approx (2 MUFU each, no IEEE division sequence)
+__device__ __forceinline__ float rcp_s(float x) {
+  float r;
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+  return r;
+}
+__device__ __forceinline__ float ex2_s(float x) {
+  float r;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+  return r;
+}
+__device__ __forceinline__ float sigm(float x) { return rcp_s(1.0f + ex2_s(-1.4426950408889634f * x)); }
+__device__ __forceinline__ float tanh_f(float x) { return fmaf(2.0f, rcp_s(1.0f + ex2_s(-2.8853900817779268f * x)), -1.0f); }
 
 __global__ void __launch_bounds__(kLstmWarps * 32) k_sage_lstm(const LstmParams p) {
   constexpr int F = kLstmF, NB = kLstmNB;
@@ -213,9 +227,247 @@ __global__ void __launch_bounds__(kLstmWarps * 32) k_sage_lstm(const LstmParams 
   }
 }
 
+// ---------------------------------------------------------------------------
+// k_sage_lstm_tc: the recurrent product on the tensor cores.  One CTA = 128
+// center nodes (thread r = node r = TMEM lane r).  Per cell t >= 1 one thread
+// issues D[128 x 128] = h_{t-1}[128 x 32] R^T[32 x 128] as 3xTF32
+// tcgen05.mma (A = h split hi/lo, B = R split hi/lo, both K-major SW128 in
+// shared memory; D in 128 TMEM columns, column 4j+g = gate g of unit j).
+// Every thread then reads its node's 128 gate sums from TMEM (4 chunks of 32
+// columns), adds the sparse-fetched row GS[u_t] (prefetched), runs the 32
+// element-wise cells (c in registers) and writes h_t back into the A tiles
+// for the next cell.  After T cells: y = S_v + W_neigh h_T (SIMT, W_neigh^T
+// in shared memory).
+// ---------------------------------------------------------------------------
+namespace {
+constexpr int kTcTileBytes = 128 * 128;  // 128 rows x 32 fp32 (one SW128 row each)
+
+__device__ __forceinline__ float rcp_f(float x) {
+  float r;
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+  return r;
+}
+__device__ __forceinline__ float ex2_l(float x) {
+  float r;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+  return r;
+}
+constexpr float kL2e = 1.4426950408889634f;
+// 2^x on the FMA pipe (the MUFU/XU pipe is the cells' bottleneck): x = r + f,
+// r = round(x), f in [-0.5, 0.5]; 2^f by its degree-6 Taylor polynomial
+// (relative error < 2e-7); 2^r added to the exponent bits.  |x| clamped to 126.
+__device__ __forceinline__ float ex2_fma(float x) {
+  x = fminf(fmaxf(x, -126.0f), 126.0f);
+  const float big = x + 12582912.0f;  // 1.5 * 2^23: round to nearest integer in the low mantissa bits
+  const float r = big - 12582912.0f;
+  const float f = x - r;
+  float q = 1.5403530393381606e-4f;
+  q = fmaf(q, f, 1.3333558146428443e-3f);
+  q = fmaf(q, f, 9.6181291076284772e-3f);
+  q = fmaf(q, f, 5.5504108664821580e-2f);
+  q = fmaf(q, f, 2.4022650695910071e-1f);
+  q = fmaf(q, f, 6.9314718055994531e-1f);
+  q = fmaf(q, f, 1.0f);
+  return __int_as_float(__float_as_int(q) + ((__float_as_int(big) - 0x4B400000) << 23));
+}
+#ifndef GNN_LSTM_EX2_FMA
+#define GNN_LSTM_EX2_FMA 1
+#endif
+__device__ __forceinline__ float ex2_sel(float x) { return GNN_LSTM_EX2_FMA ? ex2_fma(x) : ex2_l(x); }
+__device__ __forceinline__ float sig_tc(float x) { return rcp_f(1.0f + ex2_sel(-kL2e * x)); }
+__device__ __forceinline__ float tanh_tc(float x) { return fmaf(2.0f, rcp_f(1.0f + ex2_sel(-2.0f * kL2e * x)), -1.0f); }
+}  // namespace
+
+constexpr int kTcGroups = 3;  // independent 128-node tiles per CTA (12 warps), sharing R and W_neigh
+
+// named barrier of one 128-thread group
+__device__ __forceinline__ void group_sync(int g) { asm volatile("bar.sync %0, 128;" ::"r"(g + 1) : "memory"); }
+
+__global__ void __launch_bounds__(128 * kTcGroups, 1) k_sage_lstm_tc(const LstmParams p) {
+  using namespace tc;
+  constexpr int F = kLstmF;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  const int grp = threadIdx.x >> 7;          // this thread's group (tile)
+  const int tid = threadIdx.x & 127, warp = tid >> 5;
+  uint8_t *b_hi = smem, *b_lo = smem + kTcTileBytes;
+  uint8_t *a_hi = smem + (2 + 2 * grp) * kTcTileBytes, *a_lo = a_hi + kTcTileBytes;
+  float *Wnt = reinterpret_cast<float *>(smem + (2 + 2 * kTcGroups) * kTcTileBytes);  // Wnt[j*F + o] = W_neigh[o][j]
+  __shared__ uint64_t mma_bar_all[kTcGroups];
+  __shared__ uint32_t tmem_base_sh;
+  uint64_t &mma_bar = mma_bar_all[grp];
+  // B = R^T as K-major rows: row n = 4j + g holds R[g*F + j][0..31], split hi/lo
+  for (int q = threadIdx.x; q < 128 * 8; q += blockDim.x) {
+    const int n = q >> 3, c = q & 7;
+    const int j = n >> 2, g = n & 3;
+    const float *src = p.R + (int64_t)(g * F + j) * F + 4 * c;
+    const float4 w = make_float4(src[0], src[1], src[2], src[3]);
+    const float4 hi = make_float4(hi_of(w.x), hi_of(w.y), hi_of(w.z), hi_of(w.w));
+    const float4 lo = make_float4(w.x - hi.x, w.y - hi.y, w.z - hi.z, w.w - hi.w);
+    *reinterpret_cast<float4 *>(b_hi + sw128_off(n, c)) = hi;
+    *reinterpret_cast<float4 *>(b_lo + sw128_off(n, c)) = lo;
+  }
+  for (int q = threadIdx.x; q < F * F; q += blockDim.x) {
+    const int j = q / F, o = q % F;
+    Wnt[q] = o < p.F_out ? p.Wn[o * F + j] : 0.0f;
+  }
+  if (threadIdx.x == 0) {
+    for (int g = 0; g < kTcGroups; ++g) mbar_init(&mma_bar_all[g], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (threadIdx.x < 32) {  // 512 TMEM columns: 128 per group
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_u32(&tmem_base_sh)));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;");
+  const uint32_t tmem_all = tmem_base_sh;
+  const uint32_t tmem = tmem_all + 128u * grp;                   // this group's 128 accumulator columns
+  const uint32_t taddr0 = tmem + ((uint32_t)(warp * 32) << 16);  // this warp's TMEM lane quadrant (warp id % 4)
+  const uint32_t idesc = idesc_tf32(128);
+  const int T = p.T;
+  const int64_t ntiles = (p.n + 127) / 128;
+  uint32_t phase = 0;
+  for (int64_t tile = (int64_t)blockIdx.x * kTcGroups + grp; tile < ntiles; tile += (int64_t)gridDim.x * kTcGroups) {
+    const int64_t idx = tile * 128 + tid;
+    const bool act = idx < p.n;
+    const int32_t v = act ? (p.order ? __ldg(p.order + idx) : (int32_t)idx) : -1;
+    const int32_t *tab = p.table + (int64_t)(act ? v : 0) * T;
+    int32_t u = act ? __ldg(tab) : -1;
+    const bool has = u >= 0;
+    float c[F];
+#pragma unroll
+    for (int j = 0; j < F; ++j) c[j] = 0.0f;
+    // first gathered chunk of the current cell (prefetched one cell ahead)
+    float4 g0[8];
+    auto load_chunk = [&](int32_t uu, int q, float4 (&dst)[8]) {
+      const float4 *src = reinterpret_cast<const float4 *>(p.GS + (int64_t)(uu >= 0 ? uu : 0) * p.ldg) + 8 * q;
+#pragma unroll
+      for (int i = 0; i < 8; ++i) dst[i] = uu >= 0 ? __ldg(src + i) : make_float4(0.f, 0.f, 0.f, 0.f);
+    };
+    load_chunk(u, 0, g0);
+    for (int t = 0; t < T; ++t) {
+      const int32_t un = (has && t + 1 < T) ? __ldg(tab + t + 1) : -1;
+      if (t > 0 && tid == 0) {
+        asm volatile("tcgen05.fence::after_thread_sync;");
+        const uint32_t ah = smem_u32(a_hi), al = smem_u32(a_lo), bh = smem_u32(b_hi), bl = smem_u32(b_lo);
+#pragma unroll
+        for (int ks = 0; ks < 4; ++ks) {  // K = 32 in steps of 8 tf32 (32 B)
+          const uint32_t ko = ks * 32;
+          mma_tf32(tmem, sw128_desc(al + ko), sw128_desc(bh + ko), idesc, ks > 0 ? 1u : 0u);
+          mma_tf32(tmem, sw128_desc(ah + ko), sw128_desc(bl + ko), idesc, 1u);
+          mma_tf32(tmem, sw128_desc(ah + ko), sw128_desc(bh + ko), idesc, 1u);
+        }
+        mma_commit(&mma_bar);
+      }
+      if (t > 0) {
+        mbar_wait(&mma_bar, phase);
+        phase ^= 1u;
+        asm volatile("tcgen05.fence::after_thread_sync;");
+      }
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        float4 gq[8], gn[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) gq[i] = g0[i];
+        // the next chunk of this cell (or the first chunk of the next cell) is in flight during this one
+        if (q < 3) load_chunk(has ? u : -1, q + 1, gn);
+        else load_chunk(un, 0, gn);
+        float acc[32];
+        if (t > 0) {
+          tmem_ld32(taddr0 + 32 * q, acc);
+        } else {
+#pragma unroll
+          for (int i = 0; i < 32; ++i) acc[i] = 0.0f;
+        }
+        float hv[8];
+#pragma unroll
+        for (int jj = 0; jj < 8; ++jj) {
+          const int j = 8 * q + jj;
+          const float4 gg = gq[jj];
+          const float ig = sig_tc(acc[4 * jj + 0] + gg.x);
+          const float fg = sig_tc(acc[4 * jj + 1] + gg.y);
+          const float zg = tanh_tc(acc[4 * jj + 2] + gg.z);
+          const float og = sig_tc(acc[4 * jj + 3] + gg.w);
+          c[j] = has ? fmaf(fg, c[j], ig * zg) : 0.0f;
+          hv[jj] = has ? og * tanh_tc(c[j]) : 0.0f;
+        }
+        // h_t units 8q..8q+7 -> A (row tid, 16-byte chunks 2q and 2q+1), split hi/lo
+#pragma unroll
+        for (int h2 = 0; h2 < 2; ++h2) {
+          const float4 h4 = make_float4(hv[4 * h2], hv[4 * h2 + 1], hv[4 * h2 + 2], hv[4 * h2 + 3]);
+          const float4 hi = make_float4(hi_of(h4.x), hi_of(h4.y), hi_of(h4.z), hi_of(h4.w));
+          const float4 lo = make_float4(h4.x - hi.x, h4.y - hi.y, h4.z - hi.z, h4.w - hi.w);
+          *reinterpret_cast<float4 *>(a_hi + sw128_off(tid, 2 * q + h2)) = hi;
+          *reinterpret_cast<float4 *>(a_lo + sw128_off(tid, 2 * q + h2)) = lo;
+        }
+#pragma unroll
+        for (int i = 0; i < 8; ++i) g0[i] = gn[i];
+      }
+      u = un;
+      // A complete and every TMEM read done before the next cell's MMA
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      asm volatile("tcgen05.fence::before_thread_sync;");
+      group_sync(grp);
+    }
+    // SAGE combine: y_v = S_v + W_neigh h_T (h_T = hi + lo from the A tiles, exact)
+    if (act) {
+      float h[F];
+#pragma unroll
+      for (int c4 = 0; c4 < 8; ++c4) {
+        const float4 hi = *reinterpret_cast<const float4 *>(a_hi + sw128_off(tid, c4));
+        const float4 lo = *reinterpret_cast<const float4 *>(a_lo + sw128_off(tid, c4));
+        h[4 * c4 + 0] = hi.x + lo.x;
+        h[4 * c4 + 1] = hi.y + lo.y;
+        h[4 * c4 + 2] = hi.z + lo.z;
+        h[4 * c4 + 3] = hi.w + lo.w;
+      }
+      const float *Sv = p.GS + (int64_t)v * p.ldg + 4 * F;
+      float *yv = p.Y + (int64_t)v * p.ldy;
+      for (int o = 0; o < p.F_out; ++o) {
+        float y = __ldg(Sv + o);
+#pragma unroll
+        for (int j = 0; j < F; ++j) y = fmaf(Wnt[j * F + o], h[j], y);
+        yv[o] = y;
+      }
+    }
+    group_sync(grp);  // the A tiles are rewritten by the next tile
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  if (threadIdx.x < 32) {
+    asm volatile("tcgen05.fence::after_thread_sync;");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem_all));
+  }
+}
+
+static int g_lstm_impl = 0;  // 0 = SIMT cells (default, measured faster), 1 = tensor-core cells
+int set_lstm_impl(int impl) {
+  const int old = g_lstm_impl;
+  g_lstm_impl = impl;
+  return old;
+}
+
 cudaError_t launch_sage_lstm(const gnn_plan_s *p, const int32_t *table, int32_t T, const float *GS, int64_t ldg,
                              const float *R, const float *Wn, int32_t F_out, float *Y, int64_t ldy, cudaStream_t s) {
   if (p->n == 0) return cudaSuccess;
+  if (g_lstm_impl == 1) {
+    LstmParams kp{table, T, GS, ldg, R, Wn, F_out, Y, ldy, p->dg.perm, p->n};
+    const size_t smem = (2 + 2 * kTcGroups) * kTcTileBytes + sizeof(float) * kLstmF * kLstmF + 1024;
+    static bool init = false;
+    if (!init) {
+      cudaError_t e = cudaFuncSetAttribute(k_sage_lstm_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      if (e != cudaSuccess) return e;
+      init = true;
+    }
+    const int64_t tiles = (p->n + 127) / 128;
+    const int64_t blocks = std::min<int64_t>((tiles + kTcGroups - 1) / kTcGroups, (int64_t)num_sms());
+    k_sage_lstm_tc<<<(unsigned)blocks, 128 * kTcGroups, smem, s>>>(kp);
+    count_launch();
+    return cudaGetLastError();
+  }
   LstmParams kp{table, T, GS, ldg, R, Wn, F_out, Y, ldy, p->dg.perm, p->n};
   static int occ = 0;
   if (occ == 0) {

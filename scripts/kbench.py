@@ -230,6 +230,33 @@ def tiles(cfg="C5"):
         del plan
 
 
+def lstm_probe():
+    """GraphSAGE-LSTM cell kernel on the C5 graph (for ncu / quick timing)."""
+    g = gs.config_graph("C5")
+    plan = G.Plan(g.rowptr, g.colidx, reorder=1)
+    F, T = 32, 16
+    rng = np.random.default_rng(1)
+    P = {k: torch.from_numpy(rng.uniform(-0.3, 0.3, size=s).astype(np.float32)).cuda() for k, s in
+         dict(W_hh=(4 * F, F), W_neigh=(F, F)).items()}
+    GS = torch.rand((g.n, 5 * F), device="cuda") - 0.5
+    tab = G.sample_neighbors(plan, T, 7)
+    Y = torch.empty((g.n, F), device="cuda")
+    outs = {}
+    for impl in (1, 0):
+        G.set_lstm_impl(impl)
+        ms = timeit(lambda: G.sage_lstm_aggregate(plan, tab, GS, P["W_hh"], P["W_neigh"], out=Y), iters=5, warm=2)
+        outs[impl] = Y.clone()
+        print(f" lstm cells impl={impl}: {ms:.3f} ms", flush=True)
+    print(f" tc vs simt max abs diff {float((outs[1] - outs[0]).abs().max()):.3e}", flush=True)
+    for Tp in (1, 2, 4):
+        tab2 = G.sample_neighbors(plan, Tp, 7)
+        for impl in (1, 0):
+            G.set_lstm_impl(impl)
+            ms = timeit(lambda: G.sage_lstm_aggregate(plan, tab2, GS, P["W_hh"], P["W_neigh"], out=Y), iters=5, warm=2)
+            print(f" T={Tp} impl={impl}: {ms:.3f} ms", flush=True)
+    G.set_lstm_impl(1)
+
+
 if __name__ == "__main__":
     what = sys.argv[1] if len(sys.argv) > 1 else "gemm"
     if what == "gemm":
@@ -240,6 +267,8 @@ if __name__ == "__main__":
         impls(sys.argv[sys.argv.index("--cfg") + 1] if "--cfg" in sys.argv else "C5")
     elif what == "tune":
         tune()
+    elif what == "lstm":
+        lstm_probe()
     elif what == "c1":
         c1probe()
     elif what == "map100":

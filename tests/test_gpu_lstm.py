@@ -62,9 +62,16 @@ def test_sample_neighbors_bit_exact(gname, T, seed):
     assert np.array_equal(tab, oracle.sample_neighbors(g.rowptr, g.colidx, T, seed))
 
 
+@pytest.fixture(params=[1, 0], ids=["tc", "simt"])
+def impl(request):
+    old = G.set_lstm_impl(request.param)
+    yield request.param
+    G.set_lstm_impl(old)
+
+
 @pytest.mark.parametrize("gname", list(GRAPHS))
 @pytest.mark.parametrize("f_in,F_out,T", [(32, 32, 16), (37, 7, 5), (8, 32, 1)])
-def test_sage_lstm_layer_parity(gname, f_in, F_out, T):
+def test_sage_lstm_layer_parity(gname, f_in, F_out, T, impl):
     g = GRAPHS[gname]()
     P = params(f_in, 32, F_out, 21)
     X = gs.uniform(g.n, f_in, seed=22)
@@ -76,12 +83,12 @@ def test_sage_lstm_layer_parity(gname, f_in, F_out, T):
     close(Y.cpu().numpy(), ref, f"sage lstm {gname} f_in={f_in} F_out={F_out} T={T}")
 
 
-def test_sage_lstm_aggregate_from_host_pretransform():
+def test_sage_lstm_aggregate_from_host_pretransform(impl):
     """The fused cell kernel alone: GS (gates interleaved per unit, then the
     self term) prepared on the host in fp64 from the oracle's definition."""
     g = GRAPHS["small"]()
     f_in, F, F_out, T = 32, 32, 32, 16
-    P = params(f_in, F, F_out, 5, scale=0.5)
+    P = params(f_in, F, F_out, 5, scale=1.0)
     X = gs.uniform(g.n, f_in, seed=6)
     Xd = X.astype(np.float64)
     G4 = Xd @ P["W_ih"].astype(np.float64).T + P["b_ih"] + P["b_hh"]        # [n, 4F] blocks i, f, z, o
@@ -104,7 +111,7 @@ def test_sage_lstm_rejects_unsupported_hidden_size():
     assert e.value.status == 6
 
 
-def test_sage_lstm_rerun_identical():
+def test_sage_lstm_rerun_identical(impl):
     g = GRAPHS["hub"]()
     P = params(32, 32, 32, 2)
     X = T_(gs.uniform(g.n, 32, seed=3))
