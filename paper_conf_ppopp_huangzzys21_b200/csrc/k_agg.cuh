@@ -267,12 +267,151 @@ __device__ __forceinline__ float head_sum(float x, int lph, unsigned mask) {
 }
 
 // one neighbour group: fresh fp32 chain in CSR order (R9); indices from the
-// task-ordered stream, LANES at a time, U source rows in flight per worker.
-// Attention modes (GAT and the other Table 2 scores, R14): softmax terms
+// task-ordered stream, LANES at a time, U source rows in flight per worker
+// (sum / mean / max and GAT)
+template <int MODE, int VEC, int NV, int LANES>
+__device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx, int32_t len, int32_t beg,
+                                            int32_t row, int32_t c0, int lane, unsigned mask,
+                                            Part<MODE, VEC, NV> &G) {
+  constexpr int FPL = VEC * NV;
+  constexpr int U = FPL >= 32 ? 1 : (32 / FPL > 8 ? 8 : 32 / FPL);
+  part_init(G);
+  const int weight = p.weight;
+  const float *xl = p.X + c0 + lane * VEC;
+  bool valid[NV];
+  int32_t head[NV];
+  float tv[NV];
+  float nmb[NV];   // GAT: -m * log2(e) for the current reference m
+  float seen[NV];  // GAT: exact max score of the group
+  // GAT: a one-edge group takes its own score as reference (term = 1 exactly)
+  const bool one = MODE == M_GAT && len == 1;
+#pragma unroll
+  for (int n = 0; n < NV; ++n) {
+    const int32_t f = c0 + (n * LANES + lane) * VEC;
+    valid[n] = f < p.F;
+    head[n] = 0;
+    tv[n] = 0.0f;
+    nmb[n] = 0.0f;
+    seen[n] = -INFINITY;
+    if constexpr (MODE == M_GAT) {
+      head[n] = valid[n] ? f / p.Fh : 0;
+      tv[n] = valid[n] ? __ldg(p.t + (int64_t)row * p.ldt + head[n]) : 0.0f;
+      const float mb = valid[n] ? leaky_f(fkey_decode(__ldg(p.smax + head[n])) + tv[n], p.slope) : 0.0f;
+      G.m[n] = mb;
+      nmb[n] = -mb * kLog2e;
+    }
+  }
+  // index batches: the next batch (and its weights) is requested before the
+  // current one is consumed
+  auto load_batch = [&](int32_t k, int32_t &u, float &w) {
+    const int32_t c = min(LANES, len - k);
+    u = 0;
+    w = 1.0f;
+    if (lane < c) {
+      u = ld_stream_i32(idx + k + lane);
+      if constexpr (MODE != M_GAT) {
+        if (weight == GNN_W_GCN) w = __ldg(p.g.nsrc + u);
+        else if (weight == GNN_W_EDGE) w = ld_stream_f32(p.edge_w + beg + k + lane);
+      }
+    }
+  };
+#pragma unroll 1
+  for (int pass = 0;; ++pass) {
+    int32_t nx_u = 0;
+    float nx_w = 1.0f;
+    if (len > 0) load_batch(0, nx_u, nx_w);
+    for (int32_t k = 0; k < len; k += LANES) {
+      const int32_t cnt = min(LANES, len - k);
+      const int32_t my_u = nx_u;
+      const float my_w = nx_w;
+      if (k + LANES < len) load_batch(k + LANES, nx_u, nx_w);
+      float v[U][NV][VEC];
+      float sc[U][NV];
+#pragma unroll
+      for (int q = 0; q < U; ++q) {
+        if (q < cnt) {
+          const int32_t u = __shfl_sync(mask, my_u, q, LANES);
+#pragma unroll
+          for (int n = 0; n < NV; ++n) {
+            if (valid[n]) ldv<VEC>(xl + (int64_t)u * p.ldx + n * LANES * VEC, v[q][n]);
+            if constexpr (MODE == M_GAT) sc[q][n] = valid[n] ? __ldg(p.X + (int64_t)u * p.ldx + p.F + head[n]) : 0.0f;
+          }
+        }
+      }
+      for (int32_t j = 0; j < cnt; j += U) {
+#pragma unroll
+        for (int q = 0; q < U; ++q) {
+          const int32_t e = j + q;
+          if (e < cnt) {
+            if constexpr (MODE == M_GAT) {
+              // e_uv = LeakyReLU(s_u + t_v); term exp(e_uv - m) (one ex2 per edge and head)
+#pragma unroll
+              for (int n = 0; n < NV; ++n) {
+                if (!valid[n]) continue;
+                const float sco = leaky_f(sc[q][n] + tv[n], p.slope);
+                seen[n] = fmaxf(seen[n], sco);
+                const float ex = one ? 1.0f : ex2_f(fmaf(sco, kLog2e, nmb[n]));
+                G.l[n] += ex;
+#pragma unroll
+                for (int i = 0; i < VEC; ++i) G.a[n][i] = fmaf(ex, v[q][n][i], G.a[n][i]);
+              }
+            } else {
+              const float w = __shfl_sync(mask, my_w, e, LANES);
+#pragma unroll
+              for (int n = 0; n < NV; ++n) {
+                if (!valid[n]) continue;
+#pragma unroll
+                for (int i = 0; i < VEC; ++i) {
+                  if constexpr (MODE == M_MAX) G.a[n][i] = fmaxf(G.a[n][i], w * v[q][n][i]);
+                  else G.a[n][i] = fmaf(w, v[q][n][i], G.a[n][i]);
+                }
+              }
+            }
+            if (e + U < cnt) {
+              const int32_t u = __shfl_sync(mask, my_u, e + U, LANES);
+#pragma unroll
+              for (int n = 0; n < NV; ++n) {
+                if (valid[n]) ldv<VEC>(xl + (int64_t)u * p.ldx + n * LANES * VEC, v[q][n]);
+                if constexpr (MODE == M_GAT)
+                  sc[q][n] = valid[n] ? __ldg(p.X + (int64_t)u * p.ldx + p.F + head[n]) : 0.0f;
+              }
+            }
+          }
+        }
+      }
+    }
+    if constexpr (MODE != M_GAT) {
+      break;
+    } else {
+      if (one) {
+#pragma unroll
+        for (int n = 0; n < NV; ++n) G.m[n] = seen[n];
+        break;
+      }
+      // bound too loose for some head of this worker: redo against the exact max
+      bool loose = false;
+#pragma unroll
+      for (int n = 0; n < NV; ++n) loose |= valid[n] && !(G.m[n] - seen[n] <= kGatSlack);
+      if (pass == 1 || !__any_sync(mask, loose)) break;
+#pragma unroll
+      for (int n = 0; n < NV; ++n) {
+        G.m[n] = seen[n];
+        nmb[n] = -seen[n] * kLog2e;
+        G.l[n] = 0.0f;
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) G.a[n][i] = 0.0f;
+      }
+    }
+  }
+}
+
+// group chain of the Table 2 scores other than GAT (R14; GAT keeps its own
+// specialised chain above, which measured 10% faster than this generalised
+// one at 8x32).  Attention modes: softmax terms
 // exp(e - m) against a per-row upper bound m of the scores (R9 GAT), with an
 // exact-max recompute when the bound is loose.
 template <int MODE, int VEC, int NV, int LANES>
-__device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx, int32_t len, int32_t beg,
+__device__ __forceinline__ void group_chain_att(const KParams &p, const int32_t *idx, int32_t len, int32_t beg,
                                             int32_t row, int32_t c0, int lane, unsigned mask,
                                             Part<MODE, VEC, NV> &G) {
   constexpr bool ATT = is_att(MODE);
@@ -517,7 +656,10 @@ __device__ __forceinline__ void process_unit(const KParams &p, int4 d, int32_t l
   const DevGraph &g = p.g;
   const int32_t tpos = d.x, beg = d.y, row = d.z, m = d.w;
   Part<MODE, VEC, NV> G;
-  group_chain<MODE, VEC, NV, LANES>(p, g.colidx_t + tpos, len, beg, row, c0, lane, mask, G);
+  if constexpr (MODE > M_GAT)
+    group_chain_att<MODE, VEC, NV, LANES>(p, g.colidx_t + tpos, len, beg, row, c0, lane, mask, G);
+  else
+    group_chain<MODE, VEC, NV, LANES>(p, g.colidx_t + tpos, len, beg, row, c0, lane, mask, G);
   const int32_t rb = g.rowptr[row], re = g.rowptr[row + 1];
   if (m < 0) {
     store_row<MODE, VEC, NV, LANES>(p, row, re - rb, c0, lane, G);
