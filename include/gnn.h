@@ -337,22 +337,6 @@ gnn_status gnn_gcn_aggregate_prescaled(gnn_plan_t plan, const float *Hs, int64_t
  * X Wext = [Z | s | t] (Table 2 GAT scores as extra GEMM columns).
  * W: [f_in, H*Fh] row-major; Wext: [f_in, ldwe], ldwe >= H*Fh + 2H.
  */
-/*
- * GAT projection with the scores in the GEMM epilogue (a5 + Table 2 GAT):
- * Zst[u] = [Z_u | s_u | t_u], Z = X W ([m, H*Fh], 3xTF32 tcgen05), s_u[h] =
- * <Z_u^h, a_src^h>, t_u[h] = <Z_u^h, a_dst^h> (fp32 dot of the fp32 Z row).
- * The tensor-core width stays H*Fh (the folded alternative below widens it to
- * H*Fh + 2H, which costs the TMEM double buffer at H*Fh = 256).  W: [f_in,
- * H*Fh] row-major; Zst: [m, ldz], ldz >= H*Fh + 2H.  Workspace:
- * gnn_gemm_workspace_size(m, f_in, H*Fh).  GNN_ERR_UNSUPPORTED when the
- * tcgen05 GEMM does not take the shape (then fold + gnn_gemm).  Measured at
- * C5 (2.45M x 256 -> 8 x 32): 3.07 ms vs 2.95 ms for fold + gnn_gemm, so the
- * layers use the folded form; kept as an alternative entry point.
- */
-gnn_status gnn_gat_project(const float *X, int64_t ldx, int32_t f_in, const float *W, const float *a_src,
-                           const float *a_dst, int32_t H, int32_t Fh, float *Zst, int64_t ldz, int64_t m,
-                           void *ws, size_t ws_bytes, gnn_stream_t stream);
-
 gnn_status gnn_gat_fold_weights(const float *W, const float *a_src, const float *a_dst,
                                 int32_t f_in, int32_t H, int32_t Fh, float *Wext, int64_t ldwe,
                                 gnn_stream_t stream);

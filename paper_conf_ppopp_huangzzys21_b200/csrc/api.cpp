@@ -461,8 +461,7 @@ gnn_status gnn_gat_layer(gnn_plan_t p, const float *X, int64_t ldx, int32_t f_in
     float *Wext = (float *)(base + gws);
     float *Zst = (float *)(base + gws + align256(sizeof(float) * (size_t)f_in * ldwe));
     cudaStream_t s = (cudaStream_t)stream;
-    // [Z | s | t]: the scores as extra GEMM columns X (W_h a_h) (R5); the
-    // epilogue variant (gnn_gat_project) measured slower at C5 (3.07 vs 2.95 ms)
+    // [Z | s | t]: the scores as extra GEMM columns X (W_h a_h) (R5)
     cudaError_t e = launch_gat_weights(W, a_src, a_dst, f_in, H, Fh, Wext, ldwe, s);
     if (e != cudaSuccess) return cuda_status(e, "gat weights");
     gnn_status st = launch_gemm(X, ldx, Wext, ldwe, Zst, ldwe, p->n, f_in, ldwe, nullptr, nullptr, 0, base, gws, s);
@@ -865,17 +864,5 @@ gnn_status gnn_attn_aggregate(gnn_plan_t p, int score, const float *Zs, int64_t 
 }
 
 int gnn_set_lstm_impl(int impl) { return set_lstm_impl(impl); }
-
-gnn_status gnn_gat_project(const float *X, int64_t ldx, int32_t f_in, const float *W, const float *a_src,
-                           const float *a_dst, int32_t H, int32_t Fh, float *Zst, int64_t ldz, int64_t m, void *ws,
-                           size_t ws_bytes, gnn_stream_t stream) {
-  GNN_TRY({
-    if (H < 1 || Fh < 1 || f_in < 1 || m < 0) return check(false, "H, Fh, f_in >= 1 and m >= 0 required");
-    if (m > 0 && (!X || !W || !a_src || !a_dst || !Zst)) return check(false, "NULL argument");
-    if (ldx < f_in || ldz < (int64_t)H * Fh + 2 * H) return check(false, "leading dimension too small");
-    return launch_gemm_gat(X, ldx, W, (int64_t)H * Fh, Zst, ldz, m, f_in, H, Fh, a_src, a_dst, ws, ws_bytes,
-                           (cudaStream_t)stream);
-  })
-}
 
 }  // extern "C"

@@ -134,9 +134,6 @@ gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, siz
                             cudaStream_t s);
 
 // GEMM (k_gemm.cu)
-gnn_status launch_gemm_gat(const float *X, int64_t ldx, const float *W, int64_t ldw, float *Zst, int64_t ldz,
-                           int64_t m, int32_t k, int32_t H, int32_t Fh, const float *a_src, const float *a_dst,
-                           void *ws, size_t ws_bytes, cudaStream_t s);
 gnn_status launch_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H,
                        int64_t ldh, int64_t m, int32_t k, int32_t n, const float *row_scale,
                        const float *col_bias, int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s);

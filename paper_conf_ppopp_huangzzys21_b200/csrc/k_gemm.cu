@@ -124,30 +124,7 @@ int set_gemm_impl(int impl) {
 // is outside what the tcgen05 kernel takes
 cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H,
                            int64_t ldh, int64_t m, int32_t k, int32_t n, const float *row_scale,
-                           const float *col_bias, int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s,
-                           const float *att_src = nullptr, const float *att_dst = nullptr, int32_t att_H = 0,
-                           int32_t att_Fh = 0);
-
-// GAT projection [Z | s | t] = [X W | <Z^h, a_src^h> | <Z^h, a_dst^h>] with the
-// scores computed in the tcgen05 GEMM's epilogue (MMA width H*Fh, not
-// H*Fh + 2H).  GNN_ERR_UNSUPPORTED when the tcgen05 path does not take the shape.
-gnn_status launch_gemm_gat(const float *X, int64_t ldx, const float *W, int64_t ldw, float *Zst, int64_t ldz,
-                           int64_t m, int32_t k, int32_t H, int32_t Fh, const float *a_src, const float *a_dst,
-                           void *ws, size_t ws_bytes, cudaStream_t s) {
-  if (m == 0) return GNN_OK;
-  if (g_gemm_impl == 1 || !ws) {
-    set_error("GAT projection epilogue needs the tcgen05 GEMM");
-    return GNN_ERR_UNSUPPORTED;
-  }
-  cudaError_t e = launch_gemm_tc(X, ldx, W, ldw, Zst, ldz, m, k, H * Fh, nullptr, nullptr, 0, ws, ws_bytes, s,
-                                 a_src, a_dst, H, Fh);
-  if (e == cudaErrorNotSupported) {
-    (void)cudaGetLastError();
-    set_error("tcgen05 GEMM does not take this GAT projection shape");
-    return GNN_ERR_UNSUPPORTED;
-  }
-  return cuda_status(e, "gat projection launch");
-}
+                           const float *col_bias, int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s);
 
 gnn_status launch_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H,
                        int64_t ldh, int64_t m, int32_t k, int32_t n, const float *row_scale,

@@ -27,23 +27,86 @@
 #include <stdint.h>
 
 #include "gnn_internal.h"
-#include "tc_common.cuh"
 
 namespace gnn {
 namespace tc {
 
+constexpr int BM = 128;
+constexpr int BK = 32;  // fp32 elements per 128-byte swizzle row
 constexpr int NUM_PRODUCER_WARPS = 4;
-// producer groups take K blocks round-robin; each holds its next X tile in
-// registers, so PRODUCER_GROUPS K blocks of X are in flight per CTA
-#ifndef GNN_GEMM_PRODUCER_GROUPS
-#define GNN_GEMM_PRODUCER_GROUPS 2
-#endif
-constexpr int PRODUCER_GROUPS = GNN_GEMM_PRODUCER_GROUPS;
 constexpr int MMA_WARP = 4;
 constexpr int EPI_WARP0 = 5;
 constexpr int THREADS = 32 * 9;
 constexpr int TILE_A_BYTES = BM * BK * 4;  // 16 KB per hi or lo
 constexpr int MAX_STAGES = 6;
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t"
+      ".reg .pred P1;\n\t"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+      "@!P1 bra WAIT_%=;\n\t"
+      "}\n" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
+}
+
+// UMMA shared-memory descriptor: K-major, SWIZZLE_128B, 8-row atoms of 1024 B
+__device__ __forceinline__ uint64_t sw128_desc(uint32_t saddr) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr & 0x3FFFF) >> 4);  // start address >> 4 (bits 0-13)
+  d |= (uint64_t)1 << 16;                   // leading byte offset (unused: swizzled K-major)
+  d |= (uint64_t)(1024 >> 4) << 32;         // stride byte offset: 8 rows x 128 B
+  d |= (uint64_t)1 << 46;                   // descriptor version (sm_100)
+  d |= (uint64_t)2 << 61;                   // SWIZZLE_128B
+  return d;
+}
+
+// instruction descriptor: D f32, A/B tf32, both K-major, M = 128, N = n
+__host__ __device__ constexpr uint32_t idesc_tf32(int n) {
+  return (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+}
+
+__device__ __forceinline__ void mma_tf32(uint32_t tmem_d, uint64_t da, uint64_t db, uint32_t idesc,
+                                         uint32_t accumulate) {
+  asm volatile(
+      "{\n\t"
+      ".reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t"
+      "}\n" ::"r"(tmem_d),
+      "l"(da), "l"(db), "r"(idesc), "r"(accumulate));
+}
+__device__ __forceinline__ void mma_commit(uint64_t *bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
+               : "memory");
+}
+
+__device__ __forceinline__ float hi_of(float x) { return __uint_as_float(__float_as_uint(x) & 0xFFFFE000u); }
+
+// byte offset of 16-byte chunk c (0..7) of row r inside a SW128 K-major tile
+__host__ __device__ __forceinline__ uint32_t sw128_off(int r, int c) {
+  return (uint32_t)((r >> 3) * 1024 + (r & 7) * 128 + ((c ^ (r & 7)) << 4));
+}
 
 // W image: for each K block kb: [hi tile | lo tile], each NP rows (n) x 128 B,
 // K-major, swizzled exactly as in shared memory.
@@ -80,10 +143,6 @@ struct TcParams {
   const float *row_scale;
   const float *col_bias;
   int32_t relu;
-  // GAT score epilogue (att_H > 0): s_u[h] = <Z_u^h, a_src^h>, t_u[h] = <Z_u^h, a_dst^h>
-  // written to columns n + h and n + H + h of the output row (Table 2 GAT)
-  const float *att_src, *att_dst;
-  int32_t att_H, att_Fh;
 };
 
 template <bool VEC_X, bool VEC_H>
@@ -100,17 +159,10 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p) {
   const int warp = tid >> 5;
   const int lane = tid & 31;
   const int S = p.stages;
-  // GAT epilogue: a_src | a_dst (NP each, zero padded) after the pipeline stages
-  float *att_sm = reinterpret_cast<float *>(smem + (size_t)p.stages * STAGE_BYTES);
-  if (p.att_H > 0)
-    for (int i = threadIdx.x; i < 2 * NP; i += blockDim.x) {
-      const int c = i % NP;
-      att_sm[i] = c < p.n ? __ldg((i < NP ? p.att_src : p.att_dst) + c) : 0.0f;
-    }
 
   if (tid == 0) {
     for (int s = 0; s < S; ++s) {
-      mbar_init(&full_bar[s], NUM_PRODUCER_WARPS * 32 / PRODUCER_GROUPS + 1);  // one group's A arrivals + 1 expect_tx
+      mbar_init(&full_bar[s], NUM_PRODUCER_WARPS * 32 / 2 + 1);  // 64 A arrivals (one group) + 1 expect_tx
       mbar_init(&empty_bar[s], 1);
     }
     for (int b = 0; b < 2; ++b) {
@@ -134,9 +186,9 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p) {
     // the global K-block counter it = g, g+2, ...); each group loads its next
     // X tile into registers before waiting for its stage, so two K blocks of
     // X are in flight per CTA while the MMAs run.
-    constexpr int GROUP_THREADS = NUM_PRODUCER_WARPS * 32 / PRODUCER_GROUPS;
-    constexpr int PER_THREAD = BM * 8 / GROUP_THREADS;                     // float4 chunks per thread
-    const int grp = warp / (NUM_PRODUCER_WARPS / PRODUCER_GROUPS);
+    constexpr int GROUP_THREADS = NUM_PRODUCER_WARPS * 32 / 2;           // 64
+    constexpr int PER_THREAD = BM * 8 / GROUP_THREADS;                     // 16 float4 chunks
+    const int grp = warp >> 1;                                             // 0 or 1
     const int gtid = tid - grp * GROUP_THREADS;
     float4 buf[PER_THREAD];
     auto load_a = [&](int64_t m0, int kb) {
@@ -195,7 +247,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p) {
       // generic-proxy smem writes -> visible to the tensor core (async proxy)
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       mbar_arrive(&full_bar[s]);
-      it += PRODUCER_GROUPS;
+      it += 2;
       if (it < total_it) load_a((int64_t)tile_of(it) * BM, it % p.num_kb);
     }
   } else if (warp == MMA_WARP) {
@@ -251,7 +303,6 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p) {
       const float sc = (p.row_scale && gm < p.m) ? __ldg(p.row_scale + gm) : 1.0f;
       const uint32_t tbase = tmem + (uint32_t)(b * p.n_acc * p.npa) + ((uint32_t)(quad * 32) << 16);
       const int n_acc_used = p.num_kb < p.n_acc ? p.num_kb : p.n_acc;
-      float ps = 0.0f, pt = 0.0f;  // GAT score partials of the current head (Fh >= 32)
       for (int c0 = 0; c0 < NP; c0 += 32) {
         float y[32];
 #pragma unroll
@@ -281,45 +332,6 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p) {
           if (p.col_bias && col < p.n) t = t + __ldg(p.col_bias + col);
           if (p.relu) t = t > 0.0f ? t : 0.0f;
           y[i] = t;
-        }
-        if (p.att_H > 0) {
-          // GAT scores from the fp32 Z row: products with a_src (then a_dst),
-          // staged in shared memory, reduced over each head (Fh = 8, 16 or a
-          // multiple of 32) by pairwise levels
-          float *srow = p.H + gm * p.ldh + p.n;
-#pragma unroll 1
-          for (int which = 0; which < 2; ++which) {
-            const float4 *a4 = reinterpret_cast<const float4 *>(att_sm + which * NP + c0);
-            float q[32];
-#pragma unroll
-            for (int i = 0; i < 8; ++i) {
-              const float4 a = a4[i];
-              q[4 * i] = y[4 * i] * a.x;
-              q[4 * i + 1] = y[4 * i + 1] * a.y;
-              q[4 * i + 2] = y[4 * i + 2] * a.z;
-              q[4 * i + 3] = y[4 * i + 3] * a.w;
-            }
-#pragma unroll
-            for (int w = 1; w < 32; w <<= 1) {
-#pragma unroll
-              for (int i = 0; i < 32; i += 2 * w) q[i] += q[i + w];
-              if (w * 2 == p.att_Fh && p.att_Fh < 32) {
-#pragma unroll
-                for (int i = 0; i < 32; i += 2 * w) {
-                  const int hh = (c0 + i) / p.att_Fh;
-                  if (hh < p.att_H) srow[which * p.att_H + hh] = q[i];
-                }
-              }
-            }
-            if (p.att_Fh >= 32) {
-              float &acc = which ? pt : ps;
-              acc += q[0];
-              if ((c0 + 32) % p.att_Fh == 0 && c0 < p.n) {
-                srow[which * p.att_H + c0 / p.att_Fh] = acc;
-                acc = 0.0f;
-              }
-            }
-          }
         }
         float *dst = p.H + gm * p.ldh + c0;
         if (VEC_H && c0 + 32 <= p.n) {
@@ -386,8 +398,7 @@ size_t gemm_tc_workspace(int64_t m, int32_t k, int32_t n) {
 
 cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H, int64_t ldh,
                            int64_t m, int32_t k, int32_t n, const float *row_scale, const float *col_bias,
-                           int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s, const float *att_src,
-                           const float *att_dst, int32_t att_H, int32_t att_Fh) {
+                           int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s) {
   using namespace tc;
   Config c;
   if (!configure(m, k, n, c)) return cudaErrorNotSupported;
@@ -409,22 +420,15 @@ cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t 
   const int64_t num_tiles = (m + BM - 1) / BM;
   if (num_tiles > 0x7fffffff) return cudaErrorNotSupported;
   TcParams p{X, ldx, H, ldh, img, m, k, n, c.np, c.npa, c.num_kb, (int32_t)num_tiles, c.stages, c.n_acc, c.n_buf,
-             row_scale, col_bias, relu, att_src, att_dst, att_src ? att_H : 0, att_Fh};
+             row_scale, col_bias, relu};
   const bool vx = (ldx % 4 == 0) && ((uintptr_t)X % 16 == 0);
   const bool vh = (ldh % 4 == 0) && ((uintptr_t)H % 16 == 0);
   auto fn = vx ? (vh ? k_gemm_tc<true, true> : k_gemm_tc<true, false>)
                : (vh ? k_gemm_tc<false, true> : k_gemm_tc<false, false>);
-  size_t smem = c.smem;
-  if (att_src) {
-    // the epilogue reduces per head: Fh in {8, 16} or a multiple of 32
-    if (!(att_Fh == 8 || att_Fh == 16 || att_Fh % 32 == 0)) return cudaErrorNotSupported;
-    smem += sizeof(float) * 2 * (size_t)c.np;
-    if (smem > 227 * 1024) return cudaErrorNotSupported;
-  }
-  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c.smem);
   if (e != cudaSuccess) return e;
   const int grid = (int)(num_tiles < num_sms ? num_tiles : num_sms);
-  fn<<<grid, THREADS, smem, s>>>(p);
+  fn<<<grid, THREADS, c.smem, s>>>(p);
   count_launch();
   return cudaGetLastError();
 }

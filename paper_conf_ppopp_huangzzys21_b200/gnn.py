@@ -104,7 +104,6 @@ _SIGS = {
     "gnn_attn_aggregate": (ctypes.c_int, [_P, ctypes.c_int, _P, _I64, _P, _I64, _P, _I32, _I32, _F, _I32, _P, _I64,
                                           _P, _SZ, _P]),
     "gnn_set_lstm_impl": (ctypes.c_int, [ctypes.c_int]),
-    "gnn_gat_project": (ctypes.c_int, [_P, _I64, _I32, _P, _P, _P, _I32, _I32, _P, _I64, _I64, _P, _SZ, _P]),
     "gnn_sample_neighbors": (ctypes.c_int, [_P, _I32, ctypes.c_uint64, _P, _P]),
     "gnn_sage_lstm_aggregate": (ctypes.c_int, [_P, _P, _I32, _P, _I64, _I32, _P, _P, _I32, _P, _I64, _P]),
     "gnn_sage_lstm_layer": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _P, _P, _P, _P, _P, _P, _I32, _I32, _I32,

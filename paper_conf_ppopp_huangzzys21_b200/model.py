@@ -171,8 +171,7 @@ class RowPartitionedGCNGAT:
                                             self.ws_agg_b, sp), "agg2")
         rec(4)
         z_loc = self.Zst[off:off + R]
-        # [Z | s | t]: scores as extra GEMM columns X (W_h a_h) (R5).  (gnn_gat_project,
-        # the scores in the GEMM epilogue, measured 3.07 vs 2.95 ms at C5 and is not used.)
+        # [Z | s | t]: scores as extra GEMM columns X (W_h a_h) (R5)
         chk(lib.gnn_gat_fold_weights(P(self.W3), P(self.a_s), P(self.a_d), F, H, self.Fh, P(self.Wext), self.ldwe,
                                      sp), "gat fold")
         chk(lib.gnn_gemm(P(self.Y2), F, P(self.Wext), self.ldwe, P(z_loc), self.ldwe, R, F, self.ldwe, None, None, 0,

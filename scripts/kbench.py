@@ -157,44 +157,6 @@ def tune():
         del plan
 
 
-def gatproj():
-    """GAT projection: scores in the GEMM epilogue vs folded as extra columns;
-    the aggregation time on each [Z | s | t]."""
-    g = gs.config_graph("C5")
-    plan = G.Plan(g.rowptr, g.colidx, reorder=1)
-    H, Fh, F = 8, 32, 256
-    HF = H * Fh
-    ld = HF + 2 * H
-    Y2 = torch.rand((g.n, F), device="cuda") * 2 - 1
-    lim = float(np.sqrt(6 / (F + HF)))
-    W = (torch.rand((F, HF), device="cuda") * 2 - 1) * lim
-    al = float(np.sqrt(6 / (Fh + 1)))
-    a_s = (torch.rand(HF, device="cuda") * 2 - 1) * al
-    a_d = (torch.rand(HF, device="cuda") * 2 - 1) * al
-    Z1 = torch.empty((g.n, ld), device="cuda")
-    Z2 = torch.empty((g.n, ld), device="cuda")
-    Wext = torch.empty((F, ld), device="cuda")
-    ws, nb = G.gnn.gemm_workspace(g.n, F, ld, "cuda")
-    GN = G.gnn
-
-    def proj():
-        assert GN.gnn_gat_project(Y2.data_ptr(), F, F, W.data_ptr(), a_s.data_ptr(), a_d.data_ptr(), H, Fh,
-                                  Z1.data_ptr(), ld, g.n, ws.data_ptr(), nb, None) == 0
-
-    def fold():
-        assert GN.gnn_gat_fold_weights(W.data_ptr(), a_s.data_ptr(), a_d.data_ptr(), F, H, Fh, Wext.data_ptr(), ld,
-                                       None) == 0
-        G.gemm(Y2, Wext, out=Z2)
-    print(f" project (epilogue scores): {timeit(proj):.3f} ms | fold (272 columns): {timeit(fold):.3f} ms", flush=True)
-    d = (Z1 - Z2).abs()
-    print(f" max |diff| Z {float(d[:, :HF].max()):.3e} s,t {float(d[:, HF:].max()):.3e}", flush=True)
-    Y = torch.empty((g.n, HF), device="cuda")
-    for name, Z in (("project", Z1), ("fold", Z2)):
-        t = Z[:, HF + H:]
-        print(f" gat_aggregate on {name}: {timeit(lambda: G.gat_aggregate(plan, Z, t, H, Fh, out=Y)):.3f} ms",
-              flush=True)
-
-
 def c1probe():
     """C1 (Cora) aggregate calls for an ncu launch list (launch-bound config)."""
     g = gs.config_graph("C1")
@@ -307,8 +269,6 @@ if __name__ == "__main__":
         tune()
     elif what == "lstm":
         lstm_probe()
-    elif what == "gatproj":
-        gatproj()
     elif what == "c1":
         c1probe()
     elif what == "map100":
