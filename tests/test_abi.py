@@ -162,3 +162,25 @@ def test_local_csr_translation(nparts):
         for q in range(nparts):
             want[q * rmax: q * rmax + (b[q + 1] - b[q])] = d_out[b[q]:b[q + 1]]
         assert np.array_equal(sdeg, want)
+
+
+def test_new_entry_points_reject_null_plans():
+    """NEXT-1/3/4 entry points validate before touching the device."""
+    g = P.gnn
+    r = g.gnn_tune_result()
+    assert g.gnn_tune_aggregate(None, 0, 0, None, None, 1, 1, None, 1, 0, ctypes.byref(r), None) == 1
+    assert g.gnn_plan_set_group_size(None, 16) == 1
+    assert g.gnn_sample_neighbors(None, 16, 0, None, None) == 1
+    assert g.gnn_sage_lstm_aggregate(None, None, 16, None, 160, 32, None, None, 32, None, 32, None) == 1
+    assert g.gnn_sage_lstm_layer(None, None, 32, 32, None, None, None, None, None, None, None, 32, 32, 16, 0, None, 32,
+                                 None, 0, None) == 1
+    assert g.gnn_attn_aggregate(None, 0, None, 9, None, 1, None, 1, 8, 0.2, 0, None, 8, None, 0, None) == 1
+    assert g.gnn_workspace_size(None, 6, 0, 64, 8) == 0
+
+
+def test_lstm_and_agg_impl_switches_roundtrip():
+    g = P.gnn
+    old = g.gnn_set_lstm_impl(1)
+    assert g.gnn_set_lstm_impl(old) == 1
+    old = g.gnn_set_agg_impl(0)
+    assert g.gnn_set_agg_impl(old) == 0
