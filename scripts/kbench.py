@@ -157,6 +157,38 @@ def tune():
         del plan
 
 
+def c2gat():
+    """GAT mappings on the arxiv-shaped graph (C2, 8 heads x 8)."""
+    g = gs.config_graph("C2")
+    plan = G.Plan(g.rowptr, g.colidx, reorder=1)
+    H, Fh = 8, 8
+    HF = H * Fh
+    Zs = torch.rand((g.n, HF + 2 * H), device="cuda") * 2 - 1
+    t = Zs[:, HF + H:]
+    Y = torch.empty((g.n, HF), device="cuda")
+    ref = None
+    X = torch.rand((g.n, HF), device="cuda")
+    for m in [(0, 0, 0), (4, 32, 1), (2, 32, 1), (1, 32, 1)]:
+        G.set_agg_mapping(*m)
+        ms = timeit(lambda: G.aggregate(plan, X, "sum", "gcn", out=Y), iters=20, warm=3)
+        print(f" C2 sum F=64 map {m}: {ms * 1e3:.1f} us", flush=True)
+    g1 = gs.config_graph("C1")
+    p1 = G.Plan(g1.rowptr, g1.colidx, reorder=1)
+    X1 = torch.rand((g1.n, 16), device="cuda")
+    Y1 = torch.empty_like(X1)
+    for m in [(0, 0, 0), (4, 32, 1), (2, 32, 1), (1, 32, 1), (8, 4, 1)]:
+        G.set_agg_mapping(*m)
+        ms = timeit(lambda: G.aggregate(p1, X1, "sum", "gcn", out=Y1), iters=50, warm=5)
+        print(f" C1 sum F=16 map {m}: {ms * 1e3:.1f} us", flush=True)
+    for m in [(0, 0, 0), (4, 32, 1), (8, 32, 1), (2, 32, 1), (4, 16, 1), (8, 8, 1)]:
+        G.set_agg_mapping(*m)
+        ms = timeit(lambda: G.gat_aggregate(plan, Zs, t, H, Fh, out=Y), iters=20, warm=3)
+        d = 0.0 if ref is None else float((Y - ref).abs().max())
+        ref = Y.clone() if ref is None else ref
+        print(f" C2 GAT map {m}: {ms * 1e3:.1f} us  max|diff| {d:.2e}", flush=True)
+    G.set_agg_mapping(0, 0, 0)
+
+
 def c1probe():
     """C1 (Cora) aggregate calls for an ncu launch list (launch-bound config)."""
     g = gs.config_graph("C1")
@@ -269,6 +301,8 @@ if __name__ == "__main__":
         tune()
     elif what == "lstm":
         lstm_probe()
+    elif what == "c2gat":
+        c2gat()
     elif what == "c1":
         c1probe()
     elif what == "map100":
