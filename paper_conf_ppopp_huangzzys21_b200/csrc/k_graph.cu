@@ -273,12 +273,12 @@ static Mapping choose_mapping(const gnn_plan_s *p, const AggArgs &a, int32_t fh_
     }
   }
   if (m.vec == 0) return Mapping{0, 0, 0};  // only the vector scores can fail (head size)
-  // short rows (average degree < 16) and narrow features: the chain of a
+  // short rows (average degree < 32) and narrow features: the chain of a
   // group is latency-bound, so one 32-lane worker per group with 16-byte
   // vectors (32 indices per batch, 8 source rows in flight) beats narrow
   // workers (tuner on C1 F=16: 30 -> 21 us; C2 F=64: 0.226 -> 0.147 ms)
   const double avg_deg = p->n > 0 ? (double)p->nnz / (double)p->n : 0.0;
-  if (avg_deg < 16.0 && a.F <= 128 && a.mode <= M_GAT) {
+  if (avg_deg < 32.0 && a.F <= 128 && a.mode <= M_GAT) {
     // vectors of F/32 floats so that all 32 lanes hold features (C2 GAT 8x8:
     // (2, 32, 1) 170 us vs 241 us for the default (8, 8, 1))
     int v = 1;

@@ -189,6 +189,21 @@ def c2gat():
     G.set_agg_mapping(0, 0, 0)
 
 
+def c4map():
+    """EdgeConv max aggregation mappings on the kNN graph (C4, F=64, k=20)."""
+    g = gs.config_graph("C4")
+    plan = G.Plan(g.rowptr, g.colidx, reorder=1)
+    PQ = torch.rand((g.n, 128), device="cuda") * 2 - 1
+    Y = torch.empty((g.n, 64), device="cuda")
+    X = torch.rand((g.n, 64), device="cuda")
+    for m in [(0, 0, 0), (2, 32, 1), (4, 32, 1), (8, 8, 1), (4, 16, 1)]:
+        G.set_agg_mapping(*m)
+        a = timeit(lambda: G.edgeconv_aggregate(plan, PQ, 64, out=Y), iters=50, warm=5)
+        b = timeit(lambda: G.aggregate(plan, X, "sum", "gcn", out=Y), iters=50, warm=5)
+        print(f" C4 map {m}: edgeconv max {a * 1e3:.1f} us | sum gcn {b * 1e3:.1f} us", flush=True)
+    G.set_agg_mapping(0, 0, 0)
+
+
 def c1probe():
     """C1 (Cora) aggregate calls for an ncu launch list (launch-bound config)."""
     g = gs.config_graph("C1")
@@ -303,6 +318,8 @@ if __name__ == "__main__":
         lstm_probe()
     elif what == "c2gat":
         c2gat()
+    elif what == "c4map":
+        c4map()
     elif what == "c1":
         c1probe()
     elif what == "map100":
