@@ -125,8 +125,25 @@ __device__ __forceinline__ float ex2_s(float x) {
   asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
   return r;
 }
-__device__ __forceinline__ float sigm(float x) { return rcp_s(1.0f + ex2_s(-1.4426950408889634f * x)); }
-__device__ __forceinline__ float tanh_f(float x) { return fmaf(2.0f, rcp_s(1.0f + ex2_s(-2.8853900817779268f * x)), -1.0f); }
+// 1/x for x in [1, 2^64] on the FMA pipe: integer seed (relative error < 1/8)
+// and three Newton steps (error < (1/8)^8 ~ 6e-8).  The SIMT cells keep
+// rcp.approx (measured: Newton 10.8 ms vs 9.8 ms — they are issue-bound, not
+// MUFU-bound); the tensor-core cells use it (FMA pipe otherwise idle).
+__device__ __forceinline__ float rcp_nr(float x) {
+  float r = __int_as_float(0x7EF311C7 - __float_as_int(x));
+  r = r * fmaf(-x, r, 2.0f);
+  r = r * fmaf(-x, r, 2.0f);
+  r = r * fmaf(-x, r, 2.0f);
+  return r;
+}
+#ifndef GNN_LSTM_RCP_NR
+#define GNN_LSTM_RCP_NR 0
+#endif
+__device__ __forceinline__ float rcp_sel(float x) { return GNN_LSTM_RCP_NR ? rcp_nr(x) : rcp_s(x); }
+__device__ __forceinline__ float sigm(float x) { return rcp_sel(1.0f + ex2_s(fminf(-1.4426950408889634f * x, 64.0f))); }
+__device__ __forceinline__ float tanh_f(float x) {
+  return fmaf(2.0f, rcp_sel(1.0f + ex2_s(fminf(-2.8853900817779268f * x, 64.0f))), -1.0f);
+}
 
 __global__ void __launch_bounds__(kLstmWarps * 32) k_sage_lstm(const LstmParams p) {
   constexpr int F = kLstmF, NB = kLstmNB;
@@ -274,8 +291,12 @@ __device__ __forceinline__ float ex2_fma(float x) {
 #define GNN_LSTM_EX2_FMA 1
 #endif
 __device__ __forceinline__ float ex2_sel(float x) { return GNN_LSTM_EX2_FMA ? ex2_fma(x) : ex2_l(x); }
-__device__ __forceinline__ float sig_tc(float x) { return rcp_f(1.0f + ex2_sel(-kL2e * x)); }
-__device__ __forceinline__ float tanh_tc(float x) { return fmaf(2.0f, rcp_f(1.0f + ex2_sel(-2.0f * kL2e * x)), -1.0f); }
+// tensor-core cells: the FMA pipe is free, so both ex2 (polynomial) and the
+// reciprocal (Newton) run there; arguments clamped to <= 64 (see rcp_nr)
+__device__ __forceinline__ float sig_tc(float x) { return rcp_nr(1.0f + ex2_sel(fminf(-kL2e * x, 64.0f))); }
+__device__ __forceinline__ float tanh_tc(float x) {
+  return fmaf(2.0f, rcp_nr(1.0f + ex2_sel(fminf(-2.0f * kL2e * x, 64.0f))), -1.0f);
+}
 }  // namespace
 
 constexpr int kTcGroups = 3;  // independent 128-node tiles per CTA (12 warps), sharing R and W_neigh

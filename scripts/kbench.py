@@ -204,6 +204,23 @@ def c4map():
     G.set_agg_mapping(0, 0, 0)
 
 
+def pad104():
+    """agg1 of the bench (GCN weights) at F=100 vs the same rows padded to 104."""
+    g = gs.config_graph("C5")
+    plan = G.Plan(g.rowptr, g.colidx, reorder=1)
+    X = torch.rand((g.n, 104), device="cuda")
+    X[:, 100:] = 0
+    Y = torch.empty_like(X)
+    Y100 = torch.empty((g.n, 100), device="cuda")
+    X100 = X[:, :100].contiguous()
+    print(f" F=100 (ld 100): {timeit(lambda: G.aggregate(plan, X100, 'sum', 'gcn', out=Y100)):.3f} ms", flush=True)
+    for m in [(0, 0, 0), (8, 32, 1), (4, 16, 2), (4, 32, 1)]:
+        G.set_agg_mapping(*m)
+        ms = timeit(lambda: G.aggregate(plan, X, "sum", "gcn", out=Y))
+        print(f" F=104 map {m}: {ms:.3f} ms  same as F=100 {bool(torch.equal(Y[:, :100], Y100))}", flush=True)
+    G.set_agg_mapping(0, 0, 0)
+
+
 def c1probe():
     """C1 (Cora) aggregate calls for an ncu launch list (launch-bound config)."""
     g = gs.config_graph("C1")
@@ -320,6 +337,8 @@ if __name__ == "__main__":
         c2gat()
     elif what == "c4map":
         c4map()
+    elif what == "pad104":
+        pad104()
     elif what == "c1":
         c1probe()
     elif what == "map100":
