@@ -259,11 +259,6 @@ __global__ void __launch_bounds__(kLstmWarps * 32) k_sage_lstm(const LstmParams 
 namespace {
 constexpr int kTcTileBytes = 128 * 128;  // 128 rows x 32 fp32 (one SW128 row each)
 
-__device__ __forceinline__ float rcp_f(float x) {
-  float r;
-  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
-  return r;
-}
 __device__ __forceinline__ float ex2_l(float x) {
   float r;
   asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
@@ -464,7 +459,143 @@ __global__ void __launch_bounds__(128 * kTcGroups, 1) k_sage_lstm_tc(const LstmP
   }
 }
 
-static int g_lstm_impl = 0;  // 0 = SIMT cells (default, measured faster), 1 = tensor-core cells
+
+// ---------------------------------------------------------------------------
+// k_sage_lstm_mma: the recurrent product on warp-level tensor-core MMAs
+// (mma.sync m16n8k8 TF32, 3xTF32 split) inside a SIMT-style layout.  One warp
+// = 16 center nodes (the MMA's M).  Per cell, the warp computes the gate
+// pre-activations D[16 x 128] = G[u_t] + h_{t-1} R^T as 16 n-tiles of 8
+// columns (gate column 4j+g); the accumulator fragments are initialised with
+// the sparse-fetched rows G[u_t] (each lane loads 8 B of two rows per tile,
+// so a warp instruction reads 32 B of 8 rows), h_{t-1} comes from a per-warp
+// shared buffer as A fragments (hi/lo), R^T fragments from shared memory
+// (pre-split, one float4 per lane per (tile, k-step)).  A lane pair
+// (tig, tig^1) holds the four gates of one unit for two rows; one xor-shuffle
+// each gives every lane its own (row, unit) cell.
+// ---------------------------------------------------------------------------
+constexpr int kMmaWarps = 4;
+
+__device__ __forceinline__ void mma_tf32_16x8x8(float (&d)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
+  asm volatile(
+      "mma.sync.aligned.m16n8k8.row.col.f32.tf32.tf32.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+      "{%0,%1,%2,%3};"
+      : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
+      : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
+}
+
+__device__ __forceinline__ float hi19(float x) { return __uint_as_float(__float_as_uint(x) & 0xFFFFE000u); }
+
+__global__ void __launch_bounds__(kMmaWarps * 32) k_sage_lstm_mma(const LstmParams p) {
+  constexpr int F = kLstmF;
+  // B fragments of R^T per (n-tile, k-step, lane): (b0_hi, b1_hi, b0_lo, b1_lo)
+  __shared__ float4 Bf[16][4][32];
+  __shared__ float Wnt[F][F + 1];
+  __shared__ float hb[kMmaWarps][16][F + 1];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int gid = lane >> 2, tig = lane & 3;
+  for (int q = tid; q < 16 * 4 * 32; q += blockDim.x) {
+    const int nt = q / 128, ks = (q / 32) % 4, l = q % 32;
+    const int n = 8 * nt + (l >> 2);          // gate column (4j + g)
+    const int j = n >> 2, g = n & 3;
+    const int k0 = 8 * ks + (l & 3), k1 = k0 + 4;
+    const float w0 = p.R[(g * F + j) * F + k0], w1 = p.R[(g * F + j) * F + k1];
+    const float h0 = hi19(w0), h1 = hi19(w1);
+    Bf[nt][ks][l] = make_float4(h0, h1, w0 - h0, w1 - h1);
+  }
+  for (int i = tid; i < F * F; i += blockDim.x) {
+    const int j = i / F, o = i % F;
+    Wnt[j][o] = o < p.F_out ? p.Wn[o * F + j] : 0.0f;
+  }
+  __syncthreads();
+  const int T = p.T;
+  float (*h)[F + 1] = hb[warp];
+  for (int64_t base = ((int64_t)blockIdx.x * kMmaWarps + warp) * 16; base < p.n;
+       base += (int64_t)gridDim.x * kMmaWarps * 16) {
+    // rows gid and gid + 8 of this warp's 16 nodes
+    int32_t v[2];
+    bool has[2];
+#pragma unroll
+    for (int r = 0; r < 2; ++r) {
+      const int64_t idx = base + gid + 8 * r;
+      v[r] = idx < p.n ? (p.order ? __ldg(p.order + idx) : (int32_t)idx) : -1;
+      has[r] = v[r] >= 0 && __ldg(p.table + (int64_t)v[r] * T) >= 0;
+    }
+    // this lane's cells: row (tig odd ? gid + 8 : gid), units 2nt + tig/2
+    const int myr = tig & 1;
+    float c[16];
+#pragma unroll
+    for (int nt = 0; nt < 16; ++nt) c[nt] = 0.0f;
+    for (int i = lane; i < 16 * F; i += 32) h[i / F][i % F] = 0.0f;
+    __syncwarp();
+    for (int t = 0; t < T; ++t) {
+      int32_t u[2];
+#pragma unroll
+      for (int r = 0; r < 2; ++r) u[r] = has[r] ? __ldg(p.table + (int64_t)v[r] * T + t) : -1;
+      // A fragments of h_{t-1} (rows gid, gid+8; k = 8ks + tig, + 4), split hi/lo
+      uint32_t ah[4][4], al[4][4];
+#pragma unroll
+      for (int ks = 0; ks < 4; ++ks) {
+        const float x[4] = {h[gid][8 * ks + tig], h[gid + 8][8 * ks + tig], h[gid][8 * ks + tig + 4],
+                            h[gid + 8][8 * ks + tig + 4]};
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const float hi = hi19(x[i]);
+          ah[ks][i] = __float_as_uint(hi);
+          al[ks][i] = __float_as_uint(x[i] - hi);
+        }
+      }
+      __syncwarp();  // every lane has its A fragments before h is overwritten
+#pragma unroll
+      for (int nt = 0; nt < 16; ++nt) {
+        // accumulator = the gathered pre-activations G[u] (2 columns x 2 rows)
+        float d[4];
+#pragma unroll
+        for (int r = 0; r < 2; ++r) {
+          float2 gg = make_float2(0.f, 0.f);
+          if (u[r] >= 0) gg = __ldg(reinterpret_cast<const float2 *>(p.GS + (int64_t)u[r] * p.ldg + 8 * nt + 2 * tig));
+          d[2 * r] = gg.x;
+          d[2 * r + 1] = gg.y;
+        }
+        if (t > 0) {
+#pragma unroll
+          for (int ks = 0; ks < 4; ++ks) {
+            const float4 b = Bf[nt][ks][lane];
+            mma_tf32_16x8x8(d, al[ks], __float_as_uint(b.x), __float_as_uint(b.y));
+            mma_tf32_16x8x8(d, ah[ks], __float_as_uint(b.z), __float_as_uint(b.w));
+            mma_tf32_16x8x8(d, ah[ks], __float_as_uint(b.x), __float_as_uint(b.y));
+          }
+        }
+        // lanes tig even hold (i, f), odd hold (z, o) of unit 2nt + tig/2 for rows gid (d0,d1), gid+8 (d2,d3):
+        // even keeps row gid and receives (z, o) of row gid; odd keeps row gid+8 and receives (i, f)
+        const float s0 = myr ? d[0] : d[2], s1 = myr ? d[1] : d[3];
+        const float r0 = __shfl_xor_sync(0xffffffffu, s0, 1), r1 = __shfl_xor_sync(0xffffffffu, s1, 1);
+        const float gi = myr ? r0 : d[0], gf = myr ? r1 : d[1];
+        const float gz = myr ? d[2] : r0, go = myr ? d[3] : r1;
+        const int j = 2 * nt + (tig >> 1);
+        const int row = gid + 8 * myr;
+        if (has[myr]) {
+          c[nt] = fmaf(sigm(gf), c[nt], sigm(gi) * tanh_f(gz));
+          h[row][j] = sigm(go) * tanh_f(c[nt]);
+        }
+      }
+      __syncwarp();
+    }
+    // SAGE combine: lane o computes output o of the 16 nodes
+#pragma unroll 1
+    for (int r = 0; r < 16; ++r) {
+      const int64_t idx = base + r;
+      if (idx >= p.n || lane >= p.F_out) continue;
+      const int32_t vv = p.order ? __ldg(p.order + idx) : (int32_t)idx;
+      float y = __ldg(p.GS + (int64_t)vv * p.ldg + 4 * F + lane);
+#pragma unroll 8
+      for (int j = 0; j < F; ++j) y = fmaf(Wnt[j][lane], h[r][j], y);
+      p.Y[(int64_t)vv * p.ldy + lane] = y;
+    }
+    __syncwarp();
+  }
+}
+
+static int g_lstm_impl = 0;  // 0 = SIMT cells (default), 1 = tcgen05 cells, 2 = mma.sync cells
 int set_lstm_impl(int impl) {
   const int old = g_lstm_impl;
   g_lstm_impl = impl;
@@ -474,6 +605,19 @@ int set_lstm_impl(int impl) {
 cudaError_t launch_sage_lstm(const gnn_plan_s *p, const int32_t *table, int32_t T, const float *GS, int64_t ldg,
                              const float *R, const float *Wn, int32_t F_out, float *Y, int64_t ldy, cudaStream_t s) {
   if (p->n == 0) return cudaSuccess;
+  if (g_lstm_impl == 2) {
+    LstmParams kp{table, T, GS, ldg, R, Wn, F_out, Y, ldy, p->dg.perm, p->n};
+    static int occ = 0;
+    if (occ == 0) {
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sage_lstm_mma, kMmaWarps * 32, 0);
+      if (occ <= 0) occ = 1;
+    }
+    const int64_t per_cta = (int64_t)kMmaWarps * 16;
+    const int64_t blocks = std::min<int64_t>((p->n + per_cta - 1) / per_cta, (int64_t)num_sms() * occ);
+    k_sage_lstm_mma<<<(unsigned)blocks, kMmaWarps * 32, 0, s>>>(kp);
+    count_launch();
+    return cudaGetLastError();
+  }
   if (g_lstm_impl == 1) {
     LstmParams kp{table, T, GS, ldg, R, Wn, F_out, Y, ldy, p->dg.perm, p->n};
     const size_t smem = (2 + 2 * kTcGroups) * kTcTileBytes + sizeof(float) * kLstmF * kLstmF + 1024;

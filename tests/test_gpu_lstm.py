@@ -62,7 +62,7 @@ def test_sample_neighbors_bit_exact(gname, T, seed):
     assert np.array_equal(tab, oracle.sample_neighbors(g.rowptr, g.colidx, T, seed))
 
 
-@pytest.fixture(params=[1, 0], ids=["tc", "simt"])
+@pytest.fixture(params=[1, 0, 2], ids=["tc", "simt", "mma"])
 def impl(request):
     old = G.set_lstm_impl(request.param)
     yield request.param
