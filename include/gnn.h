@@ -190,7 +190,11 @@ gnn_status gnn_aggregate(gnn_plan_t plan, int reduce, int weight, const float *e
  * e_uv = LeakyReLU(s_u[h] + t_v[h], neg_slope), alpha = softmax_v(e),
  * y_v[h] = SUM_u alpha_uv z_u[h].  Edge scores never reach HBM.
  *   Zs: [n_src, ldz] rows = [z_u (H*Fh floats) | s_u (H floats)], ldz >= H*Fh+H.
- *   t:  [n, ldt] (t_v per head).  Y: [n, ldy], ldy >= H*Fh.
+ *   t:  [n, ldt] (t_v per head).  Y: [n, ldy], ldy >= H*Fh.  1 <= H <= 256.
+ * The softmax is shifted by the per-row bound LeakyReLU(max_u s_u[h] + t_v[h])
+ * (one extra pass over the n_src x H score columns; R9).  Inputs
+ * must be finite; rows of Zs that no CSR entry references still enter that
+ * maximum, so padding rows should hold finite values (zeros).
  */
 gnn_status gnn_gat_aggregate(gnn_plan_t plan, const float *Zs, int64_t ldz,
                              const float *t, int64_t ldt, int32_t H, int32_t Fh,

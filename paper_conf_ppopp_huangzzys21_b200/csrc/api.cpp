@@ -385,7 +385,7 @@ gnn_status gnn_gat_aggregate(gnn_plan_t p, const float *Zs, int64_t ldz, const f
                              size_t ws_bytes, gnn_stream_t stream) {
   GNN_TRY({
     if (!p) return check(false, "plan is NULL");
-    if (H < 1 || Fh < 1) return check(false, "H and Fh must be >= 1");
+    if (H < 1 || Fh < 1 || H > 256) return check(false, "H in [1, 256] and Fh >= 1 required");
     const int32_t F = H * Fh;
     if (!Y || !t || (p->nnz > 0 && !Zs)) return check(false, "Zs/t/Y is NULL");
     if (ldz < F + H || ldt < H || ldy < F) return check(false, "ldz < H*Fh+H or ldt < H or ldy < H*Fh");
@@ -445,7 +445,7 @@ gnn_status gnn_gat_layer(gnn_plan_t p, const float *X, int64_t ldx, int32_t f_in
   GNN_TRY({
     if (!p) return check(false, "plan is NULL");
     if (p->n != p->n_src) return check(false, "gnn_gat_layer needs a square plan (n_src == n)");
-    if (H < 1 || Fh < 1 || f_in < 1) return check(false, "H, Fh, f_in must be >= 1");
+    if (H < 1 || H > 256 || Fh < 1 || f_in < 1) return check(false, "H in [1, 256], Fh, f_in >= 1 required");
     if (!X || !W || !a_src || !a_dst || !Y) return check(false, "NULL argument");
     if (ldx < f_in || ldy < (int64_t)H * Fh) return check(false, "leading dimension too small");
     const int32_t HF = H * Fh;

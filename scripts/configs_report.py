@@ -292,6 +292,25 @@ def c3(rho, ncu_pass=False):
             Xh = np.ascontiguousarray(X[:, :F_in])
             ref1 = oracle.gcn_layer(g.rowptr, g.colidx, Xh, W1, relu=True, rows=rows)
             r["parity_layer1_sampled"] = close(Y1.cpu().numpy()[rows], ref1)
+            # epilogue fused vs separate (linear-property postponement):
+            # ndst scaling + ReLU in the aggregation's epilogue vs an extra
+            # elementwise pass over Y (torch op standing for the separate kernel)
+            Hs2 = torch.rand((g.n, F), device=DEV) - 0.5
+            Yf = torch.empty((g.n, F), device=DEV)
+            ws_f, nb_f = plan.workspace(GN.GNN_OP_AGGREGATE, 0, F, 0, DEV)
+            deg = np.diff(g.rowptr).astype(np.float32)
+            ndst = torch.from_numpy(np.where(deg > 0, 1.0 / np.sqrt(np.maximum(deg, 1)), 0).astype(np.float32)).to(DEV)
+
+            def fused():
+                GN._call("gnn_gcn_aggregate_prescaled", plan.handle, GN._tp(Hs2), F, F, GN._tp(Yf), F, 1,
+                         GN._tp(ws_f), nb_f, None)
+
+            def separate():
+                G.aggregate(plan, Hs2, "sum", "one", out=Yf)
+                Yf.mul_(ndst[:, None]).relu_()
+            r["epilogue_fused_ms"] = events_ms(fused, iters=5)[0]
+            r["epilogue_separate_ms"] = events_ms(separate, iters=5)[0]
+            del Hs2, Yf
             # layer 2 as a standalone layer on its own seeded input (no oracle
             # input ever comes from the GPU path)
             X2 = gs.uniform(g.n, F, lo=0.0, hi=1.0, seed=gs.seed_of("C3", 1) + 1)
@@ -569,6 +588,9 @@ def summary(path):
                      f"{v['aggregate_alg_GBps']:.0f} | {n.get('dram_bytes', 0) / 1e9:.1f} | "
                      f"{n.get('dram_GBps') or 0:.0f} | {n.get('l2_hit_pct')} | {v['plan_build_s']:.2f} |")
         v = c["variants"]["las_ng"]
+        if "epilogue_fused_ms" in v:
+            L += ["", f"- epilogue (x ndst, ReLU) fused into the aggregation {v['epilogue_fused_ms']:.2f} ms vs a "
+                  f"separate elementwise pass {v['epilogue_separate_ms']:.2f} ms"]
         L += ["", f"- layers: L1 {v['layer1_ms']:.2f} ms, L2 {v['layer2_ms']:.2f} ms; GEMM1 {v['gemm1_ms']:.3f} ms "
               f"({v['gemm1_TFLOPs']:.0f} TF/s), GEMM2 {v['gemm2_ms']:.3f} ms ({v['gemm2_TFLOPs']:.0f} TF/s)",
               f"- parity ({v['parity_rows']} sampled rows incl. the 32 largest): L1 {v['parity_layer1_sampled']['pass']}, "
