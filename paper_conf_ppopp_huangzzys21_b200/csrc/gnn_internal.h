@@ -10,6 +10,22 @@
 
 #include "../../include/gnn.h"
 
+#ifdef __CUDACC__
+namespace gnn {
+// Blackwell packed fp32 FMA (FFMA2): (a0, a1) = (x0, x1) * s + (a0, a1), each
+// lane rounded once exactly like fmaf, so chains stay bit-identical; one
+// instruction for two FMAs (ptxas folds the broadcast of s into the operand)
+__device__ __forceinline__ void fma2_bcast(float &a0, float &a1, float x0, float x1, float s) {
+  unsigned long long acc, xx, ss;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(acc) : "f"(a0), "f"(a1));
+  asm("mov.b64 %0, {%1, %2};" : "=l"(xx) : "f"(x0), "f"(x1));
+  asm("mov.b64 %0, {%1, %1};" : "=l"(ss) : "f"(s));
+  asm("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(acc) : "l"(xx), "l"(ss));
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(a0), "=f"(a1) : "l"(acc));
+}
+}  // namespace gnn
+#endif
+
 namespace gnn {
 
 // Device-side view of a plan handed to the graph kernels (all int32: the

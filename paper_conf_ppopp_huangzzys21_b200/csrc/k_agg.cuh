@@ -120,6 +120,18 @@ __device__ __forceinline__ float ld_stream_f32(const float *p) {
   return r;
 }
 
+// a[i] = fmaf(s, x[i], a[i]) for i < VEC, as packed FFMA2 pairs (bit-identical)
+template <int VEC>
+__device__ __forceinline__ void fma_vec(float (&a)[VEC], const float (&x)[VEC], float s) {
+  if constexpr (VEC % 2 == 0) {
+#pragma unroll
+    for (int i = 0; i < VEC; i += 2) fma2_bcast(a[i], a[i + 1], x[i], x[i + 1], s);
+  } else {
+#pragma unroll
+    for (int i = 0; i < VEC; ++i) a[i] = fmaf(s, x[i], a[i]);
+  }
+}
+
 // fixed ReLU: y > 0 ? y : +0 (matches the oracle replica, R9)
 __device__ __forceinline__ float relu_f(float y) { return y > 0.0f ? y : 0.0f; }
 
@@ -352,18 +364,18 @@ __device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx
                 seen[n] = fmaxf(seen[n], sco);
                 const float ex = one ? 1.0f : ex2_f(fmaf(sco, kLog2e, nmb[n]));
                 G.l[n] += ex;
-#pragma unroll
-                for (int i = 0; i < VEC; ++i) G.a[n][i] = fmaf(ex, v[q][n][i], G.a[n][i]);
+                fma_vec<VEC>(G.a[n], v[q][n], ex);
               }
             } else {
               const float w = __shfl_sync(mask, my_w, e, LANES);
 #pragma unroll
               for (int n = 0; n < NV; ++n) {
                 if (!valid[n]) continue;
+                if constexpr (MODE == M_MAX) {
 #pragma unroll
-                for (int i = 0; i < VEC; ++i) {
-                  if constexpr (MODE == M_MAX) G.a[n][i] = fmaxf(G.a[n][i], w * v[q][n][i]);
-                  else G.a[n][i] = fmaf(w, v[q][n][i], G.a[n][i]);
+                  for (int i = 0; i < VEC; ++i) G.a[n][i] = fmaxf(G.a[n][i], w * v[q][n][i]);
+                } else {
+                  fma_vec<VEC>(G.a[n], v[q][n], w);
                 }
               }
             }
@@ -560,18 +572,18 @@ __device__ __forceinline__ void group_chain_att(const KParams &p, const int32_t 
                 seen[n] = fmaxf(seen[n], sco[n]);
                 const float ex = one ? 1.0f : ex2_f(fmaf(sco[n], kLog2e, nmb[n]));
                 G.l[n] += ex;
-#pragma unroll
-                for (int i = 0; i < VEC; ++i) G.a[n][i] = fmaf(ex, v[q][n][i], G.a[n][i]);
+                fma_vec<VEC>(G.a[n], v[q][n], ex);
               }
             } else {
               const float w = __shfl_sync(mask, my_w, e, LANES);
 #pragma unroll
               for (int n = 0; n < NV; ++n) {
                 if (!valid[n]) continue;
+                if constexpr (MODE == M_MAX) {
 #pragma unroll
-                for (int i = 0; i < VEC; ++i) {
-                  if constexpr (MODE == M_MAX) G.a[n][i] = fmaxf(G.a[n][i], w * v[q][n][i]);
-                  else G.a[n][i] = fmaf(w, v[q][n][i], G.a[n][i]);
+                  for (int i = 0; i < VEC; ++i) G.a[n][i] = fmaxf(G.a[n][i], w * v[q][n][i]);
+                } else {
+                  fma_vec<VEC>(G.a[n], v[q][n], w);
                 }
               }
             }

@@ -200,22 +200,15 @@ __global__ void __launch_bounds__(kLstmWarps * 32) k_sage_lstm(const LstmParams 
 #pragma unroll
         for (int n = 0; n < NB; ++n) {
           const float4 h4 = *reinterpret_cast<const float4 *>(&hb[warp][n][k]);
-          acc[n].x = fmaf(r0.x, h4.x, acc[n].x);
-          acc[n].y = fmaf(r0.y, h4.x, acc[n].y);
-          acc[n].z = fmaf(r0.z, h4.x, acc[n].z);
-          acc[n].w = fmaf(r0.w, h4.x, acc[n].w);
-          acc[n].x = fmaf(r1.x, h4.y, acc[n].x);
-          acc[n].y = fmaf(r1.y, h4.y, acc[n].y);
-          acc[n].z = fmaf(r1.z, h4.y, acc[n].z);
-          acc[n].w = fmaf(r1.w, h4.y, acc[n].w);
-          acc[n].x = fmaf(r2.x, h4.z, acc[n].x);
-          acc[n].y = fmaf(r2.y, h4.z, acc[n].y);
-          acc[n].z = fmaf(r2.z, h4.z, acc[n].z);
-          acc[n].w = fmaf(r2.w, h4.z, acc[n].w);
-          acc[n].x = fmaf(r3.x, h4.w, acc[n].x);
-          acc[n].y = fmaf(r3.y, h4.w, acc[n].y);
-          acc[n].z = fmaf(r3.z, h4.w, acc[n].z);
-          acc[n].w = fmaf(r3.w, h4.w, acc[n].w);
+          // the same fmaf chains as pairs of packed FMAs (FFMA2, bit-identical)
+          fma2_bcast(acc[n].x, acc[n].y, r0.x, r0.y, h4.x);
+          fma2_bcast(acc[n].z, acc[n].w, r0.z, r0.w, h4.x);
+          fma2_bcast(acc[n].x, acc[n].y, r1.x, r1.y, h4.y);
+          fma2_bcast(acc[n].z, acc[n].w, r1.z, r1.w, h4.y);
+          fma2_bcast(acc[n].x, acc[n].y, r2.x, r2.y, h4.z);
+          fma2_bcast(acc[n].z, acc[n].w, r2.z, r2.w, h4.z);
+          fma2_bcast(acc[n].x, acc[n].y, r3.x, r3.y, h4.w);
+          fma2_bcast(acc[n].z, acc[n].w, r3.z, r3.w, h4.w);
         }
       }
       __syncwarp();
