@@ -250,6 +250,7 @@ size_t gnn_gemm_workspace_size(int64_t m, int32_t k, int32_t n);
  * 2 = tcgen05 3xTF32.  Returns the previous value. */
 int gnn_set_gemm_impl(int impl);
 
+
 /*
  * a4 mapping override (process-wide; the hook of the paper's mapping tuner,
  * P:1128-1168): every later graph op whose F, strides and pointers
