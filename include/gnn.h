@@ -247,7 +247,10 @@ gnn_status gnn_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw, fl
 size_t gnn_gemm_workspace_size(int64_t m, int32_t k, int32_t n);
 
 /* GEMM implementation selector (process-wide): 0 = auto, 1 = SIMT FFMA,
- * 2 = tcgen05 3xTF32.  Returns the previous value. */
+ * 2 = tcgen05 3xTF32, 3 = tcgen05 3xTF32 with register-fed X tiles instead
+ * of TMA (same results bit for bit; kept for A/B measurement).  Under 0 and
+ * 2 the X tiles arrive by TMA (cp.async.bulk.tensor, SWIZZLE_128B) whenever
+ * X and ldx are 16-byte aligned.  Returns the previous value. */
 int gnn_set_gemm_impl(int impl);
 
 

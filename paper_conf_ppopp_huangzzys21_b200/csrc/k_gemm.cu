@@ -112,11 +112,14 @@ __global__ void __launch_bounds__(256) k_gemm_simt(const float *__restrict__ X, 
   }
 }
 
-static int g_gemm_impl = 0;  // 0 auto, 1 simt, 2 tcgen05
+static int g_gemm_impl = 0;  // 0 auto, 1 simt, 2 tcgen05, 3 tcgen05 with register-fed X tiles
+
+void gemm_tc_set_tma(int on);  // k_gemm_tc.cu
 
 int set_gemm_impl(int impl) {
   int old = g_gemm_impl;
   g_gemm_impl = impl;
+  gemm_tc_set_tma(impl != 3);
   return old;
 }
 
@@ -134,12 +137,12 @@ gnn_status launch_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw,
     cudaError_t e = launch_gemm_tc(X, ldx, W, ldw, H, ldh, m, k, n, row_scale, col_bias, relu, ws, ws_bytes, s);
     if (e == cudaSuccess) return GNN_OK;
     if (e != cudaErrorNotSupported) return cuda_status(e, "gemm tcgen05 launch");
-    if (g_gemm_impl == 2) {
+    if (g_gemm_impl >= 2) {
       set_error("tcgen05 GEMM does not support this shape/alignment/workspace");
       return GNN_ERR_UNSUPPORTED;
     }
     (void)cudaGetLastError();
-  } else if (g_gemm_impl == 2) {
+  } else if (g_gemm_impl >= 2) {
     set_error("tcgen05 GEMM needs a workspace (gnn_gemm_workspace_size)");
     return GNN_ERR_UNSUPPORTED;
   }

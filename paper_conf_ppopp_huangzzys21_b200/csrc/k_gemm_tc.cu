@@ -6,13 +6,18 @@
 //     H = Xlo Whi + Xhi Wlo + Xhi Whi      (Xlo Wlo ~ 2^-22 relative: dropped)
 // Epilogue fused: row scale (GCN nsrc[u]), column bias, ReLU.
 //
-// Structure (persistent, one CTA per SM, 288 threads):
-//   warps 0-3  producers: per 32-wide K block, load the 128 x 32 X tile from
-//              global memory, split it into hi/lo and store both in the UMMA
-//              K-major SWIZZLE_128B layout; thread 0 also issues one bulk
-//              async copy (cp.async.bulk, the TMA engine) of the pre-split,
-//              pre-swizzled W image for that K block (built once per call by
-//              k_gemm_wimage into the caller's workspace).
+// Structure (persistent, one CTA per SM, 320 threads):
+//   warps 0-3  producers: per 32-wide K block, the 128 x 32 X tile is split
+//              into hi/lo in the UMMA K-major SWIZZLE_128B layout.  TMA path
+//              (default when X rows are 16-byte aligned): warp 9 streams the
+//              raw tile into the hi slot with one cp.async.bulk.tensor (the
+//              tensor map's SWIZZLE_128B is the UMMA layout; out-of-range K
+//              and M are zero-filled), and the producers split it in shared
+//              memory (elementwise: hi in place, lo alongside).  Register path
+//              (unaligned X): the producers load the tile from global memory.
+//              The pre-split, pre-swizzled W image of the K block (built once
+//              per call by k_gemm_wimage into the caller's workspace) arrives
+//              by one bulk async copy on the same stage barrier.
 //   warp 4     MMA issuer: one elected lane issues 3 tcgen05.mma per 8-wide K
 //              step per 256-column slice, commits stage release / tile done.
 //   warps 5-8  epilogue: tcgen05.ld (32x32b: one TMEM lane = one row per
@@ -23,8 +28,10 @@
 // round-to-nearest, so long K chains drift; K blocks are spread round-robin
 // over n_acc partial accumulators (summed in fp32 in the epilogue) so that no
 // accumulator sees more than ~8 K blocks (<= 96 MMA accumulations).
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <string.h>
 
 #include "gnn_internal.h"
 
@@ -36,7 +43,8 @@ constexpr int BK = 32;  // fp32 elements per 128-byte swizzle row
 constexpr int NUM_PRODUCER_WARPS = 4;
 constexpr int MMA_WARP = 4;
 constexpr int EPI_WARP0 = 5;
-constexpr int THREADS = 32 * 9;
+constexpr int TMA_WARP = 9;
+constexpr int THREADS = 32 * 10;
 constexpr int TILE_A_BYTES = BM * BK * 4;  // 16 KB per hi or lo
 constexpr int MAX_STAGES = 6;
 
@@ -68,6 +76,16 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t by
                    smem_u32(dst)),
                "l"(src), "r"(bytes), "r"(smem_u32(bar))
                : "memory");
+}
+
+// 2D tiled TMA load (coordinates: inner = K element, outer = row)
+__device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, int32_t c0, int32_t c1,
+                                            uint64_t *bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::
+          "r"(smem_u32(dst)),
+      "l"(map), "r"(c0), "r"(c1), "r"(smem_u32(bar))
+      : "memory");
 }
 
 // UMMA shared-memory descriptor: K-major, SWIZZLE_128B, 8-row atoms of 1024 B
@@ -145,14 +163,14 @@ struct TcParams {
   int32_t relu;
 };
 
-template <bool VEC_X, bool VEC_H>
-__global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p) {
+template <bool VEC_X, bool VEC_H, bool TMA_X>
+__global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const __grid_constant__ CUtensorMap xmap) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   const int NP = p.np;
   const int B_BYTES = NP * 128;
   const int STAGE_BYTES = 2 * TILE_A_BYTES + 2 * B_BYTES;
-  __shared__ uint64_t full_bar[MAX_STAGES], empty_bar[MAX_STAGES], tfull_bar[2], tempty_bar[2];
+  __shared__ uint64_t full_bar[MAX_STAGES], empty_bar[MAX_STAGES], xfull_bar[MAX_STAGES], tfull_bar[2], tempty_bar[2];
   __shared__ uint32_t tmem_base_sh;
 
   const int tid = threadIdx.x;
@@ -162,8 +180,10 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p) {
 
   if (tid == 0) {
     for (int s = 0; s < S; ++s) {
-      mbar_init(&full_bar[s], NUM_PRODUCER_WARPS * 32 / 2 + 1);  // 64 A arrivals (one group) + 1 expect_tx
+      // register path: 64 A arrivals (one group) + 1 expect_tx; TMA path: 128 splitters + 1 expect_tx
+      mbar_init(&full_bar[s], (TMA_X ? NUM_PRODUCER_WARPS * 32 : NUM_PRODUCER_WARPS * 32 / 2) + 1);
       mbar_init(&empty_bar[s], 1);
+      mbar_init(&xfull_bar[s], 1);
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(&tfull_bar[b], 1);
@@ -180,7 +200,53 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p) {
   asm volatile("tcgen05.fence::after_thread_sync;");
   const uint32_t tmem = tmem_base_sh;
 
-  if (warp < NUM_PRODUCER_WARPS) {
+  const int my_tiles = p.num_tiles > (int)blockIdx.x ? (p.num_tiles - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0;
+  const int total_it = my_tiles * p.num_kb;
+  auto tile_of = [&](int it) { return (int)blockIdx.x + (it / p.num_kb) * (int)gridDim.x; };
+  if (TMA_X && warp == TMA_WARP) {
+    // --------------------------- TMA issuer (X + W) ---------------------------
+    if (lane == 0) {
+      for (int it = 0; it < total_it; ++it) {
+        const int kb = it % p.num_kb;
+        const int s = it % S, use = it / S;
+        if (use > 0) mbar_wait(&empty_bar[s], (use - 1) & 1);
+        uint8_t *st = smem + (size_t)s * STAGE_BYTES;
+        mbar_arrive_expect_tx(&xfull_bar[s], TILE_A_BYTES);
+        tma_load_2d(st, &xmap, kb * BK, tile_of(it) * BM, &xfull_bar[s]);
+        mbar_arrive_expect_tx(&full_bar[s], 2 * B_BYTES);
+        const uint8_t *src = p.wimg + (size_t)kb * 2 * B_BYTES;
+        uint8_t *b_img = st + 2 * TILE_A_BYTES;
+        for (int off = 0; off < 2 * B_BYTES; off += 16384) {
+          const int bytes = 2 * B_BYTES - off < 16384 ? 2 * B_BYTES - off : 16384;
+          bulk_g2s(b_img + off, src + off, bytes, &full_bar[s]);
+        }
+      }
+    }
+  } else if (TMA_X && warp < NUM_PRODUCER_WARPS) {
+    // -------------------- splitters: raw X tile -> hi / lo --------------------
+    // The split is elementwise and hi/lo share the swizzled layout, so each
+    // thread converts fixed 16-byte chunks with no address arithmetic.
+    constexpr int NT = NUM_PRODUCER_WARPS * 32;
+    constexpr int PER = TILE_A_BYTES / 16 / NT;  // 8 chunks per thread
+    for (int it = 0; it < total_it; ++it) {
+      const int s = it % S, use = it / S;
+      mbar_wait(&xfull_bar[s], use & 1);
+      uint8_t *st = smem + (size_t)s * STAGE_BYTES;
+      float4 *a_hi = reinterpret_cast<float4 *>(st);
+      float4 *a_lo = reinterpret_cast<float4 *>(st + TILE_A_BYTES);
+      float4 x[PER];
+#pragma unroll
+      for (int i = 0; i < PER; ++i) x[i] = a_hi[tid + i * NT];
+#pragma unroll
+      for (int i = 0; i < PER; ++i) {
+        const float4 hi = make_float4(hi_of(x[i].x), hi_of(x[i].y), hi_of(x[i].z), hi_of(x[i].w));
+        a_hi[tid + i * NT] = hi;
+        a_lo[tid + i * NT] = make_float4(x[i].x - hi.x, x[i].y - hi.y, x[i].z - hi.z, x[i].w - hi.w);
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      mbar_arrive(&full_bar[s]);
+    }
+  } else if (!TMA_X && warp < NUM_PRODUCER_WARPS) {
     // ------------------------------ producers ------------------------------
     // Two producer groups of 2 warps take alternate K blocks (group g handles
     // the global K-block counter it = g, g+2, ...); each group loads its next
@@ -214,9 +280,6 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p) {
         buf[i] = x;
       }
     };
-    const int my_tiles = p.num_tiles > (int)blockIdx.x ? (p.num_tiles - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0;
-    const int total_it = my_tiles * p.num_kb;
-    auto tile_of = [&](int it) { return (int)blockIdx.x + (it / p.num_kb) * (int)gridDim.x; };
     int it = grp;
     if (it < total_it) load_a((int64_t)tile_of(it) * BM, it % p.num_kb);
     while (it < total_it) {
@@ -287,7 +350,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p) {
         __syncwarp();
       }
     }
-  } else {
+  } else if (warp >= EPI_WARP0 && warp < EPI_WARP0 + 4) {
     // ------------------------------ epilogue ------------------------------
     const int ew = warp - EPI_WARP0;  // 0..3 -> TMEM lanes 32*ew (warp % 4 == ew + 1 ... see note)
     // TMEM lane quadrant accessible by a warp is (warp id % 4): warps 5,6,7,8 -> 1,2,3,0
@@ -390,6 +453,42 @@ static bool configure(int64_t m, int32_t k, int32_t n, Config &c) {
 
 }  // namespace tc
 
+namespace tc {
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no -lcuda)
+typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                  const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+static EncodeTiledFn encode_fn() {
+  static EncodeTiledFn fn = nullptr;
+  static bool tried = false;
+  if (!tried) {
+    tried = true;
+    void *f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = (EncodeTiledFn)f;
+  }
+  return fn;
+}
+static int g_tma_mode = 1;  // 1 = TMA-fed X tiles when the layout allows, 0 = register path
+static bool tma_enabled() { return g_tma_mode != 0 && encode_fn() != nullptr; }
+// X [m, k] row stride ldx (elements): box 32 (K) x 128 (rows), SWIZZLE_128B
+// (= the UMMA K-major layout), out-of-range elements zero-filled
+static bool encode_x_map(CUtensorMap *map, const float *X, int64_t ldx, int64_t m, int32_t k) {
+  if (((uintptr_t)X & 15) || ((ldx * 4) & 15)) return false;
+  const cuuint64_t dims[2] = {(cuuint64_t)k, (cuuint64_t)m};
+  const cuuint64_t strides[1] = {(cuuint64_t)ldx * 4};
+  const cuuint32_t box[2] = {(cuuint32_t)BK, (cuuint32_t)BM};
+  const cuuint32_t estr[2] = {1, 1};
+  return encode_fn()(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void *)X, dims, strides, box, estr,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+}  // namespace tc
+
+void gemm_tc_set_tma(int on) { tc::g_tma_mode = on ? 1 : 0; }
+
 size_t gemm_tc_workspace(int64_t m, int32_t k, int32_t n) {
   tc::Config c;
   if (!tc::configure(m > 0 ? m : 1, k, n, c)) return 0;
@@ -423,12 +522,17 @@ cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t 
              row_scale, col_bias, relu};
   const bool vx = (ldx % 4 == 0) && ((uintptr_t)X % 16 == 0);
   const bool vh = (ldh % 4 == 0) && ((uintptr_t)H % 16 == 0);
-  auto fn = vx ? (vh ? k_gemm_tc<true, true> : k_gemm_tc<true, false>)
-               : (vh ? k_gemm_tc<false, true> : k_gemm_tc<false, false>);
+  CUtensorMap xmap;
+  memset(&xmap, 0, sizeof(xmap));
+  // TMA needs 16-byte aligned rows (vx) and a 32-bit row coordinate
+  const bool tma = vx && tma_enabled() && m < 0x7fffff00LL && encode_x_map(&xmap, X, ldx, m, k);
+  auto fn = tma ? (vh ? k_gemm_tc<true, true, true> : k_gemm_tc<true, false, true>)
+                : vx ? (vh ? k_gemm_tc<true, true, false> : k_gemm_tc<true, false, false>)
+                     : (vh ? k_gemm_tc<false, true, false> : k_gemm_tc<false, false, false>);
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c.smem);
   if (e != cudaSuccess) return e;
   const int grid = (int)(num_tiles < num_sms ? num_tiles : num_sms);
-  fn<<<grid, THREADS, c.smem, s>>>(p);
+  fn<<<grid, THREADS, c.smem, s>>>(p, xmap);
   count_launch();
   return cudaGetLastError();
 }

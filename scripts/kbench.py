@@ -39,7 +39,7 @@ def gemm():
         W = (torch.rand(k, n, device="cuda") * 2 - 1) * float(np.sqrt(6 / (k + n)))
         rs = torch.rand(m, device="cuda") + 0.1
         res = {}
-        for impl, name in [(1, "simt"), (2, "tc")]:
+        for impl, name in [(1, "simt"), (2, "tc"), (3, "tc_reg")]:
             G.set_gemm_impl(impl)
             try:
                 H = G.gemm(X, W, row_scale=rs, simt=(impl == 1))

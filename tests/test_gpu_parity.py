@@ -392,6 +392,27 @@ def test_gemm_parity(m, k, n):
     assert_close(H(Hh), ref, what=f"gemm {m}x{k}x{n}")
 
 
+@pytest.mark.parametrize("m,k,n,ldx", [(300, 17, 5, 17), (4099, 602, 256, 604), (5000, 100, 256, 100),
+                                       (1000, 256, 272, 256), (129, 33, 16, 36)])
+def test_gemm_tma_matches_register_path(m, k, n, ldx):
+    """TMA-fed X tiles (impl 2) and register-fed X tiles (impl 3) build the
+    same hi/lo operands, so the tcgen05 results are bit-identical."""
+    Xp = gs.uniform(m, ldx, seed=5)
+    lim = np.sqrt(6 / (k + n))
+    W = gs.uniform(k, n, lo=-lim, hi=lim, seed=6)
+    X = T(Xp)[:, :k]
+    ref = oracle.gemm(Xp[:, :k], W, np.ones(m))
+    out = {}
+    try:
+        for impl in (2, 3):
+            G.set_gemm_impl(impl)
+            out[impl] = H(G.gemm(X, T(W)))
+    finally:
+        G.set_gemm_impl(0)
+    assert np.array_equal(out[2].view(np.uint32), out[3].view(np.uint32))
+    assert_close(out[2], ref, what=f"gemm tma {m}x{k}x{n} ld {ldx}")
+
+
 @pytest.mark.parametrize("order", [1, 2])
 def test_gcn_layer_parity(order):
     g = gs.config_graph("C1")
