@@ -43,8 +43,9 @@ constexpr int BK = 32;  // fp32 elements per 128-byte swizzle row
 constexpr int NUM_PRODUCER_WARPS = 4;
 constexpr int MMA_WARP = 4;
 constexpr int EPI_WARP0 = 5;
-constexpr int TMA_WARP = 9;
-constexpr int THREADS = 32 * 10;
+constexpr int TMA_WARP = 9;   // TMA path: X tiles
+constexpr int WIMG_WARP = 10; // TMA path: W image blocks
+constexpr int THREADS = 32 * 11;
 constexpr int TILE_A_BYTES = BM * BK * 4;  // 16 KB per hi or lo
 constexpr int MAX_STAGES = 6;
 
@@ -86,6 +87,18 @@ __device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, i
           "r"(smem_u32(dst)),
       "l"(map), "r"(c0), "r"(c1), "r"(smem_u32(bar))
       : "memory");
+}
+
+// 2D tiled TMA store (smem -> global, out-of-range rows/columns clipped)
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap *map, int32_t c0, int32_t c1, const void *src) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];" ::"l"(map), "r"(c0),
+               "r"(c1), "r"(smem_u32(src))
+               : "memory");
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() {
+  asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
 }
 
 // UMMA shared-memory descriptor: K-major, SWIZZLE_128B, 8-row atoms of 1024 B
@@ -158,19 +171,26 @@ struct TcParams {
   int32_t k, n, np, npa;  // np = n rounded to 16; npa = TMEM columns per accumulator
   int32_t num_kb, num_tiles;
   int32_t stages, n_acc, n_buf;
+  int32_t sa, sb;  // TMA path: A (X hi/lo) ring and B (W image) ring depths
+  int32_t eb;      // TMA path with TMA stores: 4 KB staging buffers per epilogue warp (1 or 2)
   const float *row_scale;
   const float *col_bias;
   int32_t relu;
 };
 
 template <bool VEC_X, bool VEC_H, bool TMA_X>
-__global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const __grid_constant__ CUtensorMap xmap) {
+__global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const __grid_constant__ CUtensorMap xmap,
+                                                          const __grid_constant__ CUtensorMap hmap) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   const int NP = p.np;
   const int B_BYTES = NP * 128;
   const int STAGE_BYTES = 2 * TILE_A_BYTES + 2 * B_BYTES;
-  __shared__ uint64_t full_bar[MAX_STAGES], empty_bar[MAX_STAGES], xfull_bar[MAX_STAGES], tfull_bar[2], tempty_bar[2];
+  // register path: full/empty per unified stage [A | B].  TMA path: separate
+  // rings -- A: xfull (TMA bytes) -> afull (splitters) -> aempty (MMA);
+  // B: full (bulk bytes) -> empty (MMA)
+  __shared__ uint64_t full_bar[MAX_STAGES], empty_bar[MAX_STAGES], xfull_bar[MAX_STAGES], afull_bar[MAX_STAGES],
+      aempty_bar[MAX_STAGES], tfull_bar[2], tempty_bar[2];
   __shared__ uint32_t tmem_base_sh;
 
   const int tid = threadIdx.x;
@@ -179,11 +199,21 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const 
   const int S = p.stages;
 
   if (tid == 0) {
-    for (int s = 0; s < S; ++s) {
-      // register path: 64 A arrivals (one group) + 1 expect_tx; TMA path: 128 splitters + 1 expect_tx
-      mbar_init(&full_bar[s], (TMA_X ? NUM_PRODUCER_WARPS * 32 : NUM_PRODUCER_WARPS * 32 / 2) + 1);
-      mbar_init(&empty_bar[s], 1);
-      mbar_init(&xfull_bar[s], 1);
+    if (TMA_X) {
+      for (int s = 0; s < p.sa; ++s) {
+        mbar_init(&xfull_bar[s], 1);
+        mbar_init(&afull_bar[s], NUM_PRODUCER_WARPS * 32);
+        mbar_init(&aempty_bar[s], 1);
+      }
+      for (int s = 0; s < p.sb; ++s) {
+        mbar_init(&full_bar[s], 1);
+        mbar_init(&empty_bar[s], 1);
+      }
+    } else {
+      for (int s = 0; s < S; ++s) {
+        mbar_init(&full_bar[s], NUM_PRODUCER_WARPS * 32 / 2 + 1);  // 64 A arrivals (one group) + 1 expect_tx
+        mbar_init(&empty_bar[s], 1);
+      }
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(&tfull_bar[b], 1);
@@ -203,19 +233,27 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const 
   const int my_tiles = p.num_tiles > (int)blockIdx.x ? (p.num_tiles - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0;
   const int total_it = my_tiles * p.num_kb;
   auto tile_of = [&](int it) { return (int)blockIdx.x + (it / p.num_kb) * (int)gridDim.x; };
+  uint8_t *const b_ring = smem + (size_t)p.sa * 2 * TILE_A_BYTES;  // TMA path
   if (TMA_X && warp == TMA_WARP) {
-    // --------------------------- TMA issuer (X + W) ---------------------------
+    // ----------------------------- TMA issuer (X) -----------------------------
     if (lane == 0) {
       for (int it = 0; it < total_it; ++it) {
-        const int kb = it % p.num_kb;
-        const int s = it % S, use = it / S;
-        if (use > 0) mbar_wait(&empty_bar[s], (use - 1) & 1);
-        uint8_t *st = smem + (size_t)s * STAGE_BYTES;
+        const int s = it % p.sa, use = it / p.sa;
+        if (use > 0) mbar_wait(&aempty_bar[s], (use - 1) & 1);
         mbar_arrive_expect_tx(&xfull_bar[s], TILE_A_BYTES);
-        tma_load_2d(st, &xmap, kb * BK, tile_of(it) * BM, &xfull_bar[s]);
+        tma_load_2d(smem + (size_t)s * 2 * TILE_A_BYTES, &xmap, (it % p.num_kb) * BK, tile_of(it) * BM,
+                    &xfull_bar[s]);
+      }
+    }
+  } else if (TMA_X && warp == WIMG_WARP) {
+    // ------------------------ bulk-copy issuer (W image) ------------------------
+    if (lane == 0) {
+      for (int it = 0; it < total_it; ++it) {
+        const int s = it % p.sb, use = it / p.sb;
+        if (use > 0) mbar_wait(&empty_bar[s], (use - 1) & 1);
         mbar_arrive_expect_tx(&full_bar[s], 2 * B_BYTES);
-        const uint8_t *src = p.wimg + (size_t)kb * 2 * B_BYTES;
-        uint8_t *b_img = st + 2 * TILE_A_BYTES;
+        const uint8_t *src = p.wimg + (size_t)(it % p.num_kb) * 2 * B_BYTES;
+        uint8_t *b_img = b_ring + (size_t)s * 2 * B_BYTES;
         for (int off = 0; off < 2 * B_BYTES; off += 16384) {
           const int bytes = 2 * B_BYTES - off < 16384 ? 2 * B_BYTES - off : 16384;
           bulk_g2s(b_img + off, src + off, bytes, &full_bar[s]);
@@ -229,9 +267,9 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const 
     constexpr int NT = NUM_PRODUCER_WARPS * 32;
     constexpr int PER = TILE_A_BYTES / 16 / NT;  // 8 chunks per thread
     for (int it = 0; it < total_it; ++it) {
-      const int s = it % S, use = it / S;
+      const int s = it % p.sa, use = it / p.sa;
       mbar_wait(&xfull_bar[s], use & 1);
-      uint8_t *st = smem + (size_t)s * STAGE_BYTES;
+      uint8_t *st = smem + (size_t)s * 2 * TILE_A_BYTES;
       float4 *a_hi = reinterpret_cast<float4 *>(st);
       float4 *a_lo = reinterpret_cast<float4 *>(st + TILE_A_BYTES);
       float4 x[PER];
@@ -244,7 +282,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const 
         a_lo[tid + i * NT] = make_float4(x[i].x - hi.x, x[i].y - hi.y, x[i].z - hi.z, x[i].w - hi.w);
       }
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-      mbar_arrive(&full_bar[s]);
+      mbar_arrive(&afull_bar[s]);
     }
   } else if (!TMA_X && warp < NUM_PRODUCER_WARPS) {
     // ------------------------------ producers ------------------------------
@@ -322,12 +360,24 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const 
       asm volatile("tcgen05.fence::after_thread_sync;");
       const uint32_t tbase = tmem + (uint32_t)(b * p.n_acc * p.npa);
       for (int kb = 0; kb < p.num_kb; ++kb, ++it) {
-        const int s = it % S, use = it / S;
-        mbar_wait(&full_bar[s], use & 1);
+        int s, sA;
+        uint32_t a_hi, b_hi;
+        if (TMA_X) {
+          sA = it % p.sa;
+          s = it % p.sb;
+          mbar_wait(&afull_bar[sA], (it / p.sa) & 1);
+          mbar_wait(&full_bar[s], (it / p.sb) & 1);
+          a_hi = smem_u32(smem + (size_t)sA * 2 * TILE_A_BYTES);
+          b_hi = smem_u32(b_ring + (size_t)s * 2 * B_BYTES);
+        } else {
+          s = sA = it % S;
+          mbar_wait(&full_bar[s], (it / S) & 1);
+          a_hi = smem_u32(smem + (size_t)s * STAGE_BYTES);
+          b_hi = a_hi + 2 * TILE_A_BYTES;
+        }
         asm volatile("tcgen05.fence::after_thread_sync;");
         if (lane == 0) {
-          const uint32_t st = smem_u32(smem + (size_t)s * STAGE_BYTES);
-          const uint32_t a_hi = st, a_lo = st + TILE_A_BYTES, b_hi = st + 2 * TILE_A_BYTES, b_lo = b_hi + B_BYTES;
+          const uint32_t a_lo = a_hi + TILE_A_BYTES, b_lo = b_hi + B_BYTES;
           const int acc = kb % p.n_acc;
           const uint32_t d0 = tbase + (uint32_t)(acc * p.npa);
           const uint32_t first = (kb < p.n_acc) ? 1u : 0u;  // first K block of this accumulator
@@ -345,6 +395,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const 
             }
           }
           mma_commit(&empty_bar[s]);
+          if (TMA_X) mma_commit(&aempty_bar[sA]);
           if (kb == p.num_kb - 1) mma_commit(&tfull_bar[b]);
         }
         __syncwarp();
@@ -356,6 +407,13 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const 
     // TMEM lane quadrant accessible by a warp is (warp id % 4): warps 5,6,7,8 -> 1,2,3,0
     const int quad = warp & 3;
     (void)ew;
+    // TMA path (VEC_H): each warp stages its 32 rows x 32 columns in a
+    // SWIZZLE_128B buffer (row = lane, conflict-free float4 writes) and one
+    // lane stores it with a TMA bulk tensor store (coalesced; tails clipped)
+    constexpr bool TMA_H = TMA_X && VEC_H;
+    uint8_t *const epi_buf = smem + (size_t)p.sa * 2 * TILE_A_BYTES + (size_t)p.sb * 2 * B_BYTES +
+                             (size_t)(warp - EPI_WARP0) * p.eb * 4096;
+    int chunk = 0;
     int tcount = 0;
     for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++tcount) {
       const int b = tcount % p.n_buf, buse = tcount / p.n_buf;
@@ -386,7 +444,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const 
 #pragma unroll
           for (int i = 0; i < 32; ++i) y[i] = (a == 0) ? __uint_as_float(v[i]) : y[i] + __uint_as_float(v[i]);
         }
-        if (gm >= p.m) continue;
+        if (!TMA_H && gm >= p.m) continue;
 #pragma unroll
         for (int i = 0; i < 32; ++i) {
           const int col = c0 + i;
@@ -395,6 +453,25 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const 
           if (p.col_bias && col < p.n) t = t + __ldg(p.col_bias + col);
           if (p.relu) t = t > 0.0f ? t : 0.0f;
           y[i] = t;
+        }
+        if constexpr (TMA_H) {
+          uint8_t *buf = epi_buf + (chunk % p.eb) * 4096;
+          if (chunk >= p.eb) {
+            if (lane == 0) {
+              if (p.eb == 2) bulk_wait_read<1>();
+              else bulk_wait_read<0>();
+            }
+            __syncwarp();
+          }
+#pragma unroll
+          for (int c = 0; c < 8; ++c)
+            *reinterpret_cast<float4 *>(buf + lane * 128 + ((c ^ (lane & 7)) << 4)) =
+                make_float4(y[4 * c], y[4 * c + 1], y[4 * c + 2], y[4 * c + 3]);
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+          __syncwarp();
+          if (lane == 0) tma_store_2d(&hmap, c0, (int32_t)(tile * BM + quad * 32), buf);
+          ++chunk;
+          continue;
         }
         float *dst = p.H + gm * p.ldh + c0;
         if (VEC_H && c0 + 32 <= p.n) {
@@ -409,6 +486,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const 
       asm volatile("tcgen05.fence::before_thread_sync;");
       mbar_arrive(&tempty_bar[b]);
     }
+    if (TMA_H && lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
   }
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
@@ -420,7 +498,8 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const 
 
 struct Config {
   int np, npa, num_kb, stages, n_acc, n_buf;
-  size_t smem, wimg_bytes;
+  int sa, sb, eb;
+  size_t smem, smem_tma, wimg_bytes;
 };
 
 static bool configure(int64_t m, int32_t k, int32_t n, Config &c) {
@@ -435,6 +514,21 @@ static bool configure(int64_t m, int32_t k, int32_t n, Config &c) {
   while (c.stages > 2 && (size_t)c.stages * stage_bytes + 2048 > 200 * 1024) --c.stages;
   c.smem = (size_t)c.stages * stage_bytes + 1024;
   if (c.smem > 227 * 1024) return false;
+  // TMA path: separate rings; deepen the X ring first (HBM latency), then W
+  {
+    const size_t budget = 225 * 1024, a_bytes = 2 * TILE_A_BYTES, b_bytes = 2 * (size_t)c.np * 128;
+    c.sa = 2;
+    c.sb = 2;
+    c.eb = 2;  // epilogue staging: 4 warps x eb x 4 KB
+    auto need = [&](int sa, int sb, int eb) {
+      return (size_t)sa * a_bytes + (size_t)sb * b_bytes + (size_t)eb * 4 * 4096 + 1024;
+    };
+    if (need(2, 2, 2) > budget) c.eb = 1;
+    while (c.sa < MAX_STAGES && need(c.sa + 1, c.sb, c.eb) <= budget) ++c.sa;
+    while (c.sb < MAX_STAGES && need(c.sa, c.sb + 1, c.eb) <= budget) ++c.sb;
+    c.smem_tma = need(c.sa, c.sb, c.eb);
+    if (c.smem_tma > budget) c.sa = 0;  // TMA path unavailable for this n
+  }
   // TMEM: n_buf tile buffers x n_acc accumulators x npa columns <= 512
   const int slots = 512 / c.npa;  // accumulators that fit
   if (slots < 1) return false;
@@ -485,6 +579,18 @@ static bool encode_x_map(CUtensorMap *map, const float *X, int64_t ldx, int64_t 
                      CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
+// H [m, n] row stride ldh: box 32 (columns) x 32 (rows), SWIZZLE_128B (the
+// epilogue's staging layout); stores outside [m, n] are clipped
+static bool encode_h_map(CUtensorMap *map, float *H, int64_t ldh, int64_t m, int32_t n) {
+  if (((uintptr_t)H & 15) || ((ldh * 4) & 15)) return false;
+  const cuuint64_t dims[2] = {(cuuint64_t)n, (cuuint64_t)m};
+  const cuuint64_t strides[1] = {(cuuint64_t)ldh * 4};
+  const cuuint32_t box[2] = {32, 32};
+  const cuuint32_t estr[2] = {1, 1};
+  return encode_fn()(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void *)H, dims, strides, box, estr,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
 }  // namespace tc
 
 void gemm_tc_set_tma(int on) { tc::g_tma_mode = on ? 1 : 0; }
@@ -519,20 +625,24 @@ cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t 
   const int64_t num_tiles = (m + BM - 1) / BM;
   if (num_tiles > 0x7fffffff) return cudaErrorNotSupported;
   TcParams p{X, ldx, H, ldh, img, m, k, n, c.np, c.npa, c.num_kb, (int32_t)num_tiles, c.stages, c.n_acc, c.n_buf,
-             row_scale, col_bias, relu};
+             c.sa, c.sb, c.eb, row_scale, col_bias, relu};
   const bool vx = (ldx % 4 == 0) && ((uintptr_t)X % 16 == 0);
   const bool vh = (ldh % 4 == 0) && ((uintptr_t)H % 16 == 0);
   CUtensorMap xmap;
   memset(&xmap, 0, sizeof(xmap));
   // TMA needs 16-byte aligned rows (vx) and a 32-bit row coordinate
-  const bool tma = vx && tma_enabled() && m < 0x7fffff00LL && encode_x_map(&xmap, X, ldx, m, k);
+  CUtensorMap hmap;
+  memset(&hmap, 0, sizeof(hmap));
+  const bool tma = vx && c.sa > 0 && tma_enabled() && m < 0x7fffff00LL && encode_x_map(&xmap, X, ldx, m, k) &&
+                   (!vh || encode_h_map(&hmap, H, ldh, m, n));
   auto fn = tma ? (vh ? k_gemm_tc<true, true, true> : k_gemm_tc<true, false, true>)
                 : vx ? (vh ? k_gemm_tc<true, true, false> : k_gemm_tc<true, false, false>)
                      : (vh ? k_gemm_tc<false, true, false> : k_gemm_tc<false, false, false>);
-  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c.smem);
+  const size_t smem = tma ? c.smem_tma : c.smem;
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   const int grid = (int)(num_tiles < num_sms ? num_tiles : num_sms);
-  fn<<<grid, THREADS, c.smem, s>>>(p, xmap);
+  fn<<<grid, THREADS, smem, s>>>(p, xmap, hmap);
   count_launch();
   return cudaGetLastError();
 }
