@@ -6,23 +6,26 @@
 //     H = Xlo Whi + Xhi Wlo + Xhi Whi      (Xlo Wlo ~ 2^-22 relative: dropped)
 // Epilogue fused: row scale (GCN nsrc[u]), column bias, ReLU.
 //
-// Structure (persistent, one CTA per SM, 320 threads):
+// Structure (persistent, one CTA per SM, 352 threads):
 //   warps 0-3  producers: per 32-wide K block, the 128 x 32 X tile is split
 //              into hi/lo in the UMMA K-major SWIZZLE_128B layout.  TMA path
-//              (default when X rows are 16-byte aligned): warp 9 streams the
-//              raw tile into the hi slot with one cp.async.bulk.tensor (the
-//              tensor map's SWIZZLE_128B is the UMMA layout; out-of-range K
-//              and M are zero-filled), and the producers split it in shared
-//              memory (elementwise: hi in place, lo alongside).  Register path
-//              (unaligned X): the producers load the tile from global memory.
-//              The pre-split, pre-swizzled W image of the K block (built once
-//              per call by k_gemm_wimage into the caller's workspace) arrives
-//              by one bulk async copy on the same stage barrier.
+//              (default when X/H rows are 16-byte aligned): warp 9 streams
+//              the raw tile into the hi slot with one cp.async.bulk.tensor
+//              (the tensor map's SWIZZLE_128B is the UMMA layout; out-of-range
+//              K and M are zero-filled), and the producers split it in shared
+//              memory (elementwise: hi in place, lo alongside); warp 10 bulk-
+//              copies the pre-split, pre-swizzled W image of the K block
+//              (built once per call by k_gemm_wimage into the caller's
+//              workspace) into its own ring.  Register path (unaligned X, or
+//              gnn_set_gemm_impl(3)): the producers load the tile from global
+//              memory and one of them issues the W copy; one unified ring.
 //   warp 4     MMA issuer: one elected lane issues 3 tcgen05.mma per 8-wide K
 //              step per 256-column slice, commits stage release / tile done.
 //   warps 5-8  epilogue: tcgen05.ld (32x32b: one TMEM lane = one row per
 //              thread), fp32 sum of the partial accumulators, scale/bias/ReLU,
-//              store.  Runs concurrently with the next tile's MMAs when TMEM
+//              then (TMA path) a swizzled 32x32 staging buffer per warp and a
+//              TMA bulk tensor store, or (register path) row-per-thread
+//              stores.  Runs concurrently with the next tile's MMAs when TMEM
 //              holds two tile buffers.
 // Accumulation drift: the tensor core's internal accumulation is not IEEE
 // round-to-nearest, so long K chains drift; K blocks are spread round-robin
