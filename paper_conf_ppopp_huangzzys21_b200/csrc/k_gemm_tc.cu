@@ -34,6 +34,7 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include "gnn_internal.h"
@@ -48,7 +49,10 @@ constexpr int MMA_WARP = 4;
 constexpr int EPI_WARP0 = 5;
 constexpr int TMA_WARP = 9;   // TMA path: X tiles
 constexpr int WIMG_WARP = 10; // TMA path: W image blocks
-constexpr int THREADS = 32 * 11;
+constexpr int THREADS = 32 * 11;      // register path
+constexpr int EPI_WARP1 = 11;         // TMA path: second epilogue half (warps 11-14)
+constexpr int THREADS_TMA = 32 * 15;
+__host__ __device__ constexpr int threads_of(bool tma) { return tma ? THREADS_TMA : THREADS; }
 constexpr int TILE_A_BYTES = BM * BK * 4;  // 16 KB per hi or lo
 constexpr int MAX_STAGES = 6;
 
@@ -176,13 +180,14 @@ struct TcParams {
   int32_t stages, n_acc, n_buf;
   int32_t sa, sb;  // TMA path: A (X hi/lo) ring and B (W image) ring depths
   int32_t eb;      // TMA path with TMA stores: 4 KB staging buffers per epilogue warp (1 or 2)
+  int32_t epi8;    // TMA stores with 8 epilogue warps (two per TMEM lane quadrant, alternate column chunks)
   const float *row_scale;
   const float *col_bias;
   int32_t relu;
 };
 
 template <bool VEC_X, bool VEC_H, bool TMA_X>
-__global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const __grid_constant__ CUtensorMap xmap,
+__global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams p, const __grid_constant__ CUtensorMap xmap,
                                                           const __grid_constant__ CUtensorMap hmap) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -220,7 +225,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const 
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(&tfull_bar[b], 1);
-      mbar_init(&tempty_bar[b], 128);
+      mbar_init(&tempty_bar[b], 128 * (p.epi8 ? 2 : 1));
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -404,7 +409,8 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const 
         __syncwarp();
       }
     }
-  } else if (warp >= EPI_WARP0 && warp < EPI_WARP0 + 4) {
+  } else if ((warp >= EPI_WARP0 && warp < EPI_WARP0 + 4) ||
+             (TMA_X && VEC_H && p.epi8 && warp >= EPI_WARP1 && warp < EPI_WARP1 + 4)) {
     // ------------------------------ epilogue ------------------------------
     const int ew = warp - EPI_WARP0;  // 0..3 -> TMEM lanes 32*ew (warp % 4 == ew + 1 ... see note)
     // TMEM lane quadrant accessible by a warp is (warp id % 4): warps 5,6,7,8 -> 1,2,3,0
@@ -414,8 +420,11 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const 
     // SWIZZLE_128B buffer (row = lane, conflict-free float4 writes) and one
     // lane stores it with a TMA bulk tensor store (coalesced; tails clipped)
     constexpr bool TMA_H = TMA_X && VEC_H;
+    const int half = warp >= EPI_WARP1 ? 1 : 0;  // column chunks half, half + nhalf, ...
+    const int nhalf = p.epi8 ? 2 : 1;
+    const int widx = half ? 4 + warp - EPI_WARP1 : warp - EPI_WARP0;
     uint8_t *const epi_buf = smem + (size_t)p.sa * 2 * TILE_A_BYTES + (size_t)p.sb * 2 * B_BYTES +
-                             (size_t)(warp - EPI_WARP0) * p.eb * 4096;
+                             (size_t)widx * p.eb * 4096;
     int chunk = 0;
     int tcount = 0;
     for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++tcount) {
@@ -427,7 +436,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const 
       const float sc = (p.row_scale && gm < p.m) ? __ldg(p.row_scale + gm) : 1.0f;
       const uint32_t tbase = tmem + (uint32_t)(b * p.n_acc * p.npa) + ((uint32_t)(quad * 32) << 16);
       const int n_acc_used = p.num_kb < p.n_acc ? p.num_kb : p.n_acc;
-      for (int c0 = 0; c0 < NP; c0 += 32) {
+      for (int c0 = half * 32; c0 < NP; c0 += 32 * nhalf) {
         float y[32];
 #pragma unroll
         for (int i = 0; i < 32; ++i) y[i] = 0.0f;
@@ -501,10 +510,11 @@ __global__ void __launch_bounds__(THREADS, 1) k_gemm_tc(const TcParams p, const 
 
 struct Config {
   int np, npa, num_kb, stages, n_acc, n_buf;
-  int sa, sb, eb;
+  int sa, sb, eb, epi8;
   size_t smem, smem_tma, wimg_bytes;
 };
 
+static int g_epi8 = -1;  // 8 epilogue warps on the TMA path (A/B switch: env GNN_GEMM_EPI8=0 disables)
 static bool configure(int64_t m, int32_t k, int32_t n, Config &c) {
   if (n < 1 || n > 512 || k < 1 || m < 1) return false;
   c.np = (n + 15) / 16 * 16;
@@ -522,14 +532,24 @@ static bool configure(int64_t m, int32_t k, int32_t n, Config &c) {
     const size_t budget = 225 * 1024, a_bytes = 2 * TILE_A_BYTES, b_bytes = 2 * (size_t)c.np * 128;
     c.sa = 2;
     c.sb = 2;
-    c.eb = 2;  // epilogue staging: 4 warps x eb x 4 KB
-    auto need = [&](int sa, int sb, int eb) {
-      return (size_t)sa * a_bytes + (size_t)sb * b_bytes + (size_t)eb * 4 * 4096 + 1024;
+    // epilogue staging: (epi8 ? 8 : 4) warps x eb x 4 KB; prefer 8 warps
+    auto need = [&](int sa, int sb, int eb, int e8) {
+      return (size_t)sa * a_bytes + (size_t)sb * b_bytes + (size_t)eb * (e8 ? 8 : 4) * 4096 + 1024;
     };
-    if (need(2, 2, 2) > budget) c.eb = 1;
-    while (c.sa < MAX_STAGES && need(c.sa + 1, c.sb, c.eb) <= budget) ++c.sa;
-    while (c.sb < MAX_STAGES && need(c.sa, c.sb + 1, c.eb) <= budget) ++c.sb;
-    c.smem_tma = need(c.sa, c.sb, c.eb);
+    if (g_epi8 < 0) {
+      const char *e = getenv("GNN_GEMM_EPI8");
+      g_epi8 = (e && e[0] == '0') ? 0 : 1;
+    }
+    c.epi8 = g_epi8 ? 1 : 0;
+    c.eb = 2;
+    if (need(2, 2, c.eb, c.epi8) > budget) c.eb = 1;
+    if (c.epi8 && need(2, 2, c.eb, 1) > budget) {
+      c.epi8 = 0;
+      c.eb = need(2, 2, 2, 0) > budget ? 1 : 2;
+    }
+    while (c.sa < MAX_STAGES && need(c.sa + 1, c.sb, c.eb, c.epi8) <= budget) ++c.sa;
+    while (c.sb < MAX_STAGES && need(c.sa, c.sb + 1, c.eb, c.epi8) <= budget) ++c.sb;
+    c.smem_tma = need(c.sa, c.sb, c.eb, c.epi8);
     if (c.smem_tma > budget) c.sa = 0;  // TMA path unavailable for this n
   }
   // TMEM: n_buf tile buffers x n_acc accumulators x npa columns <= 512
@@ -628,7 +648,7 @@ cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t 
   const int64_t num_tiles = (m + BM - 1) / BM;
   if (num_tiles > 0x7fffffff) return cudaErrorNotSupported;
   TcParams p{X, ldx, H, ldh, img, m, k, n, c.np, c.npa, c.num_kb, (int32_t)num_tiles, c.stages, c.n_acc, c.n_buf,
-             c.sa, c.sb, c.eb, row_scale, col_bias, relu};
+             c.sa, c.sb, c.eb, c.epi8, row_scale, col_bias, relu};
   const bool vx = (ldx % 4 == 0) && ((uintptr_t)X % 16 == 0);
   const bool vh = (ldh % 4 == 0) && ((uintptr_t)H % 16 == 0);
   CUtensorMap xmap;
@@ -645,7 +665,8 @@ cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t 
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   const int grid = (int)(num_tiles < num_sms ? num_tiles : num_sms);
-  fn<<<grid, THREADS, smem, s>>>(p, xmap, hmap);
+  if (!(tma && vh)) p.epi8 = 0;
+  fn<<<grid, threads_of(tma), smem, s>>>(p, xmap, hmap);
   count_launch();
   return cudaGetLastError();
 }
