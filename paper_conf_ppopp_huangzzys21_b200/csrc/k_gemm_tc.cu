@@ -624,43 +624,9 @@ size_t gemm_tc_workspace(int64_t m, int32_t k, int32_t n) {
   return (c.wimg_bytes + 255) & ~(size_t)255;
 }
 
-static cudaError_t launch_gemm_tc_one(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H,
-                                      int64_t ldh, int64_t m, int32_t k, int32_t n, const float *row_scale,
-                                      const float *col_bias, int32_t relu, void *ws, size_t ws_bytes,
-                                      cudaStream_t s);
-
-// Column split: an output wider than 256 columns cannot double-buffer its
-// accumulator in TMEM (2 x 512 columns), so the epilogue would serialise with
-// the MMAs.  It runs as two launches instead -- columns [0, 256) with the
-// TMEM double buffer, then the rest -- each writing its column range of H in
-// place; the W images sit back to back in the same workspace (same total
-// size).  Costs one extra read of X.  A/B: env GNN_GEMM_SPLIT=0 disables.
 cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H, int64_t ldh,
                            int64_t m, int32_t k, int32_t n, const float *row_scale, const float *col_bias,
                            int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s) {
-  static int split = -1;
-  if (split < 0) {
-    const char *e = getenv("GNN_GEMM_SPLIT");
-    split = (e && e[0] == '0') ? 0 : 1;
-  }
-  tc::Config c, c0;
-  if (split && n > 256 && m > 0 && tc::configure(m, k, n, c) && c.n_buf == 1 && tc::configure(m, k, 256, c0) &&
-      c0.n_buf == 2) {
-    if (!ws || ws_bytes < c.wimg_bytes) return cudaErrorNotSupported;
-    cudaError_t e = launch_gemm_tc_one(X, ldx, W, ldw, H, ldh, m, k, 256, row_scale, col_bias, relu, ws,
-                                       c0.wimg_bytes, s);
-    if (e != cudaSuccess) return e;
-    return launch_gemm_tc_one(X, ldx, W + 256, ldw, H + 256, ldh, m, k, n - 256, row_scale,
-                              col_bias ? col_bias + 256 : nullptr, relu, (uint8_t *)ws + c0.wimg_bytes,
-                              ws_bytes - c0.wimg_bytes, s);
-  }
-  return launch_gemm_tc_one(X, ldx, W, ldw, H, ldh, m, k, n, row_scale, col_bias, relu, ws, ws_bytes, s);
-}
-
-static cudaError_t launch_gemm_tc_one(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H,
-                                      int64_t ldh, int64_t m, int32_t k, int32_t n, const float *row_scale,
-                                      const float *col_bias, int32_t relu, void *ws, size_t ws_bytes,
-                                      cudaStream_t s) {
   using namespace tc;
   Config c;
   if (!configure(m, k, n, c)) return cudaErrorNotSupported;
