@@ -27,6 +27,9 @@
 //              TMA bulk tensor store, or (register path) row-per-thread
 //              stores.  Runs concurrently with the next tile's MMAs when TMEM
 //              holds two tile buffers.
+// Column blocks (TMA path, n > 256, <= 8 K blocks): each row tile is two
+// work items over column slices of the W image, so both accumulators fit
+// TMEM twice and the epilogue overlaps the next item's MMAs.
 // Accumulation drift: the tensor core's internal accumulation is not IEEE
 // round-to-nearest, so long K chains drift; K blocks are spread round-robin
 // over n_acc partial accumulators (summed in fp32 in the epilogue) so that no
@@ -180,6 +183,7 @@ struct TcParams {
   int32_t stages, n_acc, n_buf;
   int32_t sa, sb;  // TMA path: A (X hi/lo) ring and B (W image) ring depths
   int32_t eb;      // TMA path with TMA stores: 4 KB staging buffers per epilogue warp (1 or 2)
+  int32_t ncb, cbw0;  // TMA path: column blocks per row tile (1 or 2) and block 0's width
   int32_t epi8;    // TMA stores with 8 epilogue warps (two per TMEM lane quadrant, alternate column chunks)
   const float *row_scale;
   const float *col_bias;
@@ -241,6 +245,11 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
   const int my_tiles = p.num_tiles > (int)blockIdx.x ? (p.num_tiles - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0;
   const int total_it = my_tiles * p.num_kb;
   auto tile_of = [&](int it) { return (int)blockIdx.x + (it / p.num_kb) * (int)gridDim.x; };
+  // TMA path: work item vt = (row tile vt / ncb, column block vt % ncb); a
+  // column block is a slice of the W image (rows cb_beg .. cb_beg + cb_w)
+  auto cb_beg = [&](int vt) { return (p.ncb > 1 && vt % p.ncb) ? p.cbw0 : 0; };
+  auto cb_w = [&](int vt) { return p.ncb > 1 ? ((vt % p.ncb) ? NP - p.cbw0 : p.cbw0) : NP; };
+  const int B_STAGE = 2 * (p.ncb > 1 ? p.cbw0 : NP) * 128;  // TMA path B ring stage
   uint8_t *const b_ring = smem + (size_t)p.sa * 2 * TILE_A_BYTES;  // TMA path
   if (TMA_X && warp == TMA_WARP) {
     // ----------------------------- TMA issuer (X) -----------------------------
@@ -249,7 +258,7 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
         const int s = it % p.sa, use = it / p.sa;
         if (use > 0) mbar_wait(&aempty_bar[s], (use - 1) & 1);
         mbar_arrive_expect_tx(&xfull_bar[s], TILE_A_BYTES);
-        tma_load_2d(smem + (size_t)s * 2 * TILE_A_BYTES, &xmap, (it % p.num_kb) * BK, tile_of(it) * BM,
+        tma_load_2d(smem + (size_t)s * 2 * TILE_A_BYTES, &xmap, (it % p.num_kb) * BK, (tile_of(it) / p.ncb) * BM,
                     &xfull_bar[s]);
       }
     }
@@ -259,13 +268,16 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
       for (int it = 0; it < total_it; ++it) {
         const int s = it % p.sb, use = it / p.sb;
         if (use > 0) mbar_wait(&empty_bar[s], (use - 1) & 1);
-        mbar_arrive_expect_tx(&full_bar[s], 2 * B_BYTES);
-        const uint8_t *src = p.wimg + (size_t)(it % p.num_kb) * 2 * B_BYTES;
-        uint8_t *b_img = b_ring + (size_t)s * 2 * B_BYTES;
-        for (int off = 0; off < 2 * B_BYTES; off += 16384) {
-          const int bytes = 2 * B_BYTES - off < 16384 ? 2 * B_BYTES - off : 16384;
-          bulk_g2s(b_img + off, src + off, bytes, &full_bar[s]);
-        }
+        const int vt = tile_of(it), w = cb_w(vt);
+        const int wb = w * 128;  // bytes of one (hi or lo) slice
+        mbar_arrive_expect_tx(&full_bar[s], 2 * wb);
+        const uint8_t *src = p.wimg + (size_t)(it % p.num_kb) * 2 * B_BYTES + (size_t)cb_beg(vt) * 128;
+        uint8_t *b_img = b_ring + (size_t)s * B_STAGE;
+        for (int part = 0; part < 2; ++part)  // hi slice, then lo slice (stage layout [hi w | lo w])
+          for (int off = 0; off < wb; off += 16384) {
+            const int bytes = wb - off < 16384 ? wb - off : 16384;
+            bulk_g2s(b_img + part * wb + off, src + (size_t)part * B_BYTES + off, bytes, &full_bar[s]);
+          }
       }
     }
   } else if (TMA_X && warp < NUM_PRODUCER_WARPS) {
@@ -367,6 +379,8 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
       if (buse > 0) mbar_wait(&tempty_bar[b], (buse - 1) & 1);
       asm volatile("tcgen05.fence::after_thread_sync;");
       const uint32_t tbase = tmem + (uint32_t)(b * p.n_acc * p.npa);
+      const int NW = TMA_X ? cb_w(tile) : NP;  // MMA width of this work item
+      const uint32_t b_lo_off = TMA_X ? (uint32_t)NW * 128 : (uint32_t)B_BYTES;
       for (int kb = 0; kb < p.num_kb; ++kb, ++it) {
         int s, sA;
         uint32_t a_hi, b_hi;
@@ -376,7 +390,7 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
           mbar_wait(&afull_bar[sA], (it / p.sa) & 1);
           mbar_wait(&full_bar[s], (it / p.sb) & 1);
           a_hi = smem_u32(smem + (size_t)sA * 2 * TILE_A_BYTES);
-          b_hi = smem_u32(b_ring + (size_t)s * 2 * B_BYTES);
+          b_hi = smem_u32(b_ring + (size_t)s * B_STAGE);
         } else {
           s = sA = it % S;
           mbar_wait(&full_bar[s], (it / S) & 1);
@@ -385,15 +399,15 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
         }
         asm volatile("tcgen05.fence::after_thread_sync;");
         if (lane == 0) {
-          const uint32_t a_lo = a_hi + TILE_A_BYTES, b_lo = b_hi + B_BYTES;
+          const uint32_t a_lo = a_hi + TILE_A_BYTES, b_lo = b_hi + b_lo_off;
           const int acc = kb % p.n_acc;
           const uint32_t d0 = tbase + (uint32_t)(acc * p.npa);
           const uint32_t first = (kb < p.n_acc) ? 1u : 0u;  // first K block of this accumulator
 #pragma unroll
           for (int j = 0; j < BK / 8; ++j) {  // 8 tf32 (32 B) per MMA K step
             const uint32_t ko = j * 32;
-            for (int n0 = 0; n0 < NP; n0 += 256) {
-              const int nn = NP - n0 < 256 ? NP - n0 : 256;
+            for (int n0 = 0; n0 < NW; n0 += 256) {
+              const int nn = NW - n0 < 256 ? NW - n0 : 256;
               const uint32_t id = idesc_tf32(nn);
               const uint32_t bo = (uint32_t)n0 * 128;
               const uint32_t d = d0 + (uint32_t)n0;
@@ -423,7 +437,7 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
     const int half = warp >= EPI_WARP1 ? 1 : 0;  // column chunks half, half + nhalf, ...
     const int nhalf = p.epi8 ? 2 : 1;
     const int widx = half ? 4 + warp - EPI_WARP1 : warp - EPI_WARP0;
-    uint8_t *const epi_buf = smem + (size_t)p.sa * 2 * TILE_A_BYTES + (size_t)p.sb * 2 * B_BYTES +
+    uint8_t *const epi_buf = smem + (size_t)p.sa * 2 * TILE_A_BYTES + (size_t)p.sb * B_STAGE +
                              (size_t)widx * p.eb * 4096;
     int chunk = 0;
     int tcount = 0;
@@ -432,11 +446,14 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
       mbar_wait(&tfull_bar[b], buse & 1);
       asm volatile("tcgen05.fence::after_thread_sync;");
       const int r = quad * 32 + lane;
-      const int64_t gm = (int64_t)tile * BM + r;
+      const int rt = TMA_H ? tile / p.ncb : tile;    // row tile
+      const int cbb = TMA_H ? cb_beg(tile) : 0;      // first global column of this work item
+      const int NW = TMA_H ? cb_w(tile) : NP;
+      const int64_t gm = (int64_t)rt * BM + r;
       const float sc = (p.row_scale && gm < p.m) ? __ldg(p.row_scale + gm) : 1.0f;
       const uint32_t tbase = tmem + (uint32_t)(b * p.n_acc * p.npa) + ((uint32_t)(quad * 32) << 16);
       const int n_acc_used = p.num_kb < p.n_acc ? p.num_kb : p.n_acc;
-      for (int c0 = half * 32; c0 < NP; c0 += 32 * nhalf) {
+      for (int c0 = half * 32; c0 < NW; c0 += 32 * nhalf) {
         float y[32];
 #pragma unroll
         for (int i = 0; i < 32; ++i) y[i] = 0.0f;
@@ -459,7 +476,7 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
         if (!TMA_H && gm >= p.m) continue;
 #pragma unroll
         for (int i = 0; i < 32; ++i) {
-          const int col = c0 + i;
+          const int col = cbb + c0 + i;
           float t = y[i];
           if (p.row_scale) t = t * sc;
           if (p.col_bias && col < p.n) t = t + __ldg(p.col_bias + col);
@@ -481,7 +498,7 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
                 make_float4(y[4 * c], y[4 * c + 1], y[4 * c + 2], y[4 * c + 3]);
           asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
           __syncwarp();
-          if (lane == 0) tma_store_2d(&hmap, c0, (int32_t)(tile * BM + quad * 32), buf);
+          if (lane == 0) tma_store_2d(&hmap, cbb + c0, (int32_t)(rt * BM + quad * 32), buf);
           ++chunk;
           continue;
         }
@@ -511,10 +528,12 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
 struct Config {
   int np, npa, num_kb, stages, n_acc, n_buf;
   int sa, sb, eb, epi8;
+  int ncb, cbw0, npa_t, nbuf_t, nacc_t;  // TMA path: column blocks and their TMEM layout
   size_t smem, smem_tma, wimg_bytes;
 };
 
 static int g_epi8 = -1;  // 8 epilogue warps on the TMA path (A/B switch: env GNN_GEMM_EPI8=0 disables)
+static int g_cb = -1;  // column blocks on the TMA path (A/B switch: env GNN_GEMM_CB=0 disables)
 static bool configure(int64_t m, int32_t k, int32_t n, Config &c) {
   if (n < 1 || n > 512 || k < 1 || m < 1) return false;
   c.np = (n + 15) / 16 * 16;
@@ -527,9 +546,28 @@ static bool configure(int64_t m, int32_t k, int32_t n, Config &c) {
   while (c.stages > 2 && (size_t)c.stages * stage_bytes + 2048 > 200 * 1024) --c.stages;
   c.smem = (size_t)c.stages * stage_bytes + 1024;
   if (c.smem > 227 * 1024) return false;
+  // TMA path, outputs wider than 256 columns with <= 8 K blocks: two column
+  // blocks per row tile (widths cbw0 = a multiple of 32, and np - cbw0), so
+  // each accumulator fits 256 TMEM columns and the epilogue of one block
+  // overlaps the MMAs of the next (a 272-column accumulator cannot be
+  // double-buffered in 512 columns).  The X tile is read twice (L2 hit).
+  if (g_cb < 0) {
+    const char *e = getenv("GNN_GEMM_CB");
+    g_cb = (e && e[0] == '0') ? 0 : 1;
+  }
+  c.ncb = 1;
+  c.cbw0 = c.np;
+  if (g_cb && c.np > 256 && c.num_kb <= 8) {
+    c.ncb = 2;
+    c.cbw0 = (c.np / 2 + 31) / 32 * 32;
+    if (c.cbw0 > 256 || c.np - c.cbw0 < 16) {
+      c.ncb = 1;
+      c.cbw0 = c.np;
+    }
+  }
   // TMA path: separate rings; deepen the X ring first (HBM latency), then W
   {
-    const size_t budget = 225 * 1024, a_bytes = 2 * TILE_A_BYTES, b_bytes = 2 * (size_t)c.np * 128;
+    const size_t budget = 225 * 1024, a_bytes = 2 * TILE_A_BYTES, b_bytes = 2 * (size_t)c.cbw0 * 128;
     c.sa = 2;
     c.sb = 2;
     // epilogue staging: (epi8 ? 8 : 4) warps x eb x 4 KB; prefer 8 warps
@@ -565,6 +603,14 @@ static bool configure(int64_t m, int32_t k, int32_t n, Config &c) {
   const int need_acc = (c.num_kb + 7) / 8;  // keep <= 8 K blocks per accumulator when possible
   if (c.n_acc > need_acc) c.n_acc = need_acc;
   if (c.n_acc < 1) c.n_acc = 1;
+  c.npa_t = c.npa;
+  c.nbuf_t = c.n_buf;
+  c.nacc_t = c.n_acc;
+  if (c.ncb > 1) {  // both blocks <= 256 columns: double buffer, one accumulator (<= 8 K blocks)
+    c.npa_t = 256;
+    c.nbuf_t = 2;
+    c.nacc_t = 1;
+  }
   return true;
 }
 
@@ -646,9 +692,9 @@ cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t 
     count_launch();
   }
   const int64_t num_tiles = (m + BM - 1) / BM;
-  if (num_tiles > 0x7fffffff) return cudaErrorNotSupported;
+  if (num_tiles > 0x3fffffff) return cudaErrorNotSupported;
   TcParams p{X, ldx, H, ldh, img, m, k, n, c.np, c.npa, c.num_kb, (int32_t)num_tiles, c.stages, c.n_acc, c.n_buf,
-             c.sa, c.sb, c.eb, c.epi8, row_scale, col_bias, relu};
+             c.sa, c.sb, c.eb, 1, c.np, c.epi8, row_scale, col_bias, relu};
   const bool vx = (ldx % 4 == 0) && ((uintptr_t)X % 16 == 0);
   const bool vh = (ldh % 4 == 0) && ((uintptr_t)H % 16 == 0);
   CUtensorMap xmap;
@@ -656,7 +702,7 @@ cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t 
   // TMA needs 16-byte aligned rows (vx) and a 32-bit row coordinate
   CUtensorMap hmap;
   memset(&hmap, 0, sizeof(hmap));
-  const bool tma = vx && c.sa > 0 && tma_enabled() && m < 0x7fffff00LL && encode_x_map(&xmap, X, ldx, m, k) &&
+  const bool tma = vx && c.sa > 0 && (vh || c.ncb == 1) && tma_enabled() && m < 0x7fffff00LL && encode_x_map(&xmap, X, ldx, m, k) &&
                    (!vh || encode_h_map(&hmap, H, ldh, m, n));
   auto fn = tma ? (vh ? k_gemm_tc<true, true, true> : k_gemm_tc<true, false, true>)
                 : vx ? (vh ? k_gemm_tc<true, true, false> : k_gemm_tc<true, false, false>)
@@ -664,8 +710,16 @@ cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t 
   const size_t smem = tma ? c.smem_tma : c.smem;
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  const int grid = (int)(num_tiles < num_sms ? num_tiles : num_sms);
+  const int grid = (int)(p.num_tiles < num_sms ? p.num_tiles : num_sms);
   if (!(tma && vh)) p.epi8 = 0;
+  if (tma && c.ncb > 1) {  // column blocks (vh holds here)
+    p.ncb = c.ncb;
+    p.cbw0 = c.cbw0;
+    p.npa = c.npa_t;
+    p.n_buf = c.nbuf_t;
+    p.n_acc = c.nacc_t;
+    p.num_tiles = (int32_t)(num_tiles * c.ncb);
+  }
   fn<<<grid, threads_of(tma), smem, s>>>(p, xmap, hmap);
   count_launch();
   return cudaGetLastError();

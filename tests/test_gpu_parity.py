@@ -393,7 +393,8 @@ def test_gemm_parity(m, k, n):
 
 
 @pytest.mark.parametrize("m,k,n,ldx", [(300, 17, 5, 17), (4099, 602, 256, 604), (5000, 100, 256, 100),
-                                       (1000, 256, 272, 256), (129, 33, 16, 36)])
+                                       (1000, 256, 272, 256), (129, 33, 16, 36), (777, 100, 304, 100),
+                                       (300, 64, 300, 64)])
 def test_gemm_tma_matches_register_path(m, k, n, ldx):
     """TMA-fed X tiles (impl 2) and register-fed X tiles (impl 3) build the
     same hi/lo operands, so the tcgen05 results are bit-identical."""
