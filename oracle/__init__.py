@@ -10,7 +10,10 @@ never imports it.
 Parity status per function (DESIGN.md §4 lists the pins):
   aggregate, aggregate_ng_f32, gemm, gcn_layer, gat_aggregate, gat_layer,
   edgeconv, minhash, lsh_pairs, las_merge, neighbor_groups,
-  partition_rows: pinned by tests/test_oracle_pins.py.
+  partition_rows: pinned by tests/test_oracle_pins.py; the LSH window and
+  within-bucket order, pair completeness/dedup, the merge's re-enqueue branch
+  and the hash family's known answers by tests/test_oracle_pins_las.py
+  (hand traces, tests/golden/fmix64_minhash.txt, the LSH S-curve).
   LAS *quality* (how much L2 reuse the schedule buys) is "parity unpinned":
   the paper's real graphs are unavailable.
 """
