@@ -363,8 +363,35 @@ def run_reference(args):
     print(json.dumps(out), flush=True)
 
 
+def relaunch_under_torchrun(n):
+    """`python bench.py --gpus N` without a launcher: re-exec this script under
+    torch.distributed.run with N local ranks (127.0.0.1 rendezvous), NCCL's INFO
+    lines on so the communicator's rank count is visible in the log."""
+    import socket
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")
+    env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd, env=env)
+
+
 def main():
     args = parse()
+    world = os.environ.get("WORLD_SIZE")
+    if world is None and args.gpus > 1:
+        if args.impl == "ours":
+            import torch
+            have = torch.cuda.device_count()
+            if have < args.gpus:
+                sys.exit(f"bench.py --gpus {args.gpus}: only {have} CUDA device(s) visible")
+        sys.exit(relaunch_under_torchrun(args.gpus))
+    if world is not None and int(world) != args.gpus:
+        sys.exit(f"bench.py: WORLD_SIZE={world} but --gpus {args.gpus}; launch one rank per GPU")
     if args.impl == "reference":
         run_reference(args)
     else:

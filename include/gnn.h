@@ -69,8 +69,8 @@ typedef struct {
   uint32_t struct_size;  /* sizeof(gnn_plan_opts), for ABI versioning */
   int32_t reorder;       /* 0 = identity task order, 1 = LAS (MinHash+LSH+merge) */
   int32_t group_size;    /* NG upper bound ng; -1 = auto (R8-ii); 0 = never split */
-  int32_t tile_groups;   /* T: max neighbor groups per work unit (a run of consecutive groups in
-                            task order streamed by one worker; capped at 32) (0 -> 32) */
+  int32_t tile_groups;   /* reserved (validated to [0, 256], otherwise unused): every neighbor
+                            group is one work unit claimed in task order (R8) */
   int32_t cluster_cap;   /* LAS cluster size cap (32) */
   int32_t minhash_k;     /* K signature length (32) */
   int32_t lsh_rows;      /* r rows per band (2); b = K / r bands */
@@ -91,8 +91,8 @@ typedef struct {
   int64_t n_src;        /* source rows (== n for gnn_plan_create) */
   int64_t nnz;
   int64_t n_groups;     /* G = sum ceil(d_v / ng) */
-  int64_t n_tiles;      /* work units (runs of <= T consecutive groups, <= E_u edges) */
-  int64_t n_split_rows; /* rows with more than T groups (combined through the workspace) */
+  int64_t n_tiles;      /* work units = neighbor groups (one unit per group, claimed in task order) */
+  int64_t n_split_rows; /* rows with more than one group (combined through the workspace, a9) */
   int64_t n_empty_rows;
   int64_t n_clusters;   /* LAS clusters (n if reorder == 0) */
   int64_t n_pairs;      /* LSH candidate pairs (0 if reorder == 0) */
@@ -104,8 +104,8 @@ typedef struct {
 } gnn_plan_info;
 
 /*
- * Build a plan (a1 CSR ingest + degrees, a2 LAS if opts->reorder, a3 NG and
- * CTA tiles).  Synchronous; copies the host CSR.  Validates in O(n + nnz):
+ * Build a plan (a1 CSR ingest + degrees, a2 LAS if opts->reorder, a3 NG work
+ * units in task order).  Synchronous; copies the host CSR.  Validates in O(n + nnz):
  * on failure returns GNN_ERR_INVALID_GRAPH and sets *out = NULL.
  * opts may be NULL (defaults).
  */
@@ -168,10 +168,11 @@ size_t gnn_workspace_size(gnn_plan_t plan, int op, int32_t f_in, int32_t f_out, 
 /*
  * a6 + a9: graph operation y_v = REDUCE_{u->v} e_uv * x_u (Table 1 x Table 2,
  * Eq 1 inner part P:217), evaluated over the plan's neighbor groups in task
- * order: persistent workers take work units (a whole row, or T groups of a
- * longer row) in task order; a row's group partials are combined in fixed
- * group order (R9) — in registers, or in the workspace by the last unit of a
- * long row to finish — or with atomics (deterministic == 0, sum/mean only).  Epilogue (linear property):
+ * order: persistent workers claim work units (one neighbor group each) in task
+ * order; a single-group row is finished by its worker; the group partials of a
+ * longer row are combined in fixed group order (R9) in the workspace by the
+ * last group to finish, or with atomics (deterministic == 0, sum/mean only).
+ * Epilogue (linear property):
  * GCN x ndst[v], mean / D_v, then + add_row[v] (nullable, EdgeConv's Q), then
  * ReLU if relu != 0.
  *   edge_w: [nnz] in CSR order, required iff weight == GNN_W_EDGE.
@@ -236,9 +237,13 @@ gnn_status gnn_edgeconv(gnn_plan_t plan, const float *X, int64_t ldx, int32_t f_
  * X: [m, ldx] (k used), W: [k, ldw] (n used), H: [m, ldh].
  * Epilogue: row_scale (nullable, [m]) multiplies row i; col_bias (nullable, [n])
  * is added after the scale; relu != 0 clamps.  H must not overlap X or W.
- * With ws (>= gnn_gemm_workspace_size(m, k, n) bytes, 256-byte aligned) and
- * n <= 512 the tcgen05 3xTF32 tensor-core kernel runs (the workspace holds the
- * split, pre-swizzled W image); with ws == NULL the SIMT fp32 FFMA kernel runs.
+ * With ws != NULL the tcgen05 3xTF32 tensor-core kernel runs for every shape
+ * (the workspace holds the split, pre-swizzled W image; outputs wider than one
+ * launch takes -- n > 320 with k > 256, or n > 512 -- run as ceil(n/256)
+ * launches over equal column slices); ws must be 16-byte aligned and hold
+ * gnn_gemm_workspace_size(m, k, n) bytes, else GNN_ERR_INVALID_ARG /
+ * GNN_ERR_WORKSPACE (never a silent fallback).  With ws == NULL the SIMT fp32
+ * FFMA kernel runs.
  */
 gnn_status gnn_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H,
                     int64_t ldh, int64_t m, int32_t k, int32_t n, const float *row_scale,
@@ -269,14 +274,6 @@ int gnn_set_gemm_impl(int impl);
  * feature and does not depend on the mapping).
  */
 gnn_status gnn_set_agg_mapping(int32_t vec, int32_t lanes, int32_t nv);
-
-/* Aggregation kernel selector for sum/mean/max (process-wide; same results
- * bit for bit): 1 = per-group kernel (default: one work unit = one neighbour
- * group), 0 = stream kernel (one worker streams a run of consecutive groups
- * with its loads in flight across group boundaries; measured slower, kept
- * for experiments).  GAT always takes the per-group kernel.  Returns the
- * previous value. */
-int gnn_set_agg_impl(int impl);
 
 /*
  * NG bound of an existing plan (reading R8): rebuilds the work
@@ -391,7 +388,6 @@ gnn_status gnn_las_host(int64_t n, const int64_t *rowptr_h, const uint64_t *sig_
 gnn_status gnn_groups_host(int64_t n, const int64_t *rowptr_h, const int32_t *perm_h, int32_t ng,
                            int64_t *n_groups, int32_t *grp_row_h, int64_t *grp_beg_h);
 
-/* Number of kernels this library launched since load (for bench accounting). */
 /*
  * NEXT-3 GraphSAGE-LSTM (Fig 6; setting P:1366-1367: 32 in /
  * 32 out, 16 sampled neighbours; reading R13).
@@ -474,6 +470,7 @@ gnn_status gnn_attn_aggregate(gnn_plan_t plan, int score, const float *Zs, int64
                               float neg_slope, int32_t head_mean, float *Y, int64_t ldy, void *ws,
                               size_t ws_bytes, gnn_stream_t stream);
 
+/* Number of kernels this library launched since load (for bench accounting). */
 uint64_t gnn_launch_count(void);
 
 const char *gnn_last_error(void);

@@ -39,15 +39,12 @@ struct DevGraph {
                                 //   tpos = offset in colidx_t, beg = CSR offset of the unit's first entry,
                                 //   m = long-row index (-1: the unit is the whole row); [n_units] = {nnz,0,0,-1}
   const int32_t *colidx_t;      // [nnz + 16] source indices in task order
-  const int32_t *pos_t;         // [nnz + 16] task position -> CSR position
-  const int32_t *sunit_beg;     // [n_sunits + 1] stream units: first group of each run
   const int32_t *multi_slot;    // [n_multi] workspace slot of a long row's first group
   const int32_t *multi_units;   // [n_multi] number of units of a long row
   const int32_t *multi_row;     // [n_multi] row id of each split row
   const int32_t *empty_rows;    // [n_empty]
   const int32_t *perm;          // [n] task (LAS) order of the rows
   int32_t n_units, n_multi, n_empty, ng;
-  int32_t n_sunits;
 };
 
 }  // namespace gnn
@@ -142,7 +139,6 @@ bool agg_override_active();
 bool agg_mapping_ok(const AggArgs &a, int32_t fh_or_0, int32_t vec, int32_t lanes, int32_t nv);
 gnn_status rebuild_schedule(gnn_plan_s *p, int64_t group_size);
 int64_t default_group_size(int64_t n, int64_t nnz);
-int set_agg_impl(int impl);
 size_t agg_workspace_bytes(const gnn_plan_s *p, int mode, int32_t F, int32_t H);
 cudaError_t launch_head_mean(const float *Yf, int64_t ldf, int64_t n, int32_t H, int32_t Fh, float *Y, int64_t ldy,
                              cudaStream_t s);

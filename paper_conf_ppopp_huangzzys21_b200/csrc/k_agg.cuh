@@ -66,10 +66,12 @@ struct KParams {
   int64_t ldk;
   const float *Wa;       // Gene: [H, Fh]
   int32_t *ws_unit;  // work-unit counters (one per feature chunk), zeroed per call
+  int32_t n_unit_ctr; // number of unit counters (>= feature chunks of any mapping)
   float *ws_acc;   // [n_multi][FW] atomic accumulators (deterministic == 0)
   float *ws_part;  // [multi slots][FW] per-group partials (deterministic)
   int32_t *ws_cnt; // [n_multi][nch] arrival counters
-  int32_t FW;      // F (+ 2H for GAT)
+  int32_t FW;      // partial slot width: F (+ 2 nmeta for attention), rounded to 8
+  int32_t nmeta;   // attention: (m, l) entries per slot = H + max chunks; entry of (chunk ci, head h) = h + ci
   int32_t deterministic;
   int32_t nch;        // feature chunks per row (arrival counters per multi-unit row)
   int32_t n_persist;  // persistent CTAs
@@ -627,7 +629,7 @@ __device__ __forceinline__ void group_chain_att(const KParams &p, const int32_t 
 // merge the group partials of a long row in group order (R9), epilogue, store
 template <int MODE, int VEC, int NV, int LANES>
 __device__ __forceinline__ void merge_row(const KParams &p, const float *base, int32_t ngrp, int32_t row,
-                                          int32_t deg, int32_t c0, int lane) {
+                                          int32_t deg, int32_t c0, int32_t ci, int lane) {
   Part<MODE, VEC, NV> A;
   part_init(A);
 #pragma unroll
@@ -638,8 +640,9 @@ __device__ __forceinline__ void merge_row(const KParams &p, const float *base, i
       float b[VEC];
       ldv_cg<VEC>(base + (size_t)q * p.FW + f, b);
       if constexpr (is_att(MODE)) {
-        const float bm = __ldcg(base + (size_t)q * p.FW + p.F + f / p.Fh);
-        const float bl = __ldcg(base + (size_t)q * p.FW + p.F + p.H + f / p.Fh);
+        const int32_t e = f / p.Fh + ci;  // (chunk, head) entry
+        const float bm = __ldcg(base + (size_t)q * p.FW + p.F + e);
+        const float bl = __ldcg(base + (size_t)q * p.FW + p.F + p.nmeta + e);
         if (q == 0) {
 #pragma unroll
           for (int i = 0; i < VEC; ++i) A.a[n][i] = b[i];
@@ -693,9 +696,13 @@ __device__ __forceinline__ void process_unit(const KParams &p, int4 d, int32_t l
     } else {
       stv<VEC>(base + (size_t)k * p.FW + f, G.a[n]);
       if constexpr (is_att(MODE)) {
-        if (f % p.Fh == 0) {
-          base[(size_t)k * p.FW + p.F + f / p.Fh] = G.m[n];
-          base[(size_t)k * p.FW + p.F + p.H + f / p.Fh] = G.l[n];
+        // the softmax state of (chunk ci, head h), written by the lane holding
+        // the head's first feature in this chunk (a head may straddle chunks;
+        // each chunk keeps its own reference and sum)
+        if (f % p.Fh == 0 || f == c0) {
+          const int32_t e = f / p.Fh + ci;
+          base[(size_t)k * p.FW + p.F + e] = G.m[n];
+          base[(size_t)k * p.FW + p.F + p.nmeta + e] = G.l[n];
         }
       }
     }
@@ -718,309 +725,9 @@ __device__ __forceinline__ void process_unit(const KParams &p, int4 d, int32_t l
     }
     store_row<MODE, VEC, NV, LANES>(p, row, re - rb, c0, lane, A);
   } else {
-    merge_row<MODE, VEC, NV, LANES>(p, base, ngrp, row, re - rb, c0, lane);
+    merge_row<MODE, VEC, NV, LANES>(p, base, ngrp, row, re - rb, c0, ci, lane);
   }
   if (lane == 0) *cnt = 0;  // leave the counter at 0 for the next call
-}
-
-// ---------------------------------------------------------------------------
-// v10 stream kernel.  A work unit is a run of consecutive neighbour groups in
-// task order (plan: <= 32 groups, <= E_u edges); its source indices are one
-// contiguous range [T0, T1) of colidx_t.  The worker streams that range with
-// U source rows in flight and never drains its load pipeline at group or row
-// boundaries: when the edge that ends a group is consumed, the group's chain
-// (R9, unchanged: a fresh fp32 chain per group in CSR order) is finished —
-// epilogue + store, or partial + fixed-order merge for split rows — while the
-// loads of the next group's first rows are already in flight.
-//
-// Index stream: three LANES-wide batches (A = being issued, B, C = loading);
-// per-edge weights (GCN nsrc[u], explicit edge_w via the task->CSR map) are
-// fetched one batch ahead from indices that already arrived, so no load in
-// the loop waits on another load.
-// ---------------------------------------------------------------------------
-template <int MODE, int VEC, int NV, int LANES, bool WGT>
-struct Stream {
-  static constexpr int FPL = VEC * NV;
-  static constexpr int U0 = FPL >= 32 ? 1 : (32 / FPL > 8 ? 8 : 32 / FPL);
-  static constexpr int U = (is_att(MODE) && U0 > 4) ? 4 : (U0 > LANES ? LANES : U0);
-};
-
-// finish one group: epilogue + store (whole row), or the group's partial to
-// its workspace slot (atomics into one accumulator row in the non-deterministic
-// variant); split rows are merged by k_merge after the stream kernel
-template <int MODE, int VEC, int NV, int LANES>
-__device__ __forceinline__ void finish_group(const KParams &p, const Part<MODE, VEC, NV> &G, int32_t row, int32_t m,
-                                             int32_t gbeg, int32_t len, int32_t c0, int32_t ci, int lane,
-                                             unsigned mask) {
-  if (m < 0) {
-    store_row<MODE, VEC, NV, LANES>(p, row, len, c0, lane, G);
-    return;
-  }
-  const DevGraph &g = p.g;
-  const int32_t k = (gbeg - __ldg(g.rowptr + row)) / g.ng;
-  const bool atomic_acc = !p.deterministic && MODE == M_SUM;
-  float *base = p.ws_part + (size_t)__ldg(g.multi_slot + m) * p.FW;
-  float *acc = p.ws_acc + (size_t)m * p.FW;
-#pragma unroll
-  for (int n = 0; n < NV; ++n) {
-    const int32_t f = c0 + (n * LANES + lane) * VEC;
-    if (f >= p.F) continue;
-    if (atomic_acc) {
-#pragma unroll
-      for (int i = 0; i < VEC; ++i) atomicAdd(acc + f + i, G.a[n][i]);
-    } else {
-      stv<VEC>(base + (size_t)k * p.FW + f, G.a[n]);
-      if constexpr (is_att(MODE)) {
-        if (f % p.Fh == 0) {
-          base[(size_t)k * p.FW + p.F + f / p.Fh] = G.m[n];
-          base[(size_t)k * p.FW + p.F + p.H + f / p.Fh] = G.l[n];
-        }
-      }
-    }
-  }
-}
-
-// split rows (more than one group): merge the group partials in group order
-// (R9) and apply the postponed epilogue.  One worker per row.
-template <int MODE, int VEC, int NV, int LANES>
-__global__ void __launch_bounds__(256) k_merge(const KParams p) {
-  constexpr int CW = LANES * VEC * NV;
-  const int lane = threadIdx.x & (LANES - 1);
-  const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / LANES;
-  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) / LANES;
-  const DevGraph &g = p.g;
-  for (int64_t m = w; m < g.n_multi; m += nw) {
-    const int32_t row = __ldg(g.multi_row + m);
-    const int32_t rb = __ldg(g.rowptr + row), re = __ldg(g.rowptr + row + 1);
-    const int32_t ngrp = 1 + (re - rb - 1) / g.ng;
-    for (int32_t c0 = 0; c0 < p.F; c0 += CW) {
-      if (!p.deterministic && MODE == M_SUM) {
-        const float *acc = p.ws_acc + (size_t)m * p.FW;
-        Part<MODE, VEC, NV> A;
-        part_init(A);
-#pragma unroll
-        for (int n = 0; n < NV; ++n) {
-          const int32_t f = c0 + (n * LANES + lane) * VEC;
-          if (f < p.F) ldv_cg<VEC>(acc + f, A.a[n]);
-        }
-        store_row<MODE, VEC, NV, LANES>(p, row, re - rb, c0, lane, A);
-      } else {
-        const float *base = p.ws_part + (size_t)__ldg(g.multi_slot + m) * p.FW;
-        merge_row<MODE, VEC, NV, LANES>(p, base, ngrp, row, re - rb, c0, lane);
-      }
-    }
-  }
-}
-
-template <int MODE, int VEC, int NV, int LANES, bool WGT>
-__device__ __forceinline__ void stream_unit(const KParams &p, int32_t g0, int32_t g1, int32_t T0, int32_t T1,
-                                            int32_t c0, int32_t ci, int lane, unsigned mask) {
-  constexpr int U = Stream<MODE, VEC, NV, LANES, WGT>::U;
-  const DevGraph &g = p.g;
-  // group table: lane j holds group gw + j
-  int32_t gw = g0;
-  int32_t gtp = 0, gend = 0, grow = 0, gm = -1, gbg = 0;
-  auto load_table = [&]() {
-    if (gw + lane < g1) {
-      const int4 d = __ldg(g.unit_desc + gw + lane);
-      gtp = d.x; gbg = d.y; grow = d.z; gm = d.w;
-      gend = __ldg(&g.unit_desc[gw + lane + 1].x);
-    }
-  };
-  load_table();
-  // index batches
-  const int32_t *idx = g.colidx_t;
-  auto ld_idx = [&](int32_t pos) -> int32_t { return pos < T1 ? ld_stream_i32(idx + pos) : 0; };
-  auto ld_pos = [&](int32_t pos) -> int32_t { return pos < T1 ? ld_stream_i32(g.pos_t + pos) : 0; };
-  auto weight_of = [&](int32_t u, int32_t cpos, int32_t pos) -> float {
-    if constexpr (WGT) {
-      if (pos >= T1) return 0.0f;
-      return p.weight == GNN_W_GCN ? __ldg(g.nsrc + u) : ld_stream_f32(p.edge_w + cpos);
-    } else {
-      return 1.0f;
-    }
-  };
-  int32_t ibase = T0;
-  int32_t a_u = ld_idx(T0 + lane), b_u = ld_idx(T0 + LANES + lane), c_u = ld_idx(T0 + 2 * LANES + lane);
-  int32_t a_c = 0, b_c = 0, c_c = 0;
-  if (WGT && p.weight == GNN_W_EDGE) {
-    a_c = ld_pos(T0 + lane); b_c = ld_pos(T0 + LANES + lane); c_c = ld_pos(T0 + 2 * LANES + lane);
-  }
-  float a_w = weight_of(a_u, a_c, T0 + lane), b_w = weight_of(b_u, b_c, T0 + LANES + lane);
-  // per-lane feature slice
-  bool valid[NV];
-  int32_t head[NV];
-#pragma unroll
-  for (int n = 0; n < NV; ++n) {
-    const int32_t f = c0 + (n * LANES + lane) * VEC;
-    valid[n] = f < p.F;
-    head[n] = (is_att(MODE) && valid[n]) ? f / p.Fh : 0;
-  }
-  const float *xl = p.X + c0 + lane * VEC;
-  // current group
-  int32_t gi = g0;
-  int32_t cur_end = __shfl_sync(mask, gend, 0, LANES);
-  float tv[NV], tvn[NV];
-  auto load_tv = [&](int32_t row, float (&out)[NV]) {
-#pragma unroll
-    for (int n = 0; n < NV; ++n) out[n] = valid[n] ? __ldg(p.t + (int64_t)row * p.ldt + head[n]) : 0.0f;
-  };
-  if constexpr (is_att(MODE)) {
-    load_tv(__shfl_sync(mask, grow, 0, LANES), tv);
-    if (g0 + 1 < g1 && 1 < LANES) load_tv(__shfl_sync(mask, grow, 1, LANES), tvn);
-  }
-  Part<MODE, VEC, NV> G;
-  part_init(G);
-  float v[U][NV][VEC];
-  float sc[U][NV];
-  float wq[U];
-  // issue the load of edge `pos` into slot q (pos is the next position in
-  // order; a macro so that q is a compile-time constant after unrolling and
-  // the slot arrays stay in registers)
-#define GNN_ISSUE(q, pos)                                                                             \
-  do {                                                                                                \
-    int32_t off_ = (pos) - ibase;                                                                     \
-    if (off_ == LANES) { /* batch A fully issued: rotate */                                          \
-      a_u = b_u; a_w = b_w; a_c = b_c;                                                                \
-      b_u = c_u; b_c = c_c;                                                                           \
-      b_w = weight_of(b_u, b_c, ibase + 2 * LANES + lane);                                            \
-      c_u = ld_idx(ibase + 3 * LANES + lane);                                                         \
-      if (WGT && p.weight == GNN_W_EDGE) c_c = ld_pos(ibase + 3 * LANES + lane);                      \
-      ibase += LANES;                                                                                 \
-      off_ = 0;                                                                                       \
-    }                                                                                                 \
-    const int32_t u_ = __shfl_sync(mask, a_u, off_, LANES);                                           \
-    if constexpr (WGT) wq[q] = __shfl_sync(mask, a_w, off_, LANES);                                   \
-    _Pragma("unroll") for (int n = 0; n < NV; ++n) {                                                  \
-      if (valid[n]) ldv<VEC>(xl + (int64_t)u_ * p.ldx + n * LANES * VEC, v[q][n]);                    \
-      if constexpr (is_att(MODE))                                                                    \
-        sc[q][n] = valid[n] ? __ldg(p.X + (int64_t)u_ * p.ldx + p.F + head[n]) : 0.0f;                \
-    }                                                                                                 \
-  } while (0)
-  int32_t pi = T0;
-#pragma unroll
-  for (int q = 0; q < U; ++q)
-    if (pi < T1) {
-      GNN_ISSUE(q, pi);
-      ++pi;
-    }
-  int32_t pe = T0;
-  while (pe < T1) {
-#pragma unroll
-    for (int q = 0; q < U; ++q) {
-      if (pe < T1) {
-        // consume edge pe (slot q)
-        if constexpr (is_att(MODE)) {
-#pragma unroll
-          for (int n = 0; n < NV; ++n) {
-            if (!valid[n]) continue;
-            float sco = sc[q][n] + tv[n];
-            sco = sco > 0.0f ? sco : p.slope * sco;  // LeakyReLU (Table 2 GAT)
-            const float d = sco - G.m[n];
-            const float ex = __expf(-fabsf(d));
-            const bool up = d > 0.0f;
-#pragma unroll
-            for (int i = 0; i < VEC; ++i)
-              G.a[n][i] = fmaf(up ? G.a[n][i] : v[q][n][i], ex, up ? v[q][n][i] : G.a[n][i]);
-            G.l[n] = fmaf(up ? G.l[n] : 1.0f, ex, up ? 1.0f : G.l[n]);
-            G.m[n] = up ? sco : G.m[n];
-          }
-        } else {
-          const float w = WGT ? wq[q] : 1.0f;
-#pragma unroll
-          for (int n = 0; n < NV; ++n) {
-            if (!valid[n]) continue;
-#pragma unroll
-            for (int i = 0; i < VEC; ++i) {
-              if constexpr (MODE == M_MAX) G.a[n][i] = fmaxf(G.a[n][i], WGT ? w * v[q][n][i] : v[q][n][i]);
-              else G.a[n][i] = WGT ? fmaf(w, v[q][n][i], G.a[n][i]) : G.a[n][i] + v[q][n][i];
-            }
-          }
-        }
-        ++pe;
-        if (pe == cur_end) {
-          const int j = gi - gw;
-          const int32_t row = __shfl_sync(mask, grow, j, LANES);
-          const int32_t m = __shfl_sync(mask, gm, j, LANES);
-          const int32_t gb = __shfl_sync(mask, gbg, j, LANES);
-          const int32_t tp = __shfl_sync(mask, gtp, j, LANES);
-          finish_group<MODE, VEC, NV, LANES>(p, G, row, m, gb, cur_end - tp, c0, ci, lane, mask);
-          part_init(G);
-          ++gi;
-          if (gi < g1) {
-            if (gi - gw == LANES) {  // next window of the group table
-              gw += LANES;
-              load_table();
-              if constexpr (is_att(MODE)) load_tv(__shfl_sync(mask, grow, 0, LANES), tvn);
-            }
-            cur_end = __shfl_sync(mask, gend, gi - gw, LANES);
-            if constexpr (is_att(MODE)) {
-#pragma unroll
-              for (int n = 0; n < NV; ++n) tv[n] = tvn[n];
-              const int jn = gi + 1 - gw;
-              const int32_t rn = __shfl_sync(mask, grow, jn < LANES ? jn : 0, LANES);
-              if (gi + 1 < g1 && jn < LANES) load_tv(rn, tvn);
-            }
-          }
-        }
-        if (pi < T1) {
-          GNN_ISSUE(q, pi);
-          ++pi;
-        }
-      }
-    }
-  }
-#undef GNN_ISSUE
-}
-
-template <int MODE, int VEC, int NV, int LANES, bool WGT>
-__global__ void __launch_bounds__(256, is_att(MODE) ? 3 : 4) k_stream(const KParams p) {
-  constexpr int CW = LANES * VEC * NV;
-  const int tid = threadIdx.x;
-  const int lane = tid & (LANES - 1);
-  const unsigned mask =
-      LANES == 32 ? 0xffffffffu : (((1u << LANES) - 1u) << ((tid & 31) & ~(LANES - 1)));
-  const DevGraph &g = p.g;
-  if ((int32_t)blockIdx.x >= p.n_persist) {
-    const int64_t r0 = (int64_t)(blockIdx.x - p.n_persist) * 32;
-    for (int64_t r = r0; r < r0 + 32 && r < g.n_empty; ++r) {
-      float *y = p.Y + (int64_t)g.empty_rows[r] * p.ldy;
-      for (int f = tid; f < p.F; f += blockDim.x) y[f] = 0.0f;
-    }
-    return;
-  }
-  const int32_t nunits = g.n_sunits;
-  int32_t ci = 0;
-  for (int32_t c0 = 0; c0 < p.F; c0 += CW, ++ci) {
-    int32_t *ctr = p.ws_unit + ci;
-    // the next unit (id, group range, index range) is claimed while the current one streams
-    int32_t u = 0;
-    if (lane == 0) u = atomicAdd(ctr, 1);
-    u = __shfl_sync(mask, u, 0, LANES);
-    int32_t g0 = 0, g1 = 0, t0 = 0, t1 = 0;
-    if (u < nunits) {
-      g0 = __ldg(g.sunit_beg + u);
-      g1 = __ldg(g.sunit_beg + u + 1);
-      t0 = __ldg(&g.unit_desc[g0].x);
-      t1 = __ldg(&g.unit_desc[g1].x);
-    }
-    while (u < nunits) {
-      int32_t un = 0;
-      if (lane == 0) un = atomicAdd(ctr, 1);
-      un = __shfl_sync(mask, un, 0, LANES);
-      int32_t h0 = 0, h1 = 0, s0 = 0, s1 = 0;
-      if (un < nunits) {
-        h0 = __ldg(g.sunit_beg + un);
-        h1 = __ldg(g.sunit_beg + un + 1);
-      }
-      stream_unit<MODE, VEC, NV, LANES, WGT>(p, g0, g1, t0, t1, c0, ci, lane, mask);
-      if (un < nunits) {
-        s0 = __ldg(&g.unit_desc[h0].x);
-        s1 = __ldg(&g.unit_desc[h1].x);
-      }
-      u = un; g0 = h0; g1 = h1; t0 = s0; t1 = s1;
-    }
-  }
 }
 
 #ifndef GNN_AGG_MINB
@@ -1086,7 +793,6 @@ struct Mapping {
   int vec, lanes, nv;
 };
 int num_sms();
-int agg_impl();
 
 template <typename KFN>
 cudaError_t launch_persistent(KFN fn, int &occ, const KParams &kp_in, int32_t units, int cw, int lanes,
@@ -1101,7 +807,8 @@ cudaError_t launch_persistent(KFN fn, int &occ, const KParams &kp_in, int32_t un
   const int64_t workers_per_cta = threads / lanes;
   kp.n_persist = (int32_t)std::min<int64_t>((int64_t)num_sms() * occ,
                                             std::max<int64_t>(1, (units + workers_per_cta - 1) / workers_per_cta));
-  cudaError_t e = cudaMemsetAsync(kp.ws_unit, 0, 256, s);
+  if (kp.nch > kp.n_unit_ctr) return cudaErrorInvalidValue;  // mapping wider than the workspace sizing
+  cudaError_t e = cudaMemsetAsync(kp.ws_unit, 0, sizeof(int32_t) * (size_t)kp.n_unit_ctr, s);
   if (e == cudaSuccess && kp.g.n_multi > 0)
     e = cudaMemsetAsync(kp.ws_cnt, 0, sizeof(int32_t) * (size_t)kp.g.n_multi * kp.nch, s);
   if (e == cudaSuccess && kp.g.n_multi > 0 && !kp.deterministic && kp.mode != M_MAX && !is_att(kp.mode))
@@ -1116,29 +823,8 @@ cudaError_t launch_persistent(KFN fn, int &occ, const KParams &kp_in, int32_t un
 template <int MODE, int VEC, int NV, int LANES>
 cudaError_t launch_one(const KParams &kp, int threads, cudaStream_t s) {
   constexpr int CW = LANES * VEC * NV;
-  if (agg_impl() == 1) {
-    static int occ = 0;
-    return launch_persistent(k_aggregate<MODE, VEC, NV, LANES>, occ, kp, kp.g.n_units, CW, LANES, threads, s);
-  }
-  const bool wgt = !is_att(MODE) && (kp.weight == GNN_W_GCN || kp.weight == GNN_W_EDGE);
-  cudaError_t e;
-  if constexpr (!is_att(MODE)) {
-    static int occ_w = 0;
-    static int occ = 0;
-    e = wgt ? launch_persistent(k_stream<MODE, VEC, NV, LANES, true>, occ_w, kp, kp.g.n_sunits, CW, LANES, threads, s)
-            : launch_persistent(k_stream<MODE, VEC, NV, LANES, false>, occ, kp, kp.g.n_sunits, CW, LANES, threads, s);
-  } else {
-    static int occ = 0;
-    e = launch_persistent(k_stream<MODE, VEC, NV, LANES, false>, occ, kp, kp.g.n_sunits, CW, LANES, threads, s);
-  }
-  if (e != cudaSuccess || kp.g.n_multi == 0) return e;
-  // split rows: fixed-order merge of the group partials (R9)
-  KParams km = kp;
-  km.nch = (kp.F + CW - 1) / CW;
-  const int64_t blocks = std::max<int64_t>(1, std::min<int64_t>((kp.g.n_multi * LANES + 255) / 256, 148 * 8));
-  k_merge<MODE, VEC, NV, LANES><<<(unsigned)blocks, 256, 0, s>>>(km);
-  count_launch();
-  return cudaGetLastError();
+  static int occ = 0;
+  return launch_persistent(k_aggregate<MODE, VEC, NV, LANES>, occ, kp, kp.g.n_units, CW, LANES, threads, s);
 }
 
 template <int MODE, int VEC>

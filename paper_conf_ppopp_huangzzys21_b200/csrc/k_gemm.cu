@@ -133,16 +133,20 @@ gnn_status launch_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw,
                        int64_t ldh, int64_t m, int32_t k, int32_t n, const float *row_scale,
                        const float *col_bias, int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s) {
   if (m == 0 || n == 0) return GNN_OK;
-  if (g_gemm_impl != 1 && ws != nullptr) {
+  if (g_gemm_impl != 1 && ws != nullptr && k > 0) {
+    // a caller that passes a workspace gets the tensor cores or an error,
+    // never a silent fallback (every n is taken, wide ones as column slices)
     cudaError_t e = launch_gemm_tc(X, ldx, W, ldw, H, ldh, m, k, n, row_scale, col_bias, relu, ws, ws_bytes, s);
     if (e == cudaSuccess) return GNN_OK;
-    if (e != cudaErrorNotSupported) return cuda_status(e, "gemm tcgen05 launch");
-    if (g_gemm_impl >= 2) {
-      set_error("tcgen05 GEMM does not support this shape/alignment/workspace");
-      return GNN_ERR_UNSUPPORTED;
+    if (e == cudaErrorInvalidValue) {
+      set_error("gemm workspace too small: need gnn_gemm_workspace_size(m, k, n) = " +
+                std::to_string(gemm_tc_workspace(m, k, n)) + " bytes");
+      return GNN_ERR_WORKSPACE;
     }
-    (void)cudaGetLastError();
-  } else if (g_gemm_impl >= 2) {
+    if (e != cudaErrorNotSupported) return cuda_status(e, "gemm tcgen05 launch");
+    set_error("tcgen05 GEMM: workspace must be 16-byte aligned");
+    return GNN_ERR_INVALID_ARG;
+  } else if (g_gemm_impl >= 2 && k > 0) {
     set_error("tcgen05 GEMM needs a workspace (gnn_gemm_workspace_size)");
     return GNN_ERR_UNSUPPORTED;
   }

@@ -664,19 +664,54 @@ static bool encode_h_map(CUtensorMap *map, float *H, int64_t ldh, int64_t m, int
 
 void gemm_tc_set_tma(int on) { tc::g_tma_mode = on ? 1 : 0; }
 
-size_t gemm_tc_workspace(int64_t m, int32_t k, int32_t n) {
+// Column slices: an output wider than one launch takes (the W image stages of
+// 2 x np x 128 B no longer fit shared memory, n > 320 with K > 256 or n > 512)
+// is computed as ceil(n / 256) launches over column slices of equal width
+// (a multiple of 32, <= 256); each re-reads X (L2 or HBM).  Returns the
+// columns per launch (n when one launch takes the whole width).
+static int32_t slice_width(int64_t m, int32_t k, int32_t n) {
   tc::Config c;
-  if (!tc::configure(m > 0 ? m : 1, k, n, c)) return 0;
+  if (tc::configure(m > 0 ? m : 1, k, n, c)) return n;
+  const int32_t nsl = (n + 255) / 256;
+  return ((n + nsl - 1) / nsl + 31) / 32 * 32;
+}
+
+size_t gemm_tc_workspace(int64_t m, int32_t k, int32_t n) {
+  if (n < 1 || k < 1) return 0;
+  tc::Config c;
+  if (!tc::configure(m > 0 ? m : 1, k, slice_width(m, k, n), c)) return 0;
   return (c.wimg_bytes + 255) & ~(size_t)255;
 }
 
+static cudaError_t launch_gemm_tc_one(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H, int64_t ldh,
+                                      int64_t m, int32_t k, int32_t n, const float *row_scale, const float *col_bias,
+                                      int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s);
+
+// Returns cudaErrorNotSupported only for shapes no launch takes (k < 1) or a
+// missing / misaligned workspace, cudaErrorInvalidValue for a workspace that
+// is too small (the caller reports GNN_ERR_WORKSPACE).
 cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H, int64_t ldh,
                            int64_t m, int32_t k, int32_t n, const float *row_scale, const float *col_bias,
                            int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s) {
+  if (k < 1 || n < 1 || !ws || ((uintptr_t)ws & 15)) return cudaErrorNotSupported;
+  if (ws_bytes < gemm_tc_workspace(m, k, n)) return cudaErrorInvalidValue;
+  const int32_t sw = slice_width(m, k, n);
+  for (int32_t c0 = 0; c0 < n; c0 += sw) {
+    const int32_t w = n - c0 < sw ? n - c0 : sw;
+    cudaError_t e = launch_gemm_tc_one(X, ldx, W + c0, ldw, H + c0, ldh, m, k, w, row_scale,
+                                       col_bias ? col_bias + c0 : nullptr, relu, ws, ws_bytes, s);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+
+static cudaError_t launch_gemm_tc_one(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H, int64_t ldh,
+                                      int64_t m, int32_t k, int32_t n, const float *row_scale, const float *col_bias,
+                                      int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s) {
   using namespace tc;
   Config c;
   if (!configure(m, k, n, c)) return cudaErrorNotSupported;
-  if (!ws || ws_bytes < c.wimg_bytes || ((uintptr_t)ws & 15)) return cudaErrorNotSupported;
+  if (ws_bytes < c.wimg_bytes) return cudaErrorInvalidValue;
   static int num_sms = 0;
   if (num_sms == 0) {
     int dev = 0;
@@ -710,7 +745,6 @@ cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t 
   const size_t smem = tma ? c.smem_tma : c.smem;
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  const int grid = (int)(p.num_tiles < num_sms ? p.num_tiles : num_sms);
   if (!(tma && vh)) p.epi8 = 0;
   if (tma && c.ncb > 1) {  // column blocks (vh holds here)
     p.ncb = c.ncb;
@@ -720,6 +754,8 @@ cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t 
     p.n_acc = c.nacc_t;
     p.num_tiles = (int32_t)(num_tiles * c.ncb);
   }
+  // one persistent CTA per SM, or one per work item when there are fewer
+  const int grid = (int)(p.num_tiles < num_sms ? p.num_tiles : num_sms);
   fn<<<grid, threads_of(tma), smem, s>>>(p, xmap, hmap);
   count_launch();
   return cudaGetLastError();

@@ -248,9 +248,11 @@ static bool mapping_ok(const AggArgs &a, int32_t fh_or_0, const Mapping &o) {
   // the Table 2 scores other than GAT are instantiated with one vector per lane
   if (a.mode > M_GAT && o.nv != 1) return false;
   if (vec_score(a.mode) && fh_or_0 / o.vec > o.lanes) return false;
-  // GAT: a chunk must hold whole heads (the softmax state is per head)
+  // GaAN / Gene: a chunk must hold whole heads (the score is a butterfly sum
+  // over the head's lanes).  Scalar scores (GAT, Sym-GAT, Linear) may split a
+  // head across chunks: each chunk keeps its own softmax state per head.
   const int cw = o.vec * o.lanes * o.nv;
-  const bool heads_ok = !fh_or_0 || cw >= a.F || cw % fh_or_0 == 0;
+  const bool heads_ok = !vec_score(a.mode) || cw >= a.F || cw % fh_or_0 == 0;
   return heads_ok && (a.F + cw - 1) / cw <= max_chunks(a.F);
 }
 
@@ -306,22 +308,40 @@ static Mapping choose_mapping(const gnn_plan_s *p, const AggArgs &a, int32_t fh_
 }
 
 
-// layout: [unit counters (256 B)][attention score maxima: H or 2H keys | pad 256]
-//         [row counters n_multi x nch | pad 256][acc n_multi x FW][slots x FW]
+// Workspace layout (every region 256-byte aligned):
+//   [unit counters: one int32 per feature chunk (<= max_chunks(F))]
+//   [attention score maxima: H or 2H order-encoded keys]
+//   [arrival counters: n_multi x max_chunks(F)]
+//   [atomic accumulators: n_multi x FW][group partial slots: multi_slots x FW]
 static size_t smax_bytes(int mode, int32_t H) {
   const size_t keys = (mode == M_GAT || mode == M_GAAN) ? (size_t)H : (mode == M_SYM ? 2 * (size_t)H : 0);
   return (sizeof(uint32_t) * keys + 255) & ~(size_t)255;
 }
-// partial-slot width: F (+ m, l per head for attention), rounded up to 8 floats
-// so that every slot row is 32-byte aligned for the vector stores
-static int32_t slot_width(int mode, int32_t F, int32_t H) { return (F + (is_att(mode) ? 2 * H : 0) + 7) / 8 * 8; }
+static size_t a256(size_t b) { return (b + 255) & ~(size_t)255; }
+// partial-slot width: F, plus for attention the softmax state (m, l) of every
+// (feature chunk, head) pair the chunk touches -- at most H + nch of them, so
+// a head split across two chunks keeps one (m, l) per chunk -- rounded up to
+// 8 floats so every slot row is 32-byte aligned for the vector stores
+static int32_t att_meta(int mode, int32_t F, int32_t H) { return is_att(mode) ? H + max_chunks(F) : 0; }
+static int32_t slot_width(int mode, int32_t F, int32_t H) { return (F + 2 * att_meta(mode, F, H) + 7) / 8 * 8; }
+
+struct WsLayout {
+  size_t unit, smax, cnt, acc, part, total;
+};
+static WsLayout ws_layout(const gnn_plan_s *p, int mode, int32_t F, int32_t H) {
+  const size_t FW = (size_t)slot_width(mode, F, H);
+  WsLayout L;
+  L.unit = 0;
+  L.smax = L.unit + a256(sizeof(int32_t) * (size_t)max_chunks(F));
+  L.cnt = L.smax + smax_bytes(mode, H);
+  L.acc = L.cnt + a256(sizeof(int32_t) * (size_t)p->n_multi * max_chunks(F));
+  L.part = L.acc + sizeof(float) * (size_t)p->n_multi * FW;
+  L.total = L.part + sizeof(float) * (size_t)p->multi_slots * FW;
+  return L;
+}
 
 size_t agg_workspace_bytes(const gnn_plan_s *p, int mode, int32_t F, int32_t H) {
-  const size_t FW = (size_t)slot_width(mode, F, H);
-  size_t b = 256 + smax_bytes(mode, H);
-  size_t c = sizeof(int32_t) * (size_t)p->n_multi * max_chunks(F);
-  b += (c + 255) & ~(size_t)255;
-  return b + sizeof(float) * ((size_t)p->multi_slots + (size_t)p->n_multi) * FW;
+  return ws_layout(p, mode, F, H).total;
 }
 
 int num_sms() {
@@ -333,14 +353,6 @@ int num_sms() {
     if (n <= 0) n = 148;
   }
   return n;
-}
-
-static int g_agg_impl = 1;  // 0 = v10 stream kernel (measured slower), 1 = v8 per-group kernel
-int agg_impl() { return g_agg_impl; }
-int set_agg_impl(int impl) {
-  const int old = g_agg_impl;
-  g_agg_impl = impl;
-  return old;
 }
 
 gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, size_t ws_bytes, cudaStream_t s) {
@@ -373,14 +385,15 @@ gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, siz
   kp.ldk = a.ldk;
   kp.Wa = a.Wa;
   kp.FW = slot_width(mode, a.F, a.H);
+  kp.nmeta = att_meta(mode, a.F, a.H);
   kp.deterministic = a.deterministic;
+  const WsLayout L = ws_layout(p, mode, a.F, a.H);
   char *w = reinterpret_cast<char *>(ws);
-  kp.ws_unit = reinterpret_cast<int32_t *>(w);
-  const size_t cnt_bytes = (sizeof(int32_t) * (size_t)p->n_multi * max_chunks(a.F) + 255) & ~(size_t)255;
-  const size_t sm_bytes = smax_bytes(mode, a.H);
-  kp.ws_cnt = reinterpret_cast<int32_t *>(w + 256 + sm_bytes);
-  kp.ws_acc = reinterpret_cast<float *>(w + 256 + sm_bytes + cnt_bytes);
-  kp.ws_part = kp.ws_acc + (size_t)p->n_multi * kp.FW;
+  kp.ws_unit = reinterpret_cast<int32_t *>(w + L.unit);
+  kp.n_unit_ctr = max_chunks(a.F);
+  kp.ws_cnt = reinterpret_cast<int32_t *>(w + L.cnt);
+  kp.ws_acc = reinterpret_cast<float *>(w + L.acc);
+  kp.ws_part = reinterpret_cast<float *>(w + L.part);
   const Mapping m = choose_mapping(p, a, is_att(mode) ? a.Fh : 0);
   if (m.vec == 0) {
     set_error("no supported lane mapping for this width / head size (GaAN, Gene: Fh/vec must be a power of 2 <= 32)");
@@ -388,7 +401,7 @@ gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, siz
   }
   const int threads = 256;
   cudaError_t e = cudaSuccess;
-  uint32_t *smax = reinterpret_cast<uint32_t *>(w + 256);
+  uint32_t *smax = reinterpret_cast<uint32_t *>(w + L.smax);
   kp.smax = smax;
   if (mode == M_GAT || mode == M_SYM) e = launch_score_max(a.X + a.F, a.ldx, p->n_src, a.H, 1, smax, s);
   if (e == cudaSuccess && mode == M_SYM) e = launch_score_max(a.X + a.F + a.H, a.ldx, p->n_src, a.H, 1, smax + a.H, s);

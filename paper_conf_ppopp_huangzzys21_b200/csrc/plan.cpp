@@ -279,33 +279,6 @@ gnn_status build_schedule(gnn_plan_s *p) {
   }
   const int64_t n_units = (int64_t)desc.size() / 4;
   desc.insert(desc.end(), {(int32_t)tpos, 0, 0, -1});
-  // stream units: runs of consecutive groups in task order (<= min(T, 32)
-  // groups and <= E_u edges, at least one group) that one worker streams as
-  // one contiguous index range, so its loads stay in flight across group and
-  // row boundaries.  E_u keeps >= ~256 units per SM for dynamic balance.
-  std::vector<int32_t> sunit{0};
-  {
-    const int64_t eu = std::max<int64_t>(32, std::min<int64_t>(512, p->nnz / (148 * 256)));
-    const int64_t gmax = std::min<int64_t>(p->T, 32);
-    int64_t cnt = 0, edges = 0;
-    for (int64_t gi = 0; gi < n_units; ++gi) {
-      const int64_t len = (int64_t)desc[(size_t)(gi + 1) * 4] - desc[(size_t)gi * 4];
-      if (cnt > 0 && (cnt == gmax || edges + len > eu)) {
-        sunit.push_back((int32_t)gi);
-        cnt = 0;
-        edges = 0;
-      }
-      ++cnt;
-      edges += len;
-    }
-    if (n_units > 0) sunit.push_back((int32_t)n_units);
-  }
-  // task position -> CSR position (explicit edge weights are indexed by CSR entry)
-  std::vector<int32_t> pos_t((size_t)p->nnz + 16, 0);
-  for (int64_t gi = 0; gi < n_units; ++gi) {
-    const int32_t tp = desc[(size_t)gi * 4], te = desc[(size_t)(gi + 1) * 4], b = desc[(size_t)gi * 4 + 1];
-    for (int32_t k = tp; k < te; ++k) pos_t[(size_t)k] = b + (k - tp);
-  }
   for (int64_t v = 0; v < n; ++v)
     if (p->rowptr[v + 1] == p->rowptr[v]) empty.push_back((int32_t)v);
   p->n_multi = (int64_t)multi_slot.size();
@@ -328,8 +301,6 @@ gnn_status build_schedule(gnn_plan_s *p) {
   p->dg.field = reinterpret_cast<decltype(p->dg.field)>(d);
   UP(desc, unit_desc)
   UP(colidx_t, colidx_t)
-  UP(sunit, sunit_beg)
-  UP(pos_t, pos_t)
   UP(multi_slot, multi_slot)
   UP(multi_units, multi_units)
   UP(multi_row, multi_row)
@@ -337,12 +308,11 @@ gnn_status build_schedule(gnn_plan_s *p) {
   UP(p->perm, perm)
 #undef UP
   p->dg.n_units = (int32_t)n_units;
-  p->dg.n_sunits = (int32_t)(sunit.size() - 1);
   p->dg.n_multi = (int32_t)p->n_multi;
   p->dg.n_empty = (int32_t)p->n_empty;
   p->dg.ng = (int32_t)ng;
   p->info.n_groups = (int64_t)p->grp_row.size();
-  p->info.n_tiles = (int64_t)(sunit.size() - 1);
+  p->info.n_tiles = n_units;  // work units (one per neighbour group)
   p->info.n_split_rows = p->n_multi;
   p->info.n_empty_rows = p->n_empty;
   return GNN_OK;

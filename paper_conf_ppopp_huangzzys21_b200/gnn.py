@@ -89,7 +89,6 @@ _SIGS = {
     "gnn_gemm_workspace_size": (_SZ, [_I64, _I32, _I32]),
     "gnn_set_gemm_impl": (ctypes.c_int, [ctypes.c_int]),
     "gnn_set_agg_mapping": (ctypes.c_int, [_I32, _I32, _I32]),
-    "gnn_set_agg_impl": (ctypes.c_int, [ctypes.c_int]),
     "gnn_gcn_layer": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _I64, _I32, _I32, _I32, _P, _I64, _P, _SZ, _P]),
     "gnn_gcn_aggregate_prescaled": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _I64, _I32, _P, _SZ, _P]),
     "gnn_gat_fold_weights": (ctypes.c_int, [_P, _P, _P, _I32, _I32, _I32, _P, _I64, _P]),
@@ -328,11 +327,6 @@ def gemm(X, W, row_scale=None, col_bias=None, relu=False, out=None, stream=None,
 
 def set_gemm_impl(impl: int) -> int:
     return _lib.gnn_set_gemm_impl(impl)
-
-
-def set_agg_impl(impl: int) -> int:
-    """0 = stream kernel (default), 1 = per-group kernel; returns the previous value."""
-    return _lib.gnn_set_agg_impl(impl)
 
 
 def set_agg_mapping(vec: int = 0, lanes: int = 0, nv: int = 0) -> None:

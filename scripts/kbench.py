@@ -233,67 +233,6 @@ def c1probe():
     print(plan.info, flush=True)
 
 
-def impls(cfg="C5"):
-    """v8 per-group kernel vs v10 stream kernel on the bench's three aggregations."""
-    t0 = time.time()
-    g = gs.config_graph(cfg)
-    print(f"{cfg}: n={g.n} nnz={g.nnz} gen {time.time() - t0:.1f}s", flush=True)
-    plan = G.Plan(g.rowptr, g.colidx, reorder=1)
-    print(f" plan: {plan.info}", flush=True)
-    X1 = torch.rand(g.n, 100, device="cuda")
-    Y1 = torch.empty_like(X1)
-    X2 = torch.rand(g.n, 256, device="cuda")
-    Y2 = torch.empty_like(X2)
-    Hh, Fh = 8, 32
-    Zs = torch.rand(g.n, Hh * Fh + 2 * Hh, device="cuda")
-    Yg = torch.empty(g.n, Hh * Fh, device="cuda")
-    t = Zs[:, Hh * Fh + Hh:]
-    res = {}
-    for impl in (1, 0, 1, 0):
-        G.set_agg_impl(impl)
-        a = timeit(lambda: G.aggregate(plan, X1, "sum", "gcn", out=Y1), iters=5, warm=2)
-        b = timeit(lambda: G.aggregate(plan, X2, "sum", "one", out=Y2), iters=5, warm=2)
-        c = timeit(lambda: G.gat_aggregate(plan, Zs, t, Hh, Fh, out=Yg), iters=5, warm=2)
-        outs = (Y1.clone(), Y2.clone(), Yg.clone())
-        if impl in res:
-            same = [bool(torch.equal(x, y)) for x, y in zip(outs, res[impl])]
-        else:
-            res[impl] = outs
-            same = None
-        print(f" impl={impl}: agg F=100 gcn {a:.3f} ms | sum F=256 {b:.3f} ms | GAT 8x32 {c:.3f} ms | rerun-identical {same}",
-              flush=True)
-    same = [bool(torch.equal(x, y)) for x, y in zip(res[0], res[1])]
-    print(f" v8 vs v10 bit-identical: {same}", flush=True)
-    G.set_agg_impl(0)
-
-
-def tiles(cfg="C5"):
-    """stream kernel vs max groups per unit (T): locality window vs per-unit overhead."""
-    g = gs.config_graph(cfg)
-    X1 = torch.rand(g.n, 100, device="cuda")
-    Y1 = torch.empty_like(X1)
-    X2 = torch.rand(g.n, 256, device="cuda")
-    Y2 = torch.empty_like(X2)
-    Hh, Fh = 8, 32
-    Zs = torch.rand(g.n, Hh * Fh + 2 * Hh, device="cuda")
-    Yg = torch.empty(g.n, Hh * Fh, device="cuda")
-    t = Zs[:, Hh * Fh + Hh:]
-    base = G.Plan(g.rowptr, g.colidx, reorder=1)
-    perm = base.export()[0]
-    del base
-    for T in [int(x) for x in os.environ.get("KB_TILES", "1,2,4,8,32").split(",")]:
-        plan = G.Plan(g.rowptr, g.colidx, reorder=1, tile_groups=T)
-        for impl in (0, 1) if T == 1 else (0,):
-            G.set_agg_impl(impl)
-            a = timeit(lambda: G.aggregate(plan, X1, "sum", "gcn", out=Y1), iters=5, warm=2)
-            b = timeit(lambda: G.aggregate(plan, X2, "sum", "one", out=Y2), iters=5, warm=2)
-            c = timeit(lambda: G.gat_aggregate(plan, Zs, t, Hh, Fh, out=Yg), iters=5, warm=2)
-            print(f" T={T} units={plan.info['n_tiles']} impl={impl}: agg F=100 gcn {a:.3f} ms | sum F=256 {b:.3f} ms"
-                  f" | GAT 8x32 {c:.3f} ms", flush=True)
-        G.set_agg_impl(0)
-        del plan
-
-
 def lstm_probe():
     """GraphSAGE-LSTM cell kernel on the C5 graph (for ncu / quick timing)."""
     g = gs.config_graph("C5")
@@ -326,10 +265,6 @@ if __name__ == "__main__":
     what = sys.argv[1] if len(sys.argv) > 1 else "gemm"
     if what == "gemm":
         gemm()
-    elif what == "tiles":
-        tiles(sys.argv[sys.argv.index("--cfg") + 1] if "--cfg" in sys.argv else "C5")
-    elif what == "impl":
-        impls(sys.argv[sys.argv.index("--cfg") + 1] if "--cfg" in sys.argv else "C5")
     elif what == "tune":
         tune()
     elif what == "lstm":

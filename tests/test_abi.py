@@ -178,9 +178,7 @@ def test_new_entry_points_reject_null_plans():
     assert g.gnn_workspace_size(None, 6, 0, 64, 8) == 0
 
 
-def test_lstm_and_agg_impl_switches_roundtrip():
+def test_lstm_impl_switch_roundtrip():
     g = P.gnn
     old = g.gnn_set_lstm_impl(1)
     assert g.gnn_set_lstm_impl(old) == 1
-    old = g.gnn_set_agg_impl(0)
-    assert g.gnn_set_agg_impl(old) == 0

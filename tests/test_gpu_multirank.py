@@ -68,6 +68,7 @@ def test_two_ranks_bit_identical_to_one_and_oracle():
     m1 = RowPartitionedGCNGAT(g.rowptr, g.colidx, W1, W2, W3, a_s, a_d, Hh, Fh, reorder=0)
     m1.load_input(torch.from_numpy(X), non_blocking=False)
     Y1 = m1.step().cpu().numpy()
+    L1, L2 = m1.Y1.cpu().numpy(), m1.Y2.cpu().numpy()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _port()
@@ -79,10 +80,13 @@ def test_two_ranks_bit_identical_to_one_and_oracle():
         p.join(timeout=120)
     assert not isinstance(Y2, str), Y2
     assert np.array_equal(Y1.view(np.uint32), Y2.view(np.uint32))
-    # P = 1 vs the oracle, layer by layer definitions composed in fp64 on sampled rows
+    # P = 1 vs the oracle layer by layer on sampled rows, each layer fed the
+    # GPU's own input to it, at the north_star tolerance (R11)
     rows = np.sort(np.random.default_rng(0).choice(g.n, 300, replace=False))
-    Y1o = oracle.gcn_layer(g.rowptr, g.colidx, X, W1, relu=True)
-    Y2o = oracle.gcn_layer(g.rowptr, g.colidx, Y1o, W2, relu=False)
-    Y3o = oracle.gat_layer(g.rowptr, g.colidx, Y2o, W3, a_s, a_d, Hh, Fh, 0.2, rows=rows)
-    err = np.abs(Y1[rows].astype(np.float64) - Y3o)
-    assert np.all(err <= 1e-4 + 1e-3 * np.abs(Y3o)), err.max()  # three layers compose: looser, see DESIGN R11
+    tol = lambda r: 1e-5 + 1e-4 * np.abs(r)  # noqa: E731
+    r1 = oracle.gcn_layer(g.rowptr, g.colidx, X, W1, relu=True, rows=rows)
+    assert np.all(np.abs(L1[rows] - r1.astype(np.float64)) <= tol(r1)), "layer 1"
+    r2 = oracle.gcn_layer(g.rowptr, g.colidx, L1, W2, relu=False, rows=rows)
+    assert np.all(np.abs(L2[rows] - r2.astype(np.float64)) <= tol(r2)), "layer 2"
+    r3 = oracle.gat_layer(g.rowptr, g.colidx, L2, W3, a_s, a_d, Hh, Fh, 0.2, rows=rows)
+    assert np.all(np.abs(Y1[rows] - r3.astype(np.float64)) <= tol(r3)), "layer 3"
