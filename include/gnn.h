@@ -124,6 +124,31 @@ gnn_status gnn_plan_create_ex(int64_t n, int64_t n_src, int64_t nnz,
                               const int32_t *src_degree_h,
                               const gnn_plan_opts *opts, gnn_plan_t *out);
 
+/*
+ * As gnn_plan_create_ex with the task order given instead of computed:
+ * perm_h int32[n] must be a permutation of [0, n) (else GNN_ERR_INVALID_ARG);
+ * opts->reorder is recorded but LAS does not run.  For schedules computed
+ * offline and reused.
+ */
+gnn_status gnn_plan_create_perm(int64_t n, int64_t n_src, int64_t nnz,
+                                const int64_t *rowptr_h, const int32_t *colidx_h,
+                                const int32_t *src_degree_h, const int32_t *perm_h,
+                                const gnn_plan_opts *opts, gnn_plan_t *out);
+
+/*
+ * Plan persistence (LAS runs once offline and is reused).
+ * gnn_plan_save writes the CSR, the source out-degrees, the options and the
+ * task order to `path` (with_las != 0 also writes the LAS intermediates
+ * exported by gnn_plan_export_las); a checksum covers the file.
+ * gnn_plan_load rebuilds the device plan on the current device from such a
+ * file without rerunning LAS: the task order, the normalisers and every
+ * result computed with the loaded plan are identical to the saved plan's.
+ * Errors: GNN_ERR_INVALID_ARG for an unreadable, truncated, corrupt or foreign
+ * file (*out = NULL); GNN_ERR_INTERNAL if writing fails.  Synchronous.
+ */
+gnn_status gnn_plan_save(gnn_plan_t plan, const char *path, int32_t with_las);
+gnn_status gnn_plan_load(const char *path, gnn_plan_t *out);
+
 gnn_status gnn_plan_get_info(gnn_plan_t plan, gnn_plan_info *info);
 
 /*

@@ -98,10 +98,16 @@ void gnn_plan_opts_default(gnn_plan_opts *o) {
   o->seed = 0;
 }
 
-gnn_status gnn_plan_create_ex(int64_t n, int64_t n_src, int64_t nnz, const int64_t *rowptr_h,
-                              const int32_t *colidx_h, const int32_t *src_degree_h,
-                              const gnn_plan_opts *opts_in, gnn_plan_t *out) {
-  GNN_TRY({
+}  // extern "C"
+
+namespace gnn {
+// Plan construction shared by gnn_plan_create_ex (perm_h == NULL: LAS or the
+// identity order per opts) and gnn_plan_create_perm / gnn_plan_load (the task
+// order given, e.g. a LAS schedule computed offline).
+gnn_status create_plan(int64_t n, int64_t n_src, int64_t nnz, const int64_t *rowptr_h, const int32_t *colidx_h,
+                       const int32_t *src_degree_h, const int32_t *perm_h, const gnn_plan_opts *opts_in,
+                       gnn_plan_t *out) {
+  {
     if (!out) return check(false, "out is NULL");
     *out = nullptr;
     auto t0 = std::chrono::steady_clock::now();
@@ -194,6 +200,7 @@ gnn_status gnn_plan_create_ex(int64_t n, int64_t n_src, int64_t nnz, const int64
     p->dg.colidx = (const int32_t *)d_colidx;
     p->dg.nsrc = (const float *)d_nsrc;
     p->dg.ndst = (const float *)d_ndst;
+    p->d_dout = (const int32_t *)d_dout;
     p->info.ms_upload = ms_since(t0);
     // a1: degrees + normalisers on the GPU
     t0 = std::chrono::steady_clock::now();
@@ -204,7 +211,20 @@ gnn_status gnn_plan_create_ex(int64_t n, int64_t n_src, int64_t nnz, const int64
     if (e != cudaSuccess) return fail(cuda_status(e, "degrees"));
     p->info.ms_degrees = ms_since(t0);
     // a2: locality-aware task scheduling
-    if (opts.reorder && n > 0) {
+    if (perm_h) {
+      // given task order: must be a permutation of [0, n)
+      std::vector<uint8_t> seen((size_t)n, 0);
+      for (int64_t i = 0; i < n; ++i) {
+        const int32_t v = perm_h[i];
+        if (v < 0 || v >= n || seen[(size_t)v]) {
+          set_error("perm is not a permutation of [0, n) (entry " + std::to_string(i) + ")");
+          return fail(GNN_ERR_INVALID_ARG);
+        }
+        seen[(size_t)v] = 1;
+      }
+      p->perm.assign(perm_h, perm_h + n);
+      p->n_clusters = 0;
+    } else if (opts.reorder && n > 0) {
       t0 = std::chrono::steady_clock::now();
       const int32_t K = opts.minhash_k;
       uint64_t *d_sig = nullptr;
@@ -247,6 +267,24 @@ gnn_status gnn_plan_create_ex(int64_t n, int64_t n_src, int64_t nnz, const int64
     p->info.reorder = opts.reorder;
     *out = p;
     return GNN_OK;
+  }
+}
+}  // namespace gnn
+
+extern "C" {
+
+gnn_status gnn_plan_create_ex(int64_t n, int64_t n_src, int64_t nnz, const int64_t *rowptr_h,
+                              const int32_t *colidx_h, const int32_t *src_degree_h,
+                              const gnn_plan_opts *opts_in, gnn_plan_t *out) {
+  GNN_TRY({ return create_plan(n, n_src, nnz, rowptr_h, colidx_h, src_degree_h, nullptr, opts_in, out); })
+}
+
+gnn_status gnn_plan_create_perm(int64_t n, int64_t n_src, int64_t nnz, const int64_t *rowptr_h,
+                                const int32_t *colidx_h, const int32_t *src_degree_h, const int32_t *perm_h,
+                                const gnn_plan_opts *opts_in, gnn_plan_t *out) {
+  GNN_TRY({
+    if (!perm_h && n > 0) return check(false, "perm_h is NULL");
+    return create_plan(n, n_src, nnz, rowptr_h, colidx_h, src_degree_h, perm_h, opts_in, out);
   })
 }
 
@@ -271,8 +309,9 @@ gnn_status gnn_plan_export(gnn_plan_t p, int32_t *perm_h, int32_t *grp_row_h, in
 
 gnn_status gnn_plan_export_las(gnn_plan_t p, uint64_t *sig_h, int32_t *pairs_h, int32_t *cluster_of_h) {
   if (!p) return check(false, "plan is NULL");
-  if (!p->opts.reorder) {
-    set_error("plan was built without reorder");
+  if (!p->opts.reorder || p->sig.empty()) {
+    set_error(p->opts.reorder ? "plan has no LAS intermediates (given order, or loaded without them)"
+                              : "plan was built without reorder");
     return GNN_ERR_INVALID_ARG;
   }
   if (sig_h) std::memcpy(sig_h, p->sig.data(), sizeof(uint64_t) * p->sig.size());

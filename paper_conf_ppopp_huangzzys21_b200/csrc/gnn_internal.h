@@ -73,6 +73,7 @@ struct gnn_plan_s {
   // (tuned_vec == 0: none)
   int32_t tuned_F = 0, tuned_vec = 0, tuned_lanes = 0, tuned_nv = 0;
   gnn::DevGraph dg{};
+  const int32_t *d_dout = nullptr;  // device source out-degrees (counted or the override)
 };
 
 namespace gnn {
@@ -81,6 +82,10 @@ namespace gnn {
 void set_error(const std::string &msg);
 gnn_status cuda_status(cudaError_t e, const char *what);
 void count_launch(uint64_t k = 1);
+
+gnn_status create_plan(int64_t n, int64_t n_src, int64_t nnz, const int64_t *rowptr_h, const int32_t *colidx_h,
+                       const int32_t *src_degree_h, const int32_t *perm_h, const gnn_plan_opts *opts_in,
+                       gnn_plan_t *out);
 
 // planner (plan.cpp) — host side
 gnn_status build_schedule(gnn_plan_s *p);

@@ -73,6 +73,10 @@ _SIGS = {
     "gnn_plan_create": (ctypes.c_int, [_I64, _I64, _P, _P, ctypes.POINTER(gnn_plan_opts), ctypes.POINTER(_P)]),
     "gnn_plan_create_ex": (ctypes.c_int, [_I64, _I64, _I64, _P, _P, _P, ctypes.POINTER(gnn_plan_opts),
                                           ctypes.POINTER(_P)]),
+    "gnn_plan_create_perm": (ctypes.c_int, [_I64, _I64, _I64, _P, _P, _P, _P, ctypes.POINTER(gnn_plan_opts),
+                                            ctypes.POINTER(_P)]),
+    "gnn_plan_save": (ctypes.c_int, [_P, ctypes.c_char_p, _I32]),
+    "gnn_plan_load": (ctypes.c_int, [ctypes.c_char_p, ctypes.POINTER(_P)]),
     "gnn_plan_get_info": (ctypes.c_int, [_P, ctypes.POINTER(gnn_plan_info)]),
     "gnn_plan_export": (ctypes.c_int, [_P, _P, _P, _P]),
     "gnn_plan_export_las": (ctypes.c_int, [_P, _P, _P, _P]),
@@ -178,7 +182,9 @@ def default_opts(**kw) -> gnn_plan_opts:
 class Plan:
     """Owns a gnn_plan_t built from a host CSR (numpy int64 rowptr, int32 colidx)."""
 
-    def __init__(self, rowptr, colidx, n_src=None, src_degree=None, **opts):
+    def __init__(self, rowptr, colidx, n_src=None, src_degree=None, perm=None, **opts):
+        """gnn_plan_create_ex, or gnn_plan_create_perm when a task order `perm`
+        (e.g. a LAS schedule computed earlier) is given."""
         rowptr = np.ascontiguousarray(rowptr, dtype=np.int64)
         colidx = np.ascontiguousarray(colidx, dtype=np.int32)
         self.n = len(rowptr) - 1
@@ -187,10 +193,32 @@ class Plan:
         self.opts = default_opts(**opts)
         h = ctypes.c_void_p()
         sd = None if src_degree is None else np.ascontiguousarray(src_degree, dtype=np.int32)
-        _call("gnn_plan_create_ex", self.n, self.n_src, self.nnz, _np_ptr(rowptr), _np_ptr(colidx), _np_ptr(sd),
-              ctypes.byref(self.opts), ctypes.byref(h))
+        if perm is None:
+            _call("gnn_plan_create_ex", self.n, self.n_src, self.nnz, _np_ptr(rowptr), _np_ptr(colidx), _np_ptr(sd),
+                  ctypes.byref(self.opts), ctypes.byref(h))
+        else:
+            pm = np.ascontiguousarray(perm, dtype=np.int32)
+            _call("gnn_plan_create_perm", self.n, self.n_src, self.nnz, _np_ptr(rowptr), _np_ptr(colidx),
+                  _np_ptr(sd), _np_ptr(pm), ctypes.byref(self.opts), ctypes.byref(h))
         self.handle = h
         self._ws = {}
+
+    @classmethod
+    def load(cls, path):
+        """gnn_plan_load: a plan saved by Plan.save (no LAS rerun)."""
+        self = cls.__new__(cls)
+        h = ctypes.c_void_p()
+        _call("gnn_plan_load", os.fsencode(path), ctypes.byref(h))
+        self.handle = h
+        self._ws = {}
+        i = self.info
+        self.n, self.n_src, self.nnz = i["n"], i["n_src"], i["nnz"]
+        self.opts = default_opts(reorder=i["reorder"])
+        return self
+
+    def save(self, path, with_las=False):
+        """gnn_plan_save: CSR, degrees, task order (+ LAS intermediates)."""
+        _call("gnn_plan_save", self.handle, os.fsencode(path), int(with_las))
 
     @property
     def info(self) -> dict:

@@ -182,3 +182,15 @@ def test_lstm_impl_switch_roundtrip():
     g = P.gnn
     old = g.gnn_set_lstm_impl(1)
     assert g.gnn_set_lstm_impl(old) == 1
+
+
+def test_plan_load_rejects_missing_and_foreign_files(tmp_path):
+    """gnn_plan_load validates the file on the host before any device work."""
+    h = ctypes.c_void_p()
+    assert P.gnn.gnn_plan_load(str(tmp_path / "none").encode(), ctypes.byref(h)) == 1
+    assert h.value is None
+    f = tmp_path / "foreign"
+    f.write_bytes(b"NOTAPLAN" + bytes(100))
+    assert P.gnn.gnn_plan_load(str(f).encode(), ctypes.byref(h)) == 1
+    assert "not a gnn plan" in P.gnn.gnn_last_error()
+    assert P.gnn.gnn_plan_save(None, b"/tmp/x", 0) == 1
