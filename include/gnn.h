@@ -228,9 +228,25 @@ gnn_status gnn_gat_aggregate(gnn_plan_t plan, const float *Zs, int64_t ldz,
                              void *ws, size_t ws_bytes, gnn_stream_t stream);
 
 /*
- * Full GAT layer: Z = X W (W: [f_in, H*Fh] row-major), s = Z_h . a_src_h,
- * t = Z_h . a_dst_h (computed as extra GEMM columns X (W_h a_h)), then
- * gnn_gat_aggregate.  Requires n_src == n.  Workspace from
+ * GAT transform (a5 for Table 2's GAT; reading R5): Zst rows =
+ * [z_v | s_v | t_v] with z = X W (W: [f_in, ldw >= H*Fh] row-major), s_v[h] =
+ * <z_v[h], a_src_h>, t_v[h] = <z_v[h], a_dst_h>.  Heads of a multiple of 32
+ * features: one tcgen05 3xTF32 GEMM of H*Fh columns whose epilogue
+ * accumulates s and t from the stored z (fp32, head order); other head sizes
+ * fold the scores into extra GEMM columns X (W_h a_h) (needs ldw == H*Fh and
+ * ldz >= round_up(H*Fh + 2H, 8)).  X: [m, ldx]; Zst: [m, ldz], ldz >= H*Fh + 2H.
+ * Workspace: gnn_gat_transform_workspace_size(m, f_in, H, Fh) bytes, 256-byte
+ * aligned.
+ */
+gnn_status gnn_gat_transform(const float *X, int64_t ldx, int64_t m, int32_t f_in, const float *W,
+                             int64_t ldw, const float *a_src, const float *a_dst, int32_t H,
+                             int32_t Fh, float *Zst, int64_t ldz, void *ws, size_t ws_bytes,
+                             gnn_stream_t stream);
+size_t gnn_gat_transform_workspace_size(int64_t m, int32_t f_in, int32_t H, int32_t Fh);
+
+/*
+ * Full GAT layer: [Z | s | t] by gnn_gat_transform, then gnn_gat_aggregate.
+ * W: [f_in, H*Fh] row-major.  Requires n_src == n.  Workspace from
  * gnn_workspace_size(plan, GNN_OP_GAT_LAYER, f_in, H * Fh, H).
  */
 gnn_status gnn_gat_layer(gnn_plan_t plan, const float *X, int64_t ldx, int32_t f_in,

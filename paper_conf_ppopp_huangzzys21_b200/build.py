@@ -36,25 +36,30 @@ def _headers():
                   [os.path.join(ROOT, "include", "gnn.h")])
 
 
-def _digest(path, hdr_digest):
+def _digest(path, hdr_digest, extra=()):
     h = hashlib.sha1(open(path, "rb").read())
     h.update(hdr_digest)
-    h.update(" ".join(ARCH + FLAGS).encode())
+    h.update(" ".join(ARCH + FLAGS + list(extra)).encode())
     return h.hexdigest()[:16]
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    os.makedirs(BUILD, exist_ok=True)
+def build(force: bool = False, verbose: bool = False, extra=(), out: str = None) -> str:
+    """Build libgnn.so; `extra` nvcc flags (e.g. -DGNN_AGG_MINB=5) and `out`
+    build an A/B variant library elsewhere (load it with GNN_LIB_PATH)."""
+    extra = list(extra)
+    so = out or SO
+    build_dir = BUILD if not extra else os.path.join(BUILD, "v_" + hashlib.sha1(" ".join(extra).encode()).hexdigest()[:8])
+    os.makedirs(build_dir, exist_ok=True)
     hd = hashlib.sha1()
     for hpath in _headers():
         hd.update(open(hpath, "rb").read())
     hdr = hd.digest()
     objs, jobs = [], []
     for src in _sources():
-        obj = os.path.join(BUILD, os.path.basename(src) + "." + _digest(src, hdr) + ".o")
+        obj = os.path.join(build_dir, os.path.basename(src) + "." + _digest(src, hdr, extra) + ".o")
         objs.append(obj)
         if force or not os.path.exists(obj):
-            cmd = [NVCC, *ARCH, *FLAGS, "-c", src, "-o", obj + ".tmp"]
+            cmd = [NVCC, *ARCH, *FLAGS, *extra, "-c", src, "-o", obj + ".tmp"]
             if verbose and src.endswith(".cu"):
                 cmd.insert(1, "-Xptxas=-v")
             jobs.append((cmd, obj))
@@ -73,23 +78,27 @@ def build(force: bool = False, verbose: bool = False) -> str:
                 if verbose and out:
                     sys.stderr.write(out)
     link_stamp = hashlib.sha1("".join(objs).encode()).hexdigest()[:16]
-    stamp_file = SO + ".stamp"
-    if force or not os.path.exists(SO) or not os.path.exists(stamp_file) or open(stamp_file).read() != link_stamp:
-        tmp = SO + f".tmp{os.getpid()}"
+    stamp_file = so + ".stamp"
+    if force or not os.path.exists(so) or not os.path.exists(stamp_file) or open(stamp_file).read() != link_stamp:
+        os.makedirs(os.path.dirname(os.path.abspath(so)), exist_ok=True)
+        tmp = so + f".tmp{os.getpid()}"
         cmd = [NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-cudart", "static", "-lpthread"]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"link failed:\n{r.stderr}")
-        os.replace(tmp, SO)
+        os.replace(tmp, so)
         with open(stamp_file, "w") as f:
             f.write(link_stamp)
     # drop stale objects
     keep = set(objs)
-    for o in glob.glob(os.path.join(BUILD, "*.o")):
+    for o in glob.glob(os.path.join(build_dir, "*.o")):
         if o not in keep:
             os.remove(o)
-    return SO
+    return so
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose="--verbose" in sys.argv))
+    args = sys.argv[1:]
+    out = args[args.index("--out") + 1] if "--out" in args else None
+    extra = [a for a in args if a.startswith("-D")]
+    print(build(force="--force" in args, verbose="--verbose" in args, extra=extra, out=out))

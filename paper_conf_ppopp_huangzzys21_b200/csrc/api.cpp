@@ -1,5 +1,6 @@
 // api.cpp — the C-ABI of libgnn.so (include/gnn.h): validation, plan
 // lifetime, dispatch to the sm_100a kernels.  No exception crosses the ABI.
+#include <algorithm>
 #include <atomic>
 #include <chrono>
 #include <climits>
@@ -334,12 +335,19 @@ gnn_status gnn_plan_destroy(gnn_plan_t p) {
   })
 }
 
-// layer workspaces: [GEMM W image][layer buffers][aggregation workspace]
+// GAT transform workspace: the tensor-core W image of the H*Fh-column GEMM
+// with the score epilogue, or (heads not a multiple of 32 wide) the folded
+// weights [W | W a_src | W a_dst] and the W image of that wider GEMM
+static size_t ws_gat_transform(int64_t m, int32_t f_in, int32_t H, int32_t Fh) {
+  const int32_t ld = ((H * Fh + 2 * H) + 7) / 8 * 8;
+  const size_t fold = align256(gemm_tc_workspace(m, f_in, ld)) + align256(sizeof(float) * (size_t)f_in * ld);
+  return std::max(align256(gemm_tc_workspace(m, f_in, H * Fh)), fold);
+}
+// layer workspaces: [transform workspace][layer buffers][aggregation workspace]
 static size_t ws_gat_layer_head(int64_t n, int32_t f_in, int32_t HF, int32_t H, int32_t *ldwe) {
   const int32_t ld = ((HF + 2 * H) + 7) / 8 * 8;
   if (ldwe) *ldwe = ld;
-  return align256(gemm_tc_workspace(n, f_in, ld)) + align256(sizeof(float) * (size_t)f_in * ld) +
-         align256(sizeof(float) * (size_t)n * ld);
+  return ws_gat_transform(n, f_in, H, HF / H) + align256(sizeof(float) * (size_t)n * ld);
 }
 static size_t ws_edgeconv_head(int64_t n, int32_t f_in, int32_t f_out) {
   const size_t ld = 2 * (size_t)f_out;
@@ -476,6 +484,67 @@ gnn_status gnn_set_agg_mapping(int32_t vec, int32_t lanes, int32_t nv) {
   })
 }
 
+}  // extern "C"
+
+namespace gnn {
+// [Z | s | t] = X W with s[h] = Z_h . a_src_h, t[h] = Z_h . a_dst_h (Table 2
+// GAT, reading R5).  Heads of a multiple of 32 features: one
+// tensor-core GEMM of H*Fh columns whose epilogue accumulates the scores from
+// the Z values it stores.  Otherwise the scores are extra GEMM columns of the
+// folded weights [W | W_h a_src_h | W_h a_dst_h] (a reassociation of Z a).
+static gnn_status gat_transform(const float *X, int64_t ldx, int64_t m, int32_t f_in, const float *W, int64_t ldw,
+                                const float *a_src, const float *a_dst, int32_t H, int32_t Fh, float *Zst,
+                                int64_t ldz, void *ws, size_t ws_bytes, cudaStream_t s) {
+  if (m == 0) return GNN_OK;
+  if (ws_bytes < ws_gat_transform(m, f_in, H, Fh)) {
+    set_error("gat transform workspace too small: need " + std::to_string(ws_gat_transform(m, f_in, H, Fh)));
+    return GNN_ERR_WORKSPACE;
+  }
+  const int32_t HF = H * Fh;
+  cudaError_t e = launch_gemm_att(X, ldx, W, ldw, Zst, ldz, m, f_in, H, Fh, a_src, a_dst, ws, ws_bytes, s);
+  if (e == cudaSuccess) return GNN_OK;
+  if (e != cudaErrorNotSupported) return cuda_status(e, "gat transform");
+  (void)cudaGetLastError();
+  const int32_t ld = ((HF + 2 * H) + 7) / 8 * 8;
+  if (ldw != HF) {
+    set_error("gat transform: the folded path needs ldw == H * Fh");
+    return GNN_ERR_UNSUPPORTED;
+  }
+  const size_t gws = align256(gemm_tc_workspace(m, f_in, ld));
+  float *Wext = (float *)((char *)ws + gws);
+  e = launch_gat_weights(W, a_src, a_dst, f_in, H, Fh, Wext, ld, s);
+  if (e != cudaSuccess) return cuda_status(e, "gat weights");
+  // the folded GEMM writes ld >= HF + 2H columns: stage through Zst only if it is wide enough
+  if (ldz < ld) {
+    set_error("gat transform: ldz must be >= round_up(H*Fh + 2H, 8) for this head size");
+    return GNN_ERR_INVALID_ARG;
+  }
+  return launch_gemm(X, ldx, Wext, ld, Zst, ldz, m, f_in, ld, nullptr, nullptr, 0, ws, gws, s);
+}
+}  // namespace gnn
+
+extern "C" {
+
+size_t gnn_gat_transform_workspace_size(int64_t m, int32_t f_in, int32_t H, int32_t Fh) {
+  if (m < 0 || f_in < 1 || H < 1 || Fh < 1) return 0;
+  return ws_gat_transform(m, f_in, H, Fh);
+}
+
+gnn_status gnn_gat_transform(const float *X, int64_t ldx, int64_t m, int32_t f_in, const float *W, int64_t ldw,
+                             const float *a_src, const float *a_dst, int32_t H, int32_t Fh, float *Zst, int64_t ldz,
+                             void *ws, size_t ws_bytes, gnn_stream_t stream) {
+  GNN_TRY({
+    if (m < 0 || f_in < 1 || H < 1 || H > 256 || Fh < 1) return check(false, "bad GAT transform sizes");
+    if (m > 0 && (!X || !W || !a_src || !a_dst || !Zst || !ws)) return check(false, "NULL argument");
+    if (ldx < f_in || ldw < (int64_t)H * Fh || ldz < (int64_t)H * Fh + 2 * H)
+      return check(false, "leading dimension too small (ldz >= H*Fh + 2H)");
+    if (overlaps(Zst, span_bytes(m, ldz, (int64_t)H * Fh + 2 * H), X, span_bytes(m, ldx, f_in)))
+      return check(false, "Zst overlaps X");
+    return gat_transform(X, ldx, m, f_in, W, ldw, a_src, a_dst, H, Fh, Zst, ldz, ws, ws_bytes,
+                         (cudaStream_t)stream);
+  })
+}
+
 gnn_status gnn_gat_layer(gnn_plan_t p, const float *X, int64_t ldx, int32_t f_in, const float *W,
                          const float *a_src, const float *a_dst, int32_t H, int32_t Fh, float neg_slope,
                          float *Y, int64_t ldy, void *ws, size_t ws_bytes, gnn_stream_t stream) {
@@ -494,14 +563,11 @@ gnn_status gnn_gat_layer(gnn_plan_t p, const float *X, int64_t ldx, int32_t f_in
       return GNN_ERR_WORKSPACE;
     }
     char *base = (char *)ws;
-    const size_t gws = align256(gemm_tc_workspace(p->n, f_in, ldwe));
-    float *Wext = (float *)(base + gws);
-    float *Zst = (float *)(base + gws + align256(sizeof(float) * (size_t)f_in * ldwe));
+    const size_t tws = ws_gat_transform(p->n, f_in, H, Fh);
+    float *Zst = (float *)(base + tws);
     cudaStream_t s = (cudaStream_t)stream;
-    // [Z | s | t]: the scores as extra GEMM columns X (W_h a_h) (R5)
-    cudaError_t e = launch_gat_weights(W, a_src, a_dst, f_in, H, Fh, Wext, ldwe, s);
-    if (e != cudaSuccess) return cuda_status(e, "gat weights");
-    gnn_status st = launch_gemm(X, ldx, Wext, ldwe, Zst, ldwe, p->n, f_in, ldwe, nullptr, nullptr, 0, base, gws, s);
+    // [Z | s | t] (R5)
+    gnn_status st = gat_transform(X, ldx, p->n, f_in, W, HF, a_src, a_dst, H, Fh, Zst, ldwe, base, tws, s);
     if (st != GNN_OK) return st;
     AggArgs a{};
     a.mode = 3;

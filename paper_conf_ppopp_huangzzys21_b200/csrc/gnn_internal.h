@@ -155,6 +155,9 @@ gnn_status launch_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw,
                        int64_t ldh, int64_t m, int32_t k, int32_t n, const float *row_scale,
                        const float *col_bias, int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s);
 size_t gemm_tc_workspace(int64_t m, int32_t k, int32_t n);
+cudaError_t launch_gemm_att(const float *X, int64_t ldx, const float *W, int64_t ldw, float *Z, int64_t ldz, int64_t m,
+                            int32_t k, int32_t H, int32_t Fh, const float *a_src, const float *a_dst, void *ws,
+                            size_t ws_bytes, cudaStream_t s);
 int set_gemm_impl(int impl);
 
 // small helper kernels (k_graph.cu)

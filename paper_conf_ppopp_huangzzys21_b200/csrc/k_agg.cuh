@@ -77,21 +77,36 @@ struct KParams {
   int32_t n_persist;  // persistent CTAs
 };
 
+// Cache policy of the three streams (A/B switches, compile time):
+//   GNN_LD_NA  gathered source rows bypass L1 allocation (L1 keeps the
+//              kernel's local memory; the rows are reused through L2)
+//   GNN_EF     the task-ordered index stream is loaded and the output rows are
+//              stored evict-first (.cs), so they do not push the reused
+//              source rows out of L2
+#ifndef GNN_LD_NA
+#define GNN_LD_NA 1
+#endif
+#ifndef GNN_EF
+#define GNN_EF 1
+#endif
+#if GNN_LD_NA
+#define GNN_LDNC "ld.global.nc.L1::no_allocate"
+#else
+#define GNN_LDNC "ld.global.nc"
+#endif
 template <int VEC>
 __device__ __forceinline__ void ldv(const float *p, float (&v)[VEC]) {
   if constexpr (VEC == 8) {
-    asm volatile("ld.global.nc.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-                 : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3]), "=f"(v[4]), "=f"(v[5]),
-                   "=f"(v[6]), "=f"(v[7])
+    asm volatile(GNN_LDNC ".v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3]), "=f"(v[4]), "=f"(v[5]), "=f"(v[6]),
+                   "=f"(v[7])
                  : "l"(p));
   } else if constexpr (VEC == 4) {
-    float4 x = __ldg(reinterpret_cast<const float4 *>(p));
-    v[0] = x.x; v[1] = x.y; v[2] = x.z; v[3] = x.w;
+    asm volatile(GNN_LDNC ".v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3]) : "l"(p));
   } else if constexpr (VEC == 2) {
-    float2 x = __ldg(reinterpret_cast<const float2 *>(p));
-    v[0] = x.x; v[1] = x.y;
+    asm volatile(GNN_LDNC ".v2.f32 {%0,%1}, [%2];" : "=f"(v[0]), "=f"(v[1]) : "l"(p));
   } else {
-    v[0] = __ldg(p);
+    asm volatile(GNN_LDNC ".f32 %0, [%1];" : "=f"(v[0]) : "l"(p));
   }
 }
 
@@ -110,10 +125,35 @@ __device__ __forceinline__ void stv(float *p, const float (&v)[VEC]) {
   }
 }
 
+// output rows: written once, read by the next kernel (evict-first in L2, GNN_EF)
+template <int VEC>
+__device__ __forceinline__ void stv_out(float *p, const float (&v)[VEC]) {
+#if GNN_EF
+  if constexpr (VEC == 8) {
+    asm volatile("st.global.cs.v8.f32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "f"(v[0]), "f"(v[1]),
+                 "f"(v[2]), "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]), "f"(v[7])
+                 : "memory");
+  } else if constexpr (VEC == 4) {
+    asm volatile("st.global.cs.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(p), "f"(v[0]), "f"(v[1]), "f"(v[2]), "f"(v[3])
+                 : "memory");
+  } else if constexpr (VEC == 2) {
+    asm volatile("st.global.cs.v2.f32 [%0], {%1,%2};" ::"l"(p), "f"(v[0]), "f"(v[1]) : "memory");
+  } else {
+    asm volatile("st.global.cs.f32 [%0], %1;" ::"l"(p), "f"(v[0]) : "memory");
+  }
+#else
+  stv<VEC>(p, v);
+#endif
+}
+
 // streaming index load: read once, do not keep in L1
 __device__ __forceinline__ int32_t ld_stream_i32(const int32_t *p) {
   int32_t r;
+#if GNN_EF
+  asm volatile("ld.global.cs.nc.s32 %0, [%1];" : "=r"(r) : "l"(p));  // evict-first in L2
+#else
   asm volatile("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(r) : "l"(p));
+#endif
   return r;
 }
 __device__ __forceinline__ float ld_stream_f32(const float *p) {
@@ -237,7 +277,7 @@ __device__ __forceinline__ void store_row(const KParams &p, int32_t row, int32_t
     if (p.add_row) ldv<VEC>(p.add_row + (int64_t)row * p.ld_add + f, addv);
 #pragma unroll
     for (int i = 0; i < VEC; ++i) y[i] = epi(p, p.mode, P.a[n][i], P.l[n], ndst, deg_f, p.add_row ? &addv[i] : nullptr);
-    stv<VEC>(p.Y + (int64_t)row * p.ldy + f, y);
+    stv_out<VEC>(p.Y + (int64_t)row * p.ldy + f, y);
   }
 }
 

@@ -57,7 +57,7 @@ constexpr int EPI_WARP1 = 11;         // TMA path: second epilogue half (warps 1
 constexpr int THREADS_TMA = 32 * 15;
 __host__ __device__ constexpr int threads_of(bool tma) { return tma ? THREADS_TMA : THREADS; }
 constexpr int TILE_A_BYTES = BM * BK * 4;  // 16 KB per hi or lo
-constexpr int MAX_STAGES = 6;
+constexpr int MAX_STAGES = 8;
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
@@ -181,13 +181,21 @@ struct TcParams {
   int32_t k, n, np, npa;  // np = n rounded to 16; npa = TMEM columns per accumulator
   int32_t num_kb, num_tiles;
   int32_t stages, n_acc, n_buf;
-  int32_t sa, sb;  // TMA path: A (X hi/lo) ring and B (W image) ring depths
+  int32_t sa, sb;  // TMA path: raw X ring (TMA destination, the A_hi operand) and B (W image) ring depths
+  int32_t sl;      // TMA path: X_lo ring depth (written by the splitters)
   int32_t eb;      // TMA path with TMA stores: 4 KB staging buffers per epilogue warp (1 or 2)
   int32_t ncb, cbw0;  // TMA path: column blocks per row tile (1 or 2) and block 0's width
   int32_t epi8;    // TMA stores with 8 epilogue warps (two per TMEM lane quadrant, alternate column chunks)
   const float *row_scale;
   const float *col_bias;
   int32_t relu;
+  // attention-score epilogue (GAT, Table 2; reading R5): when att
+  // is set, the epilogue also writes s_v[h] = <y_v[h*Fh : (h+1)*Fh], a_src_h>
+  // and t_v[h] = <y_v[h], a_dst_h> (att_dst) to columns att_col + h and
+  // att_col + att_H + h of H.  Fh is a multiple of 32, so every 32-column
+  // chunk belongs to one head, and each thread's chunks are contiguous.
+  const float *att, *att_dst;
+  int32_t att_H, att_Fh, att_col;
 };
 
 template <bool VEC_X, bool VEC_H, bool TMA_X>
@@ -198,11 +206,13 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
   const int NP = p.np;
   const int B_BYTES = NP * 128;
   const int STAGE_BYTES = 2 * TILE_A_BYTES + 2 * B_BYTES;
-  // register path: full/empty per unified stage [A | B].  TMA path: separate
-  // rings -- A: xfull (TMA bytes) -> afull (splitters) -> aempty (MMA);
-  // B: full (bulk bytes) -> empty (MMA)
+  // register path: full/empty per unified stage [A | B].  TMA path: three
+  // rings -- raw X: xfull (TMA bytes) -> aempty (MMA; the raw tile is the
+  // A_hi operand: kind::tf32 reads the top 19 bits of each fp32, which is
+  // exactly hi_of(x)); X_lo: afull (splitters) -> lempty (MMA); B: full (bulk
+  // bytes) -> empty (MMA)
   __shared__ uint64_t full_bar[MAX_STAGES], empty_bar[MAX_STAGES], xfull_bar[MAX_STAGES], afull_bar[MAX_STAGES],
-      aempty_bar[MAX_STAGES], tfull_bar[2], tempty_bar[2];
+      aempty_bar[MAX_STAGES], lempty_bar[MAX_STAGES], tfull_bar[2], tempty_bar[2];
   __shared__ uint32_t tmem_base_sh;
 
   const int tid = threadIdx.x;
@@ -214,8 +224,11 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
     if (TMA_X) {
       for (int s = 0; s < p.sa; ++s) {
         mbar_init(&xfull_bar[s], 1);
-        mbar_init(&afull_bar[s], NUM_PRODUCER_WARPS * 32);
         mbar_init(&aempty_bar[s], 1);
+      }
+      for (int s = 0; s < p.sl; ++s) {
+        mbar_init(&afull_bar[s], NUM_PRODUCER_WARPS * 32);
+        mbar_init(&lempty_bar[s], 1);
       }
       for (int s = 0; s < p.sb; ++s) {
         mbar_init(&full_bar[s], 1);
@@ -250,7 +263,9 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
   auto cb_beg = [&](int vt) { return (p.ncb > 1 && vt % p.ncb) ? p.cbw0 : 0; };
   auto cb_w = [&](int vt) { return p.ncb > 1 ? ((vt % p.ncb) ? NP - p.cbw0 : p.cbw0) : NP; };
   const int B_STAGE = 2 * (p.ncb > 1 ? p.cbw0 : NP) * 128;  // TMA path B ring stage
-  uint8_t *const b_ring = smem + (size_t)p.sa * 2 * TILE_A_BYTES;  // TMA path
+  // TMA path smem: [raw X ring sa x 16 KB][X_lo ring sl x 16 KB][W ring sb x B_STAGE][epilogue staging]
+  uint8_t *const lo_ring = smem + (size_t)p.sa * TILE_A_BYTES;
+  uint8_t *const b_ring = lo_ring + (size_t)p.sl * TILE_A_BYTES;
   if (TMA_X && warp == TMA_WARP) {
     // ----------------------------- TMA issuer (X) -----------------------------
     if (lane == 0) {
@@ -258,7 +273,7 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
         const int s = it % p.sa, use = it / p.sa;
         if (use > 0) mbar_wait(&aempty_bar[s], (use - 1) & 1);
         mbar_arrive_expect_tx(&xfull_bar[s], TILE_A_BYTES);
-        tma_load_2d(smem + (size_t)s * 2 * TILE_A_BYTES, &xmap, (it % p.num_kb) * BK, (tile_of(it) / p.ncb) * BM,
+        tma_load_2d(smem + (size_t)s * TILE_A_BYTES, &xmap, (it % p.num_kb) * BK, (tile_of(it) / p.ncb) * BM,
                     &xfull_bar[s]);
       }
     }
@@ -281,28 +296,29 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
       }
     }
   } else if (TMA_X && warp < NUM_PRODUCER_WARPS) {
-    // -------------------- splitters: raw X tile -> hi / lo --------------------
-    // The split is elementwise and hi/lo share the swizzled layout, so each
-    // thread converts fixed 16-byte chunks with no address arithmetic.
+    // ---------------------- splitters: raw X tile -> lo ----------------------
+    // The split is elementwise and lo shares the raw tile's swizzled layout,
+    // so each thread converts fixed 16-byte chunks with no address arithmetic.
+    // The raw tile stays in place as the A_hi operand.
     constexpr int NT = NUM_PRODUCER_WARPS * 32;
     constexpr int PER = TILE_A_BYTES / 16 / NT;  // 8 chunks per thread
     for (int it = 0; it < total_it; ++it) {
       const int s = it % p.sa, use = it / p.sa;
+      const int l = it % p.sl, luse = it / p.sl;
       mbar_wait(&xfull_bar[s], use & 1);
-      uint8_t *st = smem + (size_t)s * 2 * TILE_A_BYTES;
-      float4 *a_hi = reinterpret_cast<float4 *>(st);
-      float4 *a_lo = reinterpret_cast<float4 *>(st + TILE_A_BYTES);
+      const float4 *a_raw = reinterpret_cast<const float4 *>(smem + (size_t)s * TILE_A_BYTES);
       float4 x[PER];
 #pragma unroll
-      for (int i = 0; i < PER; ++i) x[i] = a_hi[tid + i * NT];
+      for (int i = 0; i < PER; ++i) x[i] = a_raw[tid + i * NT];
+      if (luse > 0) mbar_wait(&lempty_bar[l], (luse - 1) & 1);
+      float4 *a_lo = reinterpret_cast<float4 *>(lo_ring + (size_t)l * TILE_A_BYTES);
 #pragma unroll
       for (int i = 0; i < PER; ++i) {
         const float4 hi = make_float4(hi_of(x[i].x), hi_of(x[i].y), hi_of(x[i].z), hi_of(x[i].w));
-        a_hi[tid + i * NT] = hi;
         a_lo[tid + i * NT] = make_float4(x[i].x - hi.x, x[i].y - hi.y, x[i].z - hi.z, x[i].w - hi.w);
       }
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-      mbar_arrive(&afull_bar[s]);
+      mbar_arrive(&afull_bar[l]);
     }
   } else if (!TMA_X && warp < NUM_PRODUCER_WARPS) {
     // ------------------------------ producers ------------------------------
@@ -382,24 +398,28 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
       const int NW = TMA_X ? cb_w(tile) : NP;  // MMA width of this work item
       const uint32_t b_lo_off = TMA_X ? (uint32_t)NW * 128 : (uint32_t)B_BYTES;
       for (int kb = 0; kb < p.num_kb; ++kb, ++it) {
-        int s, sA;
-        uint32_t a_hi, b_hi;
+        int s, sA, sL = 0;
+        uint32_t a_hi, a_lo, b_hi;
         if (TMA_X) {
           sA = it % p.sa;
+          sL = it % p.sl;
           s = it % p.sb;
-          mbar_wait(&afull_bar[sA], (it / p.sa) & 1);
+          mbar_wait(&xfull_bar[sA], (it / p.sa) & 1);
+          mbar_wait(&afull_bar[sL], (it / p.sl) & 1);
           mbar_wait(&full_bar[s], (it / p.sb) & 1);
-          a_hi = smem_u32(smem + (size_t)sA * 2 * TILE_A_BYTES);
+          a_hi = smem_u32(smem + (size_t)sA * TILE_A_BYTES);
+          a_lo = smem_u32(lo_ring + (size_t)sL * TILE_A_BYTES);
           b_hi = smem_u32(b_ring + (size_t)s * B_STAGE);
         } else {
           s = sA = it % S;
           mbar_wait(&full_bar[s], (it / S) & 1);
           a_hi = smem_u32(smem + (size_t)s * STAGE_BYTES);
+          a_lo = a_hi + TILE_A_BYTES;
           b_hi = a_hi + 2 * TILE_A_BYTES;
         }
         asm volatile("tcgen05.fence::after_thread_sync;");
         if (lane == 0) {
-          const uint32_t a_lo = a_hi + TILE_A_BYTES, b_lo = b_hi + b_lo_off;
+          const uint32_t b_lo = b_hi + b_lo_off;
           const int acc = kb % p.n_acc;
           const uint32_t d0 = tbase + (uint32_t)(acc * p.npa);
           const uint32_t first = (kb < p.n_acc) ? 1u : 0u;  // first K block of this accumulator
@@ -417,7 +437,10 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
             }
           }
           mma_commit(&empty_bar[s]);
-          if (TMA_X) mma_commit(&aempty_bar[sA]);
+          if (TMA_X) {
+            mma_commit(&aempty_bar[sA]);
+            mma_commit(&lempty_bar[sL]);
+          }
           if (kb == p.num_kb - 1) mma_commit(&tfull_bar[b]);
         }
         __syncwarp();
@@ -434,11 +457,12 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
     // SWIZZLE_128B buffer (row = lane, conflict-free float4 writes) and one
     // lane stores it with a TMA bulk tensor store (coalesced; tails clipped)
     constexpr bool TMA_H = TMA_X && VEC_H;
-    const int half = warp >= EPI_WARP1 ? 1 : 0;  // column chunks half, half + nhalf, ...
-    const int nhalf = p.epi8 ? 2 : 1;
+    // with 8 epilogue warps the two warps of a TMEM lane quadrant take
+    // contiguous halves of the item's 32-column chunks (a head's chunks stay
+    // with one thread for the attention-score epilogue)
+    const int half = warp >= EPI_WARP1 ? 1 : 0;
     const int widx = half ? 4 + warp - EPI_WARP1 : warp - EPI_WARP0;
-    uint8_t *const epi_buf = smem + (size_t)p.sa * 2 * TILE_A_BYTES + (size_t)p.sb * B_STAGE +
-                             (size_t)widx * p.eb * 4096;
+    uint8_t *const epi_buf = b_ring + (size_t)p.sb * B_STAGE + (size_t)widx * p.eb * 4096;
     int chunk = 0;
     int tcount = 0;
     for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++tcount) {
@@ -453,7 +477,18 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
       const float sc = (p.row_scale && gm < p.m) ? __ldg(p.row_scale + gm) : 1.0f;
       const uint32_t tbase = tmem + (uint32_t)(b * p.n_acc * p.npa) + ((uint32_t)(quad * 32) << 16);
       const int n_acc_used = p.num_kb < p.n_acc ? p.num_kb : p.n_acc;
-      for (int c0 = half * 32; c0 < NW; c0 += 32 * nhalf) {
+      const int nchunk = (NW + 31) / 32;
+      const int cmid = p.epi8 ? (nchunk + 1) / 2 : nchunk;
+      float att_s = 0.0f, att_t = 0.0f;
+      int att_h = -1;
+      // attention scores of head att_h (complete): to columns att_col + h, att_col + H + h
+      auto att_flush = [&]() {
+        if (att_h >= 0 && gm < p.m) {
+          p.H[gm * p.ldh + p.att_col + att_h] = att_s;
+          p.H[gm * p.ldh + p.att_col + p.att_H + att_h] = att_t;
+        }
+      };
+      for (int c0 = (half ? cmid : 0) * 32; c0 < (half ? nchunk : cmid) * 32; c0 += 32) {
         float y[32];
 #pragma unroll
         for (int i = 0; i < 32; ++i) y[i] = 0.0f;
@@ -482,6 +517,20 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
           if (p.col_bias && col < p.n) t = t + __ldg(p.col_bias + col);
           if (p.relu) t = t > 0.0f ? t : 0.0f;
           y[i] = t;
+        }
+        if (p.att) {
+          const int h = (cbb + c0) / p.att_Fh;
+          if (h != att_h) {
+            att_flush();
+            att_h = h;
+            att_s = att_t = 0.0f;
+          }
+          const float *as = p.att + cbb + c0, *at = p.att_dst + cbb + c0;
+#pragma unroll
+          for (int i = 0; i < 32; ++i) {
+            att_s = fmaf(y[i], __ldg(as + i), att_s);
+            att_t = fmaf(y[i], __ldg(at + i), att_t);
+          }
         }
         if constexpr (TMA_H) {
           uint8_t *buf = epi_buf + (chunk % p.eb) * 4096;
@@ -512,6 +561,7 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
             if (c0 + i < p.n) dst[i] = y[i];
         }
       }
+      if (p.att) att_flush();
       asm volatile("tcgen05.fence::before_thread_sync;");
       mbar_arrive(&tempty_bar[b]);
     }
@@ -527,7 +577,7 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
 
 struct Config {
   int np, npa, num_kb, stages, n_acc, n_buf;
-  int sa, sb, eb, epi8;
+  int sa, sb, sl, eb, epi8;
   int ncb, cbw0, npa_t, nbuf_t, nacc_t;  // TMA path: column blocks and their TMEM layout
   size_t smem, smem_tma, wimg_bytes;
 };
@@ -553,11 +603,11 @@ static bool configure(int64_t m, int32_t k, int32_t n, Config &c) {
   // double-buffered in 512 columns).  The X tile is read twice (L2 hit).
   if (g_cb < 0) {
     const char *e = getenv("GNN_GEMM_CB");
-    g_cb = (e && e[0] == '0') ? 0 : 1;
+    g_cb = (e && e[0] == '0') ? 0 : (e && e[0] == '2') ? 2 : 1;
   }
   c.ncb = 1;
   c.cbw0 = c.np;
-  if (g_cb && c.np > 256 && c.num_kb <= 8) {
+  if (g_cb && (c.np > 256 || (g_cb == 2 && c.np == 256)) && c.num_kb <= 8) {
     c.ncb = 2;
     c.cbw0 = (c.np / 2 + 31) / 32 * 32;
     if (c.cbw0 > 256 || c.np - c.cbw0 < 16) {
@@ -565,28 +615,34 @@ static bool configure(int64_t m, int32_t k, int32_t n, Config &c) {
       c.cbw0 = c.np;
     }
   }
-  // TMA path: separate rings; deepen the X ring first (HBM latency), then W
+  // TMA path: raw X ring (sa x 16 KB, the TMA destination and A_hi), X_lo
+  // ring (sl = 2 x 16 KB), W ring (sb x 2 x cbw0 x 128 B), epilogue staging
+  // (8 warps x eb x 4 KB).  The X loads come from HBM and need the depth
+  // (ncu r2: the MMA warp waited on X 33% of the time with 2 stages), so the
+  // raw ring gets what is left after W (2 stages) and the staging (eb = 1).
   {
-    const size_t budget = 225 * 1024, a_bytes = 2 * TILE_A_BYTES, b_bytes = 2 * (size_t)c.cbw0 * 128;
-    c.sa = 2;
-    c.sb = 2;
-    // epilogue staging: (epi8 ? 8 : 4) warps x eb x 4 KB; prefer 8 warps
-    auto need = [&](int sa, int sb, int eb, int e8) {
-      return (size_t)sa * a_bytes + (size_t)sb * b_bytes + (size_t)eb * (e8 ? 8 : 4) * 4096 + 1024;
-    };
+    const size_t budget = 225 * 1024, b_bytes = 2 * (size_t)c.cbw0 * 128;
     if (g_epi8 < 0) {
       const char *e = getenv("GNN_GEMM_EPI8");
       g_epi8 = (e && e[0] == '0') ? 0 : 1;
     }
-    c.epi8 = g_epi8 ? 1 : 0;
-    c.eb = 2;
-    if (need(2, 2, c.eb, c.epi8) > budget) c.eb = 1;
-    if (c.epi8 && need(2, 2, c.eb, 1) > budget) {
-      c.epi8 = 0;
-      c.eb = need(2, 2, 2, 0) > budget ? 1 : 2;
+    static int env_sa = -2;
+    if (env_sa == -2) {
+      const char *e = getenv("GNN_GEMM_SA");
+      env_sa = e ? atoi(e) : -1;
     }
-    while (c.sa < MAX_STAGES && need(c.sa + 1, c.sb, c.eb, c.epi8) <= budget) ++c.sa;
-    while (c.sb < MAX_STAGES && need(c.sa, c.sb + 1, c.eb, c.epi8) <= budget) ++c.sb;
+    c.sl = 2;
+    c.sb = 2;
+    c.epi8 = g_epi8 ? 1 : 0;
+    c.eb = 1;
+    auto need = [&](int sa, int sb, int eb, int e8) {
+      return (size_t)(sa + c.sl) * TILE_A_BYTES + (size_t)sb * b_bytes + (size_t)eb * (e8 ? 8 : 4) * 4096 + 1024;
+    };
+    if (c.epi8 && need(2, 2, 1, 1) > budget) c.epi8 = 0;
+    c.sa = 2;
+    const int sa_max = env_sa > 1 && env_sa <= MAX_STAGES ? env_sa : MAX_STAGES;
+    while (c.sa < sa_max && need(c.sa + 1, c.sb, c.eb, c.epi8) <= budget) ++c.sa;
+    if (need(c.sa, c.sb, 2, c.epi8) <= budget) c.eb = 2;
     c.smem_tma = need(c.sa, c.sb, c.eb, c.epi8);
     if (c.smem_tma > budget) c.sa = 0;  // TMA path unavailable for this n
   }
@@ -683,9 +739,14 @@ size_t gemm_tc_workspace(int64_t m, int32_t k, int32_t n) {
   return (c.wimg_bytes + 255) & ~(size_t)255;
 }
 
+struct AttEpi {
+  const float *a = nullptr, *a_dst = nullptr;  // [H * Fh] each
+  int32_t H = 0, Fh = 0, col = 0;
+};
 static cudaError_t launch_gemm_tc_one(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H, int64_t ldh,
                                       int64_t m, int32_t k, int32_t n, const float *row_scale, const float *col_bias,
-                                      int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s);
+                                      int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s,
+                                      const AttEpi &att = AttEpi());
 
 // Returns cudaErrorNotSupported only for shapes no launch takes (k < 1) or a
 // missing / misaligned workspace, cudaErrorInvalidValue for a workspace that
@@ -705,9 +766,29 @@ cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t 
   return cudaSuccess;
 }
 
+// GAT transform with the attention scores in the epilogue (reading R5):
+// [Z | s | t] with Z = X W (n = H * Fh columns on the tensor cores) and
+// s[h] = Z_h . a_src_h, t[h] = Z_h . a_dst_h accumulated in fp32 from the
+// epilogue's Z values.  Needs Fh % 32 == 0 and a single launch for the width;
+// returns cudaErrorNotSupported otherwise (the caller folds the scores into
+// extra GEMM columns instead).
+cudaError_t launch_gemm_att(const float *X, int64_t ldx, const float *W, int64_t ldw, float *Z, int64_t ldz, int64_t m,
+                            int32_t k, int32_t H, int32_t Fh, const float *a_src, const float *a_dst, void *ws,
+                            size_t ws_bytes, cudaStream_t s) {
+  const int32_t n = H * Fh;
+  if (Fh % 32 != 0 || k < 1 || !ws || ((uintptr_t)ws & 15) || slice_width(m, k, n) != n) return cudaErrorNotSupported;
+  AttEpi att;
+  att.a = a_src;
+  att.a_dst = a_dst;
+  att.H = H;
+  att.Fh = Fh;
+  att.col = n;
+  return launch_gemm_tc_one(X, ldx, W, ldw, Z, ldz, m, k, n, nullptr, nullptr, 0, ws, ws_bytes, s, att);
+}
+
 static cudaError_t launch_gemm_tc_one(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H, int64_t ldh,
                                       int64_t m, int32_t k, int32_t n, const float *row_scale, const float *col_bias,
-                                      int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s) {
+                                      int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s, const AttEpi &att) {
   using namespace tc;
   Config c;
   if (!configure(m, k, n, c)) return cudaErrorNotSupported;
@@ -729,7 +810,7 @@ static cudaError_t launch_gemm_tc_one(const float *X, int64_t ldx, const float *
   const int64_t num_tiles = (m + BM - 1) / BM;
   if (num_tiles > 0x3fffffff) return cudaErrorNotSupported;
   TcParams p{X, ldx, H, ldh, img, m, k, n, c.np, c.npa, c.num_kb, (int32_t)num_tiles, c.stages, c.n_acc, c.n_buf,
-             c.sa, c.sb, c.eb, 1, c.np, c.epi8, row_scale, col_bias, relu};
+             c.sa, c.sb, c.sl, c.eb, 1, c.np, c.epi8, row_scale, col_bias, relu, att.a, att.a_dst, att.H, att.Fh, att.col};
   const bool vx = (ldx % 4 == 0) && ((uintptr_t)X % 16 == 0);
   const bool vh = (ldh % 4 == 0) && ((uintptr_t)H % 16 == 0);
   CUtensorMap xmap;
@@ -753,6 +834,14 @@ static cudaError_t launch_gemm_tc_one(const float *X, int64_t ldx, const float *
     p.n_buf = c.nbuf_t;
     p.n_acc = c.nacc_t;
     p.num_tiles = (int32_t)(num_tiles * c.ncb);
+  }
+  if (att.a) {
+    // every work item must hold whole heads, and with 8 epilogue warps the
+    // boundary between the two halves of an item's chunks must fall between heads
+    const int ws0 = p.ncb > 1 ? p.cbw0 : c.np, ws1 = p.ncb > 1 ? c.np - p.cbw0 : c.np;
+    if (ws0 % att.Fh != 0 || ws1 % att.Fh != 0) return cudaErrorNotSupported;
+    for (int w : {ws0, ws1})
+      if ((((w + 31) / 32 + 1) / 2 * 32) % att.Fh != 0) p.epi8 = 0;
   }
   // one persistent CTA per SM, or one per work item when there are fewer
   const int grid = (int)(p.num_tiles < num_sms ? p.num_tiles : num_sms);

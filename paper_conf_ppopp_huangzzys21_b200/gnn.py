@@ -96,6 +96,8 @@ _SIGS = {
     "gnn_gcn_layer": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _I64, _I32, _I32, _I32, _P, _I64, _P, _SZ, _P]),
     "gnn_gcn_aggregate_prescaled": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _I64, _I32, _P, _SZ, _P]),
     "gnn_gat_fold_weights": (ctypes.c_int, [_P, _P, _P, _I32, _I32, _I32, _P, _I64, _P]),
+    "gnn_gat_transform": (ctypes.c_int, [_P, _I64, _I64, _I32, _P, _I64, _P, _P, _I32, _I32, _P, _I64, _P, _SZ, _P]),
+    "gnn_gat_transform_workspace_size": (_SZ, [_I64, _I32, _I32, _I32]),
     "gnn_partition_rows": (ctypes.c_int, [_I64, _P, _I32, _P]),
     "gnn_local_csr": (ctypes.c_int, [_I64, _P, _P, _P, _I32, _I32, ctypes.POINTER(_I64), ctypes.POINTER(_I64),
                                      _P, _P, _P]),
@@ -304,6 +306,19 @@ def gat_layer(plan: Plan, X, W, a_src, a_dst, H, Fh, neg_slope=0.2, out=None, st
     _call("gnn_gat_layer", plan.handle, _tp(X), _ld(X, f_in), f_in, _tp(W.contiguous()), _tp(a_src.contiguous()),
           _tp(a_dst.contiguous()), H, Fh, float(neg_slope), _tp(Y), _ld(Y, F), _tp(ws), nb, _stream(stream))
     return Y
+
+
+def gat_transform(X, W, a_src, a_dst, H, Fh, out=None, stream=None):
+    """gnn_gat_transform: [Z | s | t] = X W with the GAT scores (reading R5)."""
+    torch = _torch()
+    m, f_in = X.shape
+    ldz = (H * Fh + 2 * H + 7) // 8 * 8
+    Z = out if out is not None else torch.empty((m, ldz), dtype=torch.float32, device=X.device)
+    nb = _lib.gnn_gat_transform_workspace_size(m, f_in, H, Fh)
+    ws = torch.empty(max(nb, 256), dtype=torch.uint8, device=X.device)
+    _call("gnn_gat_transform", _tp(X), _ld(X, f_in), m, f_in, _tp(W.contiguous()), H * Fh, _tp(a_src.contiguous()),
+          _tp(a_dst.contiguous()), H, Fh, _tp(Z), Z.stride(0), _tp(ws), nb, _stream(stream))
+    return Z
 
 
 def edgeconv_aggregate(plan: Plan, PQ, f_out, out=None, stream=None):

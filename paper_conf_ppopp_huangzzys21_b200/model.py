@@ -61,7 +61,6 @@ class RowPartitionedGCNGAT:
         self.Y1 = torch.empty((R, self.F), device=d)
         self.Hs2 = torch.zeros((P, self.F), device=d)
         self.Y2 = torch.empty((R, self.F), device=d)
-        self.Wext = torch.empty((self.F, self.ldwe), device=d)
         self.Zst = torch.zeros((P, self.ldwe), device=d)
         self.Y3 = torch.empty((R, self.HF), device=d)
         self.nsrc_ptr, _ = self.plan.normalizers()
@@ -69,7 +68,7 @@ class RowPartitionedGCNGAT:
         self.ws_gat, self.ws_gat_b = self.plan.workspace(_g.GNN_OP_GAT_AGGREGATE, 0, self.HF, heads, d)
         self.names = ["agg1", "gemm1", "gemm2+xchg", "agg2", "gemm3+xchg", "gat_agg"]
         gw = max(_g._lib.gnn_gemm_workspace_size(R, self.F_in, self.F), _g._lib.gnn_gemm_workspace_size(R, self.F, self.F),
-                 _g._lib.gnn_gemm_workspace_size(R, self.F, self.ldwe))
+                 _g._lib.gnn_gat_transform_workspace_size(R, self.F, heads, head_dim))
         self.ws_gemm = torch.empty(max(gw, 256), dtype=torch.uint8, device=d)
         self.ws_gemm_b = gw
 
@@ -171,11 +170,9 @@ class RowPartitionedGCNGAT:
                                             self.ws_agg_b, sp), "agg2")
         rec(4)
         z_loc = self.Zst[off:off + R]
-        # [Z | s | t]: scores as extra GEMM columns X (W_h a_h) (R5)
-        chk(lib.gnn_gat_fold_weights(P(self.W3), P(self.a_s), P(self.a_d), F, H, self.Fh, P(self.Wext), self.ldwe,
-                                     sp), "gat fold")
-        chk(lib.gnn_gemm(P(self.Y2), F, P(self.Wext), self.ldwe, P(z_loc), self.ldwe, R, F, self.ldwe, None, None, 0,
-                         *gws, sp), "gemm3")
+        # [Z | s | t] = Y2 W3 with the GAT scores from the GEMM epilogue (R5)
+        chk(lib.gnn_gat_transform(P(self.Y2), F, R, F, P(self.W3), HF, P(self.a_s), P(self.a_d), H, self.Fh, P(z_loc),
+                                  self.ldwe, *gws, sp), "gemm3 (gat transform)")
         self._allgather(self.Zst)
         rec(5)
         tptr = ctypes.c_void_p(z_loc.data_ptr() + 4 * (HF + H))

@@ -109,6 +109,31 @@ def test_gemm_small_workspace_is_an_error_not_a_fallback():
 
 
 # --------------------------------------------------------------------------- #
+# a5 for GAT: [Z | s | t] with the scores from the GEMM epilogue (heads of a
+# multiple of 32 features) or folded into extra GEMM columns (other heads)
+# --------------------------------------------------------------------------- #
+@pytest.mark.parametrize("m,f_in,Hh,Fh", [(100003, 256, 8, 32), (5000, 128, 8, 8), (3001, 100, 4, 64),
+                                          (2000, 64, 1, 256), (1500, 100, 3, 96), (1200, 64, 2, 192),
+                                          (777, 37, 5, 32)])
+def test_gat_transform(m, f_in, Hh, Fh):
+    X = gs.uniform(m, f_in, seed=f_in)
+    lim = np.sqrt(6 / (f_in + Hh * Fh))
+    W = gs.uniform(f_in, Hh * Fh, lo=-lim, hi=lim, seed=Fh)
+    al = np.sqrt(6 / (Fh + 1))
+    a_s = gs.uniform(1, Hh * Fh, lo=-al, hi=al, seed=3)[0]
+    a_d = gs.uniform(1, Hh * Fh, lo=-al, hi=al, seed=4)[0]
+    Z = H(G.gat_transform(T(X), T(W), T(a_s), T(a_d), Hh, Fh))
+    rows = sample_rows(m, 2000, seed=5, extra=np.arange(max(0, m - 130), m))
+    Zo = oracle.gemm(X[rows], W).astype(np.float64)
+    F = Hh * Fh
+    assert_close(Z[rows, :F], Zo, what=f"gat transform z {m}x{f_in} {Hh}x{Fh}")
+    s_ref = (Zo.reshape(len(rows), Hh, Fh) * a_s.reshape(Hh, Fh)).sum(2)
+    t_ref = (Zo.reshape(len(rows), Hh, Fh) * a_d.reshape(Hh, Fh)).sum(2)
+    assert_close(Z[rows, F:F + Hh], s_ref, what="s")
+    assert_close(Z[rows, F + Hh:F + 2 * Hh], t_ref, what="t")
+
+
+# --------------------------------------------------------------------------- #
 # a6 at the bench's mappings: F = 100 on a graph with average degree >= 32
 # takes (vec 4, 16 lanes, 2 vectors per lane) with 7 of 32 vector slots
 # masked; transform-first F = 256 takes (8, 16, 2)
