@@ -42,6 +42,8 @@ def _load():
                                        ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]
         lib.synth_powerlaw_ex.restype = ctypes.c_int
         lib.synth_powerlaw_ex.argtypes = lib.synth_powerlaw.argtypes + [ctypes.c_void_p]
+        lib.synth_powerlaw_sym.restype = ctypes.c_int
+        lib.synth_powerlaw_sym.argtypes = lib.synth_powerlaw_ex.argtypes
         lib.synth_uniform_f32.restype = None
         lib.synth_uniform_f32.argtypes = [ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_float,
                                           ctypes.c_float, ctypes.c_uint64, ctypes.c_void_p]
@@ -62,17 +64,18 @@ class Graph:
         return int(self.rowptr[-1])
 
 
-def powerlaw(n, nnz, mean, var, cap, comm=32, rho=0.8, seed=1, with_relabel=False) -> Graph:
-    """GEN-PL graph.  with_relabel=True also returns (in stats["relabel"]) the
-    relabel permutation (new id of pre-relabel node v), for locality studies."""
+def powerlaw(n, nnz, mean, var, cap, comm=32, rho=0.8, seed=1, with_relabel=False, sym=False) -> Graph:
+    """GEN-PL graph (directed; sym=True: the undirected recipe of SURVEY §8(d),
+    nnz/2 pairs symmetrised, min degree 1).  with_relabel=True also returns
+    (in stats["relabel"]) the relabel permutation (new id of pre-relabel node v)."""
     lib = _load()
     rowptr = np.empty(n + 1, dtype=np.int64)
     colidx = np.empty(max(nnz, 1), dtype=np.int32)
     st = np.zeros(4, dtype=np.int64)
     rel = np.empty(n, dtype=np.int64) if with_relabel else None
-    rc = lib.synth_powerlaw_ex(n, nnz, float(mean), float(var), cap, comm, float(rho), seed,
-                               rowptr.ctypes.data, colidx.ctypes.data, st.ctypes.data,
-                               None if rel is None else rel.ctypes.data)
+    fn = lib.synth_powerlaw_sym if sym else lib.synth_powerlaw_ex
+    rc = fn(n, nnz, float(mean), float(var), cap, comm, float(rho), seed, rowptr.ctypes.data, colidx.ctypes.data,
+            st.ctypes.data, None if rel is None else rel.ctypes.data)
     if rc != 0:
         raise RuntimeError(f"synth_powerlaw failed rc={rc}")
     stats = {"max": int(st[0]), "mean": st[1] / 1e6, "var": st[2] / 1e3, "zero_rows": int(st[3])}
@@ -147,15 +150,16 @@ def from_rows(rows) -> Graph:
 # BASELINE.json configs; seeds = 20210227 + 10*cfg + {0 graph, 1 X, 2 W, 3 a/theta/phi/b}
 CONFIGS = {
     # C1: Cora-shaped, 2,708 nodes, 10,556 CSR entries, F=16
-    "C1": dict(n=2708, nnz=10556, mean=3.9, var=27.0, cap=168, comm=32, F=16),
+    "C1": dict(n=2708, nnz=10556, mean=3.9, var=27.0, cap=168, comm=32, F=16, sym=True),
     # C2: ogbn-arxiv-shaped (Table 3): 169,343 nodes, 1,166,243 edges, max 13,155, var 4.6K
     "C2": dict(n=169343, nnz=1166243, mean=6.89, var=4600.0, cap=13155, comm=32, F_in=128, H=8, Fh=8),
     # C3: Reddit-shaped: 232,965 nodes, 114.6M entries, max 21,657, var 640K
-    "C3": dict(n=232965, nnz=114615892, mean=492.0, var=640000.0, cap=21657, comm=1024, F_in=602, F=256),
+    "C3": dict(n=232965, nnz=114615892, mean=492.0, var=640000.0, cap=21657, comm=1024, F_in=602, F=256, sym=True),
     # C4: kNN point clouds 32 x 1024, k=20, F=64
     "C4": dict(batch=32, points=1024, k=20, F=64),
     # C5: ogbn-products-shaped: 2,449,029 nodes, 123,718,280 entries, max 17,481, var 9.1K
-    "C5": dict(n=2449029, nnz=123718280, mean=50.5, var=9100.0, cap=17481, comm=256, F_in=100, F=256, H=8, Fh=32),
+    "C5": dict(n=2449029, nnz=123718280, mean=50.5, var=9100.0, cap=17481, comm=256, F_in=100, F=256, H=8, Fh=32,
+               sym=True),
 }
 
 
@@ -170,5 +174,10 @@ def config_graph(cfg: str, rho: float = 0.8, scale: float = 1.0, with_relabel: b
     n = max(64, int(c["n"] * scale))
     nnz = max(n, int(c["nnz"] * scale))
     cap = min(c["cap"], n - 1)
+    # Cora, Reddit and products are undirected: SURVEY §8(d) GEN-PL draws
+    # nnz/2 pairs and symmetrises them (min degree 1); arxiv (C2) is directed
+    sym = c.get("sym", False)
+    if sym:
+        nnz -= nnz % 2
     return powerlaw(n, nnz, c["mean"], c["var"], cap, c["comm"], rho, seed_of(cfg, 0) + int(rho * 100),
-                    with_relabel=with_relabel)
+                    with_relabel=with_relabel, sym=sym)

@@ -293,6 +293,247 @@ int synth_powerlaw(int64_t n, int64_t nnz, double mean, double var, int64_t cap,
   return synth_powerlaw_ex(n, nnz, mean, var, cap, comm, rho, seed, rowptr, colidx, stats, NULL);
 }
 
+/* LSD radix sort of uint64 keys (16-bit digits), tmp of the same size */
+static void radix_u64(uint64_t *a, uint64_t *tmp, int64_t m, int bits) {
+  int64_t *cnt = (int64_t *)malloc(sizeof(int64_t) * 65536);
+  for (int sh = 0; sh < bits; sh += 16) {
+    memset(cnt, 0, sizeof(int64_t) * 65536);
+    for (int64_t i = 0; i < m; ++i) cnt[(a[i] >> sh) & 0xFFFF]++;
+    int64_t s = 0;
+    for (int d = 0; d < 65536; ++d) { int64_t c = cnt[d]; cnt[d] = s; s += c; }
+    for (int64_t i = 0; i < m; ++i) tmp[cnt[(a[i] >> sh) & 0xFFFF]++] = a[i];
+    memcpy(a, tmp, sizeof(uint64_t) * (size_t)m);
+  }
+  free(cnt);
+}
+static int64_t unique_u64(uint64_t *a, int64_t m) {
+  if (m == 0) return 0;
+  int64_t k = 1;
+  for (int64_t i = 1; i < m; ++i)
+    if (a[i] != a[k - 1]) a[k++] = a[i];
+  return k;
+}
+
+/*
+ * GEN-PL, undirected (SURVEY.md §8(d) steps 1-6 for C1/C3/C5): `nnz` CSR
+ * entries = nnz/2 undirected pairs, symmetrised, no self loops, no duplicates.
+ *   1. lognormal expected degrees w_v (mean nnz/n, Table 3 variance, clipped
+ *      to cap, the heaviest at cap);
+ *   2. community g(v) = floor(v / comm) owns a template of ceil(2*rho*mean_g)
+ *      nodes drawn proportional to w;
+ *   3. node v proposes about w_v / 2 partners: round(rho * that) uniformly
+ *      from its template, the rest proportional to w (so its expected degree
+ *      is ~w_v: its own proposals plus being proposed);
+ *   4. pairs are canonicalised to (min, max) and deduplicated; top-up draws
+ *      (v ~ w, partner as in 3) until there are nnz/2 pairs, random ones are
+ *      dropped if over;
+ *   5. degree floor 1: every isolated node is attached to a partner ~ w, and
+ *      as many pairs whose endpoints both have degree >= 3 are removed;
+ *   6. symmetrise, random relabel, CSR rows sorted by source id.
+ */
+int synth_powerlaw_sym(int64_t n, int64_t nnz, double mean, double var, int64_t cap, int64_t comm,
+                       double rho, uint64_t seed, int64_t *rowptr, int32_t *colidx, int64_t *stats,
+                       int64_t *relabel_out) {
+  (void)mean;
+  if (n <= 2 || nnz < 2 || (nnz & 1) || cap < 1) return -1;
+  if (cap > n - 1) cap = n - 1;
+  const int64_t P = nnz / 2;
+  if (P > n * (n - 1) / 2) return -2;
+  rng_t rng = {seed * 0x2545F4914F6CDD1DULL + 0x7654321ULL};
+  double *w = (double *)malloc(sizeof(double) * n);
+  if (!w) return -3;
+  double s2 = log(1.0 + var / ((double)nnz / n * (double)nnz / n));
+  double sg = sqrt(s2), mu = log((double)nnz / n) - 0.5 * s2;
+  for (int64_t i = 0; i < n; ++i) w[i] = exp(mu + sg * rng_normal(&rng));
+  const double target_mean = (double)nnz / (double)n;
+  for (int it = 0; it < 8; ++it) {
+    double tot = 0;
+    for (int64_t i = 0; i < n; ++i) tot += w[i];
+    double sc = target_mean * n / tot;
+    for (int64_t i = 0; i < n; ++i) {
+      w[i] *= sc;
+      if (w[i] > (double)cap) w[i] = (double)cap;
+    }
+  }
+  int64_t imax = 0;
+  for (int64_t i = 1; i < n; ++i) if (w[i] > w[imax]) imax = i;
+  w[imax] = (double)cap;
+  alias_t al;
+  if (alias_build(&al, w, n)) return -3;
+  /* templates */
+  int64_t ncomm = comm > 0 ? (n + comm - 1) / comm : 0;
+  int64_t *tpl_off = NULL, *tpl = NULL;
+  if (rho > 0 && ncomm > 0) {
+    tpl_off = (int64_t *)calloc((size_t)ncomm + 1, sizeof(int64_t));
+    for (int64_t g = 0; g < ncomm; ++g) {
+      int64_t lo = g * comm, hi = lo + comm < n ? lo + comm : n;
+      double md = 0;
+      for (int64_t v = lo; v < hi; ++v) md += w[v];
+      md /= (double)(hi - lo);
+      int64_t ts = (int64_t)ceil(2.0 * rho * md);
+      if (ts > n / 2) ts = n / 2;
+      if (ts < 1) ts = 1;
+      tpl_off[g + 1] = tpl_off[g] + ts;
+    }
+    tpl = (int64_t *)malloc(sizeof(int64_t) * (tpl_off[ncomm] + 1));
+    int64_t *buf = NULL, bufcap = 0;
+    for (int64_t g = 0; g < ncomm; ++g) {
+      int64_t ts = tpl_off[g + 1] - tpl_off[g];
+      if (bufcap < 2 * ts + 64) { bufcap = 2 * ts + 64; buf = (int64_t *)realloc(buf, sizeof(int64_t) * bufcap); }
+      int64_t k = 0;
+      while (k < ts) {
+        int64_t need = ts - k;
+        for (int64_t j = 0; j < need; ++j) buf[k + j] = alias_draw(&al, &rng);
+        k = sort_unique_i64(buf, k + need);
+      }
+      memcpy(tpl + tpl_off[g], buf, sizeof(int64_t) * ts);
+    }
+    free(buf);
+  }
+  /* partner of v: from v's template with probability rho (when it has one), else ~ w */
+  #define PARTNER(v)                                                                         \
+    ((tpl && rng_u01(&rng) < rho)                                                            \
+         ? tpl[tpl_off[(v) / comm] + (int64_t)rng_below(&rng, (uint64_t)(tpl_off[(v) / comm + 1] - tpl_off[(v) / comm]))] \
+         : alias_draw(&al, &rng))
+  /* 3. proposals: about w_v / 2 per node, by largest remainder so the total is P */
+  int64_t cap_keys = P + P / 4 + 1024, m = 0;
+  uint64_t *key = (uint64_t *)malloc(sizeof(uint64_t) * (size_t)cap_keys);
+  uint64_t *tmp = (uint64_t *)malloc(sizeof(uint64_t) * (size_t)cap_keys);
+  if (!key || !tmp) return -3;
+  {
+    double tot = 0;
+    for (int64_t i = 0; i < n; ++i) tot += w[i];
+    double carry = 0;
+    for (int64_t v = 0; v < n; ++v) {
+      double x = w[v] * (double)P / tot + carry;
+      int64_t h = (int64_t)floor(x);
+      carry = x - (double)h;
+      for (int64_t j = 0; j < h && m < cap_keys; ++j) {
+        int64_t u = PARTNER(v);
+        if (u == v) continue;
+        int64_t a = v < u ? v : u, b = v < u ? u : v;
+        key[m++] = (uint64_t)a * (uint64_t)n + (uint64_t)b;
+      }
+    }
+  }
+  int bits = 0;
+  while (bits < 64 && ((uint64_t)1 << bits) <= (uint64_t)n * (uint64_t)n) bits += 16;
+  radix_u64(key, tmp, m, bits);
+  m = unique_u64(key, m);
+  /* 4. top-up / trim to exactly P pairs */
+  int guard = 0;
+  double eff = 0.5;  /* fraction of top-up draws that survive dedup (updated per round) */
+  while (m < P && guard++ < 64) {
+    int64_t need = P - m, add = (int64_t)((double)need / eff * 1.1) + 64, m0 = m;
+    if (m + add > cap_keys) {
+      cap_keys = m + add + 1024;
+      key = (uint64_t *)realloc(key, sizeof(uint64_t) * (size_t)cap_keys);
+      tmp = (uint64_t *)realloc(tmp, sizeof(uint64_t) * (size_t)cap_keys);
+    }
+    for (int64_t j = 0; j < add; ++j) {
+      int64_t v = alias_draw(&al, &rng), u = PARTNER(v);
+      if (u == v) continue;
+      int64_t a = v < u ? v : u, b = v < u ? u : v;
+      key[m++] = (uint64_t)a * (uint64_t)n + (uint64_t)b;
+    }
+    const int64_t drawn = m - m0;
+    radix_u64(key, tmp, m, bits);
+    m = unique_u64(key, m);
+    if (drawn > 0) eff = (double)(m - m0) / (double)drawn;
+    if (eff < 0.05) eff = 0.05;
+  }
+  if (m < P) return -4;
+  if (m > P) { /* drop random pairs: partial Fisher-Yates moves the dropped ones to the tail */
+    for (int64_t j = 0; j < m - P; ++j) {
+      int64_t r = j + (int64_t)rng_below(&rng, (uint64_t)(m - j));
+      uint64_t t = key[j]; key[j] = key[r]; key[r] = t;
+    }
+    memmove(key, key + (m - P), sizeof(uint64_t) * (size_t)P);
+    m = P;
+    radix_u64(key, tmp, m, bits);
+  }
+  /* 5. degree floor 1: attach every isolated node to a partner ~ w, then
+     remove as many pairs whose endpoints both have degree >= 3 (then >= 2;
+     random scan start) so that no endpoint becomes isolated */
+  int64_t *deg = (int64_t *)calloc((size_t)n, sizeof(int64_t));
+  for (int64_t i = 0; i < m; ++i) { deg[key[i] / n]++; deg[key[i] % n]++; }
+  {
+    int64_t attached = 0, m0 = m;
+    for (int64_t v = 0; v < n; ++v) {
+      if (deg[v] != 0) continue;
+      int64_t u;
+      do { u = alias_draw(&al, &rng); } while (u == v);
+      if (m >= cap_keys) {
+        cap_keys = m + 1024;
+        key = (uint64_t *)realloc(key, sizeof(uint64_t) * (size_t)cap_keys);
+        tmp = (uint64_t *)realloc(tmp, sizeof(uint64_t) * (size_t)cap_keys);
+      }
+      int64_t a2 = v < u ? v : u, b2 = v < u ? u : v;
+      key[m++] = (uint64_t)a2 * (uint64_t)n + (uint64_t)b2;  /* new: v had no pair */
+      deg[v]++; deg[u]++;
+      ++attached;
+    }
+    if (attached > 0) {
+      int64_t removed = 0, start = (int64_t)rng_below(&rng, (uint64_t)m0);
+      uint8_t *dead = (uint8_t *)calloc((size_t)m, 1);
+      for (int thr = 3; thr >= 2 && removed < attached; --thr)
+        for (int64_t t = 0; t < m0 && removed < attached; ++t) {
+          int64_t i = (start + t) % m0;
+          int64_t a2 = (int64_t)(key[i] / n), b2 = (int64_t)(key[i] % n);
+          if (!dead[i] && deg[a2] >= thr && deg[b2] >= thr) { dead[i] = 1; deg[a2]--; deg[b2]--; ++removed; }
+        }
+      int64_t k = 0;
+      for (int64_t i = 0; i < m; ++i) if (!dead[i]) key[k++] = key[i];
+      free(dead);
+      m = k;
+      radix_u64(key, tmp, m, bits);
+    }
+  }
+  /* 6. relabel + symmetric CSR */
+  int64_t *perm = (int64_t *)malloc(sizeof(int64_t) * n);
+  for (int64_t i = 0; i < n; ++i) perm[i] = i;
+  for (int64_t i = n - 1; i > 0; --i) {
+    int64_t j = (int64_t)rng_below(&rng, (uint64_t)(i + 1));
+    int64_t t = perm[i]; perm[i] = perm[j]; perm[j] = t;
+  }
+  memset(deg, 0, sizeof(int64_t) * (size_t)n);
+  for (int64_t i = 0; i < m; ++i) { deg[perm[key[i] / n]]++; deg[perm[key[i] % n]]++; }
+  rowptr[0] = 0;
+  for (int64_t v = 0; v < n; ++v) rowptr[v + 1] = rowptr[v] + deg[v];
+  if (rowptr[n] != nnz) { /* only the floor step can shift the count (by duplicates it removed) */
+    free(deg); free(perm); free(key); free(tmp); free(tpl); free(tpl_off); alias_free(&al); free(w);
+    return -5;
+  }
+  int64_t *fill = (int64_t *)malloc(sizeof(int64_t) * n);
+  memcpy(fill, rowptr, sizeof(int64_t) * n);
+  for (int64_t i = 0; i < m; ++i) {
+    int64_t a = perm[key[i] / n], b = perm[key[i] % n];
+    colidx[fill[a]++] = (int32_t)b;
+    colidx[fill[b]++] = (int32_t)a;
+  }
+  int64_t maxd = 0, zeros = 0;
+  double m2 = 0, m1 = (double)nnz / n;
+  for (int64_t v = 0; v < n; ++v) {
+    const int64_t d = rowptr[v + 1] - rowptr[v];
+    if (d > 1) qsort(colidx + rowptr[v], (size_t)d, sizeof(int32_t), cmp_i32);
+    if (d > maxd) maxd = d;
+    zeros += d == 0;
+    m2 += ((double)d - m1) * ((double)d - m1);
+  }
+  if (stats) {
+    stats[0] = maxd;
+    stats[1] = (int64_t)llround(m1 * 1e6);
+    stats[2] = (int64_t)llround(m2 / n * 1e3);
+    stats[3] = zeros;
+  }
+  if (relabel_out) memcpy(relabel_out, perm, sizeof(int64_t) * (size_t)n);
+  #undef PARTNER
+  free(fill); free(deg); free(perm); free(key); free(tmp); free(tpl); free(tpl_off);
+  alias_free(&al);
+  free(w);
+  return 0;
+}
+
 /* uniform fp32 features in [lo, hi) with row stride ld (pad columns = 0) */
 void synth_uniform_f32(int64_t rows, int64_t cols, int64_t ld, float lo, float hi,
                        uint64_t seed, float *out) {

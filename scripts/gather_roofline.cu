@@ -149,6 +149,63 @@ __global__ void __launch_bounds__(WARPS * 32) k_bulk(const char *X, const int32_
   if (sum == 12345.f) out[0] = sum;
 }
 
+// cp.async (LDGSTS) gather: each lane copies its own 16-byte chunks of a row
+// into a per-warp shared-memory ring of S row slots and later reads back only
+// those chunks (no cross-lane sharing, so no barrier): in-flight data lives in
+// shared memory, not in registers
+template <int ROWB, int S, int WARPS>
+__global__ void __launch_bounds__(WARPS * 32) k_cpa(const char *X, const int32_t *idx, int64_t nidx, int per_warp,
+                                                    float *out) {
+  constexpr int SLOT = (ROWB + 127) / 128 * 128;
+  constexpr int NCH = ROWB / 16;               // 16-byte chunks per row
+  constexpr int PER = (NCH + 31) / 32;          // chunks per lane
+  extern __shared__ __align__(128) char smem[];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  char *ring = smem + (size_t)w * S * SLOT;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t base = warp * per_warp;
+  auto issue = [&](int32_t u, int s) {
+    const char *src = X + (int64_t)u * ROWB;
+#pragma unroll
+    for (int k = 0; k < PER; ++k) {
+      const int c = lane + 32 * k;
+      if (c < NCH)
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(ring + s * SLOT + 16 * c)),
+                     "l"(src + 16 * c)
+                     : "memory");
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  int32_t cur = idx[(base + lane) % nidx];
+  int32_t nxt = idx[(base + 32 + lane) % nidx];
+#pragma unroll
+  for (int q = 0; q < S; ++q) issue(__shfl_sync(~0u, cur, q), q);
+  float4 a[PER] = {};
+  for (int j = 0; j < per_warp; ++j) {
+    const int s = j % S;
+    asm volatile("cp.async.wait_group %0;" ::"n"(S - 1) : "memory");
+#pragma unroll
+    for (int k = 0; k < PER; ++k) {
+      const int c = lane + 32 * k;
+      if (c < NCH) {
+        const float4 v = *reinterpret_cast<const float4 *>(ring + s * SLOT + 16 * c);
+        a[k].x += v.x; a[k].y += v.y; a[k].z += v.z; a[k].w += v.w;
+      }
+    }
+    const int jn = j + S;
+    if ((jn & 31) == 0) {
+      cur = nxt;
+      nxt = idx[(base + jn + 32 + lane) % nidx];
+    }
+    const int32_t u = __shfl_sync(~0u, cur, jn & 31);
+    if (jn < per_warp) issue(u, s);
+    else asm volatile("cp.async.commit_group;" ::: "memory");  // keep the group count uniform
+  }
+  float sum = 0;
+  for (int k = 0; k < PER; ++k) sum += a[k].x + a[k].y + a[k].z + a[k].w;
+  if (sum == 12345.f) out[0] = sum;
+}
+
 template <typename K>
 static float time_kernel(K launch) {
   cudaEvent_t a, b;
@@ -204,12 +261,27 @@ static void run_rowb(const char *X, int64_t nrows_total, int32_t *idx_d, std::ve
       printf("ROWB %4d %s bulk S=%2d warps=%d occ=%2d CTA/SM (%3zu KB smem/SM): %8.3f ms %7.0f GB/s\n", ROWB, names[si],
              S, warps, occ, sm * occ / 1024, ms, rows * ROWB / (ms * 1e-3) / 1e9);
     };
-    bulk(k_bulk<ROWB, 4, 8>, 4, 8);
-    bulk(k_bulk<ROWB, 8, 8>, 8, 8);
-    bulk(k_bulk<ROWB, 12, 8>, 12, 8);
+    auto cpa = [&](auto kern, int S, int warps) {
+      constexpr int SLOT = (ROWB + 127) / 128 * 128;
+      const size_t sm = (size_t)warps * S * SLOT;
+      cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+      int occ = 0;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, warps * 32, sm);
+      if (occ < 1) return;
+      const int blocks = 148 * occ * 2;
+      const double rows = (double)blocks * warps * per_warp;
+      const float ms = time_kernel([&] { kern<<<blocks, warps * 32, sm>>>(X, idx_d, nidx, per_warp, out); });
+      printf("ROWB %4d %s cpa  S=%2d warps=%d occ=%2d CTA/SM (%3zu KB smem/SM, %2d warps/SM): %8.3f ms %7.0f GB/s\n",
+             ROWB, names[si], S, warps, occ, sm * occ / 1024, occ * warps, ms, rows * ROWB / (ms * 1e-3) / 1e9);
+    };
+    cpa(k_cpa<ROWB, 4, 8>, 4, 8);
+    cpa(k_cpa<ROWB, 6, 8>, 6, 8);
+    cpa(k_cpa<ROWB, 8, 8>, 8, 8);
+    cpa(k_cpa<ROWB, 12, 8>, 12, 8);
+    cpa(k_cpa<ROWB, 4, 16>, 4, 16);
+    cpa(k_cpa<ROWB, 6, 16>, 6, 16);
+    cpa(k_cpa<ROWB, 3, 16>, 3, 16);
     bulk(k_bulk<ROWB, 16, 8>, 16, 8);
-    bulk(k_bulk<ROWB, 8, 4>, 8, 4);
-    bulk(k_bulk<ROWB, 24, 4>, 24, 4);
   }
 }
 
