@@ -50,6 +50,7 @@ def parse():
     ap.add_argument("--scale", type=float, default=1.0, help="graph scale (1.0 = BASELINE size; <1 only for dev)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-rho0", action="store_true", help="skip the rho = 0 control graph (SURVEY §8(d))")
     ap.add_argument("--cpu-rows", type=int, default=0, help="oracle sample rows (0 = auto)")
     return ap.parse_args()
 
@@ -276,12 +277,52 @@ def run_ours(args):
         "gpu_launches": int(launches),
         "e2e": e2e,
     }
+    if world == 1 and not args.no_rho0 and args.rho != 0.0:
+        del model
+        torch.cuda.empty_cache()
+        out["rho0"] = rho0_control(args, dev)
     if rank == 0 and world == 1 and not args.no_cpu:
         out["cpu_baseline"] = cpu_baseline(g, inp, args)
     if rank == 0:
         print(json.dumps(out), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+def rho0_control(args, dev):
+    """The same step on the rho = 0 graph (no planted neighbour similarity, the
+    control of SURVEY §8(d)): LAS has little to find there."""
+    import torch
+    from paper_conf_ppopp_huangzzys21_b200.model import RowPartitionedGCNGAT
+    g, inp = make_inputs(args.config, 0.0, args.scale)
+    t0 = time.time()
+    m = RowPartitionedGCNGAT(g.rowptr, g.colidx, inp["W1"], inp["W2"], inp["W3"], inp["a_src"], inp["a_dst"],
+                             inp["H"], inp["Fh"], reorder=args.reorder, device=dev)
+    plan_s = time.time() - t0
+    m.load_input(torch.from_numpy(inp["X"]), non_blocking=False)
+    stream = torch.cuda.current_stream(dev)
+    for _ in range(max(2, args.warmup)):
+        m.step()
+    k = max(3, min(args.steps, 5))
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(7)] for _ in range(k)]
+    torch.cuda.synchronize(dev)
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record(stream)
+    for i in range(k):
+        m.step(events=evs[i])
+    b.record(stream)
+    torch.cuda.synchronize(dev)
+    ms = a.elapsed_time(b) / k
+    names = ["agg1_F100", "gemm1", "gemm2+allgather", "agg2_F256", "gemm3+allgather", "gat_agg_8x32"]
+    parts = [sum(evs[i][j].elapsed_time(evs[i][j + 1]) for i in range(k)) / k for j in range(6)]
+    info = m.plan.info
+    del m
+    torch.cuda.empty_cache()
+    return {"rho": 0.0, "ms_per_step": round(ms, 4), "steps": k,
+            "value": round(float(g.nnz) * (inp["F_in"] + inp["F"] + inp["H"] * inp["Fh"]) / (ms * 1e-3) / 1e9, 3),
+            "breakdown_ms": {n: round(v, 4) for n, v in zip(names, parts)},
+            "plan": {"build_s": round(plan_s, 2), "gen_s": round(inp["gen_s"], 2), "n_clusters": info["n_clusters"]},
+            "note": "control graph without planted neighbour similarity (SURVEY §8(d) rho = 0); same step"}
 
 
 # --------------------------------------------------------------------------- #

@@ -317,6 +317,20 @@ int gnn_set_gemm_impl(int impl);
 gnn_status gnn_set_agg_mapping(int32_t vec, int32_t lanes, int32_t nv);
 
 /*
+ * Load-balance trace of the aggregation kernels (the "Balanced vs Actual"
+ * measurement of Fig 8; process-wide, NULL = off).  When set,
+ * every later graph-op launch resets trace_dev (device, 8 x uint64) and its
+ * persistent workers record: [0] the sum over workers of the time spent in
+ * their work units (ns, %globaltimer), [1] the number of workers, [2] the
+ * earliest worker start, [3] the latest worker end, [4] work units, [5] the
+ * longest single-worker busy time.  Balanced time = [0] / [1] (all workers
+ * are resident at once: perfect balance); actual = [3] - [2].  Costs two
+ * timer reads per unit; for measurement only.  The caller keeps the buffer
+ * alive while set.
+ */
+void gnn_set_agg_trace(void *trace_dev);
+
+/*
  * NG bound of an existing plan (reading R8): rebuilds the work
  * units and the task-ordered index stream for group_size (> 0: groups of at
  * most group_size entries; 0: never split rows; -1: the default rule); the

@@ -474,6 +474,8 @@ gnn_status gnn_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw, fl
 
 int gnn_set_gemm_impl(int impl) { return set_gemm_impl(impl); }
 
+void gnn_set_agg_trace(void *trace_dev) { set_agg_trace(trace_dev); }
+
 gnn_status gnn_set_agg_mapping(int32_t vec, int32_t lanes, int32_t nv) {
   GNN_TRY({
     if (!set_agg_mapping(vec, lanes, nv)) {

@@ -141,6 +141,7 @@ cudaError_t launch_sage_lstm(const gnn_plan_s *p, const int32_t *table, int32_t 
 bool set_agg_mapping(int32_t vec, int32_t lanes, int32_t nv);
 bool mapping_supported(int32_t vec, int32_t lanes, int32_t nv);
 bool agg_override_active();
+void set_agg_trace(void *dev_buf);
 bool agg_mapping_ok(const AggArgs &a, int32_t fh_or_0, int32_t vec, int32_t lanes, int32_t nv);
 gnn_status rebuild_schedule(gnn_plan_s *p, int64_t group_size);
 int64_t default_group_size(int64_t n, int64_t nnz);

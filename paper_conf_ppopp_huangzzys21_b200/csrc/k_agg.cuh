@@ -75,7 +75,17 @@ struct KParams {
   int32_t deterministic;
   int32_t nch;        // feature chunks per row (arrival counters per multi-unit row)
   int32_t n_persist;  // persistent CTAs
+  // load-balance trace (Fig 8 analogue), nullable: [0] sum of
+  // worker busy ns, [1] workers, [2] earliest worker start, [3] latest worker
+  // end (%globaltimer ns), [4] units, [5] longest worker busy ns
+  unsigned long long *trace;
 };
+
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
 
 // Cache policy of the three streams (A/B switches, compile time):
 //   GNN_LD_NA  gathered source rows bypass L1 allocation (L1 keeps the
@@ -666,6 +676,156 @@ __device__ __forceinline__ void group_chain_att(const KParams &p, const int32_t 
   }
 }
 
+// ---------------------------------------------------------------------------
+// cp.async-staged group chain (sum / mean / max with any weight, GAT): the
+// source rows of a group stream through a per-warp ring of S shared-memory
+// slots with cp.async (LDGSTS, L2 -> shared, bypassing L1 and registers), so
+// the bytes in flight are bounded by shared memory rather than registers
+// (scripts/gather_roofline.cu on this B200: random 1 KB rows from a 100 MB
+// working set 18.6 TB/s vs 10.9 TB/s for register loads; HBM-bound 7.3 TB/s
+// either way).  Worker = one warp; lane owns features c0 + n*128 + 4*lane
+// (n < NV): the (4, 32, NV) lane mapping, so partials, merge and epilogue
+// are shared with the register kernel and results are bit-identical (the
+// chain of R9 is per feature, in CSR order).  Every lane copies exactly the
+// 16-byte vectors it later reads; per-edge extras (GCN nsrc[u], explicit
+// edge weight, GAT scores s_u[h]) are 4-byte copies by lanes 0..H-1 into the
+// slot tail and read by all lanes after a __syncwarp.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void cp_async16(uint32_t dst, const void *src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async4(uint32_t dst, const void *src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(dst), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+// slot size in floats: NV*128 features + the extras (H <= 32 GAT scores, or one weight), 16-byte multiple
+template <int MODE, int NV>
+__host__ __device__ constexpr int cp_slot_floats() {
+  return NV * 128 + (MODE == M_GAT ? 32 : 4);
+}
+
+template <int MODE, int NV, int S>
+__device__ __forceinline__ void group_chain_cp(const KParams &p, const int32_t *idx, int32_t len, int32_t beg,
+                                               int32_t row, int32_t c0, int lane, float *ring,
+                                               Part<MODE, 4, NV> &G) {
+  constexpr int VEC = 4;
+  constexpr int SLOT = cp_slot_floats<MODE, NV>();
+  part_init(G);
+  const int weight = p.weight;
+  const uint32_t ring_s = (uint32_t)__cvta_generic_to_shared(ring);
+  bool valid[NV];
+  int32_t head[NV];
+  float tv[NV], nmb[NV], seen[NV];
+  const bool one = MODE == M_GAT && len == 1;
+#pragma unroll
+  for (int n = 0; n < NV; ++n) {
+    const int32_t f = c0 + (n * 32 + lane) * VEC;
+    valid[n] = f < p.F;
+    head[n] = 0;
+    tv[n] = 0.0f;
+    nmb[n] = 0.0f;
+    seen[n] = -INFINITY;
+    if constexpr (MODE == M_GAT) {
+      head[n] = valid[n] ? f / p.Fh : 0;
+      tv[n] = valid[n] ? __ldg(p.t + (int64_t)row * p.ldt + head[n]) : 0.0f;
+      const float mb = valid[n] ? leaky_f(fkey_decode(__ldg(p.smax + head[n])) + tv[n], p.slope) : 0.0f;
+      G.m[n] = mb;
+      nmb[n] = -mb * kLog2e;
+    }
+  }
+  const float *xl = p.X + c0 + lane * VEC;
+  // issue the copies of edge e (source row u) into slot e % S; one commit group per edge
+  auto issue = [&](int32_t u, int32_t e) {
+    const uint32_t sl = ring_s + (uint32_t)((e % S) * SLOT * 4);
+    if (e < len) {
+#pragma unroll
+      for (int n = 0; n < NV; ++n)
+        if (valid[n]) cp_async16(sl + (uint32_t)((n * 128 + lane * VEC) * 4), xl + (int64_t)u * p.ldx + n * 128);
+      if constexpr (MODE == M_GAT) {
+        if (lane < p.H) cp_async4(sl + (uint32_t)((NV * 128 + lane) * 4), p.X + (int64_t)u * p.ldx + p.F + lane);
+      } else {
+        if (lane == 0) {
+          if (weight == GNN_W_GCN) cp_async4(sl + (uint32_t)(NV * 128 * 4), p.g.nsrc + u);
+          else if (weight == GNN_W_EDGE) cp_async4(sl + (uint32_t)(NV * 128 * 4), p.edge_w + beg + e);
+        }
+      }
+    }
+    cp_commit();
+  };
+#pragma unroll 1
+  for (int pass = 0;; ++pass) {
+    int32_t cur = lane < len ? ld_stream_i32(idx + lane) : 0;
+    int32_t nxt = 32 + lane < len ? ld_stream_i32(idx + 32 + lane) : 0;
+#pragma unroll
+    for (int q = 0; q < S; ++q) issue(__shfl_sync(0xffffffffu, cur, q), q);
+    for (int32_t e = 0; e < len; ++e) {
+      cp_wait<S - 1>();
+      __syncwarp();
+      const float *sl = ring + (e % S) * SLOT;
+      if constexpr (MODE == M_GAT) {
+#pragma unroll
+        for (int n = 0; n < NV; ++n) {
+          if (!valid[n]) continue;
+          const float4 x4 = *reinterpret_cast<const float4 *>(sl + n * 128 + lane * VEC);
+          const float v[4] = {x4.x, x4.y, x4.z, x4.w};
+          const float sco = leaky_f(sl[NV * 128 + head[n]] + tv[n], p.slope);
+          seen[n] = fmaxf(seen[n], sco);
+          const float ex = one ? 1.0f : ex2_f(fmaf(sco, kLog2e, nmb[n]));
+          G.l[n] += ex;
+          fma_vec<VEC>(G.a[n], v, ex);
+        }
+      } else {
+        const float w = (weight == GNN_W_GCN || weight == GNN_W_EDGE) ? sl[NV * 128] : 1.0f;
+#pragma unroll
+        for (int n = 0; n < NV; ++n) {
+          if (!valid[n]) continue;
+          const float4 x4 = *reinterpret_cast<const float4 *>(sl + n * 128 + lane * VEC);
+          const float v[4] = {x4.x, x4.y, x4.z, x4.w};
+          if constexpr (MODE == M_MAX) {
+#pragma unroll
+            for (int i = 0; i < VEC; ++i) G.a[n][i] = fmaxf(G.a[n][i], w * v[i]);
+          } else {
+            fma_vec<VEC>(G.a[n], v, w);
+          }
+        }
+      }
+      __syncwarp();  // every lane has read slot e % S before it is refilled
+      const int32_t pe = e + S;
+      if ((pe & 31) == 0) {
+        cur = nxt;
+        nxt = pe + 32 + lane < len ? ld_stream_i32(idx + pe + 32 + lane) : 0;
+      }
+      issue(__shfl_sync(0xffffffffu, cur, pe & 31), pe);
+    }
+    if constexpr (MODE != M_GAT) {
+      break;
+    } else {
+      if (one) {
+#pragma unroll
+        for (int n = 0; n < NV; ++n) G.m[n] = seen[n];
+        break;
+      }
+      // bound too loose for some head of this warp: redo against the exact max (R9 GAT)
+      bool loose = false;
+#pragma unroll
+      for (int n = 0; n < NV; ++n) loose |= valid[n] && !(G.m[n] - seen[n] <= kGatSlack);
+      if (pass == 1 || !__any_sync(0xffffffffu, loose)) break;
+#pragma unroll
+      for (int n = 0; n < NV; ++n) {
+        G.m[n] = seen[n];
+        nmb[n] = -seen[n] * kLog2e;
+        G.l[n] = 0.0f;
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) G.a[n][i] = 0.0f;
+      }
+    }
+  }
+}
+
 // merge the group partials of a long row in group order (R9), epilogue, store
 template <int MODE, int VEC, int NV, int LANES>
 __device__ __forceinline__ void merge_row(const KParams &p, const float *base, int32_t ngrp, int32_t row,
@@ -705,13 +865,16 @@ __device__ __forceinline__ void merge_row(const KParams &p, const float *base, i
 // one computing unit).  A row with a single group is finished here (epilogue +
 // store); the groups of a longer row leave their partials in the workspace and
 // the last one to arrive merges them in group order (R9).
-template <int MODE, int VEC, int NV, int LANES>
+template <int MODE, int VEC, int NV, int LANES, int S = 0>
 __device__ __forceinline__ void process_unit(const KParams &p, int4 d, int32_t len, int32_t c0, int32_t ci, int lane,
-                                             unsigned mask) {
+                                             unsigned mask, float *ring = nullptr) {
   const DevGraph &g = p.g;
   const int32_t tpos = d.x, beg = d.y, row = d.z, m = d.w;
   Part<MODE, VEC, NV> G;
-  if constexpr (MODE > M_GAT)
+  if constexpr (S > 0) {
+    static_assert(VEC == 4 && LANES == 32 && MODE <= M_GAT, "cp.async chain: (4, 32, NV) mapping");
+    group_chain_cp<MODE, NV, S>(p, g.colidx_t + tpos, len, beg, row, c0, lane, ring, G);
+  } else if constexpr (MODE > M_GAT)
     group_chain_att<MODE, VEC, NV, LANES>(p, g.colidx_t + tpos, len, beg, row, c0, lane, mask, G);
   else
     group_chain<MODE, VEC, NV, LANES>(p, g.colidx_t + tpos, len, beg, row, c0, lane, mask, G);
@@ -776,10 +939,22 @@ __device__ __forceinline__ void process_unit(const KParams &p, int4 d, int32_t l
 #ifndef GNN_AGG_MINB_GAT
 #define GNN_AGG_MINB_GAT 4
 #endif
-template <int MODE, int VEC, int NV, int LANES>
-__global__ void __launch_bounds__(256, vec_score(MODE) ? 2 : (is_att(MODE) ? GNN_AGG_MINB_GAT : GNN_AGG_MINB))
+#ifndef GNN_AGG_MINB_CP
+#define GNN_AGG_MINB_CP 5
+#endif
+// slots per warp of the cp.async ring (S > 0 selects the cp.async chain)
+#ifndef GNN_CP_S1
+#define GNN_CP_S1 8  // NV = 1: rows <= 128 features
+#endif
+#ifndef GNN_CP_S2
+#define GNN_CP_S2 4  // NV = 2: rows <= 256 features
+#endif
+template <int MODE, int VEC, int NV, int LANES, int S = 0>
+__global__ void __launch_bounds__(256, S > 0 ? GNN_AGG_MINB_CP
+                                             : (vec_score(MODE) ? 2 : (is_att(MODE) ? GNN_AGG_MINB_GAT : GNN_AGG_MINB)))
     k_aggregate(const KParams p) {
   constexpr int CW = LANES * VEC * NV;
+  extern __shared__ __align__(16) float cp_smem[];
   const int tid = threadIdx.x;
   const int lane = tid & (LANES - 1);
   const unsigned mask =
@@ -796,6 +971,8 @@ __global__ void __launch_bounds__(256, vec_score(MODE) ? 2 : (is_att(MODE) ? GNN
   }
   const int32_t nunits = g.n_units;
   int32_t ci = 0;
+  unsigned long long t_start = 0, busy = 0, n_done = 0;
+  if (p.trace) t_start = gtimer();
   for (int32_t c0 = 0; c0 < p.F; c0 += CW, ++ci) {
     int32_t *ctr = p.ws_unit + ci;
     // the next unit (id and descriptor) is claimed while the current one streams
@@ -809,6 +986,7 @@ __global__ void __launch_bounds__(256, vec_score(MODE) ? 2 : (is_att(MODE) ? GNN
       dnx = __ldg(&g.unit_desc[u + 1].x);
     }
     while (u < nunits) {
+      const unsigned long long t_unit = p.trace ? gtimer() : 0ull;
       int32_t un = 0;
       if (lane == 0) un = atomicAdd(ctr, 1);
       un = __shfl_sync(mask, un, 0, LANES);
@@ -818,11 +996,27 @@ __global__ void __launch_bounds__(256, vec_score(MODE) ? 2 : (is_att(MODE) ? GNN
         dn = __ldg(g.unit_desc + un);
         dnxn = __ldg(&g.unit_desc[un + 1].x);
       }
-      process_unit<MODE, VEC, NV, LANES>(p, d, dnx - d.x, c0, ci, lane, mask);
+      if constexpr (S > 0)
+        process_unit<MODE, VEC, NV, LANES, S>(p, d, dnx - d.x, c0, ci, lane, mask,
+                                              cp_smem + (tid >> 5) * S * cp_slot_floats<MODE, NV>());
+      else
+        process_unit<MODE, VEC, NV, LANES>(p, d, dnx - d.x, c0, ci, lane, mask);
+      if (p.trace) {
+        busy += gtimer() - t_unit;
+        ++n_done;
+      }
       u = un;
       d = dn;
       dnx = dnxn;
     }
+  }
+  if (p.trace && lane == 0) {
+    atomicAdd(p.trace + 0, busy);
+    atomicAdd(p.trace + 1, 1ull);
+    atomicMin(p.trace + 2, t_start);
+    atomicMax(p.trace + 3, gtimer());
+    atomicAdd(p.trace + 4, n_done);
+    atomicMax(p.trace + 5, busy);
   }
 }
 
@@ -831,15 +1025,21 @@ __global__ void __launch_bounds__(256, vec_score(MODE) ? 2 : (is_att(MODE) ? GNN
 // ---------------------------------------------------------------------------
 struct Mapping {
   int vec, lanes, nv;
+  int cp = 0;  // 1: the cp.async-staged chain with the (4, 32, nv) mapping
 };
 int num_sms();
 
 template <typename KFN>
 cudaError_t launch_persistent(KFN fn, int &occ, const KParams &kp_in, int32_t units, int cw, int lanes,
-                                     int threads, cudaStream_t s) {
+                                     int threads, cudaStream_t s, size_t smem = 0) {
   if (occ == 0) {
-    cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, 0);  // all of it to L1
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, threads, 0);
+    if (smem > 0) {  // cp.async ring: shared memory first
+      cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    } else {
+      cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, 0);  // all of it to L1
+    }
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, threads, smem);
     if (occ <= 0) occ = 1;
   }
   KParams kp = kp_in;
@@ -854,8 +1054,13 @@ cudaError_t launch_persistent(KFN fn, int &occ, const KParams &kp_in, int32_t un
   if (e == cudaSuccess && kp.g.n_multi > 0 && !kp.deterministic && kp.mode != M_MAX && !is_att(kp.mode))
     e = cudaMemsetAsync(kp.ws_acc, 0, sizeof(float) * (size_t)kp.g.n_multi * kp.FW, s);
   if (e != cudaSuccess) return e;
+  if (e == cudaSuccess && kp.trace) {
+    e = cudaMemsetAsync(kp.trace, 0, 8 * sizeof(unsigned long long), s);
+    if (e == cudaSuccess) e = cudaMemsetAsync(kp.trace + 2, 0xff, sizeof(unsigned long long), s);
+  }
+  if (e != cudaSuccess) return e;
   const int64_t blocks = (int64_t)kp.n_persist + (kp.g.n_empty + 31) / 32;
-  fn<<<(unsigned)blocks, threads, 0, s>>>(kp);
+  fn<<<(unsigned)blocks, threads, smem, s>>>(kp);
   count_launch();
   return cudaGetLastError();
 }
@@ -865,6 +1070,16 @@ cudaError_t launch_one(const KParams &kp, int threads, cudaStream_t s) {
   constexpr int CW = LANES * VEC * NV;
   static int occ = 0;
   return launch_persistent(k_aggregate<MODE, VEC, NV, LANES>, occ, kp, kp.g.n_units, CW, LANES, threads, s);
+}
+
+// the cp.async-staged kernel: (4, 32, NV) mapping, S ring slots per warp
+template <int MODE, int NV>
+cudaError_t launch_cp(const KParams &kp, int threads, cudaStream_t s) {
+  constexpr int S = NV == 1 ? GNN_CP_S1 : GNN_CP_S2;
+  constexpr int CW = 32 * 4 * NV;
+  static int occ = 0;
+  const size_t smem = sizeof(float) * (size_t)(threads / 32) * S * cp_slot_floats<MODE, NV>();
+  return launch_persistent(k_aggregate<MODE, 4, NV, 32, S>, occ, kp, kp.g.n_units, CW, 32, threads, s, smem);
 }
 
 template <int MODE, int VEC>
@@ -891,6 +1106,9 @@ cudaError_t dispatch_lanes(const KParams &kp, const Mapping &m, int threads, cud
 
 template <int MODE>
 cudaError_t dispatch_vec(const KParams &kp, const Mapping &m, int threads, cudaStream_t s) {
+  if constexpr (MODE <= M_GAT) {
+    if (m.cp) return m.nv == 1 ? launch_cp<MODE, 1>(kp, threads, s) : launch_cp<MODE, 2>(kp, threads, s);
+  }
 #ifdef GNN_DEV_SUBSET  // dev builds: only the C5 bench instantiations (fast compile)
   if (m.lanes == 32 && m.nv == 1 && m.vec == 8) return launch_one<MODE, 8, 1, 32>(kp, threads, s);
   if (m.lanes == 32 && m.nv == 1 && m.vec == 4) return launch_one<MODE, 4, 1, 32>(kp, threads, s);

@@ -230,6 +230,10 @@ bool set_agg_mapping(int32_t vec, int32_t lanes, int32_t nv) {
 
 bool agg_override_active() { return g_override.vec != 0; }
 
+// process-wide load-balance trace buffer (gnn_set_agg_trace), device, 8 x u64
+static unsigned long long *g_trace = nullptr;
+void set_agg_trace(void *dev_buf) { g_trace = reinterpret_cast<unsigned long long *>(dev_buf); }
+
 static bool is_pow2(int x) { return x > 0 && (x & (x - 1)) == 0; }
 
 static bool vec_admissible(const AggArgs &a, int32_t fh_or_0, int v) {
@@ -260,12 +264,32 @@ bool agg_mapping_ok(const AggArgs &a, int32_t fh_or_0, int32_t vec, int32_t lane
   return mapping_supported(vec, lanes, nv) && mapping_ok(a, fh_or_0, Mapping{vec, lanes, nv});
 }
 
+// cp.async-staged kernel (a4 rule): sum / mean / max and
+// GAT with 16-byte vectors, rows of >= 64 features; one warp per group, 128
+// (NV = 1) or 256 (NV = 2) features per sweep.  A/B switch: env GNN_AGG_CP=0.
+static int g_agg_cp = -1;
+static bool cp_admissible(const gnn_plan_s *p, const AggArgs &a, int32_t fh_or_0) {
+  (void)p;
+  if (g_agg_cp < 0) {
+    const char *e = getenv("GNN_AGG_CP");
+    g_agg_cp = (e && e[0] == '0') ? 0 : 1;
+  }
+  if (!g_agg_cp || a.mode > M_GAT || a.F < 64) return false;
+  if (a.mode == M_GAT && (a.H > 32 || fh_or_0 % 4 != 0)) return false;
+  return vec_admissible(a, fh_or_0, 4);
+}
+
 static Mapping choose_mapping(const gnn_plan_s *p, const AggArgs &a, int32_t fh_or_0) {
   Mapping m{1, 4, 1};
   if (mapping_ok(a, fh_or_0, g_override)) return g_override;
   // the plan's tuned mapping (gnn_tune_aggregate) for this width
   const Mapping t{p->tuned_vec, p->tuned_lanes, p->tuned_nv};
   if (p->tuned_F == a.F && mapping_ok(a, fh_or_0, t)) return t;
+  if (cp_admissible(p, a, fh_or_0)) {
+    Mapping c{4, 32, a.F > 128 ? 2 : 1};
+    c.cp = 1;
+    return c;
+  }
   const int cands[4] = {8, 4, 2, 1};
   m.vec = 0;
   for (int v : cands) {
@@ -387,6 +411,7 @@ gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, siz
   kp.FW = slot_width(mode, a.F, a.H);
   kp.nmeta = att_meta(mode, a.F, a.H);
   kp.deterministic = a.deterministic;
+  kp.trace = g_trace;
   const WsLayout L = ws_layout(p, mode, a.F, a.H);
   char *w = reinterpret_cast<char *>(ws);
   kp.ws_unit = reinterpret_cast<int32_t *>(w + L.unit);

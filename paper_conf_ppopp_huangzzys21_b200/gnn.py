@@ -93,6 +93,7 @@ _SIGS = {
     "gnn_gemm_workspace_size": (_SZ, [_I64, _I32, _I32]),
     "gnn_set_gemm_impl": (ctypes.c_int, [ctypes.c_int]),
     "gnn_set_agg_mapping": (ctypes.c_int, [_I32, _I32, _I32]),
+    "gnn_set_agg_trace": (None, [_P]),
     "gnn_gcn_layer": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _I64, _I32, _I32, _I32, _P, _I64, _P, _SZ, _P]),
     "gnn_gcn_aggregate_prescaled": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _I64, _I32, _P, _SZ, _P]),
     "gnn_gat_fold_weights": (ctypes.c_int, [_P, _P, _P, _I32, _I32, _I32, _P, _I64, _P]),

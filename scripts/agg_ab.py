@@ -21,7 +21,7 @@ import paper_conf_ppopp_huangzzys21_b200 as G  # noqa: E402
 
 tag = sys.argv[1] if len(sys.argv) > 1 and not sys.argv[1].startswith("--") else os.path.basename(
     os.path.dirname(G.gnn.LIB_PATH))
-GPATH, PPATH = "/tmp/agg_ab_c5.npz", "/tmp/agg_ab_c5.gnnplan"
+GPATH, PPATH = "/tmp/agg_ab_c5_sym.npz", "/tmp/agg_ab_c5_sym.gnnplan"
 t0 = time.time()
 if os.path.exists(GPATH):
     z = np.load(GPATH)
