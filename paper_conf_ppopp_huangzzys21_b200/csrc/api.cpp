@@ -187,7 +187,7 @@ gnn_status create_plan(int64_t n, int64_t n_src, int64_t nnz, const int64_t *row
     if (e == cudaSuccess) p->dev_allocs.push_back(d_colidx);
     if (e == cudaSuccess) e = cudaMalloc(&d_nsrc, sizeof(float) * (n_src > 0 ? n_src : 1));
     if (e == cudaSuccess) p->dev_allocs.push_back(d_nsrc);
-    if (e == cudaSuccess) e = cudaMalloc(&d_ndst, sizeof(float) * (n > 0 ? n : 1));
+    if (e == cudaSuccess) e = cudaMalloc(&d_ndst, sizeof(float) * (size_t)(n + 4));  // + 4: 16-byte bulk reads
     if (e == cudaSuccess) p->dev_allocs.push_back(d_ndst);
     if (e == cudaSuccess) e = cudaMalloc(&d_dout, sizeof(int32_t) * (n_src > 0 ? n_src : 1));
     if (e == cudaSuccess) p->dev_allocs.push_back(d_dout);

@@ -7,6 +7,7 @@
 #include <cuda_runtime.h>
 #include <math.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include <algorithm>
 
@@ -275,8 +276,9 @@ __device__ __forceinline__ float epi(const KParams &p, int mode, float a, float 
 
 template <int MODE, int VEC, int NV, int LANES>
 __device__ __forceinline__ void store_row(const KParams &p, int32_t row, int32_t deg, int32_t c0,
-                                          int lane, const Part<MODE, VEC, NV> &P) {
-  const float ndst = (!is_att(MODE) && scales_dst(p.weight)) ? __ldg(p.g.ndst + row) : 1.0f;
+                                          int lane, const Part<MODE, VEC, NV> &P, const float *ndst_pre = nullptr) {
+  const float ndst =
+      (!is_att(MODE) && scales_dst(p.weight)) ? (ndst_pre ? *ndst_pre : __ldg(p.g.ndst + row)) : 1.0f;
   const float deg_f = (float)deg;
 #pragma unroll
   for (int n = 0; n < NV; ++n) {
@@ -865,6 +867,11 @@ __device__ __forceinline__ void merge_row(const KParams &p, const float *base, i
 // one computing unit).  A row with a single group is finished here (epilogue +
 // store); the groups of a longer row leave their partials in the workspace and
 // the last one to arrive merges them in group order (R9).
+template <int MODE, int VEC, int NV, int LANES>
+__device__ __forceinline__ void finish_unit(const KParams &p, const Part<MODE, VEC, NV> &G, int32_t row, int32_t beg,
+                                            int32_t m, int32_t len, int32_t c0, int32_t ci, int lane, unsigned mask,
+                                            const float *ndst_pre);
+
 template <int MODE, int VEC, int NV, int LANES, int S = 0>
 __device__ __forceinline__ void process_unit(const KParams &p, int4 d, int32_t len, int32_t c0, int32_t ci, int lane,
                                              unsigned mask, float *ring = nullptr) {
@@ -878,11 +885,22 @@ __device__ __forceinline__ void process_unit(const KParams &p, int4 d, int32_t l
     group_chain_att<MODE, VEC, NV, LANES>(p, g.colidx_t + tpos, len, beg, row, c0, lane, mask, G);
   else
     group_chain<MODE, VEC, NV, LANES>(p, g.colidx_t + tpos, len, beg, row, c0, lane, mask, G);
-  const int32_t rb = g.rowptr[row], re = g.rowptr[row + 1];
+  finish_unit<MODE, VEC, NV, LANES>(p, G, row, beg, m, len, c0, ci, lane, mask, nullptr);
+}
+
+// a finished group: a whole row -> epilogue + store (deg = len); a group of a
+// longer row -> its partial to the workspace, the last group to arrive merges
+// them in group order (R9)
+template <int MODE, int VEC, int NV, int LANES>
+__device__ __forceinline__ void finish_unit(const KParams &p, const Part<MODE, VEC, NV> &G, int32_t row, int32_t beg,
+                                            int32_t m, int32_t len, int32_t c0, int32_t ci, int lane, unsigned mask,
+                                            const float *ndst_pre) {
+  const DevGraph &g = p.g;
   if (m < 0) {
-    store_row<MODE, VEC, NV, LANES>(p, row, re - rb, c0, lane, G);
+    store_row<MODE, VEC, NV, LANES>(p, row, len, c0, lane, G, ndst_pre);
     return;
   }
+  const int32_t rb = g.rowptr[row], re = g.rowptr[row + 1];
   const int32_t ng = g.ng;
   const int32_t ngrp = 1 + (re - rb - 1) / ng;
   const int32_t k = (beg - rb) / ng;
@@ -940,14 +958,14 @@ __device__ __forceinline__ void process_unit(const KParams &p, int4 d, int32_t l
 #define GNN_AGG_MINB_GAT 4
 #endif
 #ifndef GNN_AGG_MINB_CP
-#define GNN_AGG_MINB_CP 5
+#define GNN_AGG_MINB_CP 4
 #endif
 // slots per warp of the cp.async ring (S > 0 selects the cp.async chain)
 #ifndef GNN_CP_S1
-#define GNN_CP_S1 8  // NV = 1: rows <= 128 features
+#define GNN_CP_S1 12  // NV = 1: rows <= 128 features
 #endif
 #ifndef GNN_CP_S2
-#define GNN_CP_S2 4  // NV = 2: rows <= 256 features
+#define GNN_CP_S2 6  // NV = 2: rows <= 256 features
 #endif
 template <int MODE, int VEC, int NV, int LANES, int S = 0>
 __global__ void __launch_bounds__(256, S > 0 ? GNN_AGG_MINB_CP
@@ -1020,12 +1038,45 @@ __global__ void __launch_bounds__(256, S > 0 ? GNN_AGG_MINB_CP
   }
 }
 
+// GAT, a group whose softmax bound was too loose (R9 GAT): recompute it
+// against its exact maximum with direct loads (rare path); 32 lanes, lane's
+// vector n at features c0 + (n * 32 + lane) * VEC
+template <int VEC, int NV>
+__device__ __forceinline__ void gat_recompute_v(const KParams &p, int32_t tpos, int32_t len, int32_t c0, int lane,
+                                                const bool (&valid)[NV], const int32_t (&head)[NV],
+                                                const float (&tv)[NV], Part<M_GAT, VEC, NV> &G, float (&seen)[NV]) {
+  const int32_t *idx = p.g.colidx_t + tpos;
+  float nmb[NV];
+#pragma unroll
+  for (int n = 0; n < NV; ++n) {
+    G.m[n] = seen[n];
+    nmb[n] = -seen[n] * kLog2e;
+    G.l[n] = 0.0f;
+#pragma unroll
+    for (int i = 0; i < VEC; ++i) G.a[n][i] = 0.0f;
+  }
+  const float *xl = p.X + c0 + lane * VEC;
+  for (int32_t e = 0; e < len; ++e) {
+    const int32_t u = ld_stream_i32(idx + e);
+#pragma unroll
+    for (int n = 0; n < NV; ++n) {
+      if (!valid[n]) continue;
+      float v[VEC];
+      ldv<VEC>(xl + (int64_t)u * p.ldx + n * 32 * VEC, v);
+      const float sco = leaky_f(__ldg(p.X + (int64_t)u * p.ldx + p.F + head[n]) + tv[n], p.slope);
+      const float ex = ex2_f(fmaf(sco, kLog2e, nmb[n]));
+      G.l[n] += ex;
+      fma_vec<VEC>(G.a[n], v, ex);
+    }
+  }
+}
+
 // ---------------------------------------------------------------------------
 // launch templates
 // ---------------------------------------------------------------------------
 struct Mapping {
   int vec, lanes, nv;
-  int cp = 0;  // 1: the cp.async-staged chain with the (4, 32, nv) mapping
+  int cp = 0;  // 1: the cp.async-staged chain with the (4, 32, nv) mapping; 2: the TMA gather4 streaming kernel
 };
 int num_sms();
 
@@ -1045,7 +1096,15 @@ cudaError_t launch_persistent(KFN fn, int &occ, const KParams &kp_in, int32_t un
   KParams kp = kp_in;
   kp.nch = (kp.F + cw - 1) / cw;
   const int64_t workers_per_cta = threads / lanes;
-  kp.n_persist = (int32_t)std::min<int64_t>((int64_t)num_sms() * occ,
+  // A/B knob: cap on resident CTAs per SM (fewer concurrent groups = a narrower
+  // window of the task order in flight = more L2 reuse, fewer rows in flight)
+  static int cap = -1;
+  if (cap < 0) {
+    const char *e = getenv("GNN_AGG_CTAS_PER_SM");
+    cap = e ? atoi(e) : 0;
+  }
+  const int occ_used = (cap > 0 && cap < occ) ? cap : occ;
+  kp.n_persist = (int32_t)std::min<int64_t>((int64_t)num_sms() * occ_used,
                                             std::max<int64_t>(1, (units + workers_per_cta - 1) / workers_per_cta));
   if (kp.nch > kp.n_unit_ctr) return cudaErrorInvalidValue;  // mapping wider than the workspace sizing
   cudaError_t e = cudaMemsetAsync(kp.ws_unit, 0, sizeof(int32_t) * (size_t)kp.n_unit_ctr, s);
@@ -1128,6 +1187,8 @@ cudaError_t dispatch_vec(const KParams &kp, const Mapping &m, int threads, cudaS
 }
 
 cudaError_t dispatch_sum(const KParams &kp, const Mapping &m, int threads, cudaStream_t s);
+bool g4_admissible(const KParams &kp, int32_t n_src);
+cudaError_t launch_g4(const KParams &kp, int32_t n_src, cudaStream_t s);
 cudaError_t dispatch_max(const KParams &kp, const Mapping &m, int threads, cudaStream_t s);
 cudaError_t dispatch_gat(const KParams &kp, const Mapping &m, int threads, cudaStream_t s);
 cudaError_t dispatch_att(const KParams &kp, const Mapping &m, int threads, cudaStream_t s);

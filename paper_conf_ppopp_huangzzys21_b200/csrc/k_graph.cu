@@ -272,7 +272,7 @@ static bool cp_admissible(const gnn_plan_s *p, const AggArgs &a, int32_t fh_or_0
   (void)p;
   if (g_agg_cp < 0) {
     const char *e = getenv("GNN_AGG_CP");
-    g_agg_cp = (e && e[0] == '0') ? 0 : 1;
+    g_agg_cp = (e && e[0] == '0') ? 0 : (e && e[0] == '1') ? 1 : 2;  // default: gather4 streaming where it applies
   }
   if (!g_agg_cp || a.mode > M_GAT || a.F < 64) return false;
   if (a.mode == M_GAT && (a.H > 32 || fh_or_0 % 4 != 0)) return false;
@@ -286,9 +286,14 @@ static Mapping choose_mapping(const gnn_plan_s *p, const AggArgs &a, int32_t fh_
   const Mapping t{p->tuned_vec, p->tuned_lanes, p->tuned_nv};
   if (p->tuned_F == a.F && mapping_ok(a, fh_or_0, t)) return t;
   if (cp_admissible(p, a, fh_or_0)) {
+    // rows wider than 128 features: the gather4 streaming kernel (cp = 2,
+    // launch_aggregate falls back to the cp.async chain if it cannot take the
+    // call); up to 128: the cp.async chain for sum / mean / max, the register
+    // kernel for GAT (measured faster there)
     Mapping c{4, 32, a.F > 128 ? 2 : 1};
-    c.cp = 1;
-    return c;
+    c.cp = a.F > 128 ? g_agg_cp : 1;
+    if (c.cp == 1 && a.mode == M_GAT) c.cp = 0;
+    if (c.cp) return c;
   }
   const int cands[4] = {8, 4, 2, 1};
   m.vec = 0;
@@ -419,7 +424,7 @@ gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, siz
   kp.ws_cnt = reinterpret_cast<int32_t *>(w + L.cnt);
   kp.ws_acc = reinterpret_cast<float *>(w + L.acc);
   kp.ws_part = reinterpret_cast<float *>(w + L.part);
-  const Mapping m = choose_mapping(p, a, is_att(mode) ? a.Fh : 0);
+  Mapping m = choose_mapping(p, a, is_att(mode) ? a.Fh : 0);
   if (m.vec == 0) {
     set_error("no supported lane mapping for this width / head size (GaAN, Gene: Fh/vec must be a power of 2 <= 32)");
     return GNN_ERR_UNSUPPORTED;
@@ -432,6 +437,17 @@ gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, siz
   if (e == cudaSuccess && mode == M_SYM) e = launch_score_max(a.X + a.F + a.H, a.ldx, p->n_src, a.H, 1, smax + a.H, s);
   if (e == cudaSuccess && mode == M_GAAN) e = launch_score_max(a.X + a.F, a.ldx, p->n_src, a.H, a.Fh, smax, s);
   if (e != cudaSuccess) return cuda_status(e, "score max launch");
+  if (m.cp == 2) {  // gather4 streaming kernel (k_agg_g4.cu)
+    KParams kq = kp;
+    kq.n_unit_ctr = kp.n_unit_ctr;
+    if (g4_admissible(kq, (int32_t)p->n_src)) {
+      e = launch_g4(kq, (int32_t)p->n_src, s);
+      if (e != cudaErrorNotSupported) return cuda_status(e, "aggregate launch (gather4)");
+      (void)cudaGetLastError();
+    }
+    m.cp = 1;  // the cp.async chain with the same (4, 32, NV) mapping
+    if (mode == M_GAT) m.cp = 0;
+  }
   switch (mode) {
     case M_SUM:
     case M_MEAN: e = dispatch_sum(kp, m, threads, s); break;

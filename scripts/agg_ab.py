@@ -83,6 +83,12 @@ def run(label):
           f"fp {fp(Y1)} {fp(Y2)} {fp(Yg)} (prep {prep:.0f}s)", flush=True)
 
 
+if "--once" in sys.argv:  # one call of each kernel (for ncu)
+    G.aggregate(plan, X1, "sum", "gcn", out=Y1)
+    agg2()
+    G.gat_aggregate(plan, Zs, Zs[:, 264:], Hh, Fh, out=Yg)
+    torch.cuda.synchronize()
+    sys.exit(0)
 run("")
 if "--maps" in sys.argv:
     for m in [(8, 32, 1), (8, 16, 2), (4, 32, 2), (4, 16, 2), (4, 32, 1), (8, 8, 4)]:

@@ -12,6 +12,7 @@
 // over three working sets: rows spread over 2.5 GB (HBM-bound), over 100 MB
 // and over 24 MB (L2-resident, 126 MB L2).  Prints GB/s of gathered row bytes.
 //   nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 gather_roofline.cu -o gather_roofline
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -206,6 +207,106 @@ __global__ void __launch_bounds__(WARPS * 32) k_cpa(const char *X, const int32_t
   if (sum == 12345.f) out[0] = sum;
 }
 
+// TMA tile::gather4 gather: one lane issues cp.async.bulk.tensor.2d...gather4
+// for 4 rows at a time (one request = 4 rows) into a per-warp ring of S
+// slots, completion on an mbarrier per slot
+template <int ROWB, int S>
+__global__ void __launch_bounds__(256) k_g4(const __grid_constant__ CUtensorMap map, const int32_t *idx, int64_t nidx,
+                                            int per_warp, float *out) {
+  constexpr int SLOTB = (4 * ROWB + 127) / 128 * 128;  // TMA destinations are 128-byte aligned
+  constexpr int NCH = ROWB / 16;
+  constexpr int PER = (NCH + 31) / 32;
+  extern __shared__ __align__(128) char smem[];
+  __shared__ uint64_t bar[8][S];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  char *ring = smem + (size_t)w * S * SLOTB;
+  if (lane == 0)
+    for (int s = 0; s < S; ++s) asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&bar[w][s])));
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  __syncwarp();
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t base = warp * per_warp;
+  int32_t cur = idx[(base + lane) % nidx];
+  int32_t nxt = idx[(base + 32 + lane) % nidx];
+  auto issue = [&](int q, int s) {  // rows 4q .. 4q+3 of the current batch window
+    const int j = (4 * q) & 31;
+    const int32_t r0 = __shfl_sync(~0u, cur, j), r1 = __shfl_sync(~0u, cur, j + 1),
+                  r2 = __shfl_sync(~0u, cur, j + 2), r3 = __shfl_sync(~0u, cur, j + 3);
+    if (lane == 0) {
+      const uint32_t b = smem_u32(&bar[w][s]);
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(b), "r"(SLOTB) : "memory");
+      asm volatile(
+          "cp.async.bulk.tensor.2d.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes [%0], [%1, {%2, "
+          "%3, %4, %5, %6}], [%7];" ::"r"(smem_u32(ring + s * SLOTB)),
+          "l"(&map), "r"(0), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(b)
+          : "memory");
+    }
+  };
+  const int nq = per_warp / 4;
+  for (int q = 0; q < S; ++q) issue(q, q);
+  float4 a[PER] = {};
+  for (int q = 0; q < nq; ++q) {
+    const int s = q % S;
+    const uint32_t b = smem_u32(&bar[w][s]);
+    const uint32_t par = (q / S) & 1;
+    {  // bounded wait: trap instead of hanging if a request never completes
+      uint32_t ok = 0;
+      for (int spin = 0; !ok; ++spin) {
+        asm volatile(
+            "{\n\t.reg .pred P1;\n\tmbarrier.try_wait.parity.shared::cta.b64 P1, [%1], %2;\n\tselp.u32 %0, 1, 0, P1;\n\t}\n"
+            : "=r"(ok)
+            : "r"(b), "r"(par)
+            : "memory");
+        if (spin > (1 << 22)) __trap();
+      }
+    }
+#pragma unroll
+    for (int r = 0; r < 4; ++r) {
+      const float4 *row = reinterpret_cast<const float4 *>(ring + s * SLOTB + r * ROWB);
+#pragma unroll
+      for (int k = 0; k < PER; ++k) {
+        const int c = lane + 32 * k;
+        if (c < NCH) {
+          const float4 v = row[c];
+          a[k].x += v.x; a[k].y += v.y; a[k].z += v.z; a[k].w += v.w;
+        }
+      }
+    }
+    __syncwarp();
+    const int qn = q + S;
+    if (((4 * qn) & 31) == 0) {
+      cur = nxt;
+      nxt = idx[(base + 4 * qn + 32 + lane) % nidx];
+    }
+    if (qn < nq) issue(qn, s);
+  }
+  float sum = 0;
+  for (int k = 0; k < PER; ++k) sum += a[k].x + a[k].y + a[k].z + a[k].w;
+  if (sum == 12345.f) out[0] = sum;
+}
+
+typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                  const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+static bool encode_rows(CUtensorMap *m, const void *X, int64_t nrows, int rowb) {
+  static EncodeTiledFn fn = nullptr;
+  if (!fn) {
+    void *f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) != cudaSuccess) return false;
+    fn = (EncodeTiledFn)f;
+  }
+  const cuuint64_t dims[2] = {(cuuint64_t)(rowb / 4), (cuuint64_t)nrows};
+  const cuuint64_t strides[1] = {(cuuint64_t)rowb};
+  const cuuint32_t box[2] = {(cuuint32_t)(rowb / 4), 1};
+  const cuuint32_t es[2] = {1, 1};
+  CUresult r = fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void *)X, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                  CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) printf("encode failed %d\n", (int)r);
+  return r == CUDA_SUCCESS;
+}
+
 template <typename K>
 static float time_kernel(K launch) {
   cudaEvent_t a, b;
@@ -281,7 +382,27 @@ static void run_rowb(const char *X, int64_t nrows_total, int32_t *idx_d, std::ve
     cpa(k_cpa<ROWB, 4, 16>, 4, 16);
     cpa(k_cpa<ROWB, 6, 16>, 6, 16);
     cpa(k_cpa<ROWB, 3, 16>, 3, 16);
-    bulk(k_bulk<ROWB, 16, 8>, 16, 8);
+    if constexpr (ROWB <= 1024 && ROWB % 16 == 0) {
+      CUtensorMap map;
+      if (encode_rows(&map, X, sets[0], ROWB)) {
+        auto g4 = [&](auto kern, int S) {
+          const size_t sm = (size_t)8 * S * ((4 * ROWB + 127) / 128 * 128);
+          cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+          int occ = 0;
+          cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, 256, sm);
+          if (occ < 1) return;
+          const int blocks = 148 * occ * 2;
+          const double rows = (double)blocks * 8 * per_warp;
+          const float ms = time_kernel([&] { kern<<<blocks, 256, sm>>>(map, idx_d, nidx, per_warp, out); });
+          printf("ROWB %4d %s g4   S=%2d (4 rows/slot) occ=%2d CTA/SM (%3zu KB smem/SM): %8.3f ms %7.0f GB/s  %s\n", ROWB,
+                 names[si], S, occ, sm * occ / 1024, ms, rows * ROWB / (ms * 1e-3) / 1e9,
+                 cudaGetErrorString(cudaGetLastError()));
+        };
+        g4(k_g4<ROWB, 1>, 1);
+        g4(k_g4<ROWB, 2>, 2);
+        g4(k_g4<ROWB, 3>, 3);
+      }
+    }
   }
 }
 
