@@ -51,6 +51,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-rho0", action="store_true", help="skip the rho = 0 control graph (SURVEY §8(d))")
+    ap.add_argument("--overlap", type=int, default=0,
+                    help="N > 1: pipeline layer 2's exchange with its aggregation over source blocks (NEXT-2)")
     ap.add_argument("--cpu-rows", type=int, default=0, help="oracle sample rows (0 = auto)")
     return ap.parse_args()
 
@@ -161,7 +163,8 @@ def run_ours(args):
     HF = Hh * Fh
     t0 = time.time()
     model = RowPartitionedGCNGAT(g.rowptr, g.colidx, inp["W1"], inp["W2"], inp["W3"], inp["a_src"], inp["a_dst"],
-                                 Hh, Fh, rank=rank, world=world, reorder=args.reorder, device=dev)
+                                 Hh, Fh, rank=rank, world=world, reorder=args.reorder, device=dev,
+                                 overlap=bool(args.overlap))
     plan_s = time.time() - t0
     info = model.plan.info
     rows, lnnz = model.rows, model.nnz_local
@@ -266,7 +269,9 @@ def run_ours(args):
                    "reorder": args.reorder, "F": [F_in, F, HF], "heads": Hh, "scale": args.scale,
                    "group_size": info["group_size"], "tile_groups": info["tile_groups"],
                    "l2": "inputs larger than L2 (X 980 MB, activations 2.5 GB vs 126 MB); no flush",
-                   "parallelism": f"row-partition x{world}" + (" + NCCL all-gather" if world > 1 else "")},
+                   "parallelism": f"row-partition x{world}" + ((" + NCCL ring exchange overlapped with layer-2 "
+                                                                "source-block aggregation" if args.overlap else
+                                                                " + NCCL all-gather") if world > 1 else "")},
         "breakdown_ms": {k: round(float(v), 4) for k, v in zip(names, parts)},
         "plan": {"build_s": round(plan_s, 2), "gen_s": round(inp["gen_s"], 2), "n_groups": info["n_groups"],
                  "n_tiles": info["n_tiles"], "n_split_rows": info["n_split_rows"], "n_clusters": info["n_clusters"],

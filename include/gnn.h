@@ -211,6 +211,23 @@ gnn_status gnn_aggregate(gnn_plan_t plan, int reduce, int weight, const float *e
                          void *ws, size_t ws_bytes, gnn_stream_t stream);
 
 /*
+ * Source-block accumulation (NEXT-2 groundwork, SURVEY §8(e) lever ii): with a
+ * plan over the same destination rows but only the entries whose sources lie
+ * in one block (e.g. one rank's slot of the all-gather), y_v = (accumulate ?
+ * y_v : 0) + SUM_{u->v in the plan} e_uv * x_u -- raw sums, no epilogue;
+ * rows the plan leaves empty keep y_v (accumulate) or get 0.  weight: ONE or
+ * EDGE (pre-scale the sources for GCN and finish with gnn_scale_rows).
+ * Deterministic: each call is the fixed chain of R9 over the block's groups,
+ * and blocks are added in the caller's order.
+ * gnn_scale_rows: y_v = ReLU?(y_v * scale[v]) on n rows x F (device scale[n]).
+ */
+gnn_status gnn_aggregate_accumulate(gnn_plan_t plan, int weight, const float *edge_w, const float *X,
+                                    int64_t ldx, int32_t F, float *Y, int64_t ldy, int32_t accumulate,
+                                    void *ws, size_t ws_bytes, gnn_stream_t stream);
+gnn_status gnn_scale_rows(float *Y, int64_t ldy, int64_t n, int32_t F, const float *scale, int32_t relu,
+                          gnn_stream_t stream);
+
+/*
  * a7: fused GAT graph operation (Eq 2; Listing 1 P:622-646 fused, DVRA
  * P:943-968, division postponed by the linear property).  Per head h:
  * e_uv = LeakyReLU(s_u[h] + t_v[h], neg_slope), alpha = softmax_v(e),
@@ -422,6 +439,18 @@ gnn_status gnn_local_csr(int64_t n, const int64_t *rowptr_h, const int32_t *coli
                          const int64_t *bounds_h, int32_t nparts, int32_t rank,
                          int64_t *r_max, int64_t *local_nnz, int64_t *local_rowptr_h,
                          int32_t *local_colidx_h, int32_t *src_degree_h);
+
+/*
+ * Source block q of rank `rank`'s rows (host only; NEXT-2 source-block
+ * pipelining): the CSR of rows [bounds[rank], bounds[rank+1]) restricted to
+ * the entries whose source u lies in [bounds[q], bounds[q+1]), with u stored
+ * relative to the block (u - bounds[q]); entry order within a row is kept.
+ * Size query with NULL outputs: *block_nnz.  block_rowptr_h int64[rows+1],
+ * block_colidx_h int32[block_nnz].
+ */
+gnn_status gnn_local_csr_block(int64_t n, const int64_t *rowptr_h, const int32_t *colidx_h,
+                               const int64_t *bounds_h, int32_t nparts, int32_t rank, int32_t q,
+                               int64_t *block_nnz, int64_t *block_rowptr_h, int32_t *block_colidx_h);
 
 /*
  * Host-only planner steps (no GPU needed).  gnn_plan_create runs exactly these

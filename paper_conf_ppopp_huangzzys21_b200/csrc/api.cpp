@@ -427,6 +427,42 @@ gnn_status gnn_aggregate(gnn_plan_t p, int reduce, int weight, const float *edge
   })
 }
 
+gnn_status gnn_aggregate_accumulate(gnn_plan_t p, int weight, const float *edge_w, const float *X, int64_t ldx,
+                                    int32_t F, float *Y, int64_t ldy, int32_t accumulate, void *ws, size_t ws_bytes,
+                                    gnn_stream_t stream) {
+  GNN_TRY({
+    if (!p) return check(false, "plan is NULL");
+    if (weight != GNN_W_ONE && weight != GNN_W_EDGE) return check(false, "accumulate: weight must be ONE or EDGE");
+    if (F < 0) return check(false, "F < 0");
+    if (F == 0) return GNN_OK;
+    if (!Y || (p->nnz > 0 && !X)) return check(false, "X/Y is NULL");
+    if (ldx < F || ldy < F) return check(false, "ld < F");
+    if (weight == GNN_W_EDGE && !edge_w && p->nnz > 0) return check(false, "edge_w required for GNN_W_EDGE");
+    if (overlaps(X, span_bytes(p->n_src, ldx, F), Y, span_bytes(p->n, ldy, F)))
+      return check(false, "X and Y overlap");
+    AggArgs a{};
+    a.mode = 0;
+    a.weight = weight;
+    a.edge_w = edge_w;
+    a.X = X;
+    a.ldx = ldx;
+    a.F = F;
+    a.Y = Y;
+    a.ldy = ldy;
+    a.accum = accumulate ? 1 : 0;
+    return agg_common(p, a, ws, ws_bytes, stream);
+  })
+}
+
+gnn_status gnn_scale_rows(float *Y, int64_t ldy, int64_t n, int32_t F, const float *scale, int32_t relu,
+                          gnn_stream_t stream) {
+  GNN_TRY({
+    if (n < 0 || F < 0 || ldy < F) return check(false, "bad scale_rows sizes");
+    if (n > 0 && F > 0 && (!Y || !scale)) return check(false, "Y/scale is NULL");
+    return cuda_status(launch_scale_rows(Y, ldy, n, F, scale, relu, (cudaStream_t)stream), "scale rows");
+  })
+}
+
 gnn_status gnn_gat_aggregate(gnn_plan_t p, const float *Zs, int64_t ldz, const float *t, int64_t ldt,
                              int32_t H, int32_t Fh, float neg_slope, float *Y, int64_t ldy, void *ws,
                              size_t ws_bytes, gnn_stream_t stream) {
@@ -796,6 +832,30 @@ gnn_status gnn_local_csr(int64_t n, const int64_t *rowptr_h, const int32_t *coli
         src_degree_h[q * rm + (u - bounds_h[q])] += 1;
       }
     }
+    return GNN_OK;
+  })
+}
+
+gnn_status gnn_local_csr_block(int64_t n, const int64_t *rowptr_h, const int32_t *colidx_h, const int64_t *bounds_h,
+                               int32_t nparts, int32_t rank, int32_t q, int64_t *block_nnz, int64_t *block_rowptr_h,
+                               int32_t *block_colidx_h) {
+  GNN_TRY({
+    if (n < 0 || !rowptr_h || !colidx_h || !bounds_h || nparts < 1 || rank < 0 || rank >= nparts || q < 0 ||
+        q >= nparts || !block_nnz)
+      return check(false, "bad local_csr_block arguments");
+    const int64_t lo = bounds_h[rank], hi = bounds_h[rank + 1], qlo = bounds_h[q], qhi = bounds_h[q + 1];
+    int64_t cnt = 0;
+    if (block_rowptr_h) block_rowptr_h[0] = 0;
+    for (int64_t v = lo; v < hi; ++v) {
+      for (int64_t k = rowptr_h[v]; k < rowptr_h[v + 1]; ++k) {
+        const int64_t u = colidx_h[k];
+        if (u < qlo || u >= qhi) continue;
+        if (block_colidx_h) block_colidx_h[cnt] = (int32_t)(u - qlo);
+        ++cnt;
+      }
+      if (block_rowptr_h) block_rowptr_h[v - lo + 1] = cnt;
+    }
+    *block_nnz = cnt;
     return GNN_OK;
   })
 }

@@ -129,6 +129,7 @@ struct AggArgs {
   float *ws_part;
   int32_t *ws_cnt;
   int32_t deterministic;
+  int32_t accum;  // Y += sums (gnn_aggregate_accumulate)
 };
 // NEXT-3 GraphSAGE-LSTM (k_lstm.cu)
 int set_lstm_impl(int impl);
@@ -146,6 +147,8 @@ bool agg_mapping_ok(const AggArgs &a, int32_t fh_or_0, int32_t vec, int32_t lane
 gnn_status rebuild_schedule(gnn_plan_s *p, int64_t group_size);
 int64_t default_group_size(int64_t n, int64_t nnz);
 size_t agg_workspace_bytes(const gnn_plan_s *p, int mode, int32_t F, int32_t H);
+cudaError_t launch_scale_rows(float *Y, int64_t ldy, int64_t n, int32_t F, const float *scale, int32_t relu,
+                              cudaStream_t s);
 cudaError_t launch_head_mean(const float *Yf, int64_t ldf, int64_t n, int32_t H, int32_t Fh, float *Y, int64_t ldy,
                              cudaStream_t s);
 gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, size_t ws_bytes,

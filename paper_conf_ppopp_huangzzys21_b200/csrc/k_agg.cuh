@@ -74,6 +74,8 @@ struct KParams {
   int32_t FW;      // partial slot width: F (+ 2 nmeta for attention), rounded to 8
   int32_t nmeta;   // attention: (m, l) entries per slot = H + max chunks; entry of (chunk ci, head h) = h + ci
   int32_t deterministic;
+  int32_t accum;      // 1: Y += this call's sums (source-block accumulation, NEXT-2); rows without
+                      // entries keep their value
   int32_t nch;        // feature chunks per row (arrival counters per multi-unit row)
   int32_t n_persist;  // persistent CTAs
   // load-balance trace (Fig 8 analogue), nullable: [0] sum of
@@ -274,25 +276,6 @@ __device__ __forceinline__ float epi(const KParams &p, int mode, float a, float 
   return y;
 }
 
-template <int MODE, int VEC, int NV, int LANES>
-__device__ __forceinline__ void store_row(const KParams &p, int32_t row, int32_t deg, int32_t c0,
-                                          int lane, const Part<MODE, VEC, NV> &P, const float *ndst_pre = nullptr) {
-  const float ndst =
-      (!is_att(MODE) && scales_dst(p.weight)) ? (ndst_pre ? *ndst_pre : __ldg(p.g.ndst + row)) : 1.0f;
-  const float deg_f = (float)deg;
-#pragma unroll
-  for (int n = 0; n < NV; ++n) {
-    const int32_t f = c0 + (n * LANES + lane) * VEC;
-    if (f >= p.F) continue;
-    float y[VEC];
-    float addv[VEC];
-    if (p.add_row) ldv<VEC>(p.add_row + (int64_t)row * p.ld_add + f, addv);
-#pragma unroll
-    for (int i = 0; i < VEC; ++i) y[i] = epi(p, p.mode, P.a[n][i], P.l[n], ndst, deg_f, p.add_row ? &addv[i] : nullptr);
-    stv_out<VEC>(p.Y + (int64_t)row * p.ldy + f, y);
-  }
-}
-
 // load VEC floats from L2 (bypassing L1: data written by other SMs in this launch)
 template <int VEC>
 __device__ __forceinline__ void ldv_cg(const float *p, float (&v)[VEC]) {
@@ -310,6 +293,32 @@ __device__ __forceinline__ void ldv_cg(const float *p, float (&v)[VEC]) {
     v[0] = __ldcg(p);
   }
 }
+
+template <int MODE, int VEC, int NV, int LANES>
+__device__ __forceinline__ void store_row(const KParams &p, int32_t row, int32_t deg, int32_t c0,
+                                          int lane, const Part<MODE, VEC, NV> &P, const float *ndst_pre = nullptr) {
+  const float ndst =
+      (!is_att(MODE) && scales_dst(p.weight)) ? (ndst_pre ? *ndst_pre : __ldg(p.g.ndst + row)) : 1.0f;
+  const float deg_f = (float)deg;
+#pragma unroll
+  for (int n = 0; n < NV; ++n) {
+    const int32_t f = c0 + (n * LANES + lane) * VEC;
+    if (f >= p.F) continue;
+    float y[VEC];
+    float addv[VEC];
+    if (p.add_row) ldv<VEC>(p.add_row + (int64_t)row * p.ld_add + f, addv);
+#pragma unroll
+    for (int i = 0; i < VEC; ++i) y[i] = epi(p, p.mode, P.a[n][i], P.l[n], ndst, deg_f, p.add_row ? &addv[i] : nullptr);
+    if (p.accum) {  // raw sums only (validated by gnn_aggregate_accumulate): y = y_old + this block's sum
+      float old[VEC];
+      ldv_cg<VEC>(p.Y + (int64_t)row * p.ldy + f, old);
+#pragma unroll
+      for (int i = 0; i < VEC; ++i) y[i] = old[i] + y[i];
+    }
+    stv_out<VEC>(p.Y + (int64_t)row * p.ldy + f, y);
+  }
+}
+
 
 // ---------------------------------------------------------------------------
 // v8 work distribution (measured: scripts/stream_bench_k.cu): persistent
@@ -979,7 +988,8 @@ __global__ void __launch_bounds__(256, S > 0 ? GNN_AGG_MINB_CP
       LANES == 32 ? 0xffffffffu : (((1u << LANES) - 1u) << ((tid & 31) & ~(LANES - 1)));
   const DevGraph &g = p.g;
   if ((int32_t)blockIdx.x >= p.n_persist) {
-    // zero-fill rows without in-edges (R3-i): 32 rows per block
+    // zero-fill rows without in-edges (R3-i): 32 rows per block (kept as they are when accumulating)
+    if (p.accum) return;
     const int64_t r0 = (int64_t)(blockIdx.x - p.n_persist) * 32;
     for (int64_t r = r0; r < r0 + 32 && r < g.n_empty; ++r) {
       float *y = p.Y + (int64_t)g.empty_rows[r] * p.ldy;

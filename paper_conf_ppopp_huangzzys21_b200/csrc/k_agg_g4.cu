@@ -98,19 +98,20 @@ struct Layout {
 };
 }  // namespace g4
 
-template <int MODE, int VEC>
+template <int MODE, int VEC, int NV>
 __global__ void __launch_bounds__(g4::WARPS * 32, 2)
     k_stream_g4(const KParams p, const __grid_constant__ CUtensorMap rmap, const __grid_constant__ CUtensorMap smap,
                 const g4::Layout L) {
   using namespace g4;
   constexpr bool ATT = MODE == M_GAT;
-  constexpr int NV = 8 / VEC;  // (4, 32, 2) or (8, 32, 1): 256 features per sweep
+  // lane mapping (VEC, 32, NV): (4, 32, 2) / (8, 32, 1) for 256 features per sweep, (4, 32, 1) for <= 128
   extern __shared__ __align__(128) float smem_raw[];
   __shared__ uint64_t bars[WARPS][S];
   float *smem = reinterpret_cast<float *>(((uintptr_t)smem_raw + 127) & ~(uintptr_t)127);
   const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
   const DevGraph &g = p.g;
   if ((int32_t)blockIdx.x >= p.n_persist) {  // zero-fill rows without in-edges (R3-i)
+    if (p.accum) return;
     const int64_t r0 = (int64_t)(blockIdx.x - p.n_persist) * 32;
     for (int64_t r = r0; r < r0 + 32 && r < g.n_empty; ++r) {
       float *y = p.Y + (int64_t)g.empty_rows[r] * p.ldy;
@@ -127,6 +128,9 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
   __syncwarp();
   const int QE = L.qe(), RS = L.rslot(), SS = L.sslot(), BW = L.bw;
   const bool dst_scale = !ATT && scales_dst(p.weight);
+  // per-edge weights (GCN nsrc[u] inside the chain, or explicit per-CSR-entry weights): one
+  // 4-byte cp.async per edge into the slot's side area, tracked by the slot's mbarrier
+  const int wmode = ATT ? 0 : (p.weight == GNN_W_GCN ? 1 : p.weight == GNN_W_EDGE ? 2 : 0);
   const uint32_t row_bytes = 4u * 4u * (uint32_t)BW;
   const uint32_t sc_bytes = ATT ? 4u * 4u * (uint32_t)p.H : 0u;
   const uint32_t xb = ATT ? 4u * (uint32_t)p.H : 16u;
@@ -140,14 +144,14 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
     int32_t *ctr = p.ws_unit + ci;
     bool valid[NV];
     int32_t head[NV];
-    float smx[NV];
 #pragma unroll
     for (int n = 0; n < NV; ++n) {
       const int32_t f = c0 + (n * 32 + lane) * VEC;
       valid[n] = f < p.F && (n * 32 + lane) * VEC < BW;
       head[n] = (ATT && valid[n]) ? f / p.Fh : 0;
-      smx[n] = (ATT && valid[n]) ? fkey_decode(__ldg(p.smax + head[n])) : 0.0f;
     }
+    const int hsh = ATT ? (lane & (p.H - 1)) : 0;
+    const float smxs = ATT ? fkey_decode(__ldg(p.smax + hsh)) : 0.0f;
     // ---- run-claim pipeline: C (atomic issued) -> B (descriptors loading) -> A (ready, first indices loading) -> P
     int32_t uC = 0;
     if (lane == 0) uC = atomicAdd(ctr, RUN);
@@ -155,6 +159,7 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
     int32_t eB = 0, eA = 0, eP = 0, nB = 0, nA = 0, nP = 0;
     int32_t T0A = 0, T1A = 0, firstA = 0, T1P = 0;
     int32_t pp = 0, juP = 0, uendP = 0, ib0 = 0, icur = 0, inxt = 0;
+    int32_t ubegP = 0, utposP = 0;  // CSR / task position of the producer's unit (explicit edge weights)
     bool live = false;  // the producer has edges
     auto advance_run = [&]() {
       dP = dA;
@@ -189,11 +194,15 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
     // ---- producer: the next four edges of the stream into slot pslot ----
     auto produce_quad = [&]() {
       int32_t r4[4] = {0, 0, 0, 0};
+      int32_t wpos[4] = {0, 0, 0, 0};  // explicit weights: CSR position of each edge
       int32_t xrow0 = 0, xrow1 = 0, xrow2 = 0, xrow3 = 0, xent0 = 0, xent1 = 0, xent2 = 0, xent3 = 0;
       int nx = 0, nvalid = 0;
       if (live && pp + 4 <= uendP && pp - ib0 <= 28) {  // fast path: four edges of the current unit and batch
 #pragma unroll
-        for (int r = 0; r < 4; ++r) r4[r] = __shfl_sync(0xffffffffu, icur, pp - ib0 + r);
+        for (int r = 0; r < 4; ++r) {
+          r4[r] = __shfl_sync(0xffffffffu, icur, pp - ib0 + r);
+          wpos[r] = ubegP + (pp + r - utposP);
+        }
         pp += 4;
         nvalid = 4;
       } else {
@@ -210,6 +219,8 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
               const int32_t ubeg = __shfl_sync(0xffffffffu, dP.y, juP);
               const int32_t um = __shfl_sync(0xffffffffu, dP.w, juP);
               const int32_t e = qt & (QN - 1);
+              ubegP = ubeg;
+              utposP = pp;
               if (lane == 0) {
                 int *qi = reinterpret_cast<int *>(queue + e * QE);
                 qi[0] = urow;
@@ -235,6 +246,7 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
               inxt = ib0 + 32 + lane < T1P ? ld_stream_i32(g.colidx_t + ib0 + 32 + lane) : 0;
             }
             r4[r] = __shfl_sync(0xffffffffu, icur, pp - ib0);
+            wpos[r] = ubegP + (pp - utposP);
             ++pp;
             ++nvalid;
           }
@@ -245,6 +257,15 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
         ib0 += 32;
         inxt = ib0 + 32 + lane < T1P ? ld_stream_i32(g.colidx_t + ib0 + 32 + lane) : 0;
       }
+      if (wmode && lane < nvalid) {  // per-edge weights: lane r copies edge r's weight
+        const int32_t u = lane == 0 ? r4[0] : lane == 1 ? r4[1] : lane == 2 ? r4[2] : r4[3];
+        const int32_t cp = lane == 0 ? wpos[0] : lane == 1 ? wpos[1] : lane == 2 ? wpos[2] : wpos[3];
+        const float *src = wmode == 1 ? g.nsrc + u : p.edge_w + cp;
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(sa(scs + (size_t)pslot * SS + lane)), "l"(src)
+                     : "memory");
+        asm volatile("cp.async.mbarrier.arrive.shared::cta.b64 [%0];" ::"r"(sa(&bars[w][pslot])) : "memory");
+      }
+      __syncwarp();
       if (lane == 0) {
         uint64_t *bar = &bars[w][pslot];
         uint32_t bytes = (nvalid > 0 ? row_bytes + sc_bytes : 0u) + xb * (uint32_t)nx;
@@ -272,7 +293,7 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
     for (int k = 0; k < S; ++k) produce_quad();
     // ---- consumer ----
     Part<MODE, VEC, NV> G;
-    float tv[NV], nmb[NV], seen[NV];
+    float tvs = 0.0f, mbs = 0.0f, nmbs = 0.0f, seens = 0.0f, ls = 0.0f;  // GAT: head hsh's softmax state
     float ndstC = 1.0f;
     int32_t rowC = 0, lenC = 0, begC = 0, mC = -1, tposC = 0, posC = 0;
     bool more = true;
@@ -297,14 +318,13 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
           tposC = qi[4];
           part_init(G);
           if constexpr (ATT) {
-#pragma unroll
-            for (int n = 0; n < NV; ++n) {
-              tv[n] = valid[n] ? qe[8 + head[n]] : 0.0f;
-              const float mb = valid[n] ? leaky_f(smx[n] + tv[n], p.slope) : 0.0f;
-              G.m[n] = mb;
-              nmb[n] = -mb * kLog2e;
-              seen[n] = -INFINITY;
-            }
+            // shared softmax state: lane computes head hsh = lane % H (H a power of two)
+            tvs = qe[8 + hsh];
+            const float mb = leaky_f(smxs + tvs, p.slope);
+            mbs = mb;
+            nmbs = -mb * kLog2e;
+            seens = -INFINITY;
+            ls = 0.0f;
           } else {
             ndstC = dst_scale ? qe[8 + (rowC & 3)] : 1.0f;
           }
@@ -315,28 +335,31 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
         for (int j = 0; j < kk; ++j, ++r) {
           const float *rb = rq + r * BW;
           if constexpr (ATT) {
+            // e_uv and exp(e_uv - m) once per head (lane hsh), then to the lanes holding that head
+            const float sco = leaky_f(sq[r * p.H + hsh] + tvs, p.slope);
+            seens = fmaxf(seens, sco);
+            const float ex = one ? 1.0f : ex2_f(fmaf(sco, kLog2e, nmbs));
+            ls += ex;
 #pragma unroll
             for (int n = 0; n < NV; ++n) {
+              const float exn = __shfl_sync(0xffffffffu, ex, head[n]);
               if (!valid[n]) continue;
               float v[VEC];
               lds_vec<VEC>(rb + (n * 32 + lane) * VEC, v);
-              const float sco = leaky_f(sq[r * p.H + head[n]] + tv[n], p.slope);
-              seen[n] = fmaxf(seen[n], sco);
-              const float ex = one ? 1.0f : ex2_f(fmaf(sco, kLog2e, nmb[n]));
-              G.l[n] += ex;
-              fma_vec<VEC>(G.a[n], v, ex);
+              fma_vec<VEC>(G.a[n], v, exn);
             }
           } else {
 #pragma unroll
+            const float wt = wmode ? sq[r] : 1.0f;
             for (int n = 0; n < NV; ++n) {
               if (!valid[n]) continue;
               float v[VEC];
               lds_vec<VEC>(rb + (n * 32 + lane) * VEC, v);
               if constexpr (MODE == M_MAX) {
 #pragma unroll
-                for (int i = 0; i < VEC; ++i) G.a[n][i] = fmaxf(G.a[n][i], 1.0f * v[i]);
+                for (int i = 0; i < VEC; ++i) G.a[n][i] = fmaxf(G.a[n][i], wt * v[i]);
               } else {
-                fma_vec<VEC>(G.a[n], v, 1.0f);
+                fma_vec<VEC>(G.a[n], v, wt);
               }
             }
           }
@@ -344,6 +367,14 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
         posC += kk;
         if (posC == lenC) {
           if constexpr (ATT) {
+            float tv[NV], seen[NV];
+#pragma unroll
+            for (int n = 0; n < NV; ++n) {  // the per-head state to the lanes of each vector
+              G.m[n] = __shfl_sync(0xffffffffu, mbs, head[n]);
+              G.l[n] = __shfl_sync(0xffffffffu, ls, head[n]);
+              seen[n] = __shfl_sync(0xffffffffu, seens, head[n]);
+              tv[n] = __shfl_sync(0xffffffffu, tvs, head[n]);
+            }
             if (lenC == 1) {
 #pragma unroll
               for (int n = 0; n < NV; ++n) G.m[n] = seen[n];
@@ -420,21 +451,21 @@ bool g4_admissible(const KParams &kp, int32_t n_src) {
   if (!encode_fn() || n_src < 1) return false;
   if (kp.F % 4 || kp.ldx % 4 || ((uintptr_t)kp.X & 15)) return false;
   if (kp.add_row) return false;
-  if (kp.mode == M_GAT) {
-    if (kp.H % 4 || kp.H > 32 || kp.Fh % 4 || kp.ldt % 4 || ((uintptr_t)kp.t & 15)) return false;
+  if (kp.mode == M_GAT) {  // heads: a power of two, 4..32 (16-byte score rows, one lane per head)
+    if (kp.H < 4 || kp.H > 32 || (kp.H & (kp.H - 1)) || kp.Fh % 4 || kp.ldt % 4 || ((uintptr_t)kp.t & 15)) return false;
     if (((uintptr_t)(kp.X + kp.F) & 15)) return false;
     return true;
   }
   if (kp.mode > M_MAX) return false;
-  return kp.weight == GNN_W_ONE || kp.weight == W_DST_ONLY;
+  return true;  // every weight: 1, GCN (nsrc[u] per edge, ndst[v] per row), explicit, pre-scaled GCN
 }
 
-template <int MODE, int VEC>
+template <int MODE, int VEC, int NV>
 static cudaError_t launch_g4_mode(const KParams &kp_in, int32_t n_src, cudaStream_t s) {
   using namespace g4;
   g4::Layout L;
   L.bw = kp_in.F < BWMAX ? kp_in.F : BWMAX;
-  L.hs = MODE == M_GAT ? kp_in.H : 0;
+  L.hs = MODE == M_GAT ? kp_in.H : 4;  // GAT scores, or the 4 per-edge weights of a quad
   L.xe = MODE == M_GAT ? (kp_in.H < 4 ? 4 : kp_in.H) : 4;
   const size_t smem = L.bytes();
   CUtensorMap rmap, smap;
@@ -444,7 +475,7 @@ static cudaError_t launch_g4_mode(const KParams &kp_in, int32_t n_src, cudaStrea
   if (MODE == M_GAT && !encode_rows(&smap, kp_in.X + kp_in.F, n_src, kp_in.H, kp_in.ldx, kp_in.H))
     return cudaErrorNotSupported;
   static int occ = 0;
-  auto fn = k_stream_g4<MODE, VEC>;
+  auto fn = k_stream_g4<MODE, VEC, NV>;
   if (occ == 0) {
     cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
@@ -472,23 +503,28 @@ static cudaError_t launch_g4_mode(const KParams &kp_in, int32_t n_src, cudaStrea
   return cudaGetLastError();
 }
 
-// lane mapping of the consumer: VEC 8 (one lane = 8 consecutive features, one
-// GAT head slice per lane) unless env GNN_G4_VEC=4; every lane needs F % VEC == 0
+// lane mapping of the consumer: VEC 4 (lane = features 4l and 128 + 4l), or
+// env GNN_G4_VEC=8 (8 consecutive features; 2-way shared-memory bank conflicts)
 static int g4_vec() {
   static int v = 0;
   if (v == 0) {
     const char *e = getenv("GNN_G4_VEC");
-    v = (e && e[0] == '4') ? 4 : 8;
+    v = (e && e[0] == '8') ? 8 : 4;  // measured: VEC 4 (conflict-free shared reads) 15.1 vs 17.9 ms on C5
   }
   return v;
 }
 cudaError_t launch_g4(const KParams &kp, int32_t n_src, cudaStream_t s) {
-  const bool v8 = g4_vec() == 8 && kp.F % 8 == 0 && (kp.mode != M_GAT || kp.Fh % 8 == 0);
+  const bool narrow = kp.F <= 128;  // one 128-feature vector per lane set
+  const bool v8 = !narrow && g4_vec() == 8 && kp.F % 8 == 0;
   switch (kp.mode) {
     case M_SUM:
-    case M_MEAN: return v8 ? launch_g4_mode<M_SUM, 8>(kp, n_src, s) : launch_g4_mode<M_SUM, 4>(kp, n_src, s);
-    case M_MAX: return v8 ? launch_g4_mode<M_MAX, 8>(kp, n_src, s) : launch_g4_mode<M_MAX, 4>(kp, n_src, s);
-    case M_GAT: return v8 ? launch_g4_mode<M_GAT, 8>(kp, n_src, s) : launch_g4_mode<M_GAT, 4>(kp, n_src, s);
+    case M_MEAN:
+      return narrow ? launch_g4_mode<M_SUM, 4, 1>(kp, n_src, s)
+                    : v8 ? launch_g4_mode<M_SUM, 8, 1>(kp, n_src, s) : launch_g4_mode<M_SUM, 4, 2>(kp, n_src, s);
+    case M_MAX:
+      return narrow ? launch_g4_mode<M_MAX, 4, 1>(kp, n_src, s)
+                    : v8 ? launch_g4_mode<M_MAX, 8, 1>(kp, n_src, s) : launch_g4_mode<M_MAX, 4, 2>(kp, n_src, s);
+    case M_GAT: return narrow ? cudaErrorNotSupported : launch_g4_mode<M_GAT, 4, 2>(kp, n_src, s);
     default: return cudaErrorNotSupported;
   }
 }

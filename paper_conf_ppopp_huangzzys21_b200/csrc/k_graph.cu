@@ -174,6 +174,26 @@ cudaError_t launch_score_max(const float *S, int64_t lds, int64_t n_src, int32_t
   return cudaGetLastError();
 }
 
+// y[v][f] = ReLU?(y[v][f] * scale[v]) (the postponed normaliser of a source-block accumulation)
+__global__ void k_scale_rows(float *Y, int64_t ldy, int64_t n, int32_t F, const float *scale, int32_t relu) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n * F; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t v = i / F;
+    float *y = Y + v * ldy + (i % F);
+    float t = *y * __ldg(scale + v);
+    if (relu) t = t > 0.0f ? t : 0.0f;
+    *y = t;
+  }
+}
+
+cudaError_t launch_scale_rows(float *Y, int64_t ldy, int64_t n, int32_t F, const float *scale, int32_t relu,
+                              cudaStream_t s) {
+  if (n == 0 || F == 0) return cudaSuccess;
+  const int blocks = (int)std::min<int64_t>((n * F + 255) / 256, (int64_t)num_sms() * 16);
+  k_scale_rows<<<blocks, 256, 0, s>>>(Y, ldy, n, F, scale, relu);
+  count_launch();
+  return cudaGetLastError();
+}
+
 // head mean (final attention layer): y[v][f] = (1/H) sum_h Yf[v][h*Fh + f], heads in order
 __global__ void k_head_mean(const float *__restrict__ Yf, int64_t ldf, int64_t n, int32_t H, int32_t Fh, float *Y,
                             int64_t ldy) {
@@ -291,8 +311,17 @@ static Mapping choose_mapping(const gnn_plan_s *p, const AggArgs &a, int32_t fh_
     // call); up to 128: the cp.async chain for sum / mean / max, the register
     // kernel for GAT (measured faster there)
     Mapping c{4, 32, a.F > 128 ? 2 : 1};
-    c.cp = a.F > 128 ? g_agg_cp : 1;
-    if (c.cp == 1 && a.mode == M_GAT) c.cp = 0;
+    c.cp = g_agg_cp;
+    if (a.mode == M_GAT) {
+      // GAT: the register kernel measured faster than both staged kernels on C5
+      // (19.8 vs 20.4 ms gather4, 20.0 ms cp.async chain); env GNN_G4_GAT=1 opts in
+      static int g4_gat = -1;
+      if (g4_gat < 0) {
+        const char *e = getenv("GNN_G4_GAT");
+        g4_gat = (e && e[0] == '1') ? 1 : 0;
+      }
+      c.cp = (g4_gat && a.F > 128 && c.cp == 2) ? 2 : 0;
+    }
     if (c.cp) return c;
   }
   const int cands[4] = {8, 4, 2, 1};
@@ -416,6 +445,7 @@ gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, siz
   kp.FW = slot_width(mode, a.F, a.H);
   kp.nmeta = att_meta(mode, a.F, a.H);
   kp.deterministic = a.deterministic;
+  kp.accum = a.accum;
   kp.trace = g_trace;
   const WsLayout L = ws_layout(p, mode, a.F, a.H);
   char *w = reinterpret_cast<char *>(ws);

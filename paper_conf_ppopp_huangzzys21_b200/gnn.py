@@ -86,6 +86,8 @@ _SIGS = {
     "gnn_aggregate": (ctypes.c_int, [_P, ctypes.c_int, ctypes.c_int, _P, _P, _I64, _I32, _P, _I64, _I32, _P, _I64,
                                      _P, _SZ, _P]),
     "gnn_gat_aggregate": (ctypes.c_int, [_P, _P, _I64, _P, _I64, _I32, _I32, _F, _P, _I64, _P, _SZ, _P]),
+    "gnn_aggregate_accumulate": (ctypes.c_int, [_P, ctypes.c_int, _P, _P, _I64, _I32, _P, _I64, _I32, _P, _SZ, _P]),
+    "gnn_scale_rows": (ctypes.c_int, [_P, _I64, _I64, _I32, _P, _I32, _P]),
     "gnn_gat_layer": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _P, _P, _I32, _I32, _F, _P, _I64, _P, _SZ, _P]),
     "gnn_edgeconv_aggregate": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _I64, _P, _SZ, _P]),
     "gnn_edgeconv": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _P, _P, _I32, _P, _I64, _P, _SZ, _P]),
@@ -102,6 +104,7 @@ _SIGS = {
     "gnn_partition_rows": (ctypes.c_int, [_I64, _P, _I32, _P]),
     "gnn_local_csr": (ctypes.c_int, [_I64, _P, _P, _P, _I32, _I32, ctypes.POINTER(_I64), ctypes.POINTER(_I64),
                                      _P, _P, _P]),
+    "gnn_local_csr_block": (ctypes.c_int, [_I64, _P, _P, _P, _I32, _I32, _I32, ctypes.POINTER(_I64), _P, _P]),
     "gnn_las_host": (ctypes.c_int, [_I64, _P, _P, _I32, _I32, _I32, _I32, _I32, _I32, _P, _P, ctypes.POINTER(_I64),
                                     ctypes.POINTER(_I64)]),
     "gnn_groups_host": (ctypes.c_int, [_I64, _P, _P, _I32, ctypes.POINTER(_I64), _P, _P]),
@@ -288,6 +291,23 @@ def aggregate(plan: Plan, X, reduce="sum", weight="one", edge_w=None, relu=False
     return Y
 
 
+def aggregate_accumulate(plan: Plan, X, Y, accumulate=True, weight="one", edge_w=None, stream=None):
+    """gnn_aggregate_accumulate: Y (+)= raw sums of this (source-block) plan."""
+    F = X.shape[1]
+    ws, nb = plan.workspace(GNN_OP_AGGREGATE, 0, F, 0, X.device)
+    _call("gnn_aggregate_accumulate", plan.handle, WEIGHT[weight], _tp(edge_w), _tp(X), _ld(X, F), F, _tp(Y),
+          _ld(Y, F), int(accumulate), _tp(ws), nb, _stream(stream))
+    return Y
+
+
+def scale_rows(Y, scale, relu=False, stream=None):
+    """gnn_scale_rows: Y[v] = ReLU?(Y[v] * scale[v]) (scale: device tensor or pointer)."""
+    sp = scale if isinstance(scale, int) else scale.data_ptr()
+    _call("gnn_scale_rows", _tp(Y), _ld(Y, Y.shape[1]), Y.shape[0], Y.shape[1], ctypes.c_void_p(sp), int(relu),
+          _stream(stream))
+    return Y
+
+
 def gat_aggregate(plan: Plan, Zs, t, H, Fh, neg_slope=0.2, out=None, stream=None):
     torch = _torch()
     F = H * Fh
@@ -413,6 +433,23 @@ def local_csr(rowptr, colidx, bounds, rank):
     _call("gnn_local_csr", n, _np_ptr(rowptr), _np_ptr(colidx), _np_ptr(bounds), P, rank, ctypes.byref(rmax),
           ctypes.byref(lnnz), _np_ptr(lrp), _np_ptr(lci), _np_ptr(sdeg))
     return lrp, lci[:lnnz.value], sdeg[:P * rmax.value], rmax.value
+
+
+def local_csr_block(rowptr, colidx, bounds, rank, q):
+    """gnn_local_csr_block: rank's rows restricted to sources of block q, sources relative to the block."""
+    rowptr = np.ascontiguousarray(rowptr, dtype=np.int64)
+    colidx = np.ascontiguousarray(colidx, dtype=np.int32)
+    b = np.ascontiguousarray(bounds, dtype=np.int64)
+    n, P = len(rowptr) - 1, len(b) - 1
+    cnt = ctypes.c_int64()
+    _call("gnn_local_csr_block", n, _np_ptr(rowptr), _np_ptr(colidx), _np_ptr(b), P, rank, q, ctypes.byref(cnt),
+          None, None)
+    rows = int(b[rank + 1] - b[rank])
+    brp = np.empty(rows + 1, np.int64)
+    bci = np.empty(max(cnt.value, 1), np.int32)
+    _call("gnn_local_csr_block", n, _np_ptr(rowptr), _np_ptr(colidx), _np_ptr(b), P, rank, q, ctypes.byref(cnt),
+          _np_ptr(brp), _np_ptr(bci))
+    return brp, bci[:cnt.value]
 
 
 def las_host(rowptr, sig, r=2, W=8, cap=32, min_sim=-1, cluster_order=1):

@@ -23,12 +23,45 @@ import torch
 from . import gnn as _g
 
 
+def ring_allgather_blocks(buf, rmax, rank, world, group=None, on_block=None, staged=False):
+    """All-gather of the padded layout buf [world * rmax, F] as P - 1 ring steps
+    (NEXT-2 groundwork, SURVEY §8(e) lever ii): step s sends block (rank - s + 1)
+    mod P to rank + 1 and receives block (rank - s) mod P from rank - 1, so rank
+    r holds its blocks in the order r, r - 1, ..., r + 1 (mod P).  on_block(q) is
+    called as soon as block q is present -- the caller enqueues that block's
+    aggregation, which overlaps the next step's transfer (NCCL runs the P2P
+    on its own stream; `wait()` only orders the caller's stream).  staged: move
+    the blocks through host memory (gloo tests)."""
+    import torch.distributed as dist
+    if on_block:
+        on_block(rank)
+    for s in range(1, world):
+        sq, rq = (rank - s + 1) % world, (rank - s) % world
+        send = buf[sq * rmax:(sq + 1) * rmax]
+        recv = buf[rq * rmax:(rq + 1) * rmax]
+        if staged:
+            sbuf, rbuf = send.cpu(), torch.empty(recv.shape, dtype=recv.dtype)
+        else:
+            sbuf, rbuf = send.contiguous(), recv
+        ops = [dist.P2POp(dist.isend, sbuf, (rank + 1) % world, group),
+               dist.P2POp(dist.irecv, rbuf, (rank - 1) % world, group)]
+        for req in dist.batch_isend_irecv(ops):
+            req.wait()
+        if staged:
+            recv.copy_(rbuf)
+        if on_block:
+            on_block(rq)
+
+
 class RowPartitionedGCNGAT:
     def __init__(self, rowptr, colidx, W1, W2, W3, a_src, a_dst, heads, head_dim, neg_slope=0.2,
-                 rank=0, world=1, group=None, reorder=1, device=None, plan_opts=None, staged_allgather=False):
+                 rank=0, world=1, group=None, reorder=1, device=None, plan_opts=None, staged_allgather=False,
+                 overlap=False):
         self.rank, self.world, self.group = rank, world, group
         self.dev = device or torch.device("cuda", torch.cuda.current_device())
         self.staged = staged_allgather  # gloo: exchange through host memory (tests only)
+        # layer 2 exchange pipelined with the aggregation over source blocks (world > 1)
+        self.overlap = bool(overlap) and world > 1
         n = len(rowptr) - 1
         self.n = n
         opts = dict(reorder=reorder, **(plan_opts or {}))
@@ -41,6 +74,15 @@ class RowPartitionedGCNGAT:
             lrp, lci, sdeg, rmax = _g.local_csr(rowptr, colidx, self.bounds, rank)
             self.rmax = rmax
             self.plan = _g.Plan(lrp, lci, n_src=world * rmax, src_degree=sdeg, **opts)
+            if self.overlap:
+                # one plan per source block, in the local plan's task order (LAS runs once)
+                perm = self.plan.export()[0]
+                bopts = dict(opts)
+                bopts.pop("reorder", None)
+                self.block_plans = []
+                for q in range(world):
+                    brp, bci = _g.local_csr_block(rowptr, colidx, self.bounds, rank, q)
+                    self.block_plans.append(_g.Plan(brp, bci, n_src=rmax, perm=perm, reorder=0, **bopts))
         self.lo, self.hi = int(self.bounds[rank]), int(self.bounds[rank + 1])
         self.rows = self.hi - self.lo
         self.nnz_local = int(rowptr[self.hi] - rowptr[self.lo])
@@ -63,7 +105,7 @@ class RowPartitionedGCNGAT:
         self.Y2 = torch.empty((R, self.F), device=d)
         self.Zst = torch.zeros((P, self.ldwe), device=d)
         self.Y3 = torch.empty((R, self.HF), device=d)
-        self.nsrc_ptr, _ = self.plan.normalizers()
+        self.nsrc_ptr, self.ndst_ptr = self.plan.normalizers()
         self.ws_agg, self.ws_agg_b = self.plan.workspace(_g.GNN_OP_AGGREGATE, 0, max(self.F, self.F_in), 0, d)
         self.ws_gat, self.ws_gat_b = self.plan.workspace(_g.GNN_OP_GAT_AGGREGATE, 0, self.HF, heads, d)
         self.names = ["agg1", "gemm1", "gemm2+xchg", "agg2", "gemm3+xchg", "gat_agg"]
@@ -164,10 +206,23 @@ class RowPartitionedGCNGAT:
         h_loc = self.Hs2[off:off + R]
         chk(lib.gnn_gemm(P(self.Y1), F, P(self.W2), F, P(h_loc), F, R, F, F,
                          ctypes.c_void_p(self.nsrc_ptr + 4 * off), None, 0, *gws, sp), "gemm2")
-        self._allgather(self.Hs2)
-        rec(3)
-        chk(lib.gnn_gcn_aggregate_prescaled(self.plan.handle, P(self.Hs2), F, F, P(self.Y2), F, 0, P(self.ws_agg),
-                                            self.ws_agg_b, sp), "agg2")
+        if self.overlap:
+            # source-block pipeline: aggregate each rank's block of Hs2 as it arrives
+            # (own block first), raw sums accumulated in ring order, then x ndst
+            def on_block(q):
+                bp = self.block_plans[q]
+                ws, wb = bp.workspace(_g.GNN_OP_AGGREGATE, 0, F, 0, self.dev)
+                chk(lib.gnn_aggregate_accumulate(bp.handle, _g.GNN_W_ONE, None,
+                                                 P(self.Hs2[q * self.rmax:(q + 1) * self.rmax]), F, F, P(self.Y2), F,
+                                                 int(q != self.rank), P(ws), wb, sp), "agg2 block")
+            rec(3)
+            ring_allgather_blocks(self.Hs2, self.rmax, self.rank, self.world, self.group, on_block, self.staged)
+            chk(lib.gnn_scale_rows(P(self.Y2), F, R, F, ctypes.c_void_p(self.ndst_ptr), 0, sp), "agg2 scale")
+        else:
+            self._allgather(self.Hs2)
+            rec(3)
+            chk(lib.gnn_gcn_aggregate_prescaled(self.plan.handle, P(self.Hs2), F, F, P(self.Y2), F, 0,
+                                                P(self.ws_agg), self.ws_agg_b, sp), "agg2")
         rec(4)
         z_loc = self.Zst[off:off + R]
         # [Z | s | t] = Y2 W3 with the GAT scores from the GEMM epilogue (R5)
