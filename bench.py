@@ -51,6 +51,7 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-rho0", action="store_true", help="skip the rho = 0 control graph (SURVEY §8(d))")
+    ap.add_argument("--no-traffic", action="store_true", help="skip the ncu DRAM-traffic capture of the dominant kernel")
     ap.add_argument("--overlap", type=int, default=0,
                     help="N > 1: pipeline layer 2's exchange with its aggregation over source blocks (NEXT-2)")
     ap.add_argument("--cpu-rows", type=int, default=0, help="oracle sample rows (0 = auto)")
@@ -223,11 +224,9 @@ def run_ours(args):
         pass
     peak = float(peaks.get("hbm_gbs", 6650.0))
     achieved = per_launch[dom_name] / (parts[dom] * 1e-3) / 1e9
-    traffic = None
-    try:  # ncu DRAM bytes per launch of this kernel, from the committed profile summary
-        traffic = json.load(open(os.path.join(ROOT, "profiles", "traffic.json"))).get(dom_name)
-    except Exception:
-        pass
+    traffic, traffic_src = None, "not measured"
+    if world == 1 and not args.no_traffic:
+        traffic, traffic_src = measure_traffic(g, inp, model, dom_name)
     roofline = {"bound": "hbm", "kernel": dom_name, "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(achieved / peak, 4), "traffic": traffic,
                 "dram_gbs": round(traffic / (parts[dom] * 1e-3) / 1e9, 1) if traffic else None,
@@ -236,6 +235,7 @@ def run_ours(args):
                         "launch's event time; LAS + L2 serve part of them, so it can exceed the HBM peak. "
                         "dram_gbs = ncu DRAM bytes (traffic, cold-cache capture) / the same time.",
                 "algorithmic_bytes": int(per_launch[dom_name]), "launch_ms": round(float(parts[dom]), 4),
+                "traffic_source": traffic_src,
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)" if "hbm_gbs" in peaks else "fallback 6650"}
 
     # e2e: the same steps through the public API from pinned host input to
@@ -292,6 +292,50 @@ def run_ours(args):
         print(json.dumps(out), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+def measure_traffic(g, inp, model, kernel):
+    """ncu DRAM bytes (read + write) of one launch of the dominant kernel on this
+    run's graph and plan: the plan is saved (gnn_plan_save) and a probe process
+    repeats the launch under `ncu --metrics dram__bytes_*` (cold cache, like the
+    driver's launch list).  Returns (bytes or None, how)."""
+    import shutil
+    import tempfile
+    ncu = shutil.which("ncu") or "/usr/local/cuda/bin/ncu"
+    if not os.path.exists(ncu):
+        return None, "ncu not found"
+    d = tempfile.mkdtemp(prefix="gnn_traffic_")
+    try:
+        model.plan.save(os.path.join(d, "plan.gnnplan"))
+        np.savez(os.path.join(d, "meta.npz"), n=g.n, F_in=inp["F_in"], F=inp["F"], H=inp["H"], Fh=inp["Fh"])
+        regex = {"gat_agg_8x32": "k_aggregate<3|k_stream_g4<3", "agg2_F256": "k_aggregate<0|k_stream_g4<0",
+                 "agg1_F100": "k_aggregate<0|k_stream_g4<0"}[kernel]
+        cmd = [ncu, "--metrics", "dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum",
+               "--clock-control", "none", "-k", f"regex:{regex}", "-s", "1", "-c", "1", "--csv", "--page", "raw",
+               sys.executable, os.path.join(ROOT, "scripts", "traffic_probe.py"), d, kernel]
+        r = subprocess.run(cmd, capture_output=True, text=True, timeout=300)
+        import csv
+        import io
+        rows = [ln for ln in r.stdout.splitlines() if ln.startswith('"')]
+        rec = list(csv.reader(io.StringIO("\n".join(rows))))
+        if len(rec) < 3:
+            return None, f"ncu produced no record (rc {r.returncode})"
+        h, units, vals = rec[0], rec[1], rec[2]
+        scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
+
+        def val(name):
+            i = h.index(name)
+            return float(vals[i].replace(",", "")) * scale.get(units[i], 1)
+        tot = val("dram__bytes_read.sum") + val("dram__bytes_write.sum")
+        it = h.index("gpu__time_duration.sum")
+        t_ms = float(vals[it].replace(",", "")) * {"nsecond": 1e-6, "usecond": 1e-3, "msecond": 1.0,
+                                                   "second": 1e3}.get(units[it], 1.0)
+        return int(tot), (f"ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum on one launch of "
+                          f"{vals[h.index('Kernel Name')]} (this run's plan; cold cache; {t_ms:.3f} ms under ncu)")
+    except Exception as e:  # noqa: BLE001
+        return None, f"ncu capture failed: {e!r}"[:200]
+    finally:
+        shutil.rmtree(d, ignore_errors=True)
 
 
 def rho0_control(args, dev):

@@ -311,7 +311,11 @@ static Mapping choose_mapping(const gnn_plan_s *p, const AggArgs &a, int32_t fh_
     // call); up to 128: the cp.async chain for sum / mean / max, the register
     // kernel for GAT (measured faster there)
     Mapping c{4, 32, a.F > 128 ? 2 : 1};
-    c.cp = g_agg_cp;
+    // rows of > 128 features: the gather4 streaming kernel (C5 agg2 F = 256:
+    // 15.0 vs 16.8 ms for the register kernel); 64..128: the cp.async chain
+    // (C5 agg1 F = 100 with per-edge GCN weights: 11.0 vs 11.9 register, 13.8
+    // gather4)
+    c.cp = a.F > 128 ? g_agg_cp : std::min(g_agg_cp, 1);
     if (a.mode == M_GAT) {
       // GAT: the register kernel measured faster than both staged kernels on C5
       // (19.8 vs 20.4 ms gather4, 20.0 ms cp.async chain); env GNN_G4_GAT=1 opts in
