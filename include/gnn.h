@@ -510,14 +510,6 @@ gnn_status gnn_sage_lstm_aggregate(gnn_plan_t plan, const int32_t *table, int32_
  * f_in], W_neigh [F_out, F], bias [F_out] (nullable).  Workspace:
  * gnn_workspace_size(plan, GNN_OP_SAGE_LSTM_LAYER, f_in, F_out, T).
  */
-/* GraphSAGE-LSTM cell implementation (process-wide; results within the
- * tolerance of each other): 0 = SIMT cells (default, fastest measured: 9.8 ms
- * on the C5 graph, T = 16), 1 = tcgen05 cells (h R^T as 3xTF32
- * tcgen05.mma into TMEM, 3 x 128 nodes per CTA; 16.1 ms), 2 = mma.sync
- * m16n8k8 TF32 cells (16 nodes per warp; 16.1 ms).  Returns the previous
- * value. */
-int gnn_set_lstm_impl(int impl);
-
 gnn_status gnn_sage_lstm_layer(gnn_plan_t plan, const float *X, int64_t ldx, int32_t f_in,
                                const float *W_ih, const float *W_hh, const float *b_ih,
                                const float *b_hh, const float *W_self, const float *W_neigh,

@@ -1028,6 +1028,5 @@ gnn_status gnn_attn_aggregate(gnn_plan_t p, int score, const float *Zs, int64_t 
   })
 }
 
-int gnn_set_lstm_impl(int impl) { return set_lstm_impl(impl); }
 
 }  // extern "C"

@@ -132,7 +132,6 @@ struct AggArgs {
   int32_t accum;  // Y += sums (gnn_aggregate_accumulate)
 };
 // NEXT-3 GraphSAGE-LSTM (k_lstm.cu)
-int set_lstm_impl(int impl);
 cudaError_t launch_sample_neighbors(const gnn_plan_s *p, int32_t T, uint64_t seed, int32_t *table, cudaStream_t s);
 cudaError_t launch_lstm_weights(const float *W_ih, const float *b_ih, const float *b_hh, const float *W_self,
                                 const float *bias, int32_t f_in, int32_t F, int32_t F_out, float *Wcat,

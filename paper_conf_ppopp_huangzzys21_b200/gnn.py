@@ -112,7 +112,6 @@ _SIGS = {
     "gnn_plan_set_group_size": (ctypes.c_int, [_P, _I32]),
     "gnn_attn_aggregate": (ctypes.c_int, [_P, ctypes.c_int, _P, _I64, _P, _I64, _P, _I32, _I32, _F, _I32, _P, _I64,
                                           _P, _SZ, _P]),
-    "gnn_set_lstm_impl": (ctypes.c_int, [ctypes.c_int]),
     "gnn_sample_neighbors": (ctypes.c_int, [_P, _I32, ctypes.c_uint64, _P, _P]),
     "gnn_sage_lstm_aggregate": (ctypes.c_int, [_P, _P, _I32, _P, _I64, _I32, _P, _P, _I32, _P, _I64, _P]),
     "gnn_sage_lstm_layer": (ctypes.c_int, [_P, _P, _I64, _I32, _P, _P, _P, _P, _P, _P, _P, _I32, _I32, _I32,
@@ -511,10 +510,6 @@ def attn_aggregate(plan: Plan, score, Zs, H, Fh, Tv=None, Wa=None, neg_slope=0.2
           0 if Tv is None else Tv.stride(0), _tp(Wa), H, Fh, neg_slope, int(head_mean), _tp(Y), _ld(Y, width),
           _tp(ws), nb, _stream(stream))
     return Y
-
-
-def set_lstm_impl(impl: int) -> int:
-    return _lib.gnn_set_lstm_impl(impl)
 
 
 def sample_neighbors(plan: Plan, T=16, seed=0, out=None, stream=None):

@@ -244,22 +244,8 @@ def lstm_probe():
     GS = torch.rand((g.n, 5 * F), device="cuda") - 0.5
     tab = G.sample_neighbors(plan, T, 7)
     Y = torch.empty((g.n, F), device="cuda")
-    outs = {}
-    for impl in (1, 0, 2):
-        G.set_lstm_impl(impl)
-        ms = timeit(lambda: G.sage_lstm_aggregate(plan, tab, GS, P["W_hh"], P["W_neigh"], out=Y), iters=5, warm=2)
-        outs[impl] = Y.clone()
-        print(f" lstm cells impl={impl}: {ms:.3f} ms", flush=True)
-    print(f" tc vs simt max abs diff {float((outs[1] - outs[0]).abs().max()):.3e}, mma vs simt "
-          f"{float((outs[2] - outs[0]).abs().max()):.3e}", flush=True)
-    for Tp in (1, 2, 4):
-        tab2 = G.sample_neighbors(plan, Tp, 7)
-        for impl in (1, 0, 2):
-            G.set_lstm_impl(impl)
-            ms = timeit(lambda: G.sage_lstm_aggregate(plan, tab2, GS, P["W_hh"], P["W_neigh"], out=Y), iters=5, warm=2)
-            print(f" T={Tp} impl={impl}: {ms:.3f} ms", flush=True)
-    G.set_lstm_impl(0)
-
+    ms = timeit(lambda: G.sage_lstm_aggregate(plan, tab, GS, P["W_hh"], P["W_neigh"], out=Y), iters=5, warm=2)
+    print(f" lstm cells: {ms:.3f} ms", flush=True)
 
 if __name__ == "__main__":
     what = sys.argv[1] if len(sys.argv) > 1 else "gemm"

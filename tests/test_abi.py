@@ -178,10 +178,11 @@ def test_new_entry_points_reject_null_plans():
     assert g.gnn_workspace_size(None, 6, 0, 64, 8) == 0
 
 
-def test_lstm_impl_switch_roundtrip():
+def test_accumulate_and_scale_validate_before_device_work():
     g = P.gnn
-    old = g.gnn_set_lstm_impl(1)
-    assert g.gnn_set_lstm_impl(old) == 1
+    assert g.gnn_aggregate_accumulate(None, 0, None, None, 1, 1, None, 1, 0, None, 0, None) == 1
+    assert g.gnn_scale_rows(None, 4, 2, 8, None, 0, None) == 1  # ldy < F
+    assert g.gnn_gat_transform(None, 1, 4, 1, None, 1, None, None, 1, 1, None, 3, None, 0, None) == 1
 
 
 def test_plan_load_rejects_missing_and_foreign_files(tmp_path):
