@@ -43,9 +43,10 @@ __device__ __forceinline__ void mbar_init(uint64_t *bar) {
 __device__ __forceinline__ void mbar_expect(uint64_t *bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(sa(bar)), "r"(bytes) : "memory");
 }
-// wait for a phase; a request that never completes traps (an error the
-// caller sees) instead of hanging the GPU
+// wait for a phase; a request that has not completed after 20 s of wall
+// time traps (an error the caller sees) instead of hanging the GPU
 __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+  unsigned long long t0 = 0;
   for (uint32_t spin = 0;; ++spin) {
     uint32_t ok;
     asm volatile(
@@ -54,7 +55,11 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
         : "r"(sa(bar)), "r"(parity)
         : "memory");
     if (ok) return;
-    if (spin > (1u << 26)) __trap();
+    if ((spin & 1023) == 1023) {
+      const unsigned long long t = gtimer();
+      if (t0 == 0) t0 = t;
+      else if (t - t0 > 20000000000ull) __trap();
+    }
   }
 }
 __device__ __forceinline__ void gather4(void *dst, const CUtensorMap *map, int32_t col, int32_t r0, int32_t r1,
@@ -128,9 +133,6 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
   __syncwarp();
   const int QE = L.qe(), RS = L.rslot(), SS = L.sslot(), BW = L.bw;
   const bool dst_scale = !ATT && scales_dst(p.weight);
-  // per-edge weights (GCN nsrc[u] inside the chain, or explicit per-CSR-entry weights): one
-  // 4-byte cp.async per edge into the slot's side area, tracked by the slot's mbarrier
-  const int wmode = ATT ? 0 : (p.weight == GNN_W_GCN ? 1 : p.weight == GNN_W_EDGE ? 2 : 0);
   const uint32_t row_bytes = 4u * 4u * (uint32_t)BW;
   const uint32_t sc_bytes = ATT ? 4u * 4u * (uint32_t)p.H : 0u;
   const uint32_t xb = ATT ? 4u * (uint32_t)p.H : 16u;
@@ -159,7 +161,6 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
     int32_t eB = 0, eA = 0, eP = 0, nB = 0, nA = 0, nP = 0;
     int32_t T0A = 0, T1A = 0, firstA = 0, T1P = 0;
     int32_t pp = 0, juP = 0, uendP = 0, ib0 = 0, icur = 0, inxt = 0;
-    int32_t ubegP = 0, utposP = 0;  // CSR / task position of the producer's unit (explicit edge weights)
     bool live = false;  // the producer has edges
     auto advance_run = [&]() {
       dP = dA;
@@ -194,15 +195,11 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
     // ---- producer: the next four edges of the stream into slot pslot ----
     auto produce_quad = [&]() {
       int32_t r4[4] = {0, 0, 0, 0};
-      int32_t wpos[4] = {0, 0, 0, 0};  // explicit weights: CSR position of each edge
       int32_t xrow0 = 0, xrow1 = 0, xrow2 = 0, xrow3 = 0, xent0 = 0, xent1 = 0, xent2 = 0, xent3 = 0;
       int nx = 0, nvalid = 0;
       if (live && pp + 4 <= uendP && pp - ib0 <= 28) {  // fast path: four edges of the current unit and batch
 #pragma unroll
-        for (int r = 0; r < 4; ++r) {
-          r4[r] = __shfl_sync(0xffffffffu, icur, pp - ib0 + r);
-          wpos[r] = ubegP + (pp + r - utposP);
-        }
+        for (int r = 0; r < 4; ++r) r4[r] = __shfl_sync(0xffffffffu, icur, pp - ib0 + r);
         pp += 4;
         nvalid = 4;
       } else {
@@ -219,8 +216,6 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
               const int32_t ubeg = __shfl_sync(0xffffffffu, dP.y, juP);
               const int32_t um = __shfl_sync(0xffffffffu, dP.w, juP);
               const int32_t e = qt & (QN - 1);
-              ubegP = ubeg;
-              utposP = pp;
               if (lane == 0) {
                 int *qi = reinterpret_cast<int *>(queue + e * QE);
                 qi[0] = urow;
@@ -246,7 +241,6 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
               inxt = ib0 + 32 + lane < T1P ? ld_stream_i32(g.colidx_t + ib0 + 32 + lane) : 0;
             }
             r4[r] = __shfl_sync(0xffffffffu, icur, pp - ib0);
-            wpos[r] = ubegP + (pp - utposP);
             ++pp;
             ++nvalid;
           }
@@ -257,15 +251,6 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
         ib0 += 32;
         inxt = ib0 + 32 + lane < T1P ? ld_stream_i32(g.colidx_t + ib0 + 32 + lane) : 0;
       }
-      if (wmode && lane < nvalid) {  // per-edge weights: lane r copies edge r's weight
-        const int32_t u = lane == 0 ? r4[0] : lane == 1 ? r4[1] : lane == 2 ? r4[2] : r4[3];
-        const int32_t cp = lane == 0 ? wpos[0] : lane == 1 ? wpos[1] : lane == 2 ? wpos[2] : wpos[3];
-        const float *src = wmode == 1 ? g.nsrc + u : p.edge_w + cp;
-        asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(sa(scs + (size_t)pslot * SS + lane)), "l"(src)
-                     : "memory");
-        asm volatile("cp.async.mbarrier.arrive.shared::cta.b64 [%0];" ::"r"(sa(&bars[w][pslot])) : "memory");
-      }
-      __syncwarp();
       if (lane == 0) {
         uint64_t *bar = &bars[w][pslot];
         uint32_t bytes = (nvalid > 0 ? row_bytes + sc_bytes : 0u) + xb * (uint32_t)nx;
@@ -350,7 +335,7 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
             }
           } else {
 #pragma unroll
-            const float wt = wmode ? sq[r] : 1.0f;
+            const float wt = 1.0f;  // weight 1 (pre-scaled GCN: ndst in the epilogue)
             for (int n = 0; n < NV; ++n) {
               if (!valid[n]) continue;
               float v[VEC];
@@ -457,7 +442,10 @@ bool g4_admissible(const KParams &kp, int32_t n_src) {
     return true;
   }
   if (kp.mode > M_MAX) return false;
-  return true;  // every weight: 1, GCN (nsrc[u] per edge, ndst[v] per row), explicit, pre-scaled GCN
+  // weight 1 or the pre-scaled GCN form (ndst per row); per-edge weights take the
+  // cp.async chain (their 4-byte copies would need cp.async.mbarrier.arrive
+  // tracking, which compute-sanitizer synccheck flags, and measured slower)
+  return kp.weight == GNN_W_ONE || kp.weight == W_DST_ONLY;
 }
 
 template <int MODE, int VEC, int NV>
@@ -465,7 +453,7 @@ static cudaError_t launch_g4_mode(const KParams &kp_in, int32_t n_src, cudaStrea
   using namespace g4;
   g4::Layout L;
   L.bw = kp_in.F < BWMAX ? kp_in.F : BWMAX;
-  L.hs = MODE == M_GAT ? kp_in.H : 4;  // GAT scores, or the 4 per-edge weights of a quad
+  L.hs = MODE == M_GAT ? kp_in.H : 0;  // GAT score columns
   L.xe = MODE == M_GAT ? (kp_in.H < 4 ? 4 : kp_in.H) : 4;
   const size_t smem = L.bytes();
   CUtensorMap rmap, smap;
