@@ -68,7 +68,8 @@ struct KParams {
   const float *Wa;       // Gene: [H, Fh]
   int32_t *ws_unit;  // work-unit counters (one per feature chunk), zeroed per call
   int32_t n_unit_ctr; // number of unit counters (>= feature chunks of any mapping)
-  float *ws_acc;   // [n_multi][FW] atomic accumulators (deterministic == 0)
+  float *ws_acc;   // [n_multi][FW] atomic accumulators (deterministic == 0): sum / max keys / GAT a | l
+  float *ws_rowmax;  // [n_multi][H] GAT, deterministic == 0: exact row maxima of the scores (pre-pass)
   float *ws_part;  // [multi slots][FW] per-group partials (deterministic)
   int32_t *ws_cnt; // [n_multi][nch] arrival counters
   int32_t FW;      // partial slot width: F (+ 2 nmeta for attention), rounded to 8
@@ -347,7 +348,7 @@ __device__ __forceinline__ float head_sum(float x, int lph, unsigned mask) {
 template <int MODE, int VEC, int NV, int LANES>
 __device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx, int32_t len, int32_t beg,
                                             int32_t row, int32_t c0, int lane, unsigned mask,
-                                            Part<MODE, VEC, NV> &G) {
+                                            Part<MODE, VEC, NV> &G, int32_t m = -1) {
   constexpr int FPL = VEC * NV;
   constexpr int U = FPL >= 32 ? 1 : (32 / FPL > 8 ? 8 : 32 / FPL);
   part_init(G);
@@ -358,8 +359,12 @@ __device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx
   float tv[NV];
   float nmb[NV];   // GAT: -m * log2(e) for the current reference m
   float seen[NV];  // GAT: exact max score of the group
+  // GAT, atomic variant (deterministic == 0) on a split row: every group of the
+  // row uses the row's exact score maximum from the pre-pass, so their (a, l)
+  // partials can be added with atomics; never loose
+  const bool rowmax = MODE == M_GAT && !p.deterministic && m >= 0;
   // GAT: a one-edge group takes its own score as reference (term = 1 exactly)
-  const bool one = MODE == M_GAT && len == 1;
+  const bool one = MODE == M_GAT && len == 1 && !rowmax;
 #pragma unroll
   for (int n = 0; n < NV; ++n) {
     const int32_t f = c0 + (n * LANES + lane) * VEC;
@@ -371,7 +376,9 @@ __device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx
     if constexpr (MODE == M_GAT) {
       head[n] = valid[n] ? f / p.Fh : 0;
       tv[n] = valid[n] ? __ldg(p.t + (int64_t)row * p.ldt + head[n]) : 0.0f;
-      const float mb = valid[n] ? leaky_f(fkey_decode(__ldg(p.smax + head[n])) + tv[n], p.slope) : 0.0f;
+      const float mb = !valid[n] ? 0.0f
+                       : rowmax  ? __ldcg(p.ws_rowmax + (size_t)m * p.H + head[n])
+                                 : leaky_f(fkey_decode(__ldg(p.smax + head[n])) + tv[n], p.slope);
       G.m[n] = mb;
       nmb[n] = -mb * kLog2e;
     }
@@ -467,7 +474,7 @@ __device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx
       bool loose = false;
 #pragma unroll
       for (int n = 0; n < NV; ++n) loose |= valid[n] && !(G.m[n] - seen[n] <= kGatSlack);
-      if (pass == 1 || !__any_sync(mask, loose)) break;
+      if (pass == 1 || rowmax || !__any_sync(mask, loose)) break;
 #pragma unroll
       for (int n = 0; n < NV; ++n) {
         G.m[n] = seen[n];
@@ -893,7 +900,7 @@ __device__ __forceinline__ void process_unit(const KParams &p, int4 d, int32_t l
   } else if constexpr (MODE > M_GAT)
     group_chain_att<MODE, VEC, NV, LANES>(p, g.colidx_t + tpos, len, beg, row, c0, lane, mask, G);
   else
-    group_chain<MODE, VEC, NV, LANES>(p, g.colidx_t + tpos, len, beg, row, c0, lane, mask, G);
+    group_chain<MODE, VEC, NV, LANES>(p, g.colidx_t + tpos, len, beg, row, c0, lane, mask, G, m);
   finish_unit<MODE, VEC, NV, LANES>(p, G, row, beg, m, len, c0, ci, lane, mask, nullptr);
 }
 
@@ -913,7 +920,10 @@ __device__ __forceinline__ void finish_unit(const KParams &p, const Part<MODE, V
   const int32_t ng = g.ng;
   const int32_t ngrp = 1 + (re - rb - 1) / ng;
   const int32_t k = (beg - rb) / ng;
-  const bool atomic_acc = !p.deterministic && MODE == M_SUM;
+  // non-deterministic variant: partials meet in one accumulator row
+  // by atomics -- sum / mean: float adds; max: atomicMax on order-preserving
+  // keys (exact); GAT: a and l added against the shared exact row maximum
+  const bool atomic_acc = !p.deterministic && (MODE == M_SUM || MODE == M_MAX || MODE == M_GAT);
   float *base = p.ws_part + (size_t)g.multi_slot[m] * p.FW;
   float *acc = p.ws_acc + (size_t)m * p.FW;
 #pragma unroll
@@ -921,8 +931,16 @@ __device__ __forceinline__ void finish_unit(const KParams &p, const Part<MODE, V
     const int32_t f = c0 + (n * LANES + lane) * VEC;
     if (f >= p.F) continue;
     if (atomic_acc) {
+      if constexpr (MODE == M_MAX) {
 #pragma unroll
-      for (int i = 0; i < VEC; ++i) atomicAdd(acc + f + i, G.a[n][i]);
+        for (int i = 0; i < VEC; ++i) atomicMax(reinterpret_cast<uint32_t *>(acc) + f + i, fkey(G.a[n][i]));
+      } else {
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) atomicAdd(acc + f + i, G.a[n][i]);
+        if constexpr (MODE == M_GAT) {
+          if (f % p.Fh == 0) atomicAdd(acc + p.F + f / p.Fh, G.l[n]);  // heads never straddle chunks here
+        }
+      }
     } else {
       stv<VEC>(base + (size_t)k * p.FW + f, G.a[n]);
       if constexpr (is_att(MODE)) {
@@ -951,7 +969,13 @@ __device__ __forceinline__ void finish_unit(const KParams &p, const Part<MODE, V
 #pragma unroll
     for (int n = 0; n < NV; ++n) {
       const int32_t f = c0 + (n * LANES + lane) * VEC;
-      if (f < p.F) ldv_cg<VEC>(acc + f, A.a[n]);
+      if (f >= p.F) continue;
+      ldv_cg<VEC>(acc + f, A.a[n]);
+      if constexpr (MODE == M_MAX) {
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) A.a[n][i] = fkey_decode(__float_as_uint(A.a[n][i]));
+      }
+      if constexpr (MODE == M_GAT) A.l[n] = __ldcg(acc + p.F + f / p.Fh);
     }
     store_row<MODE, VEC, NV, LANES>(p, row, re - rb, c0, lane, A);
   } else {
@@ -1120,7 +1144,7 @@ cudaError_t launch_persistent(KFN fn, int &occ, const KParams &kp_in, int32_t un
   cudaError_t e = cudaMemsetAsync(kp.ws_unit, 0, sizeof(int32_t) * (size_t)kp.n_unit_ctr, s);
   if (e == cudaSuccess && kp.g.n_multi > 0)
     e = cudaMemsetAsync(kp.ws_cnt, 0, sizeof(int32_t) * (size_t)kp.g.n_multi * kp.nch, s);
-  if (e == cudaSuccess && kp.g.n_multi > 0 && !kp.deterministic && kp.mode != M_MAX && !is_att(kp.mode))
+  if (e == cudaSuccess && kp.g.n_multi > 0 && !kp.deterministic)  // max keys: 0 is below every key
     e = cudaMemsetAsync(kp.ws_acc, 0, sizeof(float) * (size_t)kp.g.n_multi * kp.FW, s);
   if (e != cudaSuccess) return e;
   if (e == cudaSuccess && kp.trace) {
@@ -1198,6 +1222,7 @@ cudaError_t dispatch_vec(const KParams &kp, const Mapping &m, int threads, cudaS
 
 cudaError_t dispatch_sum(const KParams &kp, const Mapping &m, int threads, cudaStream_t s);
 bool g4_admissible(const KParams &kp, int32_t n_src);
+cudaError_t launch_row_score_max(const KParams &kp, cudaStream_t s);
 cudaError_t launch_g4(const KParams &kp, int32_t n_src, cudaStream_t s);
 cudaError_t dispatch_max(const KParams &kp, const Mapping &m, int threads, cudaStream_t s);
 cudaError_t dispatch_gat(const KParams &kp, const Mapping &m, int threads, cudaStream_t s);

@@ -194,6 +194,37 @@ cudaError_t launch_scale_rows(float *Y, int64_t ldy, int64_t n, int32_t F, const
   return cudaGetLastError();
 }
 
+// GAT atomic variant: exact per-row score maxima of the split rows,
+// ws_rowmax[m][h] = max over the row's entries of LeakyReLU(s_u[h] + t_v[h])
+// (monotone: the same value the deterministic merge reaches).  One warp per row.
+__global__ void k_row_score_max(const KParams p) {
+  const int lane = threadIdx.x & 31;
+  const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const DevGraph &g = p.g;
+  for (int64_t m = w; m < g.n_multi; m += nw) {
+    const int32_t row = g.multi_row[m];
+    const int32_t rb = g.rowptr[row], re = g.rowptr[row + 1];
+    for (int32_t h = 0; h < p.H; ++h) {
+      const float tv = __ldg(p.t + (int64_t)row * p.ldt + h);
+      float mx = -INFINITY;
+      for (int32_t k = rb + lane; k < re; k += 32) {
+        const int32_t u = __ldg(g.colidx + k);
+        mx = fmaxf(mx, leaky_f(__ldg(p.X + (int64_t)u * p.ldx + p.F + h) + tv, p.slope));
+      }
+      for (int off = 16; off > 0; off >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, off));
+      if (lane == 0) p.ws_rowmax[m * p.H + h] = mx;
+    }
+  }
+}
+
+cudaError_t launch_row_score_max(const KParams &kp, cudaStream_t s) {
+  const int64_t blocks = std::min<int64_t>((kp.g.n_multi * 32 + 255) / 256, (int64_t)num_sms() * 8);
+  k_row_score_max<<<(unsigned)std::max<int64_t>(1, blocks), 256, 0, s>>>(kp);
+  count_launch();
+  return cudaGetLastError();
+}
+
 // head mean (final attention layer): y[v][f] = (1/H) sum_h Yf[v][h*Fh + f], heads in order
 __global__ void k_head_mean(const float *__restrict__ Yf, int64_t ldf, int64_t n, int32_t H, int32_t Fh, float *Y,
                             int64_t ldy) {
@@ -388,7 +419,7 @@ static int32_t att_meta(int mode, int32_t F, int32_t H) { return is_att(mode) ? 
 static int32_t slot_width(int mode, int32_t F, int32_t H) { return (F + 2 * att_meta(mode, F, H) + 7) / 8 * 8; }
 
 struct WsLayout {
-  size_t unit, smax, cnt, acc, part, total;
+  size_t unit, smax, cnt, acc, part, rowmax, total;
 };
 static WsLayout ws_layout(const gnn_plan_s *p, int mode, int32_t F, int32_t H) {
   const size_t FW = (size_t)slot_width(mode, F, H);
@@ -398,7 +429,8 @@ static WsLayout ws_layout(const gnn_plan_s *p, int mode, int32_t F, int32_t H) {
   L.cnt = L.smax + smax_bytes(mode, H);
   L.acc = L.cnt + a256(sizeof(int32_t) * (size_t)p->n_multi * max_chunks(F));
   L.part = L.acc + sizeof(float) * (size_t)p->n_multi * FW;
-  L.total = L.part + sizeof(float) * (size_t)p->multi_slots * FW;
+  L.rowmax = L.part + sizeof(float) * (size_t)p->multi_slots * FW;
+  L.total = L.rowmax + (is_att(mode) ? sizeof(float) * (size_t)p->n_multi * (size_t)(H > 0 ? H : 0) : 0);
   return L;
 }
 
@@ -458,6 +490,7 @@ gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, siz
   kp.ws_cnt = reinterpret_cast<int32_t *>(w + L.cnt);
   kp.ws_acc = reinterpret_cast<float *>(w + L.acc);
   kp.ws_part = reinterpret_cast<float *>(w + L.part);
+  kp.ws_rowmax = reinterpret_cast<float *>(w + L.rowmax);
   Mapping m = choose_mapping(p, a, is_att(mode) ? a.Fh : 0);
   if (m.vec == 0) {
     set_error("no supported lane mapping for this width / head size (GaAN, Gene: Fh/vec must be a power of 2 <= 32)");
@@ -471,6 +504,21 @@ gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, siz
   if (e == cudaSuccess && mode == M_SYM) e = launch_score_max(a.X + a.F + a.H, a.ldx, p->n_src, a.H, 1, smax + a.H, s);
   if (e == cudaSuccess && mode == M_GAAN) e = launch_score_max(a.X + a.F, a.ldx, p->n_src, a.H, a.Fh, smax, s);
   if (e != cudaSuccess) return cuda_status(e, "score max launch");
+  if (!kp.deterministic && is_att(mode)) {
+    // atomic variant for GAT only, when no head straddles a feature chunk (the
+    // l of a head is added by the chunk holding it); otherwise the
+    // deterministic merge.  The register kernel computes the rowmax chains.
+    const int cw = m.vec * m.lanes * m.nv;
+    if (mode != M_GAT || !(cw >= a.F || cw % a.Fh == 0)) {
+      kp.deterministic = 1;
+    } else {
+      m.cp = 0;
+      if (p->n_multi > 0) {
+        e = launch_row_score_max(kp, s);
+        if (e != cudaSuccess) return cuda_status(e, "row score max launch");
+      }
+    }
+  }
   if (m.cp == 2) {  // gather4 streaming kernel (k_agg_g4.cu)
     KParams kq = kp;
     kq.n_unit_ctr = kp.n_unit_ctr;

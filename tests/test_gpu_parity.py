@@ -224,6 +224,29 @@ def test_nondeterministic_variant_within_tolerance(graphs):
     assert_close(H(G.aggregate(plan, T(X), "sum", "one")), ref, what="atomic raw sum", S=S, deg=np.diff(g.rowptr))
 
 
+@pytest.mark.parametrize("F", [32, 64, 100, 256])
+def test_nondeterministic_max_and_gat(graphs, F):
+    """a9 fast variant: split rows combined with atomics -- max by
+    atomicMax on order-preserving keys (still exact, so bit-identical to the
+    oracle), GAT by atomically added (a, l) against the row's exact score
+    maximum from a pre-pass (tolerance R11); sum at the staged kernels' widths."""
+    g = graphs["hub"]
+    plan = G.Plan(g.rowptr, g.colidx, group_size=16, deterministic=0)
+    X = gs.uniform(g.n, F, seed=F + 1)
+    ref = oracle.aggregate(g.rowptr, g.colidx, X, "max", "one")
+    assert np.array_equal(H(G.aggregate(plan, T(X), "max", "one")), ref)
+    ref, S = oracle.aggregate(g.rowptr, g.colidx, X, "sum", "one", return_abs=True)
+    assert_close(H(G.aggregate(plan, T(X), "sum", "one")), ref, what=f"atomic sum F={F}", S=S,
+                 deg=np.diff(g.rowptr))
+    Hh = 8 if F % 8 == 0 else 4
+    Fh = F // Hh
+    Zs = gs.uniform(g.n, F + Hh, seed=3)
+    Zs[:, F:] *= 3.0
+    t = gs.uniform(g.n, Hh, lo=-3, hi=3, seed=4)
+    refg = oracle.gat_aggregate(g.rowptr, g.colidx, Zs, t, Hh, Fh, 0.2)
+    assert_close(H(G.gat_aggregate(plan, T(Zs), T(t), Hh, Fh, 0.2)), refg, what=f"atomic GAT {Hh}x{Fh}")
+
+
 def test_strided_and_offset_views():
     """ld > F and unaligned column offsets fall back to narrower vectors."""
     g = gs.random_small(200, avg_deg=6, seed=9)
