@@ -308,10 +308,11 @@ def measure_traffic(g, inp, model, kernel):
     try:
         model.plan.save(os.path.join(d, "plan.gnnplan"))
         np.savez(os.path.join(d, "meta.npz"), n=g.n, F_in=inp["F_in"], F=inp["F"], H=inp["H"], Fh=inp["Fh"])
-        regex = {"gat_agg_8x32": "k_aggregate<3|k_stream_g4<3", "agg2_F256": "k_aggregate<0|k_stream_g4<0",
-                 "agg1_F100": "k_aggregate<0|k_stream_g4<0"}[kernel]
+        # the probe launches the kernel twice (k_score_max for GAT is not matched):
+        # profile the second launch
         cmd = [ncu, "--metrics", "dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum",
-               "--clock-control", "none", "-k", f"regex:{regex}", "-s", "1", "-c", "1", "--csv", "--page", "raw",
+               "--clock-control", "none", "-k", "regex:k_aggregate|k_stream_g4", "-s", "1", "-c", "1", "--csv",
+               "--page", "raw",
                sys.executable, os.path.join(ROOT, "scripts", "traffic_probe.py"), d, kernel]
         r = subprocess.run(cmd, capture_output=True, text=True, timeout=300)
         import csv
@@ -319,7 +320,8 @@ def measure_traffic(g, inp, model, kernel):
         rows = [ln for ln in r.stdout.splitlines() if ln.startswith('"')]
         rec = list(csv.reader(io.StringIO("\n".join(rows))))
         if len(rec) < 3:
-            return None, f"ncu produced no record (rc {r.returncode})"
+            tail = (r.stdout[-300:] + r.stderr[-300:]).replace("\n", " ")
+            return None, f"ncu produced no record (rc {r.returncode}): {tail}"
         h, units, vals = rec[0], rec[1], rec[2]
         scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
 

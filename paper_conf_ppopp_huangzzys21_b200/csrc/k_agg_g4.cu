@@ -478,7 +478,7 @@ static cudaError_t launch_g4_mode(const KParams &kp_in, int32_t n_src, cudaStrea
   cudaError_t e = cudaMemsetAsync(kp.ws_unit, 0, sizeof(int32_t) * (size_t)kp.n_unit_ctr, s);
   if (e == cudaSuccess && kp.g.n_multi > 0)
     e = cudaMemsetAsync(kp.ws_cnt, 0, sizeof(int32_t) * (size_t)kp.g.n_multi * kp.nch, s);
-  if (e == cudaSuccess && kp.g.n_multi > 0 && !kp.deterministic && kp.mode == M_SUM)
+  if (e == cudaSuccess && kp.g.n_multi > 0 && !kp.deterministic)  // sums and max keys start at 0
     e = cudaMemsetAsync(kp.ws_acc, 0, sizeof(float) * (size_t)kp.g.n_multi * kp.FW, s);
   if (e == cudaSuccess && kp.trace) {
     e = cudaMemsetAsync(kp.trace, 0, 8 * sizeof(unsigned long long), s);
