@@ -330,8 +330,9 @@ def measure_traffic(g, inp, model, kernel):
             return float(vals[i].replace(",", "")) * scale.get(units[i], 1)
         tot = val("dram__bytes_read.sum") + val("dram__bytes_write.sum")
         it = h.index("gpu__time_duration.sum")
-        t_ms = float(vals[it].replace(",", "")) * {"nsecond": 1e-6, "usecond": 1e-3, "msecond": 1.0,
-                                                   "second": 1e3}.get(units[it], 1.0)
+        t_ms = float(vals[it].replace(",", "")) * {"nsecond": 1e-6, "ns": 1e-6, "usecond": 1e-3, "us": 1e-3,
+                                                   "msecond": 1.0, "ms": 1.0, "second": 1e3,
+                                                   "s": 1e3}.get(units[it].strip(), 1e-6)
         return int(tot), (f"ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum on one launch of "
                           f"{vals[h.index('Kernel Name')]} (this run's plan; cold cache; {t_ms:.3f} ms under ncu)")
     except Exception as e:  # noqa: BLE001
