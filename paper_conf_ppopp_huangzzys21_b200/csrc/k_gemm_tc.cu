@@ -107,7 +107,7 @@ struct TcParams {
   int32_t att_H, att_Fh, att_col;
 };
 
-template <bool VEC_X, bool VEC_H, bool TMA_X>
+template <bool VEC_X, bool VEC_H, bool TMA_X, bool CTA2 = false>
 __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams p, const __grid_constant__ CUtensorMap xmap,
                                                           const __grid_constant__ CUtensorMap hmap) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -122,12 +122,22 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
   // bytes) -> empty (MMA)
   __shared__ uint64_t full_bar[MAX_STAGES], empty_bar[MAX_STAGES], xfull_bar[MAX_STAGES], afull_bar[MAX_STAGES],
       aempty_bar[MAX_STAGES], lempty_bar[MAX_STAGES], tfull_bar[2], tempty_bar[2];
+  // CTA pair: the peer's "stage it complete" gate, arrived remotely on the leader
+  __shared__ uint64_t peer_bar[MAX_STAGES];
   __shared__ uint32_t tmem_base_sh;
 
   const int tid = threadIdx.x;
   const int warp = tid >> 5;
   const int lane = tid & 31;
   const int S = p.stages;
+  // CTA pair (TMA path, cluster of 2): a row tile is 256 rows, 128 per CTA;
+  // each CTA holds its rows of X and half of the item's W columns; the
+  // leader (rank 0) issues the cta_group::2 MMAs for both
+  const uint32_t crank = CTA2 ? cluster_ctarank() : 0u;
+  const int cta_id = CTA2 ? (int)(blockIdx.x >> 1) : (int)blockIdx.x;
+  const int n_cta = CTA2 ? (int)(gridDim.x >> 1) : (int)gridDim.x;
+  constexpr int ROWS = CTA2 ? 2 * BM : BM;
+  const int n_epi_warps = p.epi8 ? 8 : 4;
 
   if (tid == 0) {
     if (TMA_X) {
@@ -151,27 +161,36 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(&tfull_bar[b], 1);
-      mbar_init(&tempty_bar[b], 128 * (p.epi8 ? 2 : 1));
+      // pair: one arrival per epilogue warp of both CTAs (on the leader's barrier)
+      mbar_init(&tempty_bar[b], CTA2 ? 2 * n_epi_warps : 128 * (p.epi8 ? 2 : 1));
     }
+    if (CTA2)
+      for (int s = 0; s < MAX_STAGES; ++s) mbar_init(&peer_bar[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == MMA_WARP) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_u32(&tmem_base_sh)));
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    if (CTA2) {
+      asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_u32(&tmem_base_sh)));
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
+    } else {
+      asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_u32(&tmem_base_sh)));
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
   }
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
+  if (CTA2) cluster_sync_all();  // both CTAs' barriers initialised before any remote arrive
   asm volatile("tcgen05.fence::after_thread_sync;");
   const uint32_t tmem = tmem_base_sh;
 
-  const int my_tiles = p.num_tiles > (int)blockIdx.x ? (p.num_tiles - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0;
+  const int my_tiles = p.num_tiles > cta_id ? (p.num_tiles - 1 - cta_id) / n_cta + 1 : 0;
   const int total_it = my_tiles * p.num_kb;
-  auto tile_of = [&](int it) { return (int)blockIdx.x + (it / p.num_kb) * (int)gridDim.x; };
+  auto tile_of = [&](int it) { return cta_id + (it / p.num_kb) * n_cta; };
   // TMA path: work item vt = (row tile vt / ncb, column block vt % ncb); a
   // column block is a slice of the W image (rows cb_beg .. cb_beg + cb_w)
   auto cb_beg = [&](int vt) { return (p.ncb > 1 && vt % p.ncb) ? p.cbw0 : 0; };
   auto cb_w = [&](int vt) { return p.ncb > 1 ? ((vt % p.ncb) ? NP - p.cbw0 : p.cbw0) : NP; };
-  const int B_STAGE = 2 * (p.ncb > 1 ? p.cbw0 : NP) * 128;  // TMA path B ring stage
+  const int B_STAGE = 2 * (p.ncb > 1 ? p.cbw0 : NP) * 128 / (CTA2 ? 2 : 1);  // TMA path B ring stage
   // TMA path smem: [raw X ring sa x 16 KB][X_lo ring sl x 16 KB][W ring sb x B_STAGE][epilogue staging]
   uint8_t *const lo_ring = smem + (size_t)p.sa * TILE_A_BYTES;
   uint8_t *const b_ring = lo_ring + (size_t)p.sl * TILE_A_BYTES;
@@ -182,8 +201,8 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
         const int s = it % p.sa, use = it / p.sa;
         if (use > 0) mbar_wait(&aempty_bar[s], (use - 1) & 1);
         mbar_arrive_expect_tx(&xfull_bar[s], TILE_A_BYTES);
-        tma_load_2d(smem + (size_t)s * TILE_A_BYTES, &xmap, (it % p.num_kb) * BK, (tile_of(it) / p.ncb) * BM,
-                    &xfull_bar[s]);
+        tma_load_2d(smem + (size_t)s * TILE_A_BYTES, &xmap, (it % p.num_kb) * BK,
+                    (tile_of(it) / p.ncb) * ROWS + (int)crank * BM, &xfull_bar[s]);
       }
     }
   } else if (TMA_X && warp == WIMG_WARP) {
@@ -192,10 +211,13 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
       for (int it = 0; it < total_it; ++it) {
         const int s = it % p.sb, use = it / p.sb;
         if (use > 0) mbar_wait(&empty_bar[s], (use - 1) & 1);
-        const int vt = tile_of(it), w = cb_w(vt);
+        const int vt = tile_of(it), w = cb_w(vt) / (CTA2 ? 2 : 1);  // pair: this CTA's half of the columns
         const int wb = w * 128;  // bytes of one (hi or lo) slice
+#ifdef GNN_GEMM_DBG_NOW
+        if (use >= p.sb) { mbar_arrive(&full_bar[s]); continue; }  // first fill only: MMAs read stale W
+#endif
         mbar_arrive_expect_tx(&full_bar[s], 2 * wb);
-        const uint8_t *src = p.wimg + (size_t)(it % p.num_kb) * 2 * B_BYTES + (size_t)cb_beg(vt) * 128;
+        const uint8_t *src = p.wimg + (size_t)(it % p.num_kb) * 2 * B_BYTES + (size_t)(cb_beg(vt) + (int)crank * w) * 128;
         uint8_t *b_img = b_ring + (size_t)s * B_STAGE;
         for (int part = 0; part < 2; ++part)  // hi slice, then lo slice (stage layout [hi w | lo w])
           for (int off = 0; off < wb; off += 16384) {
@@ -215,6 +237,11 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
       const int s = it % p.sa, use = it / p.sa;
       const int l = it % p.sl, luse = it / p.sl;
       mbar_wait(&xfull_bar[s], use & 1);
+#ifdef GNN_GEMM_DBG_NOSPLIT
+      if (luse > 0) mbar_wait(&lempty_bar[l], (luse - 1) & 1);
+      mbar_arrive(&afull_bar[l]);
+      continue;
+#endif
       const float4 *a_raw = reinterpret_cast<const float4 *>(smem + (size_t)s * TILE_A_BYTES);
       float4 x[PER];
 #pragma unroll
@@ -296,16 +323,29 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
       it += 2;
       if (it < total_it) load_a((int64_t)tile_of(it) * BM, it % p.num_kb);
     }
+  } else if (CTA2 && warp == MMA_WARP && crank != 0) {
+    // ------------------- pair peer: gate its stages to the leader -------------------
+    if (lane == 0)
+      for (int it = 0; it < total_it; ++it) {
+        mbar_wait(&xfull_bar[it % p.sa], (it / p.sa) & 1);
+        mbar_wait(&afull_bar[it % p.sl], (it / p.sl) & 1);
+        mbar_wait(&full_bar[it % p.sb], (it / p.sb) & 1);
+        mbar_arrive_cluster(&peer_bar[it % MAX_STAGES], 0);
+      }
+    __syncwarp();
   } else if (warp == MMA_WARP) {
     // ------------------------------ MMA issuer ------------------------------
     int it = 0, tcount = 0;
-    for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++tcount) {
+    for (int tile = cta_id; tile < p.num_tiles; tile += n_cta, ++tcount) {
       const int b = tcount % p.n_buf, buse = tcount / p.n_buf;
-      if (buse > 0) mbar_wait(&tempty_bar[b], (buse - 1) & 1);
+      if (buse > 0) {
+        if (CTA2) mbar_wait_cluster(&tempty_bar[b], (buse - 1) & 1);
+        else mbar_wait(&tempty_bar[b], (buse - 1) & 1);
+      }
       asm volatile("tcgen05.fence::after_thread_sync;");
       const uint32_t tbase = tmem + (uint32_t)(b * p.n_acc * p.npa);
       const int NW = TMA_X ? cb_w(tile) : NP;  // MMA width of this work item
-      const uint32_t b_lo_off = TMA_X ? (uint32_t)NW * 128 : (uint32_t)B_BYTES;
+      const uint32_t b_lo_off = TMA_X ? (uint32_t)(NW / (CTA2 ? 2 : 1)) * 128 : (uint32_t)B_BYTES;
       for (int kb = 0; kb < p.num_kb; ++kb, ++it) {
         int s, sA, sL = 0;
         uint32_t a_hi, a_lo, b_hi;
@@ -316,6 +356,7 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
           mbar_wait(&xfull_bar[sA], (it / p.sa) & 1);
           mbar_wait(&afull_bar[sL], (it / p.sl) & 1);
           mbar_wait(&full_bar[s], (it / p.sb) & 1);
+          if (CTA2) mbar_wait_cluster(&peer_bar[it % MAX_STAGES], (it / MAX_STAGES) & 1);
           a_hi = smem_u32(smem + (size_t)sA * TILE_A_BYTES);
           a_lo = smem_u32(lo_ring + (size_t)sL * TILE_A_BYTES);
           b_hi = smem_u32(b_ring + (size_t)s * B_STAGE);
@@ -332,9 +373,17 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
           const int acc = kb % p.n_acc;
           const uint32_t d0 = tbase + (uint32_t)(acc * p.npa);
           const uint32_t first = (kb < p.n_acc) ? 1u : 0u;  // first K block of this accumulator
+#ifndef GNN_GEMM_DBG_NOMMA
 #pragma unroll
           for (int j = 0; j < BK / 8; ++j) {  // 8 tf32 (32 B) per MMA K step
             const uint32_t ko = j * 32;
+            if (CTA2) {  // NW <= 256: one pair MMA per term
+              const uint32_t id = idesc_tf32_pair(NW);
+              mma_tf32_pair(d0, sw128_desc(a_lo + ko), sw128_desc(b_hi + ko), id, (first && j == 0) ? 0u : 1u);
+              mma_tf32_pair(d0, sw128_desc(a_hi + ko), sw128_desc(b_lo + ko), id, 1u);
+              mma_tf32_pair(d0, sw128_desc(a_hi + ko), sw128_desc(b_hi + ko), id, 1u);
+              continue;
+            }
             for (int n0 = 0; n0 < NW; n0 += 256) {
               const int nn = NW - n0 < 256 ? NW - n0 : 256;
               const uint32_t id = idesc_tf32(nn);
@@ -345,12 +394,20 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
               mma_tf32(d, sw128_desc(a_hi + ko), sw128_desc(b_hi + bo + ko), id, 1u);
             }
           }
-          mma_commit(&empty_bar[s]);
-          if (TMA_X) {
-            mma_commit(&aempty_bar[sA]);
-            mma_commit(&lempty_bar[sL]);
+#endif
+          if (CTA2) {
+            mma_commit_pair(&empty_bar[s]);
+            mma_commit_pair(&aempty_bar[sA]);
+            mma_commit_pair(&lempty_bar[sL]);
+            if (kb == p.num_kb - 1) mma_commit_pair(&tfull_bar[b]);
+          } else {
+            mma_commit(&empty_bar[s]);
+            if (TMA_X) {
+              mma_commit(&aempty_bar[sA]);
+              mma_commit(&lempty_bar[sL]);
+            }
+            if (kb == p.num_kb - 1) mma_commit(&tfull_bar[b]);
           }
-          if (kb == p.num_kb - 1) mma_commit(&tfull_bar[b]);
         }
         __syncwarp();
       }
@@ -365,7 +422,11 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
     // TMA path (VEC_H): each warp stages its 32 rows x 32 columns in a
     // SWIZZLE_128B buffer (row = lane, conflict-free float4 writes) and one
     // lane stores it with a TMA bulk tensor store (coalesced; tails clipped)
+#ifdef GNN_GEMM_DBG_REGSTORE
+    constexpr bool TMA_H = false;
+#else
     constexpr bool TMA_H = TMA_X && VEC_H;
+#endif
     // with 8 epilogue warps the two warps of a TMEM lane quadrant take
     // contiguous halves of the item's 32-column chunks (a head's chunks stay
     // with one thread for the attention-score epilogue)
@@ -374,7 +435,7 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
     uint8_t *const epi_buf = b_ring + (size_t)p.sb * B_STAGE + (size_t)widx * p.eb * 4096;
     int chunk = 0;
     int tcount = 0;
-    for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++tcount) {
+    for (int tile = cta_id; tile < p.num_tiles; tile += n_cta, ++tcount) {
       const int b = tcount % p.n_buf, buse = tcount / p.n_buf;
       mbar_wait(&tfull_bar[b], buse & 1);
       asm volatile("tcgen05.fence::after_thread_sync;");
@@ -382,7 +443,8 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
       const int rt = TMA_H ? tile / p.ncb : tile;    // row tile
       const int cbb = TMA_H ? cb_beg(tile) : 0;      // first global column of this work item
       const int NW = TMA_H ? cb_w(tile) : NP;
-      const int64_t gm = (int64_t)rt * BM + r;
+      const int64_t row0 = (int64_t)rt * ROWS + (int64_t)crank * BM;  // this CTA's first row of the tile
+      const int64_t gm = row0 + r;
       const float sc = (p.row_scale && gm < p.m) ? __ldg(p.row_scale + gm) : 1.0f;
       const uint32_t tbase = tmem + (uint32_t)(b * p.n_acc * p.npa) + ((uint32_t)(quad * 32) << 16);
       const int n_acc_used = p.num_kb < p.n_acc ? p.num_kb : p.n_acc;
@@ -397,6 +459,17 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
           p.H[gm * p.ldh + p.att_col + p.att_H + att_h] = att_t;
         }
       };
+#ifdef GNN_GEMM_DBG_NOEPI
+      (void)att_flush;
+      asm volatile("tcgen05.fence::before_thread_sync;");
+      if (CTA2) {
+        __syncwarp();
+        if (lane == 0) mbar_arrive_cluster(&tempty_bar[b], 0);
+      } else {
+        mbar_arrive(&tempty_bar[b]);
+      }
+      continue;
+#endif
       for (int c0 = (half ? cmid : 0) * 32; c0 < (half ? nchunk : cmid) * 32; c0 += 32) {
         float y[32];
 #pragma unroll
@@ -456,7 +529,7 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
                 make_float4(y[4 * c], y[4 * c + 1], y[4 * c + 2], y[4 * c + 3]);
           asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
           __syncwarp();
-          if (lane == 0) tma_store_2d(&hmap, cbb + c0, (int32_t)(rt * BM + quad * 32), buf);
+          if (lane == 0) tma_store_2d(&hmap, cbb + c0, (int32_t)(row0 + quad * 32), buf);
           ++chunk;
           continue;
         }
@@ -472,15 +545,22 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
       }
       if (p.att) att_flush();
       asm volatile("tcgen05.fence::before_thread_sync;");
-      mbar_arrive(&tempty_bar[b]);
+      if (CTA2) {
+        __syncwarp();
+        if (lane == 0) mbar_arrive_cluster(&tempty_bar[b], 0);
+      } else {
+        mbar_arrive(&tempty_bar[b]);
+      }
     }
     if (TMA_H && lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
   }
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
+  if (CTA2) cluster_sync_all();  // the leader's last commits land in the peer; the peer's arrives in the leader
   if (warp == MMA_WARP) {
     asm volatile("tcgen05.fence::after_thread_sync;");
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem));
+    if (CTA2) asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, 512;" ::"r"(tmem));
+    else asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem));
   }
 }
 
@@ -488,11 +568,13 @@ struct Config {
   int np, npa, num_kb, stages, n_acc, n_buf;
   int sa, sb, sl, eb, epi8;
   int ncb, cbw0, npa_t, nbuf_t, nacc_t;  // TMA path: column blocks and their TMEM layout
+  int cta2;                              // TMA path: CTA pairs (cta_group::2)
   size_t smem, smem_tma, wimg_bytes;
 };
 
 static int g_epi8 = -1;  // 8 epilogue warps on the TMA path (A/B switch: env GNN_GEMM_EPI8=0 disables)
 static int g_cb = -1;  // column blocks on the TMA path (A/B switch: env GNN_GEMM_CB=0 disables)
+static int g_cta2 = -1;  // CTA pairs on the TMA path (A/B switch: env GNN_GEMM_CTA2=0/1)
 static bool configure(int64_t m, int32_t k, int32_t n, Config &c) {
   if (n < 1 || n > 512 || k < 1 || m < 1) return false;
   c.np = (n + 15) / 16 * 16;
@@ -524,24 +606,40 @@ static bool configure(int64_t m, int32_t k, int32_t n, Config &c) {
       c.cbw0 = c.np;
     }
   }
+  // CTA pairs (cta_group::2): every work item <= 256 columns and >= 32 (the
+  // pair MMA's N), so each CTA holds half of the item's W columns
+  if (g_cta2 < 0) {
+    const char *e = getenv("GNN_GEMM_CTA2");
+    g_cta2 = (e && e[0] == '0') ? 0 : (e && e[0] == '1') ? 1 : 0;
+  }
+  c.cta2 = 0;
+  if (g_cta2) {
+    const bool ok1 = c.ncb == 1 && c.np >= 32 && c.np <= 256;
+    const bool ok2 = c.ncb == 2 && c.cbw0 >= 32 && c.cbw0 <= 256 && c.np - c.cbw0 >= 32 && c.np - c.cbw0 <= 256;
+    c.cta2 = (ok1 || ok2) ? 1 : 0;
+  }
   // TMA path: raw X ring (sa x 16 KB, the TMA destination and A_hi), X_lo
   // ring (sl = 2 x 16 KB), W ring (sb x 2 x cbw0 x 128 B), epilogue staging
   // (8 warps x eb x 4 KB).  The X loads come from HBM and need the depth
   // (ncu r2: the MMA warp waited on X 33% of the time with 2 stages), so the
   // raw ring gets what is left after W (2 stages) and the staging (eb = 1).
   {
-    const size_t budget = 225 * 1024, b_bytes = 2 * (size_t)c.cbw0 * 128;
+    const size_t budget = 225 * 1024, b_bytes = 2 * (size_t)c.cbw0 * 128 / (c.cta2 ? 2 : 1);
     if (g_epi8 < 0) {
       const char *e = getenv("GNN_GEMM_EPI8");
       g_epi8 = (e && e[0] == '0') ? 0 : 1;
     }
-    static int env_sa = -2;
+    static int env_sa = -2, env_sb = -2, env_sl = -2;
     if (env_sa == -2) {
       const char *e = getenv("GNN_GEMM_SA");
       env_sa = e ? atoi(e) : -1;
+      e = getenv("GNN_GEMM_SB");
+      env_sb = e ? atoi(e) : -1;
+      e = getenv("GNN_GEMM_SL");
+      env_sl = e ? atoi(e) : -1;
     }
-    c.sl = 2;
-    c.sb = 2;
+    c.sl = env_sl >= 2 && env_sl <= MAX_STAGES ? env_sl : 2;
+    c.sb = env_sb >= 2 && env_sb <= MAX_STAGES ? env_sb : 2;
     c.epi8 = g_epi8 ? 1 : 0;
     c.eb = 1;
     auto need = [&](int sa, int sb, int eb, int e8) {
@@ -716,9 +814,10 @@ static cudaError_t launch_gemm_tc_one(const float *X, int64_t ldx, const float *
     k_gemm_wimage<<<blocks, 256, 0, s>>>(W, ldw, k, n, c.np, c.num_kb, img);
     count_launch();
   }
-  const int64_t num_tiles = (m + BM - 1) / BM;
-  if (num_tiles > 0x3fffffff) return cudaErrorNotSupported;
-  TcParams p{X, ldx, H, ldh, img, m, k, n, c.np, c.npa, c.num_kb, (int32_t)num_tiles, c.stages, c.n_acc, c.n_buf,
+  const int64_t rows_per_tile = c.cta2 ? 2 * BM : BM;  // a pair tile is 256 rows
+  const int64_t num_tiles0 = (m + BM - 1) / BM;
+  if (num_tiles0 > 0x3fffffff) return cudaErrorNotSupported;
+  TcParams p{X, ldx, H, ldh, img, m, k, n, c.np, c.npa, c.num_kb, (int32_t)num_tiles0, c.stages, c.n_acc, c.n_buf,
              c.sa, c.sb, c.sl, c.eb, 1, c.np, c.epi8, row_scale, col_bias, relu, att.a, att.a_dst, att.H, att.Fh, att.col};
   const bool vx = (ldx % 4 == 0) && ((uintptr_t)X % 16 == 0);
   const bool vh = (ldh % 4 == 0) && ((uintptr_t)H % 16 == 0);
@@ -729,7 +828,11 @@ static cudaError_t launch_gemm_tc_one(const float *X, int64_t ldx, const float *
   memset(&hmap, 0, sizeof(hmap));
   const bool tma = vx && c.sa > 0 && (vh || c.ncb == 1) && tma_enabled() && m < 0x7fffff00LL && encode_x_map(&xmap, X, ldx, m, k) &&
                    (!vh || encode_h_map(&hmap, H, ldh, m, n));
-  auto fn = tma ? (vh ? k_gemm_tc<true, true, true> : k_gemm_tc<true, false, true>)
+  const bool pair = tma && c.cta2;
+  const int64_t num_tiles = pair ? (m + rows_per_tile - 1) / rows_per_tile : num_tiles0;
+  p.num_tiles = (int32_t)num_tiles;
+  auto fn = pair ? (vh ? k_gemm_tc<true, true, true, true> : k_gemm_tc<true, false, true, true>)
+          : tma ? (vh ? k_gemm_tc<true, true, true> : k_gemm_tc<true, false, true>)
                 : vx ? (vh ? k_gemm_tc<true, true, false> : k_gemm_tc<true, false, false>)
                      : (vh ? k_gemm_tc<false, true, false> : k_gemm_tc<false, false, false>);
   const size_t smem = tma ? c.smem_tma : c.smem;
@@ -751,6 +854,37 @@ static cudaError_t launch_gemm_tc_one(const float *X, int64_t ldx, const float *
     if (ws0 % att.Fh != 0 || ws1 % att.Fh != 0) return cudaErrorNotSupported;
     for (int w : {ws0, ws1})
       if ((((w + 31) / 32 + 1) / 2 * 32) % att.Fh != 0) p.epi8 = 0;
+  }
+  if (pair) {
+    // one persistent CTA pair per co-resident cluster slot (clusters of 2
+    // share a TPC), or one per work item when there are fewer
+    cudaLaunchConfig_t cfg = {};
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = 2;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.blockDim = dim3(threads_of(true));
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    static int max_clusters[2] = {0, 0};  // per epilogue variant (vh)
+    int &mc = max_clusters[vh ? 1 : 0];
+    cfg.gridDim = dim3(2 * (num_sms / 2));
+    if (mc == 0) {
+      int nc = 0;
+      if (cudaOccupancyMaxActiveClusters(&nc, fn, &cfg) != cudaSuccess || nc < 1) {
+        (void)cudaGetLastError();
+        nc = num_sms / 2;
+      }
+      mc = nc;
+    }
+    const int clusters = (int)(p.num_tiles < mc ? p.num_tiles : mc);
+    cfg.gridDim = dim3(2 * clusters);
+    e = cudaLaunchKernelEx(&cfg, fn, p, xmap, hmap);
+    count_launch();
+    return e != cudaSuccess ? e : cudaGetLastError();
   }
   // one persistent CTA per SM, or one per work item when there are fewer
   const int grid = (int)(p.num_tiles < num_sms ? p.num_tiles : num_sms);

@@ -30,7 +30,7 @@ def timeit(fn, iters=10, warm=3):
     return a.elapsed_time(b) / iters
 
 
-tag = " ".join(f"{k}={os.environ[k]}" for k in ("GNN_GEMM_CB", "GNN_GEMM_SA", "GNN_GEMM_EPI8") if k in os.environ)
+tag = " ".join(f"{k}={os.path.basename(os.environ[k])}" for k in ("GNN_GEMM_CB", "GNN_GEMM_SA", "GNN_GEMM_EPI8", "GNN_LIB_PATH") if k in os.environ)
 torch.manual_seed(0)
 for name, m, k, n, relu, scale in SHAPES:
     X = torch.rand(m, k, device="cuda") * 2 - 1
