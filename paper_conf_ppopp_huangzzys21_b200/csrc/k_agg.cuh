@@ -720,10 +720,98 @@ template <int N>
 __device__ __forceinline__ void cp_wait() {
   asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
 }
+// branch-free forms for the lean chain: a 16-byte copy that zero-fills (reads
+// nothing) when src_bytes == 0, and a predicated 4-byte copy
+__device__ __forceinline__ void cp_async16_zfill(uint32_t dst, const void *src, uint32_t src_bytes) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
+}
+__device__ __forceinline__ void cp_async4_if(uint32_t dst, const void *src, uint32_t pred) {
+  asm volatile(
+      "{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %2, 0;\n\t@q cp.async.ca.shared.global [%0], [%1], 4;\n\t}" ::"r"(dst),
+      "l"(src), "r"(pred)
+      : "memory");
+}
 // slot size in floats: NV*128 features + the extras (H <= 32 GAT scores, or one weight), 16-byte multiple
 template <int MODE, int NV>
 __host__ __device__ constexpr int cp_slot_floats() {
   return NV * 128 + (MODE == M_GAT ? 32 : 4);
+}
+
+// Lean chain for sum / mean / max (no GAT): the per-edge issue is branch-free
+// (row copies zero-fill on the lanes past F, the weight copy is one predicated
+// instruction by lane 0) and the ring slots are running counters, which cuts
+// the instructions per edge of the F <= 128 gather (C5 agg1 is issue-bound,
+// not byte-bound).  Same copies, same arithmetic order as group_chain_cp.
+template <int MODE, int NV, int S>
+__device__ __forceinline__ void group_chain_cp_lean(const KParams &p, const int32_t *idx, int32_t len, int32_t beg,
+                                                    int32_t c0, int lane, float *ring, Part<MODE, 4, NV> &G) {
+  constexpr int VEC = 4;
+  constexpr int SLOT = cp_slot_floats<MODE, NV>();
+  static_assert(MODE != M_GAT, "lean chain: sum / mean / max only");
+  part_init(G);
+  const int weight = p.weight;
+  const bool has_w = weight == GNN_W_GCN || weight == GNN_W_EDGE;
+  const uint32_t ring_s = (uint32_t)__cvta_generic_to_shared(ring);
+  uint32_t nbytes[NV];
+#pragma unroll
+  for (int n = 0; n < NV; ++n) nbytes[n] = (c0 + (n * 32 + lane) * VEC < p.F) ? 16u : 0u;
+  const float *xl = p.X + c0 + lane * VEC;
+  const int32_t ldx32 = (int32_t)p.ldx;  // cp_admissible: ldx <= INT32_MAX
+  const float *wbase = weight == GNN_W_GCN ? p.g.nsrc : p.edge_w + beg;  // + u or + e
+  const uint32_t wlane = (lane == 0 && has_w) ? 1u : 0u;
+  const uint32_t my_off = (uint32_t)(lane * VEC * 4);
+  uint32_t slot_w = ring_s;  // issue slot address
+  int slot_i = 0;
+  auto issue = [&](int32_t u, int32_t e) {
+    const uint32_t live = e < len ? 1u : 0u;
+#pragma unroll
+    for (int n = 0; n < NV; ++n)
+      cp_async16_zfill(slot_w + my_off + (uint32_t)(n * 512), xl + (int64_t)u * ldx32 + n * 128, live ? nbytes[n] : 0u);
+    cp_async4_if(slot_w + (uint32_t)(NV * 512), wbase + (weight == GNN_W_GCN ? (int64_t)u : (int64_t)e),
+                 wlane & live);
+    cp_commit();
+    if (++slot_i == S) {
+      slot_i = 0;
+      slot_w = ring_s;
+    } else {
+      slot_w += (uint32_t)(SLOT * 4);
+    }
+  };
+  int32_t cur = lane < len ? ld_stream_i32(idx + lane) : 0;
+  int32_t nxt = 32 + lane < len ? ld_stream_i32(idx + 32 + lane) : 0;
+#pragma unroll
+  for (int q = 0; q < S; ++q) issue(__shfl_sync(0xffffffffu, cur, q), q);
+  const float *rd = ring;
+  int rd_i = 0;
+  for (int32_t e = 0; e < len; ++e) {
+    cp_wait<S - 1>();
+    __syncwarp();
+    const float w = has_w ? rd[NV * 128] : 1.0f;
+#pragma unroll
+    for (int n = 0; n < NV; ++n) {
+      const float4 x4 = *reinterpret_cast<const float4 *>(rd + n * 128 + lane * VEC);
+      const float v[4] = {x4.x, x4.y, x4.z, x4.w};
+      if constexpr (MODE == M_MAX) {
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) G.a[n][i] = fmaxf(G.a[n][i], w * v[i]);
+      } else {
+        fma_vec<VEC>(G.a[n], v, w);
+      }
+    }
+    __syncwarp();  // every lane has read the slot before it is refilled
+    if (++rd_i == S) {
+      rd_i = 0;
+      rd = ring;
+    } else {
+      rd += SLOT;
+    }
+    const int32_t pe = e + S;
+    if ((pe & 31) == 0) {
+      cur = nxt;
+      nxt = pe + 32 + lane < len ? ld_stream_i32(idx + pe + 32 + lane) : 0;
+    }
+    issue(__shfl_sync(0xffffffffu, cur, pe & 31), pe);
+  }
 }
 
 template <int MODE, int NV, int S>
@@ -732,6 +820,13 @@ __device__ __forceinline__ void group_chain_cp(const KParams &p, const int32_t *
                                                Part<MODE, 4, NV> &G) {
   constexpr int VEC = 4;
   constexpr int SLOT = cp_slot_floats<MODE, NV>();
+  if constexpr (MODE != M_GAT) {
+#ifndef GNN_CP_LEGACY
+    (void)row;
+    group_chain_cp_lean<MODE, NV, S>(p, idx, len, beg, c0, lane, ring, G);
+    return;
+#endif
+  }
   part_init(G);
   const int weight = p.weight;
   const uint32_t ring_s = (uint32_t)__cvta_generic_to_shared(ring);

@@ -30,6 +30,13 @@
 // Column blocks (TMA path, n > 256, <= 8 K blocks): each row tile is two
 // work items over column slices of the W image, so both accumulators fit
 // TMEM twice and the epilogue overlaps the next item's MMAs.
+// CTA pairs (TMA path, default; env GNN_GEMM_CTA2=0 disables): clusters of 2
+// CTAs, 256-row work items (128 rows per CTA), each CTA stages its X rows
+// and half of the item's W columns; the leader's MMA warp issues
+// tcgen05.mma.cta_group::2 (M = 256) once the peer's gate warp has arrived
+// (remotely) on its per-stage barrier, and commits with .multicast::cluster
+// to both CTAs' stage / tile barriers.  Halving the W stage halves the
+// shared-memory operand reads per SM and leaves room for a third W stage.
 // Accumulation drift: the tensor core's internal accumulation is not IEEE
 // round-to-nearest, so long K chains drift; K blocks are spread round-robin
 // over n_acc partial accumulators (summed in fp32 in the epilogue) so that no
@@ -508,10 +515,20 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
             att_s = att_t = 0.0f;
           }
           const float *as = p.att + cbb + c0, *at = p.att_dst + cbb + c0;
+          if (!(((uintptr_t)p.att | (uintptr_t)p.att_dst) & 15)) {  // 16-byte loads (warp-uniform)
 #pragma unroll
-          for (int i = 0; i < 32; ++i) {
-            att_s = fmaf(y[i], __ldg(as + i), att_s);
-            att_t = fmaf(y[i], __ldg(at + i), att_t);
+            for (int i = 0; i < 32; i += 4) {
+              const float4 a4 = __ldg(reinterpret_cast<const float4 *>(as + i));
+              const float4 t4 = __ldg(reinterpret_cast<const float4 *>(at + i));
+              att_s = fmaf(y[i + 3], a4.w, fmaf(y[i + 2], a4.z, fmaf(y[i + 1], a4.y, fmaf(y[i], a4.x, att_s))));
+              att_t = fmaf(y[i + 3], t4.w, fmaf(y[i + 2], t4.z, fmaf(y[i + 1], t4.y, fmaf(y[i], t4.x, att_t))));
+            }
+          } else {
+#pragma unroll
+            for (int i = 0; i < 32; ++i) {
+              att_s = fmaf(y[i], __ldg(as + i), att_s);
+              att_t = fmaf(y[i], __ldg(at + i), att_t);
+            }
           }
         }
         if constexpr (TMA_H) {
@@ -610,7 +627,7 @@ static bool configure(int64_t m, int32_t k, int32_t n, Config &c) {
   // pair MMA's N), so each CTA holds half of the item's W columns
   if (g_cta2 < 0) {
     const char *e = getenv("GNN_GEMM_CTA2");
-    g_cta2 = (e && e[0] == '0') ? 0 : (e && e[0] == '1') ? 1 : 0;
+    g_cta2 = (e && e[0] == '0') ? 0 : 1;
   }
   c.cta2 = 0;
   if (g_cta2) {
@@ -638,8 +655,15 @@ static bool configure(int64_t m, int32_t k, int32_t n, Config &c) {
       e = getenv("GNN_GEMM_SL");
       env_sl = e ? atoi(e) : -1;
     }
+    static int env_eb = -2;
+    if (env_eb == -2) {
+      const char *e = getenv("GNN_GEMM_EB");
+      env_eb = e ? atoi(e) : -1;
+    }
     c.sl = env_sl >= 2 && env_sl <= MAX_STAGES ? env_sl : 2;
-    c.sb = env_sb >= 2 && env_sb <= MAX_STAGES ? env_sb : 2;
+    // W ring: 3 stages when the pair halves them (measured: GEMM1/2/3 0.97 /
+    // 1.50 / 1.67 ms vs 1.05 / 1.56 / 1.71 with 2; profiles/r02_gemm_pair.txt)
+    c.sb = env_sb >= 2 && env_sb <= MAX_STAGES ? env_sb : (c.cta2 ? 3 : 2);
     c.epi8 = g_epi8 ? 1 : 0;
     c.eb = 1;
     auto need = [&](int sa, int sb, int eb, int e8) {
@@ -649,6 +673,9 @@ static bool configure(int64_t m, int32_t k, int32_t n, Config &c) {
     c.sa = 2;
     const int sa_max = env_sa > 1 && env_sa <= MAX_STAGES ? env_sa : MAX_STAGES;
     while (c.sa < sa_max && need(c.sa + 1, c.sb, c.eb, c.epi8) <= budget) ++c.sa;
+    if (env_eb == 2) {  // A/B: two staging buffers per epilogue warp before X depth
+      while (c.sa > 2 && need(c.sa, c.sb, 2, c.epi8) > budget) --c.sa;
+    }
     if (need(c.sa, c.sb, 2, c.epi8) <= budget) c.eb = 2;
     c.smem_tma = need(c.sa, c.sb, c.eb, c.epi8);
     if (c.smem_tma > budget) c.sa = 0;  // TMA path unavailable for this n

@@ -325,7 +325,7 @@ static bool cp_admissible(const gnn_plan_s *p, const AggArgs &a, int32_t fh_or_0
     const char *e = getenv("GNN_AGG_CP");
     g_agg_cp = (e && e[0] == '0') ? 0 : (e && e[0] == '1') ? 1 : 2;  // default: gather4 streaming where it applies
   }
-  if (!g_agg_cp || a.mode > M_GAT || a.F < 64) return false;
+  if (!g_agg_cp || a.mode > M_GAT || a.F < 64 || a.ldx > INT32_MAX) return false;  // (32-bit row stride)
   if (a.mode == M_GAT && (a.H > 32 || fh_or_0 % 4 != 0)) return false;
   return vec_admissible(a, fh_or_0, 4);
 }
