@@ -157,6 +157,8 @@ def run_ours(args):
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
+        os.environ.setdefault("NCCL_DEBUG", "INFO")  # the communicator lines show the rank count
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
         dist.init_process_group("nccl", device_id=dev)
     g, inp = make_inputs(args.config, args.rho, args.scale)
     n, nnz = g.n, g.nnz

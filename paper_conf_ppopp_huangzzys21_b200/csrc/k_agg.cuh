@@ -742,12 +742,20 @@ __host__ __device__ constexpr int cp_slot_floats() {
 // instruction by lane 0) and the ring slots are running counters, which cuts
 // the instructions per edge of the F <= 128 gather (C5 agg1 is issue-bound,
 // not byte-bound).  Same copies, same arithmetic order as group_chain_cp.
+#ifndef GNN_CP_U
+#define GNN_CP_U 4  // edges per cp.async commit group (C5 agg1, same box: U = 1 / 2 / 4 -> 10.1 / 9.5 / 8.5 ms)
+#endif
 template <int MODE, int NV, int S>
 __device__ __forceinline__ void group_chain_cp_lean(const KParams &p, const int32_t *idx, int32_t len, int32_t beg,
                                                     int32_t c0, int lane, float *ring, Part<MODE, 4, NV> &G) {
   constexpr int VEC = 4;
   constexpr int SLOT = cp_slot_floats<MODE, NV>();
+  // U consecutive edges share one commit group, one wait and one pair of
+  // warp barriers; the R9 chain still adds them one by one in CSR order
+  constexpr int U = (S % GNN_CP_U == 0) ? GNN_CP_U : 1;
+  constexpr int NG = S / U;  // commit groups in flight
   static_assert(MODE != M_GAT, "lean chain: sum / mean / max only");
+  static_assert(32 % U == 0 && S <= 32, "U divides the 32-entry index window, S fits it");
   part_init(G);
   const int weight = p.weight;
   const bool has_w = weight == GNN_W_GCN || weight == GNN_W_EDGE;
@@ -760,57 +768,70 @@ __device__ __forceinline__ void group_chain_cp_lean(const KParams &p, const int3
   const float *wbase = weight == GNN_W_GCN ? p.g.nsrc : p.edge_w + beg;  // + u or + e
   const uint32_t wlane = (lane == 0 && has_w) ? 1u : 0u;
   const uint32_t my_off = (uint32_t)(lane * VEC * 4);
-  uint32_t slot_w = ring_s;  // issue slot address
+  uint32_t slot_w = ring_s;  // next issue slot (address)
   int slot_i = 0;
-  auto issue = [&](int32_t u, int32_t e) {
-    const uint32_t live = e < len ? 1u : 0u;
+  int32_t cur = lane < len ? ld_stream_i32(idx + lane) : 0;
+  int32_t nxt = 32 + lane < len ? ld_stream_i32(idx + 32 + lane) : 0;
+  // issue edges e0 .. e0+U-1 (e0 % U == 0) as one commit group; indices from
+  // the 32-entry window `cur` (refilled from `nxt` at multiples of 32)
+  auto issue = [&](int32_t e0) {
+    if ((e0 & 31) == 0 && e0 >= 32) {
+      cur = nxt;
+      nxt = e0 + 32 + lane < len ? ld_stream_i32(idx + e0 + 32 + lane) : 0;
+    }
 #pragma unroll
-    for (int n = 0; n < NV; ++n)
-      cp_async16_zfill(slot_w + my_off + (uint32_t)(n * 512), xl + (int64_t)u * ldx32 + n * 128, live ? nbytes[n] : 0u);
-    cp_async4_if(slot_w + (uint32_t)(NV * 512), wbase + (weight == GNN_W_GCN ? (int64_t)u : (int64_t)e),
-                 wlane & live);
+    for (int j = 0; j < U; ++j) {
+      const int32_t e = e0 + j;
+      const int32_t u = __shfl_sync(0xffffffffu, cur, e & 31);
+      const uint32_t live = e < len ? 1u : 0u;
+      const uint32_t sw = slot_w + (uint32_t)(j * SLOT * 4);
+#pragma unroll
+      for (int n = 0; n < NV; ++n)
+        cp_async16_zfill(sw + my_off + (uint32_t)(n * 512), xl + (int64_t)u * ldx32 + n * 128, live ? nbytes[n] : 0u);
+      cp_async4_if(sw + (uint32_t)(NV * 512), wbase + (weight == GNN_W_GCN ? (int64_t)u : (int64_t)e), wlane & live);
+    }
     cp_commit();
-    if (++slot_i == S) {
+    slot_i += U;
+    if (slot_i == S) {
       slot_i = 0;
       slot_w = ring_s;
     } else {
-      slot_w += (uint32_t)(SLOT * 4);
+      slot_w += (uint32_t)(U * SLOT * 4);
     }
   };
-  int32_t cur = lane < len ? ld_stream_i32(idx + lane) : 0;
-  int32_t nxt = 32 + lane < len ? ld_stream_i32(idx + 32 + lane) : 0;
 #pragma unroll
-  for (int q = 0; q < S; ++q) issue(__shfl_sync(0xffffffffu, cur, q), q);
+  for (int q = 0; q < NG; ++q) issue(q * U);
   const float *rd = ring;
   int rd_i = 0;
-  for (int32_t e = 0; e < len; ++e) {
-    cp_wait<S - 1>();
+  for (int32_t e0 = 0; e0 < len; e0 += U) {
+    cp_wait<NG - 1>();
     __syncwarp();
-    const float w = has_w ? rd[NV * 128] : 1.0f;
 #pragma unroll
-    for (int n = 0; n < NV; ++n) {
-      const float4 x4 = *reinterpret_cast<const float4 *>(rd + n * 128 + lane * VEC);
-      const float v[4] = {x4.x, x4.y, x4.z, x4.w};
-      if constexpr (MODE == M_MAX) {
+    for (int j = 0; j < U; ++j) {
+      if (U > 1 && e0 + j >= len) break;
+      const float *sl = rd + j * SLOT;
+      const float w = has_w ? sl[NV * 128] : 1.0f;
 #pragma unroll
-        for (int i = 0; i < VEC; ++i) G.a[n][i] = fmaxf(G.a[n][i], w * v[i]);
-      } else {
-        fma_vec<VEC>(G.a[n], v, w);
+      for (int n = 0; n < NV; ++n) {
+        const float4 x4 = *reinterpret_cast<const float4 *>(sl + n * 128 + lane * VEC);
+        const float v[4] = {x4.x, x4.y, x4.z, x4.w};
+        if constexpr (MODE == M_MAX) {
+#pragma unroll
+          for (int i = 0; i < VEC; ++i) G.a[n][i] = fmaxf(G.a[n][i], w * v[i]);
+        } else {
+          fma_vec<VEC>(G.a[n], v, w);
+        }
       }
     }
-    __syncwarp();  // every lane has read the slot before it is refilled
-    if (++rd_i == S) {
+    __syncwarp();  // every lane has read the slots (incl. lane 0's weight words) before they are refilled
+    rd_i += U;
+    if (rd_i == S) {
       rd_i = 0;
       rd = ring;
     } else {
-      rd += SLOT;
+      rd += U * SLOT;
     }
-    const int32_t pe = e + S;
-    if ((pe & 31) == 0) {
-      cur = nxt;
-      nxt = pe + 32 + lane < len ? ld_stream_i32(idx + pe + 32 + lane) : 0;
-    }
-    issue(__shfl_sync(0xffffffffu, cur, pe & 31), pe);
+    issue(e0 + S);
   }
 }
 
