@@ -345,12 +345,17 @@ __device__ __forceinline__ float head_sum(float x, int lph, unsigned mask) {
 // one neighbour group: fresh fp32 chain in CSR order (R9); indices from the
 // task-ordered stream, LANES at a time, U source rows in flight per worker
 // (sum / mean / max and GAT)
+#ifndef GNN_GAT_U
+#define GNN_GAT_U 0  // 0: the GAT chain keeps the generic rows-in-flight rule
+#endif
 template <int MODE, int VEC, int NV, int LANES>
 __device__ __forceinline__ void group_chain(const KParams &p, const int32_t *idx, int32_t len, int32_t beg,
                                             int32_t row, int32_t c0, int lane, unsigned mask,
                                             Part<MODE, VEC, NV> &G, int32_t m = -1) {
   constexpr int FPL = VEC * NV;
-  constexpr int U = FPL >= 32 ? 1 : (32 / FPL > 8 ? 8 : 32 / FPL);
+  constexpr int U0 = FPL >= 32 ? 1 : (32 / FPL > 8 ? 8 : 32 / FPL);
+  // rows in flight per worker; GAT may take fewer (GNN_GAT_U) to stay in registers
+  constexpr int U = (MODE == M_GAT && GNN_GAT_U > 0 && GNN_GAT_U < U0) ? GNN_GAT_U : U0;
   part_init(G);
   const int weight = p.weight;
   const float *xl = p.X + c0 + lane * VEC;
@@ -752,7 +757,7 @@ __device__ __forceinline__ void group_chain_cp_lean(const KParams &p, const int3
   constexpr int SLOT = cp_slot_floats<MODE, NV>();
   // U consecutive edges share one commit group, one wait and one pair of
   // warp barriers; the R9 chain still adds them one by one in CSR order
-  constexpr int U = (S % GNN_CP_U == 0) ? GNN_CP_U : 1;
+  constexpr int U = (S % GNN_CP_U == 0) ? GNN_CP_U : (S % 2 == 0 ? 2 : 1);
   constexpr int NG = S / U;  // commit groups in flight
   static_assert(MODE != M_GAT, "lean chain: sum / mean / max only");
   static_assert(32 % U == 0 && S <= 32, "U divides the 32-entry index window, S fits it");
@@ -1139,8 +1144,15 @@ __global__ void __launch_bounds__(256, S > 0 ? GNN_AGG_MINB_CP
   }
   const int32_t nunits = g.n_units;
   int32_t ci = 0;
-  unsigned long long t_start = 0, busy = 0, n_done = 0;
-  if (p.trace) t_start = gtimer();
+  // load-balance trace state lives in shared memory (one slot per worker), so
+  // the untraced kernel carries no extra registers across the unit loop
+  __shared__ unsigned long long trace_sh[256 / LANES][3];  // t_unit, busy, n_done
+  unsigned long long *const tr = trace_sh[tid / LANES];
+  unsigned long long t_start = 0;
+  if (p.trace) {
+    t_start = gtimer();
+    if (lane == 0) tr[1] = tr[2] = 0ull;
+  }
   for (int32_t c0 = 0; c0 < p.F; c0 += CW, ++ci) {
     int32_t *ctr = p.ws_unit + ci;
     // the next unit (id and descriptor) is claimed while the current one streams
@@ -1154,7 +1166,7 @@ __global__ void __launch_bounds__(256, S > 0 ? GNN_AGG_MINB_CP
       dnx = __ldg(&g.unit_desc[u + 1].x);
     }
     while (u < nunits) {
-      const unsigned long long t_unit = p.trace ? gtimer() : 0ull;
+      if (p.trace && lane == 0) tr[0] = gtimer();
       int32_t un = 0;
       if (lane == 0) un = atomicAdd(ctr, 1);
       un = __shfl_sync(mask, un, 0, LANES);
@@ -1169,9 +1181,9 @@ __global__ void __launch_bounds__(256, S > 0 ? GNN_AGG_MINB_CP
                                               cp_smem + (tid >> 5) * S * cp_slot_floats<MODE, NV>());
       else
         process_unit<MODE, VEC, NV, LANES>(p, d, dnx - d.x, c0, ci, lane, mask);
-      if (p.trace) {
-        busy += gtimer() - t_unit;
-        ++n_done;
+      if (p.trace && lane == 0) {
+        tr[1] += gtimer() - tr[0];
+        tr[2] += 1ull;
       }
       u = un;
       d = dn;
@@ -1179,11 +1191,12 @@ __global__ void __launch_bounds__(256, S > 0 ? GNN_AGG_MINB_CP
     }
   }
   if (p.trace && lane == 0) {
+    const unsigned long long busy = tr[1];
     atomicAdd(p.trace + 0, busy);
     atomicAdd(p.trace + 1, 1ull);
     atomicMin(p.trace + 2, t_start);
     atomicMax(p.trace + 3, gtimer());
-    atomicAdd(p.trace + 4, n_done);
+    atomicAdd(p.trace + 4, tr[2]);
     atomicMax(p.trace + 5, busy);
   }
 }

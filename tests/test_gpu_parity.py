@@ -488,3 +488,37 @@ def test_full_size_gcn_aggregate(cfg):
     rows = sample_rows(g, 2048)
     ref = oracle.aggregate(g.rowptr, g.colidx, Hs, "sum", "gcn", relu=True, rows=rows)
     assert_close(Y[rows], ref, what=f"{cfg} aggregate")
+
+
+# --------------------------------------------------------------------------- #
+# aux: load-balance trace (gnn_set_agg_trace, Fig 8 "Balanced vs Actual")
+# --------------------------------------------------------------------------- #
+@pytest.mark.parametrize("F,kind", [(64, "sum"), (100, "sum"), (256, "sum"), (256, "gat")])
+def test_agg_trace_counters(graphs, F, kind):
+    """Tracing changes no output bit; its counters are consistent: every work
+    unit is recorded, per-worker busy time fits inside the kernel span, the
+    balanced time ([0]/[1]) is at most the actual span ([3]-[2])."""
+    g = graphs["hub"]
+    plan = G.Plan(g.rowptr, g.colidx, group_size=16)
+    if kind == "gat":
+        Hh, Fh = 8, F // 8
+        Zs = T(gs.uniform(g.n, F + 2 * Hh, seed=5))
+        run = lambda: G.gat_aggregate(plan, Zs, Zs[:, F + Hh:], Hh, Fh)  # noqa: E731
+    else:
+        X = T(gs.uniform(g.n, F, seed=6))
+        run = lambda: G.aggregate(plan, X, "sum", "gcn")  # noqa: E731
+    ref = H(run())
+    trace = torch.zeros(8, dtype=torch.int64, device="cuda")
+    G.gnn.gnn_set_agg_trace(trace.data_ptr())
+    try:
+        got = H(run())
+        torch.cuda.synchronize()
+        busy, workers, t0, t1, units, longest = trace.cpu().tolist()[:6]
+    finally:
+        G.gnn.gnn_set_agg_trace(None)
+    assert np.array_equal(got, ref)
+    assert workers > 0 and units >= plan.info["n_tiles"]
+    span = t1 - t0
+    assert span > 0 and 0 <= longest <= span
+    assert busy <= workers * span
+    assert busy / workers <= span
