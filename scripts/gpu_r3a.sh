@@ -1,0 +1,10 @@
+# re-entry check of HEAD: GPU tests, smoke, bench
+TAG=${1:-r3a}
+cd $GRAFT_REPO_ROOT; mkdir -p gpurun_out
+nvidia-smi > gpurun_out/smi_$TAG.txt 2>&1
+timeout 1500 python -m pytest tests -m gpu -q -p no:cacheprovider > gpurun_out/pytest_gpu_$TAG.log 2>&1
+echo "pytest rc=$?" >> gpurun_out/pytest_gpu_$TAG.log
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke_$TAG.log 2>&1
+echo "smoke rc=$?" >> gpurun_out/smoke_$TAG.log
+timeout 900 python bench.py --steps 10 --warmup 3 > gpurun_out/bench_$TAG.log 2>&1
+echo "bench rc=$?" >> gpurun_out/bench_$TAG.log
