@@ -10,6 +10,7 @@
 #include <stdlib.h>
 
 #include <algorithm>
+#include <type_traits>
 
 #include "gnn_internal.h"
 
@@ -743,10 +744,12 @@ __host__ __device__ constexpr int cp_slot_floats() {
 }
 
 // Lean chain for sum / mean / max (no GAT): the per-edge issue is branch-free
-// (row copies zero-fill on the lanes past F, the weight copy is one predicated
-// instruction by lane 0) and the ring slots are running counters, which cuts
-// the instructions per edge of the F <= 128 gather (C5 agg1 is issue-bound,
-// not byte-bound).  Same copies, same arithmetic order as group_chain_cp.
+// (row copies zero-fill on the lanes past F), the per-edge weights ride in
+// registers (one load per lane per 32 edges, one shuffle per edge, instead of
+// a 4-byte copy and a shared read per edge) and the ring slots are running
+// counters, which cuts the instructions per edge of the F <= 128 gather (C5
+// agg1 is issue-bound, not byte-bound).  Same rows, same arithmetic order as
+// group_chain_cp.
 #ifndef GNN_CP_U
 #define GNN_CP_U 4  // edges per cp.async commit group (C5 agg1, same box: U = 1 / 2 / 4 -> 10.1 / 9.5 / 8.5 ms)
 #endif
@@ -768,32 +771,50 @@ __device__ __forceinline__ void group_chain_cp_lean(const KParams &p, const int3
   uint32_t nbytes[NV];
 #pragma unroll
   for (int n = 0; n < NV; ++n) nbytes[n] = (c0 + (n * 32 + lane) * VEC < p.F) ? 16u : 0u;
-  const float *xl = p.X + c0 + lane * VEC;
-  const int32_t ldx32 = (int32_t)p.ldx;  // cp_admissible: ldx <= INT32_MAX
-  const float *wbase = weight == GNN_W_GCN ? p.g.nsrc : p.edge_w + beg;  // + u or + e
-  const uint32_t wlane = (lane == 0 && has_w) ? 1u : 0u;
+  // row addresses: one IMAD.WIDE.U32 per edge (u unsigned x the row pitch in
+  // bytes, cp_admissible: ldx * 4 < 2^32)
+  const char *xl = reinterpret_cast<const char *>(p.X + c0 + lane * VEC);
+  const uint32_t ldxb = (uint32_t)p.ldx * 4u;
   const uint32_t my_off = (uint32_t)(lane * VEC * 4);
   uint32_t slot_w = ring_s;  // next issue slot (address)
   int slot_i = 0;
+  // per-edge weights travel in registers, one 32-edge window per lane set:
+  // lane l of `wi` holds the weight of edge 32k + l of the window the issue
+  // side is in (GCN: nsrc[u], loaded when the window's indices become current,
+  // 32 edges after they were requested; explicit: edge_w[beg + e], coalesced);
+  // the consume side takes the window over (`wc`) when it reaches it, at most
+  // S edges later, and broadcasts edge e's weight with one shuffle
+  auto wload = [&](int32_t e_base, int32_t u_lane) -> float {
+    if (!has_w || e_base + lane >= len) return 1.0f;
+    return weight == GNN_W_GCN ? __ldg(p.g.nsrc + u_lane) : ld_stream_f32(p.edge_w + beg + e_base + lane);
+  };
   int32_t cur = lane < len ? ld_stream_i32(idx + lane) : 0;
   int32_t nxt = 32 + lane < len ? ld_stream_i32(idx + 32 + lane) : 0;
+  float wi = wload(0, cur);
+  float wc = wi;
   // issue edges e0 .. e0+U-1 (e0 % U == 0) as one commit group; indices from
-  // the 32-entry window `cur` (refilled from `nxt` at multiples of 32)
-  auto issue = [&](int32_t e0) {
+  // the 32-entry window `cur` (refilled from `nxt` at multiples of 32); a
+  // batch wholly inside the group needs no per-edge checks (FULL), the last
+  // ones zero-fill the copies of edges past the end
+  auto issue = [&](int32_t e0, auto full) {
     if ((e0 & 31) == 0 && e0 >= 32) {
       cur = nxt;
       nxt = e0 + 32 + lane < len ? ld_stream_i32(idx + e0 + 32 + lane) : 0;
+      wi = wload(e0, cur);
     }
 #pragma unroll
     for (int j = 0; j < U; ++j) {
       const int32_t e = e0 + j;
-      const int32_t u = __shfl_sync(0xffffffffu, cur, e & 31);
-      const uint32_t live = e < len ? 1u : 0u;
+      const uint32_t u = (uint32_t)__shfl_sync(0xffffffffu, cur, (e0 & 31) + j);
       const uint32_t sw = slot_w + (uint32_t)(j * SLOT * 4);
+      const char *src = xl + (uint64_t)u * ldxb;
 #pragma unroll
-      for (int n = 0; n < NV; ++n)
-        cp_async16_zfill(sw + my_off + (uint32_t)(n * 512), xl + (int64_t)u * ldx32 + n * 128, live ? nbytes[n] : 0u);
-      cp_async4_if(sw + (uint32_t)(NV * 512), wbase + (weight == GNN_W_GCN ? (int64_t)u : (int64_t)e), wlane & live);
+      for (int n = 0; n < NV; ++n) {
+        if constexpr (decltype(full)::value)
+          cp_async16_zfill(sw + my_off + (uint32_t)(n * 512), src + n * 512, nbytes[n]);
+        else
+          cp_async16_zfill(sw + my_off + (uint32_t)(n * 512), src + n * 512, e < len ? nbytes[n] : 0u);
+      }
     }
     cp_commit();
     slot_i += U;
@@ -804,31 +825,42 @@ __device__ __forceinline__ void group_chain_cp_lean(const KParams &p, const int3
       slot_w += (uint32_t)(U * SLOT * 4);
     }
   };
+  auto issue_any = [&](int32_t e0) {
+    if (e0 + U <= len) issue(e0, std::true_type{});
+    else issue(e0, std::false_type{});
+  };
 #pragma unroll
-  for (int q = 0; q < NG; ++q) issue(q * U);
+  for (int q = 0; q < NG; ++q) issue_any(q * U);
   const float *rd = ring;
   int rd_i = 0;
-  for (int32_t e0 = 0; e0 < len; e0 += U) {
-    cp_wait<NG - 1>();
-    __syncwarp();
+  auto consume = [&](int32_t e0, int j) {
+    const float *sl = rd + j * SLOT;
+    const float w = has_w ? __shfl_sync(0xffffffffu, wc, (e0 & 31) + j) : 1.0f;
 #pragma unroll
-    for (int j = 0; j < U; ++j) {
-      if (U > 1 && e0 + j >= len) break;
-      const float *sl = rd + j * SLOT;
-      const float w = has_w ? sl[NV * 128] : 1.0f;
+    for (int n = 0; n < NV; ++n) {
+      const float4 x4 = *reinterpret_cast<const float4 *>(sl + n * 128 + lane * VEC);
+      const float v[4] = {x4.x, x4.y, x4.z, x4.w};
+      if constexpr (MODE == M_MAX) {
 #pragma unroll
-      for (int n = 0; n < NV; ++n) {
-        const float4 x4 = *reinterpret_cast<const float4 *>(sl + n * 128 + lane * VEC);
-        const float v[4] = {x4.x, x4.y, x4.z, x4.w};
-        if constexpr (MODE == M_MAX) {
-#pragma unroll
-          for (int i = 0; i < VEC; ++i) G.a[n][i] = fmaxf(G.a[n][i], w * v[i]);
-        } else {
-          fma_vec<VEC>(G.a[n], v, w);
-        }
+        for (int i = 0; i < VEC; ++i) G.a[n][i] = fmaxf(G.a[n][i], w * v[i]);
+      } else {
+        fma_vec<VEC>(G.a[n], v, w);
       }
     }
-    __syncwarp();  // every lane has read the slots (incl. lane 0's weight words) before they are refilled
+  };
+  for (int32_t e0 = 0; e0 < len; e0 += U) {
+    // the issue side is at most S <= 32 edges ahead, so at a window start it
+    // is still inside this window: `wi` holds this window's weights
+    if ((e0 & 31) == 0) wc = wi;
+    cp_wait<NG - 1>();
+    __syncwarp();
+    if (e0 + U <= len) {
+#pragma unroll
+      for (int j = 0; j < U; ++j) consume(e0, j);
+    } else {
+      for (int j = 0; j < len - e0; ++j) consume(e0, j);
+    }
+    __syncwarp();  // every lane has read the slots before they are refilled
     rd_i += U;
     if (rd_i == S) {
       rd_i = 0;
@@ -836,7 +868,7 @@ __device__ __forceinline__ void group_chain_cp_lean(const KParams &p, const int3
     } else {
       rd += U * SLOT;
     }
-    issue(e0 + S);
+    issue_any(e0 + S);
   }
 }
 

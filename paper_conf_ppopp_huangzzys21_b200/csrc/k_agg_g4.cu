@@ -89,7 +89,11 @@ __device__ __forceinline__ void lds_vec(const float *p, float (&v)[VEC]) {
 // shared-memory layout in floats (runtime: box width bw, score width hs = H for GAT); every TMA
 // destination slot starts on a 128-byte boundary
 struct Layout {
-  int bw, hs, xe;  // row floats per edge, score floats per edge, extras floats per queue entry
+  // row floats per edge (GAT merged: the F features + the H scores of the row,
+  // one gather4 of 8-byte elements), score floats per edge in the separate
+  // score slots (0: none / merged), extras floats per queue entry, log2 of the
+  // row map's element size in floats (0: fp32 elements, 1: 8-byte elements)
+  int bw, hs, xe, esh;
   __host__ __device__ static int r32(int x) { return (x + 31) / 32 * 32; }
   __host__ __device__ int rslot() const { return r32(4 * bw); }  // floats per quad of rows
   __host__ __device__ int sslot() const { return r32(4 * hs); }  // floats per quad of scores
@@ -134,7 +138,7 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
   const int QE = L.qe(), RS = L.rslot(), SS = L.sslot(), BW = L.bw;
   const bool dst_scale = !ATT && scales_dst(p.weight);
   const uint32_t row_bytes = 4u * 4u * (uint32_t)BW;
-  const uint32_t sc_bytes = ATT ? 4u * 4u * (uint32_t)p.H : 0u;
+  const uint32_t sc_bytes = (ATT && L.hs) ? 4u * 4u * (uint32_t)p.H : 0u;  // separate score gather
   const uint32_t xb = ATT ? 4u * (uint32_t)p.H : 16u;
   const int32_t nunits = g.n_units;
   unsigned long long t_start = 0, busy = 0, n_done = 0, t_unit = 0;
@@ -153,6 +157,10 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
       head[n] = (ATT && valid[n]) ? f / p.Fh : 0;
     }
     const int hsh = ATT ? (lane & (p.H - 1)) : 0;
+    // GAT scores of edge r of a quad: in the gathered row after the features
+    // (merged map) or in the separate score slot
+    const bool merged = ATT && L.hs == 0;
+    const int sstr = merged ? BW : p.H;
     const float smxs = ATT ? fkey_decode(__ldg(p.smax + hsh)) : 0.0f;
     // ---- run-claim pipeline: C (atomic issued) -> B (descriptors loading) -> A (ready, first indices loading) -> P
     int32_t uC = 0;
@@ -257,8 +265,8 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic reads of the slot -> async writes
         mbar_expect(bar, bytes);
         if (nvalid > 0) {
-          gather4(rows + (size_t)pslot * RS, &rmap, c0, r4[0], r4[1], r4[2], r4[3], bar);
-          if (ATT) gather4(scs + (size_t)pslot * SS, &smap, 0, r4[0], r4[1], r4[2], r4[3], bar);
+          gather4(rows + (size_t)pslot * RS, &rmap, c0 >> L.esh, r4[0], r4[1], r4[2], r4[3], bar);
+          if (ATT && !merged) gather4(scs + (size_t)pslot * SS, &smap, 0, r4[0], r4[1], r4[2], r4[3], bar);
         }
         for (int j = 0; j < nx; ++j) {
           const int32_t xr = j == 0 ? xrow0 : j == 1 ? xrow1 : j == 2 ? xrow2 : xrow3;
@@ -286,7 +294,7 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
       if (posC == 0 && qh == qt) break;  // every queued unit done and the producer is exhausted
       mbar_wait(&bars[w][cslot], cpar);
       const float *rq = rows + (size_t)cslot * RS;
-      const float *sq = scs + (size_t)cslot * SS;
+      const float *sq = merged ? rq + (p.F - c0) : scs + (size_t)cslot * SS;
       int r = 0;
       while (r < 4) {
         if (posC == 0) {  // first edge of the next queued unit: its entry and extras have landed
@@ -317,11 +325,56 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
         }
         const int kk = min(4 - r, lenC - posC);  // edges of this unit in the rest of the quad
         const bool one = lenC == 1;
+        if (kk == 4) {
+          // a whole quad of one unit (the common case): the four edges' terms
+          // are independent, so they are issued back to back; the chain still
+          // adds them in CSR order (bit-identical to the per-edge loop below)
+          if constexpr (ATT) {
+            float ex4[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              const float sco = leaky_f(sq[j * sstr + hsh] + tvs, p.slope);
+              seens = fmaxf(seens, sco);
+              ex4[j] = ex2_f(fmaf(sco, kLog2e, nmbs));
+            }
+#pragma unroll
+            for (int j = 0; j < 4; ++j) ls += ex4[j];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+#pragma unroll
+              for (int n = 0; n < NV; ++n) {
+                const float exn = __shfl_sync(0xffffffffu, ex4[j], head[n]);
+                if (!valid[n]) continue;
+                float v[VEC];
+                lds_vec<VEC>(rq + j * BW + (n * 32 + lane) * VEC, v);
+                fma_vec<VEC>(G.a[n], v, exn);
+              }
+            }
+          } else {
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              const float wt = 1.0f;  // weight 1 (pre-scaled GCN: ndst in the epilogue)
+#pragma unroll
+              for (int n = 0; n < NV; ++n) {
+                if (!valid[n]) continue;
+                float v[VEC];
+                lds_vec<VEC>(rq + j * BW + (n * 32 + lane) * VEC, v);
+                if constexpr (MODE == M_MAX) {
+#pragma unroll
+                  for (int i = 0; i < VEC; ++i) G.a[n][i] = fmaxf(G.a[n][i], wt * v[i]);
+                } else {
+                  fma_vec<VEC>(G.a[n], v, wt);
+                }
+              }
+            }
+          }
+          r = 4;
+        } else
         for (int j = 0; j < kk; ++j, ++r) {
           const float *rb = rq + r * BW;
           if constexpr (ATT) {
             // e_uv and exp(e_uv - m) once per head (lane hsh), then to the lanes holding that head
-            const float sco = leaky_f(sq[r * p.H + hsh] + tvs, p.slope);
+            const float sco = leaky_f(sq[r * sstr + hsh] + tvs, p.slope);
             seens = fmaxf(seens, sco);
             const float ex = one ? 1.0f : ex2_f(fmaf(sco, kLog2e, nmbs));
             ls += ex;
@@ -334,8 +387,8 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
               fma_vec<VEC>(G.a[n], v, exn);
             }
           } else {
-#pragma unroll
             const float wt = 1.0f;  // weight 1 (pre-scaled GCN: ndst in the epilogue)
+#pragma unroll
             for (int n = 0; n < NV; ++n) {
               if (!valid[n]) continue;
               float v[VEC];
@@ -416,21 +469,50 @@ EncodeTiledFn encode_fn() {
   }
   return fn;
 }
-// rows of `width` fp32 features, row stride ld (elements), boxes of box_w x 1 (gather4 takes 4 box rows)
-bool encode_rows(CUtensorMap *m, const float *base, int64_t nrows, int32_t width, int64_t ld, int32_t box_w) {
+// L2 promotion of the gathered rows' misses: a miss is fetched as the whole
+// aligned 256-byte block when every row starts on one (C5 agg2: 1 KB rows);
+// otherwise the largest block size the row starts stay aligned to, so at most
+// the tail block of a row reaches outside it (GAT [z | s] rows of 1056 B at a
+// 1088-byte stride: 256-byte promotion fetched 1280 B per row, 64-byte 1088).  env GNN_G4_PROMO = 0 / 64 / 128 / 256 forces one (A/B).
+CUtensorMapL2promotion promotion(const float *base, int64_t ld) {
+  static int forced = -2;
+  if (forced == -2) {
+    const char *e = getenv("GNN_G4_PROMO");
+    forced = e ? atoi(e) : -1;
+  }
+  int blk = 256;
+  if (forced >= 0) {
+    blk = forced;
+  } else {
+    const uint64_t a = (uint64_t)(uintptr_t)base | (uint64_t)(ld * 4);
+    while (blk > 32 && (a & (uint64_t)(blk - 1))) blk >>= 1;
+  }
+  return blk >= 256 ? CU_TENSOR_MAP_L2_PROMOTION_L2_256B
+         : blk >= 128 ? CU_TENSOR_MAP_L2_PROMOTION_L2_128B
+         : blk >= 64  ? CU_TENSOR_MAP_L2_PROMOTION_L2_64B
+                      : CU_TENSOR_MAP_L2_PROMOTION_NONE;
+}
+// rows of `width` fp32 features, row stride ld (floats), boxes of box_w x 1
+// (gather4 takes 4 box rows); esh = 1: the same bytes as 8-byte elements
+// (width and box_w still in floats, even), so a box may span 512 floats
+bool encode_rows(CUtensorMap *m, const float *base, int64_t nrows, int32_t width, int64_t ld, int32_t box_w,
+                 int esh = 0) {
   if (!encode_fn() || ((uintptr_t)base & 15) || ((ld * 4) & 15) || nrows < 1 || nrows > 0x7fffffffLL) return false;
-  const cuuint64_t dims[2] = {(cuuint64_t)width, (cuuint64_t)nrows};
+  if (esh && ((width | box_w) & 1)) return false;
+  if ((box_w >> esh) > 256 || ((box_w * 4) & 15)) return false;
+  const cuuint64_t dims[2] = {(cuuint64_t)(width >> esh), (cuuint64_t)nrows};
   const cuuint64_t strides[1] = {(cuuint64_t)ld * 4};
-  const cuuint32_t box[2] = {(cuuint32_t)box_w, 1};
+  const cuuint32_t box[2] = {(cuuint32_t)(box_w >> esh), 1};
   const cuuint32_t es[2] = {1, 1};
-  return encode_fn()(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void *)base, dims, strides, box, es,
-                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+  return encode_fn()(m, esh ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void *)base,
+                     dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                     promotion(base, ld),
                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 }  // namespace
 
 // Does the gather4 kernel take this call?  Sum / mean / max with weight 1 or
-// the pre-scaled GCN form (no per-edge weight), or GAT with H % 4 == 0 <= 32;
+// the pre-scaled GCN form, or GAT with H a power of two in 4..32;
 // 16-byte aligned rows, F % 4 == 0 (DESIGN.md §5.2 rule).
 bool g4_admissible(const KParams &kp, int32_t n_src) {
   if (!encode_fn() || n_src < 1) return false;
@@ -442,9 +524,9 @@ bool g4_admissible(const KParams &kp, int32_t n_src) {
     return true;
   }
   if (kp.mode > M_MAX) return false;
-  // weight 1 or the pre-scaled GCN form (ndst per row); per-edge weights take the
-  // cp.async chain (their 4-byte copies would need cp.async.mbarrier.arrive
-  // tracking, which compute-sanitizer synccheck flags, and measured slower)
+  // weight 1 or the pre-scaled GCN form (ndst per row); per-edge weights take
+  // the cp.async chain (GCN nsrc[u] by 4-byte cp.async per edge tracked with
+  // commit groups measured slower there: C3 13.6 vs 11.9 ms; agg1 12.9 vs 7.9)
   return kp.weight == GNN_W_ONE || kp.weight == W_DST_ONLY;
 }
 
@@ -455,13 +537,31 @@ static cudaError_t launch_g4_mode(const KParams &kp_in, int32_t n_src, cudaStrea
   L.bw = kp_in.F < BWMAX ? kp_in.F : BWMAX;
   L.hs = MODE == M_GAT ? kp_in.H : 0;  // GAT score columns
   L.xe = MODE == M_GAT ? (kp_in.H < 4 ? 4 : kp_in.H) : 4;
-  const size_t smem = L.bytes();
+  L.esh = 0;
+  // GAT with one sweep (F <= 256): the H score columns that follow the
+  // features ride in the same gather4 as the row (F + H floats as 8-byte
+  // elements), one TMA request per quad instead of two (env GNN_G4_MERGED=0: two)
+  static int merged_ok = -1;
+  if (merged_ok < 0) {
+    const char *e = getenv("GNN_G4_MERGED");
+    merged_ok = (e && e[0] == '0') ? 0 : 1;
+  }
+  const bool merged = MODE == M_GAT && merged_ok && kp_in.F <= BWMAX && (kp_in.F + kp_in.H) % 4 == 0 &&
+                      kp_in.F + kp_in.H <= 512 && kp_in.F + kp_in.H <= kp_in.ldx;
   CUtensorMap rmap, smap;
   memset(&rmap, 0, sizeof(rmap));
   memset(&smap, 0, sizeof(smap));
-  if (!encode_rows(&rmap, kp_in.X, n_src, kp_in.F, kp_in.ldx, L.bw)) return cudaErrorNotSupported;
-  if (MODE == M_GAT && !encode_rows(&smap, kp_in.X + kp_in.F, n_src, kp_in.H, kp_in.ldx, kp_in.H))
-    return cudaErrorNotSupported;
+  if (merged) {
+    L.bw = kp_in.F + kp_in.H;
+    L.hs = 0;
+    L.esh = 1;
+    if (!encode_rows(&rmap, kp_in.X, n_src, L.bw, kp_in.ldx, L.bw, 1)) return cudaErrorNotSupported;
+  } else {
+    if (!encode_rows(&rmap, kp_in.X, n_src, kp_in.F, kp_in.ldx, L.bw)) return cudaErrorNotSupported;
+    if (MODE == M_GAT && !encode_rows(&smap, kp_in.X + kp_in.F, n_src, kp_in.H, kp_in.ldx, kp_in.H))
+      return cudaErrorNotSupported;
+  }
+  const size_t smem = L.bytes();
   static int occ = 0;
   auto fn = k_stream_g4<MODE, VEC, NV>;
   if (occ == 0) {

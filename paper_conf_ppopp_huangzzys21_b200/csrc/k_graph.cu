@@ -325,7 +325,7 @@ static bool cp_admissible(const gnn_plan_s *p, const AggArgs &a, int32_t fh_or_0
     const char *e = getenv("GNN_AGG_CP");
     g_agg_cp = (e && e[0] == '0') ? 0 : (e && e[0] == '1') ? 1 : 2;  // default: gather4 streaming where it applies
   }
-  if (!g_agg_cp || a.mode > M_GAT || a.F < 64 || a.ldx > INT32_MAX) return false;  // (32-bit row stride)
+  if (!g_agg_cp || a.mode > M_GAT || a.F < 64 || a.ldx >= (1LL << 30)) return false;  // (32-bit row pitch in bytes)
   if (a.mode == M_GAT && (a.H > 32 || fh_or_0 % 4 != 0)) return false;
   return vec_admissible(a, fh_or_0, 4);
 }
@@ -346,14 +346,21 @@ static Mapping choose_mapping(const gnn_plan_s *p, const AggArgs &a, int32_t fh_
     // 15.0 vs 16.8 ms for the register kernel); 64..128: the cp.async chain
     // (C5 agg1 F = 100 with per-edge GCN weights: 11.0 vs 11.9 register, 13.8
     // gather4)
-    c.cp = a.F > 128 ? g_agg_cp : std::min(g_agg_cp, 1);
+    static int g4_narrow = -1;  // A/B: env GNN_G4_NARROW=1 sends 64..128-feature rows to gather4 too
+    if (g4_narrow < 0) {
+      const char *e = getenv("GNN_G4_NARROW");
+      g4_narrow = (e && e[0] == '1') ? 1 : 0;
+    }
+    c.cp = (a.F > 128 || g4_narrow) ? g_agg_cp : std::min(g_agg_cp, 1);
     if (a.mode == M_GAT) {
-      // GAT: the register kernel measured faster than both staged kernels on C5
-      // (19.8 vs 20.4 ms gather4, 20.0 ms cp.async chain); env GNN_G4_GAT=1 opts in
+      // GAT, rows > 128 features: gather4 with the H score columns in the same
+      // request as the row and 64-byte L2 promotion for the 1056-byte [z | s]
+      // rows (C5 8x32, same box: 18.7-19.0 vs 19.6-19.7 ms for the register
+      // kernel; profiles/r02_r3d_*); env GNN_G4_GAT=0 takes the register kernel
       static int g4_gat = -1;
       if (g4_gat < 0) {
         const char *e = getenv("GNN_G4_GAT");
-        g4_gat = (e && e[0] == '1') ? 1 : 0;
+        g4_gat = (e && e[0] == '0') ? 0 : 1;
       }
       c.cp = (g4_gat && a.F > 128 && c.cp == 2) ? 2 : 0;
     }
