@@ -261,6 +261,14 @@ gnn_status gnn_gat_transform(const float *X, int64_t ldx, int64_t m, int32_t f_i
                              gnn_stream_t stream);
 size_t gnn_gat_transform_workspace_size(int64_t m, int32_t f_in, int32_t H, int32_t Fh);
 
+/* gnn_gat_transform whose epilogue also writes [z | s | t] to n_mirrors peer
+ * replicas (NEXT-2; mirror contract as gnn_gemm_mirrored, laid out like Zst). */
+gnn_status gnn_gat_transform_mirrored(const float *X, int64_t ldx, int64_t m, int32_t f_in,
+                                      const float *W, int64_t ldw, const float *a_src,
+                                      const float *a_dst, int32_t H, int32_t Fh, float *Zst,
+                                      int64_t ldz, float *const *mirrors, int32_t n_mirrors,
+                                      void *ws, size_t ws_bytes, gnn_stream_t stream);
+
 /*
  * Full GAT layer: [Z | s | t] by gnn_gat_transform, then gnn_gat_aggregate.
  * W: [f_in, H*Fh] row-major.  Requires n_src == n.  Workspace from
@@ -308,6 +316,37 @@ gnn_status gnn_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw, fl
                     const float *col_bias, int32_t relu, void *ws, size_t ws_bytes,
                     gnn_stream_t stream);
 size_t gnn_gemm_workspace_size(int64_t m, int32_t k, int32_t n);
+
+/*
+ * NEXT-2 (SURVEY §8(e) lever iii, §8(f)): the all-gather of a row-partitioned
+ * layer fused into the producer.  gnn_gemm whose epilogue also writes every
+ * output tile to n_mirrors (<= 7) extra destinations -- the same rows of the
+ * peer GPUs' replica buffers, opened with gnn_ipc_open -- with the same TMA
+ * bulk-tensor stores that write H, so the rows leave over NVLink as soon as
+ * each tile is done instead of in a separate collective.  mirrors[q]: device
+ * pointer (local or peer), 16-byte aligned, laid out like H (ldh, m rows, n
+ * columns), not overlapping X or H.  Needs the tcgen05 path (ws from
+ * gnn_gemm_workspace_size) with 16-byte aligned X/H rows, else
+ * GNN_ERR_UNSUPPORTED (never a silent non-mirrored run).  The kernel's stores
+ * are complete (and fenced at system scope) when it ends; consumers on other
+ * GPUs must order after it (e.g. a stream-ordered NCCL all_reduce of a flag).
+ */
+gnn_status gnn_gemm_mirrored(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H,
+                             int64_t ldh, int64_t m, int32_t k, int32_t n, const float *row_scale,
+                             const float *col_bias, int32_t relu, float *const *mirrors,
+                             int32_t n_mirrors, void *ws, size_t ws_bytes, gnn_stream_t stream);
+
+/*
+ * Device memory shareable across processes (CUDA IPC) for the mirrors:
+ * gnn_ipc_alloc returns a fresh cudaMalloc allocation and its 64-byte IPC
+ * handle (written to `handle`); another process on this or a peer GPU maps
+ * it with gnn_ipc_open (peer access enabled lazily) and unmaps it with
+ * gnn_ipc_close; the owner releases it with gnn_ipc_free.
+ */
+gnn_status gnn_ipc_alloc(size_t bytes, void **ptr, void *handle);
+gnn_status gnn_ipc_free(void *ptr);
+gnn_status gnn_ipc_open(const void *handle, void **ptr);
+gnn_status gnn_ipc_close(void *ptr);
 
 /* GEMM implementation selector (process-wide): 0 = auto, 1 = SIMT FFMA,
  * 2 = tcgen05 3xTF32, 3 = tcgen05 3xTF32 with register-fed X tiles instead

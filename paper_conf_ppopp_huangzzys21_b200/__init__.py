@@ -10,7 +10,7 @@ Python binding.  Touching any public name loads the library and fails loudly
 if it is not built — there is no CPU fallback.  (The submodule ``build`` can
 be imported without loading the library, so it can rebuild it.)
 """
-_PUBLIC = ("Plan", "aggregate", "aggregate_accumulate", "scale_rows", "gat_aggregate", "gat_layer", "gat_transform", "edgeconv", "edgeconv_aggregate", "gemm",
+_PUBLIC = ("Plan", "aggregate", "aggregate_accumulate", "scale_rows", "gat_aggregate", "gat_layer", "gat_transform", "edgeconv", "edgeconv_aggregate", "gemm", "gemm_mirrored", "IpcBuffer", "ipc_open", "ipc_close",
            "gcn_layer", "partition_rows", "local_csr", "local_csr_block", "launch_count", "set_gemm_impl", "set_agg_mapping", "set_group_size", "tune_aggregate", "attn_aggregate", "sample_neighbors", "sage_lstm_aggregate", "sage_lstm_layer", "las_host", "groups_host",
            "GnnError")
 __all__ = ["gnn", *_PUBLIC]

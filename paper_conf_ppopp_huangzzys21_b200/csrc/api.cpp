@@ -12,6 +12,10 @@
 #include "gnn_internal.h"
 
 namespace gnn {
+static gnn_status pack_mirrors(float *const *mirrors, int32_t n_mirrors, GemmMirrors &m);
+}
+
+namespace gnn {
 
 static thread_local std::string t_last_error;
 static std::atomic<uint64_t> g_launches{0};
@@ -508,7 +512,68 @@ gnn_status gnn_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw, fl
   })
 }
 
+gnn_status gnn_gemm_mirrored(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H, int64_t ldh,
+                             int64_t m, int32_t k, int32_t n, const float *row_scale, const float *col_bias,
+                             int32_t relu, float *const *mirrors, int32_t n_mirrors, void *ws, size_t ws_bytes,
+                             gnn_stream_t stream) {
+  GNN_TRY({
+    if (m < 0 || k < 1 || n < 0) return check(false, "GEMM sizes: m, n >= 0, k >= 1");
+    if (m == 0 || n == 0) return GNN_OK;
+    if (!H || !X || !W) return check(false, "X/W/H is NULL");
+    if (ldx < k || ldw < n || ldh < n) return check(false, "GEMM leading dimension too small");
+    if (overlaps(H, span_bytes(m, ldh, n), X, span_bytes(m, ldx, k)) ||
+        overlaps(H, span_bytes(m, ldh, n), W, span_bytes(k, ldw, n)))
+      return check(false, "H overlaps X or W");
+    GemmMirrors mir;
+    gnn_status st = pack_mirrors(mirrors, n_mirrors, mir);
+    if (st != GNN_OK) return st;
+    for (int32_t q = 0; q < n_mirrors; ++q)
+      if (overlaps(mirrors[q], span_bytes(m, ldh, n), X, span_bytes(m, ldx, k)) ||
+          overlaps(mirrors[q], span_bytes(m, ldh, n), H, span_bytes(m, ldh, n)))
+        return check(false, "a mirror overlaps X or H");
+    if (!ws) return check(false, "the mirrored GEMM needs the tcgen05 workspace");
+    return launch_gemm(X, ldx, W, ldw, H, ldh, m, k, n, row_scale, col_bias, relu, ws, ws_bytes,
+                       (cudaStream_t)stream, &mir);
+  })
+}
+
 int gnn_set_gemm_impl(int impl) { return set_gemm_impl(impl); }
+
+// CUDA IPC for the mirrors of a multi-process exchange (NEXT-2)
+gnn_status gnn_ipc_alloc(size_t bytes, void **ptr, void *handle) {
+  GNN_TRY({
+    if (!ptr || !handle || bytes == 0) return check(false, "gnn_ipc_alloc: NULL argument or zero size");
+    *ptr = nullptr;
+    cudaError_t e = cudaMalloc(ptr, bytes);
+    if (e != cudaSuccess) return cuda_status(e, "gnn_ipc_alloc cudaMalloc");
+    cudaIpcMemHandle_t h;
+    e = cudaIpcGetMemHandle(&h, *ptr);
+    if (e != cudaSuccess) {
+      cudaFree(*ptr);
+      *ptr = nullptr;
+      return cuda_status(e, "gnn_ipc_alloc cudaIpcGetMemHandle");
+    }
+    memcpy(handle, &h, sizeof(h));
+    return GNN_OK;
+  })
+}
+
+gnn_status gnn_ipc_free(void *ptr) {
+  GNN_TRY({ return ptr ? cuda_status(cudaFree(ptr), "gnn_ipc_free") : GNN_OK; })
+}
+
+gnn_status gnn_ipc_open(const void *handle, void **ptr) {
+  GNN_TRY({
+    if (!ptr || !handle) return check(false, "gnn_ipc_open: NULL argument");
+    cudaIpcMemHandle_t h;
+    memcpy(&h, handle, sizeof(h));
+    return cuda_status(cudaIpcOpenMemHandle(ptr, h, cudaIpcMemLazyEnablePeerAccess), "gnn_ipc_open");
+  })
+}
+
+gnn_status gnn_ipc_close(void *ptr) {
+  GNN_TRY({ return ptr ? cuda_status(cudaIpcCloseMemHandle(ptr), "gnn_ipc_close") : GNN_OK; })
+}
 
 void gnn_set_agg_trace(void *trace_dev) { set_agg_trace(trace_dev); }
 
@@ -532,14 +597,15 @@ namespace gnn {
 // folded weights [W | W_h a_src_h | W_h a_dst_h] (a reassociation of Z a).
 static gnn_status gat_transform(const float *X, int64_t ldx, int64_t m, int32_t f_in, const float *W, int64_t ldw,
                                 const float *a_src, const float *a_dst, int32_t H, int32_t Fh, float *Zst,
-                                int64_t ldz, void *ws, size_t ws_bytes, cudaStream_t s) {
+                                int64_t ldz, void *ws, size_t ws_bytes, cudaStream_t s,
+                                const GemmMirrors *mir = nullptr) {
   if (m == 0) return GNN_OK;
   if (ws_bytes < ws_gat_transform(m, f_in, H, Fh)) {
     set_error("gat transform workspace too small: need " + std::to_string(ws_gat_transform(m, f_in, H, Fh)));
     return GNN_ERR_WORKSPACE;
   }
   const int32_t HF = H * Fh;
-  cudaError_t e = launch_gemm_att(X, ldx, W, ldw, Zst, ldz, m, f_in, H, Fh, a_src, a_dst, ws, ws_bytes, s);
+  cudaError_t e = launch_gemm_att(X, ldx, W, ldw, Zst, ldz, m, f_in, H, Fh, a_src, a_dst, ws, ws_bytes, s, mir);
   if (e == cudaSuccess) return GNN_OK;
   if (e != cudaErrorNotSupported) return cuda_status(e, "gat transform");
   (void)cudaGetLastError();
@@ -557,7 +623,25 @@ static gnn_status gat_transform(const float *X, int64_t ldx, int64_t m, int32_t 
     set_error("gat transform: ldz must be >= round_up(H*Fh + 2H, 8) for this head size");
     return GNN_ERR_INVALID_ARG;
   }
-  return launch_gemm(X, ldx, Wext, ld, Zst, ldz, m, f_in, ld, nullptr, nullptr, 0, ws, gws, s);
+  return launch_gemm(X, ldx, Wext, ld, Zst, ldz, m, f_in, ld, nullptr, nullptr, 0, ws, gws, s, mir);
+}
+
+// validate and pack the mirror pointers of the *_mirrored entry points
+static gnn_status pack_mirrors(float *const *mirrors, int32_t n_mirrors, GemmMirrors &m) {
+  memset(&m, 0, sizeof(m));
+  if (n_mirrors < 0 || n_mirrors > kMaxMirrors || (n_mirrors > 0 && !mirrors)) {
+    set_error("n_mirrors must be in [0, 7] with a mirror pointer array");
+    return GNN_ERR_INVALID_ARG;
+  }
+  for (int32_t q = 0; q < n_mirrors; ++q) {
+    if (!mirrors[q] || ((uintptr_t)mirrors[q] & 15)) {
+      set_error("mirror pointers must be non-NULL and 16-byte aligned");
+      return GNN_ERR_INVALID_ARG;
+    }
+    m.dst[q] = mirrors[q];
+  }
+  m.count = n_mirrors;
+  return GNN_OK;
 }
 }  // namespace gnn
 
@@ -580,6 +664,25 @@ gnn_status gnn_gat_transform(const float *X, int64_t ldx, int64_t m, int32_t f_i
       return check(false, "Zst overlaps X");
     return gat_transform(X, ldx, m, f_in, W, ldw, a_src, a_dst, H, Fh, Zst, ldz, ws, ws_bytes,
                          (cudaStream_t)stream);
+  })
+}
+
+gnn_status gnn_gat_transform_mirrored(const float *X, int64_t ldx, int64_t m, int32_t f_in, const float *W,
+                                      int64_t ldw, const float *a_src, const float *a_dst, int32_t H, int32_t Fh,
+                                      float *Zst, int64_t ldz, float *const *mirrors, int32_t n_mirrors, void *ws,
+                                      size_t ws_bytes, gnn_stream_t stream) {
+  GNN_TRY({
+    if (m < 0 || f_in < 1 || H < 1 || H > 256 || Fh < 1) return check(false, "bad GAT transform sizes");
+    if (m > 0 && (!X || !W || !a_src || !a_dst || !Zst || !ws)) return check(false, "NULL argument");
+    if (ldx < f_in || ldw < (int64_t)H * Fh || ldz < (int64_t)H * Fh + 2 * H)
+      return check(false, "leading dimension too small (ldz >= H*Fh + 2H)");
+    if (overlaps(Zst, span_bytes(m, ldz, (int64_t)H * Fh + 2 * H), X, span_bytes(m, ldx, f_in)))
+      return check(false, "Zst overlaps X");
+    GemmMirrors mir;
+    gnn_status st = pack_mirrors(mirrors, n_mirrors, mir);
+    if (st != GNN_OK) return st;
+    return gat_transform(X, ldx, m, f_in, W, ldw, a_src, a_dst, H, Fh, Zst, ldz, ws, ws_bytes,
+                         (cudaStream_t)stream, &mir);
   })
 }
 

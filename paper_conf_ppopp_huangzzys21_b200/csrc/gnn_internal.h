@@ -154,13 +154,23 @@ gnn_status launch_aggregate(const gnn_plan_s *p, const AggArgs &a, void *ws, siz
                             cudaStream_t s);
 
 // GEMM (k_gemm.cu)
+// Mirrors (NEXT-2): extra destinations with the output's layout (ldh, rows,
+// columns) -- the same rows of peer GPUs' replica buffers -- that the tcgen05
+// epilogue writes with the same TMA stores as H (all-gather fused into the
+// producer).  Only the TMA-store epilogue takes them.
+constexpr int kMaxMirrors = 7;
+struct GemmMirrors {
+  float *dst[kMaxMirrors];
+  int32_t count;
+};
 gnn_status launch_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H,
                        int64_t ldh, int64_t m, int32_t k, int32_t n, const float *row_scale,
-                       const float *col_bias, int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s);
+                       const float *col_bias, int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s,
+                       const GemmMirrors *mir = nullptr);
 size_t gemm_tc_workspace(int64_t m, int32_t k, int32_t n);
 cudaError_t launch_gemm_att(const float *X, int64_t ldx, const float *W, int64_t ldw, float *Z, int64_t ldz, int64_t m,
                             int32_t k, int32_t H, int32_t Fh, const float *a_src, const float *a_dst, void *ws,
-                            size_t ws_bytes, cudaStream_t s);
+                            size_t ws_bytes, cudaStream_t s, const GemmMirrors *mir = nullptr);
 int set_gemm_impl(int impl);
 
 // small helper kernels (k_graph.cu)

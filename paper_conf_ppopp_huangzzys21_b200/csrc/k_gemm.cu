@@ -127,16 +127,22 @@ int set_gemm_impl(int impl) {
 // is outside what the tcgen05 kernel takes
 cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H,
                            int64_t ldh, int64_t m, int32_t k, int32_t n, const float *row_scale,
-                           const float *col_bias, int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s);
+                           const float *col_bias, int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s,
+                           const GemmMirrors *mir);
 
 gnn_status launch_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H,
                        int64_t ldh, int64_t m, int32_t k, int32_t n, const float *row_scale,
-                       const float *col_bias, int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s) {
+                       const float *col_bias, int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s,
+                       const GemmMirrors *mir) {
   if (m == 0 || n == 0) return GNN_OK;
+  if (mir && mir->count > 0 && (g_gemm_impl == 1 || !ws || k < 1)) {
+    set_error("mirrored GEMM: only the tcgen05 TMA-store epilogue writes mirrors (pass a workspace)");
+    return GNN_ERR_UNSUPPORTED;
+  }
   if (g_gemm_impl != 1 && ws != nullptr && k > 0) {
     // a caller that passes a workspace gets the tensor cores or an error,
     // never a silent fallback (every n is taken, wide ones as column slices)
-    cudaError_t e = launch_gemm_tc(X, ldx, W, ldw, H, ldh, m, k, n, row_scale, col_bias, relu, ws, ws_bytes, s);
+    cudaError_t e = launch_gemm_tc(X, ldx, W, ldw, H, ldh, m, k, n, row_scale, col_bias, relu, ws, ws_bytes, s, mir);
     if (e == cudaSuccess) return GNN_OK;
     if (e == cudaErrorInvalidValue) {
       set_error("gemm workspace too small: need gnn_gemm_workspace_size(m, k, n) = " +
@@ -144,6 +150,10 @@ gnn_status launch_gemm(const float *X, int64_t ldx, const float *W, int64_t ldw,
       return GNN_ERR_WORKSPACE;
     }
     if (e != cudaErrorNotSupported) return cuda_status(e, "gemm tcgen05 launch");
+    if (mir && mir->count > 0) {
+      set_error("mirrored GEMM: needs the TMA-store epilogue (16-byte aligned X, H, mirrors and leading dimensions)");
+      return GNN_ERR_UNSUPPORTED;
+    }
     set_error("tcgen05 GEMM: workspace must be 16-byte aligned");
     return GNN_ERR_INVALID_ARG;
   } else if (g_gemm_impl >= 2 && k > 0) {

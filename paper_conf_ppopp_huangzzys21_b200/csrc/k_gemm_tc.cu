@@ -87,6 +87,14 @@ __global__ void k_gemm_wimage(const float *__restrict__ W, int64_t ldw, int32_t 
   }
 }
 
+// mirror destinations (NEXT-2) as kernel parameters: one TMA map per mirror
+// (same box as hmap) and its base pointer for the scalar score stores
+struct MirrorMaps {
+  CUtensorMap map[kMaxMirrors];
+  float *base[kMaxMirrors];
+  int32_t count;
+};
+
 struct TcParams {
   const float *X;
   int64_t ldx;
@@ -116,7 +124,8 @@ struct TcParams {
 
 template <bool VEC_X, bool VEC_H, bool TMA_X, bool CTA2 = false>
 __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams p, const __grid_constant__ CUtensorMap xmap,
-                                                          const __grid_constant__ CUtensorMap hmap) {
+                                                          const __grid_constant__ CUtensorMap hmap,
+                                                          const __grid_constant__ MirrorMaps mir) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   const int NP = p.np;
@@ -464,6 +473,10 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
         if (att_h >= 0 && gm < p.m) {
           p.H[gm * p.ldh + p.att_col + att_h] = att_s;
           p.H[gm * p.ldh + p.att_col + p.att_H + att_h] = att_t;
+          for (int q = 0; q < mir.count; ++q) {  // the same scores into the mirrors (NEXT-2)
+            mir.base[q][gm * p.ldh + p.att_col + att_h] = att_s;
+            mir.base[q][gm * p.ldh + p.att_col + p.att_H + att_h] = att_t;
+          }
         }
       };
 #ifdef GNN_GEMM_DBG_NOEPI
@@ -546,7 +559,12 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
                 make_float4(y[4 * c], y[4 * c + 1], y[4 * c + 2], y[4 * c + 3]);
           asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
           __syncwarp();
-          if (lane == 0) tma_store_2d(&hmap, cbb + c0, (int32_t)(row0 + quad * 32), buf);
+          if (lane == 0) {
+            // the chunk to H and to every mirror (peer replicas, NEXT-2), one bulk group
+            tma_store_2d_nc(&hmap, cbb + c0, (int32_t)(row0 + quad * 32), buf);
+            for (int q = 0; q < mir.count; ++q) tma_store_2d_nc(&mir.map[q], cbb + c0, (int32_t)(row0 + quad * 32), buf);
+            asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+          }
           ++chunk;
           continue;
         }
@@ -570,6 +588,7 @@ __global__ void __launch_bounds__(threads_of(TMA_X), 1) k_gemm_tc(const TcParams
       }
     }
     if (TMA_H && lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    if (mir.count > 0) __threadfence_system();  // peer stores performed before the kernel ends
   }
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
@@ -780,21 +799,22 @@ struct AttEpi {
 static cudaError_t launch_gemm_tc_one(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H, int64_t ldh,
                                       int64_t m, int32_t k, int32_t n, const float *row_scale, const float *col_bias,
                                       int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s,
-                                      const AttEpi &att = AttEpi());
+                                      const AttEpi &att = AttEpi(), const GemmMirrors *mir = nullptr,
+                                      int32_t mir_col = 0);
 
 // Returns cudaErrorNotSupported only for shapes no launch takes (k < 1) or a
 // missing / misaligned workspace, cudaErrorInvalidValue for a workspace that
 // is too small (the caller reports GNN_ERR_WORKSPACE).
 cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H, int64_t ldh,
                            int64_t m, int32_t k, int32_t n, const float *row_scale, const float *col_bias,
-                           int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s) {
+                           int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s, const GemmMirrors *mir) {
   if (k < 1 || n < 1 || !ws || ((uintptr_t)ws & 15)) return cudaErrorNotSupported;
   if (ws_bytes < gemm_tc_workspace(m, k, n)) return cudaErrorInvalidValue;
   const int32_t sw = slice_width(m, k, n);
   for (int32_t c0 = 0; c0 < n; c0 += sw) {
     const int32_t w = n - c0 < sw ? n - c0 : sw;
     cudaError_t e = launch_gemm_tc_one(X, ldx, W + c0, ldw, H + c0, ldh, m, k, w, row_scale,
-                                       col_bias ? col_bias + c0 : nullptr, relu, ws, ws_bytes, s);
+                                       col_bias ? col_bias + c0 : nullptr, relu, ws, ws_bytes, s, AttEpi(), mir, c0);
     if (e != cudaSuccess) return e;
   }
   return cudaSuccess;
@@ -808,7 +828,7 @@ cudaError_t launch_gemm_tc(const float *X, int64_t ldx, const float *W, int64_t 
 // extra GEMM columns instead).
 cudaError_t launch_gemm_att(const float *X, int64_t ldx, const float *W, int64_t ldw, float *Z, int64_t ldz, int64_t m,
                             int32_t k, int32_t H, int32_t Fh, const float *a_src, const float *a_dst, void *ws,
-                            size_t ws_bytes, cudaStream_t s) {
+                            size_t ws_bytes, cudaStream_t s, const GemmMirrors *mir) {
   const int32_t n = H * Fh;
   if (Fh % 32 != 0 || k < 1 || !ws || ((uintptr_t)ws & 15) || slice_width(m, k, n) != n) return cudaErrorNotSupported;
   AttEpi att;
@@ -817,12 +837,13 @@ cudaError_t launch_gemm_att(const float *X, int64_t ldx, const float *W, int64_t
   att.H = H;
   att.Fh = Fh;
   att.col = n;
-  return launch_gemm_tc_one(X, ldx, W, ldw, Z, ldz, m, k, n, nullptr, nullptr, 0, ws, ws_bytes, s, att);
+  return launch_gemm_tc_one(X, ldx, W, ldw, Z, ldz, m, k, n, nullptr, nullptr, 0, ws, ws_bytes, s, att, mir, 0);
 }
 
 static cudaError_t launch_gemm_tc_one(const float *X, int64_t ldx, const float *W, int64_t ldw, float *H, int64_t ldh,
                                       int64_t m, int32_t k, int32_t n, const float *row_scale, const float *col_bias,
-                                      int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s, const AttEpi &att) {
+                                      int32_t relu, void *ws, size_t ws_bytes, cudaStream_t s, const AttEpi &att,
+                                      const GemmMirrors *mir, int32_t mir_col) {
   using namespace tc;
   Config c;
   if (!configure(m, k, n, c)) return cudaErrorNotSupported;
@@ -855,6 +876,18 @@ static cudaError_t launch_gemm_tc_one(const float *X, int64_t ldx, const float *
   memset(&hmap, 0, sizeof(hmap));
   const bool tma = vx && c.sa > 0 && (vh || c.ncb == 1) && tma_enabled() && m < 0x7fffff00LL && encode_x_map(&xmap, X, ldx, m, k) &&
                    (!vh || encode_h_map(&hmap, H, ldh, m, n));
+  // mirrors: one TMA map each over the same rows / columns (needs the TMA-store epilogue)
+  MirrorMaps mm;
+  memset(&mm, 0, sizeof(mm));
+  if (mir && mir->count > 0) {
+    if (!(tma && vh) || mir->count > kMaxMirrors) return cudaErrorNotSupported;
+    for (int q = 0; q < mir->count; ++q) {
+      float *d = mir->dst[q] + mir_col;
+      if (!d || ((uintptr_t)d & 15) || !encode_h_map(&mm.map[q], d, ldh, m, n)) return cudaErrorNotSupported;
+      mm.base[q] = d;
+    }
+    mm.count = mir->count;
+  }
   const bool pair = tma && c.cta2;
   const int64_t num_tiles = pair ? (m + rows_per_tile - 1) / rows_per_tile : num_tiles0;
   p.num_tiles = (int32_t)num_tiles;
@@ -909,13 +942,13 @@ static cudaError_t launch_gemm_tc_one(const float *X, int64_t ldx, const float *
     }
     const int clusters = (int)(p.num_tiles < mc ? p.num_tiles : mc);
     cfg.gridDim = dim3(2 * clusters);
-    e = cudaLaunchKernelEx(&cfg, fn, p, xmap, hmap);
+    e = cudaLaunchKernelEx(&cfg, fn, p, xmap, hmap, mm);
     count_launch();
     return e != cudaSuccess ? e : cudaGetLastError();
   }
   // one persistent CTA per SM, or one per work item when there are fewer
   const int grid = (int)(p.num_tiles < num_sms ? p.num_tiles : num_sms);
-  fn<<<grid, threads_of(tma), smem, s>>>(p, xmap, hmap);
+  fn<<<grid, threads_of(tma), smem, s>>>(p, xmap, hmap, mm);
   count_launch();
   return cudaGetLastError();
 }

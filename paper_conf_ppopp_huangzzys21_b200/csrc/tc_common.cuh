@@ -58,6 +58,12 @@ __device__ __forceinline__ void tma_store_2d(const CUtensorMap *map, int32_t c0,
                : "memory");
   asm volatile("cp.async.bulk.commit_group;" ::: "memory");
 }
+// the same store without its own bulk group (the caller commits once for several)
+__device__ __forceinline__ void tma_store_2d_nc(const CUtensorMap *map, int32_t c0, int32_t c1, const void *src) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];" ::"l"(map), "r"(c0),
+               "r"(c1), "r"(smem_u32(src))
+               : "memory");
+}
 template <int N>
 __device__ __forceinline__ void bulk_wait_read() {
   asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");

@@ -118,6 +118,14 @@ _SIGS = {
                                            ctypes.c_uint64, _P, _I64, _P, _SZ, _P]),
     "gnn_tune_aggregate": (ctypes.c_int, [_P, ctypes.c_int, ctypes.c_int, _P, _P, _I64, _I32, _P, _I64, _I32,
                                           ctypes.POINTER(gnn_tune_result), _P]),
+    "gnn_gemm_mirrored": (ctypes.c_int, [_P, _I64, _P, _I64, _P, _I64, _I64, _I32, _I32, _P, _P, _I32, _P, _I32, _P,
+                                         _SZ, _P]),
+    "gnn_gat_transform_mirrored": (ctypes.c_int, [_P, _I64, _I64, _I32, _P, _I64, _P, _P, _I32, _I32, _P, _I64, _P,
+                                                  _I32, _P, _SZ, _P]),
+    "gnn_ipc_alloc": (ctypes.c_int, [_SZ, ctypes.POINTER(_P), _P]),
+    "gnn_ipc_free": (ctypes.c_int, [_P]),
+    "gnn_ipc_open": (ctypes.c_int, [_P, ctypes.POINTER(_P)]),
+    "gnn_ipc_close": (ctypes.c_int, [_P]),
     "gnn_last_error": (ctypes.c_char_p, []),
     "gnn_version": (ctypes.c_char_p, []),
 }
@@ -386,6 +394,64 @@ def gemm(X, W, row_scale=None, col_bias=None, relu=False, out=None, stream=None,
     _call("gnn_gemm", _tp(X), _ld(X, k), _tp(W), _ld(W, n), _tp(H), _ld(H, n), m, k, n, _tp(row_scale),
           _tp(col_bias), int(relu), _tp(ws), nb, _stream(stream))
     return H
+
+
+def _ptr_array(ptrs):
+    arr = (ctypes.c_void_p * max(1, len(ptrs)))(*[int(p) for p in ptrs])
+    return arr, len(ptrs)
+
+
+def gemm_mirrored(X, W, mirrors, row_scale=None, col_bias=None, relu=False, out=None, stream=None):
+    """gnn_gemm_mirrored: H = X W written to `out` and to every mirror (device
+    pointers laid out like `out`: the same rows of peer replicas; NEXT-2)."""
+    torch = _torch()
+    m, k = X.shape
+    n = W.shape[1]
+    H = out if out is not None else torch.empty((m, n), dtype=torch.float32, device=X.device)
+    ws, nb = gemm_workspace(m, k, n, X.device)
+    arr, cnt = _ptr_array(mirrors)
+    _call("gnn_gemm_mirrored", _tp(X), _ld(X, k), _tp(W), _ld(W, n), _tp(H), _ld(H, n), m, k, n, _tp(row_scale),
+          _tp(col_bias), int(relu), arr, cnt, _tp(ws), nb, _stream(stream))
+    return H
+
+
+class IpcBuffer:
+    """A device buffer shareable across processes (gnn_ipc_alloc), viewed as a
+    torch fp32 tensor of `shape` (zero-copy, __cuda_array_interface__)."""
+
+    def __init__(self, shape, device):
+        torch = _torch()
+        self.shape = tuple(int(x) for x in shape)
+        nbytes = int(np.prod(self.shape)) * 4
+        self.handle = ctypes.create_string_buffer(64)
+        p = ctypes.c_void_p()
+        with torch.cuda.device(device):
+            _call("gnn_ipc_alloc", nbytes, ctypes.byref(p), self.handle)
+        self.ptr = p.value
+        self.__cuda_array_interface__ = {"shape": self.shape, "typestr": "<f4", "data": (self.ptr, False),
+                                         "version": 3, "strides": None}
+        self.tensor = torch.as_tensor(self, device=device)
+
+    def handle_bytes(self) -> bytes:
+        return self.handle.raw
+
+    def free(self):
+        if self.ptr:
+            self.tensor = None
+            _call("gnn_ipc_free", ctypes.c_void_p(self.ptr))
+            self.ptr = None
+
+
+def ipc_open(handle: bytes) -> int:
+    """Map a peer process's gnn_ipc_alloc buffer; returns the device pointer."""
+    p = ctypes.c_void_p()
+    hb = ctypes.create_string_buffer(handle, 64)
+    _call("gnn_ipc_open", hb, ctypes.byref(p))
+    return p.value
+
+
+def ipc_close(ptr: int) -> None:
+    _call("gnn_ipc_close", ctypes.c_void_p(ptr))
 
 
 def set_gemm_impl(impl: int) -> int:

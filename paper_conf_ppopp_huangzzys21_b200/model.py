@@ -56,12 +56,20 @@ def ring_allgather_blocks(buf, rmax, rank, world, group=None, on_block=None, sta
 class RowPartitionedGCNGAT:
     def __init__(self, rowptr, colidx, W1, W2, W3, a_src, a_dst, heads, head_dim, neg_slope=0.2,
                  rank=0, world=1, group=None, reorder=1, device=None, plan_opts=None, staged_allgather=False,
-                 overlap=False):
+                 overlap=False, exchange="nccl"):
         self.rank, self.world, self.group = rank, world, group
         self.dev = device or torch.device("cuda", torch.cuda.current_device())
         self.staged = staged_allgather  # gloo: exchange through host memory (tests only)
         # layer 2 exchange pipelined with the aggregation over source blocks (world > 1)
         self.overlap = bool(overlap) and world > 1
+        # exchange of layers 2 and 3: "nccl" (all_gather_into_tensor, or the ring
+        # with overlap) or "peer" (NEXT-2: the GEMM epilogue stores its rows into
+        # every peer's replica buffer through CUDA IPC, then a barrier)
+        if exchange not in ("nccl", "peer"):
+            raise ValueError("exchange must be 'nccl' or 'peer'")
+        self.peer = exchange == "peer" and world > 1
+        if self.peer and self.overlap:
+            raise ValueError("exchange='peer' replaces the ring exchange (overlap)")
         n = len(rowptr) - 1
         self.n = n
         opts = dict(reorder=reorder, **(plan_opts or {}))
@@ -101,9 +109,12 @@ class RowPartitionedGCNGAT:
         self.Xs = torch.zeros((P, self.F_in), device=d)          # replicated input, padded layout
         self.A1 = torch.empty((R, self.F_in), device=d)
         self.Y1 = torch.empty((R, self.F), device=d)
-        self.Hs2 = torch.zeros((P, self.F), device=d)
         self.Y2 = torch.empty((R, self.F), device=d)
-        self.Zst = torch.zeros((P, self.ldwe), device=d)
+        if self.peer:
+            self._setup_peer(P, d)
+        else:
+            self.Hs2 = torch.zeros((P, self.F), device=d)
+            self.Zst = torch.zeros((P, self.ldwe), device=d)
         self.Y3 = torch.empty((R, self.HF), device=d)
         self.nsrc_ptr, self.ndst_ptr = self.plan.normalizers()
         self.ws_agg, self.ws_agg_b = self.plan.workspace(_g.GNN_OP_AGGREGATE, 0, max(self.F, self.F_in), 0, d)
@@ -170,6 +181,61 @@ class RowPartitionedGCNGAT:
             self.Xs[q * self.rmax:q * self.rmax + (b - a)].copy_(X_host_or_dev[a:b], non_blocking=non_blocking)
 
     # -- exchange -----------------------------------------------------------
+    def _setup_peer(self, P, d):
+        """NEXT-2: the replica buffers Hs2 / Zst live in IPC-shareable memory;
+        every rank maps its peers' buffers and keeps, per layer, the list of
+        peer addresses of its own row block (the GEMM epilogue's mirrors)."""
+        import torch.distributed as dist
+        self._ipc = [_g.IpcBuffer((P, self.F), d), _g.IpcBuffer((P, self.ldwe), d)]
+        self.Hs2, self.Zst = self._ipc[0].tensor, self._ipc[1].tensor
+        self.Hs2.zero_()
+        self.Zst.zero_()
+        handles = [None] * self.world
+        dist.all_gather_object(handles, [b.handle_bytes() for b in self._ipc], group=self.group)
+        self._peer_ptrs = []
+        off = self.rank * self.rmax
+        self.mirrors2, self.mirrors3 = [], []
+        with torch.cuda.device(d):
+            for q in range(self.world):
+                if q == self.rank:
+                    continue
+                p2, p3 = _g.ipc_open(handles[q][0]), _g.ipc_open(handles[q][1])
+                self._peer_ptrs += [p2, p3]
+                self.mirrors2.append(p2 + 4 * off * self.F)
+                self.mirrors3.append(p3 + 4 * off * self.ldwe)
+        self._mir2 = _g._ptr_array(self.mirrors2)
+        self._mir3 = _g._ptr_array(self.mirrors3)
+        self._flag = torch.zeros(1, device=d)
+        torch.cuda.synchronize(d)
+        dist.barrier(group=self.group)
+
+    def _peer_barrier(self):
+        """Every rank's mirrored GEMM has finished (its stores are performed and
+        fenced at system scope) before any rank reads its replica: a
+        stream-ordered NCCL all_reduce of a flag (the aggregation queued after
+        it waits on the device, not the host); gloo: host barrier."""
+        import torch.distributed as dist
+        if dist.get_backend(self.group) == "nccl":
+            dist.all_reduce(self._flag, group=self.group)
+        else:
+            torch.cuda.synchronize(self.dev)
+            dist.barrier(group=self.group)
+
+    def close(self):
+        """Unmap the peers' buffers and free the IPC buffers (peer exchange)."""
+        if getattr(self, "_peer_ptrs", None):
+            import torch.distributed as dist
+            torch.cuda.synchronize(self.dev)
+            dist.barrier(group=self.group)  # no peer still writes into our buffers
+            for ptr in self._peer_ptrs:
+                _g.ipc_close(ptr)
+            self._peer_ptrs = []
+            dist.barrier(group=self.group)  # every peer has unmapped ours
+            self.Hs2 = self.Zst = None
+            for b in self._ipc:
+                b.free()
+            self._ipc = []
+
     def _allgather(self, buf):
         if self.world == 1:
             return
@@ -204,8 +270,13 @@ class RowPartitionedGCNGAT:
         chk(lib.gnn_gemm(P(self.A1), Fi, P(self.W1), F, P(self.Y1), F, R, Fi, F, None, None, 1, *gws, sp), "gemm1")
         rec(2)
         h_loc = self.Hs2[off:off + R]
-        chk(lib.gnn_gemm(P(self.Y1), F, P(self.W2), F, P(h_loc), F, R, F, F,
-                         ctypes.c_void_p(self.nsrc_ptr + 4 * off), None, 0, *gws, sp), "gemm2")
+        if self.peer:  # NEXT-2: the epilogue writes the rows into every peer's replica too
+            chk(lib.gnn_gemm_mirrored(P(self.Y1), F, P(self.W2), F, P(h_loc), F, R, F, F,
+                                      ctypes.c_void_p(self.nsrc_ptr + 4 * off), None, 0, self._mir2[0],
+                                      self._mir2[1], *gws, sp), "gemm2 (mirrored)")
+        else:
+            chk(lib.gnn_gemm(P(self.Y1), F, P(self.W2), F, P(h_loc), F, R, F, F,
+                             ctypes.c_void_p(self.nsrc_ptr + 4 * off), None, 0, *gws, sp), "gemm2")
         if self.overlap:
             # source-block pipeline: aggregate each rank's block of Hs2 as it arrives
             # (own block first), raw sums accumulated in ring order, then x ndst
@@ -219,16 +290,25 @@ class RowPartitionedGCNGAT:
             ring_allgather_blocks(self.Hs2, self.rmax, self.rank, self.world, self.group, on_block, self.staged)
             chk(lib.gnn_scale_rows(P(self.Y2), F, R, F, ctypes.c_void_p(self.ndst_ptr), 0, sp), "agg2 scale")
         else:
-            self._allgather(self.Hs2)
+            if self.peer:
+                self._peer_barrier()
+            else:
+                self._allgather(self.Hs2)
             rec(3)
             chk(lib.gnn_gcn_aggregate_prescaled(self.plan.handle, P(self.Hs2), F, F, P(self.Y2), F, 0,
                                                 P(self.ws_agg), self.ws_agg_b, sp), "agg2")
         rec(4)
         z_loc = self.Zst[off:off + R]
         # [Z | s | t] = Y2 W3 with the GAT scores from the GEMM epilogue (R5)
-        chk(lib.gnn_gat_transform(P(self.Y2), F, R, F, P(self.W3), HF, P(self.a_s), P(self.a_d), H, self.Fh, P(z_loc),
-                                  self.ldwe, *gws, sp), "gemm3 (gat transform)")
-        self._allgather(self.Zst)
+        if self.peer:
+            chk(lib.gnn_gat_transform_mirrored(P(self.Y2), F, R, F, P(self.W3), HF, P(self.a_s), P(self.a_d), H,
+                                               self.Fh, P(z_loc), self.ldwe, self._mir3[0], self._mir3[1], *gws, sp),
+                "gemm3 (gat transform, mirrored)")
+            self._peer_barrier()
+        else:
+            chk(lib.gnn_gat_transform(P(self.Y2), F, R, F, P(self.W3), HF, P(self.a_s), P(self.a_d), H, self.Fh,
+                                      P(z_loc), self.ldwe, *gws, sp), "gemm3 (gat transform)")
+            self._allgather(self.Zst)
         rec(5)
         tptr = ctypes.c_void_p(z_loc.data_ptr() + 4 * (HF + H))
         chk(lib.gnn_gat_aggregate(self.plan.handle, P(self.Zst), self.ldwe, tptr, self.ldwe, H, self.Fh,

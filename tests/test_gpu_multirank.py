@@ -16,9 +16,9 @@ if not torch.cuda.is_available():  # pragma: no cover
     pytest.skip("needs a CUDA device", allow_module_level=True)
 
 
-def _inputs():
+def _inputs(Fh=16):
     g = gs.powerlaw(30000, 600000, 20, 4000, 3000, comm=64, rho=0.8, seed=5)
-    F_in, F, Hh, Fh = 100, 64, 4, 16
+    F_in, F, Hh = 100, 64, 4
     X = gs.uniform(g.n, F_in, seed=1)
     W1 = gs.uniform(F_in, F, lo=-0.2, hi=0.2, seed=2)
     W2 = gs.uniform(F, F, lo=-0.25, hi=0.25, seed=3)
@@ -36,7 +36,7 @@ def _port():
     return p
 
 
-def _worker(rank, world, port, q, overlap=False):
+def _worker(rank, world, port, q, overlap=False, exchange="nccl", Fh=16):
     try:
         import torch.distributed as dist
         from paper_conf_ppopp_huangzzys21_b200.model import RowPartitionedGCNGAT
@@ -44,11 +44,15 @@ def _worker(rank, world, port, q, overlap=False):
         os.environ["MASTER_PORT"] = str(port)
         dist.init_process_group("gloo", rank=rank, world_size=world)
         torch.cuda.set_device(0)
-        g, X, W1, W2, W3, a_s, a_d, Hh, Fh = _inputs()
+        g, X, W1, W2, W3, a_s, a_d, Hh, Fh = _inputs(Fh)
         m = RowPartitionedGCNGAT(g.rowptr, g.colidx, W1, W2, W3, a_s, a_d, Hh, Fh, rank=rank, world=world,
-                                 reorder=1, staged_allgather=True, overlap=overlap)
+                                 reorder=1, staged_allgather=True, overlap=overlap, exchange=exchange)
         m.load_input(torch.from_numpy(X), non_blocking=False)
         Y = m.step().cpu().numpy()
+        if exchange == "peer":  # a second step over the same IPC buffers, then unmap / free
+            Y2 = m.step().cpu().numpy()
+            assert np.array_equal(Y.view(np.uint32), Y2.view(np.uint32)), "peer exchange rerun differs"
+            m.close()
         if overlap:  # layer outputs too (the overlapped path is checked layer by layer)
             Y = (m.Y1.cpu().numpy(), m.Y2.cpu().numpy(), Y, m.step().cpu().numpy())
         parts = [None] * world
@@ -93,6 +97,34 @@ def test_two_ranks_bit_identical_to_one_and_oracle():
     assert np.all(np.abs(L2[rows] - r2.astype(np.float64)) <= tol(r2)), "layer 2"
     r3 = oracle.gat_layer(g.rowptr, g.colidx, L2, W3, a_s, a_d, Hh, Fh, 0.2, rows=rows)
     assert np.all(np.abs(Y1[rows] - r3.astype(np.float64)) <= tol(r3)), "layer 3"
+
+
+@pytest.mark.parametrize("Fh", [16, 32])
+def test_two_ranks_peer_exchange_bit_identical_to_one(Fh):
+    """NEXT-2: the exchange fused into the producers -- each rank's GEMM2 and
+    GAT-transform epilogues also store their rows into the peer's replica
+    buffer (CUDA IPC mapping, gnn_gemm_mirrored / gnn_gat_transform_mirrored),
+    then a barrier -- is bit-identical to P = 1.  Two processes share this
+    B200 (no kernel waits on the other rank: the barrier is on the host).
+    Fh = 16 takes the folded-score GEMM, Fh = 32 the score epilogue."""
+    import torch.multiprocessing as mp
+
+    from paper_conf_ppopp_huangzzys21_b200.model import RowPartitionedGCNGAT
+    g, X, W1, W2, W3, a_s, a_d, Hh, Fh = _inputs(Fh)
+    m1 = RowPartitionedGCNGAT(g.rowptr, g.colidx, W1, W2, W3, a_s, a_d, Hh, Fh, reorder=0)
+    m1.load_input(torch.from_numpy(X), non_blocking=False)
+    Y1 = m1.step().cpu().numpy()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q, False, "peer", Fh)) for r in range(2)]
+    for p in procs:
+        p.start()
+    Y2 = q.get(timeout=600)
+    for p in procs:
+        p.join(timeout=120)
+    assert not isinstance(Y2, str), Y2
+    assert np.array_equal(Y1.view(np.uint32), Y2.view(np.uint32))
 
 
 def test_two_ranks_overlapped_exchange_vs_oracle():
