@@ -23,18 +23,19 @@ namespace gnn {
 // is LANES consecutive lanes (LANES in {4, 8, 16, 32}); each lane owns NV
 // vectors of VEC consecutive features (VEC in {1,2,4,8}; VEC = 8 is one
 // 256-bit LDG per lane).  Chunk width CW = LANES*VEC*NV features; wider rows
-// loop over chunks.  One CTA processes one plan tile (<= T neighbor groups,
-// P:855-884) per launch block; workers take groups round-robin.
+// loop over chunks.  A persistent grid of workers claims work units (one
+// neighbour group each) in task (LAS) order from one atomic
+// counter per feature chunk.
 //
 // Per group: indices are loaded LANES at a time (one coalesced load), then
-// broadcast with sub-warp shuffles; U source rows are in flight per worker.
-// Group partial = sequential fp32 chain in CSR order (reading R9).
-// Single-group rows finish in the worker (epilogue + store).  Multi-group
-// rows inside one tile are combined in shared memory in group order (TB-level
-// data-visible-range adapter).  Rows spanning several tiles write
-// per-group partials to the workspace; the last-arriving CTA (per-row counter)
-// merges them in group order (P:885-894 with a fixed order) and applies the
-// postponed epilogue (linear property).
+// broadcast with sub-warp shuffles; U source rows are in flight per worker
+// (register kernel) or S rows in a per-warp shared-memory ring (cp.async
+// chain).  Group partial = sequential fp32 chain in CSR order (reading R9).
+// Single-group rows finish in the worker (epilogue + store).  The groups of
+// a longer row write their partials to the workspace; the last to arrive
+// (per-row arrival counter) merges them in group order (P:885-894 with a
+// fixed order) and applies the postponed epilogue (linear property,
+// P:970-986).  The atomic variant adds the partials into one accumulator row.
 // ---------------------------------------------------------------------------
 enum { M_SUM = 0, M_MEAN = 1, M_MAX = 2, M_GAT = 3, M_SYM = 4, M_LIN = 5, M_GAAN = 6, M_GENE = 7 };
 // attention modes (softmax aggregation of Table 1 with a Table 2 score, R9/R14)

@@ -116,7 +116,10 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
   // lane mapping (VEC, 32, NV): (4, 32, 2) / (8, 32, 1) for 256 features per sweep, (4, 32, 1) for <= 128
   extern __shared__ __align__(128) float smem_raw[];
   __shared__ uint64_t bars[WARPS][S];
-  float *smem = reinterpret_cast<float *>(((uintptr_t)smem_raw + 127) & ~(uintptr_t)127);
+  // 128-byte aligned base as an offset from the shared array, so every slot
+  // pointer stays in the shared window (LDS, 32-bit addresses) instead of
+  // decaying to a generic pointer (LD.E with 64-bit address arithmetic)
+  float *smem = smem_raw + (((128u - (sa(smem_raw) & 127u)) & 127u) >> 2);
   const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
   const DevGraph &g = p.g;
   if ((int32_t)blockIdx.x >= p.n_persist) {  // zero-fill rows without in-edges (R3-i)
@@ -339,12 +342,14 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
             }
 #pragma unroll
             for (int j = 0; j < 4; ++j) ls += ex4[j];
+            // no per-lane guards in the fast path: a lane past F reads bytes
+            // inside this warp's shared region (the slot's tail / the next
+            // slot / the score and queue regions) and its sums are never stored
 #pragma unroll
             for (int j = 0; j < 4; ++j) {
 #pragma unroll
               for (int n = 0; n < NV; ++n) {
                 const float exn = __shfl_sync(0xffffffffu, ex4[j], head[n]);
-                if (!valid[n]) continue;
                 float v[VEC];
                 lds_vec<VEC>(rq + j * BW + (n * 32 + lane) * VEC, v);
                 fma_vec<VEC>(G.a[n], v, exn);
@@ -355,8 +360,7 @@ __global__ void __launch_bounds__(g4::WARPS * 32, 2)
             for (int j = 0; j < 4; ++j) {
               const float wt = 1.0f;  // weight 1 (pre-scaled GCN: ndst in the epilogue)
 #pragma unroll
-              for (int n = 0; n < NV; ++n) {
-                if (!valid[n]) continue;
+              for (int n = 0; n < NV; ++n) {  // unguarded, as above
                 float v[VEC];
                 lds_vec<VEC>(rq + j * BW + (n * 32 + lane) * VEC, v);
                 if constexpr (MODE == M_MAX) {

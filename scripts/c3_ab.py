@@ -34,7 +34,15 @@ gen = torch.Generator(device="cuda")
 gen.manual_seed(3)
 Hs = torch.rand((n, 256), device="cuda", generator=gen) * 2 - 1
 H1 = torch.empty_like(Hs)
-fn = lambda: G.aggregate(plan, Hs, "sum", "gcn", out=H1)  # noqa: E731
+if "--prescaled" in sys.argv:  # the transform-first layer's form: rows pre-scaled by nsrc, x ndst in the epilogue
+    import ctypes
+    ws, wb = plan.workspace(G.gnn.GNN_OP_AGGREGATE, 0, 256, 0, Hs.device)
+    P = lambda t: ctypes.c_void_p(t.data_ptr())  # noqa: E731
+    fn = lambda: G.gnn._lib.gnn_gcn_aggregate_prescaled(plan.handle, P(Hs), 256, 256, P(H1), 256, 0, P(ws), wb,  # noqa
+                                                      None)
+    tag += " prescaled"
+else:
+    fn = lambda: G.aggregate(plan, Hs, "sum", "gcn", out=H1)  # noqa: E731
 if "--once" in sys.argv:
     fn()
     torch.cuda.synchronize()
