@@ -732,6 +732,12 @@ __device__ __forceinline__ void cp_wait() {
 __device__ __forceinline__ void cp_async16_zfill(uint32_t dst, const void *src, uint32_t src_bytes) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
 }
+__device__ __forceinline__ void cp_async16_if(uint32_t dst, const void *src, uint32_t pred) {
+  asm volatile(
+      "{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %2, 0;\n\t@q cp.async.cg.shared.global [%0], [%1], 16;\n\t}" ::"r"(dst),
+      "l"(src), "r"(pred)
+      : "memory");
+}
 __device__ __forceinline__ void cp_async4_if(uint32_t dst, const void *src, uint32_t pred) {
   asm volatile(
       "{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %2, 0;\n\t@q cp.async.ca.shared.global [%0], [%1], 4;\n\t}" ::"r"(dst),
@@ -742,6 +748,17 @@ __device__ __forceinline__ void cp_async4_if(uint32_t dst, const void *src, uint
 template <int MODE, int NV>
 __host__ __device__ constexpr int cp_slot_floats() {
   return NV * 128 + (MODE == M_GAT ? 32 : 4);
+}
+// lean chain (sum / mean / max): a slot holds only the row's features of one
+// chunk, min(F, NV*128) rounded to 16 bytes (C5 agg1: 400 B instead of 528 B,
+// so the ring holds more rows in the same shared memory); lanes past F issue
+// no copy and their reads of the next slot's bytes are never stored.  The
+// per-CTA allocation is padded by one full-width slot for the last lane's reads.
+template <int MODE, int NV>
+__host__ __device__ inline int cp_ring_slot(int32_t F) {
+  if (MODE == M_GAT) return cp_slot_floats<MODE, NV>();
+  const int w = F < NV * 128 ? F : NV * 128;
+  return (w + 3) & ~3;
 }
 
 // Lean chain for sum / mean / max (no GAT): the per-edge issue is branch-free
@@ -758,7 +775,7 @@ template <int MODE, int NV, int S>
 __device__ __forceinline__ void group_chain_cp_lean(const KParams &p, const int32_t *idx, int32_t len, int32_t beg,
                                                     int32_t c0, int lane, float *ring, Part<MODE, 4, NV> &G) {
   constexpr int VEC = 4;
-  constexpr int SLOT = cp_slot_floats<MODE, NV>();
+  const int SLOT = cp_ring_slot<MODE, NV>(p.F);
   // U consecutive edges share one commit group, one wait and one pair of
   // warp barriers; the R9 chain still adds them one by one in CSR order
   constexpr int U = (S % GNN_CP_U == 0) ? GNN_CP_U : (S % 2 == 0 ? 2 : 1);
@@ -769,9 +786,9 @@ __device__ __forceinline__ void group_chain_cp_lean(const KParams &p, const int3
   const int weight = p.weight;
   const bool has_w = weight == GNN_W_GCN || weight == GNN_W_EDGE;
   const uint32_t ring_s = (uint32_t)__cvta_generic_to_shared(ring);
-  uint32_t nbytes[NV];
+  uint32_t lv[NV];  // this lane copies vector n (inside F)
 #pragma unroll
-  for (int n = 0; n < NV; ++n) nbytes[n] = (c0 + (n * 32 + lane) * VEC < p.F) ? 16u : 0u;
+  for (int n = 0; n < NV; ++n) lv[n] = (c0 + (n * 32 + lane) * VEC < p.F) ? 1u : 0u;
   // row addresses: one IMAD.WIDE.U32 per edge (u unsigned x the row pitch in
   // bytes, cp_admissible: ldx * 4 < 2^32)
   const char *xl = reinterpret_cast<const char *>(p.X + c0 + lane * VEC);
@@ -796,7 +813,7 @@ __device__ __forceinline__ void group_chain_cp_lean(const KParams &p, const int3
   // issue edges e0 .. e0+U-1 (e0 % U == 0) as one commit group; indices from
   // the 32-entry window `cur` (refilled from `nxt` at multiples of 32); a
   // batch wholly inside the group needs no per-edge checks (FULL), the last
-  // ones zero-fill the copies of edges past the end
+  // ones copy nothing for edges past the end
   auto issue = [&](int32_t e0, auto full) {
     if ((e0 & 31) == 0 && e0 >= 32) {
       cur = nxt;
@@ -812,9 +829,9 @@ __device__ __forceinline__ void group_chain_cp_lean(const KParams &p, const int3
 #pragma unroll
       for (int n = 0; n < NV; ++n) {
         if constexpr (decltype(full)::value)
-          cp_async16_zfill(sw + my_off + (uint32_t)(n * 512), src + n * 512, nbytes[n]);
+          cp_async16_if(sw + my_off + (uint32_t)(n * 512), src + n * 512, lv[n]);
         else
-          cp_async16_zfill(sw + my_off + (uint32_t)(n * 512), src + n * 512, e < len ? nbytes[n] : 0u);
+          cp_async16_if(sw + my_off + (uint32_t)(n * 512), src + n * 512, e < len ? lv[n] : 0u);
       }
     }
     cp_commit();
@@ -1211,7 +1228,7 @@ __global__ void __launch_bounds__(256, S > 0 ? GNN_AGG_MINB_CP
       }
       if constexpr (S > 0)
         process_unit<MODE, VEC, NV, LANES, S>(p, d, dnx - d.x, c0, ci, lane, mask,
-                                              cp_smem + (tid >> 5) * S * cp_slot_floats<MODE, NV>());
+                                              cp_smem + (tid >> 5) * S * cp_ring_slot<MODE, NV>(p.F));
       else
         process_unit<MODE, VEC, NV, LANES>(p, d, dnx - d.x, c0, ci, lane, mask);
       if (p.trace && lane == 0) {
@@ -1278,10 +1295,10 @@ int num_sms();
 
 template <typename KFN>
 cudaError_t launch_persistent(KFN fn, int &occ, const KParams &kp_in, int32_t units, int cw, int lanes,
-                                     int threads, cudaStream_t s, size_t smem = 0) {
+                                     int threads, cudaStream_t s, size_t smem = 0, size_t smem_attr = 0) {
   if (occ == 0) {
-    if (smem > 0) {  // cp.async ring: shared memory first
-      cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (smem > 0) {  // cp.async ring: shared memory first (attribute: the largest ring this kernel takes)
+      cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)std::max(smem, smem_attr));
       cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
     } else {
       cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, 0);  // all of it to L1
@@ -1332,9 +1349,21 @@ template <int MODE, int NV>
 cudaError_t launch_cp(const KParams &kp, int threads, cudaStream_t s) {
   constexpr int S = NV == 1 ? GNN_CP_S1 : GNN_CP_S2;
   constexpr int CW = 32 * 4 * NV;
-  static int occ = 0;
-  const size_t smem = sizeof(float) * (size_t)(threads / 32) * S * cp_slot_floats<MODE, NV>();
-  return launch_persistent(k_aggregate<MODE, 4, NV, 32, S>, occ, kp, kp.g.n_units, CW, 32, threads, s, smem);
+  const size_t smem = sizeof(float) * ((size_t)(threads / 32) * S * cp_ring_slot<MODE, NV>(kp.F) + NV * 128);
+  // the ring size depends on F: occupancy (and the dynamic shared-memory
+  // attribute, set when occ == 0) cached per ring size
+  static size_t occ_smem[8] = {0};
+  static int occ_val[8] = {0};
+  int slot = 0;
+  while (slot < 8 && occ_smem[slot] != 0 && occ_smem[slot] != smem) ++slot;
+  if (slot == 8) slot = 7;  // more sizes than slots: recompute in the last one
+  if (occ_smem[slot] != smem) {
+    occ_smem[slot] = smem;
+    occ_val[slot] = 0;
+  }
+  const size_t smem_max = sizeof(float) * ((size_t)(threads / 32) * S * cp_slot_floats<MODE, NV>() + NV * 128);
+  return launch_persistent(k_aggregate<MODE, 4, NV, 32, S>, occ_val[slot], kp, kp.g.n_units, CW, 32, threads, s,
+                           smem, smem_max);
 }
 
 template <int MODE, int VEC>

@@ -59,8 +59,9 @@ def fp(t):
 
 gen = torch.Generator(device="cuda")
 gen.manual_seed(1)
-X1 = torch.rand(n, 100, device="cuda", generator=gen) * 2 - 1
-Y1 = torch.empty_like(X1)
+LDX1 = int(os.environ.get("AGG_AB_LDX1", "100"))  # row pitch of agg1's X (the bench pads 100 -> 104)
+X1 = (torch.rand(n, LDX1, device="cuda", generator=gen) * 2 - 1)[:, :100]
+Y1 = torch.empty((n, 100), device="cuda")
 X2 = torch.rand(n, 256, device="cuda", generator=gen) * 2 - 1
 Y2 = torch.empty_like(X2)
 Hh, Fh = 8, 32
