@@ -195,3 +195,30 @@ def test_plan_load_rejects_missing_and_foreign_files(tmp_path):
     assert P.gnn.gnn_plan_load(str(f).encode(), ctypes.byref(h)) == 1
     assert "not a gnn plan" in P.gnn.gnn_last_error()
     assert P.gnn.gnn_plan_save(None, b"/tmp/x", 0) == 1
+
+
+def test_mirrored_entry_points_validate_before_device_work():
+    """NEXT-2 entry points (gnn_gemm_mirrored, gnn_gat_transform_mirrored,
+    gnn_ipc_*) reject bad arguments on the host, with fake device pointers."""
+    g = P.gnn
+    fake = lambda off: ctypes.c_void_p(0x7f0000000000 + off)  # noqa: E731 (never dereferenced)
+    X, W, H, ws = fake(0), fake(1 << 30), fake(2 << 30), fake(3 << 30)
+    m, k, n = 1000, 64, 64
+    arr8, _ = g._ptr_array([0x7f1000000000 + 4096 * i for i in range(8)])
+    assert g.gnn_gemm_mirrored(X, k, W, n, H, n, m, k, n, None, None, 0, arr8, 8, ws, 1 << 20, None) == 1  # > 7
+    assert "n_mirrors" in g.gnn_last_error()
+    bad, _ = g._ptr_array([0x7f1000000004])
+    assert g.gnn_gemm_mirrored(X, k, W, n, H, n, m, k, n, None, None, 0, bad, 1, ws, 1 << 20, None) == 1  # misaligned
+    null, _ = g._ptr_array([0])
+    assert g.gnn_gemm_mirrored(X, k, W, n, H, n, m, k, n, None, None, 0, null, 1, ws, 1 << 20, None) == 1
+    ok, _ = g._ptr_array([0x7f1000000000])
+    assert g.gnn_gemm_mirrored(X, k, W, n, H, n, m, k, n, None, None, 0, ok, 1, None, 0, None) == 1  # no workspace
+    assert g.gnn_gemm_mirrored(X, k, W, n, X, n, m, k, n, None, None, 0, ok, 1, ws, 1 << 20, None) == 1  # H == X
+    over, _ = g._ptr_array([0x7f0000000000 + 64])  # inside X
+    assert g.gnn_gemm_mirrored(X, k, W, n, H, n, m, k, n, None, None, 0, over, 1, ws, 1 << 20, None) == 1
+    assert g.gnn_gemm_mirrored(X, k, W, n, H, n, m, 0, n, None, None, 0, ok, 1, ws, 1 << 20, None) == 1  # k < 1
+    assert g.gnn_gat_transform_mirrored(X, 64, m, 64, W, 256, fake(5 << 30), fake(6 << 30), 8, 32, H, 272, arr8, 8,
+                                        ws, 1 << 20, None) == 1
+    assert g.gnn_ipc_alloc(0, None, None) == 1
+    assert g.gnn_ipc_open(None, None) == 1
+    assert g.gnn_ipc_free(None) == 0 and g.gnn_ipc_close(None) == 0
