@@ -42,6 +42,7 @@ static void free_plan(gnn_plan_s *p) {
   cudaSetDevice(p->device);
   for (void *d : p->dev_allocs) cudaFree(d);
   for (void *d : p->sched_allocs) cudaFree(d);
+  if (p->d_hot) cudaFree(p->d_hot);
   cudaSetDevice(cur);
   delete p;
 }

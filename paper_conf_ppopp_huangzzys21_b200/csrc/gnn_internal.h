@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <mutex>
 #include <string>
 #include <vector>
 
@@ -74,6 +75,12 @@ struct gnn_plan_s {
   int32_t tuned_F = 0, tuned_vec = 0, tuned_lanes = 0, tuned_nv = 0;
   gnn::DevGraph dg{};
   const int32_t *d_dout = nullptr;  // device source out-degrees (counted or the override)
+  // hot source rows (the highest out-degrees, in degree order) whose L2 lines
+  // an aggregation marks evict_last for its duration (k_graph.cu); built on
+  // first use from d_dout, freed with the plan
+  mutable std::once_flag hot_once;
+  mutable int32_t *d_hot = nullptr;
+  mutable int32_t n_hot = 0;
 };
 
 namespace gnn {
