@@ -1169,7 +1169,7 @@ __device__ __forceinline__ void finish_unit(const KParams &p, const Part<MODE, V
 #define GNN_CP_S1 12  // NV = 1: rows <= 128 features
 #endif
 #ifndef GNN_CP_S2
-#define GNN_CP_S2 6  // NV = 2: rows <= 256 features
+#define GNN_CP_S2 8  // NV = 2: rows <= 256 features (C3 F=256 GCN, same box: S = 4 / 6 / 8 / 12 -> 9.7-9.8 / 10.0-10.1 / 9.2-9.5 / 9.65 ms)
 #endif
 template <int MODE, int VEC, int NV, int LANES, int S = 0>
 __global__ void __launch_bounds__(256, S > 0 ? GNN_AGG_MINB_CP
