@@ -279,7 +279,11 @@ def test_plan_bit_exact_vs_oracle(rho):
 # --------------------------------------------------------------------------- #
 # a7 fused GAT
 # --------------------------------------------------------------------------- #
-@pytest.mark.parametrize("Hh,Fh", [(8, 8), (8, 32), (1, 1), (2, 3), (4, 16)])
+# rows > 128 features with 4..32 heads take the gather4 kernel: scores in the
+# row's request for F <= 256 ((4,64), (16,16), (32,8), (4,48), (16,12)), a
+# separate score gather and two feature sweeps for F = 320 ((8,40))
+@pytest.mark.parametrize("Hh,Fh", [(8, 8), (8, 32), (1, 1), (2, 3), (4, 16), (4, 64), (16, 16), (32, 8), (4, 48),
+                                   (8, 40), (16, 12)])
 @pytest.mark.parametrize("gname", ["small", "hub"])
 def test_gat_aggregate_parity(graphs, Hh, Fh, gname):
     g = graphs[gname]
