@@ -890,6 +890,145 @@ __device__ __forceinline__ void group_chain_cp_lean(const KParams &p, const int3
   }
 }
 
+// Lean chain for GAT (same structure as group_chain_cp_lean): U = 4 edges per
+// commit group, predicated 16-byte row copies, the H scores s_u[h] of each
+// edge by 16-byte copies of lanes 0 .. H/4-1 (4-byte copies when H % 4 != 0)
+// into the slot tail; each lane computes e and exp(e - m) for the head of each
+// of its vectors (same expression and order as the register and gather4
+// kernels: bit-identical).  A group whose softmax bound was too loose for
+// some head is streamed a second time against its exact maxima (R9 GAT).
+template <int NV, int S>
+__device__ __forceinline__ void group_chain_cp_lean_gat(const KParams &p, const int32_t *idx, int32_t len,
+                                                        int32_t row, int32_t c0, int lane, float *ring,
+                                                        Part<M_GAT, 4, NV> &G) {
+  constexpr int VEC = 4;
+  constexpr int SLOT = cp_slot_floats<M_GAT, NV>();
+  constexpr int U = (S % GNN_CP_U == 0) ? GNN_CP_U : (S % 2 == 0 ? 2 : 1);
+  constexpr int NG = S / U;
+  static_assert(32 % U == 0 && S <= 32, "U divides the 32-entry index window, S fits it");
+  const uint32_t ring_s = (uint32_t)__cvta_generic_to_shared(ring);
+  uint32_t lv[NV];
+  bool valid[NV];
+  int32_t head[NV];
+  float tv[NV], nmb[NV], seen[NV];
+  const bool one = len == 1;
+#pragma unroll
+  for (int n = 0; n < NV; ++n) {
+    const int32_t f = c0 + (n * 32 + lane) * VEC;
+    valid[n] = f < p.F;
+    lv[n] = valid[n] ? 1u : 0u;
+    head[n] = valid[n] ? f / p.Fh : 0;
+    tv[n] = valid[n] ? __ldg(p.t + (int64_t)row * p.ldt + head[n]) : 0.0f;
+    const float mb = valid[n] ? leaky_f(fkey_decode(__ldg(p.smax + head[n])) + tv[n], p.slope) : 0.0f;
+    G.m[n] = mb;
+    nmb[n] = -mb * kLog2e;
+  }
+  const char *xl = reinterpret_cast<const char *>(p.X + c0 + lane * VEC);
+  const char *sxl = reinterpret_cast<const char *>(p.X + p.F);
+  const uint32_t ldxb = (uint32_t)p.ldx * 4u;
+  const uint32_t my_off = (uint32_t)(lane * VEC * 4);
+  const bool s16 = (p.H & 3) == 0;
+  const uint32_t sc_lane = s16 ? ((lane < (p.H >> 2)) ? 1u : 0u) : ((lane < p.H) ? 1u : 0u);
+  const uint32_t sc_off = s16 ? (uint32_t)(lane * 16) : (uint32_t)(lane * 4);
+#pragma unroll 1
+  for (int pass = 0;; ++pass) {
+#pragma unroll
+    for (int n = 0; n < NV; ++n) {
+      G.l[n] = 0.0f;
+      seen[n] = -INFINITY;
+#pragma unroll
+      for (int i = 0; i < VEC; ++i) G.a[n][i] = 0.0f;
+    }
+    uint32_t slot_w = ring_s;
+    int slot_i = 0;
+    int32_t cur = lane < len ? ld_stream_i32(idx + lane) : 0;
+    int32_t nxt = 32 + lane < len ? ld_stream_i32(idx + 32 + lane) : 0;
+    auto issue = [&](int32_t e0) {
+      if ((e0 & 31) == 0 && e0 >= 32) {
+        cur = nxt;
+        nxt = e0 + 32 + lane < len ? ld_stream_i32(idx + e0 + 32 + lane) : 0;
+      }
+#pragma unroll
+      for (int j = 0; j < U; ++j) {
+        const int32_t e = e0 + j;
+        const uint32_t u = (uint32_t)__shfl_sync(0xffffffffu, cur, (e0 & 31) + j);
+        const uint32_t sw = slot_w + (uint32_t)(j * SLOT * 4);
+        const uint32_t live = e < len ? 1u : 0u;
+        const char *src = xl + (uint64_t)u * ldxb;
+#pragma unroll
+        for (int n = 0; n < NV; ++n) cp_async16_if(sw + my_off + (uint32_t)(n * 512), src + n * 512, live & lv[n]);
+        const char *ss = sxl + (uint64_t)u * ldxb + sc_off;
+        if (s16) cp_async16_if(sw + (uint32_t)(NV * 512) + sc_off, ss, live & sc_lane);
+        else cp_async4_if(sw + (uint32_t)(NV * 512) + sc_off, ss, live & sc_lane);
+      }
+      cp_commit();
+      slot_i += U;
+      if (slot_i == S) {
+        slot_i = 0;
+        slot_w = ring_s;
+      } else {
+        slot_w += (uint32_t)(U * SLOT * 4);
+      }
+    };
+#pragma unroll
+    for (int q = 0; q < NG; ++q) issue(q * U);
+    const float *rd = ring;
+    int rd_i = 0;
+    auto consume = [&](int j) {
+      const float *sl = rd + j * SLOT;
+#pragma unroll
+      for (int n = 0; n < NV; ++n) {
+        const float4 x4 = *reinterpret_cast<const float4 *>(sl + n * 128 + lane * VEC);
+        const float v[4] = {x4.x, x4.y, x4.z, x4.w};
+        const float sco = leaky_f(sl[NV * 128 + head[n]] + tv[n], p.slope);
+        seen[n] = fmaxf(seen[n], sco);
+        const float ex = one ? 1.0f : ex2_f(fmaf(sco, kLog2e, nmb[n]));
+        G.l[n] += ex;
+        fma_vec<VEC>(G.a[n], v, ex);
+      }
+    };
+    for (int32_t e0 = 0; e0 < len; e0 += U) {
+      cp_wait<NG - 1>();
+      __syncwarp();
+      if (e0 + U <= len) {
+#pragma unroll
+        for (int j = 0; j < U; ++j) consume(j);
+      } else {
+        for (int j = 0; j < len - e0; ++j) consume(j);
+      }
+      __syncwarp();  // every lane has read the slots before they are refilled
+      rd_i += U;
+      if (rd_i == S) {
+        rd_i = 0;
+        rd = ring;
+      } else {
+        rd += U * SLOT;
+      }
+      issue(e0 + S);
+    }
+    cp_wait<0>();  // nothing of this pass is still landing in the ring
+    if (one) {
+#pragma unroll
+      for (int n = 0; n < NV; ++n) G.m[n] = seen[n];
+      break;
+    }
+    // bound too loose for some head of this warp: redo against the exact max (R9 GAT)
+    bool loose = false;
+#pragma unroll
+    for (int n = 0; n < NV; ++n) loose |= valid[n] && !(G.m[n] - seen[n] <= kGatSlack);
+    if (pass == 1 || !__any_sync(0xffffffffu, loose)) break;
+#pragma unroll
+    for (int n = 0; n < NV; ++n) {
+      G.m[n] = seen[n];
+      nmb[n] = -seen[n] * kLog2e;
+    }
+    __syncwarp();
+  }
+}
+
+#ifndef GNN_CP_GAT_LEAN
+#define GNN_CP_GAT_LEAN 1  // 0: the per-edge GAT chain below
+#endif
 template <int MODE, int NV, int S>
 __device__ __forceinline__ void group_chain_cp(const KParams &p, const int32_t *idx, int32_t len, int32_t beg,
                                                int32_t row, int32_t c0, int lane, float *ring,
@@ -902,6 +1041,10 @@ __device__ __forceinline__ void group_chain_cp(const KParams &p, const int32_t *
     group_chain_cp_lean<MODE, NV, S>(p, idx, len, beg, c0, lane, ring, G);
     return;
 #endif
+  } else if constexpr (GNN_CP_GAT_LEAN) {
+    (void)beg;
+    group_chain_cp_lean_gat<NV, S>(p, idx, len, row, c0, lane, ring, G);
+    return;
   }
   part_init(G);
   const int weight = p.weight;

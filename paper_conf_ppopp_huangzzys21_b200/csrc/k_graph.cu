@@ -407,32 +407,40 @@ static Mapping choose_mapping(const gnn_plan_s *p, const AggArgs &a, int32_t fh_
   const Mapping t{p->tuned_vec, p->tuned_lanes, p->tuned_nv};
   if (p->tuned_F == a.F && mapping_ok(a, fh_or_0, t)) return t;
   if (cp_admissible(p, a, fh_or_0)) {
-    // rows wider than 128 features: the gather4 streaming kernel (cp = 2,
-    // launch_aggregate falls back to the cp.async chain if it cannot take the
-    // call); up to 128: the cp.async chain for sum / mean / max, the register
-    // kernel for GAT (measured faster there)
+    // staged kernels with the (4, 32, NV) lane mapping: cp = 1 the cp.async
+    // chain, cp = 2 the gather4 streaming kernel (launch_aggregate falls back
+    // to the cp.async chain if gather4 cannot take the call)
     Mapping c{4, 32, a.F > 128 ? 2 : 1};
-    // rows of > 128 features: the gather4 streaming kernel (C5 agg2 F = 256:
-    // 15.0 vs 16.8 ms for the register kernel); 64..128: the cp.async chain
-    // (C5 agg1 F = 100 with per-edge GCN weights: 11.0 vs 11.9 register, 13.8
-    // gather4)
-    static int g4_narrow = -1;  // A/B: env GNN_G4_NARROW=1 sends 64..128-feature rows to gather4 too
-    if (g4_narrow < 0) {
-      const char *e = getenv("GNN_G4_NARROW");
+    // sum / mean / max: the cp.async chain for every width (two 128-feature
+    // vectors per lane, 256-feature chunks, 8-slot ring): it measured faster
+    // than gather4 at every F in 144..256 on C5 (agg2 F=256 prescaled 13.9 vs
+    // 14.5 ms, DRAM 84.4 vs 93.6 GB: a narrower window of the task order in
+    // flight); A/B: env GNN_G4_SUM=1 sends rows of > 128 features to gather4,
+    // GNN_G4_NARROW=1 also the 64..128-feature rows
+    static int g4_sum = -1, g4_narrow = -1;
+    if (g4_sum < 0) {
+      const char *e = getenv("GNN_G4_SUM");
+      g4_sum = (e && e[0] == '1') ? 1 : 0;
+      e = getenv("GNN_G4_NARROW");
       g4_narrow = (e && e[0] == '1') ? 1 : 0;
     }
-    c.cp = (a.F > 128 || g4_narrow) ? g_agg_cp : std::min(g_agg_cp, 1);
+    c.cp = ((a.F > 128 && g4_sum) || g4_narrow) ? g_agg_cp : std::min(g_agg_cp, 1);
     if (a.mode == M_GAT) {
-      // GAT, rows > 128 features: gather4 with the H score columns in the same
-      // request as the row and 64-byte L2 promotion for the 1056-byte [z | s]
-      // rows (C5 8x32, same box: 18.7-19.0 vs 19.6-19.7 ms for the register
-      // kernel; profiles/r02_r3d_*); env GNN_G4_GAT=0 takes the register kernel
-      static int g4_gat = -1;
+      // GAT, rows of > 128 features: the lean cp.async chain (C5 8x32, same
+      // box: 16.9-17.4 vs 17.4-17.6 ms on gather4, DRAM 96.7 vs 101.5 GB; the
+      // register kernel 19.6-19.7 ms); A/B: env GNN_G4_GAT=1 takes gather4
+      // (scores in the row's request, 64-byte L2 promotion), GNN_CP_GAT=0 the
+      // register kernel; up to 128 features the register kernel
+      static int g4_gat = -1, cp_gat = -1;
       if (g4_gat < 0) {
         const char *e = getenv("GNN_G4_GAT");
-        g4_gat = (e && e[0] == '0') ? 0 : 1;
+        g4_gat = (e && e[0] == '1') ? 1 : 0;
+        e = getenv("GNN_CP_GAT");
+        cp_gat = (e && e[0] == '0') ? 0 : 1;
       }
-      c.cp = (g4_gat && a.F > 128 && c.cp == 2) ? 2 : 0;
+      if (a.F > 128 && g4_gat) c.cp = g_agg_cp == 2 ? 2 : 0;
+      else if (a.F > 128 && cp_gat) c.cp = g_agg_cp ? 1 : 0;
+      else c.cp = 0;
     }
     if (c.cp) return c;
   }
