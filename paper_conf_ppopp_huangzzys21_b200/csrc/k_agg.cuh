@@ -1315,7 +1315,10 @@ __device__ __forceinline__ void finish_unit(const KParams &p, const Part<MODE, V
 #define GNN_CP_S2 8  // NV = 2: rows <= 256 features (C3 F=256 GCN, same box: S = 4 / 6 / 8 / 12 -> 9.7-9.8 / 10.0-10.1 / 9.2-9.5 / 9.65 ms)
 #endif
 template <int MODE, int VEC, int NV, int LANES, int S = 0>
-__global__ void __launch_bounds__(256, S > 0 ? GNN_AGG_MINB_CP
+#ifndef GNN_AGG_MINB_CP2
+#define GNN_AGG_MINB_CP2 3  // NV = 2 rings (8 slots of 1 KB per warp) fit 3 CTAs per SM: 80 registers, no spills
+#endif
+__global__ void __launch_bounds__(256, S > 0 ? (NV >= 2 ? GNN_AGG_MINB_CP2 : GNN_AGG_MINB_CP)
                                              : (vec_score(MODE) ? 2 : (is_att(MODE) ? GNN_AGG_MINB_GAT : GNN_AGG_MINB)))
     k_aggregate(const KParams p) {
   constexpr int CW = LANES * VEC * NV;
