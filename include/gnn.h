@@ -204,6 +204,15 @@ size_t gnn_workspace_size(gnn_plan_t plan, int op, int32_t f_in, int32_t f_out, 
  *   X: [n_src, ldx] with F <= ldx; Y: [n, ldy]; X and Y must not overlap.
  *   add_row: [n, ld_add] or NULL.
  * F == 0 is a no-op.
+ * Kernels (results bit-identical across them): rows of >= 64
+ * features stream through a per-warp shared-memory ring (cp.async), narrower
+ * rows use the register kernel.  When the source rows exceed L2 (n_src * row
+ * bytes > 128 MB), the plan's highest out-degree sources (up to 32 MB of rows,
+ * the list built on the first such call) are marked evict_last in L2 for the
+ * duration of the call and returned to evict_normal after it (cache hints
+ * only; env GNN_L2_PIN=0 disables).  Every aggregation entry point below
+ * (gnn_gat_aggregate, gnn_attn_aggregate, gnn_gcn_aggregate_prescaled,
+ * gnn_aggregate_accumulate, gnn_edgeconv_aggregate) behaves the same way.
  */
 gnn_status gnn_aggregate(gnn_plan_t plan, int reduce, int weight, const float *edge_w,
                          const float *X, int64_t ldx, int32_t F, float *Y, int64_t ldy,
