@@ -431,15 +431,17 @@ static Mapping choose_mapping(const gnn_plan_s *p, const AggArgs &a, int32_t fh_
       // register kernel 19.6-19.7 ms); A/B: env GNN_G4_GAT=1 takes gather4
       // (scores in the row's request, 64-byte L2 promotion), GNN_CP_GAT=0 the
       // register kernel; up to 128 features the register kernel
-      static int g4_gat = -1, cp_gat = -1;
+      static int g4_gat = -1, cp_gat = -1, cp_gat_narrow = -1;
       if (g4_gat < 0) {
         const char *e = getenv("GNN_G4_GAT");
         g4_gat = (e && e[0] == '1') ? 1 : 0;
         e = getenv("GNN_CP_GAT");
         cp_gat = (e && e[0] == '0') ? 0 : 1;
+        e = getenv("GNN_CP_GAT_NARROW");  // A/B: 64..128-feature GAT rows on the lean chain too
+        cp_gat_narrow = (e && e[0] == '1') ? 1 : 0;
       }
       if (a.F > 128 && g4_gat) c.cp = g_agg_cp == 2 ? 2 : 0;
-      else if (a.F > 128 && cp_gat) c.cp = g_agg_cp ? 1 : 0;
+      else if ((a.F > 128 || cp_gat_narrow) && cp_gat) c.cp = g_agg_cp ? 1 : 0;
       else c.cp = 0;
     }
     if (c.cp) return c;
